@@ -1,0 +1,255 @@
+"""Pins for the fp64 CPU oracle (no GPU).
+
+The oracle (oracle/ncc_oracle.c) is checked against things other than itself:
+  * hand-derived closed forms (tests/golden/hand_cases.json),
+  * numpy.corrcoef (library Pearson) on random non-square cases,
+  * invariants the corr2 definition fixes (planted = 1, |r| <= 1, affine invariance,
+    symmetry, flat -> 0),
+  * an independent algebra (oracle/ncc_fft.py: FFT numerator + fp64 SAT denominator),
+  * PIV: planted integer shifts, the window-grid count by enumeration, sub-pixel closed
+    forms (Gaussian / parabola triples are recovered exactly).
+Citations: PAPER.md Fig 5.1 caption P:132-137 (definition), Listing 5.1 caption
+P:250-251 (corr2 per shift), PIV Figs 5.9-5.12 captions P:165-171; SURVEY.md 8(c).
+"""
+import json
+import math
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+from oracle.ncc_fft import ncc_surface_fft, window_sums
+import synth
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden", "hand_cases.json")
+
+
+def _closed(expr: str) -> float:
+    return float(eval(expr, {"sqrt": math.sqrt}))
+
+
+def _cases():
+    with open(GOLD) as f:
+        return json.load(f)
+
+
+# ---------------------------------------------------------------- hand cases
+def test_hand_case_A():
+    c = _cases()["case_A"]
+    s = oracle.ncc_surface(np.array(c["image"], np.float32), np.array(c["template"], np.float32))
+    exp = np.array([[_closed(e) for e in row] for row in c["expected"]])
+    np.testing.assert_allclose(s, exp, rtol=0, atol=1e-14)
+
+
+def test_hand_case_B():
+    c = _cases()["case_B"]
+    s = oracle.ncc_surface(np.array(c["image"], np.float32), np.array(c["template"], np.float32))
+    for u, v, e in c["expected_at"]:
+        assert abs(s[u, v] - _closed(e)) < 1e-14, (u, v, s[u, v], e)
+    # negated image -> -1 at the plant (alpha < 0 flips the sign)
+    s2 = oracle.ncc_surface(-np.array(c["image"], np.float32), np.array(c["template"], np.float32))
+    assert abs(s2[1, 1] + 1.0) < 1e-14
+
+
+def test_hand_case_E_flat():
+    c = _cases()["case_E_flat"]
+    s = oracle.ncc_surface(np.array(c["image"], np.float32), np.array(c["template"], np.float32))
+    exp = np.array([[_closed(e) for e in row] for row in c["expected"]])
+    np.testing.assert_allclose(s, exp, rtol=0, atol=1e-14)
+
+
+# ---------------------------------------------------------------- library routine
+@pytest.mark.parametrize("H,W,h,w,seed", [(9, 11, 3, 5, 1), (12, 7, 4, 2, 2), (10, 10, 7, 3, 3), (6, 13, 1, 6, 4)])
+def test_matches_numpy_corrcoef(H, W, h, w, seed):
+    g = synth.rng(seed)
+    I = g.random((H, W), dtype=np.float32)
+    T = g.random((h, w), dtype=np.float32) * 3 - 1
+    s = oracle.ncc_surface(I, T)
+    assert s.shape == (H - h + 1, W - w + 1)
+    for u in range(H - h + 1):
+        for v in range(W - w + 1):
+            ref = np.corrcoef(T.astype(np.float64).ravel(), I[u:u + h, v:v + w].astype(np.float64).ravel())[0, 1]
+            assert abs(s[u, v] - ref) < 1e-12
+
+
+def test_ncc_at_matches_surface():
+    I, T, _, _ = synth.tm_inputs(1)
+    s = oracle.ncc_surface(I, T)
+    g = synth.rng(5)
+    us = g.integers(0, s.shape[0], 50)
+    vs = g.integers(0, s.shape[1], 50)
+    np.testing.assert_array_equal(oracle.ncc_at(I, T, us, vs), s[us, vs])
+
+
+def test_band_rows():
+    I, T, _, _ = synth.tm_inputs(1)
+    s = oracle.ncc_surface(I, T)
+    np.testing.assert_array_equal(oracle.ncc_surface(I, T, 10, 23), s[10:23])
+
+
+# ---------------------------------------------------------------- invariants
+def test_planted_scores_one_and_is_peak():
+    I, T, u0, v0 = synth.tm_inputs(1)
+    s, pk = oracle.ncc_match(I, T)
+    assert abs(s[u0, v0] - 1.0) < 1e-12
+    assert (pk.u, pk.v) == (u0, v0) and pk.valid
+    assert np.all(np.abs(s) <= 1.0 + 1e-12)
+
+
+def test_affine_invariance():
+    g = synth.rng(11)
+    I = g.random((20, 23), dtype=np.float32)
+    T = g.random((5, 7), dtype=np.float32)
+    s = oracle.ncc_surface(I, T)
+    np.testing.assert_allclose(oracle.ncc_surface(2.5 * I - 7, T), s, atol=1e-6)  # fp32 input rounding
+    np.testing.assert_allclose(oracle.ncc_surface(I, 0.25 * T + 3), s, atol=1e-6)
+    np.testing.assert_allclose(oracle.ncc_surface(-I, T), -s, atol=1e-12)
+    np.testing.assert_allclose(oracle.ncc_surface(I, -T), -s, atol=1e-12)
+    # exactly representable affine maps (power-of-two scale, small shift) -> tight agreement
+    Iq = synth.quantize(I)
+    sq = oracle.ncc_surface(Iq, T)
+    np.testing.assert_allclose(oracle.ncc_surface(4 * Iq + 1, T), sq, atol=1e-13)
+
+
+def test_symmetry_template_window():
+    g = synth.rng(12)
+    A = g.random((6, 9), dtype=np.float32)
+    B = g.random((6, 9), dtype=np.float32)
+    assert abs(oracle.ncc_surface(A, B)[0, 0] - oracle.ncc_surface(B, A)[0, 0]) < 1e-15
+
+
+def test_flat_template_all_zero_and_invalid():
+    I = synth.uniform_image(16, 16, 3)
+    T = np.full((4, 4), 0.3, np.float32)
+    s, pk = oracle.ncc_match(I, T)
+    assert np.all(s == 0.0) and not pk.valid and (pk.u, pk.v) == (0, 0)
+
+
+def test_flat_window_zero():
+    I = synth.uniform_image(16, 16, 4)
+    I[2:8, 3:9] = 0.75
+    T = synth.uniform_image(4, 4, 5)
+    s = oracle.ncc_surface(I, T)
+    assert np.all(s[2:5, 3:6] == 0.0)
+    assert np.all(s[6:, :] != 0.0)
+
+
+def test_argmax_tie_smallest_index():
+    s = np.zeros((5, 7))
+    s[3, 1] = s[1, 4] = s[4, 6] = 0.9
+    assert oracle.argmax(s) == 1 * 7 + 4
+
+
+# ---------------------------------------------------------------- independent algebra
+@pytest.mark.parametrize("smooth", [False, True])
+def test_bruteforce_equals_fft_route(smooth):
+    img = synth.smooth_image(96, 80, 21) if smooth else synth.uniform_image(96, 80, 21)
+    T, _, _ = synth.planted_template(img, 17, 13, 22)
+    s = oracle.ncc_surface(img, T)
+    f = ncc_surface_fft(img, T)
+    assert np.max(np.abs(s - f)) < 1e-10
+
+
+def test_window_sums_exact_on_quantized():
+    img = synth.quantize(synth.uniform_image(40, 33, 7))
+    S1, S2 = window_sums(img, 9, 5)
+    I = img.astype(np.float64)
+    for u in (0, 5, 31):
+        for v in (0, 11, 28):
+            assert S1[u, v] == I[u:u + 9, v:v + 5].sum()
+            assert S2[u, v] == (I[u:u + 9, v:v + 5] ** 2).sum()
+
+
+# ---------------------------------------------------------------- PIV
+def test_piv_grid_by_enumeration():
+    for (H, W, h, w, my, mx, sy, sx) in [(1024, 1024, 32, 32, 16, 16, 16, 16), (2048, 2048, 64, 64, 32, 32, 32, 32),
+                                         (100, 77, 8, 6, 3, 2, 5, 4)]:
+        ny = len([y for y in range(my, H, sy) if y + h + my <= H])
+        nx = len([x for x in range(mx, W, sx) if x + w + mx <= W])
+        assert oracle.piv_grid(H, W, h, w, my, mx, sy, sx) == (ny, nx)
+    assert oracle.piv_grid(1024, 1024, 32, 32, 16, 16, 16, 16) == (61, 61)
+    assert oracle.piv_grid(2048, 2048, 64, 64, 32, 32, 32, 32) == (61, 61)
+
+
+def test_piv_planted_integer_shift():
+    dy, dx = 3, -5
+    p = synth.particle_pair_integer(160, 176, dy, dx, seed=31)
+    v = oracle.piv_pair(p.A, p.B, 32, 32, 8, 8, 16, 16)
+    assert np.all(v["iy"] == dy) and np.all(v["ix"] == dx)
+    assert np.all(np.abs(v["score"] - 1.0) < 1e-9)
+    assert np.all(v["flags"] & (oracle.EDGE_Y | oracle.EDGE_X | oracle.INVALID) == 0)
+    # Integer-shift peaks have symmetric-ish neighbours; the fit stays inside (-0.5, 0.5)
+    assert np.all(np.abs(v["dy"] - dy) < 0.5) and np.all(np.abs(v["dx"] - dx) < 0.5)
+
+
+def test_piv_zero_shift():
+    p = synth.particle_pair_integer(96, 96, 0, 0, seed=32)
+    v = oracle.piv_pair(p.A, p.A, 16, 16, 4, 4, 16, 16)
+    assert np.all(v["iy"] == 0) and np.all(v["ix"] == 0)
+    assert np.all(np.abs(v["score"] - 1.0) < 1e-12)
+
+
+def test_piv_scores_are_tm_surface_of_search_region():
+    p = synth.particle_pair_integer(128, 128, 2, 1, seed=33)
+    h = w = 16
+    m = 6
+    s = 16
+    ky, kx = 2, 3
+    y, x = m + ky * s, m + kx * s
+    sc = oracle.piv_window_scores(p.A, p.B, h, w, m, m, s, s, ky, kx)
+    ref = oracle.ncc_surface(p.B[y - m:y + h + m, x - m:x + w + m], p.A[y:y + h, x:x + w])
+    np.testing.assert_array_equal(sc, ref)
+
+
+def test_piv_edge_flags():
+    # true shift beyond the search radius -> peak can land on the border
+    p = synth.particle_pair_integer(128, 128, 9, 0, seed=34)
+    v = oracle.piv_pair(p.A, p.B, 16, 16, 4, 4, 16, 16)
+    on_edge = np.abs(v["iy"]) == 4
+    assert on_edge.any()
+    assert np.all((v["flags"][on_edge] & oracle.EDGE_Y) != 0)
+    assert np.all(v["dy"][on_edge] == v["iy"][on_edge])
+
+
+def test_piv_flat_mask_invalid():
+    A = np.zeros((64, 64), np.float32)
+    B = synth.uniform_image(64, 64, 35)
+    v = oracle.piv_pair(A, B, 16, 16, 4, 4, 16, 16)
+    assert np.all(v["flags"] & oracle.INVALID) and np.all(v["score"] == 0.0)
+
+
+# ---------------------------------------------------------------- sub-pixel
+def test_subpixel_symmetric_is_zero():
+    assert oracle.subpixel3(0.5, 0.9, 0.5) == (0.0, False)
+    assert oracle.subpixel3(-0.2, 0.9, -0.2) == (0.0, True)
+
+
+@pytest.mark.parametrize("delta,sigma", [(0.3, 1.0), (-0.17, 0.8), (0.45, 1.6), (-0.49, 1.2)])
+def test_subpixel_gaussian_exact(delta, sigma):
+    c = [math.exp(-((k - delta) ** 2) / (2 * sigma * sigma)) for k in (-1, 0, 1)]
+    d, par = oracle.subpixel3(*c)
+    assert not par and abs(d - delta) < 1e-12
+
+
+@pytest.mark.parametrize("delta", [0.21, -0.33, 0.05])
+def test_subpixel_parabola_fallback_exact(delta):
+    a, b = 0.3, 0.5
+    c = [a - b * (k - delta) ** 2 for k in (-1, 0, 1)]
+    assert min(c) <= 0  # forces the parabolic branch
+    d, par = oracle.subpixel3(*c)
+    assert par and abs(d - delta) < 1e-12
+
+
+def test_subpixel_not_a_maximum():
+    assert oracle.subpixel3(0.9, 0.5, 0.9)[0] == 0.0
+    assert oracle.subpixel3(0.5, 0.5, 0.5)[0] == 0.0
+
+
+def test_piv_subpixel_recovers_fractional_shift():
+    p = synth.particle_pair_subpixel(160, 160, 2.3, -1.6, seed=36)
+    v = oracle.piv_pair(p.A, p.B, 32, 32, 6, 6, 16, 16)
+    assert np.all(v["iy"] == 2) and np.all(v["ix"] == -2)
+    # method accuracy (reported, not a parity bound): Gaussian fit within 0.1 px here
+    assert np.median(np.abs(v["dy"] - 2.3)) < 0.1
+    assert np.median(np.abs(v["dx"] + 1.6)) < 0.1
