@@ -1,0 +1,611 @@
+// ncc_api.cu -- C ABI (include/ncc.h) over the sm_100a kernels in ncc_kernels.cuh.
+//
+// Lifecycle follows GPU-PF: ncc_plan_create = specification +
+// refresh (validate, choose the specialised variant, allocate scratch, set kernel
+// attributes); ncc_match / piv_correlate = execution (launches only, no allocation);
+// ncc_plan_destroy.  Variant selection (Ch. 4): problem
+// parameters that control loop structure (template size, search radius) are baked into
+// pre-instantiated kernels ("SK"); anything else runs the run-time-evaluated generic kernel
+// ("RE").  Pointers and template values always stay run-time.
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/ncc.h"
+#include "ncc_kernels.cuh"
+
+using namespace nccb;
+
+static_assert(sizeof(ncc_peak) == 16, "ncc_peak must be 16 B");
+static_assert(sizeof(piv_vector) == 24, "piv_vector must be 24 B");
+static_assert(sizeof(PeakOut) == sizeof(ncc_peak), "PeakOut layout");
+static_assert(sizeof(VecOut) == sizeof(piv_vector), "VecOut layout");
+
+namespace {
+
+thread_local std::string g_last_cuda_error;
+
+ncc_status cuda_fail(cudaError_t e, const char* where) {
+  g_last_cuda_error = std::string(where) + ": " + cudaGetErrorString(e);
+  return e == cudaErrorMemoryAllocation ? NCC_ERR_OUT_OF_MEMORY : NCC_ERR_CUDA;
+}
+#define NCC_CUDA(call)                                   \
+  do {                                                   \
+    cudaError_t _e = (call);                             \
+    if (_e != cudaSuccess) return cuda_fail(_e, #call);  \
+  } while (0)
+
+// ------------------------------------------------------------------ variant tables
+struct TmVariant {
+  const char* name;
+  int TH, TW;                 // 0 = run-time (RE)
+  int RV, LX, WX, WY, CH, CW;
+  void (*kernel)(TmArgs);
+  int nt, bu, bv, smem;
+};
+
+#define TM_VARIANT(NAME, TH, TW, RV, LX, WX, WY, CH, CW)                                                  \
+  TmVariant {                                                                                          \
+    NAME, TH, TW, RV, LX, WX, WY, CH, CW, tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW>,                 \
+        TmTile<RV, LX, WX, WY, CH, CW>::NT, TmTile<RV, LX, WX, WY, CH, CW>::BU,                        \
+        TmTile<RV, LX, WX, WY, CH, CW>::BV, TmTile<RV, LX, WX, WY, CH, CW>::SMEM                       \
+  }
+
+const TmVariant kTmVariants[] = {
+    // generic run-time-evaluated kernel (any h, w)
+    TM_VARIANT("tm_re_rv12_lx4_4x1_c32x32", 0, 0, 12, 4, 1, 4, 32, 32),
+    // specialised instances for the BASELINE configurations
+    TM_VARIANT("tm_sk_16x16_rv4_lx16_4x1_c16x16", 16, 16, 4, 16, 1, 4, 16, 16),
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c32x64", 128, 128, 12, 4, 1, 4, 32, 64),
+    TM_VARIANT("tm_sk_512x512_rv12_lx4_4x1_c32x64", 512, 512, 12, 4, 1, 4, 32, 64),
+};
+
+struct PivVariant {
+  const char* name;
+  int TH, TW, MY, MX;  // 0 = run-time (RE)
+  int RV, CW, NT;
+  void (*kernel)(PivArgs);
+};
+#define PIV_VARIANT(NAME, TH, TW, MY, MX, RV, CW, NT, MINB) \
+  PivVariant { NAME, TH, TW, MY, MX, RV, CW, NT, piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, MINB> }
+
+const PivVariant kPivVariants[] = {
+    PIV_VARIANT("piv_re_rv12_cw16_nt256", 0, 0, 0, 0, 12, 16, 256, 1),
+    PIV_VARIANT("piv_sk_32x32_m16_rv12_nt128", 32, 32, 16, 16, 12, 32, 128, 4),
+    PIV_VARIANT("piv_sk_64x64_m32_rv12_nt416", 64, 64, 32, 32, 12, 64, 416, 2),
+};
+
+constexpr int kBoxRowsNT = 256, kBoxRowsSEG = 4096;
+constexpr int kBoxColsNT = 128, kBoxColsRB = 64;
+
+int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
+
+}  // namespace
+
+// ------------------------------------------------------------------ plan object
+struct ncc_plan_s {
+  ncc_problem p;
+  int device;
+  ncc_plan_info info;
+  // TM
+  int U, V, u_begin, u_end, Ub, Hs, HP, WP;
+  const TmVariant* tmv;
+  float* tplC;
+  TemplateStats* tst;
+  unsigned long long* keys;
+  // PIV
+  int Ky, Kx, OY, OX, sub_batch, piv_bp, piv_smem, map_w, map_h;
+  const PivVariant* pivv;
+  // shared scratch (window sums)
+  double *RS1, *RS2, *S1, *S2;
+  int64_t rs_frame_stride, s_frame_stride;
+  // timing (NCC_F_TIMING)
+  std::vector<cudaEvent_t> ev;
+  int n_ev_used;
+  int timing_kind;  // 0 none, 1 TM, 2 PIV
+  int piv_nsub;
+  // host staging (lazy)
+  float *st_a, *st_b, *st_t, *st_s;
+  void* st_out;
+  size_t st_a_bytes, st_b_bytes, st_t_bytes, st_s_bytes, st_out_bytes;
+};
+
+namespace {
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) cudaSetDevice(dev);
+    else prev = -1;
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+void free_plan(ncc_plan pl) {
+  cudaFree(pl->tplC);
+  cudaFree(pl->tst);
+  cudaFree(pl->keys);
+  cudaFree(pl->RS1);
+  cudaFree(pl->RS2);
+  cudaFree(pl->S1);
+  cudaFree(pl->S2);
+  cudaFree(pl->st_a);
+  cudaFree(pl->st_b);
+  cudaFree(pl->st_t);
+  cudaFree(pl->st_s);
+  cudaFree(pl->st_out);
+  for (cudaEvent_t e : pl->ev) cudaEventDestroy(e);
+  delete pl;
+}
+
+ncc_status validate(const ncc_problem& p) {
+  if (p.score != NCC_SCORE_NCC) return p.score == NCC_SCORE_SSD ? NCC_ERR_UNSUPPORTED : NCC_ERR_INVALID_ARGUMENT;
+  if (p.mode != NCC_MODE_MATCH && p.mode != NCC_MODE_PIV) return NCC_ERR_INVALID_ARGUMENT;
+  if (p.image_h <= 0 || p.image_w <= 0 || p.tmpl_h <= 0 || p.tmpl_w <= 0) return NCC_ERR_INVALID_ARGUMENT;
+  if (p.image_pitch < p.image_w) return NCC_ERR_INVALID_ARGUMENT;
+  if (p.tmpl_h > p.image_h || p.tmpl_w > p.image_w) return NCC_ERR_INVALID_ARGUMENT;
+  if (p.batch < 1 || p.shard_count < 1 || p.shard_rank < 0 || p.shard_rank >= p.shard_count)
+    return NCC_ERR_INVALID_ARGUMENT;
+  if (p.mode == NCC_MODE_MATCH) {
+    if (p.search_y != 0 || p.search_x != 0) return NCC_ERR_INVALID_ARGUMENT;
+    const int64_t U = p.image_h - p.tmpl_h + 1, V = p.image_w - p.tmpl_w + 1;
+    if (U * V >= (int64_t)0xFFFFFFF0ll) return NCC_ERR_INVALID_ARGUMENT;  // 32-bit key index
+    if (p.shard_count > U) return NCC_ERR_INVALID_ARGUMENT;               // every band has rows
+  } else {
+    if (p.search_y < 0 || p.search_x < 0 || p.step_y <= 0 || p.step_x <= 0) return NCC_ERR_INVALID_ARGUMENT;
+    if (p.image_h - p.tmpl_h - 2 * p.search_y < 0 || p.image_w - p.tmpl_w - 2 * p.search_x < 0)
+      return NCC_ERR_INVALID_ARGUMENT;
+    if (p.shard_count != 1 || p.shard_rank != 0) return NCC_ERR_INVALID_ARGUMENT;
+    if (p.subpix < 0 || p.subpix > 2) return NCC_ERR_INVALID_ARGUMENT;
+  }
+  return NCC_OK;
+}
+
+template <class T>
+ncc_status dalloc(T** ptr, size_t count) {
+  *ptr = nullptr;
+  if (count == 0) return NCC_OK;
+  cudaError_t e = cudaMalloc((void**)ptr, count * sizeof(T));
+  if (e != cudaSuccess) {
+    *ptr = nullptr;
+    return cuda_fail(e, "cudaMalloc");
+  }
+  return NCC_OK;
+}
+
+void fill_kernel_info(ncc_plan pl, const void* fn, int nt, int smem, int gx, int gy, int gz) {
+  cudaFuncAttributes fa;
+  if (cudaFuncGetAttributes(&fa, fn) == cudaSuccess) pl->info.regs_per_thread = fa.numRegs;
+  pl->info.threads_per_block = nt;
+  pl->info.smem_per_block = smem;
+  pl->info.grid_x = gx;
+  pl->info.grid_y = gy;
+  pl->info.grid_z = gz;
+}
+
+ncc_status create_tm(ncc_plan pl) {
+  const ncc_problem& p = pl->p;
+  const int h = p.tmpl_h, w = p.tmpl_w;
+  pl->U = p.image_h - h + 1;
+  pl->V = p.image_w - w + 1;
+  const int band = ceil_div(pl->U, p.shard_count);
+  pl->u_begin = p.shard_rank * band;
+  pl->u_end = pl->u_begin + band < pl->U ? pl->u_begin + band : pl->U;
+  if (pl->u_begin >= pl->u_end) return NCC_ERR_INVALID_ARGUMENT;
+  pl->Ub = pl->u_end - pl->u_begin;
+  pl->Hs = pl->Ub + h - 1;
+
+  const TmVariant* v = &kTmVariants[0];
+  if (!(p.flags & NCC_F_GENERIC_KERNEL))
+    for (const TmVariant& c : kTmVariants)
+      if (c.TH == h && c.TW == w) v = &c;
+  pl->tmv = v;
+  const int nCH = ceil_div(h, v->CH), nCW = ceil_div(w, v->CW);
+  pl->HP = nCH * v->CH;
+  pl->WP = nCW * v->CW;
+
+  int maxsm = 0;
+  NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
+  if (v->smem > maxsm) return NCC_ERR_UNSUPPORTED;
+  NCC_CUDA(cudaFuncSetAttribute((const void*)v->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, v->smem));
+  const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
+  if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
+  NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT, kBoxRowsSEG>,
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem));
+
+  ncc_status st;
+  if ((st = dalloc(&pl->tplC, (size_t)pl->HP * pl->WP))) return st;
+  if ((st = dalloc(&pl->tst, 1))) return st;
+  if ((st = dalloc(&pl->keys, (size_t)p.batch))) return st;
+  pl->rs_frame_stride = (int64_t)pl->Hs * pl->V;
+  pl->s_frame_stride = (int64_t)pl->Ub * pl->V;
+  if ((st = dalloc(&pl->RS1, (size_t)p.batch * pl->rs_frame_stride))) return st;
+  if ((st = dalloc(&pl->RS2, (size_t)p.batch * pl->rs_frame_stride))) return st;
+  if ((st = dalloc(&pl->S1, (size_t)p.batch * pl->s_frame_stride))) return st;
+  if ((st = dalloc(&pl->S2, (size_t)p.batch * pl->s_frame_stride))) return st;
+
+  ncc_plan_info& in = pl->info;
+  in.U = pl->U;
+  in.V = pl->V;
+  in.u_begin = pl->u_begin;
+  in.u_end = pl->u_end;
+  in.outputs_per_call = (int64_t)pl->Ub * pl->V * p.batch;
+  in.flops_per_call = 2.0 * h * (double)w * (double)in.outputs_per_call;
+  in.specialized = v->TH != 0;
+  in.variant_id = (int)(v - kTmVariants);
+  snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
+  fill_kernel_info(pl, (const void*)v->kernel, v->nt, v->smem, ceil_div(pl->V, v->bv), ceil_div(pl->Ub, v->bu),
+                   p.batch);
+  return NCC_OK;
+}
+
+ncc_status create_piv(ncc_plan pl) {
+  const ncc_problem& p = pl->p;
+  const int h = p.tmpl_h, w = p.tmpl_w, my = p.search_y, mx = p.search_x;
+  pl->Ky = (p.image_h - h - 2 * my) / p.step_y + 1;
+  pl->Kx = (p.image_w - w - 2 * mx) / p.step_x + 1;
+  pl->OY = 2 * my + 1;
+  pl->OX = 2 * mx + 1;
+  pl->map_h = p.image_h - h + 1;
+  pl->map_w = p.image_w - w + 1;
+
+  const PivVariant* v = &kPivVariants[0];
+  if (!(p.flags & NCC_F_GENERIC_KERNEL))
+    for (const PivVariant& c : kPivVariants)
+      if (c.TH == h && c.TW == w && c.MY == my && c.MX == mx) v = &c;
+  pl->pivv = v;
+  const int RV = v->RV, CW = v->CW;
+  const int NG = (pl->OX + RV - 1) / RV, OXP = NG * RV, WP = ((w + CW - 1) / CW) * CW;
+  pl->piv_bp = piv_pick_pitch(OXP + WP, RV, NG);
+  const int64_t smem_f = (int64_t)h * WP + (int64_t)(h + 2 * my) * pl->piv_bp + (int64_t)pl->OY * OXP;
+  pl->piv_smem = (int)(smem_f * 4);
+  int maxsm = 0;
+  NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
+  if (smem_f * 4 > maxsm) return NCC_ERR_UNSUPPORTED;
+  NCC_CUDA(cudaFuncSetAttribute((const void*)v->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
+  const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
+  if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
+  NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT, kBoxRowsSEG>,
+                                cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem));
+
+  // window-sum maps of frame B, processed in sub-batches of pairs (scratch budget ~2 GiB)
+  pl->rs_frame_stride = (int64_t)p.image_h * pl->map_w;
+  pl->s_frame_stride = (int64_t)pl->map_h * pl->map_w;
+  const double per_pair = 16.0 * (double)(pl->rs_frame_stride + pl->s_frame_stride);
+  int sb = (int)(2.0 * 1024 * 1024 * 1024 / per_pair);
+  if (sb < 1) sb = 1;
+  if (sb > p.batch) sb = p.batch;
+  pl->sub_batch = sb;
+  ncc_status st;
+  if ((st = dalloc(&pl->RS1, (size_t)sb * pl->rs_frame_stride))) return st;
+  if ((st = dalloc(&pl->RS2, (size_t)sb * pl->rs_frame_stride))) return st;
+  if ((st = dalloc(&pl->S1, (size_t)sb * pl->s_frame_stride))) return st;
+  if ((st = dalloc(&pl->S2, (size_t)sb * pl->s_frame_stride))) return st;
+
+  ncc_plan_info& in = pl->info;
+  in.U = pl->OY;
+  in.V = pl->OX;
+  in.Ky = pl->Ky;
+  in.Kx = pl->Kx;
+  in.outputs_per_call = (int64_t)pl->Ky * pl->Kx * p.batch;
+  in.flops_per_call = 2.0 * h * (double)w * pl->OY * (double)pl->OX * (double)in.outputs_per_call;
+  in.specialized = v->TH != 0;
+  in.variant_id = (int)(v - kPivVariants);
+  snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
+  fill_kernel_info(pl, (const void*)v->kernel, v->NT, pl->piv_smem, pl->Kx, pl->Ky, sb);
+  return NCC_OK;
+}
+
+ncc_status ensure_events(ncc_plan pl, int n) {
+  while ((int)pl->ev.size() < n) {
+    cudaEvent_t e;
+    NCC_CUDA(cudaEventCreate(&e));
+    pl->ev.push_back(e);
+  }
+  return NCC_OK;
+}
+
+inline void mark(ncc_plan pl, cudaStream_t s, int i) {
+  if (pl->p.flags & NCC_F_TIMING) cudaEventRecord(pl->ev[i], s);
+}
+
+// window sums of `batch` frames over rows [row0, row0 + rows_out + h - 1)
+void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_out, cudaStream_t s) {
+  const ncc_problem& p = pl->p;
+  const int h = p.tmpl_h, w = p.tmpl_w;
+  const int V = p.image_w - w + 1;
+  const int rows_in = rows_out + h - 1;
+  const int smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
+  dim3 g1(ceil_div(V, kBoxRowsSEG), rows_in, batch);
+  box_rows_kernel<kBoxRowsNT, kBoxRowsSEG><<<g1, kBoxRowsNT, smem, s>>>(
+      frames, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, row0, w, V, pl->RS1, pl->RS2,
+      pl->rs_frame_stride);
+  dim3 g2(ceil_div(V, kBoxColsNT), ceil_div(rows_out, kBoxColsRB), batch);
+  box_cols_kernel<kBoxColsNT, kBoxColsRB><<<g2, kBoxColsNT, 0, s>>>(pl->RS1, pl->RS2, pl->rs_frame_stride, V, h,
+                                                                    rows_out, pl->S1, pl->S2, pl->s_frame_stride);
+}
+
+ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, int64_t tmpl_pitch, float* d_scores,
+                     ncc_peak* d_peaks, cudaStream_t s) {
+  const ncc_problem& p = pl->p;
+  const TmVariant* v = pl->tmv;
+  if (p.flags & NCC_F_TIMING) {
+    ncc_status st = ensure_events(pl, 5);
+    if (st) return st;
+  }
+  pl->timing_kind = 1;
+  mark(pl, s, 0);
+  tm_template_prep<<<1, 1024, 0, s>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP, pl->tst,
+                                      pl->keys, p.batch);
+  mark(pl, s, 1);
+  launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
+  mark(pl, s, 2);
+  TmArgs a;
+  a.img = d_images;
+  a.pitch = p.image_pitch;
+  a.frame_stride = (int64_t)p.image_h * p.image_pitch;
+  a.H = p.image_h;
+  a.W = p.image_w;
+  a.tplC = pl->tplC;
+  a.tplP = pl->WP;
+  a.h = p.tmpl_h;
+  a.w = p.tmpl_w;
+  a.nCH = pl->HP / v->CH;
+  a.nCW = pl->WP / v->CW;
+  a.S1 = pl->S1;
+  a.S2 = pl->S2;
+  a.stat_frame_stride = pl->s_frame_stride;
+  a.tst = pl->tst;
+  a.U = pl->U;
+  a.V = pl->V;
+  a.u_begin = pl->u_begin;
+  a.u_end = pl->u_end;
+  a.scores = (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr;
+  a.score_frame_stride = (int64_t)pl->Ub * pl->V;
+  a.keys = pl->keys;
+  dim3 grid(ceil_div(pl->V, v->bv), ceil_div(pl->Ub, v->bu), p.batch);
+  v->kernel<<<grid, v->nt, v->smem, s>>>(a);
+  mark(pl, s, 3);
+  tm_finalize<<<ceil_div(p.batch, 128), 128, 0, s>>>(pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks),
+                                                     p.batch);
+  mark(pl, s, 4);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch");
+  return NCC_OK;
+}
+
+ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores, piv_vector* d_vec, cudaStream_t s) {
+  const ncc_problem& p = pl->p;
+  const PivVariant* v = pl->pivv;
+  const int nsub = ceil_div(p.batch, pl->sub_batch);
+  if (p.flags & NCC_F_TIMING) {
+    ncc_status st = ensure_events(pl, 3 * nsub + 1);
+    if (st) return st;
+  }
+  pl->timing_kind = 2;
+  pl->piv_nsub = nsub;
+  const int64_t fs = (int64_t)p.image_h * p.image_pitch;
+  const int64_t wins = (int64_t)pl->Ky * pl->Kx;
+  PivArgs a;
+  a.pitch = p.image_pitch;
+  a.frame_stride = fs;
+  a.H = p.image_h;
+  a.W = p.image_w;
+  a.h = p.tmpl_h;
+  a.w = p.tmpl_w;
+  a.my = p.search_y;
+  a.mx = p.search_x;
+  a.sy = p.step_y;
+  a.sx = p.step_x;
+  a.Ky = pl->Ky;
+  a.Kx = pl->Kx;
+  a.S1 = pl->S1;
+  a.S2 = pl->S2;
+  a.map_pitch = pl->map_w;
+  a.map_frame_stride = pl->s_frame_stride;
+  a.subpix = p.subpix;
+  a.BP = pl->piv_bp;
+  mark(pl, s, 0);
+  for (int sb = 0; sb < nsub; ++sb) {
+    const int p0 = sb * pl->sub_batch;
+    const int np = (p0 + pl->sub_batch <= p.batch) ? pl->sub_batch : p.batch - p0;
+    launch_box(pl, B + p0 * fs, np, 0, pl->map_h, s);
+    mark(pl, s, 3 * sb + 1);
+    a.A = A + p0 * fs;
+    a.B = B + p0 * fs;
+    a.vec = reinterpret_cast<VecOut*>(d_vec) + p0 * wins;
+    a.scores = d_scores ? d_scores + p0 * wins * pl->OY * pl->OX : nullptr;
+    dim3 grid(pl->Kx, pl->Ky, np);
+    v->kernel<<<grid, v->NT, pl->piv_smem, s>>>(a);
+    mark(pl, s, 3 * sb + 2);
+    if (p.flags & NCC_F_TIMING) mark(pl, s, 3 * sb + 3);
+  }
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return cuda_fail(e, "piv_correlate launch");
+  return NCC_OK;
+}
+
+ncc_status stage(void** buf, size_t* have, size_t need) {
+  if (*have >= need) return NCC_OK;
+  cudaFree(*buf);
+  *buf = nullptr;
+  *have = 0;
+  cudaError_t e = cudaMalloc(buf, need);
+  if (e != cudaSuccess) {
+    *buf = nullptr;
+    return cuda_fail(e, "cudaMalloc(staging)");
+  }
+  *have = need;
+  return NCC_OK;
+}
+
+}  // namespace
+
+// ================================================================== extern "C"
+extern "C" {
+
+const char* ncc_status_string(ncc_status s) {
+  switch (s) {
+    case NCC_OK: return "NCC_OK";
+    case NCC_ERR_INVALID_ARGUMENT: return "NCC_ERR_INVALID_ARGUMENT";
+    case NCC_ERR_UNSUPPORTED: return "NCC_ERR_UNSUPPORTED";
+    case NCC_ERR_OUT_OF_MEMORY: return "NCC_ERR_OUT_OF_MEMORY";
+    case NCC_ERR_CUDA: return "NCC_ERR_CUDA";
+    case NCC_ERR_COMPILE: return "NCC_ERR_COMPILE";
+    case NCC_ERR_WRONG_MODE: return "NCC_ERR_WRONG_MODE";
+  }
+  return "NCC_ERR_UNKNOWN";
+}
+
+const char* ncc_last_cuda_error(void) { return g_last_cuda_error.c_str(); }
+
+int32_t ncc_build_arch(void) { return 100; }
+
+ncc_status ncc_plan_create(const ncc_problem* p, int device, ncc_plan* out) {
+  if (!out) return NCC_ERR_INVALID_ARGUMENT;
+  *out = nullptr;
+  if (!p) return NCC_ERR_INVALID_ARGUMENT;
+  ncc_status st = validate(*p);
+  if (st) return st;
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaGetDeviceCount");
+  if (device < 0 || device >= ndev) return NCC_ERR_INVALID_ARGUMENT;
+  DeviceGuard g(device);
+  ncc_plan pl = new (std::nothrow) ncc_plan_s();
+  if (!pl) return NCC_ERR_OUT_OF_MEMORY;
+  pl->p = *p;
+  pl->device = device;
+  memset(&pl->info, 0, sizeof(pl->info));
+  pl->info.mode = p->mode;
+  pl->info.batch = p->batch;
+  st = p->mode == NCC_MODE_MATCH ? create_tm(pl) : create_piv(pl);
+  if (st) {
+    free_plan(pl);
+    return st;
+  }
+  *out = pl;
+  return NCC_OK;
+}
+
+ncc_status ncc_plan_destroy(ncc_plan pl) {
+  if (!pl) return NCC_OK;
+  DeviceGuard g(pl->device);
+  cudaDeviceSynchronize();
+  free_plan(pl);
+  return NCC_OK;
+}
+
+ncc_status ncc_plan_query(ncc_plan pl, void* info, size_t info_size) {
+  if (!pl || !info) return NCC_ERR_INVALID_ARGUMENT;
+  memcpy(info, &pl->info, info_size < sizeof(ncc_plan_info) ? info_size : sizeof(ncc_plan_info));
+  return NCC_OK;
+}
+
+ncc_status ncc_plan_timing(ncc_plan pl, ncc_timing* out) {
+  if (!pl || !out) return NCC_ERR_INVALID_ARGUMENT;
+  memset(out, 0, sizeof(*out));
+  if (!(pl->p.flags & NCC_F_TIMING) || pl->timing_kind == 0) return NCC_OK;
+  DeviceGuard g(pl->device);
+  float ms = 0.f;
+  if (pl->timing_kind == 1) {
+    NCC_CUDA(cudaEventSynchronize(pl->ev[4]));
+    cudaEventElapsedTime(&ms, pl->ev[0], pl->ev[1]); out->prep_ms = ms;
+    cudaEventElapsedTime(&ms, pl->ev[1], pl->ev[2]); out->stats_ms = ms;
+    cudaEventElapsedTime(&ms, pl->ev[2], pl->ev[3]); out->numerator_ms = ms;
+    cudaEventElapsedTime(&ms, pl->ev[3], pl->ev[4]); out->finalize_ms = ms;
+    cudaEventElapsedTime(&ms, pl->ev[0], pl->ev[4]); out->total_ms = ms;
+    out->numerator_launches = 1;
+  } else {
+    const int nsub = pl->piv_nsub;
+    NCC_CUDA(cudaEventSynchronize(pl->ev[3 * nsub]));
+    cudaEvent_t prev = pl->ev[0];
+    for (int sb = 0; sb < nsub; ++sb) {
+      cudaEventElapsedTime(&ms, prev, pl->ev[3 * sb + 1]); out->stats_ms += ms;
+      cudaEventElapsedTime(&ms, pl->ev[3 * sb + 1], pl->ev[3 * sb + 2]); out->numerator_ms += ms;
+      prev = pl->ev[3 * sb + 3];
+    }
+    cudaEventElapsedTime(&ms, pl->ev[0], pl->ev[3 * nsub]); out->total_ms = ms;
+    out->numerator_launches = nsub;
+  }
+  return NCC_OK;
+}
+
+ncc_status ncc_match(ncc_plan pl, const float* d_images, const float* d_tmpl, int64_t tmpl_pitch, float* d_scores,
+                     ncc_peak* d_peaks, void* stream) {
+  if (!pl) return NCC_ERR_INVALID_ARGUMENT;
+  if (pl->p.mode != NCC_MODE_MATCH) return NCC_ERR_WRONG_MODE;
+  if (!d_images || !d_tmpl || !d_peaks || tmpl_pitch < pl->p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
+  if ((pl->p.flags & NCC_F_WRITE_SURFACE) && !d_scores) return NCC_ERR_INVALID_ARGUMENT;
+  DeviceGuard g(pl->device);
+  return run_match(pl, d_images, d_tmpl, tmpl_pitch, d_scores, d_peaks, (cudaStream_t)stream);
+}
+
+ncc_status piv_correlate_ex(ncc_plan pl, const float* d_a, const float* d_b, float* d_scores, piv_vector* d_vec,
+                            void* stream) {
+  if (!pl) return NCC_ERR_INVALID_ARGUMENT;
+  if (pl->p.mode != NCC_MODE_PIV) return NCC_ERR_WRONG_MODE;
+  if (!d_a || !d_b || !d_vec) return NCC_ERR_INVALID_ARGUMENT;
+  DeviceGuard g(pl->device);
+  return run_piv(pl, d_a, d_b, d_scores, d_vec, (cudaStream_t)stream);
+}
+
+ncc_status piv_correlate(ncc_plan pl, const float* d_a, const float* d_b, piv_vector* d_vec, void* stream) {
+  return piv_correlate_ex(pl, d_a, d_b, nullptr, d_vec, stream);
+}
+
+ncc_status ncc_match_host(ncc_plan pl, const float* h_images, const float* h_tmpl, int64_t tmpl_pitch,
+                          float* h_scores, ncc_peak* h_peaks, void* stream) {
+  if (!pl) return NCC_ERR_INVALID_ARGUMENT;
+  if (pl->p.mode != NCC_MODE_MATCH) return NCC_ERR_WRONG_MODE;
+  const ncc_problem& p = pl->p;
+  if (!h_images || !h_tmpl || !h_peaks || tmpl_pitch < p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
+  DeviceGuard g(pl->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t img_bytes = (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float);
+  const size_t t_bytes = (size_t)p.tmpl_h * p.tmpl_w * sizeof(float);
+  const bool surf = (p.flags & NCC_F_WRITE_SURFACE) != 0;
+  const size_t s_bytes = surf ? (size_t)p.batch * pl->Ub * pl->V * sizeof(float) : 0;
+  ncc_status st;
+  if ((st = stage((void**)&pl->st_a, &pl->st_a_bytes, img_bytes))) return st;
+  if ((st = stage((void**)&pl->st_t, &pl->st_t_bytes, t_bytes))) return st;
+  if (surf && (st = stage((void**)&pl->st_s, &pl->st_s_bytes, s_bytes))) return st;
+  if ((st = stage(&pl->st_out, &pl->st_out_bytes, (size_t)p.batch * sizeof(ncc_peak)))) return st;
+  NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_images, img_bytes, cudaMemcpyHostToDevice, s));
+  NCC_CUDA(cudaMemcpy2DAsync(pl->st_t, p.tmpl_w * sizeof(float), h_tmpl, tmpl_pitch * sizeof(float),
+                             p.tmpl_w * sizeof(float), p.tmpl_h, cudaMemcpyHostToDevice, s));
+  st = run_match(pl, pl->st_a, pl->st_t, p.tmpl_w, pl->st_s, (ncc_peak*)pl->st_out, s);
+  if (st) return st;
+  NCC_CUDA(cudaMemcpyAsync(h_peaks, pl->st_out, (size_t)p.batch * sizeof(ncc_peak), cudaMemcpyDeviceToHost, s));
+  if (surf && h_scores) NCC_CUDA(cudaMemcpyAsync(h_scores, pl->st_s, s_bytes, cudaMemcpyDeviceToHost, s));
+  return NCC_OK;
+}
+
+ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, piv_vector* h_vec, void* stream) {
+  if (!pl) return NCC_ERR_INVALID_ARGUMENT;
+  if (pl->p.mode != NCC_MODE_PIV) return NCC_ERR_WRONG_MODE;
+  const ncc_problem& p = pl->p;
+  if (!h_a || !h_b || !h_vec) return NCC_ERR_INVALID_ARGUMENT;
+  DeviceGuard g(pl->device);
+  cudaStream_t s = (cudaStream_t)stream;
+  const size_t fb = (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float);
+  const size_t vb = (size_t)p.batch * pl->Ky * pl->Kx * sizeof(piv_vector);
+  ncc_status st;
+  if ((st = stage((void**)&pl->st_a, &pl->st_a_bytes, fb))) return st;
+  if ((st = stage((void**)&pl->st_b, &pl->st_b_bytes, fb))) return st;
+  if ((st = stage(&pl->st_out, &pl->st_out_bytes, vb))) return st;
+  NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_a, fb, cudaMemcpyHostToDevice, s));
+  NCC_CUDA(cudaMemcpyAsync(pl->st_b, h_b, fb, cudaMemcpyHostToDevice, s));
+  st = run_piv(pl, pl->st_a, pl->st_b, nullptr, (piv_vector*)pl->st_out, s);
+  if (st) return st;
+  NCC_CUDA(cudaMemcpyAsync(h_vec, pl->st_out, vb, cudaMemcpyDeviceToHost, s));
+  return NCC_OK;
+}
+
+}  // extern "C"

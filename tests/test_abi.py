@@ -1,0 +1,97 @@
+"""C-ABI library checks that need no GPU: it loads, exports every symbol include/ncc.h
+declares, struct layouts match, and argument validation runs before any device work."""
+import ctypes
+import os
+import re
+
+import pytest
+
+from paper_conf_ipps_moorelk13_b200 import _native as N
+from paper_conf_ipps_moorelk13_b200 import build as B
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def L():
+    B.build()
+    return N.lib()
+
+
+def declared_functions():
+    src = open(os.path.join(ROOT, "include", "ncc.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"^\s*(?:ncc_status|const char\*|int32_t)\s+(\w+)\s*\(", src, flags=re.M)))
+
+
+def test_exports_every_declared_symbol(L):
+    names = declared_functions()
+    assert len(names) >= 12
+    for n in names:
+        assert hasattr(L, n), n
+    assert set(names) == set(N.EXPORTS)
+
+
+def test_build_arch(L):
+    assert L.ncc_build_arch() == 100
+
+
+def test_struct_sizes():
+    assert ctypes.sizeof(N.NccPeak) == 16
+    assert ctypes.sizeof(N.PivVector) == 24
+    assert ctypes.sizeof(N.NccProblem) == 72  # 5 x i32, pad, i64, 10 x 32-bit
+
+
+def test_sm100a_cubin_in_library(L):
+    import subprocess
+    out = subprocess.run(["cuobjdump", "--list-elf", N.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_status_strings(L):
+    for k, v in N.STATUS.items():
+        assert N.ncc_status_string(k) == v
+
+
+def _create(**kw):
+    base = dict(mode=N.NCC_MODE_MATCH, image_h=64, image_w=64, tmpl_h=16, tmpl_w=16)
+    base.update(kw)
+    p = N.make_problem(**base)
+    h = ctypes.c_void_p()
+    return N.lib().ncc_plan_create(ctypes.byref(p), 0, ctypes.byref(h)), h.value
+
+
+@pytest.mark.parametrize("kw", [
+    dict(tmpl_h=65), dict(tmpl_w=0), dict(image_h=0), dict(image_pitch=10), dict(batch=0),
+    dict(shard_count=0), dict(shard_rank=2, shard_count=2), dict(search_y=3),
+    dict(mode=N.NCC_MODE_PIV, search_y=-1, search_x=2, step_y=4, step_x=4),
+    dict(mode=N.NCC_MODE_PIV, search_y=40, search_x=2, step_y=4, step_x=4),
+    dict(mode=N.NCC_MODE_PIV, search_y=2, search_x=2, step_y=0, step_x=4),
+    dict(mode=N.NCC_MODE_PIV, search_y=2, search_x=2, step_y=4, step_x=4, shard_count=2),
+    dict(mode=7), dict(shard_count=50, shard_rank=0),
+])
+def test_invalid_arguments_rejected_before_device(L, kw):
+    st, h = _create(**kw)
+    assert st == 1 and not h  # NCC_ERR_INVALID_ARGUMENT, *out == NULL
+
+
+def test_ssd_unsupported(L):
+    st, h = _create(score=N.NCC_SCORE_SSD)
+    assert st == 2 and not h
+
+
+def test_null_arguments(L):
+    assert L.ncc_plan_create(None, 0, None) == 1
+    assert L.ncc_plan_destroy(None) == 0
+    assert L.ncc_match(None, None, None, 16, None, None, None) == 1
+    assert L.piv_correlate(None, None, None, None, None) == 1
+    assert L.ncc_plan_query(None, None, 0) == 1
+
+
+def test_product_package_does_not_import_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_ipps_moorelk13_b200")
+    for dp, _, fs in os.walk(pkg):
+        for f in fs:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                txt = open(os.path.join(dp, f)).read()
+                assert "import oracle" not in txt and "from oracle" not in txt and "ncc_oracle" not in txt, f

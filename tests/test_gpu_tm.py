@@ -1,0 +1,178 @@
+"""GPU parity: template matching (TM) through the C ABI vs the fp64 oracle.
+
+Bar (BASELINE.json north_star): max |dNCC| <= 1e-4 element by element; peak locations
+bit-exact on planted inputs.  Sizes: the oracle full surface where it finishes in seconds
+(several tiles + ragged tails), and at full BASELINE sizes the independent FFT route
+(itself pinned to the brute force in test_oracle.py) plus brute-force samples.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from oracle.ncc_fft import ncc_surface_fft
+import synth
+from paper_conf_ipps_moorelk13_b200 import build as B
+from paper_conf_ipps_moorelk13_b200.api import MatchPlan, decode_peaks
+
+pytestmark = pytest.mark.gpu
+TOL = 1e-4
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _lib():
+    B.build()
+
+
+def run_match(img, T, generic=False, batch_imgs=None, shard=(0, 1)):
+    imgs = np.stack(batch_imgs) if batch_imgs is not None else img[None]
+    H, W = imgs.shape[1:]
+    h, w = T.shape
+    dev = torch.device("cuda", 0)
+    with MatchPlan(H, W, h, w, batch=imgs.shape[0], write_surface=True, generic=generic,
+                   shard_rank=shard[0], shard_count=shard[1]) as plan:
+        d_img = torch.from_numpy(imgs).to(dev)
+        d_t = torch.from_numpy(np.ascontiguousarray(T)).to(dev)
+        peaks, scores = plan.match(d_img, d_t)
+        torch.cuda.synchronize()
+        info = plan.info.as_dict()
+        return {k: v.cpu().numpy() for k, v in decode_peaks(peaks).items()}, scores.cpu().numpy(), info
+
+
+@pytest.mark.parametrize("generic", [False, True])
+def test_cfg1_full_surface(generic):
+    img, T, u0, v0 = synth.tm_inputs(1)
+    ref, pk = oracle.ncc_match(img, T)
+    peaks, s, info = run_match(img, T, generic)
+    assert info["specialized"] == (0 if generic else 1)
+    assert np.max(np.abs(s[0] - ref)) <= TOL
+    assert (peaks["u"][0], peaks["v"][0]) == (u0, v0) == (pk.u, pk.v)
+    assert peaks["flags"][0] == 0
+    assert abs(peaks["score"][0] - 1.0) <= TOL
+
+
+@pytest.mark.parametrize("H,W,h,w,smooth", [(100, 137, 23, 17, False), (157, 123, 33, 41, True),
+                                            (300, 280, 156, 116, False), (70, 90, 1, 1, False),
+                                            (64, 64, 64, 64, False), (41, 300, 7, 290, False)])
+def test_generic_ragged_shapes(H, W, h, w, smooth):
+    img = synth.smooth_image(H, W, 7) if smooth else synth.uniform_image(H, W, 7)
+    T, u0, v0 = synth.planted_template(img, h, w, 8)
+    ref, pk = oracle.ncc_match(img, T)
+    peaks, s, info = run_match(img, T)
+    assert info["specialized"] == 0
+    assert np.max(np.abs(s[0] - ref)) <= TOL
+    if h * w > 1:
+        assert (peaks["u"][0], peaks["v"][0]) == (u0, v0)
+
+
+@pytest.mark.parametrize("smooth", [False, True])
+def test_cfg2_full_surface_fft_and_samples(smooth):
+    img, T, u0, v0 = synth.tm_inputs(2, smooth=smooth)
+    peaks, s, info = run_match(img, T)
+    assert info["specialized"] == 1
+    f = ncc_surface_fft(img, T)
+    assert np.max(np.abs(s[0] - f)) <= TOL
+    g = synth.rng(99)
+    us = np.concatenate([g.integers(0, 897, 300), np.arange(u0 - 2, u0 + 3).repeat(5), [0, 896, 896]])
+    vs = np.concatenate([g.integers(0, 897, 300), np.tile(np.arange(v0 - 2, v0 + 3), 5), [896, 0, 896]])
+    ok = (us >= 0) & (us < 897) & (vs >= 0) & (vs < 897)
+    us, vs = us[ok], vs[ok]
+    bf = oracle.ncc_at(img, T, us, vs)
+    assert np.max(np.abs(s[0][us, vs] - bf)) <= TOL
+    assert (peaks["u"][0], peaks["v"][0]) == (u0, v0)
+
+
+def test_cfg2_rows_vs_bruteforce_band():
+    img, T, u0, v0 = synth.tm_inputs(2, k=1)
+    peaks, s, _ = run_match(img, T)
+    ref = oracle.ncc_surface(img, T, 0, 40)  # full rows, all columns, including the ragged tail
+    assert np.max(np.abs(s[0][:40] - ref)) <= TOL
+
+
+@pytest.mark.slow
+def test_cfg5_full_surface_fft_and_samples():
+    img, T, u0, v0 = synth.tm_inputs(5)
+    peaks, s, info = run_match(img, T)
+    assert info["specialized"] == 1
+    f = ncc_surface_fft(img, T)
+    assert np.max(np.abs(s[0] - f)) <= TOL
+    g = synth.rng(98)
+    us = np.concatenate([g.integers(0, 3585, 48), [u0, u0 - 1, u0 + 1, 3584, 0]])
+    vs = np.concatenate([g.integers(0, 3585, 48), [v0, v0 + 1, v0 - 1, 3584, 3584]])
+    bf = oracle.ncc_at(img, T, us, vs)
+    assert np.max(np.abs(s[0][us, vs] - bf)) <= TOL
+    assert (peaks["u"][0], peaks["v"][0]) == (u0, v0)
+
+
+def test_batch_frames_and_host_path():
+    imgs = [synth.uniform_image(200, 180, 40 + k) for k in range(3)]
+    T, _, _ = synth.planted_template(imgs[1], 24, 20, 3)
+    peaks, s, _ = run_match(None, T, batch_imgs=imgs)
+    for k in range(3):
+        ref, pk = oracle.ncc_match(imgs[k], T)
+        assert np.max(np.abs(s[k] - ref)) <= TOL
+        assert (peaks["u"][k], peaks["v"][k]) == (pk.u, pk.v)
+    # host-buffer entry point gives the same peaks
+    stack = torch.from_numpy(np.stack(imgs)).pin_memory()
+    tt = torch.from_numpy(T).pin_memory()
+    hp = torch.empty((3, 4), dtype=torch.int32).pin_memory()
+    with MatchPlan(200, 180, 24, 20, batch=3) as plan:
+        plan.match_host(stack, tt, hp)
+        torch.cuda.synchronize()
+    d = decode_peaks(hp)
+    np.testing.assert_array_equal(d["u"].numpy(), peaks["u"])
+    np.testing.assert_array_equal(d["v"].numpy(), peaks["v"])
+    np.testing.assert_array_equal(d["score"].numpy(), peaks["score"])
+
+
+def test_band_shards_cover_and_merge():
+    img, T, u0, v0 = synth.tm_inputs(1, k=3)
+    full_peaks, full, _ = run_match(img, T)
+    parts, keys = [], []
+    for r in range(3):
+        pk, s, info = run_match(img, T, shard=(r, 3))
+        assert s.shape[1] == info["u_end"] - info["u_begin"]
+        parts.append(s[0])
+        keys.append((pk["score"][0], -(pk["u"][0] * 49 + pk["v"][0]), pk["u"][0], pk["v"][0]))
+    np.testing.assert_array_equal(np.concatenate(parts, axis=0), full[0])  # bitwise: order independent of band
+    best = max(keys)
+    assert (best[2], best[3]) == (full_peaks["u"][0], full_peaks["v"][0]) == (u0, v0)
+
+
+def test_flat_template_and_flat_windows():
+    img = synth.uniform_image(80, 90, 50)
+    img[10:40, 20:60] = 0.25
+    T = synth.uniform_image(8, 8, 51)
+    peaks, s, _ = run_match(img, T)
+    ref = oracle.ncc_surface(img, T)
+    assert np.max(np.abs(s[0] - ref)) <= TOL
+    assert np.all(s[0][10:33, 20:53] == 0.0)
+    Tf = np.full((8, 8), 0.5, np.float32)
+    peaks, s, _ = run_match(img, Tf)
+    assert np.all(s[0] == 0.0)
+    assert peaks["flags"][0] & 1 and peaks["flags"][0] & 32
+    assert (peaks["u"][0], peaks["v"][0]) == (0, 0)
+
+
+def test_tie_break_smallest_index():
+    # periodic image: the template matches exactly at several offsets -> smallest u*V+v
+    tile = synth.quantize(synth.uniform_image(8, 8, 60))  # exact window sums -> bitwise-equal ties
+    img = np.tile(tile, (6, 6))
+    T = np.ascontiguousarray(img[8:16, 8:16])
+    peaks, s, _ = run_match(img, T)
+    ones = np.argwhere(s[0] >= 1.0 - 1e-6)
+    assert len(ones) > 1
+    assert (peaks["u"][0], peaks["v"][0]) == tuple(ones[0])
+
+
+def test_timing_and_info():
+    img, T, _, _ = synth.tm_inputs(2)
+    dev = torch.device("cuda", 0)
+    with MatchPlan(1024, 1024, 128, 128, timing=True) as plan:
+        d_img = torch.from_numpy(img).to(dev)
+        d_t = torch.from_numpy(T).to(dev)
+        plan.match(d_img, d_t)
+        t = plan.timing()
+        assert t.numerator_ms > 0 and t.total_ms >= t.numerator_ms and t.numerator_launches == 1
+        assert plan.info.regs_per_thread > 0
+        assert abs(plan.info.flops_per_call - 2 * 128 * 128 * 897 * 897) < 1
