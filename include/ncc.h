@@ -89,7 +89,8 @@ typedef struct {
     int32_t step_y;  /* PIV: window step s_y (= (1-overlap)*window); TM: ignored           */
     int32_t step_x;  /* PIV: window step s_x                                               */
     int32_t batch;   /* TM: frames per call; PIV: frame pairs per call (per shard)        */
-    int32_t shard_rank;  /* TM: this rank's band of offset rows; PIV: must be 0            */
+    int32_t shard_rank;  /* TM: band r = offset rows [r*U/n, (r+1)*U/n), n = shard_count;  */
+                         /*     PIV: must be 0 (shard PIV by passing each rank its pairs) */
     int32_t shard_count; /* >= 1                                                            */
     uint32_t flags;  /* NCC_F_*                                                              */
 } ncc_problem;

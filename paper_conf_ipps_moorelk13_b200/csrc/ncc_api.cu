@@ -194,9 +194,9 @@ ncc_status create_tm(ncc_plan pl) {
   const int h = p.tmpl_h, w = p.tmpl_w;
   pl->U = p.image_h - h + 1;
   pl->V = p.image_w - w + 1;
-  const int band = ceil_div(pl->U, p.shard_count);
-  pl->u_begin = p.shard_rank * band;
-  pl->u_end = pl->u_begin + band < pl->U ? pl->u_begin + band : pl->U;
+  // balanced contiguous bands of offset rows: [r*U/n, (r+1)*U/n) (every band non-empty for n <= U)
+  pl->u_begin = (int)((int64_t)p.shard_rank * pl->U / p.shard_count);
+  pl->u_end = (int)((int64_t)(p.shard_rank + 1) * pl->U / p.shard_count);
   if (pl->u_begin >= pl->u_end) return NCC_ERR_INVALID_ARGUMENT;
   pl->Ub = pl->u_end - pl->u_begin;
   pl->Hs = pl->Ub + h - 1;

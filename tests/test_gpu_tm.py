@@ -13,6 +13,7 @@ import oracle
 from oracle.ncc_fft import ncc_surface_fft
 import synth
 from paper_conf_ipps_moorelk13_b200 import build as B
+from paper_conf_ipps_moorelk13_b200 import shard
 from paper_conf_ipps_moorelk13_b200.api import MatchPlan, decode_peaks
 
 pytestmark = pytest.mark.gpu
@@ -132,6 +133,7 @@ def test_band_shards_cover_and_merge():
     for r in range(3):
         pk, s, info = run_match(img, T, shard=(r, 3))
         assert s.shape[1] == info["u_end"] - info["u_begin"]
+        assert (info["u_begin"], info["u_end"]) == shard.band_range(49, r, 3)
         parts.append(s[0])
         keys.append((pk["score"][0], -(pk["u"][0] * 49 + pk["v"][0]), pk["u"][0], pk["v"][0]))
     np.testing.assert_array_equal(np.concatenate(parts, axis=0), full[0])  # bitwise: order independent of band
