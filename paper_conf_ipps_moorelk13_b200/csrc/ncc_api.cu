@@ -44,15 +44,19 @@ struct TmVariant {
   const char* name;
   int TH, TW;                 // 0 = run-time (RE)
   int RV, LX, WX, WY, CH, CW;
-  void (*kernel)(TmArgs);
-  int nt, bu, bv, smem;
+  void (*k_tma)(TmArgs, CUtensorMap, CUtensorMap);
+  void (*k_ldg)(TmArgs, CUtensorMap, CUtensorMap);
+  int nt, bu, bv, ir, ip, smem_tma, smem_ldg;
+  int rv_nt() const { return RV * nt; }
 };
 
 #define TM_VARIANT(NAME, TH, TW, RV, LX, WX, WY, CH, CW)                                                  \
   TmVariant {                                                                                          \
-    NAME, TH, TW, RV, LX, WX, WY, CH, CW, tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW>,                 \
-        TmTile<RV, LX, WX, WY, CH, CW>::NT, TmTile<RV, LX, WX, WY, CH, CW>::BU,                        \
-        TmTile<RV, LX, WX, WY, CH, CW>::BV, TmTile<RV, LX, WX, WY, CH, CW>::SMEM                       \
+    NAME, TH, TW, RV, LX, WX, WY, CH, CW, tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW, true>,           \
+        tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW, false>, TmTile<RV, LX, WX, WY, CH, CW>::NT,         \
+        TmTile<RV, LX, WX, WY, CH, CW>::BU, TmTile<RV, LX, WX, WY, CH, CW>::BV,                           \
+        TmTile<RV, LX, WX, WY, CH, CW>::IR, TmTile<RV, LX, WX, WY, CH, CW>::IP,                           \
+        TmTile<RV, LX, WX, WY, CH, CW>::SMEM_TMA, TmTile<RV, LX, WX, WY, CH, CW>::SMEM_LDG                \
   }
 
 const TmVariant kTmVariants[] = {
@@ -63,6 +67,41 @@ const TmVariant kTmVariants[] = {
     TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c32x64", 128, 128, 12, 4, 1, 4, 32, 64),
     TM_VARIANT("tm_sk_512x512_rv12_lx4_4x1_c32x64", 512, 512, 12, 4, 1, 4, 32, 64),
 };
+
+// cuTensorMapEncodeTiled through the runtime's driver entry point (no -lcuda needed).
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                  const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                  CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+EncodeTiledFn encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  }
+  return fn;
+}
+
+// fp32 tensor map of `rank` dims (innermost first), strides in bytes for dims 1..rank-1.
+bool encode_f32(CUtensorMap* m, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
+                const uint32_t* box) {
+  EncodeTiledFn fn = encode_fn();
+  if (!fn) return false;
+  cuuint64_t gd[3], gs[2];
+  cuuint32_t bx[3], es[3] = {1, 1, 1};
+  for (int i = 0; i < rank; ++i) {
+    gd[i] = dims[i];
+    bx[i] = box[i];
+  }
+  for (int i = 0; i + 1 < rank; ++i) gs[i] = strides_bytes[i];
+  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (cuuint32_t)rank, const_cast<void*>(base), gd, gs, bx, es,
+            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+}
 
 struct PivVariant {
   const char* name;
@@ -93,6 +132,11 @@ struct ncc_plan_s {
   ncc_plan_info info;
   // TM
   int U, V, u_begin, u_end, Ub, Hs, HP, WP;
+  int tiles_u, tiles_v, split;
+  bool tma_ok;
+  CUtensorMap map_tpl;
+  float* part;
+  unsigned int* cnt;
   const TmVariant* tmv;
   float* tplC;
   TemplateStats* tst;
@@ -129,6 +173,8 @@ struct DeviceGuard {
 
 void free_plan(ncc_plan pl) {
   cudaFree(pl->tplC);
+  cudaFree(pl->part);
+  cudaFree(pl->cnt);
   cudaFree(pl->tst);
   cudaFree(pl->keys);
   cudaFree(pl->RS1);
@@ -210,25 +256,64 @@ ncc_status create_tm(ncc_plan pl) {
   pl->HP = nCH * v->CH;
   pl->WP = nCW * v->CW;
 
-  int maxsm = 0;
+  int maxsm = 0, nsm = 0;
   NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
-  if (v->smem > maxsm) return NCC_ERR_UNSUPPORTED;
-  NCC_CUDA(cudaFuncSetAttribute((const void*)v->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, v->smem));
+  NCC_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, pl->device));
+  if (v->smem_tma > maxsm || v->smem_ldg > maxsm) return NCC_ERR_UNSUPPORTED;
+  NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, v->smem_tma));
+  NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, v->smem_ldg));
   const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
   if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
   NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT, kBoxRowsSEG>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem));
 
+  // tiles of this band; split-K factor S from the FULL problem's tile count (so every shard
+  // of a problem uses the same S and the same per-offset accumulation order): the smallest
+  // S <= chunks whose unit count fills whole "rounds" of resident CTAs to >= 97 %.
+  pl->tiles_u = ceil_div(pl->Ub, v->bu);
+  pl->tiles_v = ceil_div(pl->V, v->bv);
+  {
+    int per_sm = 0;
+    NCC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, v->k_tma, v->nt, v->smem_tma));
+    const int64_t slots = (int64_t)(per_sm > 0 ? per_sm : 1) * nsm;
+    const int64_t tiles_full = (int64_t)ceil_div(pl->U, v->bu) * ceil_div(pl->V, v->bv);
+    const int nq = nCH * nCW;
+    int best_s = 1;
+    double best_e = 0.0;
+    for (int S = 1; S <= nq && S <= 8; ++S) {
+      const int64_t units = tiles_full * S;
+      const double e = (double)units / (double)(((units + slots - 1) / slots) * slots);
+      if (e > best_e + 0.02) {
+        best_e = e;
+        best_s = S;
+      }
+      if (e >= 0.97) break;
+    }
+    pl->split = best_s;
+  }
+
   ncc_status st;
   if ((st = dalloc(&pl->tplC, (size_t)pl->HP * pl->WP))) return st;
   if ((st = dalloc(&pl->tst, 1))) return st;
   if ((st = dalloc(&pl->keys, (size_t)p.batch))) return st;
+  const int64_t ntiles = (int64_t)pl->tiles_u * pl->tiles_v * p.batch;
+  if (pl->split > 1) {
+    if ((st = dalloc(&pl->part, (size_t)ntiles * pl->split * v->rv_nt()))) return st;
+    if ((st = dalloc(&pl->cnt, (size_t)ntiles))) return st;
+    NCC_CUDA(cudaMemset(pl->cnt, 0, (size_t)ntiles * sizeof(unsigned int)));
+  }
   pl->rs_frame_stride = (int64_t)pl->Hs * pl->V;
   pl->s_frame_stride = (int64_t)pl->Ub * pl->V;
   if ((st = dalloc(&pl->RS1, (size_t)p.batch * pl->rs_frame_stride))) return st;
   if ((st = dalloc(&pl->RS2, (size_t)p.batch * pl->rs_frame_stride))) return st;
   if ((st = dalloc(&pl->S1, (size_t)p.batch * pl->s_frame_stride))) return st;
   if ((st = dalloc(&pl->S2, (size_t)p.batch * pl->s_frame_stride))) return st;
+  {  // template chunks: 2D map over the zero-padded centred template
+    const uint64_t dims[2] = {(uint64_t)pl->WP, (uint64_t)pl->HP};
+    const uint64_t strides[1] = {(uint64_t)pl->WP * 4};
+    const uint32_t box[2] = {(uint32_t)v->CW, (uint32_t)v->CH};
+    pl->tma_ok = encode_f32(&pl->map_tpl, pl->tplC, 2, dims, strides, box);
+  }
 
   ncc_plan_info& in = pl->info;
   in.U = pl->U;
@@ -240,8 +325,9 @@ ncc_status create_tm(ncc_plan pl) {
   in.specialized = v->TH != 0;
   in.variant_id = (int)(v - kTmVariants);
   snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
-  fill_kernel_info(pl, (const void*)v->kernel, v->nt, v->smem, ceil_div(pl->V, v->bv), ceil_div(pl->Ub, v->bu),
-                   p.batch);
+  snprintf(in.variant_name + strlen(in.variant_name), sizeof(in.variant_name) - strlen(in.variant_name), "_s%d",
+           pl->split);
+  fill_kernel_info(pl, (const void*)v->k_tma, v->nt, v->smem_tma, pl->tiles_u * pl->tiles_v * pl->split, p.batch, 1);
   return NCC_OK;
 }
 
@@ -366,11 +452,29 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   a.V = pl->V;
   a.u_begin = pl->u_begin;
   a.u_end = pl->u_end;
+  a.tiles_u = pl->tiles_u;
+  a.tiles_v = pl->tiles_v;
   a.scores = (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr;
   a.score_frame_stride = (int64_t)pl->Ub * pl->V;
   a.keys = pl->keys;
-  dim3 grid(ceil_div(pl->V, v->bv), ceil_div(pl->Ub, v->bu), p.batch);
-  v->kernel<<<grid, v->nt, v->smem, s>>>(a);
+  a.part = pl->part;
+  a.cnt = pl->cnt;
+  a.S = pl->split;
+  // TMA needs a 16-B aligned base and a pitch that is a multiple of 16 B; else plain loads.
+  CUtensorMap map_img;
+  memset(&map_img, 0, sizeof(map_img));
+  bool use_tma = pl->tma_ok && (reinterpret_cast<uintptr_t>(d_images) % 16 == 0) && (p.image_pitch % 4 == 0);
+  if (use_tma) {
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
+    const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)p.image_h * p.image_pitch * 4};
+    const uint32_t box[3] = {(uint32_t)v->ip, (uint32_t)v->ir, 1u};
+    use_tma = encode_f32(&map_img, d_images, 3, dims, strides, box);
+  }
+  dim3 grid(pl->tiles_u * pl->tiles_v * pl->split, p.batch);
+  if (use_tma)
+    v->k_tma<<<grid, v->nt, v->smem_tma, s>>>(a, map_img, pl->map_tpl);
+  else
+    v->k_ldg<<<grid, v->nt, v->smem_ldg, s>>>(a, map_img, pl->map_tpl);
   mark(pl, s, 3);
   tm_finalize<<<ceil_div(p.batch, 128), 128, 0, s>>>(pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks),
                                                      p.batch);

@@ -20,6 +20,7 @@
 // running total, bounding fp32 error growth.  Denominator from fp64 window
 // sums; normalisation in fp64; packed 64-bit (score, -index) keys for a deterministic argmax.
 #pragma once
+#include <cuda.h>  // CUtensorMap (type only; encoded on the host through the runtime entry point)
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -117,6 +118,49 @@ __device__ __forceinline__ float ncc_normalize(float num, double s1, double s2, 
   return (float)r;
 }
 
+
+// ------------------------------------------------------------------ TMA / mbarrier (sm_100a PTX)
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void fence_mbar_init() {
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "@!P bra WAIT_%=;\n}" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+// 2D / 3D tiled TMA loads global -> shared, completion on an mbarrier (out-of-bounds = 0).
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::
+          "r"(smem_u32(dst)),
+      "l"(map), "r"(x), "r"(y), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_3d(void* dst, const CUtensorMap* map, int x, int y, int z, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];" ::
+          "r"(smem_u32(dst)),
+      "l"(map), "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void tma_prefetch_desc(const CUtensorMap* map) {
+  asm volatile("prefetch.tensormap [%0];" ::"l"(map) : "memory");
+}
+
 // ------------------------------------------------------------------ numerator core
 // acc[c] += sum_{j<CW} tpl[j] * img[c + j],  c < RV.
 // img: shared, 16-B aligned, >= RV + CW readable values; tpl: shared, 16-B aligned (broadcast).
@@ -185,9 +229,13 @@ struct TmArgs {
   int64_t stat_frame_stride;
   const TemplateStats* tst;
   int U, V, u_begin, u_end;
+  int tiles_u, tiles_v;      // output tiles of the band
   float* scores;             // nullable: [batch][u_end-u_begin][V]
   int64_t score_frame_stride;
   unsigned long long* keys;  // [batch] argmax keys (reset by tm_template_prep)
+  float* part;               // split-K partial totals [batch][tiles][S][RV][NT]   (S > 1)
+  unsigned int* cnt;         // split-K arrival counters [batch][tiles], zero between calls
+  int S;                     // split-K factor (fixed per variant: accumulation order depends on it)
 };
 
 template <int RV, int LX, int WX, int WY, int CH, int CW>
@@ -196,21 +244,33 @@ struct TmTile {
   static constexpr int LY = 32 / LX;
   static constexpr int BU = WY * LY;              // output rows per CTA
   static constexpr int BV = WX * LX * RV;         // output cols per CTA
-  static constexpr int IR = BU + CH - 1;          // staged image rows
-  static constexpr int IP = pick_pitch(BV + CW, RV, LX);  // staged image pitch (floats)
-  static constexpr int SMEM = (CH * CW + IR * IP) * 4;
+  static constexpr int IR = BU + CH - 1;          // staged image rows (= TMA box rows)
+  static constexpr int IP = pick_pitch(BV + CW, RV, LX);  // staged image pitch (= TMA box cols)
+  static constexpr int T_BYTES = CH * CW * 4;
+  static constexpr int I_BYTES = IR * IP * 4;
+  static constexpr int STAGE = ((T_BYTES + 127) / 128) * 128 + ((I_BYTES + 127) / 128) * 128;
+  static constexpr int SMEM_TMA = 2 * STAGE;      // double-buffered (TMA path)
+  static constexpr int SMEM_LDG = T_BYTES + I_BYTES;
+  static_assert(IR <= 256 && IP <= 256 && CW <= 256 && CH <= 256, "TMA box dims are limited to 256");
 };
 
 // Numerator + fused normalise / clamp / optional surface store / CTA argmax (Fig 5.3-5.6).
 // TH, TW: compile-time template size (specialised, "SK") or 0 (run-time evaluated, "RE").
-template <int RV, int LX, int WX, int WY, int CH, int CW, int TH, int TW>
+// S: split of the (row-chunk, col-chunk) sequence of a tile over S CTAs; chunk ranges are fixed
+//    per tile and the S partial totals are combined in index order by the last CTA to arrive, so
+//    the result is deterministic and independent of scheduling and of the band (shard).
+// TMA: stage image / template chunks with double-buffered cp.async.bulk.tensor + mbarrier;
+//      otherwise (pitch not 16-B aligned) plain coalesced loads, single buffer.
+// One CTA = one (tile, split) unit: blockIdx.x = tile * S + split, blockIdx.y = frame.
+template <int RV, int LX, int WX, int WY, int CH, int CW, int TH, int TW, bool TMA>
 __global__ void __launch_bounds__(WX* WY * 32)
-    tm_ncc_kernel(const TmArgs a) {
+    tm_ncc_kernel(const TmArgs a, const __grid_constant__ CUtensorMap map_img,
+                  const __grid_constant__ CUtensorMap map_tpl) {
   using T = TmTile<RV, LX, WX, WY, CH, CW>;
-  extern __shared__ float4 smem_f4[];
-  float* Ts = reinterpret_cast<float*>(smem_f4);  // [CH][CW]
-  float* Is = Ts + CH * CW;                       // [IR][IP]
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
   __shared__ unsigned long long red_key[32];
+  __shared__ __align__(8) uint64_t full_bar[2];
+  __shared__ unsigned int last_flag;
 
   const int h = TH ? TH : a.h;
   const int w = TW ? TW : a.w;
@@ -223,22 +283,71 @@ __global__ void __launch_bounds__(WX* WY * 32)
   const int ly = lane / LX, lx = lane % LX;
   const int lu = wy * T::LY + ly;         // local output row
   const int lv = (wx * LX + lx) * RV;     // local output col (first of RV)
-  const int f = blockIdx.z;
-  const int u0 = a.u_begin + blockIdx.y * T::BU;
-  const int v0 = blockIdx.x * T::BV;
-  const float* img = a.img + (int64_t)f * a.frame_stride;
+  const int f = blockIdx.y;
+  const int S = a.S;
+  const int tile = blockIdx.x / S, split = blockIdx.x % S;
+  const int ty = tile / a.tiles_v, tx = tile % a.tiles_v;
+  const int u0 = a.u_begin + ty * T::BU;
+  const int v0 = tx * T::BV;
+  const int nq = nCH * nCW;
+  const int q0 = (split * nq) / S, q1 = ((split + 1) * nq) / S;  // this unit's chunk range
 
   float total[RV];
 #pragma unroll
   for (int c = 0; c < RV; ++c) total[c] = 0.0f;
 
-  for (int ic = 0; ic < nCH; ++ic) {
-    for (int jc = 0; jc < nCW; ++jc) {
+  auto compute_chunk = [&](const float* Ts, const float* Is) {
+    const float* irow = Is + lu * T::IP + lv;
+#pragma unroll 1
+    for (int i = 0; i < CH; ++i) {
+      float part[RV];
+#pragma unroll
+      for (int c = 0; c < RV; ++c) part[c] = 0.0f;
+      row_dot<RV, CW>(irow + i * T::IP, Ts + i * CW, part);
+#pragma unroll
+      for (int c = 0; c < RV; ++c) total[c] += part[c];
+    }
+  };
+
+  if constexpr (TMA) {
+    auto stage_t = [&](int s) { return reinterpret_cast<float*>(smem_raw + s * T::STAGE); };
+    auto stage_i = [&](int s) {
+      return reinterpret_cast<float*>(smem_raw + s * T::STAGE + ((T::T_BYTES + 127) / 128) * 128);
+    };
+    auto issue = [&](int q, int s) {  // one thread: chunk q -> stage s
+      const int ic = q / nCW, jc = q % nCW;
+      mbar_expect_tx(&full_bar[s], (uint32_t)(T::T_BYTES + T::I_BYTES));
+      tma_load_2d(stage_t(s), &map_tpl, jc * CW, ic * CH, &full_bar[s]);
+      tma_load_3d(stage_i(s), &map_img, v0 + jc * CW, u0 + ic * CH, f, &full_bar[s]);
+    };
+    if (tid == 0) {
+      tma_prefetch_desc(&map_img);
+      tma_prefetch_desc(&map_tpl);
+      mbar_init(&full_bar[0], 1);
+      mbar_init(&full_bar[1], 1);
+      fence_mbar_init();
+    }
+    __syncthreads();
+    if (tid == 0) {
+      if (q0 < q1) issue(q0, 0);
+      if (q0 + 1 < q1) issue(q0 + 1, 1);
+    }
+    for (int q = q0; q < q1; ++q) {
+      const int k = q - q0, s = k & 1;
+      mbar_wait(&full_bar[s], (uint32_t)((k >> 1) & 1));
+      compute_chunk(stage_t(s), stage_i(s));
+      __syncthreads();  // every warp is done with stage s
+      if (tid == 0 && q + 2 < q1) issue(q + 2, s);
+    }
+  } else {
+    float* Ts = reinterpret_cast<float*>(smem_raw);
+    float* Is = Ts + CH * CW;
+    const float* img = a.img + (int64_t)f * a.frame_stride;
+    for (int q = q0; q < q1; ++q) {
+      const int ic = q / nCW, jc = q % nCW;
       __syncthreads();
-      // stage the template chunk (zero-padded in global: no bounds checks)
       const float* tsrc = a.tplC + (int64_t)(ic * CH) * tplP + jc * CW;
       for (int k = tid; k < CH * CW; k += T::NT) Ts[k] = tsrc[(k / CW) * tplP + (k % CW)];
-      // stage image rows [u0 + ic*CH, +IR) x cols [v0 + jc*CW, +IP), zero outside the frame
       const int gr0 = u0 + ic * CH, gc0 = v0 + jc * CW;
       for (int k = tid; k < T::IR * T::IP; k += T::NT) {
         const int r = k / T::IP, c = k % T::IP;
@@ -246,17 +355,30 @@ __global__ void __launch_bounds__(WX* WY * 32)
         Is[k] = (gr < a.H && gc < a.W) ? __ldg(img + (int64_t)gr * a.pitch + gc) : 0.0f;
       }
       __syncthreads();
-      const float* irow = Is + lu * T::IP + lv;
-#pragma unroll 1
-      for (int i = 0; i < CH; ++i) {
-        float part[RV];
-#pragma unroll
-        for (int c = 0; c < RV; ++c) part[c] = 0.0f;
-        row_dot<RV, CW>(irow + i * T::IP, Ts + i * CW, part);
-#pragma unroll
-        for (int c = 0; c < RV; ++c) total[c] += part[c];
-      }
+      compute_chunk(Ts, Is);
     }
+  }
+
+  // ---- split-K combine: partials in fixed split order, by the last unit of the tile
+  if (S > 1) {
+    float* pbase = a.part + (((int64_t)f * a.tiles_u * a.tiles_v + tile) * S) * (RV * T::NT);
+#pragma unroll
+    for (int c = 0; c < RV; ++c) pbase[(int64_t)split * RV * T::NT + c * T::NT + tid] = total[c];
+    __threadfence();
+    __syncthreads();
+    unsigned int* cnt = a.cnt + (int64_t)f * a.tiles_u * a.tiles_v + tile;
+    if (tid == 0) last_flag = (atomicAdd(cnt, 1u) == (unsigned)(S - 1)) ? 1u : 0u;
+    __syncthreads();
+    if (!last_flag) return;
+    __threadfence();
+#pragma unroll
+    for (int c = 0; c < RV; ++c) {
+      float t = 0.0f;
+      for (int sp = 0; sp < S; ++sp)
+        t += (sp == split) ? total[c] : __ldcg(pbase + (int64_t)sp * RV * T::NT + c * T::NT + tid);
+      total[c] = t;
+    }
+    if (tid == 0) *cnt = 0u;  // ready for the next call (stream-ordered)
   }
 
   // ---- fused epilogue: normalise, clamp, optional surface, argmax key
