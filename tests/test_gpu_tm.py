@@ -178,3 +178,32 @@ def test_timing_and_info():
         assert t.numerator_ms > 0 and t.total_ms >= t.numerator_ms and t.numerator_launches == 1
         assert plan.info.regs_per_thread > 0
         assert abs(plan.info.flops_per_call - 2 * 128 * 128 * 897 * 897) < 1
+
+
+def test_unaligned_pitch_uses_plain_loads():
+    """pitch % 4 != 0 -> no TMA (plain-load kernel); same numbers as the oracle."""
+    img, T, u0, v0 = synth.tm_inputs(1, k=7)
+    H, W = img.shape
+    P = W + 3
+    buf = np.zeros((H, P), np.float32)
+    buf[:, :W] = img
+    dev = torch.device("cuda", 0)
+    with MatchPlan(H, W, 16, 16, write_surface=True, image_pitch=P) as plan:
+        peaks, s = plan.match(torch.from_numpy(buf).to(dev), torch.from_numpy(T).to(dev))
+        torch.cuda.synchronize()
+    ref, pk = oracle.ncc_match(img, T)
+    assert np.max(np.abs(s[0].cpu().numpy() - ref)) <= TOL
+    d = decode_peaks(peaks)
+    assert (int(d["u"][0]), int(d["v"][0])) == (u0, v0)
+
+
+def test_cfg2_split_k_bands_bitwise():
+    """Split-K units + band shards: per-offset accumulation order is fixed per problem."""
+    img, T, u0, v0 = synth.tm_inputs(2, k=2)
+    full_peaks, full, info = run_match(img, T)
+    assert info["variant_name"].endswith(tuple(f"_s{k}" for k in range(1, 9)))
+    parts = []
+    for r in range(2):
+        pk, s, inf = run_match(img, T, shard=(r, 2))
+        parts.append(s[0])
+    np.testing.assert_array_equal(np.concatenate(parts, axis=0), full[0])
