@@ -134,8 +134,8 @@ typedef struct {
 
 /* Per-stage device time of the most recent execute call (NCC_F_TIMING plans). */
 typedef struct {
-    float prep_ms;      /* template prep (TM)                                    */
-    float stats_ms;     /* window sums (box statistics, both passes)             */
+    float prep_ms;      /* template prep (TM; side stream, concurrent with stats) */
+    float stats_ms;     /* call start -> window sums and template prep both done  */
     float numerator_ms; /* numerator + fused normalise/argmax (+ PIV sub-pixel)  */
     float finalize_ms;  /* peak finalisation (TM)                                */
     float total_ms;     /* whole call                                            */

@@ -10,6 +10,7 @@
 #include <cuda_runtime.h>
 
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 #include <string>
@@ -65,6 +66,11 @@ const TmVariant kTmVariants[] = {
     // specialised instances for the BASELINE configurations
     TM_VARIANT("tm_sk_16x16_rv4_lx16_4x1_c16x16", 16, 16, 4, 16, 1, 4, 16, 16),
     TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c32x64", 128, 128, 12, 4, 1, 4, 32, 64),
+    // alternative 128x128 tilings (selected with NCC_FORCE_VARIANT for sweeps)
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_8x1_c32x64", 128, 128, 12, 4, 1, 8, 32, 64),
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c16x64", 128, 128, 12, 4, 1, 4, 16, 64),
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_8x1_c16x64", 128, 128, 12, 4, 1, 8, 16, 64),
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x2_c32x64", 128, 128, 12, 4, 2, 4, 32, 64),
     TM_VARIANT("tm_sk_512x512_rv12_lx4_4x1_c32x64", 512, 512, 12, 4, 1, 4, 32, 64),
 };
 
@@ -106,20 +112,26 @@ bool encode_f32(CUtensorMap* m, const void* base, int rank, const uint64_t* dims
 struct PivVariant {
   const char* name;
   int TH, TW, MY, MX;  // 0 = run-time (RE)
-  int RV, CW, NT;
-  void (*kernel)(PivArgs);
+  int RV, CW, NT, WPB;
+  void (*k_tma)(PivArgs, CUtensorMap, CUtensorMap);  // nullptr: no TMA form (RE)
+  void (*k_ldg)(PivArgs, CUtensorMap, CUtensorMap);
 };
-#define PIV_VARIANT(NAME, TH, TW, MY, MX, RV, CW, NT, MINB) \
-  PivVariant { NAME, TH, TW, MY, MX, RV, CW, NT, piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, MINB> }
+#define PIV_VARIANT_SK(NAME, TH, TW, MY, MX, RV, CW, NT, WPB, MINB)                                      \
+  PivVariant {                                                                                          \
+    NAME, TH, TW, MY, MX, RV, CW, NT, WPB, piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, true>,   \
+        piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, false>                                     \
+  }
+#define PIV_VARIANT_RE(NAME, RV, CW, NT, MINB) \
+  PivVariant { NAME, 0, 0, 0, 0, RV, CW, NT, 1, nullptr, piv_ncc_kernel<0, 0, 0, 0, RV, CW, NT, 1, MINB, false> }
 
 const PivVariant kPivVariants[] = {
-    PIV_VARIANT("piv_re_rv12_cw16_nt256", 0, 0, 0, 0, 12, 16, 256, 1),
-    PIV_VARIANT("piv_sk_32x32_m16_rv12_nt128", 32, 32, 16, 16, 12, 32, 128, 4),
-    PIV_VARIANT("piv_sk_64x64_m32_rv12_nt416", 64, 64, 32, 32, 12, 64, 416, 2),
+    PIV_VARIANT_RE("piv_re_rv12_cw16_nt256", 12, 16, 256, 1),
+    PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt416_w4", 32, 32, 16, 16, 12, 32, 416, 4, 2),
+    PIV_VARIANT_SK("piv_sk_64x64_m32_rv12_nt416_w1", 64, 64, 32, 32, 12, 64, 416, 1, 2),
 };
 
-constexpr int kBoxRowsNT = 256, kBoxRowsSEG = 4096;
-constexpr int kBoxColsNT = 128, kBoxColsRB = 64;
+constexpr int kBoxRowsNT = 256, kBoxRowsSEG = 2048;  // max segment; actual = min(V, SEG)
+constexpr int kBoxColsNT = 128, kBoxColsRB = 32;
 
 int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
@@ -147,6 +159,9 @@ struct ncc_plan_s {
   // shared scratch (window sums)
   double *RS1, *RS2, *S1, *S2;
   int64_t rs_frame_stride, s_frame_stride;
+  // side stream for work independent of the main chain (template prep || window sums)
+  cudaStream_t side;
+  cudaEvent_t ev_fork, ev_join;
   // timing (NCC_F_TIMING)
   std::vector<cudaEvent_t> ev;
   int n_ev_used;
@@ -187,6 +202,9 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->st_s);
   cudaFree(pl->st_out);
   for (cudaEvent_t e : pl->ev) cudaEventDestroy(e);
+  if (pl->ev_fork) cudaEventDestroy(pl->ev_fork);
+  if (pl->ev_join) cudaEventDestroy(pl->ev_join);
+  if (pl->side) cudaStreamDestroy(pl->side);
   delete pl;
 }
 
@@ -250,7 +268,13 @@ ncc_status create_tm(ncc_plan pl) {
   const TmVariant* v = &kTmVariants[0];
   if (!(p.flags & NCC_F_GENERIC_KERNEL))
     for (const TmVariant& c : kTmVariants)
-      if (c.TH == h && c.TW == w) v = &c;
+      if (c.TH == h && c.TW == w) {
+        v = &c;
+        break;  // first matching specialised instance is the default
+      }
+  if (const char* force = getenv("NCC_FORCE_VARIANT"))  // sweeps: any instance valid for (h, w)
+    for (const TmVariant& c : kTmVariants)
+      if (strcmp(force, c.name) == 0 && (c.TH == 0 || (c.TH == h && c.TW == w))) v = &c;
   pl->tmv = v;
   const int nCH = ceil_div(h, v->CH), nCW = ceil_div(w, v->CW);
   pl->HP = nCH * v->CH;
@@ -264,7 +288,7 @@ ncc_status create_tm(ncc_plan pl) {
   NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, v->smem_ldg));
   const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
   if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
-  NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT, kBoxRowsSEG>,
+  NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem));
 
   // tiles of this band; split-K factor S from the FULL problem's tile count (so every shard
@@ -290,8 +314,15 @@ ncc_status create_tm(ncc_plan pl) {
       if (e >= 0.97) break;
     }
     pl->split = best_s;
+    if (const char* fs = getenv("NCC_FORCE_SPLIT")) {
+      const int f = atoi(fs);
+      if (f >= 1 && f <= nq) pl->split = f;
+    }
   }
 
+  NCC_CUDA(cudaStreamCreateWithFlags(&pl->side, cudaStreamNonBlocking));
+  NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_fork, cudaEventDisableTiming));
+  NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_join, cudaEventDisableTiming));
   ncc_status st;
   if ((st = dalloc(&pl->tplC, (size_t)pl->HP * pl->WP))) return st;
   if ((st = dalloc(&pl->tst, 1))) return st;
@@ -347,17 +378,23 @@ ncc_status create_piv(ncc_plan pl) {
       if (c.TH == h && c.TW == w && c.MY == my && c.MX == mx) v = &c;
   pl->pivv = v;
   const int RV = v->RV, CW = v->CW;
-  const int NG = (pl->OX + RV - 1) / RV, OXP = NG * RV, WP = ((w + CW - 1) / CW) * CW;
-  pl->piv_bp = piv_pick_pitch(OXP + WP, RV, NG);
-  const int64_t smem_f = (int64_t)h * WP + (int64_t)(h + 2 * my) * pl->piv_bp + (int64_t)pl->OY * OXP;
-  pl->piv_smem = (int)(smem_f * 4);
+  const int NG = (pl->OX + RV - 1) / RV;
+  pl->piv_bp = v->TH ? piv_sk_pitch(v->TW, v->MX, RV, CW) : piv_pick_pitch(NG * RV + ((w + CW - 1) / CW) * CW, RV, NG);
+  const int64_t win_fl = [&] {
+    if (RV == 12 && CW == 16) return (int64_t)PivShape<12, 16>(h, w, my, mx, pl->piv_bp).win_fl;
+    if (RV == 12 && CW == 32) return (int64_t)PivShape<12, 32>(h, w, my, mx, pl->piv_bp).win_fl;
+    return (int64_t)PivShape<12, 64>(h, w, my, mx, pl->piv_bp).win_fl;
+  }();
+  pl->piv_smem = (int)(win_fl * 4 * v->WPB);
   int maxsm = 0;
   NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
-  if (smem_f * 4 > maxsm) return NCC_ERR_UNSUPPORTED;
-  NCC_CUDA(cudaFuncSetAttribute((const void*)v->kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
+  if (win_fl * 4 * v->WPB > maxsm) return NCC_ERR_UNSUPPORTED;
+  if (v->k_tma)
+    NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
+  NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
   const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
   if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
-  NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT, kBoxRowsSEG>,
+  NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem));
 
   // window-sum maps of frame B, processed in sub-batches of pairs (scratch budget ~2 GiB)
@@ -384,7 +421,7 @@ ncc_status create_piv(ncc_plan pl) {
   in.specialized = v->TH != 0;
   in.variant_id = (int)(v - kPivVariants);
   snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
-  fill_kernel_info(pl, (const void*)v->kernel, v->NT, pl->piv_smem, pl->Kx, pl->Ky, sb);
+  fill_kernel_info(pl, (const void*)v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
   return NCC_OK;
 }
 
@@ -407,11 +444,12 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
   const int h = p.tmpl_h, w = p.tmpl_w;
   const int V = p.image_w - w + 1;
   const int rows_in = rows_out + h - 1;
-  const int smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
-  dim3 g1(ceil_div(V, kBoxRowsSEG), rows_in, batch);
-  box_rows_kernel<kBoxRowsNT, kBoxRowsSEG><<<g1, kBoxRowsNT, smem, s>>>(
-      frames, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, row0, w, V, pl->RS1, pl->RS2,
-      pl->rs_frame_stride);
+  const int seg = V < kBoxRowsSEG ? V : kBoxRowsSEG;
+  const int smem = (int)((seg + w + 1) * 2 * sizeof(double));
+  dim3 g1(ceil_div(V, seg), rows_in, batch);
+  box_rows_kernel<kBoxRowsNT><<<g1, kBoxRowsNT, smem, s>>>(frames, p.image_pitch, (int64_t)p.image_h * p.image_pitch,
+                                                           p.image_w, row0, w, V, seg, pl->RS1, pl->RS2,
+                                                           pl->rs_frame_stride);
   dim3 g2(ceil_div(V, kBoxColsNT), ceil_div(rows_out, kBoxColsRB), batch);
   box_cols_kernel<kBoxColsNT, kBoxColsRB><<<g2, kBoxColsNT, 0, s>>>(pl->RS1, pl->RS2, pl->rs_frame_stride, V, h,
                                                                     rows_out, pl->S1, pl->S2, pl->s_frame_stride);
@@ -426,11 +464,16 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     if (st) return st;
   }
   pl->timing_kind = 1;
+  // fork: template prep on the side stream, window sums on the main stream, join
   mark(pl, s, 0);
-  tm_template_prep<<<1, 1024, 0, s>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP, pl->tst,
-                                      pl->keys, p.batch);
-  mark(pl, s, 1);
+  NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
+  NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
+  tm_template_prep<<<1, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
+                                             pl->tst, pl->keys, p.batch);
+  mark(pl, pl->side, 1);
+  NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
   launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
+  NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
   mark(pl, s, 2);
   TmArgs a;
   a.img = d_images;
@@ -495,8 +538,9 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   pl->timing_kind = 2;
   pl->piv_nsub = nsub;
   const int64_t fs = (int64_t)p.image_h * p.image_pitch;
-  const int64_t wins = (int64_t)pl->Ky * pl->Kx;
   PivArgs a;
+  a.A = A;
+  a.B = B;
   a.pitch = p.image_pitch;
   a.frame_stride = fs;
   a.H = p.image_h;
@@ -513,22 +557,39 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   a.S2 = pl->S2;
   a.map_pitch = pl->map_w;
   a.map_frame_stride = pl->s_frame_stride;
+  a.vec = reinterpret_cast<VecOut*>(d_vec);
+  a.scores = d_scores;
   a.subpix = p.subpix;
   a.BP = pl->piv_bp;
+  // TMA maps over all frames of the call (3D: cols, rows, pair); plain loads otherwise
+  CUtensorMap mA, mB;
+  memset(&mA, 0, sizeof(mA));
+  memset(&mB, 0, sizeof(mB));
+  bool use_tma = v->k_tma != nullptr && p.image_pitch % 4 == 0 && reinterpret_cast<uintptr_t>(A) % 16 == 0 &&
+                 reinterpret_cast<uintptr_t>(B) % 16 == 0;
+  if (use_tma) {
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
+    const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)fs * 4};
+    const uint32_t boxA[3] = {(uint32_t)p.tmpl_w, (uint32_t)p.tmpl_h, 1u};
+    const uint32_t boxB[3] = {(uint32_t)pl->piv_bp, (uint32_t)(p.tmpl_h + 2 * p.search_y), 1u};
+    use_tma = boxB[1] <= 256 && boxB[0] <= 256 && encode_f32(&mA, A, 3, dims, strides, boxA) &&
+              encode_f32(&mB, B, 3, dims, strides, boxB);
+  }
+  const int groups = ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB);
   mark(pl, s, 0);
   for (int sb = 0; sb < nsub; ++sb) {
     const int p0 = sb * pl->sub_batch;
     const int np = (p0 + pl->sub_batch <= p.batch) ? pl->sub_batch : p.batch - p0;
     launch_box(pl, B + p0 * fs, np, 0, pl->map_h, s);
     mark(pl, s, 3 * sb + 1);
-    a.A = A + p0 * fs;
-    a.B = B + p0 * fs;
-    a.vec = reinterpret_cast<VecOut*>(d_vec) + p0 * wins;
-    a.scores = d_scores ? d_scores + p0 * wins * pl->OY * pl->OX : nullptr;
-    dim3 grid(pl->Kx, pl->Ky, np);
-    v->kernel<<<grid, v->NT, pl->piv_smem, s>>>(a);
+    a.pair0 = p0;
+    dim3 grid(groups, 1, np);
+    if (use_tma)
+      v->k_tma<<<grid, v->NT, pl->piv_smem, s>>>(a, mA, mB);
+    else
+      v->k_ldg<<<grid, v->NT, pl->piv_smem, s>>>(a, mA, mB);
     mark(pl, s, 3 * sb + 2);
-    if (p.flags & NCC_F_TIMING) mark(pl, s, 3 * sb + 3);
+    mark(pl, s, 3 * sb + 3);
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "piv_correlate launch");
@@ -621,7 +682,7 @@ ncc_status ncc_plan_timing(ncc_plan pl, ncc_timing* out) {
   if (pl->timing_kind == 1) {
     NCC_CUDA(cudaEventSynchronize(pl->ev[4]));
     cudaEventElapsedTime(&ms, pl->ev[0], pl->ev[1]); out->prep_ms = ms;
-    cudaEventElapsedTime(&ms, pl->ev[1], pl->ev[2]); out->stats_ms = ms;
+    cudaEventElapsedTime(&ms, pl->ev[0], pl->ev[2]); out->stats_ms = ms;  // prep || window sums
     cudaEventElapsedTime(&ms, pl->ev[2], pl->ev[3]); out->numerator_ms = ms;
     cudaEventElapsedTime(&ms, pl->ev[3], pl->ev[4]); out->finalize_ms = ms;
     cudaEventElapsedTime(&ms, pl->ev[0], pl->ev[4]); out->total_ms = ms;

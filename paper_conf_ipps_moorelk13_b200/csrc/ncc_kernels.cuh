@@ -461,54 +461,57 @@ __global__ void tm_finalize(const unsigned long long* __restrict__ keys, const T
 }
 
 // ================================================================== window sums (a2)
+// Inclusive warp scan (fp64, shuffle-up tree).
+__device__ __forceinline__ double warp_incl_scan_d(double v) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const double t = __shfl_up_sync(0xffffffffu, v, o);
+    if (lane >= o) v += t;
+  }
+  return v;
+}
+
 // Horizontal pass: RS[f][r][v] = sum_{j<w} I[row0 + r][v + j] for v < V (fp64), via a
 // segment-local fp64 prefix sum staged in shared memory (exact for 2^-8-quantised inputs).
-// grid = (ceil(V / SEG), rows, batch), block = NT.
-template <int NT, int SEG>
+// grid = (ceil(V / seg), rows, batch), block = NT, dynamic smem = 2 * (seg + w + 1) doubles.
+template <int NT>
 __global__ void __launch_bounds__(NT)
     box_rows_kernel(const float* __restrict__ img, int64_t pitch, int64_t frame_stride, int W, int row0, int w,
-                    int V, double* __restrict__ RS1, double* __restrict__ RS2, int64_t rs_frame_stride) {
+                    int V, int seg, double* __restrict__ RS1, double* __restrict__ RS2, int64_t rs_frame_stride) {
   extern __shared__ double sm_d[];
-  const int L = SEG + w;  // prefix entries P[0..L-1], P[k] = sum of the first k inputs
+  __shared__ double wt1[NT / 32], wt2[NT / 32];
+  const int L = seg + w;  // prefix entries P[0..L-1], P[k] = sum of the first k inputs
   double* P1 = sm_d;
   double* P2 = sm_d + L + 1;
-  __shared__ double tot1[NT], tot2[NT];
   const int f = blockIdx.z, r = blockIdx.y;
-  const int c0 = blockIdx.x * SEG;
-  const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch;
-  const int cnt = min(L - 1, W - c0);  // inputs in this segment
-  // per-thread contiguous block of inputs
+  const int c0 = blockIdx.x * seg;
+  const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch + c0;
+  const int cnt = min(L - 1, W - c0);  // inputs available in this segment
   const int per = (L - 1 + NT - 1) / NT;
   const int b0 = threadIdx.x * per;
   double a1 = 0.0, a2 = 0.0;
   for (int k = 0; k < per; ++k) {
     const int idx = b0 + k;
     if (idx < cnt) {
-      const double x = src[c0 + idx];
+      const double x = src[idx];
       a1 += x;
       a2 += x * x;
     }
   }
-  tot1[threadIdx.x] = a1;
-  tot2[threadIdx.x] = a2;
+  // block exclusive scan of the per-thread totals: warp shuffle scan + warp totals
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const double i1 = warp_incl_scan_d(a1), i2 = warp_incl_scan_d(a2);
+  if (lane == 31) { wt1[wid] = i1; wt2[wid] = i2; }
   __syncthreads();
-  if (threadIdx.x == 0) {  // exclusive scan of the NT block totals (serial, deterministic)
-    double s1 = 0.0, s2 = 0.0;
-    for (int t = 0; t < NT; ++t) {
-      const double q1 = tot1[t], q2 = tot2[t];
-      tot1[t] = s1;
-      tot2[t] = s2;
-      s1 += q1;
-      s2 += q2;
-    }
-  }
-  __syncthreads();
-  double s1 = tot1[threadIdx.x], s2 = tot2[threadIdx.x];
+  double o1 = 0.0, o2 = 0.0;
+  for (int q = 0; q < wid; ++q) { o1 += wt1[q]; o2 += wt2[q]; }
+  double s1 = o1 + i1 - a1, s2 = o2 + i2 - a2;
   if (threadIdx.x == 0) { P1[0] = 0.0; P2[0] = 0.0; }
   for (int k = 0; k < per; ++k) {
     const int idx = b0 + k;
     if (idx < L - 1) {
-      const double x = idx < cnt ? (double)src[c0 + idx] : 0.0;
+      const double x = idx < cnt ? (double)src[idx] : 0.0;
       s1 += x;
       s2 += x * x;
       P1[idx + 1] = s1;
@@ -516,13 +519,13 @@ __global__ void __launch_bounds__(NT)
     }
   }
   __syncthreads();
-  double* o1 = RS1 + (int64_t)f * rs_frame_stride + (int64_t)r * V;
-  double* o2 = RS2 + (int64_t)f * rs_frame_stride + (int64_t)r * V;
-  for (int k = threadIdx.x; k < SEG; k += NT) {
+  double* q1 = RS1 + (int64_t)f * rs_frame_stride + (int64_t)r * V;
+  double* q2 = RS2 + (int64_t)f * rs_frame_stride + (int64_t)r * V;
+  for (int k = threadIdx.x; k < seg; k += NT) {
     const int v = c0 + k;
     if (v < V) {
-      o1[v] = P1[k + w] - P1[k];
-      o2[v] = P2[k + w] - P2[k];
+      q1[v] = P1[k + w] - P1[k];
+      q2[v] = P2[k + w] - P2[k];
     }
   }
 }
@@ -543,16 +546,18 @@ __global__ void __launch_bounds__(NT)
   double* o1 = S1 + (int64_t)f * s_frame_stride + v;
   double* o2 = S2 + (int64_t)f * s_frame_stride + v;
   double a1 = 0.0, a2 = 0.0;
+#pragma unroll 8
   for (int i = 0; i < h; ++i) {
-    a1 += r1[(int64_t)(ub + i) * V];
-    a2 += r2[(int64_t)(ub + i) * V];
+    a1 += __ldg(r1 + (int64_t)(ub + i) * V);
+    a2 += __ldg(r2 + (int64_t)(ub + i) * V);
   }
   const int ue = min(ub + RB, rows_out);
-  for (int u = ub; u < ue; ++u) {
-    if (u > ub) {
-      a1 += r1[(int64_t)(u + h - 1) * V] - r1[(int64_t)(u - 1) * V];
-      a2 += r2[(int64_t)(u + h - 1) * V] - r2[(int64_t)(u - 1) * V];
-    }
+  o1[(int64_t)ub * V] = a1;
+  o2[(int64_t)ub * V] = a2;
+#pragma unroll 4
+  for (int u = ub + 1; u < ue; ++u) {
+    a1 += __ldg(r1 + (int64_t)(u + h - 1) * V) - __ldg(r1 + (int64_t)(u - 1) * V);
+    a2 += __ldg(r2 + (int64_t)(u + h - 1) * V) - __ldg(r2 + (int64_t)(u - 1) * V);
     o1[(int64_t)u * V] = a1;
     o2[(int64_t)u * V] = a2;
   }
@@ -560,11 +565,12 @@ __global__ void __launch_bounds__(NT)
 
 // ================================================================== PIV kernel (a6, a7)
 struct PivArgs {
-  const float* A;  // frames A (pairs), row pitch, frame stride in elements
-  const float* B;
+  const float* A;  // all frames A of the call, row pitch, frame stride in elements
+  const float* B;  // all frames B of the call
   int64_t pitch, frame_stride;
   int H, W, h, w, my, mx, sy, sx, Ky, Kx;
-  const double* S1;  // window sums of frame B at every valid position: [pair][H-h+1][W-w+1]
+  int pair0;         // first pair of this launch (sub-batch); blockIdx.z = pair - pair0
+  const double* S1;  // window sums of frame B at every valid position: [pair-pair0][H-h+1][W-w+1]
   const double* S2;
   int64_t map_pitch, map_frame_stride;
   VecOut* vec;       // [pair][Ky][Kx]
@@ -573,14 +579,19 @@ struct PivArgs {
   int BP;            // RE: staged B pitch (floats), chosen on the host
 };
 
+// Per-window shared-memory geometry (floats); regions rounded to 128 B for TMA destinations.
 template <int RV, int CW>
 struct PivShape {
-  int h, w, my, mx, OY, OX, NG, OXP, WP, BR, BP, items;
+  int h, w, my, mx, OY, OX, NG, OXP, WP, BR, BP, items, a_fl, b_fl, s_fl, win_fl;
   __host__ __device__ PivShape(int h_, int w_, int my_, int mx_, int BP_)
       : h(h_), w(w_), my(my_), mx(mx_), OY(2 * my_ + 1), OX(2 * mx_ + 1), NG((2 * mx_ + 1 + RV - 1) / RV),
         OXP(((2 * mx_ + 1 + RV - 1) / RV) * RV), WP(((w_ + CW - 1) / CW) * CW), BR(h_ + 2 * my_), BP(BP_),
-        items((2 * my_ + 1) * ((2 * mx_ + 1 + RV - 1) / RV)) {}
-  __host__ __device__ int smem_floats() const { return h * WP + BR * BP + OY * OXP; }
+        items((2 * my_ + 1) * ((2 * mx_ + 1 + RV - 1) / RV)) {
+    a_fl = ((h * WP + 31) / 32) * 32;
+    b_fl = ((BR * BP + 31) / 32) * 32;
+    s_fl = ((OY * OXP + 31) / 32) * 32;
+    win_fl = a_fl + b_fl + s_fl;
+  }
 };
 
 // Bank-conflict model of the PIV image loads (flattened items: lane l -> row l/NG, group l%NG).
@@ -605,6 +616,10 @@ __host__ __device__ constexpr int piv_pick_pitch(int minp, int RV, int NG) {
   }
   return best;
 }
+__host__ __device__ constexpr int piv_sk_pitch(int TW, int MX, int RV, int CW) {
+  return piv_pick_pitch((((2 * MX + 1 + RV - 1) / RV) * RV) + (((TW + CW - 1) / CW) * CW), RV,
+                        (2 * MX + 1 + RV - 1) / RV);
+}
 
 // Three-point sub-pixel fit along one axis (S8c step 3); fp64 from the fp32 score tile.
 __device__ __forceinline__ double subpix3(double cm, double c0, double cp, int mode, bool* parabola) {
@@ -624,79 +639,168 @@ __device__ __forceinline__ double subpix3(double cm, double c0, double cp, int m
   return num / den;
 }
 
-// One CTA per (window k_x, window k_y, pair).  TH/TW/MY/MX: compile-time window and search
-// sizes (SK) or 0 (RE).  CW = template columns per fp32 partial (and per unrolled row_dot).
-template <int TH, int TW, int MY, int MX, int RV, int CW, int NT, int MINB>
-__global__ void __launch_bounds__(NT, MINB) piv_ncc_kernel(const PivArgs a) {
-  constexpr bool SK = TH > 0;
-  const int BPc = SK ? piv_pick_pitch((((2 * MX + 1 + RV - 1) / RV) * RV) + (((TW + CW - 1) / CW) * CW), RV,
-                                      (2 * MX + 1 + RV - 1) / RV)
-                     : 0;
-  const PivShape<RV, CW> sh(SK ? TH : a.h, SK ? TW : a.w, SK ? MY : a.my, SK ? MX : a.mx, SK ? BPc : a.BP);
-  extern __shared__ float4 smem_f4[];
-  float* As = reinterpret_cast<float*>(smem_f4);  // [h][WP]   mask A -> A_C
-  float* Bs = As + sh.h * sh.WP;                  // [BR][BP]  search region of B
-  float* Sc = Bs + sh.BR * sh.BP;                 // [OY][OXP] score tile
-  __shared__ double red[32];
-  __shared__ unsigned long long red_key[32];
+// NCC with the fp64 window sums and a fp32 rsqrt (PIV epilogue): |error| <= ~4e-7 absolute.
+__device__ __forceinline__ float ncc_normalize_fast(float num, double s1, double s2, double inv_n, double csum,
+                                                    double energy, bool flat) {
+  const double var = s2 - s1 * s1 * inv_n;
+  if (flat || !(var > kFlatRel * s2)) return 0.0f;
+  const float numc = (float)((double)num - csum * s1 * inv_n);
+  float r = numc * rsqrtf((float)(energy * var));
+  return r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+}
 
-  const int tid = threadIdx.x;
-  const int kx = blockIdx.x, ky = blockIdx.y, pr = blockIdx.z;
-  const int y = sh.my + ky * a.sy, x = sh.mx + kx * a.sx;
-  const float* Af = a.A + (int64_t)pr * a.frame_stride;
-  const float* Bf = a.B + (int64_t)pr * a.frame_stride;
-
-  // ---- stage mask (zero-padded to WP) and search region (zero beyond the frame)
-  for (int k = tid; k < sh.h * sh.WP; k += NT) {
-    const int i = k / sh.WP, j = k % sh.WP;
-    As[k] = j < sh.w ? __ldg(Af + (int64_t)(y + i) * a.pitch + (x + j)) : 0.0f;
-  }
-  const int by0 = y - sh.my, bx0 = x - sh.mx;
-  for (int k = tid; k < sh.BR * sh.BP; k += NT) {
-    const int i = k / sh.BP, j = k % sh.BP;
-    const int gc = bx0 + j;
-    Bs[k] = gc < a.W ? __ldg(Bf + (int64_t)(by0 + i) * a.pitch + gc) : 0.0f;
+// Deterministic block sums of K values per thread (red: >= nwarps*K doubles).
+template <int K>
+__device__ __forceinline__ void block_sum_k(double (&v)[K], double* red) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5, nw = (blockDim.x + 31) >> 5;
+#pragma unroll
+  for (int k = 0; k < K; ++k) v[k] = warp_sum_d(v[k]);
+  __syncthreads();
+  if (lane == 0) {
+#pragma unroll
+    for (int k = 0; k < K; ++k) red[wid * K + k] = v[k];
   }
   __syncthreads();
-
-  // ---- mask statistics (Fig 5.2): mean, A_C in place, A_D, sum of fp32 A_C
-  double s = 0.0, s2 = 0.0;
-  for (int k = tid; k < sh.h * sh.WP; k += NT) {
-    const double t = As[k];
-    s += t;
-    s2 += t * t;
+#pragma unroll
+  for (int k = 0; k < K; ++k) {
+    double r = 0.0;
+    for (int q = 0; q < nw; ++q) r += red[q * K + k];
+    v[k] = r;
   }
-  s = block_sum_d(s, red);
-  s2 = block_sum_d(s2, red);
-  const double n = (double)sh.h * (double)sh.w;
-  const double mean = s / n;
-  double e = 0.0, cs = 0.0;
-  for (int k = tid; k < sh.h * sh.WP; k += NT) {
-    if (k % sh.WP < sh.w) {
-      const double d = (double)As[k] - mean;
-      e += d * d;
-      const float ac = (float)d;
-      cs += (double)ac;
-      As[k] = ac;
+}
+
+// WPB windows per CTA: blockIdx.x = window group, blockIdx.z = pair - pair0.
+// TH/TW/MY/MX: compile-time window and search sizes (SK) or 0 (RE).  CW = template columns
+// per fp32 partial (and per unrolled row_dot).  TMA: stage mask + search region with
+// cp.async.bulk.tensor (requires CW | TW so the staged mask has no padding columns).
+template <int TH, int TW, int MY, int MX, int RV, int CW, int NT, int WPB, int MINB, bool TMA>
+__global__ void __launch_bounds__(NT, MINB)
+    piv_ncc_kernel(const PivArgs a, const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB) {
+  constexpr bool SK = TH > 0;
+  static_assert(!TMA || (SK && TW % CW == 0), "TMA staging needs a specialised, unpadded mask");
+  const PivShape<RV, CW> sh(SK ? TH : a.h, SK ? TW : a.w, SK ? MY : a.my, SK ? MX : a.mx,
+                            SK ? piv_sk_pitch(TW, MX, RV, CW) : a.BP);
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  float* smem = reinterpret_cast<float*>(smem_raw);
+  constexpr int NW = (NT + 31) / 32;
+  __shared__ double red[NW * 2 * WPB];
+  __shared__ unsigned long long red_key[NW * WPB];
+  __shared__ double s_mean[WPB], s_energy[WPB], s_csum[WPB];
+  __shared__ int s_flat[WPB];
+  __shared__ __align__(8) uint64_t bar;
+
+  const int tid = threadIdx.x;
+  const int nwin = a.Ky * a.Kx;
+  const int lz = blockIdx.z, pr = a.pair0 + lz;
+  const int lin0 = blockIdx.x * WPB;
+  const int nvalid = min(WPB, nwin - lin0);
+  auto wy = [&](int wi) { return sh.my + ((lin0 + wi) / a.Kx) * a.sy; };
+  auto wx = [&](int wi) { return sh.mx + ((lin0 + wi) % a.Kx) * a.sx; };
+  auto As = [&](int wi) { return smem + wi * sh.win_fl; };
+  auto Bs = [&](int wi) { return smem + wi * sh.win_fl + sh.a_fl; };
+  auto Sc = [&](int wi) { return smem + wi * sh.win_fl + sh.a_fl + sh.b_fl; };
+
+  // ---- stage masks and search regions
+  if constexpr (TMA) {
+    if (tid == 0) {
+      tma_prefetch_desc(&mapA);
+      tma_prefetch_desc(&mapB);
+      mbar_init(&bar, 1);
+      fence_mbar_init();
     }
+    __syncthreads();
+    if (tid == 0) {
+      mbar_expect_tx(&bar, (uint32_t)(nvalid * (sh.h * sh.WP + sh.BR * sh.BP) * 4));
+      for (int wi = 0; wi < nvalid; ++wi) {
+        tma_load_3d(As(wi), &mapA, wx(wi), wy(wi), pr, &bar);
+        tma_load_3d(Bs(wi), &mapB, wx(wi) - sh.mx, wy(wi) - sh.my, pr, &bar);
+      }
+    }
+    mbar_wait(&bar, 0);
+  } else {
+    const float* Af = a.A + (int64_t)pr * a.frame_stride;
+    const float* Bf = a.B + (int64_t)pr * a.frame_stride;
+    for (int wi = 0; wi < nvalid; ++wi) {
+      const int y = wy(wi), x = wx(wi);
+      float* as = As(wi);
+      float* bs = Bs(wi);
+      for (int k = tid; k < sh.h * sh.WP; k += NT) {
+        const int i = k / sh.WP, j = k % sh.WP;
+        as[k] = j < sh.w ? __ldg(Af + (int64_t)(y + i) * a.pitch + (x + j)) : 0.0f;
+      }
+      const int by0 = y - sh.my, bx0 = x - sh.mx;
+      for (int k = tid; k < sh.BR * sh.BP; k += NT) {
+        const int i = k / sh.BP, j = k % sh.BP;
+        const int gc = bx0 + j;
+        bs[k] = gc < a.W ? __ldg(Bf + (int64_t)(by0 + i) * a.pitch + gc) : 0.0f;
+      }
+    }
+    __syncthreads();
   }
-  e = block_sum_d(e, red);  // contains __syncthreads: A_C visible afterwards
-  cs = block_sum_d(cs, red);
-  TemplateStats ts;
-  ts.sum = s; ts.sumsq = s2; ts.energy = e; ts.csum = cs;
-  ts.flat = (e <= kFlatRel * s2) ? 1 : 0;
-  ts.pad = 0;
 
-  // ---- numerator over flattened items (row, group of RV shifts) + normalisation
+  // ---- mask statistics (Fig 5.2) for all windows at once: mean, A_C, A_D, sum of fp32 A_C
+  const int per_win = sh.h * sh.WP;
+  {
+    double v[2 * WPB];
+#pragma unroll
+    for (int q = 0; q < 2 * WPB; ++q) v[q] = 0.0;
+    for (int e = tid; e < nvalid * per_win; e += NT) {
+      const int wi = e / per_win, k = e % per_win;
+      const double t = As(wi)[k];  // padding columns hold 0
+#pragma unroll
+      for (int q = 0; q < WPB; ++q)
+        if (q == wi) { v[2 * q] += t; v[2 * q + 1] += t * t; }
+    }
+    block_sum_k<2 * WPB>(v, red);
+    const double n = (double)sh.h * (double)sh.w;
+    double m[WPB];
+#pragma unroll
+    for (int q = 0; q < WPB; ++q) m[q] = v[2 * q] / n;
+    double sumsq[WPB];
+#pragma unroll
+    for (int q = 0; q < WPB; ++q) { sumsq[q] = v[2 * q + 1]; v[2 * q] = 0.0; v[2 * q + 1] = 0.0; }
+    for (int e = tid; e < nvalid * per_win; e += NT) {
+      const int wi = e / per_win, k = e % per_win;
+      if (k % sh.WP < sh.w) {
+        float* as = As(wi);
+        double mm = 0.0;
+#pragma unroll
+        for (int q = 0; q < WPB; ++q) mm = (q == wi) ? m[q] : mm;
+        const double d = (double)as[k] - mm;
+        const float ac = (float)d;
+        as[k] = ac;
+#pragma unroll
+        for (int q = 0; q < WPB; ++q)
+          if (q == wi) { v[2 * q] += d * d; v[2 * q + 1] += (double)ac; }
+      }
+    }
+    block_sum_k<2 * WPB>(v, red);  // (its barriers also publish the A_C writes)
+    if (tid < WPB) {
+      double e = 0, c = 0, mm = 0, ss = 0;
+#pragma unroll
+      for (int q = 0; q < WPB; ++q)
+        if (q == tid) { e = v[2 * q]; c = v[2 * q + 1]; mm = m[q]; ss = sumsq[q]; }
+      s_mean[tid] = mm;
+      s_energy[tid] = e;
+      s_csum[tid] = c;
+      s_flat[tid] = (e <= kFlatRel * ss) ? 1 : 0;
+    }
+    __syncthreads();
+  }
+
+  // ---- numerator over flattened items (window, row, group of RV shifts) + normalisation
   const int nCW = sh.WP / CW;
-  const double* S1f = a.S1 + (int64_t)pr * a.map_frame_stride;
-  const double* S2f = a.S2 + (int64_t)pr * a.map_frame_stride;
-  for (int it = tid; it < sh.items; it += NT) {
-    const int row = it / sh.NG, g = it % sh.NG;
+  const double inv_n = 1.0 / ((double)sh.h * (double)sh.w);
+  const double* S1f = a.S1 + (int64_t)lz * a.map_frame_stride;
+  const double* S2f = a.S2 + (int64_t)lz * a.map_frame_stride;
+  for (int it = tid; it < nvalid * sh.items; it += NT) {
+    const int wi = it / sh.items, r = it % sh.items;
+    const int row = r / sh.NG, g = r % sh.NG;
     float total[RV];
 #pragma unroll
     for (int c = 0; c < RV; ++c) total[c] = 0.0f;
-    const float* brow = Bs + row * sh.BP + g * RV;
+    const float* brow = Bs(wi) + row * sh.BP + g * RV;
+    const float* arow = As(wi);
 #pragma unroll 1
     for (int i = 0; i < sh.h; ++i) {
 #pragma unroll 1
@@ -704,55 +808,74 @@ __global__ void __launch_bounds__(NT, MINB) piv_ncc_kernel(const PivArgs a) {
         float part[RV];
 #pragma unroll
         for (int c = 0; c < RV; ++c) part[c] = 0.0f;
-        row_dot<RV, CW>(brow + i * sh.BP + jc * CW, As + i * sh.WP + jc * CW, part);
+        row_dot<RV, CW>(brow + i * sh.BP + jc * CW, arow + i * sh.WP + jc * CW, part);
 #pragma unroll
         for (int c = 0; c < RV; ++c) total[c] += part[c];
       }
     }
-    const int64_t mrow = (int64_t)(y - sh.my + row) * a.map_pitch + (x - sh.mx);
+    const double csum = s_csum[wi], energy = s_energy[wi];
+    const bool flat = s_flat[wi] != 0;
+    const int64_t mrow = (int64_t)(wy(wi) - sh.my + row) * a.map_pitch + (wx(wi) - sh.mx);
+    float* sc = Sc(wi) + row * sh.OXP;
 #pragma unroll
     for (int c = 0; c < RV; ++c) {
       const int col = g * RV + c;
-      float sc = 0.0f;
-      if (col < sh.OX) sc = ncc_normalize(total[c], S1f[mrow + col], S2f[mrow + col], n, ts);
-      Sc[row * sh.OXP + col] = sc;
+      float s = 0.0f;
+      if (col < sh.OX)
+        s = ncc_normalize_fast(total[c], __ldg(S1f + mrow + col), __ldg(S2f + mrow + col), inv_n, csum, energy, flat);
+      sc[col] = s;
     }
   }
   __syncthreads();
 
-  // ---- argmax over the tile (tie -> smallest row-major index), optional surface store
-  const int64_t wlin = ((int64_t)pr * a.Ky + ky) * a.Kx + kx;
-  float* gsc = a.scores ? a.scores + wlin * sh.OY * sh.OX : nullptr;
-  unsigned long long best = 0ull;
-  for (int k = tid; k < sh.OY * sh.OX; k += NT) {
+  // ---- argmax per window (tie -> smallest row-major index), optional surface store
+  const int tile = sh.OY * sh.OX;
+  unsigned long long best[WPB];
+#pragma unroll
+  for (int q = 0; q < WPB; ++q) best[q] = 0ull;
+  for (int e = tid; e < nvalid * tile; e += NT) {
+    const int wi = e / tile, k = e % tile;
     const int row = k / sh.OX, col = k % sh.OX;
-    const float sc = Sc[row * sh.OXP + col];
-    if (gsc) gsc[k] = sc;
-    const unsigned long long key = make_key(sc, (uint32_t)k);
-    best = key > best ? key : best;
+    const float s = Sc(wi)[row * sh.OXP + col];
+    if (a.scores) a.scores[((int64_t)pr * nwin + lin0 + wi) * tile + k] = s;
+    const unsigned long long key = make_key(s, (uint32_t)k);
+#pragma unroll
+    for (int q = 0; q < WPB; ++q)
+      if (q == wi) best[q] = key > best[q] ? key : best[q];
   }
-  best = block_max_key(best, red_key);
+  {
+    const int lane = tid & 31, wid = tid >> 5;
+#pragma unroll
+    for (int q = 0; q < WPB; ++q) best[q] = warp_max_key(best[q]);
+    if (lane == 0) {
+#pragma unroll
+      for (int q = 0; q < WPB; ++q) red_key[wid * WPB + q] = best[q];
+    }
+    __syncthreads();
+  }
 
-  // ---- sub-pixel fit and the 24-B vector
-  if (tid == 0) {
-    const uint32_t k = key_index(best);
+  // ---- sub-pixel fit and the 24-B vector: one thread per window
+  if (tid < nvalid) {
+    const int wi = tid;
+    unsigned long long bk = 0ull;
+    for (int q = 0; q < NW; ++q) bk = red_key[q * WPB + wi] > bk ? red_key[q * WPB + wi] : bk;
+    const float* S = Sc(wi);
+    const uint32_t k = key_index(bk);
     const int row = (int)(k / sh.OX), col = (int)(k % sh.OX);
     const int iy = row - sh.my, ix = col - sh.mx;
-    uint32_t flags = ts.flat ? (kFlatTemplate | kInvalid) : 0u;
+    uint32_t flags = s_flat[wi] ? (kFlatTemplate | kInvalid) : 0u;
     double ddy = 0.0, ddx = 0.0;
     bool par;
     if (row == 0 || row == sh.OY - 1) {
       flags |= kEdgeY;
     } else {
-      ddy = subpix3(Sc[(row - 1) * sh.OXP + col], Sc[row * sh.OXP + col], Sc[(row + 1) * sh.OXP + col], a.subpix,
-                    &par);
+      ddy = subpix3(S[(row - 1) * sh.OXP + col], S[row * sh.OXP + col], S[(row + 1) * sh.OXP + col], a.subpix, &par);
       if (par) flags |= kParabolaY;
     }
     if (col == 0 || col == sh.OX - 1) {
       flags |= kEdgeX;
     } else {
-      ddx = subpix3(Sc[row * sh.OXP + col - 1], Sc[row * sh.OXP + col], Sc[row * sh.OXP + col + 1], a.subpix,
-                    &par);
+      ddx = subpix3(S[row * sh.OXP + col - 1], S[row * sh.OXP + col], S[row * sh.OXP + col + 1], a.subpix, &par);
       if (par) flags |= kParabolaX;
     }
     VecOut o;
@@ -760,9 +883,9 @@ __global__ void __launch_bounds__(NT, MINB) piv_ncc_kernel(const PivArgs a) {
     o.ix = ix;
     o.dy = (float)(iy + ddy);
     o.dx = (float)(ix + ddx);
-    o.score = key_score(best);
+    o.score = key_score(bk);
     o.flags = flags;
-    a.vec[wlin] = o;
+    a.vec[(int64_t)pr * nwin + lin0 + wi] = o;
   }
 }
 

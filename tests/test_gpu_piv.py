@@ -147,3 +147,33 @@ def test_host_path_matches_device_path():
     d = decode_vectors(hv)
     np.testing.assert_array_equal(d["iy"].numpy(), v["iy"])
     np.testing.assert_array_equal(d["dy"].numpy(), v["dy"])
+
+
+def test_unaligned_pitch_plain_loads():
+    p = synth.particle_pair_integer(256, 256, 5, 2, seed=8000)
+    P = 259
+    A = np.zeros((1, 256, P), np.float32)
+    B_ = np.zeros((1, 256, P), np.float32)
+    A[0, :, :256] = p.A
+    B_[0, :, :256] = p.B
+    dev = torch.device("cuda", 0)
+    with PivPlan(256, 256, 32, 16, 16, pairs=1, image_pitch=P) as plan:
+        vec, sc = plan.correlate(torch.from_numpy(A).to(dev), torch.from_numpy(B_).to(dev), scores=True)
+        torch.cuda.synchronize()
+        assert plan.info.specialized == 1
+    d = {k: v.cpu().numpy() for k, v in decode_vectors(vec).items()}
+    ref = oracle.piv_pair(p.A, p.B, 32, 32, 16, 16, 16, 16)
+    np.testing.assert_array_equal(d["iy"][0], ref["iy"])
+    np.testing.assert_array_equal(d["ix"][0], ref["ix"])
+    rs = oracle.piv_window_scores(p.A, p.B, 32, 32, 16, 16, 16, 16, 5, 6)
+    assert np.max(np.abs(sc[0, 5, 6].cpu().numpy() - rs)) <= TOL
+
+
+def test_partial_last_window_group():
+    # Ky*Kx not a multiple of the windows-per-CTA of the specialised cfg3 kernel
+    p = synth.particle_pair_integer(32 * 7 + 32, 32 * 5 + 32, -3, 4, seed=8100)
+    H, W = p.A.shape
+    v, sc, info = run_piv([p.A], [p.B], 32, 16, 16)
+    Ky, Kx = oracle.piv_grid(H, W, 32, 32, 16, 16, 16, 16)
+    assert (Ky * Kx) % 4 != 0
+    assert np.all(v["iy"][0] == -3) and np.all(v["ix"][0] == 4)
