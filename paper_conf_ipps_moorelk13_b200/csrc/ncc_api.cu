@@ -45,19 +45,23 @@ struct TmVariant {
   const char* name;
   int TH, TW;                 // 0 = run-time (RE)
   int RV, LX, WX, WY, CH, CW;
-  void (*k_tma)(TmArgs, CUtensorMap, CUtensorMap);
-  void (*k_ldg)(TmArgs, CUtensorMap, CUtensorMap);
-  int nt, bu, bv, ir, ip, smem_tma, smem_ldg;
+  void (*k[2][2])(TmArgs, CUtensorMap, CUtensorMap);  // [tma][const template]
+  int smem[2][2];
+  int nt, bu, bv, ir, ip;
   int rv_nt() const { return RV * nt; }
 };
 
-#define TM_VARIANT(NAME, TH, TW, RV, LX, WX, WY, CH, CW)                                                  \
-  TmVariant {                                                                                          \
-    NAME, TH, TW, RV, LX, WX, WY, CH, CW, tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW, true>,           \
-        tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW, false>, TmTile<RV, LX, WX, WY, CH, CW>::NT,         \
-        TmTile<RV, LX, WX, WY, CH, CW>::BU, TmTile<RV, LX, WX, WY, CH, CW>::BV,                           \
-        TmTile<RV, LX, WX, WY, CH, CW>::IR, TmTile<RV, LX, WX, WY, CH, CW>::IP,                           \
-        TmTile<RV, LX, WX, WY, CH, CW>::SMEM_TMA, TmTile<RV, LX, WX, WY, CH, CW>::SMEM_LDG                \
+#define TM_K(RV, LX, WX, WY, CH, CW, TH, TW, TMA, CT) tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW, TMA, CT>
+#define TM_VARIANT(NAME, TH, TW, RV, LX, WX, WY, CH, CW)                                                     \
+  TmVariant {                                                                                             \
+    NAME, TH, TW, RV, LX, WX, WY, CH, CW,                                                                 \
+        {{TM_K(RV, LX, WX, WY, CH, CW, TH, TW, false, false), TM_K(RV, LX, WX, WY, CH, CW, TH, TW, false, true)}, \
+         {TM_K(RV, LX, WX, WY, CH, CW, TH, TW, true, false), TM_K(RV, LX, WX, WY, CH, CW, TH, TW, true, true)}},  \
+        {{TmTile<RV, LX, WX, WY, CH, CW>::smem_ldg(false), TmTile<RV, LX, WX, WY, CH, CW>::smem_ldg(true)},    \
+         {TmTile<RV, LX, WX, WY, CH, CW>::smem_tma(false), TmTile<RV, LX, WX, WY, CH, CW>::smem_tma(true)}},   \
+        TmTile<RV, LX, WX, WY, CH, CW>::NT, TmTile<RV, LX, WX, WY, CH, CW>::BU,                              \
+        TmTile<RV, LX, WX, WY, CH, CW>::BV, TmTile<RV, LX, WX, WY, CH, CW>::IR,                              \
+        TmTile<RV, LX, WX, WY, CH, CW>::IP                                                                   \
   }
 
 const TmVariant kTmVariants[] = {
@@ -68,8 +72,6 @@ const TmVariant kTmVariants[] = {
     TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c32x64", 128, 128, 12, 4, 1, 4, 32, 64),
     // alternative 128x128 tilings (selected with NCC_FORCE_VARIANT for sweeps)
     TM_VARIANT("tm_sk_128x128_rv12_lx4_8x1_c32x64", 128, 128, 12, 4, 1, 8, 32, 64),
-    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c16x64", 128, 128, 12, 4, 1, 4, 16, 64),
-    TM_VARIANT("tm_sk_128x128_rv12_lx4_8x1_c16x64", 128, 128, 12, 4, 1, 8, 16, 64),
     TM_VARIANT("tm_sk_128x128_rv12_lx4_4x2_c32x64", 128, 128, 12, 4, 2, 4, 32, 64),
     TM_VARIANT("tm_sk_512x512_rv12_lx4_4x1_c32x64", 512, 512, 12, 4, 1, 4, 32, 64),
 };
@@ -146,6 +148,8 @@ struct ncc_plan_s {
   int U, V, u_begin, u_end, Ub, Hs, HP, WP;
   int tiles_u, tiles_v, split;
   bool tma_ok;
+  int use_ct, slab_rows, n_slabs;  // constant-template slabs (rows per slab, slab count)
+  float* carry;
   CUtensorMap map_tpl;
   float* part;
   unsigned int* cnt;
@@ -190,6 +194,7 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->tplC);
   cudaFree(pl->part);
   cudaFree(pl->cnt);
+  cudaFree(pl->carry);
   cudaFree(pl->tst);
   cudaFree(pl->keys);
   cudaFree(pl->RS1);
@@ -283,13 +288,22 @@ ncc_status create_tm(ncc_plan pl) {
   int maxsm = 0, nsm = 0;
   NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
   NCC_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, pl->device));
-  if (v->smem_tma > maxsm || v->smem_ldg > maxsm) return NCC_ERR_UNSUPPORTED;
-  NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, v->smem_tma));
-  NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, v->smem_ldg));
+  for (int t = 0; t < 2; ++t)
+    for (int c = 0; c < 2; ++c) {
+      if (v->smem[t][c] > maxsm) return NCC_ERR_UNSUPPORTED;
+      NCC_CUDA(cudaFuncSetAttribute((const void*)v->k[t][c], cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    v->smem[t][c]));
+    }
   const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
   if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
   NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem));
+
+  // constant-bank template: slabs of whole row-chunks that fit 64 KB (NCC_NO_CONST_TPL=1 disables)
+  pl->slab_rows = (kConstTplFloats / pl->WP) / v->CH * v->CH;
+  pl->use_ct = pl->slab_rows >= v->CH && !getenv("NCC_NO_CONST_TPL");
+  if (pl->slab_rows > pl->HP) pl->slab_rows = pl->HP;
+  pl->n_slabs = pl->use_ct ? ceil_div(pl->HP, pl->slab_rows) : 1;
 
   // tiles of this band; split-K factor S from the FULL problem's tile count (so every shard
   // of a problem uses the same S and the same per-offset accumulation order): the smallest
@@ -298,10 +312,11 @@ ncc_status create_tm(ncc_plan pl) {
   pl->tiles_v = ceil_div(pl->V, v->bv);
   {
     int per_sm = 0;
-    NCC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, v->k_tma, v->nt, v->smem_tma));
+    const int ct = pl->use_ct ? 1 : 0;
+    NCC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, v->k[1][ct], v->nt, v->smem[1][ct]));
     const int64_t slots = (int64_t)(per_sm > 0 ? per_sm : 1) * nsm;
     const int64_t tiles_full = (int64_t)ceil_div(pl->U, v->bu) * ceil_div(pl->V, v->bv);
-    const int nq = nCH * nCW;
+    const int nq = pl->n_slabs > 1 ? 1 : nCH * nCW;  // slab launches carry totals: no split
     int best_s = 1;
     double best_e = 0.0;
     for (int S = 1; S <= nq && S <= 8; ++S) {
@@ -333,6 +348,8 @@ ncc_status create_tm(ncc_plan pl) {
     if ((st = dalloc(&pl->cnt, (size_t)ntiles))) return st;
     NCC_CUDA(cudaMemset(pl->cnt, 0, (size_t)ntiles * sizeof(unsigned int)));
   }
+  if (pl->n_slabs > 1)
+    if ((st = dalloc(&pl->carry, (size_t)ntiles * v->rv_nt()))) return st;
   pl->rs_frame_stride = (int64_t)pl->Hs * pl->V;
   pl->s_frame_stride = (int64_t)pl->Ub * pl->V;
   if ((st = dalloc(&pl->RS1, (size_t)p.batch * pl->rs_frame_stride))) return st;
@@ -356,9 +373,13 @@ ncc_status create_tm(ncc_plan pl) {
   in.specialized = v->TH != 0;
   in.variant_id = (int)(v - kTmVariants);
   snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
-  snprintf(in.variant_name + strlen(in.variant_name), sizeof(in.variant_name) - strlen(in.variant_name), "_s%d",
-           pl->split);
-  fill_kernel_info(pl, (const void*)v->k_tma, v->nt, v->smem_tma, pl->tiles_u * pl->tiles_v * pl->split, p.batch, 1);
+  snprintf(in.variant_name + strlen(in.variant_name), sizeof(in.variant_name) - strlen(in.variant_name), "_s%d%s",
+           pl->split, pl->use_ct ? (pl->n_slabs > 1 ? "_cslab" : "_ctpl") : "_stpl");
+  {
+    const int ct = pl->use_ct ? 1 : 0;
+    fill_kernel_info(pl, (const void*)v->k[1][ct], v->nt, v->smem[1][ct], pl->tiles_u * pl->tiles_v * pl->split,
+                     p.batch, 1);
+  }
   return NCC_OK;
 }
 
@@ -514,10 +535,22 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     use_tma = encode_f32(&map_img, d_images, 3, dims, strides, box);
   }
   dim3 grid(pl->tiles_u * pl->tiles_v * pl->split, p.batch);
-  if (use_tma)
-    v->k_tma<<<grid, v->nt, v->smem_tma, s>>>(a, map_img, pl->map_tpl);
-  else
-    v->k_ldg<<<grid, v->nt, v->smem_ldg, s>>>(a, map_img, pl->map_tpl);
+  const int t = use_tma ? 1 : 0, ct = pl->use_ct ? 1 : 0;
+  const int nCWl = pl->WP / v->CW;
+  a.carry = pl->carry;
+  for (int sl = 0; sl < pl->n_slabs; ++sl) {
+    const int r0 = sl * pl->slab_rows;
+    const int r1 = (r0 + pl->slab_rows < pl->HP) ? r0 + pl->slab_rows : pl->HP;
+    a.q_begin = ct ? (r0 / v->CH) * nCWl : 0;
+    a.q_end = ct ? (r1 / v->CH) * nCWl : a.nCH * a.nCW;
+    a.c_row0 = r0;
+    a.first = sl == 0;
+    a.last = sl == pl->n_slabs - 1;
+    if (ct)  // template rows [r0, r1) into the constant bank (stream-ordered after the prep)
+      NCC_CUDA(cudaMemcpyToSymbolAsync(c_tpl, pl->tplC + (size_t)r0 * pl->WP, (size_t)(r1 - r0) * pl->WP * 4, 0,
+                                       cudaMemcpyDeviceToDevice, s));
+    v->k[t][ct]<<<grid, v->nt, v->smem[t][ct], s>>>(a, map_img, pl->map_tpl);
+  }
   mark(pl, s, 3);
   tm_finalize<<<ceil_div(p.batch, 128), 128, 0, s>>>(pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks),
                                                      p.batch);

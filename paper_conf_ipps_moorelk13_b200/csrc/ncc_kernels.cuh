@@ -235,8 +235,43 @@ struct TmArgs {
   unsigned long long* keys;  // [batch] argmax keys (reset by tm_template_prep)
   float* part;               // split-K partial totals [batch][tiles][S][RV][NT]   (S > 1)
   unsigned int* cnt;         // split-K arrival counters [batch][tiles], zero between calls
-  int S;                     // split-K factor (fixed per variant: accumulation order depends on it)
+  int S;                     // split-K factor (fixed per problem: accumulation order depends on it)
+  // constant-template slabs: this launch covers chunks [q_begin, q_end) of every tile; the
+  // template rows [c_row0, c_row0 + rows) are resident in c_tpl (pitch tplP).  A running
+  // total is carried between slab launches in `carry` ([batch][tiles][RV][NT]).
+  int q_begin, q_end, c_row0, first, last;
+  float* carry;
 };
+
+// Template chunks in the constant bank: FFMA takes the template from uniform registers
+// (LDCU), so each FFMA reads only two vector registers and the register-bank conflicts
+// of the shared-memory-template form (ncu 'dispatch stall', tools/sass_banks.py) vanish.
+constexpr int kConstTplFloats = 16384;  // 64 KB
+__constant__ float c_tpl[kConstTplFloats];
+
+template <int RV, int CW>
+__device__ __forceinline__ void row_dot_c(const float* __restrict__ img, int toff, float (&acc)[RV]) {
+  float x[RV];
+#pragma unroll
+  for (int c = 0; c < RV; c += 4) {
+    const float4 v = *reinterpret_cast<const float4*>(img + c);
+    x[c] = v.x; x[c + 1] = v.y; x[c + 2] = v.z; x[c + 3] = v.w;
+  }
+#pragma unroll
+  for (int j = 0; j < CW; j += 4) {
+    const float4 nx = *reinterpret_cast<const float4*>(img + RV + j);
+    const float tt[4] = {c_tpl[toff + j], c_tpl[toff + j + 1], c_tpl[toff + j + 2], c_tpl[toff + j + 3]};
+    const float nn[4] = {nx.x, nx.y, nx.z, nx.w};
+#pragma unroll
+    for (int s = 0; s < 4; ++s) {
+#pragma unroll
+      for (int c = 0; c < RV; ++c) acc[c] = fmaf(tt[s], x[c], acc[c]);
+#pragma unroll
+      for (int c = 0; c < RV - 1; ++c) x[c] = x[c + 1];
+      x[RV - 1] = nn[s];
+    }
+  }
+}
 
 template <int RV, int LX, int WX, int WY, int CH, int CW>
 struct TmTile {
@@ -248,21 +283,26 @@ struct TmTile {
   static constexpr int IP = pick_pitch(BV + CW, RV, LX);  // staged image pitch (= TMA box cols)
   static constexpr int T_BYTES = CH * CW * 4;
   static constexpr int I_BYTES = IR * IP * 4;
-  static constexpr int STAGE = ((T_BYTES + 127) / 128) * 128 + ((I_BYTES + 127) / 128) * 128;
-  static constexpr int SMEM_TMA = 2 * STAGE;      // double-buffered (TMA path)
-  static constexpr int SMEM_LDG = T_BYTES + I_BYTES;
+  static constexpr int T_AL = ((T_BYTES + 127) / 128) * 128;
+  static constexpr int I_AL = ((I_BYTES + 127) / 128) * 128;
+  __host__ __device__ static constexpr int stage(bool ct) { return (ct ? 0 : T_AL) + I_AL; }
+  __host__ __device__ static constexpr int smem_tma(bool ct) { return 2 * stage(ct); }  // double-buffered
+  __host__ __device__ static constexpr int smem_ldg(bool ct) { return (ct ? 0 : T_BYTES) + I_BYTES; }
   static_assert(IR <= 256 && IP <= 256 && CW <= 256 && CH <= 256, "TMA box dims are limited to 256");
 };
 
 // Numerator + fused normalise / clamp / optional surface store / CTA argmax (Fig 5.3-5.6).
 // TH, TW: compile-time template size (specialised, "SK") or 0 (run-time evaluated, "RE").
-// S: split of the (row-chunk, col-chunk) sequence of a tile over S CTAs; chunk ranges are fixed
-//    per tile and the S partial totals are combined in index order by the last CTA to arrive, so
-//    the result is deterministic and independent of scheduling and of the band (shard).
-// TMA: stage image / template chunks with double-buffered cp.async.bulk.tensor + mbarrier;
+// CT:  template from the constant bank (slabs of <= 64 KB) instead of shared memory.
+// S:   split of the tile's (row-chunk, col-chunk) sequence over S CTAs; ranges are fixed per
+//      tile and the S partial totals are combined in index order by the last CTA to arrive, so
+//      the result is deterministic and independent of scheduling and of the band (shard).
+// TMA: stage image (and template) chunks with double-buffered cp.async.bulk.tensor + mbarrier;
 //      otherwise (pitch not 16-B aligned) plain coalesced loads, single buffer.
+// Per-offset order: partial per (template row, column chunk) added to the total in chunk
+// order; slab launches carry the running total, so the order equals the single-launch one.
 // One CTA = one (tile, split) unit: blockIdx.x = tile * S + split, blockIdx.y = frame.
-template <int RV, int LX, int WX, int WY, int CH, int CW, int TH, int TW, bool TMA>
+template <int RV, int LX, int WX, int WY, int CH, int CW, int TH, int TW, bool TMA, bool CT>
 __global__ void __launch_bounds__(WX* WY * 32)
     tm_ncc_kernel(const TmArgs a, const __grid_constant__ CUtensorMap map_img,
                   const __grid_constant__ CUtensorMap map_tpl) {
@@ -274,7 +314,6 @@ __global__ void __launch_bounds__(WX* WY * 32)
 
   const int h = TH ? TH : a.h;
   const int w = TW ? TW : a.w;
-  const int nCH = TH ? (TH + CH - 1) / CH : a.nCH;
   const int nCW = TW ? (TW + CW - 1) / CW : a.nCW;
   const int tplP = TW ? ((TW + CW - 1) / CW) * CW : a.tplP;
 
@@ -289,40 +328,50 @@ __global__ void __launch_bounds__(WX* WY * 32)
   const int ty = tile / a.tiles_v, tx = tile % a.tiles_v;
   const int u0 = a.u_begin + ty * T::BU;
   const int v0 = tx * T::BV;
-  const int nq = nCH * nCW;
-  const int q0 = (split * nq) / S, q1 = ((split + 1) * nq) / S;  // this unit's chunk range
+  const int nq = a.q_end - a.q_begin;
+  const int q0 = a.q_begin + (split * nq) / S, q1 = a.q_begin + ((split + 1) * nq) / S;
+  const int64_t tile_lin = (int64_t)f * a.tiles_u * a.tiles_v + tile;
 
   float total[RV];
+  if (a.first) {
 #pragma unroll
-  for (int c = 0; c < RV; ++c) total[c] = 0.0f;
+    for (int c = 0; c < RV; ++c) total[c] = 0.0f;
+  } else {  // continue the running total of the previous slab launch (S == 1)
+    const float* cp = a.carry + tile_lin * (RV * T::NT);
+#pragma unroll
+    for (int c = 0; c < RV; ++c) total[c] = __ldcg(cp + c * T::NT + tid);
+  }
 
-  auto compute_chunk = [&](const float* Ts, const float* Is) {
+  auto compute_chunk = [&](int q, const float* Ts, const float* Is) {
     const float* irow = Is + lu * T::IP + lv;
+    const int ic = q / nCW, jc = q % nCW;
 #pragma unroll 1
     for (int i = 0; i < CH; ++i) {
       float part[RV];
 #pragma unroll
       for (int c = 0; c < RV; ++c) part[c] = 0.0f;
-      row_dot<RV, CW>(irow + i * T::IP, Ts + i * CW, part);
+      if constexpr (CT)
+        row_dot_c<RV, CW>(irow + i * T::IP, (ic * CH + i - a.c_row0) * tplP + jc * CW, part);
+      else
+        row_dot<RV, CW>(irow + i * T::IP, Ts + i * CW, part);
 #pragma unroll
       for (int c = 0; c < RV; ++c) total[c] += part[c];
     }
   };
 
   if constexpr (TMA) {
-    auto stage_t = [&](int s) { return reinterpret_cast<float*>(smem_raw + s * T::STAGE); };
-    auto stage_i = [&](int s) {
-      return reinterpret_cast<float*>(smem_raw + s * T::STAGE + ((T::T_BYTES + 127) / 128) * 128);
-    };
+    constexpr int STG = T::stage(CT);
+    auto stage_t = [&](int s) { return reinterpret_cast<float*>(smem_raw + s * STG); };
+    auto stage_i = [&](int s) { return reinterpret_cast<float*>(smem_raw + s * STG + (CT ? 0 : T::T_AL)); };
     auto issue = [&](int q, int s) {  // one thread: chunk q -> stage s
       const int ic = q / nCW, jc = q % nCW;
-      mbar_expect_tx(&full_bar[s], (uint32_t)(T::T_BYTES + T::I_BYTES));
-      tma_load_2d(stage_t(s), &map_tpl, jc * CW, ic * CH, &full_bar[s]);
+      mbar_expect_tx(&full_bar[s], (uint32_t)((CT ? 0 : T::T_BYTES) + T::I_BYTES));
+      if constexpr (!CT) tma_load_2d(stage_t(s), &map_tpl, jc * CW, ic * CH, &full_bar[s]);
       tma_load_3d(stage_i(s), &map_img, v0 + jc * CW, u0 + ic * CH, f, &full_bar[s]);
     };
     if (tid == 0) {
       tma_prefetch_desc(&map_img);
-      tma_prefetch_desc(&map_tpl);
+      if constexpr (!CT) tma_prefetch_desc(&map_tpl);
       mbar_init(&full_bar[0], 1);
       mbar_init(&full_bar[1], 1);
       fence_mbar_init();
@@ -335,19 +384,21 @@ __global__ void __launch_bounds__(WX* WY * 32)
     for (int q = q0; q < q1; ++q) {
       const int k = q - q0, s = k & 1;
       mbar_wait(&full_bar[s], (uint32_t)((k >> 1) & 1));
-      compute_chunk(stage_t(s), stage_i(s));
+      compute_chunk(q, stage_t(s), stage_i(s));
       __syncthreads();  // every warp is done with stage s
       if (tid == 0 && q + 2 < q1) issue(q + 2, s);
     }
   } else {
     float* Ts = reinterpret_cast<float*>(smem_raw);
-    float* Is = Ts + CH * CW;
+    float* Is = Ts + (CT ? 0 : CH * CW);
     const float* img = a.img + (int64_t)f * a.frame_stride;
     for (int q = q0; q < q1; ++q) {
       const int ic = q / nCW, jc = q % nCW;
       __syncthreads();
-      const float* tsrc = a.tplC + (int64_t)(ic * CH) * tplP + jc * CW;
-      for (int k = tid; k < CH * CW; k += T::NT) Ts[k] = tsrc[(k / CW) * tplP + (k % CW)];
+      if constexpr (!CT) {
+        const float* tsrc = a.tplC + (int64_t)(ic * CH) * tplP + jc * CW;
+        for (int k = tid; k < CH * CW; k += T::NT) Ts[k] = tsrc[(k / CW) * tplP + (k % CW)];
+      }
       const int gr0 = u0 + ic * CH, gc0 = v0 + jc * CW;
       for (int k = tid; k < T::IR * T::IP; k += T::NT) {
         const int r = k / T::IP, c = k % T::IP;
@@ -355,18 +406,25 @@ __global__ void __launch_bounds__(WX* WY * 32)
         Is[k] = (gr < a.H && gc < a.W) ? __ldg(img + (int64_t)gr * a.pitch + gc) : 0.0f;
       }
       __syncthreads();
-      compute_chunk(Ts, Is);
+      compute_chunk(q, Ts, Is);
     }
+  }
+
+  if (!a.last) {  // hand the running total to the next slab launch
+    float* cp = a.carry + tile_lin * (RV * T::NT);
+#pragma unroll
+    for (int c = 0; c < RV; ++c) cp[c * T::NT + tid] = total[c];
+    return;
   }
 
   // ---- split-K combine: partials in fixed split order, by the last unit of the tile
   if (S > 1) {
-    float* pbase = a.part + (((int64_t)f * a.tiles_u * a.tiles_v + tile) * S) * (RV * T::NT);
+    float* pbase = a.part + tile_lin * S * (RV * T::NT);
 #pragma unroll
     for (int c = 0; c < RV; ++c) pbase[(int64_t)split * RV * T::NT + c * T::NT + tid] = total[c];
     __threadfence();
     __syncthreads();
-    unsigned int* cnt = a.cnt + (int64_t)f * a.tiles_u * a.tiles_v + tile;
+    unsigned int* cnt = a.cnt + tile_lin;
     if (tid == 0) last_flag = (atomicAdd(cnt, 1u) == (unsigned)(S - 1)) ? 1u : 0u;
     __syncthreads();
     if (!last_flag) return;

@@ -55,7 +55,11 @@ def tm(cfg, variants, splits):
 if __name__ == "__main__":
     kind, cfg = sys.argv[1], int(sys.argv[2])
     if kind == "tm":
-        vs = [None, "tm_sk_128x128_rv12_lx4_8x1_c32x64", "tm_sk_128x128_rv12_lx4_4x1_c16x64",
-              "tm_sk_128x128_rv12_lx4_8x1_c16x64", "tm_sk_128x128_rv12_lx4_4x2_c32x64",
+        vs = [None, "tm_sk_128x128_rv12_lx4_8x1_c32x64", "tm_sk_128x128_rv12_lx4_4x2_c32x64",
               "tm_re_rv12_lx4_4x1_c32x32"] if cfg == 2 else [None, "tm_re_rv12_lx4_4x1_c32x32"]
-        tm(cfg, vs, [None, 1, 2, 4, 8])
+        for ct in ("1", None):
+            if ct:
+                os.environ["NCC_NO_CONST_TPL"] = ct
+            else:
+                os.environ.pop("NCC_NO_CONST_TPL", None)
+            tm(cfg, vs, [None, 1, 2, 4, 8] if cfg == 2 else [None])
