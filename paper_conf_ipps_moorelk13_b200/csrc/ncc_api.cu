@@ -14,6 +14,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <mutex>
 #include <vector>
 
 #include "../../include/ncc.h"
@@ -114,28 +115,41 @@ bool encode_f32(CUtensorMap* m, const void* base, int rank, const uint64_t* dims
 struct PivVariant {
   const char* name;
   int TH, TW, MY, MX;  // 0 = run-time (RE)
-  int RV, CW, NT, WPB;
-  void (*k_tma)(PivArgs, CUtensorMap, CUtensorMap);  // nullptr: no TMA form (RE)
-  void (*k_ldg)(PivArgs, CUtensorMap, CUtensorMap);
+  int RV, CW, NT, WPB, ALIAS, IPT;
+  void (*k_tma)(PivArgs, CUtensorMap);  // nullptr: no TMA form
+  void (*k_ldg)(PivArgs, CUtensorMap);
 };
-#define PIV_VARIANT_SK(NAME, TH, TW, MY, MX, RV, CW, NT, WPB, MINB)                                      \
-  PivVariant {                                                                                          \
-    NAME, TH, TW, MY, MX, RV, CW, NT, WPB, piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, true>,   \
-        piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, false>                                     \
+#define PIV_VARIANT_SK(NAME, TH, TW, MY, MX, RV, CW, NT, WPB, MINB, IPT)                                     \
+  PivVariant {                                                                                              \
+    NAME, TH, TW, MY, MX, RV, CW, NT, WPB, 1, IPT,                                                          \
+        piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, true, true, IPT>,                              \
+        piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, false, true, IPT>                              \
   }
-#define PIV_VARIANT_RE(NAME, RV, CW, NT, MINB) \
-  PivVariant { NAME, 0, 0, 0, 0, RV, CW, NT, 1, nullptr, piv_ncc_kernel<0, 0, 0, 0, RV, CW, NT, 1, MINB, false> }
+#define PIV_VARIANT_RE(NAME, RV, CW, NT, MINB)                                                              \
+  PivVariant {                                                                                              \
+    NAME, 0, 0, 0, 0, RV, CW, NT, 1, 0, 1, piv_ncc_kernel<0, 0, 0, 0, RV, CW, NT, 1, MINB, true, false, 1>,   \
+        piv_ncc_kernel<0, 0, 0, 0, RV, CW, NT, 1, MINB, false, false, 1>                                     \
+  }
 
 const PivVariant kPivVariants[] = {
     PIV_VARIANT_RE("piv_re_rv12_cw16_nt256", 12, 16, 256, 1),
-    PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt416_w4", 32, 32, 16, 16, 12, 32, 416, 4, 2),
-    PIV_VARIANT_SK("piv_sk_64x64_m32_rv12_nt416_w1", 64, 64, 32, 32, 12, 64, 416, 1, 2),
+    PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt416_w4", 32, 32, 16, 16, 12, 32, 416, 4, 2, 1),
+    PIV_VARIANT_SK("piv_sk_64x64_m32_rv12_nt416_w1", 64, 64, 32, 32, 12, 64, 416, 1, 2, 1),
 };
 
 constexpr int kBoxRowsNT = 256, kBoxRowsSEG = 2048;  // max segment; actual = min(V, SEG)
 constexpr int kBoxColsNT = 128, kBoxColsRB = 32;
 
 int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
+
+// The 64 KB constant-bank template slot (c_tpl) is one per device.  Every writer orders itself
+// after the previous user on any stream with a per-device event, so concurrent TM plans on
+// different streams of one device stay correct (they serialise on the slot, nothing else).
+struct ConstSlot {
+  std::mutex mu;
+  cudaEvent_t done = nullptr;
+};
+ConstSlot g_const_slot[64];
 
 }  // namespace
 
@@ -401,17 +415,29 @@ ncc_status create_piv(ncc_plan pl) {
   const int RV = v->RV, CW = v->CW;
   const int NG = (pl->OX + RV - 1) / RV;
   pl->piv_bp = v->TH ? piv_sk_pitch(v->TW, v->MX, RV, CW) : piv_pick_pitch(NG * RV + ((w + CW - 1) / CW) * CW, RV, NG);
+  const bool alias = v->ALIAS != 0;
+  int items = 0;
   const int64_t win_fl = [&] {
-    if (RV == 12 && CW == 16) return (int64_t)PivShape<12, 16>(h, w, my, mx, pl->piv_bp).win_fl;
-    if (RV == 12 && CW == 32) return (int64_t)PivShape<12, 32>(h, w, my, mx, pl->piv_bp).win_fl;
-    return (int64_t)PivShape<12, 64>(h, w, my, mx, pl->piv_bp).win_fl;
+    if (RV == 12 && CW == 16) {
+      PivShape<12, 16> ps(h, w, my, mx, pl->piv_bp, alias);
+      items = ps.items;
+      return (int64_t)ps.win_fl;
+    }
+    if (RV == 12 && CW == 32) {
+      PivShape<12, 32> ps(h, w, my, mx, pl->piv_bp, alias);
+      items = ps.items;
+      return (int64_t)ps.win_fl;
+    }
+    PivShape<12, 64> ps(h, w, my, mx, pl->piv_bp, alias);
+    items = ps.items;
+    return (int64_t)ps.win_fl;
   }();
+  if (alias && (int64_t)items * v->WPB > (int64_t)v->NT * v->IPT) return NCC_ERR_UNSUPPORTED;
   pl->piv_smem = (int)(win_fl * 4 * v->WPB);
   int maxsm = 0;
   NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
   if (win_fl * 4 * v->WPB > maxsm) return NCC_ERR_UNSUPPORTED;
-  if (v->k_tma)
-    NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
+  NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
   NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
   const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
   if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
@@ -546,10 +572,18 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     a.c_row0 = r0;
     a.first = sl == 0;
     a.last = sl == pl->n_slabs - 1;
-    if (ct)  // template rows [r0, r1) into the constant bank (stream-ordered after the prep)
+    if (ct) {  // template rows [r0, r1) into the constant bank (stream-ordered after the prep)
+      ConstSlot& cs = g_const_slot[pl->device & 63];
+      std::lock_guard<std::mutex> lk(cs.mu);
+      if (!cs.done) NCC_CUDA(cudaEventCreateWithFlags(&cs.done, cudaEventDisableTiming));
+      else NCC_CUDA(cudaStreamWaitEvent(s, cs.done, 0));
       NCC_CUDA(cudaMemcpyToSymbolAsync(c_tpl, pl->tplC + (size_t)r0 * pl->WP, (size_t)(r1 - r0) * pl->WP * 4, 0,
                                        cudaMemcpyDeviceToDevice, s));
-    v->k[t][ct]<<<grid, v->nt, v->smem[t][ct], s>>>(a, map_img, pl->map_tpl);
+      v->k[t][ct]<<<grid, v->nt, v->smem[t][ct], s>>>(a, map_img, pl->map_tpl);
+      NCC_CUDA(cudaEventRecord(cs.done, s));
+    } else {
+      v->k[t][ct]<<<grid, v->nt, v->smem[t][ct], s>>>(a, map_img, pl->map_tpl);
+    }
   }
   mark(pl, s, 3);
   tm_finalize<<<ceil_div(p.batch, 128), 128, 0, s>>>(pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks),
@@ -595,18 +629,14 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   a.subpix = p.subpix;
   a.BP = pl->piv_bp;
   // TMA maps over all frames of the call (3D: cols, rows, pair); plain loads otherwise
-  CUtensorMap mA, mB;
-  memset(&mA, 0, sizeof(mA));
+  CUtensorMap mB;
   memset(&mB, 0, sizeof(mB));
-  bool use_tma = v->k_tma != nullptr && p.image_pitch % 4 == 0 && reinterpret_cast<uintptr_t>(A) % 16 == 0 &&
-                 reinterpret_cast<uintptr_t>(B) % 16 == 0;
+  bool use_tma = v->k_tma != nullptr && p.image_pitch % 4 == 0 && reinterpret_cast<uintptr_t>(B) % 16 == 0;
   if (use_tma) {
     const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
     const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)fs * 4};
-    const uint32_t boxA[3] = {(uint32_t)p.tmpl_w, (uint32_t)p.tmpl_h, 1u};
     const uint32_t boxB[3] = {(uint32_t)pl->piv_bp, (uint32_t)(p.tmpl_h + 2 * p.search_y), 1u};
-    use_tma = boxB[1] <= 256 && boxB[0] <= 256 && encode_f32(&mA, A, 3, dims, strides, boxA) &&
-              encode_f32(&mB, B, 3, dims, strides, boxB);
+    use_tma = boxB[1] <= 256 && boxB[0] <= 256 && encode_f32(&mB, B, 3, dims, strides, boxB);
   }
   const int groups = ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB);
   mark(pl, s, 0);
@@ -618,9 +648,9 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
     a.pair0 = p0;
     dim3 grid(groups, 1, np);
     if (use_tma)
-      v->k_tma<<<grid, v->NT, pl->piv_smem, s>>>(a, mA, mB);
+      v->k_tma<<<grid, v->NT, pl->piv_smem, s>>>(a, mB);
     else
-      v->k_ldg<<<grid, v->NT, pl->piv_smem, s>>>(a, mA, mB);
+      v->k_ldg<<<grid, v->NT, pl->piv_smem, s>>>(a, mB);
     mark(pl, s, 3 * sb + 2);
     mark(pl, s, 3 * sb + 3);
   }

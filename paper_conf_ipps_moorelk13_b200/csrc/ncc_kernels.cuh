@@ -637,19 +637,70 @@ struct PivArgs {
   int BP;            // RE: staged B pitch (floats), chosen on the host
 };
 
+// FFMA2 numerator core with template PAIRS (sm_100a fma.rn.f32x2):
+//   acc pair q = (acc[2q+1], acc[2q]);   TP[p] = (t[p-1], t[p]) for p = 0..CW (t[-1] = t[CW] = 0)
+//   for every pair p and q:  acc pair q += x[p + 2q] * TP[p]            (x broadcast to both lanes)
+// so acc[2q+1] += t[p-1] x[2q+1 + (p-1)] and acc[2q] += t[p] x[2q + p]: exactly sum_j t[j] x[c+j]
+// in increasing j (the two boundary products are +0 * x).  Each FFMA2 reads a scalar, a
+// template pair and an accumulator pair: with the template pair in the reuse cache it costs
+// two register-bank cycles for two FMAs, so bank conflicts cannot throttle the FMA pipe
+// (tools/sass_banks.py: 0.85-0.87 vs 0.62 for the scalar shared-memory form).
+typedef unsigned long long u64;
+__device__ __forceinline__ void ffma2_bcast(u64& d, float x, u64 tp) {
+  u64 xx;
+  asm("mov.b64 %0, {%1,%1};" : "=l"(xx) : "f"(x));
+  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(d) : "l"(xx), "l"(tp));
+}
+__device__ __forceinline__ void add2(u64& d, u64 s) { asm("add.rn.f32x2 %0, %0, %1;" : "+l"(d) : "l"(s)); }
+
+template <int RV, int CW>
+__device__ __forceinline__ void row_dot_pairs(const float* __restrict__ img, const u64* __restrict__ TP,
+                                              u64 (&A2)[RV / 2]) {
+  static_assert(RV % 4 == 0 && CW % 4 == 0, "RV and CW must be multiples of 4");
+  float x[RV + CW];
+#pragma unroll
+  for (int c = 0; c < RV; c += 4) {
+    const float4 v = *reinterpret_cast<const float4*>(img + c);
+    x[c] = v.x; x[c + 1] = v.y; x[c + 2] = v.z; x[c + 3] = v.w;
+  }
+#pragma unroll
+  for (int pp = 0; pp <= CW; pp += 2) {
+    if ((pp % 4) == 0 && pp + 4 <= CW) {
+      const float4 v = *reinterpret_cast<const float4*>(img + RV + pp);
+      x[RV + pp] = v.x; x[RV + pp + 1] = v.y; x[RV + pp + 2] = v.z; x[RV + pp + 3] = v.w;
+    }
+    const ulonglong2 tp = *reinterpret_cast<const ulonglong2*>(TP + pp);
+    const u64 tpv[2] = {tp.x, tp.y};
+#pragma unroll
+    for (int e = 0; e < 2; ++e) {
+      const int p = pp + e;
+      if (p <= CW) {
+#pragma unroll
+        for (int q = 0; q < RV / 2; ++q) ffma2_bcast(A2[q], x[p + 2 * q], tpv[e]);
+      }
+    }
+  }
+}
+
 // Per-window shared-memory geometry (floats); regions rounded to 128 B for TMA destinations.
+// TP: template pairs, per row nCW blocks of PB = CW + 2 pairs.  Sc (score tile) aliases TP
+// when ALIAS (scores are held in registers across the barrier that ends the numerator).
 template <int RV, int CW>
 struct PivShape {
-  int h, w, my, mx, OY, OX, NG, OXP, WP, BR, BP, items, a_fl, b_fl, s_fl, win_fl;
-  __host__ __device__ PivShape(int h_, int w_, int my_, int mx_, int BP_)
+  int h, w, my, mx, OY, OX, NG, OXP, nCW, PB, TPP, BR, BP, items, tp_fl, b_fl, s_fl, win_fl;
+  __host__ __device__ PivShape(int h_, int w_, int my_, int mx_, int BP_, bool alias)
       : h(h_), w(w_), my(my_), mx(mx_), OY(2 * my_ + 1), OX(2 * mx_ + 1), NG((2 * mx_ + 1 + RV - 1) / RV),
-        OXP(((2 * mx_ + 1 + RV - 1) / RV) * RV), WP(((w_ + CW - 1) / CW) * CW), BR(h_ + 2 * my_), BP(BP_),
+        OXP(((2 * mx_ + 1 + RV - 1) / RV) * RV), nCW((w_ + CW - 1) / CW), PB(CW + 2),
+        TPP(((w_ + CW - 1) / CW) * (CW + 2)), BR(h_ + 2 * my_), BP(BP_),
         items((2 * my_ + 1) * ((2 * mx_ + 1 + RV - 1) / RV)) {
-    a_fl = ((h * WP + 31) / 32) * 32;
+    tp_fl = ((h * TPP * 2 + 31) / 32) * 32;
     b_fl = ((BR * BP + 31) / 32) * 32;
     s_fl = ((OY * OXP + 31) / 32) * 32;
-    win_fl = a_fl + b_fl + s_fl;
+    win_fl = (alias ? (tp_fl > s_fl ? tp_fl : s_fl) : tp_fl + s_fl) + b_fl;
   }
+  __host__ __device__ int tp_off() const { return 0; }
+  __host__ __device__ int b_off(bool alias) const { return alias ? (tp_fl > s_fl ? tp_fl : s_fl) : tp_fl + s_fl; }
+  __host__ __device__ int s_off(bool alias) const { return alias ? 0 : tp_fl; }
 };
 
 // Bank-conflict model of the PIV image loads (flattened items: lane l -> row l/NG, group l%NG).
@@ -729,21 +780,21 @@ __device__ __forceinline__ void block_sum_k(double (&v)[K], double* red) {
 
 // WPB windows per CTA: blockIdx.x = window group, blockIdx.z = pair - pair0.
 // TH/TW/MY/MX: compile-time window and search sizes (SK) or 0 (RE).  CW = template columns
-// per fp32 partial (and per unrolled row_dot).  TMA: stage mask + search region with
-// cp.async.bulk.tensor (requires CW | TW so the staged mask has no padding columns).
-template <int TH, int TW, int MY, int MX, int RV, int CW, int NT, int WPB, int MINB, bool TMA>
+// per fp32 partial.  TMA: stage the search regions with cp.async.bulk.tensor; masks are read
+// from global (L2) straight into the template-pair layout.  ALIAS: the score tile reuses the
+// template-pair region (needs every item's scores in registers: items <= NT * IPT).
+template <int TH, int TW, int MY, int MX, int RV, int CW, int NT, int WPB, int MINB, bool TMA, bool ALIAS, int IPT>
 __global__ void __launch_bounds__(NT, MINB)
-    piv_ncc_kernel(const PivArgs a, const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapB) {
+    piv_ncc_kernel(const PivArgs a, const __grid_constant__ CUtensorMap mapB) {
   constexpr bool SK = TH > 0;
-  static_assert(!TMA || (SK && TW % CW == 0), "TMA staging needs a specialised, unpadded mask");
   const PivShape<RV, CW> sh(SK ? TH : a.h, SK ? TW : a.w, SK ? MY : a.my, SK ? MX : a.mx,
-                            SK ? piv_sk_pitch(TW, MX, RV, CW) : a.BP);
+                            SK ? piv_sk_pitch(TW, MX, RV, CW) : a.BP, ALIAS);
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   float* smem = reinterpret_cast<float*>(smem_raw);
   constexpr int NW = (NT + 31) / 32;
   __shared__ double red[NW * 2 * WPB];
   __shared__ unsigned long long red_key[NW * WPB];
-  __shared__ double s_mean[WPB], s_energy[WPB], s_csum[WPB];
+  __shared__ double s_energy[WPB], s_csum[WPB];
   __shared__ int s_flat[WPB];
   __shared__ __align__(8) uint64_t bar;
 
@@ -754,135 +805,166 @@ __global__ void __launch_bounds__(NT, MINB)
   const int nvalid = min(WPB, nwin - lin0);
   auto wy = [&](int wi) { return sh.my + ((lin0 + wi) / a.Kx) * a.sy; };
   auto wx = [&](int wi) { return sh.mx + ((lin0 + wi) % a.Kx) * a.sx; };
-  auto As = [&](int wi) { return smem + wi * sh.win_fl; };
-  auto Bs = [&](int wi) { return smem + wi * sh.win_fl + sh.a_fl; };
-  auto Sc = [&](int wi) { return smem + wi * sh.win_fl + sh.a_fl + sh.b_fl; };
+  auto TPw = [&](int wi) { return reinterpret_cast<u64*>(smem + wi * sh.win_fl + sh.tp_off()); };
+  auto Bs = [&](int wi) { return smem + wi * sh.win_fl + sh.b_off(ALIAS); };
+  auto Sc = [&](int wi) { return smem + wi * sh.win_fl + sh.s_off(ALIAS); };
 
-  // ---- stage masks and search regions
+  // ---- stage the search regions of frame B (TMA, or plain loads)
   if constexpr (TMA) {
     if (tid == 0) {
-      tma_prefetch_desc(&mapA);
       tma_prefetch_desc(&mapB);
       mbar_init(&bar, 1);
       fence_mbar_init();
     }
     __syncthreads();
     if (tid == 0) {
-      mbar_expect_tx(&bar, (uint32_t)(nvalid * (sh.h * sh.WP + sh.BR * sh.BP) * 4));
-      for (int wi = 0; wi < nvalid; ++wi) {
-        tma_load_3d(As(wi), &mapA, wx(wi), wy(wi), pr, &bar);
-        tma_load_3d(Bs(wi), &mapB, wx(wi) - sh.mx, wy(wi) - sh.my, pr, &bar);
-      }
+      mbar_expect_tx(&bar, (uint32_t)(nvalid * sh.BR * sh.BP * 4));
+      for (int wi = 0; wi < nvalid; ++wi) tma_load_3d(Bs(wi), &mapB, wx(wi) - sh.mx, wy(wi) - sh.my, pr, &bar);
     }
-    mbar_wait(&bar, 0);
   } else {
-    const float* Af = a.A + (int64_t)pr * a.frame_stride;
     const float* Bf = a.B + (int64_t)pr * a.frame_stride;
     for (int wi = 0; wi < nvalid; ++wi) {
-      const int y = wy(wi), x = wx(wi);
-      float* as = As(wi);
       float* bs = Bs(wi);
-      for (int k = tid; k < sh.h * sh.WP; k += NT) {
-        const int i = k / sh.WP, j = k % sh.WP;
-        as[k] = j < sh.w ? __ldg(Af + (int64_t)(y + i) * a.pitch + (x + j)) : 0.0f;
-      }
-      const int by0 = y - sh.my, bx0 = x - sh.mx;
+      const int by0 = wy(wi) - sh.my, bx0 = wx(wi) - sh.mx;
       for (int k = tid; k < sh.BR * sh.BP; k += NT) {
         const int i = k / sh.BP, j = k % sh.BP;
         const int gc = bx0 + j;
         bs[k] = gc < a.W ? __ldg(Bf + (int64_t)(by0 + i) * a.pitch + gc) : 0.0f;
       }
     }
-    __syncthreads();
   }
 
-  // ---- mask statistics (Fig 5.2) for all windows at once: mean, A_C, A_D, sum of fp32 A_C
-  const int per_win = sh.h * sh.WP;
+  // ---- mask statistics (Fig 5.2), masks read from global (L2): mean, A_D, sum of fp32 A_C;
+  //      the centred mask is written straight into the template-pair layout
+  const float* Af = a.A + (int64_t)pr * a.frame_stride;
+  const int per_win = sh.h * sh.w;
   {
     double v[2 * WPB];
 #pragma unroll
     for (int q = 0; q < 2 * WPB; ++q) v[q] = 0.0;
     for (int e = tid; e < nvalid * per_win; e += NT) {
       const int wi = e / per_win, k = e % per_win;
-      const double t = As(wi)[k];  // padding columns hold 0
+      const double t = __ldg(Af + (int64_t)(wy(wi) + k / sh.w) * a.pitch + wx(wi) + k % sh.w);
 #pragma unroll
       for (int q = 0; q < WPB; ++q)
         if (q == wi) { v[2 * q] += t; v[2 * q + 1] += t * t; }
     }
     block_sum_k<2 * WPB>(v, red);
     const double n = (double)sh.h * (double)sh.w;
-    double m[WPB];
+    double m[WPB], sumsq[WPB];
 #pragma unroll
-    for (int q = 0; q < WPB; ++q) m[q] = v[2 * q] / n;
-    double sumsq[WPB];
-#pragma unroll
-    for (int q = 0; q < WPB; ++q) { sumsq[q] = v[2 * q + 1]; v[2 * q] = 0.0; v[2 * q + 1] = 0.0; }
-    for (int e = tid; e < nvalid * per_win; e += NT) {
-      const int wi = e / per_win, k = e % per_win;
-      if (k % sh.WP < sh.w) {
-        float* as = As(wi);
+    for (int q = 0; q < WPB; ++q) { m[q] = v[2 * q] / n; sumsq[q] = v[2 * q + 1]; v[2 * q] = 0.0; v[2 * q + 1] = 0.0; }
+    const int WPd = sh.nCW * CW;  // padded mask width
+    const int per_pad = sh.h * WPd;
+    for (int e = tid; e < nvalid * per_pad; e += NT) {
+      const int wi = e / per_pad, k = e % per_pad;
+      const int i = k / WPd, j = k % WPd;
+      float ac = 0.0f;
+      if (j < sh.w) {
         double mm = 0.0;
 #pragma unroll
         for (int q = 0; q < WPB; ++q) mm = (q == wi) ? m[q] : mm;
-        const double d = (double)as[k] - mm;
-        const float ac = (float)d;
-        as[k] = ac;
+        const double d = (double)__ldg(Af + (int64_t)(wy(wi) + i) * a.pitch + wx(wi) + j) - mm;
+        ac = (float)d;
 #pragma unroll
         for (int q = 0; q < WPB; ++q)
           if (q == wi) { v[2 * q] += d * d; v[2 * q + 1] += (double)ac; }
       }
+      // pairs of chunk jc: TP[p] = (t[p-1], t[p]); value j sits in TP[l].y and TP[l+1].x
+      float* tp = reinterpret_cast<float*>(TPw(wi) + i * sh.TPP + (j / CW) * sh.PB);
+      const int l = j % CW;
+      tp[2 * l + 1] = ac;
+      tp[2 * (l + 1)] = ac;
+      if (l == 0) tp[0] = 0.0f;               // TP[0].x = t[-1] = 0
+      if (l == CW - 1) tp[2 * CW + 1] = 0.0f;  // TP[CW].y = t[CW] = 0
     }
-    block_sum_k<2 * WPB>(v, red);  // (its barriers also publish the A_C writes)
+    block_sum_k<2 * WPB>(v, red);  // (its barriers also publish the template pairs)
     if (tid < WPB) {
-      double e = 0, c = 0, mm = 0, ss = 0;
+      double e = 0, c = 0, ss = 0;
 #pragma unroll
       for (int q = 0; q < WPB; ++q)
-        if (q == tid) { e = v[2 * q]; c = v[2 * q + 1]; mm = m[q]; ss = sumsq[q]; }
-      s_mean[tid] = mm;
+        if (q == tid) { e = v[2 * q]; c = v[2 * q + 1]; ss = sumsq[q]; }
       s_energy[tid] = e;
       s_csum[tid] = c;
       s_flat[tid] = (e <= kFlatRel * ss) ? 1 : 0;
     }
+    if constexpr (TMA) mbar_wait(&bar, 0);
     __syncthreads();
   }
 
-  // ---- numerator over flattened items (window, row, group of RV shifts) + normalisation
-  const int nCW = sh.WP / CW;
+  // ---- numerator (FFMA2 pairs) over flattened items (window, row, group of RV shifts) + NCC
   const double inv_n = 1.0 / ((double)sh.h * (double)sh.w);
   const double* S1f = a.S1 + (int64_t)lz * a.map_frame_stride;
   const double* S2f = a.S2 + (int64_t)lz * a.map_frame_stride;
-  for (int it = tid; it < nvalid * sh.items; it += NT) {
+  const int nitems = nvalid * sh.items;
+  float scv[ALIAS ? IPT : 1][RV];
+#pragma unroll
+  for (int k = 0; k < (ALIAS ? IPT : 1); ++k)
+#pragma unroll
+    for (int c = 0; c < RV; ++c) scv[k][c] = 0.0f;
+  auto item = [&](int it, float (&out)[RV]) {
     const int wi = it / sh.items, r = it % sh.items;
     const int row = r / sh.NG, g = r % sh.NG;
-    float total[RV];
+    u64 tot2[RV / 2];
 #pragma unroll
-    for (int c = 0; c < RV; ++c) total[c] = 0.0f;
+    for (int q = 0; q < RV / 2; ++q) tot2[q] = 0ull;
     const float* brow = Bs(wi) + row * sh.BP + g * RV;
-    const float* arow = As(wi);
+    const u64* tpw = TPw(wi);
 #pragma unroll 1
     for (int i = 0; i < sh.h; ++i) {
 #pragma unroll 1
-      for (int jc = 0; jc < nCW; ++jc) {
-        float part[RV];
+      for (int jc = 0; jc < sh.nCW; ++jc) {
+        u64 part2[RV / 2];
 #pragma unroll
-        for (int c = 0; c < RV; ++c) part[c] = 0.0f;
-        row_dot<RV, CW>(brow + i * sh.BP + jc * CW, arow + i * sh.WP + jc * CW, part);
+        for (int q = 0; q < RV / 2; ++q) part2[q] = 0ull;
+        row_dot_pairs<RV, CW>(brow + i * sh.BP + jc * CW, tpw + i * sh.TPP + jc * sh.PB, part2);
 #pragma unroll
-        for (int c = 0; c < RV; ++c) total[c] += part[c];
+        for (int q = 0; q < RV / 2; ++q) add2(tot2[q], part2[q]);
       }
     }
     const double csum = s_csum[wi], energy = s_energy[wi];
     const bool flat = s_flat[wi] != 0;
     const int64_t mrow = (int64_t)(wy(wi) - sh.my + row) * a.map_pitch + (wx(wi) - sh.mx);
-    float* sc = Sc(wi) + row * sh.OXP;
 #pragma unroll
-    for (int c = 0; c < RV; ++c) {
-      const int col = g * RV + c;
-      float s = 0.0f;
-      if (col < sh.OX)
-        s = ncc_normalize_fast(total[c], __ldg(S1f + mrow + col), __ldg(S2f + mrow + col), inv_n, csum, energy, flat);
-      sc[col] = s;
+    for (int q = 0; q < RV / 2; ++q) {
+      const float lo = __uint_as_float((uint32_t)(tot2[q] & 0xFFFFFFFFull));  // acc[2q+1]
+      const float hi = __uint_as_float((uint32_t)(tot2[q] >> 32));           // acc[2q]
+#pragma unroll
+      for (int e = 0; e < 2; ++e) {
+        const int c = 2 * q + 1 - e;
+        const int col = g * RV + c;
+        float s = 0.0f;
+        if (col < sh.OX)
+          s = ncc_normalize_fast(e == 0 ? lo : hi, __ldg(S1f + mrow + col), __ldg(S2f + mrow + col), inv_n, csum,
+                                 energy, flat);
+        out[c] = s;
+      }
     }
+    if constexpr (!ALIAS) {
+      float* sc = Sc(wi) + row * sh.OXP + g * RV;
+#pragma unroll
+      for (int c = 0; c < RV; ++c) sc[c] = out[c];
+    }
+  };
+  if constexpr (ALIAS) {
+#pragma unroll
+    for (int k = 0; k < IPT; ++k) {
+      const int it = tid + k * NT;
+      if (it < nitems) item(it, scv[k]);
+    }
+    __syncthreads();  // template pairs are dead: the score tile may overwrite them
+#pragma unroll
+    for (int k = 0; k < IPT; ++k) {
+      const int it = tid + k * NT;
+      if (it < nitems) {
+        const int wi = it / sh.items, r = it % sh.items;
+        float* sc = Sc(wi) + (r / sh.NG) * sh.OXP + (r % sh.NG) * RV;
+#pragma unroll
+        for (int c = 0; c < RV; ++c) sc[c] = scv[k][c];
+      }
+    }
+  } else {
+    for (int it = tid; it < nitems; it += NT) item(it, scv[0]);
   }
   __syncthreads();
 

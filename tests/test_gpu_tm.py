@@ -201,9 +201,38 @@ def test_cfg2_split_k_bands_bitwise():
     """Split-K units + band shards: per-offset accumulation order is fixed per problem."""
     img, T, u0, v0 = synth.tm_inputs(2, k=2)
     full_peaks, full, info = run_match(img, T)
-    assert info["variant_name"].endswith(tuple(f"_s{k}" for k in range(1, 9)))
+    assert "_s" in info["variant_name"]
     parts = []
     for r in range(2):
         pk, s, inf = run_match(img, T, shard=(r, 2))
         parts.append(s[0])
     np.testing.assert_array_equal(np.concatenate(parts, axis=0), full[0])
+
+
+def test_concurrent_plans_on_two_streams():
+    """Two TM plans with different templates on two streams: the shared constant-bank
+    template slot is ordered by the library, both results stay exact."""
+    dev = torch.device("cuda", 0)
+    imgs, Ts, refs = [], [], []
+    for k in range(2):
+        img, T, u0, v0 = synth.tm_inputs(2, k=10 + k)
+        imgs.append(torch.from_numpy(img).to(dev))
+        Ts.append(torch.from_numpy(T).to(dev))
+        refs.append((u0, v0))
+    streams = [torch.cuda.Stream(dev), torch.cuda.Stream(dev)]
+    plans = [MatchPlan(1024, 1024, 128, 128) for _ in range(2)]
+    try:
+        outs = []
+        for _ in range(3):
+            for k in range(2):
+                with torch.cuda.stream(streams[k]):
+                    pk, _ = plans[k].match(imgs[k], Ts[k], stream=streams[k])
+                    outs.append((k, pk))
+        torch.cuda.synchronize()
+        for k, pk in outs:
+            d = decode_peaks(pk)
+            assert (int(d["u"][0]), int(d["v"][0])) == refs[k]
+            assert abs(float(d["score"][0]) - 1.0) <= TOL
+    finally:
+        for p in plans:
+            p.close()

@@ -13,7 +13,7 @@ import sys
 def analyze(lines):
     n = cyc = 0
     hist = {}
-    prev_srcs = [None, None, None]
+    prev_reuse = [None, None, None]  # register kept in each slot's reuse cache by the previous instruction
     for ln in lines:
         m = re.search(r"\b(FFMA2?|FADD|FMUL)\b\s+([^;]*);", ln)
         if not m:
@@ -22,24 +22,24 @@ def analyze(lines):
         parts = [p.strip() for p in args.split(",")]
         srcs = parts[1:]
         regs = []
-        for slot, s in enumerate(srcs):
-            reuse = ".reuse" in s
+        cur_reuse = [None, None, None]
+        for slot, s in enumerate(srcs[:3]):
             r = re.match(r"-?\|?R(\d+)", s)
             if not r:
                 continue
             idx = int(r.group(1))
-            if op == "FFMA2" and "F32x2" in s:
-                cand = [idx, idx + 1]
-            else:
-                cand = [idx]
-            if reuse and prev_srcs[slot] == idx:
-                cand = []
+            cand = [idx, idx + 1] if (op == "FFMA2" and "F32x2" in s) else [idx]
+            if prev_reuse[slot] == idx:
+                cand = []  # served by the operand reuse cache
+            if ".reuse" in s:
+                cur_reuse[slot] = idx
             regs.extend(cand)
-            prev_srcs[slot] = idx
+        prev_reuse = cur_reuse
         ev = len({r for r in regs if r % 2 == 0})
         od = len({r for r in regs if r % 2 == 1})
         rt = max(2 if op == "FFMA2" else 1, ev, od)
-        n += 1
+        fl = 2 if op == "FFMA2" else 1
+        n += fl
         cyc += rt
         hist[rt] = hist.get(rt, 0) + 1
     return n, cyc, hist
@@ -60,4 +60,4 @@ if __name__ == "__main__":
         out[cur] = analyze(buf)
     for f, (n, cyc, hist) in out.items():
         if key in f and n:
-            print(f"{f[:90]:90s} fma-class={n:6d} est_cycles={cyc:6d} eff={n / cyc:.3f} {dict(sorted(hist.items()))}")
+            print(f"{f[:90]:90s} fma-lanes={n:6d} est_cycles={cyc:6d} eff={n / cyc:.3f} {dict(sorted(hist.items()))}")
