@@ -77,6 +77,46 @@ static double corr2_window(const float *img, int64_t pitch, int r0, int c0,
     return num / sqrt(st * sw);
 }
 
+/* Sum of squared differences of the template against one window: the paper's own PIV
+ * similarity score (Fig 5.10 caption: "the per-mask offset sum of squared
+ * differences similarity score").  Plain definition, fp64, row-major serial sum. */
+static double ssd_window(const float *img, int64_t pitch, int r0, int c0,
+                         const float *tmpl, int64_t tpitch, int h, int w)
+{
+    double s = 0.0;
+    for (int i = 0; i < h; ++i)
+        for (int j = 0; j < w; ++j) {
+            double d = (double)tmpl[(int64_t)i * tpitch + j] -
+                       (double)img[(int64_t)(r0 + i) * pitch + (c0 + j)];
+            s += d * d;
+        }
+    return s;
+}
+
+/* SSD surface for offset rows [u_begin, u_end) (valid offsets, as oracle_ncc_surface). */
+int oracle_ssd_surface(const float *img, int H, int W, int64_t pitch,
+                       const float *tmpl, int h, int w, int64_t tpitch,
+                       int u_begin, int u_end, double *scores)
+{
+    if (h <= 0 || w <= 0 || h > H || w > W) return -1;
+    const int U = H - h + 1, V = W - w + 1;
+    if (u_begin < 0 || u_end > U || u_begin > u_end) return -1;
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int u = u_begin; u < u_end; ++u)
+        for (int v = 0; v < V; ++v)
+            scores[(int64_t)(u - u_begin) * V + v] = ssd_window(img, pitch, u, v, tmpl, tpitch, h, w);
+    return 0;
+}
+
+/* Peak of an SSD surface: argmin, ties -> smallest linear index. */
+int64_t oracle_argmin(const double *scores, int64_t count)
+{
+    int64_t best = 0;
+    for (int64_t k = 1; k < count; ++k)
+        if (scores[k] < scores[best]) best = k;
+    return best;
+}
+
 /* Is the template flat?  (S8c reading 4; same energy test as corr2_window.) */
 int oracle_template_is_flat(const float *tmpl, int64_t tpitch, int h, int w)
 {
@@ -212,6 +252,47 @@ static void piv_one_window(const float *A, const float *B, int64_t pitch,
     out->flags = flags;
 }
 
+/* PIV with the SSD score (the paper's metric, Fig 5.10): argmin over the search range
+ * (tie -> smallest row-major index), 3-point parabolic sub-pixel fit of the minimum per axis
+ * (delta = (c- - c+) / (2 (c- - 2 c0 + c+)), 0 if that denominator <= 0), no fit on the border. */
+static void piv_one_window_ssd(const float *A, const float *B, int64_t pitch,
+                               int h, int w, int my, int mx, int y, int x,
+                               double *scratch, oracle_piv_vector *out)
+{
+    const int OY = 2 * my + 1, OX = 2 * mx + 1;
+    const float *tmpl = A + (int64_t)y * pitch + x;
+    for (int dy = -my; dy <= my; ++dy)
+        for (int dx = -mx; dx <= mx; ++dx)
+            scratch[(dy + my) * OX + (dx + mx)] =
+                ssd_window(B, pitch, y + dy, x + dx, tmpl, pitch, h, w);
+    const int64_t k = oracle_argmin(scratch, (int64_t)OY * OX);
+    const int iy = (int)(k / OX) - my, ix = (int)(k % OX) - mx;
+    uint32_t flags = 0;
+    double ddy = 0.0, ddx = 0.0;
+    if (iy == -my || iy == my) {
+        flags |= OF_EDGE_Y;
+    } else {
+        const double cm = scratch[(iy + my - 1) * OX + (ix + mx)], c0 = scratch[(iy + my) * OX + (ix + mx)],
+                     cp = scratch[(iy + my + 1) * OX + (ix + mx)];
+        const double den = 2.0 * (cm - 2.0 * c0 + cp);
+        if (den > 0.0) ddy = (cm - cp) / den;
+    }
+    if (ix == -mx || ix == mx) {
+        flags |= OF_EDGE_X;
+    } else {
+        const double cm = scratch[(iy + my) * OX + (ix + mx - 1)], c0 = scratch[(iy + my) * OX + (ix + mx)],
+                     cp = scratch[(iy + my) * OX + (ix + mx + 1)];
+        const double den = 2.0 * (cm - 2.0 * c0 + cp);
+        if (den > 0.0) ddx = (cm - cp) / den;
+    }
+    out->iy = iy;
+    out->ix = ix;
+    out->dy = iy + ddy;
+    out->dx = ix + ddx;
+    out->score = scratch[k];
+    out->flags = flags;
+}
+
 /* Window grid (S8 notation): K = floor((S - w - 2m)/s) + 1 per axis, window (ky,kx)
  * has its A-origin at (my + ky*sy, mx + kx*sx).  Interior windows only (S8c #9). */
 int oracle_piv_grid(int H, int W, int h, int w, int my, int mx, int sy, int sx,
@@ -276,6 +357,23 @@ int oracle_piv_window_scores(const float *A, const float *B, int H, int W, int64
         for (int dx = -mx; dx <= mx; ++dx)
             scores[(dy + my) * OX + (dx + mx)] =
                 corr2_window(B, pitch, y + dy, x + dx, tmpl, pitch, h, w);
+    return 0;
+}
+
+int oracle_piv_windows_ssd(const float *A, const float *B, int H, int W, int64_t pitch,
+                           int h, int w, int my, int mx, int sy, int sx,
+                           const int *kys, const int *kxs, int count,
+                           double *scratch, oracle_piv_vector *out)
+{
+    int Ky, Kx;
+    if (oracle_piv_grid(H, W, h, w, my, mx, sy, sx, &Ky, &Kx)) return -1;
+    for (int i = 0; i < count; ++i)
+        if (kys[i] < 0 || kys[i] >= Ky || kxs[i] < 0 || kxs[i] >= Kx) return -1;
+    const int64_t per = (int64_t)(2 * my + 1) * (2 * mx + 1);
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int i = 0; i < count; ++i)
+        piv_one_window_ssd(A, B, pitch, h, w, my, mx, my + kys[i] * sy, mx + kxs[i] * sx,
+                           scratch + (int64_t)i * per, &out[i]);
     return 0;
 }
 

@@ -253,3 +253,46 @@ def test_piv_subpixel_recovers_fractional_shift():
     # method accuracy (reported, not a parity bound): Gaussian fit within 0.1 px here
     assert np.median(np.abs(v["dy"] - 2.3)) < 0.1
     assert np.median(np.abs(v["dx"] + 1.6)) < 0.1
+
+
+# ---------------------------------------------------------------- SSD (paper's PIV metric, Fig 5.10)
+def test_ssd_hand_case():
+    # case A windows are [[a,a+1],[a+3,a+4]] (a = 1,2,4,5) vs T = [[1,2],[3,4]]:
+    # T - W = [[1-a, 1-a], [-a, -a]] -> SSD = 2(1-a)^2 + 2a^2 = 2, 10, 50, 82
+    c = _cases()["case_A"]
+    s = oracle.ssd_surface(np.array(c["image"], np.float32), np.array(c["template"], np.float32))
+    np.testing.assert_array_equal(s, np.array([[2.0, 10.0], [50.0, 82.0]]))
+
+
+def test_ssd_invariants():
+    img, T, u0, v0 = synth.tm_inputs(1)
+    s, pk = oracle.ssd_match(img, T)
+    assert s[u0, v0] == 0.0 and (pk.u, pk.v) == (u0, v0)
+    assert np.all(s >= 0.0)
+    # symmetry and the expansion sum T^2 - 2 sum T W + sum W^2 through an independent path
+    g = synth.rng(44)
+    A = g.random((5, 7), dtype=np.float32)
+    B = g.random((5, 7), dtype=np.float32)
+    assert oracle.ssd_surface(A, B)[0, 0] == oracle.ssd_surface(B, A)[0, 0]
+    a, b = A.astype(np.float64), B.astype(np.float64)
+    assert abs(oracle.ssd_surface(A, B)[0, 0] - ((a * a).sum() - 2 * (a * b).sum() + (b * b).sum())) < 1e-12
+    # shift invariance: adding c to both template and image leaves SSD unchanged
+    sq = oracle.ssd_surface(synth.quantize(img), synth.quantize(T))
+    np.testing.assert_allclose(oracle.ssd_surface(synth.quantize(img) + 2, synth.quantize(T) + 2), sq, atol=1e-9)
+
+
+def test_argmin_tie_smallest_index():
+    s = np.ones((4, 6))
+    s[2, 1] = s[0, 5] = s[3, 3] = 0.1
+    assert oracle.argmin(s) == 5
+
+
+def test_piv_ssd_planted_shift_and_parabola():
+    p = synth.particle_pair_integer(160, 176, -2, 4, seed=45)
+    v = oracle.piv_windows_ssd(p.A, p.B, 32, 32, 8, 8, 16, 16, [1, 2, 3], [1, 4, 2])
+    assert np.all(v["iy"] == -2) and np.all(v["ix"] == 4) and np.all(v["score"] < 1e-9)
+    # parabola fit of an exact parabola minimum recovers delta
+    for d in (0.3, -0.2):
+        c = [1.0 + 2.0 * (k - d) ** 2 for k in (-1, 0, 1)]
+        den = 2 * (c[0] - 2 * c[1] + c[2])
+        assert abs((c[0] - c[2]) / den - d) < 1e-12
