@@ -272,7 +272,7 @@ def main():
         step = lambda: plan.match(d_img, d_t, stream=stream, peaks=peaks)  # noqa: E731
         units_per_step = plan.info.outputs_per_call
         metric, unit = "NCC offsets/sec", "offsets/s"
-        launches_per_step = 5
+        launches_per_step = plan.info.launches_per_call
         h2d = wl["img"].nbytes + wl["T"].nbytes
         d2h = 16
         # host buffers for the end-to-end arm (pinned)
@@ -288,8 +288,7 @@ def main():
         step = lambda: plan.correlate(A, Bf, stream=stream, vectors=vec)  # noqa: E731
         units_per_step = plan.info.outputs_per_call
         metric, unit = "PIV vectors/sec", "vectors/s"
-        nsub = math.ceil(wl["pairs"] / plan.info.grid_z)
-        launches_per_step = 3 * nsub
+        launches_per_step = plan.info.launches_per_call
         h2d = 2 * A.numel() * 4
         d2h = vec.numel() * 4
         e2e_step = None

@@ -45,7 +45,7 @@ typedef struct ncc_plan_s* ncc_plan;
 typedef enum {
     NCC_OK = 0,
     NCC_ERR_INVALID_ARGUMENT = 1, /* bad sizes / pointers / ranges                        */
-    NCC_ERR_UNSUPPORTED = 2,      /* valid problem this build cannot run (e.g. SSD score)  */
+    NCC_ERR_UNSUPPORTED = 2,      /* valid problem this build cannot run (smem limits)     */
     NCC_ERR_OUT_OF_MEMORY = 3,    /* scratch allocation failed                             */
     NCC_ERR_CUDA = 4,             /* CUDA runtime / launch error (see ncc_last_cuda_error) */
     NCC_ERR_COMPILE = 5,          /* run-time specialisation failed                        */
@@ -53,7 +53,11 @@ typedef enum {
 } ncc_status;
 
 enum { NCC_MODE_MATCH = 0, NCC_MODE_PIV = 1 };
-enum { NCC_SCORE_NCC = 0, NCC_SCORE_SSD = 1 /* not built yet: NCC_ERR_UNSUPPORTED */ };
+/* Score.  NCC: corr2 (Fig 5.1), peak = argmax.  SSD: sum (T - W)^2, the paper's own PIV
+ * similarity score (Fig 5.10 caption), peak = argmin (tie -> smallest index);
+ * computed from the same numerator as sum T^2 - 2 (sum A_C W + Tbar S1) + S2; PIV sub-pixel
+ * for SSD is the 3-point parabola through the minimum; no flat-template flags for SSD. */
+enum { NCC_SCORE_NCC = 0, NCC_SCORE_SSD = 1 };
 enum { NCC_SUBPIX_GAUSS3 = 0, NCC_SUBPIX_PARABOLA3 = 1, NCC_SUBPIX_NONE = 2 };
 
 /* ncc_problem.flags */
@@ -77,7 +81,7 @@ enum {
 /* Problem statement (P:1290-1311 GPU-PF parameter analog). */
 typedef struct {
     int32_t mode;    /* NCC_MODE_MATCH or NCC_MODE_PIV                                    */
-    int32_t score;   /* NCC_SCORE_NCC                                                      */
+    int32_t score;   /* NCC_SCORE_NCC or NCC_SCORE_SSD                                     */
     int32_t subpix;  /* PIV: NCC_SUBPIX_GAUSS3 (Gaussian, parabolic fallback) / PARABOLA3 / NONE */
     int32_t image_h; /* H: rows of every frame                                             */
     int32_t image_w; /* W: columns of every frame                                          */
@@ -129,6 +133,10 @@ typedef struct {
     int32_t threads_per_block; /* numerator kernel block size                               */
     int32_t smem_per_block;    /* numerator kernel dynamic shared memory (bytes)            */
     int32_t grid_x, grid_y, grid_z; /* numerator launch grid (per sub-batch for PIV)        */
+    int32_t launches_per_call; /* kernels this library launches per execute call          */
+    int32_t split;             /* TM: split-K units per tile (accumulation order is fixed by it) */
+    int32_t const_template;    /* TM: template read from the constant bank (1) or shared memory (0) */
+    int32_t slabs;             /* TM: constant-bank template slabs (numerator launches)   */
     char variant_name[96];
 } ncc_plan_info;
 
@@ -146,7 +154,8 @@ typedef struct {
  * Returns NCC_ERR_INVALID_ARGUMENT for: any size <= 0; h > H or w > W; pitch < W;
  * batch < 1; shard_count < 1 or shard_rank outside [0, shard_count) or a band with no
  * rows; PIV: search < 0, step <= 0, no window fits, shard_count != 1; TM: search != 0.
- * NCC_ERR_UNSUPPORTED for score != NCC_SCORE_NCC. *out is NULL on failure. */
+ * NCC_ERR_UNSUPPORTED when the problem needs more shared memory than the device has.
+ * *out is NULL on failure. */
 ncc_status ncc_plan_create(const ncc_problem* p, int device, ncc_plan* out);
 
 /* TM on `batch` frames with one template.

@@ -56,6 +56,8 @@ class NccPlanInfo(ctypes.Structure):
                 ("variant_id", ctypes.c_int32), ("regs_per_thread", ctypes.c_int32),
                 ("threads_per_block", ctypes.c_int32), ("smem_per_block", ctypes.c_int32),
                 ("grid_x", ctypes.c_int32), ("grid_y", ctypes.c_int32), ("grid_z", ctypes.c_int32),
+                ("launches_per_call", ctypes.c_int32), ("split", ctypes.c_int32),
+                ("const_template", ctypes.c_int32), ("slabs", ctypes.c_int32),
                 ("variant_name", ctypes.c_char * 96)]
 
     def as_dict(self):

@@ -60,11 +60,12 @@ class MatchPlan(_Plan):
     """Template matching: corr2 at every valid offset of each frame (Listing 5.1)."""
 
     def __init__(self, H, W, h, w, batch=1, device=0, shard_rank=0, shard_count=1, write_surface=False,
-                 generic=False, timing=False, image_pitch=None):
+                 generic=False, timing=False, image_pitch=None, score=N.NCC_SCORE_NCC):
         flags = (N.NCC_F_WRITE_SURFACE if write_surface else 0) | (N.NCC_F_GENERIC_KERNEL if generic else 0) | \
                 (N.NCC_F_TIMING if timing else 0)
         super().__init__(N.make_problem(N.NCC_MODE_MATCH, H, W, image_pitch, h, w, batch=batch,
-                                        shard_rank=shard_rank, shard_count=shard_count, flags=flags), device)
+                                        shard_rank=shard_rank, shard_count=shard_count, flags=flags,
+                                        score=score), device)
         self.write_surface = write_surface
 
     @property
@@ -92,13 +93,13 @@ class PivPlan(_Plan):
     """PIV: per-window NCC over a search range, peak + 3-point sub-pixel fit (Figs 5.8-5.12)."""
 
     def __init__(self, H, W, win, search, step, pairs=1, device=0, subpix=N.NCC_SUBPIX_GAUSS3, generic=False,
-                 timing=False, image_pitch=None):
+                 timing=False, image_pitch=None, score=N.NCC_SCORE_NCC):
         wh, ww = (win, win) if isinstance(win, int) else win
         my, mx = (search, search) if isinstance(search, int) else search
         sy, sx = (step, step) if isinstance(step, int) else step
         flags = (N.NCC_F_GENERIC_KERNEL if generic else 0) | (N.NCC_F_TIMING if timing else 0)
         super().__init__(N.make_problem(N.NCC_MODE_PIV, H, W, image_pitch, wh, ww, my, mx, sy, sx, batch=pairs,
-                                        flags=flags, subpix=subpix), device)
+                                        flags=flags, subpix=subpix, score=score), device)
 
     @property
     def grid(self):

@@ -228,7 +228,7 @@ void free_plan(ncc_plan pl) {
 }
 
 ncc_status validate(const ncc_problem& p) {
-  if (p.score != NCC_SCORE_NCC) return p.score == NCC_SCORE_SSD ? NCC_ERR_UNSUPPORTED : NCC_ERR_INVALID_ARGUMENT;
+  if (p.score != NCC_SCORE_NCC && p.score != NCC_SCORE_SSD) return NCC_ERR_INVALID_ARGUMENT;
   if (p.mode != NCC_MODE_MATCH && p.mode != NCC_MODE_PIV) return NCC_ERR_INVALID_ARGUMENT;
   if (p.image_h <= 0 || p.image_w <= 0 || p.tmpl_h <= 0 || p.tmpl_w <= 0) return NCC_ERR_INVALID_ARGUMENT;
   if (p.image_pitch < p.image_w) return NCC_ERR_INVALID_ARGUMENT;
@@ -393,6 +393,10 @@ ncc_status create_tm(ncc_plan pl) {
     const int ct = pl->use_ct ? 1 : 0;
     fill_kernel_info(pl, (const void*)v->k[1][ct], v->nt, v->smem[1][ct], pl->tiles_u * pl->tiles_v * pl->split,
                      p.batch, 1);
+    in.split = pl->split;
+    in.const_template = pl->use_ct;
+    in.slabs = pl->n_slabs;
+    in.launches_per_call = 4 + pl->n_slabs;  // prep, 2 window-sum passes, numerator(s), finalize
   }
   return NCC_OK;
 }
@@ -469,6 +473,7 @@ ncc_status create_piv(ncc_plan pl) {
   in.variant_id = (int)(v - kPivVariants);
   snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
   fill_kernel_info(pl, (const void*)v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
+  in.launches_per_call = 3 * ceil_div(p.batch, sb);  // per sub-batch: 2 window-sum passes + PIV kernel
   return NCC_OK;
 }
 
@@ -550,6 +555,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   a.part = pl->part;
   a.cnt = pl->cnt;
   a.S = pl->split;
+  a.ssd = p.score == NCC_SCORE_SSD;
   // TMA needs a 16-B aligned base and a pitch that is a multiple of 16 B; else plain loads.
   CUtensorMap map_img;
   memset(&map_img, 0, sizeof(map_img));
@@ -587,7 +593,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   mark(pl, s, 3);
   tm_finalize<<<ceil_div(p.batch, 128), 128, 0, s>>>(pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks),
-                                                     p.batch);
+                                                     p.batch, p.score == NCC_SCORE_SSD);
   mark(pl, s, 4);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch");
@@ -628,6 +634,7 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   a.scores = d_scores;
   a.subpix = p.subpix;
   a.BP = pl->piv_bp;
+  a.ssd = p.score == NCC_SCORE_SSD;
   // TMA maps over all frames of the call (3D: cols, rows, pair); plain loads otherwise
   CUtensorMap mB;
   memset(&mB, 0, sizeof(mB));

@@ -241,6 +241,7 @@ struct TmArgs {
   // total is carried between slab launches in `carry` ([batch][tiles][RV][NT]).
   int q_begin, q_end, c_row0, first, last;
   float* carry;
+  int ssd;                   // 0: NCC (argmax), 1: SSD = sum (T - W)^2 (argmin; Fig 5.10)
 };
 
 // Template chunks in the constant bank: FFMA takes the template from uniform registers
@@ -452,9 +453,14 @@ __global__ void __launch_bounds__(WX* WY * 32)
     for (int c = 0; c < RV; ++c) {
       const int v = v0 + lv + c;
       if (v < a.V) {
-        const float sc = ncc_normalize(total[c], a.S1[rowoff + v], a.S2[rowoff + v], n, ts);
+        const double s1 = a.S1[rowoff + v], s2 = a.S2[rowoff + v];
+        float sc;
+        if (a.ssd)  // sum T^2 - 2 sum T W + sum W^2, with sum T W = sum A_C W + Tbar S1
+          sc = (float)(ts.sumsq - 2.0 * ((double)total[c] + ts.sum / n * s1) + s2);
+        else
+          sc = ncc_normalize(total[c], s1, s2, n, ts);
         if (srow) srow[v] = sc;
-        const unsigned long long k = make_key(sc, (uint32_t)((int64_t)u * a.V + v));
+        const unsigned long long k = make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)u * a.V + v));
         best = k > best ? k : best;
       }
     }
@@ -505,16 +511,16 @@ __global__ void tm_template_prep(const float* __restrict__ tmpl, int64_t tpitch,
 }
 
 __global__ void tm_finalize(const unsigned long long* __restrict__ keys, const TemplateStats* ts, int V,
-                            PeakOut* __restrict__ peaks, int batch) {
+                            PeakOut* __restrict__ peaks, int batch, int ssd) {
   const int f = blockIdx.x * blockDim.x + threadIdx.x;
   if (f >= batch) return;
   const unsigned long long k = keys[f];
   const uint32_t idx = key_index(k);
   PeakOut p;
-  p.score = key_score(k);
+  p.score = ssd ? -key_score(k) : key_score(k);
   p.u = (int32_t)(idx / (uint32_t)V);
   p.v = (int32_t)(idx % (uint32_t)V);
-  p.flags = ts->flat ? (kFlatTemplate | kInvalid) : 0u;
+  p.flags = (ts->flat && !ssd) ? (kFlatTemplate | kInvalid) : 0u;
   peaks[f] = p;
 }
 
@@ -635,6 +641,7 @@ struct PivArgs {
   float* scores;     // nullable: [pair][Ky][Kx][OY][OX]
   int subpix;        // 0 Gauss3 (parabolic fallback), 1 parabola, 2 none
   int BP;            // RE: staged B pitch (floats), chosen on the host
+  int ssd;           // 0: NCC (argmax), 1: SSD (argmin, parabolic fit of the minimum)
 };
 
 // FFMA2 numerator core with template PAIRS (sm_100a fma.rn.f32x2):
@@ -747,6 +754,13 @@ __device__ __forceinline__ double subpix3(double cm, double c0, double cp, int m
   if (den >= 0.0) return 0.0;
   return num / den;
 }
+// SSD: three-point parabola through a minimum (0 if not a minimum or mode == none).
+__device__ __forceinline__ double subpix3_min(double cm, double c0, double cp, int mode) {
+  if (mode == 2) return 0.0;
+  const double den = 2.0 * (cm - 2.0 * c0 + cp);
+  if (den <= 0.0) return 0.0;
+  return (cm - cp) / den;
+}
 
 // NCC with the fp64 window sums and a fp32 rsqrt (PIV epilogue): |error| <= ~4e-7 absolute.
 __device__ __forceinline__ float ncc_normalize_fast(float num, double s1, double s2, double inv_n, double csum,
@@ -794,7 +808,7 @@ __global__ void __launch_bounds__(NT, MINB)
   constexpr int NW = (NT + 31) / 32;
   __shared__ double red[NW * 2 * WPB];
   __shared__ unsigned long long red_key[NW * WPB];
-  __shared__ double s_energy[WPB], s_csum[WPB];
+  __shared__ double s_energy[WPB], s_csum[WPB], s_mean[WPB], s_sumsq[WPB];
   __shared__ int s_flat[WPB];
   __shared__ __align__(8) uint64_t bar;
 
@@ -835,55 +849,92 @@ __global__ void __launch_bounds__(NT, MINB)
   }
 
   // ---- mask statistics (Fig 5.2), masks read from global (L2): mean, A_D, sum of fp32 A_C;
-  //      the centred mask is written straight into the template-pair layout
+  //      the centred mask is written straight into the template-pair layout.  Specialised
+  //      kernels know the element count at compile time: each thread issues all its loads up
+  //      front (latency overlapped) and keeps the values in registers for the second pass.
   const float* Af = a.A + (int64_t)pr * a.frame_stride;
   const int per_win = sh.h * sh.w;
   {
+    constexpr int PERT = SK ? (WPB * TH * TW + NT - 1) / NT : 1;
+    float mv[PERT];
     double v[2 * WPB];
 #pragma unroll
     for (int q = 0; q < 2 * WPB; ++q) v[q] = 0.0;
-    for (int e = tid; e < nvalid * per_win; e += NT) {
-      const int wi = e / per_win, k = e % per_win;
-      const double t = __ldg(Af + (int64_t)(wy(wi) + k / sh.w) * a.pitch + wx(wi) + k % sh.w);
+    if constexpr (SK) {
 #pragma unroll
-      for (int q = 0; q < WPB; ++q)
-        if (q == wi) { v[2 * q] += t; v[2 * q + 1] += t * t; }
+      for (int k = 0; k < PERT; ++k) {
+        const int e = tid + k * NT;
+        const int wi = e / per_win, r = e % per_win;
+        mv[k] = (wi < nvalid) ? __ldg(Af + (int64_t)(wy(wi) + r / sh.w) * a.pitch + wx(wi) + r % sh.w) : 0.0f;
+      }
+#pragma unroll
+      for (int k = 0; k < PERT; ++k) {
+        const int wi = (tid + k * NT) / per_win;
+        const double t = mv[k];
+#pragma unroll
+        for (int q = 0; q < WPB; ++q)
+          if (q == wi) { v[2 * q] += t; v[2 * q + 1] += t * t; }
+      }
+    } else {
+      for (int e = tid; e < nvalid * per_win; e += NT) {
+        const int wi = e / per_win, k = e % per_win;
+        const double t = __ldg(Af + (int64_t)(wy(wi) + k / sh.w) * a.pitch + wx(wi) + k % sh.w);
+#pragma unroll
+        for (int q = 0; q < WPB; ++q)
+          if (q == wi) { v[2 * q] += t; v[2 * q + 1] += t * t; }
+      }
     }
     block_sum_k<2 * WPB>(v, red);
     const double n = (double)sh.h * (double)sh.w;
     double m[WPB], sumsq[WPB];
 #pragma unroll
     for (int q = 0; q < WPB; ++q) { m[q] = v[2 * q] / n; sumsq[q] = v[2 * q + 1]; v[2 * q] = 0.0; v[2 * q + 1] = 0.0; }
-    const int WPd = sh.nCW * CW;  // padded mask width
-    const int per_pad = sh.h * WPd;
-    for (int e = tid; e < nvalid * per_pad; e += NT) {
-      const int wi = e / per_pad, k = e % per_pad;
-      const int i = k / WPd, j = k % WPd;
-      float ac = 0.0f;
-      if (j < sh.w) {
-        double mm = 0.0;
-#pragma unroll
-        for (int q = 0; q < WPB; ++q) mm = (q == wi) ? m[q] : mm;
-        const double d = (double)__ldg(Af + (int64_t)(wy(wi) + i) * a.pitch + wx(wi) + j) - mm;
-        ac = (float)d;
-#pragma unroll
-        for (int q = 0; q < WPB; ++q)
-          if (q == wi) { v[2 * q] += d * d; v[2 * q + 1] += (double)ac; }
-      }
-      // pairs of chunk jc: TP[p] = (t[p-1], t[p]); value j sits in TP[l].y and TP[l+1].x
+    // centred value j of row i of window wi -> pairs TP[l].y and TP[l+1].x of its chunk
+    auto put = [&](int wi, int i, int j, float ac) {
       float* tp = reinterpret_cast<float*>(TPw(wi) + i * sh.TPP + (j / CW) * sh.PB);
       const int l = j % CW;
       tp[2 * l + 1] = ac;
       tp[2 * (l + 1)] = ac;
       if (l == 0) tp[0] = 0.0f;               // TP[0].x = t[-1] = 0
       if (l == CW - 1) tp[2 * CW + 1] = 0.0f;  // TP[CW].y = t[CW] = 0
+    };
+    auto centre = [&](int wi, double x) {
+      double mm = 0.0;
+#pragma unroll
+      for (int q = 0; q < WPB; ++q) mm = (q == wi) ? m[q] : mm;
+      const double d = x - mm;
+      const float ac = (float)d;
+#pragma unroll
+      for (int q = 0; q < WPB; ++q)
+        if (q == wi) { v[2 * q] += d * d; v[2 * q + 1] += (double)ac; }
+      return ac;
+    };
+    if constexpr (SK && (TW % CW == 0)) {  // no padding columns: every element is a mask value
+#pragma unroll
+      for (int k = 0; k < PERT; ++k) {
+        const int e = tid + k * NT;
+        const int wi = e / per_win, r = e % per_win;
+        if (wi < nvalid) put(wi, r / sh.w, r % sh.w, centre(wi, (double)mv[k]));
+      }
+    } else {
+      const int WPd = sh.nCW * CW;  // padded mask width
+      const int per_pad = sh.h * WPd;
+      for (int e = tid; e < nvalid * per_pad; e += NT) {
+        const int wi = e / per_pad, k = e % per_pad;
+        const int i = k / WPd, j = k % WPd;
+        float ac = 0.0f;
+        if (j < sh.w) ac = centre(wi, (double)__ldg(Af + (int64_t)(wy(wi) + i) * a.pitch + wx(wi) + j));
+        put(wi, i, j, ac);
+      }
     }
     block_sum_k<2 * WPB>(v, red);  // (its barriers also publish the template pairs)
     if (tid < WPB) {
-      double e = 0, c = 0, ss = 0;
+      double e = 0, c = 0, ss = 0, mm = 0;
 #pragma unroll
       for (int q = 0; q < WPB; ++q)
-        if (q == tid) { e = v[2 * q]; c = v[2 * q + 1]; ss = sumsq[q]; }
+        if (q == tid) { e = v[2 * q]; c = v[2 * q + 1]; ss = sumsq[q]; mm = m[q]; }
+      s_mean[tid] = mm;
+      s_sumsq[tid] = ss;
       s_energy[tid] = e;
       s_csum[tid] = c;
       s_flat[tid] = (e <= kFlatRel * ss) ? 1 : 0;
@@ -934,9 +985,12 @@ __global__ void __launch_bounds__(NT, MINB)
         const int c = 2 * q + 1 - e;
         const int col = g * RV + c;
         float s = 0.0f;
-        if (col < sh.OX)
-          s = ncc_normalize_fast(e == 0 ? lo : hi, __ldg(S1f + mrow + col), __ldg(S2f + mrow + col), inv_n, csum,
-                                 energy, flat);
+        if (col < sh.OX) {
+          const double s1 = __ldg(S1f + mrow + col), s2 = __ldg(S2f + mrow + col);
+          const float num = e == 0 ? lo : hi;
+          s = a.ssd ? (float)(s_sumsq[wi] - 2.0 * ((double)num + s_mean[wi] * s1) + s2)
+                    : ncc_normalize_fast(num, s1, s2, inv_n, csum, energy, flat);
+        }
         out[c] = s;
       }
     }
@@ -978,7 +1032,7 @@ __global__ void __launch_bounds__(NT, MINB)
     const int row = k / sh.OX, col = k % sh.OX;
     const float s = Sc(wi)[row * sh.OXP + col];
     if (a.scores) a.scores[((int64_t)pr * nwin + lin0 + wi) * tile + k] = s;
-    const unsigned long long key = make_key(s, (uint32_t)k);
+    const unsigned long long key = make_key(a.ssd ? -s : s, (uint32_t)k);
 #pragma unroll
     for (int q = 0; q < WPB; ++q)
       if (q == wi) best[q] = key > best[q] ? key : best[q];
@@ -1003,19 +1057,21 @@ __global__ void __launch_bounds__(NT, MINB)
     const uint32_t k = key_index(bk);
     const int row = (int)(k / sh.OX), col = (int)(k % sh.OX);
     const int iy = row - sh.my, ix = col - sh.mx;
-    uint32_t flags = s_flat[wi] ? (kFlatTemplate | kInvalid) : 0u;
+    uint32_t flags = (s_flat[wi] && !a.ssd) ? (kFlatTemplate | kInvalid) : 0u;
     double ddy = 0.0, ddx = 0.0;
-    bool par;
+    bool par = false;
     if (row == 0 || row == sh.OY - 1) {
       flags |= kEdgeY;
     } else {
-      ddy = subpix3(S[(row - 1) * sh.OXP + col], S[row * sh.OXP + col], S[(row + 1) * sh.OXP + col], a.subpix, &par);
+      const double cm = S[(row - 1) * sh.OXP + col], c0 = S[row * sh.OXP + col], cp = S[(row + 1) * sh.OXP + col];
+      ddy = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
       if (par) flags |= kParabolaY;
     }
     if (col == 0 || col == sh.OX - 1) {
       flags |= kEdgeX;
     } else {
-      ddx = subpix3(S[row * sh.OXP + col - 1], S[row * sh.OXP + col], S[row * sh.OXP + col + 1], a.subpix, &par);
+      const double cm = S[row * sh.OXP + col - 1], c0 = S[row * sh.OXP + col], cp = S[row * sh.OXP + col + 1];
+      ddx = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
       if (par) flags |= kParabolaX;
     }
     VecOut o;
@@ -1023,7 +1079,7 @@ __global__ void __launch_bounds__(NT, MINB)
     o.ix = ix;
     o.dy = (float)(iy + ddy);
     o.dx = (float)(ix + ddx);
-    o.score = key_score(bk);
+    o.score = a.ssd ? -key_score(bk) : key_score(bk);
     o.flags = flags;
     a.vec[(int64_t)pr * nwin + lin0 + wi] = o;
   }

@@ -75,9 +75,9 @@ def test_invalid_arguments_rejected_before_device(L, kw):
     assert st == 1 and not h  # NCC_ERR_INVALID_ARGUMENT, *out == NULL
 
 
-def test_ssd_unsupported(L):
-    st, h = _create(score=N.NCC_SCORE_SSD)
-    assert st == 2 and not h
+def test_bad_score_rejected(L):
+    st, h = _create(score=5)
+    assert st == 1 and not h
 
 
 def test_null_arguments(L):
