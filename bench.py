@@ -373,7 +373,8 @@ def main():
 
     line = {"metric": metric, "value": value, "unit": unit, "n_gpus": ws, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": "strong" if cfg == 4 else "weak", "vs_baseline": None, "dtype": "f32",
+            "data": "synthetic",
             "config": {"workload": f"cfg{cfg}", **{k: v for k, v in synth.CONFIGS[cfg].items()},
                        "units_per_step_per_gpu": units_per_step, "l2": "flushed between steps (512 MiB write)",
                        "variant": plan.info.variant_name.decode(), "regs_per_thread": plan.info.regs_per_thread,
