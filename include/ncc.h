@@ -195,6 +195,15 @@ ncc_status ncc_plan_query(ncc_plan plan, void* info, size_t info_size);
 /* Timings of the most recent execute call (requires NCC_F_TIMING; otherwise zeros). */
 ncc_status ncc_plan_timing(ncc_plan plan, ncc_timing* out);
 
+/* Run-time specialisation ahead of use (no device needed): selects the kernel variant for
+ * *p exactly as ncc_plan_create would and, if that is a run-time specialised (NVRTC) kernel,
+ * compiles it into the on-disk binary cache (NCC_CACHE_DIR, default ~/.cache/ncc_b200; the
+ * paper's GPU-PF binary cache).  Writes the variant name (NUL-terminated) and
+ * *compiled_now = 1 if NVRTC ran in this call (0: ahead-of-time instance or cache hit).
+ * NCC_ERR_COMPILE if NVRTC is missing or fails (log in ncc_last_cuda_error); the plan would
+ * then use the generic kernel. */
+ncc_status ncc_specialize(const ncc_problem* p, char* variant_name, size_t name_size, int32_t* compiled_now);
+
 /* Library build facts: 100 = sm_100a build. */
 int32_t ncc_build_arch(void);
 

@@ -26,7 +26,7 @@ FLAG_FLAT_TEMPLATE, FLAG_EDGE_Y, FLAG_EDGE_X, FLAG_PARABOLA_Y, FLAG_PARABOLA_X, 
 
 EXPORTS = ["ncc_plan_create", "ncc_match", "piv_correlate", "piv_correlate_ex", "ncc_match_host",
            "piv_correlate_host", "ncc_plan_destroy", "ncc_status_string", "ncc_last_cuda_error",
-           "ncc_plan_query", "ncc_plan_timing", "ncc_build_arch"]
+           "ncc_plan_query", "ncc_plan_timing", "ncc_build_arch", "ncc_specialize"]
 
 
 class NccProblem(ctypes.Structure):
@@ -108,6 +108,8 @@ def lib():
         L.ncc_plan_query.argtypes = [P, P, ctypes.c_size_t]
         L.ncc_plan_timing.argtypes = [P, ctypes.POINTER(NccTiming)]
         L.ncc_build_arch.restype = ctypes.c_int32
+        L.ncc_specialize.argtypes = [ctypes.POINTER(NccProblem), ctypes.c_char_p, ctypes.c_size_t,
+                                     ctypes.POINTER(ctypes.c_int32)]
         for fn in EXPORTS:
             if fn not in ("ncc_status_string", "ncc_last_cuda_error", "ncc_build_arch"):
                 getattr(L, fn).restype = ctypes.c_int
@@ -194,3 +196,11 @@ def piv_correlate_host(plan, h_a, h_b, h_vectors, stream) -> None:
 
 def ncc_status_string(s: int) -> str:
     return lib().ncc_status_string(int(s)).decode()
+
+
+def ncc_specialize(problem: NccProblem) -> tuple[str, bool]:
+    """Compile (or find) the specialised kernel for `problem` into the binary cache (no GPU)."""
+    buf = ctypes.create_string_buffer(96)
+    now = ctypes.c_int32(0)
+    _check(lib().ncc_specialize(ctypes.byref(problem), buf, 96, ctypes.byref(now)), "ncc_specialize")
+    return buf.value.decode(), bool(now.value)

@@ -14,10 +14,12 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libncc_b200.so")
 SOURCES = [os.path.join(CSRC, "ncc_api.cu")]
-DEPS = SOURCES + [os.path.join(CSRC, "ncc_kernels.cuh"), os.path.join(ROOT, "include", "ncc.h")]
+KERNELS = os.path.join(CSRC, "ncc_kernels.cuh")
+SRC_INC = os.path.join(CSRC, "ncc_kernels_src.inc")  # generated: the kernel source for NVRTC
+DEPS = SOURCES + [KERNELS, os.path.join(CSRC, "ncc_jit.inc"), os.path.join(ROOT, "include", "ncc.h")]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
-              "--shared", "-Xcompiler", "-fPIC", "-Xptxas", "-v"]
+              "--shared", "-Xcompiler", "-fPIC", "-Xptxas", "-v", "-ldl"]
 
 
 def nvcc() -> str:
@@ -34,7 +36,19 @@ def needs_build() -> bool:
     return any(os.path.getmtime(d) > t for d in DEPS)
 
 
+def write_source_inc() -> None:
+    """Embed ncc_kernels.cuh as a string: the run-time specialiser (NVRTC) compiles the very
+    source the ahead-of-time instances come from."""
+    src = open(KERNELS).read()
+    assert ")NCC_SRC\"" not in src
+    body = 'static const char kNccKernelSource[] = R"NCC_SRC(' + src + ')NCC_SRC";\n'
+    if not os.path.exists(SRC_INC) or open(SRC_INC).read() != body:
+        with open(SRC_INC, "w") as f:
+            f.write(body)
+
+
 def build(force: bool = False, verbose: bool = False) -> str:
+    write_source_inc()
     if not force and not needs_build():
         return LIB
     tmp = LIB + f".tmp{os.getpid()}"

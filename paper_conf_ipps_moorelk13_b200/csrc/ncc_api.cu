@@ -9,6 +9,15 @@
 // ("RE").  Pointers and template values always stay run-time.
 #include <cuda_runtime.h>
 
+#include <dlfcn.h>
+#include <sys/stat.h>
+#include <sys/types.h>
+#include <unistd.h>
+
+#include <fstream>
+#include <sstream>
+
+#include <chrono>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -46,13 +55,14 @@ struct TmVariant {
   const char* name;
   int TH, TW;                 // 0 = run-time (RE)
   int RV, LX, WX, WY, CH, CW;
-  void (*k[2][2])(TmArgs, CUtensorMap, CUtensorMap);  // [tma][const template]
+  const void* k[2][2];  // [tma][const template] kernels (AOT function or JIT cudaKernel_t)
   int smem[2][2];
   int nt, bu, bv, ir, ip;
   int rv_nt() const { return RV * nt; }
 };
 
-#define TM_K(RV, LX, WX, WY, CH, CW, TH, TW, TMA, CT) tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW, TMA, CT>
+#define TM_K(RV, LX, WX, WY, CH, CW, TH, TW, TMA, CT) \
+  reinterpret_cast<const void*>(&tm_ncc_kernel<RV, LX, WX, WY, CH, CW, TH, TW, TMA, CT>)
 #define TM_VARIANT(NAME, TH, TW, RV, LX, WX, WY, CH, CW)                                                     \
   TmVariant {                                                                                             \
     NAME, TH, TW, RV, LX, WX, WY, CH, CW,                                                                 \
@@ -116,19 +126,20 @@ struct PivVariant {
   const char* name;
   int TH, TW, MY, MX;  // 0 = run-time (RE)
   int RV, CW, NT, WPB, ALIAS, IPT;
-  void (*k_tma)(PivArgs, CUtensorMap);  // nullptr: no TMA form
-  void (*k_ldg)(PivArgs, CUtensorMap);
+  const void* k_tma;  // AOT function or JIT cudaKernel_t
+  const void* k_ldg;
 };
 #define PIV_VARIANT_SK(NAME, TH, TW, MY, MX, RV, CW, NT, WPB, MINB, IPT)                                     \
   PivVariant {                                                                                              \
     NAME, TH, TW, MY, MX, RV, CW, NT, WPB, 1, IPT,                                                          \
-        piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, true, true, IPT>,                              \
-        piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, false, true, IPT>                              \
+        reinterpret_cast<const void*>(&piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, true, true, IPT>),  \
+        reinterpret_cast<const void*>(&piv_ncc_kernel<TH, TW, MY, MX, RV, CW, NT, WPB, MINB, false, true, IPT>)  \
   }
 #define PIV_VARIANT_RE(NAME, RV, CW, NT, MINB)                                                              \
   PivVariant {                                                                                              \
-    NAME, 0, 0, 0, 0, RV, CW, NT, 1, 0, 1, piv_ncc_kernel<0, 0, 0, 0, RV, CW, NT, 1, MINB, true, false, 1>,   \
-        piv_ncc_kernel<0, 0, 0, 0, RV, CW, NT, 1, MINB, false, false, 1>                                     \
+    NAME, 0, 0, 0, 0, RV, CW, NT, 1, 0, 1,                                                                 \
+        reinterpret_cast<const void*>(&piv_ncc_kernel<0, 0, 0, 0, RV, CW, NT, 1, MINB, true, false, 1>),       \
+        reinterpret_cast<const void*>(&piv_ncc_kernel<0, 0, 0, 0, RV, CW, NT, 1, MINB, false, false, 1>)       \
   }
 
 const PivVariant kPivVariants[] = {
@@ -151,6 +162,88 @@ struct ConstSlot {
 };
 ConstSlot g_const_slot[64];
 
+// Run-time mirror of TmTile<> (same formulas) for run-time specialised variants.
+TmVariant tm_geom(int RV, int LX, int WX, int WY, int CH, int CW) {
+  TmVariant v{};
+  v.RV = RV; v.LX = LX; v.WX = WX; v.WY = WY; v.CH = CH; v.CW = CW;
+  v.nt = WX * WY * 32;
+  v.bu = WY * (32 / LX);
+  v.bv = WX * LX * RV;
+  v.ir = v.bu + CH - 1;
+  v.ip = pick_pitch(v.bv + CW, RV, LX);
+  const int tb = CH * CW * 4, ib = v.ir * v.ip * 4;
+  const int tal = ((tb + 127) / 128) * 128, ial = ((ib + 127) / 128) * 128;
+  v.smem[0][0] = tb + ib;
+  v.smem[0][1] = ib;
+  v.smem[1][0] = 2 * (tal + ial);
+  v.smem[1][1] = 2 * ial;
+  return v;
+}
+
+// Smallest-padding chunk width / height from the candidates (ties -> the larger chunk).
+int pick_chunk(int n, const int* cands, int nc) {
+  int best = cands[0], bp = 1 << 30;
+  for (int i = 0; i < nc; ++i) {
+    const int pad = ((n + cands[i] - 1) / cands[i]) * cands[i] - n;
+    if (pad < bp) { bp = pad; best = cands[i]; }
+  }
+  return best;
+}
+
+struct TmJitChoice {
+  int RV, LX, WX, WY, CH, CW;
+  bool ct;
+};
+TmJitChoice tm_jit_choice(int h, int w) {
+  static const int cw[] = {64, 32, 16}, ch[] = {32, 16};
+  TmJitChoice c{12, 4, 1, 4, pick_chunk(h, ch, 2), pick_chunk(w, cw, 3), false};
+  const int WP = ((w + c.CW - 1) / c.CW) * c.CW;
+  c.ct = (kConstTplFloats / WP) / c.CH * c.CH >= c.CH;
+  return c;
+}
+
+struct PivJitChoice {
+  int RV, CW, NT, WPB, MINB, BP, items;
+  int64_t win_fl;
+  bool ok;
+};
+template <int CW>
+PivShape<12, CW> piv_shape(int h, int w, int my, int mx, int BP) { return PivShape<12, CW>(h, w, my, mx, BP, true); }
+PivJitChoice piv_jit_choice(int h, int w, int my, int mx) {
+  static const int cw[] = {64, 32, 16};
+  PivJitChoice c{};
+  c.RV = 12;
+  c.CW = pick_chunk(w, cw, 3);
+  const int OX = 2 * mx + 1, NG = (OX + 11) / 12;
+  c.BP = piv_pick_pitch(NG * 12 + ((w + c.CW - 1) / c.CW) * c.CW, 12, NG);
+  int items;
+  if (c.CW == 64) { auto ps = piv_shape<64>(h, w, my, mx, c.BP); items = ps.items; c.win_fl = ps.win_fl; }
+  else if (c.CW == 32) { auto ps = piv_shape<32>(h, w, my, mx, c.BP); items = ps.items; c.win_fl = ps.win_fl; }
+  else { auto ps = piv_shape<16>(h, w, my, mx, c.BP); items = ps.items; c.win_fl = ps.win_fl; }
+  c.items = items;
+  c.ok = false;
+  if (items > 1024) return c;  // one item per thread (score tile aliased on the template pairs)
+  const int64_t kTwoPerSm = 113 * 1024, kOnePerSm = 227 * 1024;
+  double best = -1.0;
+  for (int k = 1; k <= 8; ++k) {
+    const int nt = ((k * items + 31) / 32) * 32;
+    const int64_t smem = (int64_t)k * c.win_fl * 4;
+    if (nt > 1024 || smem > kOnePerSm) break;
+    double util = (double)(k * items) / nt;
+    if (smem <= kTwoPerSm) util += 0.05;  // prefer two resident CTAs per SM (phase overlap)
+    if (util > best + 1e-9) {
+      best = util;
+      c.WPB = k;
+      c.NT = nt;
+      c.MINB = smem <= kTwoPerSm ? 2 : 1;
+      c.ok = true;
+    }
+  }
+  return c;
+}
+
+#include "ncc_jit.inc"
+
 }  // namespace
 
 // ------------------------------------------------------------------ plan object
@@ -168,6 +261,13 @@ struct ncc_plan_s {
   float* part;
   unsigned int* cnt;
   const TmVariant* tmv;
+  TmVariant tmv_store;  // run-time specialised variant
+  PivVariant pivv_store;
+  cudaLibrary_t jit_lib;
+  void* jit_ctpl;  // the JIT library's own constant-bank template slot (nullptr: AOT, global slot)
+  double jit_ms;   // NVRTC compile time (0 when loaded from the cache)
+  int jit_ct;      // JIT TM: template mode compiled (1 = constant bank)
+  char jit_name[96];
   float* tplC;
   TemplateStats* tst;
   unsigned long long* keys;
@@ -224,6 +324,7 @@ void free_plan(ncc_plan pl) {
   if (pl->ev_fork) cudaEventDestroy(pl->ev_fork);
   if (pl->ev_join) cudaEventDestroy(pl->ev_join);
   if (pl->side) cudaStreamDestroy(pl->side);
+  if (pl->jit_lib) cudaLibraryUnload(pl->jit_lib);
   delete pl;
 }
 
@@ -284,16 +385,55 @@ ncc_status create_tm(ncc_plan pl) {
   pl->Ub = pl->u_end - pl->u_begin;
   pl->Hs = pl->Ub + h - 1;
 
+  // variant selection (a8): AOT specialised instance > run-time specialised (NVRTC) > generic RE
   const TmVariant* v = &kTmVariants[0];
+  bool aot = false;
   if (!(p.flags & NCC_F_GENERIC_KERNEL))
     for (const TmVariant& c : kTmVariants)
       if (c.TH == h && c.TW == w) {
         v = &c;
+        aot = true;
         break;  // first matching specialised instance is the default
       }
   if (const char* force = getenv("NCC_FORCE_VARIANT"))  // sweeps: any instance valid for (h, w)
     for (const TmVariant& c : kTmVariants)
-      if (strcmp(force, c.name) == 0 && (c.TH == 0 || (c.TH == h && c.TW == w))) v = &c;
+      if (strcmp(force, c.name) == 0 && (c.TH == 0 || (c.TH == h && c.TW == w))) {
+        v = &c;
+        aot = c.TH != 0;
+      }
+  if (!aot && jit_allowed(p.flags)) {
+    const TmJitChoice jc = tm_jit_choice(h, w);
+    const std::vector<std::string> names = {tm_name(jc.RV, jc.LX, jc.WX, jc.WY, jc.CH, jc.CW, h, w, false, jc.ct),
+                                            tm_name(jc.RV, jc.LX, jc.WX, jc.WY, jc.CH, jc.CW, h, w, true, jc.ct),
+                                            "&nccb::c_tpl"};
+    JitResult jr;
+    std::string err;
+    if (jit_build(names, &jr, &err) == NCC_OK) {
+      NCC_CUDA(cudaLibraryLoadData(&pl->jit_lib, jr.cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
+      TmVariant jv = tm_geom(jc.RV, jc.LX, jc.WX, jc.WY, jc.CH, jc.CW);
+      jv.TH = h;
+      jv.TW = w;
+      cudaKernel_t k0, k1;
+      NCC_CUDA(cudaLibraryGetKernel(&k0, pl->jit_lib, jr.lowered[0].c_str()));
+      NCC_CUDA(cudaLibraryGetKernel(&k1, pl->jit_lib, jr.lowered[1].c_str()));
+      const int ct = jc.ct ? 1 : 0;
+      pl->jit_ct = ct;
+      jv.k[0][ct] = reinterpret_cast<const void*>(k0);
+      jv.k[1][ct] = reinterpret_cast<const void*>(k1);
+      jv.k[0][1 - ct] = jv.k[0][ct];  // only the chosen template source is compiled
+      jv.k[1][1 - ct] = jv.k[1][ct];
+      size_t csz = 0;
+      NCC_CUDA(cudaLibraryGetGlobal(&pl->jit_ctpl, &csz, pl->jit_lib, jr.lowered[2].c_str()));
+      pl->jit_ms = jr.cached ? 0.0 : jr.compile_ms;
+      snprintf(pl->jit_name, sizeof(pl->jit_name), "tm_jit_%dx%d_rv%d_lx%d_%dx%d_c%dx%d%s", h, w, jc.RV, jc.LX, jc.WY,
+               jc.WX, jc.CH, jc.CW, jr.cached ? "_cached" : "");
+      jv.name = pl->jit_name;
+      pl->tmv_store = jv;
+      v = &pl->tmv_store;
+    } else {
+      g_last_cuda_error = err;  // reported via ncc_last_cuda_error; fall back to the generic kernel
+    }
+  }
   pl->tmv = v;
   const int nCH = ceil_div(h, v->CH), nCW = ceil_div(w, v->CW);
   pl->HP = nCH * v->CH;
@@ -304,9 +444,9 @@ ncc_status create_tm(ncc_plan pl) {
   NCC_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, pl->device));
   for (int t = 0; t < 2; ++t)
     for (int c = 0; c < 2; ++c) {
+      if (pl->jit_lib && c != pl->jit_ct) continue;  // JIT: only the chosen template mode is compiled
       if (v->smem[t][c] > maxsm) return NCC_ERR_UNSUPPORTED;
-      NCC_CUDA(cudaFuncSetAttribute((const void*)v->k[t][c], cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                    v->smem[t][c]));
+      NCC_CUDA(cudaFuncSetAttribute(v->k[t][c], cudaFuncAttributeMaxDynamicSharedMemorySize, v->smem[t][c]));
     }
   const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
   if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
@@ -315,7 +455,7 @@ ncc_status create_tm(ncc_plan pl) {
 
   // constant-bank template: slabs of whole row-chunks that fit 64 KB (NCC_NO_CONST_TPL=1 disables)
   pl->slab_rows = (kConstTplFloats / pl->WP) / v->CH * v->CH;
-  pl->use_ct = pl->slab_rows >= v->CH && !getenv("NCC_NO_CONST_TPL");
+  pl->use_ct = pl->slab_rows >= v->CH && (pl->jit_lib ? true : !getenv("NCC_NO_CONST_TPL"));
   if (pl->slab_rows > pl->HP) pl->slab_rows = pl->HP;
   pl->n_slabs = pl->use_ct ? ceil_div(pl->HP, pl->slab_rows) : 1;
 
@@ -384,14 +524,14 @@ ncc_status create_tm(ncc_plan pl) {
   in.u_end = pl->u_end;
   in.outputs_per_call = (int64_t)pl->Ub * pl->V * p.batch;
   in.flops_per_call = 2.0 * h * (double)w * (double)in.outputs_per_call;
-  in.specialized = v->TH != 0;
-  in.variant_id = (int)(v - kTmVariants);
+  in.specialized = pl->jit_lib ? 2 : (v->TH != 0);
+  in.variant_id = pl->jit_lib ? -1 : (int)(v - kTmVariants);
   snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
   snprintf(in.variant_name + strlen(in.variant_name), sizeof(in.variant_name) - strlen(in.variant_name), "_s%d%s",
            pl->split, pl->use_ct ? (pl->n_slabs > 1 ? "_cslab" : "_ctpl") : "_stpl");
   {
     const int ct = pl->use_ct ? 1 : 0;
-    fill_kernel_info(pl, (const void*)v->k[1][ct], v->nt, v->smem[1][ct], pl->tiles_u * pl->tiles_v * pl->split,
+    fill_kernel_info(pl, v->k[1][ct], v->nt, v->smem[1][ct], pl->tiles_u * pl->tiles_v * pl->split,
                      p.batch, 1);
     in.split = pl->split;
     in.const_template = pl->use_ct;
@@ -411,14 +551,45 @@ ncc_status create_piv(ncc_plan pl) {
   pl->map_h = p.image_h - h + 1;
   pl->map_w = p.image_w - w + 1;
 
+  // variant selection (a8): AOT specialised instance > run-time specialised (NVRTC) > generic RE
   const PivVariant* v = &kPivVariants[0];
+  bool aot = false;
   if (!(p.flags & NCC_F_GENERIC_KERNEL))
     for (const PivVariant& c : kPivVariants)
-      if (c.TH == h && c.TW == w && c.MY == my && c.MX == mx) v = &c;
+      if (c.TH == h && c.TW == w && c.MY == my && c.MX == mx) {
+        v = &c;
+        aot = true;
+      }
+  if (!aot && jit_allowed(p.flags)) {
+    const PivJitChoice jc = piv_jit_choice(h, w, my, mx);
+    if (jc.ok) {
+      const std::vector<std::string> names = {
+          piv_name(h, w, my, mx, jc.RV, jc.CW, jc.NT, jc.WPB, jc.MINB, true, true, 1),
+          piv_name(h, w, my, mx, jc.RV, jc.CW, jc.NT, jc.WPB, jc.MINB, false, true, 1)};
+      JitResult jr;
+      std::string err;
+      if (jit_build(names, &jr, &err) == NCC_OK) {
+        NCC_CUDA(cudaLibraryLoadData(&pl->jit_lib, jr.cubin.data(), nullptr, nullptr, 0, nullptr, nullptr, 0));
+        cudaKernel_t k0, k1;
+        NCC_CUDA(cudaLibraryGetKernel(&k0, pl->jit_lib, jr.lowered[0].c_str()));
+        NCC_CUDA(cudaLibraryGetKernel(&k1, pl->jit_lib, jr.lowered[1].c_str()));
+        pl->jit_ms = jr.cached ? 0.0 : jr.compile_ms;
+        snprintf(pl->jit_name, sizeof(pl->jit_name), "piv_jit_%dx%d_m%dx%d_rv%d_cw%d_nt%d_w%d%s", h, w, my, mx, jc.RV,
+                 jc.CW, jc.NT, jc.WPB, jr.cached ? "_cached" : "");
+        PivVariant jv{pl->jit_name, h, w, my, mx, jc.RV, jc.CW, jc.NT, jc.WPB, 1, 1,
+                      reinterpret_cast<const void*>(k0), reinterpret_cast<const void*>(k1)};
+        pl->pivv_store = jv;
+        v = &pl->pivv_store;
+      } else {
+        g_last_cuda_error = err;
+      }
+    }
+  }
   pl->pivv = v;
   const int RV = v->RV, CW = v->CW;
   const int NG = (pl->OX + RV - 1) / RV;
   pl->piv_bp = v->TH ? piv_sk_pitch(v->TW, v->MX, RV, CW) : piv_pick_pitch(NG * RV + ((w + CW - 1) / CW) * CW, RV, NG);
+  (void)NG;
   const bool alias = v->ALIAS != 0;
   int items = 0;
   const int64_t win_fl = [&] {
@@ -441,8 +612,8 @@ ncc_status create_piv(ncc_plan pl) {
   int maxsm = 0;
   NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
   if (win_fl * 4 * v->WPB > maxsm) return NCC_ERR_UNSUPPORTED;
-  NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
-  NCC_CUDA(cudaFuncSetAttribute((const void*)v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
+  NCC_CUDA(cudaFuncSetAttribute(v->k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
+  NCC_CUDA(cudaFuncSetAttribute(v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
   const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
   if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
   NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT>,
@@ -469,10 +640,10 @@ ncc_status create_piv(ncc_plan pl) {
   in.Kx = pl->Kx;
   in.outputs_per_call = (int64_t)pl->Ky * pl->Kx * p.batch;
   in.flops_per_call = 2.0 * h * (double)w * pl->OY * (double)pl->OX * (double)in.outputs_per_call;
-  in.specialized = v->TH != 0;
-  in.variant_id = (int)(v - kPivVariants);
+  in.specialized = pl->jit_lib ? 2 : (v->TH != 0);
+  in.variant_id = pl->jit_lib ? -1 : (int)(v - kPivVariants);
   snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
-  fill_kernel_info(pl, (const void*)v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
+  fill_kernel_info(pl, v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
   in.launches_per_call = 3 * ceil_div(p.batch, sb);  // per sub-batch: 2 window-sum passes + PIV kernel
   return NCC_OK;
 }
@@ -570,6 +741,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   const int t = use_tma ? 1 : 0, ct = pl->use_ct ? 1 : 0;
   const int nCWl = pl->WP / v->CW;
   a.carry = pl->carry;
+  void* args[3] = {&a, &map_img, &pl->map_tpl};
   for (int sl = 0; sl < pl->n_slabs; ++sl) {
     const int r0 = sl * pl->slab_rows;
     const int r1 = (r0 + pl->slab_rows < pl->HP) ? r0 + pl->slab_rows : pl->HP;
@@ -578,17 +750,21 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     a.c_row0 = r0;
     a.first = sl == 0;
     a.last = sl == pl->n_slabs - 1;
-    if (ct) {  // template rows [r0, r1) into the constant bank (stream-ordered after the prep)
+    if (ct && pl->jit_ctpl) {  // the plan's own constant slot (JIT library): stream order suffices
+      NCC_CUDA(cudaMemcpyAsync(pl->jit_ctpl, pl->tplC + (size_t)r0 * pl->WP, (size_t)(r1 - r0) * pl->WP * 4,
+                               cudaMemcpyDeviceToDevice, s));
+      NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
+    } else if (ct) {  // template rows [r0, r1) into the constant bank (stream-ordered after the prep)
       ConstSlot& cs = g_const_slot[pl->device & 63];
       std::lock_guard<std::mutex> lk(cs.mu);
       if (!cs.done) NCC_CUDA(cudaEventCreateWithFlags(&cs.done, cudaEventDisableTiming));
       else NCC_CUDA(cudaStreamWaitEvent(s, cs.done, 0));
       NCC_CUDA(cudaMemcpyToSymbolAsync(c_tpl, pl->tplC + (size_t)r0 * pl->WP, (size_t)(r1 - r0) * pl->WP * 4, 0,
                                        cudaMemcpyDeviceToDevice, s));
-      v->k[t][ct]<<<grid, v->nt, v->smem[t][ct], s>>>(a, map_img, pl->map_tpl);
+      NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
       NCC_CUDA(cudaEventRecord(cs.done, s));
     } else {
-      v->k[t][ct]<<<grid, v->nt, v->smem[t][ct], s>>>(a, map_img, pl->map_tpl);
+      NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
     }
   }
   mark(pl, s, 3);
@@ -654,10 +830,8 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
     mark(pl, s, 3 * sb + 1);
     a.pair0 = p0;
     dim3 grid(groups, 1, np);
-    if (use_tma)
-      v->k_tma<<<grid, v->NT, pl->piv_smem, s>>>(a, mB);
-    else
-      v->k_ldg<<<grid, v->NT, pl->piv_smem, s>>>(a, mB);
+    void* args[2] = {&a, &mB};
+    NCC_CUDA(cudaLaunchKernel(use_tma ? v->k_tma : v->k_ldg, grid, dim3(v->NT), args, (size_t)pl->piv_smem, s));
     mark(pl, s, 3 * sb + 2);
     mark(pl, s, 3 * sb + 3);
   }
@@ -701,6 +875,58 @@ const char* ncc_status_string(ncc_status s) {
 const char* ncc_last_cuda_error(void) { return g_last_cuda_error.c_str(); }
 
 int32_t ncc_build_arch(void) { return 100; }
+
+ncc_status ncc_specialize(const ncc_problem* p, char* variant_name, size_t name_size, int32_t* compiled_now) {
+  if (!p) return NCC_ERR_INVALID_ARGUMENT;
+  ncc_status st = validate(*p);
+  if (st) return st;
+  if (compiled_now) *compiled_now = 0;
+  const int h = p->tmpl_h, w = p->tmpl_w, my = p->search_y, mx = p->search_x;
+  std::string name;
+  std::vector<std::string> names;
+  if (p->mode == NCC_MODE_MATCH) {
+    for (const TmVariant& c : kTmVariants)
+      if (!(p->flags & NCC_F_GENERIC_KERNEL) && c.TH == h && c.TW == w) {
+        name = c.name;
+        break;
+      }
+    if (name.empty() && jit_allowed(p->flags)) {
+      const TmJitChoice jc = tm_jit_choice(h, w);
+      names = {tm_name(jc.RV, jc.LX, jc.WX, jc.WY, jc.CH, jc.CW, h, w, false, jc.ct),
+               tm_name(jc.RV, jc.LX, jc.WX, jc.WY, jc.CH, jc.CW, h, w, true, jc.ct), "&nccb::c_tpl"};
+      char b[96];
+      snprintf(b, sizeof(b), "tm_jit_%dx%d_rv%d_lx%d_%dx%d_c%dx%d", h, w, jc.RV, jc.LX, jc.WY, jc.WX, jc.CH, jc.CW);
+      name = b;
+    }
+    if (name.empty()) name = kTmVariants[0].name;
+  } else {
+    for (const PivVariant& c : kPivVariants)
+      if (!(p->flags & NCC_F_GENERIC_KERNEL) && c.TH == h && c.TW == w && c.MY == my && c.MX == mx) name = c.name;
+    if (name.empty() && jit_allowed(p->flags)) {
+      const PivJitChoice jc = piv_jit_choice(h, w, my, mx);
+      if (jc.ok) {
+        names = {piv_name(h, w, my, mx, jc.RV, jc.CW, jc.NT, jc.WPB, jc.MINB, true, true, 1),
+                 piv_name(h, w, my, mx, jc.RV, jc.CW, jc.NT, jc.WPB, jc.MINB, false, true, 1)};
+        char b[96];
+        snprintf(b, sizeof(b), "piv_jit_%dx%d_m%dx%d_rv%d_cw%d_nt%d_w%d", h, w, my, mx, jc.RV, jc.CW, jc.NT, jc.WPB);
+        name = b;
+      }
+    }
+    if (name.empty()) name = kPivVariants[0].name;
+  }
+  if (!names.empty()) {
+    JitResult jr;
+    std::string err;
+    st = jit_build(names, &jr, &err);
+    if (st) {
+      g_last_cuda_error = err;
+      return st;
+    }
+    if (compiled_now) *compiled_now = jr.cached ? 0 : 1;
+  }
+  if (variant_name && name_size) snprintf(variant_name, name_size, "%s", name.c_str());
+  return NCC_OK;
+}
 
 ncc_status ncc_plan_create(const ncc_problem* p, int device, ncc_plan* out) {
   if (!out) return NCC_ERR_INVALID_ARGUMENT;

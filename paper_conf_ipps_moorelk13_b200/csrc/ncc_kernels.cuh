@@ -20,9 +20,21 @@
 // running total, bounding fp32 error growth.  Denominator from fp64 window
 // sums; normalisation in fp64; packed 64-bit (score, -index) keys for a deterministic argmax.
 #pragma once
+#ifdef __CUDACC_RTC__
+// Run-time specialisation (NVRTC, csrc/ncc_jit.inc): no host headers; the few types used here.
+typedef int int32_t;
+typedef unsigned int uint32_t;
+typedef long long int64_t;
+typedef unsigned long long uint64_t;
+struct alignas(64) CUtensorMap_st {
+  unsigned long long opaque[16];
+};
+typedef CUtensorMap_st CUtensorMap;
+#else
 #include <cuda.h>  // CUtensorMap (type only; encoded on the host through the runtime entry point)
 #include <cuda_runtime.h>
 #include <stdint.h>
+#endif
 
 namespace nccb {
 

@@ -55,12 +55,14 @@ def test_cfg1_full_surface(generic):
 @pytest.mark.parametrize("H,W,h,w,smooth", [(100, 137, 23, 17, False), (157, 123, 33, 41, True),
                                             (300, 280, 156, 116, False), (70, 90, 1, 1, False),
                                             (64, 64, 64, 64, False), (41, 300, 7, 290, False)])
-def test_generic_ragged_shapes(H, W, h, w, smooth):
+@pytest.mark.parametrize("generic", [True, False])
+def test_ragged_shapes_generic_and_runtime_specialised(H, W, h, w, smooth, generic):
+    """generic=True: run-time-evaluated kernel; False: NVRTC-specialised for (h, w)."""
     img = synth.smooth_image(H, W, 7) if smooth else synth.uniform_image(H, W, 7)
     T, u0, v0 = synth.planted_template(img, h, w, 8)
     ref, pk = oracle.ncc_match(img, T)
-    peaks, s, info = run_match(img, T)
-    assert info["specialized"] == 0
+    peaks, s, info = run_match(img, T, generic=generic)
+    assert info["specialized"] == (0 if generic else 2), info["variant_name"]
     assert np.max(np.abs(s[0] - ref)) <= TOL
     if h * w > 1:
         assert (peaks["u"][0], peaks["v"][0]) == (u0, v0)
