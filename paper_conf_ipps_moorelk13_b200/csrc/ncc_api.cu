@@ -146,6 +146,10 @@ const PivVariant kPivVariants[] = {
     PIV_VARIANT_RE("piv_re_rv12_cw16_nt256", 12, 16, 256, 1),
     PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt416_w4", 32, 32, 16, 16, 12, 32, 416, 4, 2, 1),
     PIV_VARIANT_SK("piv_sk_64x64_m32_rv12_nt416_w1", 64, 64, 32, 32, 12, 64, 416, 1, 2, 1),
+    // alternatives with warp counts that are multiples of 4 (even SMSP load; NCC_FORCE_VARIANT)
+    PIV_VARIANT_SK("piv_sk_64x64_m32_rv12_nt512_w1", 64, 64, 32, 32, 12, 64, 512, 1, 2, 1),
+    PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt512_w5", 32, 32, 16, 16, 12, 32, 512, 5, 1, 1),
+    PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt512_w4", 32, 32, 16, 16, 12, 32, 512, 4, 2, 1),
 };
 
 constexpr int kBoxRowsNT = 256, kBoxRowsSEG = 2048;  // max segment; actual = min(V, SEG)
@@ -556,9 +560,15 @@ ncc_status create_piv(ncc_plan pl) {
   bool aot = false;
   if (!(p.flags & NCC_F_GENERIC_KERNEL))
     for (const PivVariant& c : kPivVariants)
-      if (c.TH == h && c.TW == w && c.MY == my && c.MX == mx) {
-        v = &c;
+      if (c.TH == h && c.TW == w && c.MY == my && c.MX == mx && !aot) {
+        v = &c;  // first matching specialised instance is the default
         aot = true;
+      }
+  if (const char* force = getenv("NCC_FORCE_VARIANT"))  // sweeps: any instance valid for the shape
+    for (const PivVariant& c : kPivVariants)
+      if (strcmp(force, c.name) == 0 && (c.TH == 0 || (c.TH == h && c.TW == w && c.MY == my && c.MX == mx))) {
+        v = &c;
+        aot = c.TH != 0;
       }
   if (!aot && jit_allowed(p.flags)) {
     const PivJitChoice jc = piv_jit_choice(h, w, my, mx);

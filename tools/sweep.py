@@ -52,7 +52,7 @@ def tm(cfg, variants, splits):
                                   "grid": plan.info.grid_x}), flush=True)
 
 
-if __name__ == "__main__":
+if __name__ == "__main__" and sys.argv[1] == "tm":
     kind, cfg = sys.argv[1], int(sys.argv[2])
     if kind == "tm":
         vs = [None, "tm_sk_128x128_rv12_lx4_8x1_c32x64", "tm_sk_128x128_rv12_lx4_4x2_c32x64",
@@ -63,3 +63,28 @@ if __name__ == "__main__":
             else:
                 os.environ.pop("NCC_NO_CONST_TPL", None)
             tm(cfg, vs, [None, 1, 2, 4, 8] if cfg == 2 else [None])
+
+
+def piv(cfg, variants, pairs):
+    import bench
+    c = synth.CONFIGS[cfg]
+    wl = dict(cfg=cfg, H=c["H"], W=c["W"], h=c["h"], w=c["w"], m=c["m"], step=c["step"], pairs=pairs, rank=0)
+    dev = torch.device("cuda", 0)
+    A, B, _ = bench.piv_frames_device(wl, dev, torch)
+    for v in variants:
+        if v:
+            os.environ["NCC_FORCE_VARIANT"] = v
+        else:
+            os.environ.pop("NCC_FORCE_VARIANT", None)
+        with PivPlan(c["H"], c["W"], c["h"], c["m"], c["step"], pairs=pairs, timing=True) as plan:
+            ms = time_plan(plan, lambda: plan.correlate(A, B), reps=5)
+            print(json.dumps({"cfg": cfg, "variant": plan.info.variant_name.decode(), "ms": ms,
+                              "tflops": plan.info.flops_per_call / ms / 1e9, "regs": plan.info.regs_per_thread,
+                              "smem": plan.info.smem_per_block, "grid": plan.info.grid_x}), flush=True)
+
+
+if __name__ == "__main__" and sys.argv[1] == "piv":
+    cfg = int(sys.argv[2])
+    vs = {3: [None, "piv_sk_32x32_m16_rv12_nt512_w5", "piv_sk_32x32_m16_rv12_nt512_w4", "piv_re_rv12_cw16_nt256"],
+          4: [None, "piv_sk_64x64_m32_rv12_nt512_w1", "piv_re_rv12_cw16_nt256"]}[cfg]
+    piv(cfg, vs, 1 if cfg == 3 else 16)
