@@ -367,7 +367,10 @@ def main():
     prof = os.path.join(ROOT, "profiles", "roofline_traffic.json")
     if os.path.exists(prof):
         try:
-            traffic = json.load(open(prof)).get(f"cfg{cfg}")
+            tj = json.load(open(prof))
+            traffic = tj.get(f"cfg{cfg}")
+            if traffic is None and f"cfg{cfg}_per_pair" in tj:
+                traffic = tj[f"cfg{cfg}_per_pair"] * plan.info.grid_z
         except Exception:
             traffic = None
 
