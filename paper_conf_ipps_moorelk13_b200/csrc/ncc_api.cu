@@ -84,6 +84,8 @@ const TmVariant kTmVariants[] = {
     // alternative 128x128 tilings (selected with NCC_FORCE_VARIANT for sweeps)
     TM_VARIANT("tm_sk_128x128_rv12_lx4_8x1_c32x64", 128, 128, 12, 4, 1, 8, 32, 64),
     TM_VARIANT("tm_sk_128x128_rv12_lx4_4x2_c32x64", 128, 128, 12, 4, 2, 4, 32, 64),
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c16x64", 128, 128, 12, 4, 1, 4, 16, 64),
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_8x1_c16x64", 128, 128, 12, 4, 1, 8, 16, 64),
     TM_VARIANT("tm_sk_512x512_rv12_lx4_4x1_c32x64", 512, 512, 12, 4, 1, 4, 32, 64),
 };
 
@@ -477,7 +479,7 @@ ncc_status create_tm(ncc_plan pl) {
     const int nq = pl->n_slabs > 1 ? 1 : nCH * nCW;  // slab launches carry totals: no split
     int best_s = 1;
     double best_e = 0.0;
-    for (int S = 1; S <= nq && S <= 8; ++S) {
+    for (int S = 1; S <= nq && S <= 16; ++S) {
       const int64_t units = tiles_full * S;
       const double e = (double)units / (double)(((units + slots - 1) / slots) * slots);
       if (e > best_e + 0.02) {

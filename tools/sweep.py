@@ -56,13 +56,13 @@ if __name__ == "__main__" and sys.argv[1] == "tm":
     kind, cfg = sys.argv[1], int(sys.argv[2])
     if kind == "tm":
         vs = [None, "tm_sk_128x128_rv12_lx4_8x1_c32x64", "tm_sk_128x128_rv12_lx4_4x2_c32x64",
-              "tm_re_rv12_lx4_4x1_c32x32"] if cfg == 2 else [None, "tm_re_rv12_lx4_4x1_c32x32"]
-        for ct in ("1", None):
+              "tm_sk_128x128_rv12_lx4_4x1_c16x64", "tm_sk_128x128_rv12_lx4_8x1_c16x64"] if cfg == 2 else [None]
+        for ct in (None,):
             if ct:
                 os.environ["NCC_NO_CONST_TPL"] = ct
             else:
                 os.environ.pop("NCC_NO_CONST_TPL", None)
-            tm(cfg, vs, [None, 1, 2, 4, 8] if cfg == 2 else [None])
+            tm(cfg, vs, [None, 1, 2, 4, 6, 8, 12, 16] if cfg == 2 else [None])
 
 
 def piv(cfg, variants, pairs):
