@@ -80,11 +80,11 @@ const TmVariant kTmVariants[] = {
     TM_VARIANT("tm_re_rv12_lx4_4x1_c32x32", 0, 0, 12, 4, 1, 4, 32, 32),
     // specialised instances for the BASELINE configurations
     TM_VARIANT("tm_sk_16x16_rv4_lx16_4x1_c16x16", 16, 16, 4, 16, 1, 4, 16, 16),
-    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c32x64", 128, 128, 12, 4, 1, 4, 32, 64),
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c16x64", 128, 128, 12, 4, 1, 4, 16, 64),
     // alternative 128x128 tilings (selected with NCC_FORCE_VARIANT for sweeps)
+    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c32x64", 128, 128, 12, 4, 1, 4, 32, 64),
     TM_VARIANT("tm_sk_128x128_rv12_lx4_8x1_c32x64", 128, 128, 12, 4, 1, 8, 32, 64),
     TM_VARIANT("tm_sk_128x128_rv12_lx4_4x2_c32x64", 128, 128, 12, 4, 2, 4, 32, 64),
-    TM_VARIANT("tm_sk_128x128_rv12_lx4_4x1_c16x64", 128, 128, 12, 4, 1, 4, 16, 64),
     TM_VARIANT("tm_sk_128x128_rv12_lx4_8x1_c16x64", 128, 128, 12, 4, 1, 8, 16, 64),
     TM_VARIANT("tm_sk_512x512_rv12_lx4_4x1_c32x64", 512, 512, 12, 4, 1, 4, 32, 64),
 };
@@ -477,16 +477,13 @@ ncc_status create_tm(ncc_plan pl) {
     const int64_t slots = (int64_t)(per_sm > 0 ? per_sm : 1) * nsm;
     const int64_t tiles_full = (int64_t)ceil_div(pl->U, v->bu) * ceil_div(pl->V, v->bv);
     const int nq = pl->n_slabs > 1 ? 1 : nCH * nCW;  // slab launches carry totals: no split
+    // Equal-size units are scheduled dynamically; the tail is about half a unit's duration at
+    // the per-SM concurrency, so aim for >= 6 "rounds" of resident units (measured on B200:
+    // cfg2 54 -> 57 TFLOP/s from S = 4 to S = 8), then stop splitting.
     int best_s = 1;
-    double best_e = 0.0;
     for (int S = 1; S <= nq && S <= 16; ++S) {
-      const int64_t units = tiles_full * S;
-      const double e = (double)units / (double)(((units + slots - 1) / slots) * slots);
-      if (e > best_e + 0.02) {
-        best_e = e;
-        best_s = S;
-      }
-      if (e >= 0.97) break;
+      best_s = S;
+      if (tiles_full * S >= 6 * slots) break;
     }
     pl->split = best_s;
     if (const char* fs = getenv("NCC_FORCE_SPLIT")) {
