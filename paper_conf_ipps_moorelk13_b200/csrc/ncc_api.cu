@@ -130,6 +130,8 @@ struct PivVariant {
   int RV, CW, NT, WPB, ALIAS, IPT;
   const void* k_tma;  // AOT function or JIT cudaKernel_t
   const void* k_ldg;
+  const void* k_ws = nullptr;  // persistent warp-specialised form (TMA only), if instantiated
+  int ws_ncw = 0, ws_npw = 0;
 };
 #define PIV_VARIANT_SK(NAME, TH, TW, MY, MX, RV, CW, NT, WPB, MINB, IPT)                                     \
   PivVariant {                                                                                              \
@@ -147,6 +149,10 @@ struct PivVariant {
 const PivVariant kPivVariants[] = {
     PIV_VARIANT_RE("piv_re_rv12_cw16_nt256", 12, 16, 256, 1),
     PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt416_w4", 32, 32, 16, 16, 12, 32, 416, 4, 2, 1),
+    PivVariant{"piv_ws_64x64_m32_rv12_c13p4", 64, 64, 32, 32, 12, 64, 416, 1, 1, 1,
+               reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, true, true, 1>),
+               reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, false, true, 1>),
+               reinterpret_cast<const void*>(&piv_ws_kernel<64, 64, 32, 32, 12, 64, 13, 4>), 13, 4},
     PIV_VARIANT_SK("piv_sk_64x64_m32_rv12_nt416_w1", 64, 64, 32, 32, 12, 64, 416, 1, 2, 1),
     // alternatives with warp counts that are multiples of 4 (even SMSP load; NCC_FORCE_VARIANT)
     PIV_VARIANT_SK("piv_sk_64x64_m32_rv12_nt512_w1", 64, 64, 32, 32, 12, 64, 512, 1, 2, 1),
@@ -279,6 +285,7 @@ struct ncc_plan_s {
   unsigned long long* keys;
   // PIV
   int Ky, Kx, OY, OX, sub_batch, piv_bp, piv_smem, map_w, map_h;
+  int ws_smem, ws_grid;  // persistent warp-specialised PIV kernel (0: not used)
   const PivVariant* pivv;
   // shared scratch (window sums)
   double *RS1, *RS2, *S1, *S2;
@@ -623,6 +630,17 @@ ncc_status create_piv(ncc_plan pl) {
   if (win_fl * 4 * v->WPB > maxsm) return NCC_ERR_UNSUPPORTED;
   NCC_CUDA(cudaFuncSetAttribute(v->k_tma, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
   NCC_CUDA(cudaFuncSetAttribute(v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
+  if (v->k_ws && !getenv("NCC_NO_WS")) {  // persistent warp-specialised form: 2 stages + score tile
+    PivShape<12, 64> ps(h, w, my, mx, pl->piv_bp, false);
+    const int64_t ws_bytes = (2 * (int64_t)(ps.tp_fl + ps.b_fl) + ps.s_fl) * 4;
+    int nsm = 0;
+    NCC_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, pl->device));
+    if (ws_bytes <= maxsm && v->CW == 64 && v->RV == 12) {
+      NCC_CUDA(cudaFuncSetAttribute(v->k_ws, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ws_bytes));
+      pl->ws_smem = (int)ws_bytes;
+      pl->ws_grid = nsm;
+    }
+  }
   const int rows_smem = (int)((kBoxRowsSEG + w + 1) * 2 * sizeof(double));
   if (rows_smem > maxsm) return NCC_ERR_UNSUPPORTED;
   NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT>,
@@ -839,8 +857,15 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
     mark(pl, s, 3 * sb + 1);
     a.pair0 = p0;
     dim3 grid(groups, 1, np);
-    void* args[2] = {&a, &mB};
-    NCC_CUDA(cudaLaunchKernel(use_tma ? v->k_tma : v->k_ldg, grid, dim3(v->NT), args, (size_t)pl->piv_smem, s));
+    if (use_tma && pl->ws_smem) {
+      int total = (int)((int64_t)np * pl->Ky * pl->Kx);
+      void* wargs[3] = {&a, &mB, &total};
+      const int g = total < pl->ws_grid ? total : pl->ws_grid;
+      NCC_CUDA(cudaLaunchKernel(v->k_ws, dim3(g), dim3((v->ws_ncw + v->ws_npw) * 32), wargs, (size_t)pl->ws_smem, s));
+    } else {
+      void* args[2] = {&a, &mB};
+      NCC_CUDA(cudaLaunchKernel(use_tma ? v->k_tma : v->k_ldg, grid, dim3(v->NT), args, (size_t)pl->piv_smem, s));
+    }
     mark(pl, s, 3 * sb + 2);
     mark(pl, s, 3 * sb + 3);
   }

@@ -154,6 +154,28 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
+// Bounded wait for the warp-specialised pipelines: a protocol bug traps (launch error)
+// instead of hanging the device.
+__device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  for (long long it = 0; it < (1ll << 30); ++it) {
+    asm volatile(
+        "{\n\t.reg .pred P;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, P;\n}"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    if (done) return;
+  }
+  __trap();
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
 // 2D / 3D tiled TMA loads global -> shared, completion on an mbarrier (out-of-bounds = 0).
 __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, int x, int y, uint64_t* bar) {
   asm volatile(
@@ -1094,6 +1116,247 @@ __global__ void __launch_bounds__(NT, MINB)
     o.score = a.ssd ? -key_score(bk) : key_score(bk);
     o.flags = flags;
     a.vec[(int64_t)pr * nwin + lin0 + wi] = o;
+  }
+}
+
+
+// ================================================================== PIV, persistent + warp-specialised
+// One CTA per SM loops over the windows of the launch.  NPW producer warps prepare window k+1
+// (TMA of the search region, mask statistics, template pairs) and finish window k-1 (argmax,
+// sub-pixel, vector store) while NCW consumer warps correlate window k -- the per-window
+// prologue / epilogue that left the FMA pipe idle in piv_ncc_kernel is overlapped.
+// Pipelines (mbarriers, parity = use index & 1):
+//   full[s]  producer -> consumers: stage s (template pairs, B region, stats) ready
+//   empty[s] consumers -> producer: stage s no longer read
+//   scfull   consumers -> producer: score tile of window k written
+//   scempty  producer -> consumers: score tile free again
+template <int TH, int TW, int MY, int MX, int RV, int CW, int NCW, int NPW>
+__global__ void __launch_bounds__((NCW + NPW) * 32, 1)
+    piv_ws_kernel(const PivArgs a, const __grid_constant__ CUtensorMap mapB, int nwin_total) {
+  constexpr int NCT = NCW * 32, NPT = NPW * 32;
+  constexpr int BPc = piv_sk_pitch(TW, MX, RV, CW);
+  const PivShape<RV, CW> sh(TH, TW, MY, MX, BPc, false);
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  float* smem = reinterpret_cast<float*>(smem_raw);
+  __shared__ __align__(8) uint64_t full_b[2], empty_b[2], scfull_b, scempty_b;
+  __shared__ double st_mean[2], st_sumsq[2], st_energy[2], st_csum[2];
+  __shared__ int st_flat[2];
+  __shared__ double pred[NPW * 4];
+  __shared__ unsigned long long pkey[NPW];
+  auto TPs = [&](int s) { return reinterpret_cast<u64*>(smem + s * (sh.tp_fl + sh.b_fl)); };
+  auto Bs = [&](int s) { return smem + s * (sh.tp_fl + sh.b_fl) + sh.tp_fl; };
+  float* Sc = smem + 2 * (sh.tp_fl + sh.b_fl);
+
+  const int tid = threadIdx.x;
+  const int nwin = a.Ky * a.Kx;
+  if (tid == 0) {
+    tma_prefetch_desc(&mapB);
+    mbar_init(&full_b[0], 2);
+    mbar_init(&full_b[1], 2);
+    mbar_init(&empty_b[0], NCT);
+    mbar_init(&empty_b[1], NCT);
+    mbar_init(&scfull_b, NCT);
+    mbar_init(&scempty_b, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  const int nlocal = (nwin_total - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+  auto win_of = [&](int k, int& lz, int& lin) {
+    const int wdx = (int)blockIdx.x + k * (int)gridDim.x;
+    lz = wdx / nwin;
+    lin = wdx % nwin;
+  };
+
+  if (tid >= NCT) {
+    // =============================== producers
+    const int pt = tid - NCT, lane = tid & 31, pw = pt >> 5;
+    constexpr int PERT = (TH * TW + NPT - 1) / NPT;
+    auto reduce2 = [&](double& x0, double& x1) {  // deterministic sum over the producer threads
+      x0 = warp_sum_d(x0);
+      x1 = warp_sum_d(x1);
+      named_bar_sync(1, NPT);
+      if (lane == 0) { pred[pw * 2] = x0; pred[pw * 2 + 1] = x1; }
+      named_bar_sync(1, NPT);
+      x0 = 0.0;
+      x1 = 0.0;
+      for (int q = 0; q < NPW; ++q) { x0 += pred[q * 2]; x1 += pred[q * 2 + 1]; }
+    };
+    auto epilogue = [&](int k) {
+      int lz, lin;
+      win_of(k, lz, lin);
+      const int s = k & 1;
+      mbar_wait_bounded(&scfull_b, (uint32_t)(k & 1));
+      const int tile = sh.OY * sh.OX;
+      unsigned long long best = 0ull;
+      const int pr = a.pair0 + lz;
+      for (int e = pt; e < tile; e += NPT) {
+        const int row = e / sh.OX, col = e % sh.OX;
+        const float sv = Sc[row * sh.OXP + col];
+        if (a.scores) a.scores[((int64_t)pr * nwin + lin) * tile + e] = sv;
+        const unsigned long long key = make_key(a.ssd ? -sv : sv, (uint32_t)e);
+        best = key > best ? key : best;
+      }
+      best = warp_max_key(best);
+      if (lane == 0) pkey[pw] = best;
+      named_bar_sync(1, NPT);
+      if (pt == 0) {
+        unsigned long long bk = 0ull;
+        for (int q = 0; q < NPW; ++q) bk = pkey[q] > bk ? pkey[q] : bk;
+        const uint32_t kk = key_index(bk);
+        const int row = (int)(kk / sh.OX), col = (int)(kk % sh.OX);
+        const int iy = row - sh.my, ix = col - sh.mx;
+        uint32_t flags = (st_flat[s] && !a.ssd) ? (kFlatTemplate | kInvalid) : 0u;
+        double ddy = 0.0, ddx = 0.0;
+        bool par = false;
+        if (row == 0 || row == sh.OY - 1) {
+          flags |= kEdgeY;
+        } else {
+          const double cm = Sc[(row - 1) * sh.OXP + col], c0 = Sc[row * sh.OXP + col],
+                       cp = Sc[(row + 1) * sh.OXP + col];
+          ddy = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
+          if (par) flags |= kParabolaY;
+        }
+        par = false;
+        if (col == 0 || col == sh.OX - 1) {
+          flags |= kEdgeX;
+        } else {
+          const double cm = Sc[row * sh.OXP + col - 1], c0 = Sc[row * sh.OXP + col], cp = Sc[row * sh.OXP + col + 1];
+          ddx = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
+          if (par) flags |= kParabolaX;
+        }
+        VecOut o;
+        o.iy = iy;
+        o.ix = ix;
+        o.dy = (float)(iy + ddy);
+        o.dx = (float)(ix + ddx);
+        o.score = a.ssd ? -key_score(bk) : key_score(bk);
+        o.flags = flags;
+        a.vec[(int64_t)pr * nwin + lin] = o;
+        mbar_arrive(&scempty_b);  // the score tile may be overwritten
+      }
+      named_bar_sync(1, NPT);  // pkey / stats reuse
+    };
+    for (int k = 0; k < nlocal; ++k) {
+      const int s = k & 1;
+      int lz, lin;
+      win_of(k, lz, lin);
+      const int pr = a.pair0 + lz;
+      const int y = sh.my + (lin / a.Kx) * a.sy, x = sh.mx + (lin % a.Kx) * a.sx;
+      if (k >= 2) mbar_wait_bounded(&empty_b[s], (uint32_t)(((k >> 1) - 1) & 1));
+      if (pt == 0) {
+        mbar_expect_tx(&full_b[s], (uint32_t)(sh.BR * sh.BP * 4));
+        tma_load_3d(Bs(s), &mapB, x - sh.mx, y - sh.my, pr, &full_b[s]);
+      }
+      // mask statistics and template pairs (as piv_ncc_kernel)
+      const float* Af = a.A + (int64_t)pr * a.frame_stride;
+      float mv[PERT];
+#pragma unroll
+      for (int q = 0; q < PERT; ++q) {
+        const int e = pt + q * NPT;
+        mv[q] = e < TH * TW ? __ldg(Af + (int64_t)(y + e / TW) * a.pitch + x + e % TW) : 0.0f;
+      }
+      double s1 = 0.0, s2 = 0.0;
+#pragma unroll
+      for (int q = 0; q < PERT; ++q) { s1 += (double)mv[q]; s2 += (double)mv[q] * (double)mv[q]; }
+      reduce2(s1, s2);
+      const double n = (double)TH * (double)TW;
+      const double mean = s1 / n;
+      double e2 = 0.0, cs = 0.0;
+      u64* tpw = TPs(s);
+#pragma unroll
+      for (int q = 0; q < PERT; ++q) {
+        const int e = pt + q * NPT;
+        if (e < TH * TW) {
+          const int i = e / TW, j = e % TW;
+          const double d = (double)mv[q] - mean;
+          const float ac = (float)d;
+          e2 += d * d;
+          cs += (double)ac;
+          float* tp = reinterpret_cast<float*>(tpw + i * sh.TPP + (j / CW) * sh.PB);
+          const int l = j % CW;
+          tp[2 * l + 1] = ac;
+          tp[2 * (l + 1)] = ac;
+          if (l == 0) tp[0] = 0.0f;
+          if (l == CW - 1) tp[2 * CW + 1] = 0.0f;
+        }
+      }
+      reduce2(e2, cs);
+      if (pt == 0) {
+        st_mean[s] = mean;
+        st_sumsq[s] = s2;
+        st_energy[s] = e2;
+        st_csum[s] = cs;
+        st_flat[s] = (e2 <= kFlatRel * s2) ? 1 : 0;
+      }
+      named_bar_sync(1, NPT);  // template pairs + stats of all producers written
+      if (pt == 0) mbar_arrive(&full_b[s]);
+      if (k >= 1) epilogue(k - 1);
+    }
+    if (nlocal >= 1) epilogue(nlocal - 1);
+  } else {
+    // =============================== consumers
+    const int ct = tid;
+    const bool has = ct < sh.items;
+    const int row = has ? ct / sh.NG : 0, g = has ? ct % sh.NG : 0;
+    const double inv_n = 1.0 / ((double)TH * (double)TW);
+    for (int k = 0; k < nlocal; ++k) {
+      const int s = k & 1;
+      int lz, lin;
+      win_of(k, lz, lin);
+      const int y = sh.my + (lin / a.Kx) * a.sy, x = sh.mx + (lin % a.Kx) * a.sx;
+      mbar_wait_bounded(&full_b[s], (uint32_t)((k >> 1) & 1));
+      float out[RV];
+      if (has) {
+        u64 tot2[RV / 2];
+#pragma unroll
+        for (int q = 0; q < RV / 2; ++q) tot2[q] = 0ull;
+        const float* brow = Bs(s) + row * sh.BP + g * RV;
+        const u64* tpw = TPs(s);
+#pragma unroll 1
+        for (int i = 0; i < TH; ++i) {
+#pragma unroll
+          for (int jc = 0; jc < (TW + CW - 1) / CW; ++jc) {
+            u64 part2[RV / 2];
+#pragma unroll
+            for (int q = 0; q < RV / 2; ++q) part2[q] = 0ull;
+            row_dot_pairs<RV, CW>(brow + i * sh.BP + jc * CW, tpw + i * sh.TPP + jc * sh.PB, part2);
+#pragma unroll
+            for (int q = 0; q < RV / 2; ++q) add2(tot2[q], part2[q]);
+          }
+        }
+        const double csum = st_csum[s], energy = st_energy[s], tmean = st_mean[s], tsq = st_sumsq[s];
+        const bool flat = st_flat[s] != 0;
+        const double* S1f = a.S1 + (int64_t)lz * a.map_frame_stride;
+        const double* S2f = a.S2 + (int64_t)lz * a.map_frame_stride;
+        const int64_t mrow = (int64_t)(y - sh.my + row) * a.map_pitch + (x - sh.mx);
+#pragma unroll
+        for (int q = 0; q < RV / 2; ++q) {
+          const float lo = __uint_as_float((uint32_t)(tot2[q] & 0xFFFFFFFFull));
+          const float hi = __uint_as_float((uint32_t)(tot2[q] >> 32));
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int c = 2 * q + 1 - e;
+            const int col = g * RV + c;
+            float v = 0.0f;
+            if (col < sh.OX) {
+              const double s1 = __ldg(S1f + mrow + col), s2 = __ldg(S2f + mrow + col);
+              const float num = e == 0 ? lo : hi;
+              v = a.ssd ? (float)(tsq - 2.0 * ((double)num + tmean * s1) + s2)
+                        : ncc_normalize_fast(num, s1, s2, inv_n, csum, energy, flat);
+            }
+            out[c] = v;
+          }
+        }
+      }
+      mbar_arrive(&empty_b[s]);  // done reading stage s (pairs, region, stats)
+      if (k >= 1) mbar_wait_bounded(&scempty_b, (uint32_t)((k - 1) & 1));
+      if (has) {
+        float* sc = Sc + row * sh.OXP + g * RV;
+#pragma unroll
+        for (int c = 0; c < RV; ++c) sc[c] = out[c];
+      }
+      mbar_arrive(&scfull_b);
+    }
   }
 }
 
