@@ -237,7 +237,7 @@ PivJitChoice piv_jit_choice(int h, int w, int my, int mx) {
   if (items > 1024) return c;  // one item per thread (score tile aliased on the template pairs)
   const int64_t kTwoPerSm = 113 * 1024, kOnePerSm = 227 * 1024;
   double best = -1.0;
-  for (int k = 1; k <= 8; ++k) {
+  for (int k = 1; k <= 4; ++k) {  // more windows per CTA blow up the per-window register arrays
     const int nt = ((k * items + 31) / 32) * 32;
     const int64_t smem = (int64_t)k * c.win_fl * 4;
     if (nt > 1024 || smem > kOnePerSm) break;
