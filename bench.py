@@ -218,7 +218,8 @@ def main():
         r = run_reference(args, cfg)
         line = {"metric": r["metric"], "value": r["value"], "unit": r["unit"], "n_gpus": args.gpus,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": r["ms_per_step"],
-                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+                "higher_is_better": True, "scaling": "strong" if cfg == 4 else "weak", "vs_baseline": None,
+                "dtype": "f64",
                 "data": "synthetic", "impl": "reference",
                 "config": {"workload": f"cfg{cfg}", **{k: v for k, v in synth.CONFIGS[cfg].items()}},
                 "cpu_baseline": {"value": r["value"], "unit": r["unit"], "cores": r["cores"], "kind": "oracle",
