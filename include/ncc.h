@@ -97,6 +97,14 @@ typedef struct {
                          /*     PIV: must be 0 (shard PIV by passing each rank its pairs) */
     int32_t shard_count; /* >= 1                                                            */
     uint32_t flags;  /* NCC_F_*                                                              */
+    /* Multi-template / ROI matching (the paper's TM runtime operation: several templates per
+     * frame, each searched within its region of interest -- Tab 5.1 caption P:190-191,
+     * 5.1.3.4 P:91).  n_templates = 0 or 1 with roi_h = roi_w = 0: plain full/band search
+     * (ncc_match).  n_templates >= 1 and roi_h, roi_w >= 1: ROI mode (ncc_match_rois), all
+     * templates h x w, every (frame, template) searched over the offsets
+     * [u0, u0+roi_h) x [v0, v0+roi_w) clipped to the valid range; shard_count must be 1. */
+    int32_t n_templates;
+    int32_t roi_h, roi_w;
 } ncc_problem;
 
 /* TM result per frame: argmax over the (band of) valid offsets, tie -> smallest u*V+v.
@@ -164,6 +172,14 @@ ncc_status ncc_plan_create(const ncc_problem* p, int device, ncc_plan* out);
  *           ignored (may be NULL).  d_peaks: [batch] ncc_peak (device). */
 ncc_status ncc_match(ncc_plan plan, const float* d_images, const float* d_tmpl,
                      int64_t tmpl_pitch, float* d_scores, ncc_peak* d_peaks, void* stream);
+
+/* ROI mode (n_templates, roi_h, roi_w set): d_tmpls = n_templates templates, template t at
+ * d_tmpls + t*tmpl_h*tmpl_pitch; d_rois = int32 [batch][n_templates][2] offset-space origins
+ * (u0, v0) of the ROIs, each in [0, U) x [0, V) (device); d_scores (if NCC_F_WRITE_SURFACE)
+ * [batch][n_templates][roi_h][roi_w] fp32; d_peaks [batch][n_templates], global (u, v),
+ * argmax (NCC) / argmin (SSD) inside the clipped ROI, tie -> smallest u*V+v. */
+ncc_status ncc_match_rois(ncc_plan plan, const float* d_images, const float* d_tmpls, int64_t tmpl_pitch,
+                          const int32_t* d_rois, float* d_scores, ncc_peak* d_peaks, void* stream);
 
 /* PIV on `batch` frame pairs: d_frames_a / d_frames_b (device), d_vectors [batch][Ky][Kx]. */
 ncc_status piv_correlate(ncc_plan plan, const float* d_frames_a, const float* d_frames_b,

@@ -24,7 +24,7 @@ NCC_SUBPIX_GAUSS3, NCC_SUBPIX_PARABOLA3, NCC_SUBPIX_NONE = 0, 1, 2
 NCC_F_WRITE_SURFACE, NCC_F_GENERIC_KERNEL, NCC_F_NO_JIT, NCC_F_TIMING = 1, 2, 4, 8
 FLAG_FLAT_TEMPLATE, FLAG_EDGE_Y, FLAG_EDGE_X, FLAG_PARABOLA_Y, FLAG_PARABOLA_X, FLAG_INVALID = 1, 2, 4, 8, 16, 32
 
-EXPORTS = ["ncc_plan_create", "ncc_match", "piv_correlate", "piv_correlate_ex", "ncc_match_host",
+EXPORTS = ["ncc_plan_create", "ncc_match", "ncc_match_rois", "piv_correlate", "piv_correlate_ex", "ncc_match_host",
            "piv_correlate_host", "ncc_plan_destroy", "ncc_status_string", "ncc_last_cuda_error",
            "ncc_plan_query", "ncc_plan_timing", "ncc_build_arch", "ncc_specialize"]
 
@@ -36,7 +36,8 @@ class NccProblem(ctypes.Structure):
                 ("search_y", ctypes.c_int32), ("search_x", ctypes.c_int32),
                 ("step_y", ctypes.c_int32), ("step_x", ctypes.c_int32),
                 ("batch", ctypes.c_int32), ("shard_rank", ctypes.c_int32), ("shard_count", ctypes.c_int32),
-                ("flags", ctypes.c_uint32)]
+                ("flags", ctypes.c_uint32), ("n_templates", ctypes.c_int32), ("roi_h", ctypes.c_int32),
+                ("roi_w", ctypes.c_int32)]
 
 
 class NccPeak(ctypes.Structure):
@@ -97,6 +98,7 @@ def lib():
         P, V = ctypes.c_void_p, ctypes.c_void_p
         L.ncc_plan_create.argtypes = [ctypes.POINTER(NccProblem), ctypes.c_int, ctypes.POINTER(P)]
         L.ncc_match.argtypes = [P, P, P, ctypes.c_int64, P, P, V]
+        L.ncc_match_rois.argtypes = [P, P, P, ctypes.c_int64, P, P, P, V]
         L.piv_correlate.argtypes = [P, P, P, P, V]
         L.piv_correlate_ex.argtypes = [P, P, P, P, P, V]
         L.ncc_match_host.argtypes = [P, P, P, ctypes.c_int64, P, P, V]
@@ -141,11 +143,12 @@ def _stream(stream, device):
 
 def make_problem(mode=NCC_MODE_MATCH, image_h=0, image_w=0, image_pitch=None, tmpl_h=0, tmpl_w=0, search_y=0,
                  search_x=0, step_y=0, step_x=0, batch=1, shard_rank=0, shard_count=1, flags=0,
-                 score=NCC_SCORE_NCC, subpix=NCC_SUBPIX_GAUSS3) -> NccProblem:
+                 score=NCC_SCORE_NCC, subpix=NCC_SUBPIX_GAUSS3, n_templates=0, roi_h=0, roi_w=0) -> NccProblem:
     return NccProblem(mode=mode, score=score, subpix=subpix, image_h=image_h, image_w=image_w,
                       image_pitch=image_w if image_pitch is None else image_pitch, tmpl_h=tmpl_h, tmpl_w=tmpl_w,
                       search_y=search_y, search_x=search_x, step_y=step_y, step_x=step_x, batch=batch,
-                      shard_rank=shard_rank, shard_count=shard_count, flags=flags)
+                      shard_rank=shard_rank, shard_count=shard_count, flags=flags, n_templates=n_templates,
+                      roi_h=roi_h, roi_w=roi_w)
 
 
 # ---------------------------------------------------------------- C-ABI names
@@ -174,6 +177,11 @@ def ncc_plan_timing(plan) -> NccTiming:
 def ncc_match(plan, images, tmpl, tmpl_pitch, scores, peaks, stream) -> None:
     _check(lib().ncc_match(plan, _ptr(images), _ptr(tmpl), int(tmpl_pitch), _ptr(scores), _ptr(peaks), stream),
            "ncc_match")
+
+
+def ncc_match_rois(plan, images, tmpls, tmpl_pitch, rois, scores, peaks, stream) -> None:
+    _check(lib().ncc_match_rois(plan, _ptr(images), _ptr(tmpls), int(tmpl_pitch), _ptr(rois), _ptr(scores),
+                                _ptr(peaks), stream), "ncc_match_rois")
 
 
 def piv_correlate(plan, frames_a, frames_b, vectors, stream) -> None:

@@ -60,12 +60,14 @@ class MatchPlan(_Plan):
     """Template matching: corr2 at every valid offset of each frame (Listing 5.1)."""
 
     def __init__(self, H, W, h, w, batch=1, device=0, shard_rank=0, shard_count=1, write_surface=False,
-                 generic=False, timing=False, image_pitch=None, score=N.NCC_SCORE_NCC):
+                 generic=False, timing=False, image_pitch=None, score=N.NCC_SCORE_NCC, n_templates=0, roi=None):
+        """roi=(roi_h, roi_w) with n_templates >= 1 selects ROI mode (match_rois)."""
         flags = (N.NCC_F_WRITE_SURFACE if write_surface else 0) | (N.NCC_F_GENERIC_KERNEL if generic else 0) | \
                 (N.NCC_F_TIMING if timing else 0)
+        rh, rw = roi if roi is not None else (0, 0)
         super().__init__(N.make_problem(N.NCC_MODE_MATCH, H, W, image_pitch, h, w, batch=batch,
                                         shard_rank=shard_rank, shard_count=shard_count, flags=flags,
-                                        score=score), device)
+                                        score=score, n_templates=n_templates, roi_h=rh, roi_w=rw), device)
         self.write_surface = write_surface
 
     @property
@@ -81,6 +83,19 @@ class MatchPlan(_Plan):
         if self.write_surface and scores is None:
             scores = torch.empty((p.batch, self.band_rows, self.info.V), dtype=torch.float32, device=dev)
         N.ncc_match(self.handle, images, tmpl, tmpl.stride(0), scores, peaks, self._stream(stream))
+        return peaks, scores
+
+    def match_rois(self, images: torch.Tensor, tmpls: torch.Tensor, rois: torch.Tensor, stream=None, peaks=None,
+                   scores=None):
+        """images (batch, H, pitch); tmpls (T, h, w); rois int32 (batch, T, 2) origins (u0, v0)."""
+        p = self.problem
+        dev = torch.device("cuda", self.device)
+        T = max(1, p.n_templates)
+        if peaks is None:
+            peaks = torch.empty((p.batch, T, 4), dtype=torch.int32, device=dev)
+        if self.write_surface and scores is None:
+            scores = torch.empty((p.batch, T, p.roi_h, p.roi_w), dtype=torch.float32, device=dev)
+        N.ncc_match_rois(self.handle, images, tmpls, tmpls.stride(1), rois, scores, peaks, self._stream(stream))
         return peaks, scores
 
     def match_host(self, h_images: torch.Tensor, h_tmpl: torch.Tensor, h_peaks: torch.Tensor, h_scores=None,

@@ -161,7 +161,7 @@ const PivVariant kPivVariants[] = {
 };
 
 constexpr int kBoxRowsNT = 256, kBoxRowsSEG = 2048;  // max segment; actual = min(V, SEG)
-constexpr int kBoxColsNT = 128, kBoxColsRB = 32;
+constexpr int kBoxColsNW = 8, kBoxColsL = 16;  // 32 columns x 8 warps x 16 rows per CTA
 
 int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
@@ -266,6 +266,8 @@ struct ncc_plan_s {
   // TM
   int U, V, u_begin, u_end, Ub, Hs, HP, WP;
   int tiles_u, tiles_v, split;
+  int n_tmpl;     // templates per frame (ROI mode) or 1
+  bool roi_mode;
   bool tma_ok;
   int use_ct, slab_rows, n_slabs;  // constant-template slabs (rows per slab, slab count)
   float* carry;
@@ -349,8 +351,13 @@ ncc_status validate(const ncc_problem& p) {
   if (p.tmpl_h > p.image_h || p.tmpl_w > p.image_w) return NCC_ERR_INVALID_ARGUMENT;
   if (p.batch < 1 || p.shard_count < 1 || p.shard_rank < 0 || p.shard_rank >= p.shard_count)
     return NCC_ERR_INVALID_ARGUMENT;
+  if (p.n_templates < 0 || p.roi_h < 0 || p.roi_w < 0) return NCC_ERR_INVALID_ARGUMENT;
   if (p.mode == NCC_MODE_MATCH) {
     if (p.search_y != 0 || p.search_x != 0) return NCC_ERR_INVALID_ARGUMENT;
+    if (p.roi_h > 0 || p.roi_w > 0 || p.n_templates > 1) {  // ROI mode
+      if (p.roi_h < 1 || p.roi_w < 1 || p.n_templates < 1 || p.shard_count != 1) return NCC_ERR_INVALID_ARGUMENT;
+      if (p.roi_h > p.image_h - p.tmpl_h + 1 || p.roi_w > p.image_w - p.tmpl_w + 1) return NCC_ERR_INVALID_ARGUMENT;
+    }
     const int64_t U = p.image_h - p.tmpl_h + 1, V = p.image_w - p.tmpl_w + 1;
     if (U * V >= (int64_t)0xFFFFFFF0ll) return NCC_ERR_INVALID_ARGUMENT;  // 32-bit key index
     if (p.shard_count > U) return NCC_ERR_INVALID_ARGUMENT;               // every band has rows
@@ -360,6 +367,7 @@ ncc_status validate(const ncc_problem& p) {
       return NCC_ERR_INVALID_ARGUMENT;
     if (p.shard_count != 1 || p.shard_rank != 0) return NCC_ERR_INVALID_ARGUMENT;
     if (p.subpix < 0 || p.subpix > 2) return NCC_ERR_INVALID_ARGUMENT;
+    if (p.n_templates > 1 || p.roi_h > 0 || p.roi_w > 0) return NCC_ERR_INVALID_ARGUMENT;
   }
   return NCC_OK;
 }
@@ -397,6 +405,8 @@ ncc_status create_tm(ncc_plan pl) {
   if (pl->u_begin >= pl->u_end) return NCC_ERR_INVALID_ARGUMENT;
   pl->Ub = pl->u_end - pl->u_begin;
   pl->Hs = pl->Ub + h - 1;
+  pl->roi_mode = p.roi_h > 0;
+  pl->n_tmpl = p.n_templates > 1 ? p.n_templates : 1;
 
   // variant selection (a8): AOT specialised instance > run-time specialised (NVRTC) > generic RE
   const TmVariant* v = &kTmVariants[0];
@@ -415,7 +425,11 @@ ncc_status create_tm(ncc_plan pl) {
         aot = c.TH != 0;
       }
   if (!aot && jit_allowed(p.flags)) {
-    const TmJitChoice jc = tm_jit_choice(h, w);
+    TmJitChoice jc = tm_jit_choice(h, w);
+    if (p.n_templates > 1) {  // several templates share the 64 KB constant bank or use shared memory
+      const int64_t hp = ((h + jc.CH - 1) / jc.CH) * jc.CH, wp = ((w + jc.CW - 1) / jc.CW) * jc.CW;
+      jc.ct = jc.ct && (int64_t)p.n_templates * hp * wp <= kConstTplFloats;
+    }
     const std::vector<std::string> names = {tm_name(jc.RV, jc.LX, jc.WX, jc.WY, jc.CH, jc.CW, h, w, false, jc.ct),
                                             tm_name(jc.RV, jc.LX, jc.WX, jc.WY, jc.CH, jc.CW, h, w, true, jc.ct),
                                             "&nccb::c_tpl"};
@@ -468,21 +482,28 @@ ncc_status create_tm(ncc_plan pl) {
 
   // constant-bank template: slabs of whole row-chunks that fit 64 KB (NCC_NO_CONST_TPL=1 disables)
   pl->slab_rows = (kConstTplFloats / pl->WP) / v->CH * v->CH;
-  pl->use_ct = pl->slab_rows >= v->CH && (pl->jit_lib ? true : !getenv("NCC_NO_CONST_TPL"));
+  pl->use_ct = pl->jit_lib ? (pl->jit_ct != 0) : (pl->slab_rows >= v->CH && !getenv("NCC_NO_CONST_TPL"));
   if (pl->slab_rows > pl->HP) pl->slab_rows = pl->HP;
   pl->n_slabs = pl->use_ct ? ceil_div(pl->HP, pl->slab_rows) : 1;
+  if (pl->n_tmpl > 1) {  // several templates: all of them resident in the constant bank, or shared memory
+    const bool fits = (int64_t)pl->n_tmpl * pl->HP * pl->WP <= kConstTplFloats;
+    pl->use_ct = pl->use_ct && fits;
+    pl->slab_rows = pl->HP;
+    pl->n_slabs = 1;
+  }
 
   // tiles of this band; split-K factor S from the FULL problem's tile count (so every shard
   // of a problem uses the same S and the same per-offset accumulation order): the smallest
   // S <= chunks whose unit count fills whole "rounds" of resident CTAs to >= 97 %.
-  pl->tiles_u = ceil_div(pl->Ub, v->bu);
-  pl->tiles_v = ceil_div(pl->V, v->bv);
+  pl->tiles_u = ceil_div(pl->roi_mode ? p.roi_h : pl->Ub, v->bu);
+  pl->tiles_v = ceil_div(pl->roi_mode ? p.roi_w : pl->V, v->bv);
   {
     int per_sm = 0;
     const int ct = pl->use_ct ? 1 : 0;
     NCC_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, v->k[1][ct], v->nt, v->smem[1][ct]));
     const int64_t slots = (int64_t)(per_sm > 0 ? per_sm : 1) * nsm;
-    const int64_t tiles_full = (int64_t)ceil_div(pl->U, v->bu) * ceil_div(pl->V, v->bv);
+    const int64_t tiles_full = pl->roi_mode ? (int64_t)pl->tiles_u * pl->tiles_v * pl->n_tmpl
+                                            : (int64_t)ceil_div(pl->U, v->bu) * ceil_div(pl->V, v->bv);
     const int nq = pl->n_slabs > 1 ? 1 : nCH * nCW;  // slab launches carry totals: no split
     // Equal-size units are scheduled dynamically; the tail is about half a unit's duration at
     // the per-SM concurrency, so aim for >= 6 "rounds" of resident units (measured on B200:
@@ -503,10 +524,10 @@ ncc_status create_tm(ncc_plan pl) {
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_fork, cudaEventDisableTiming));
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_join, cudaEventDisableTiming));
   ncc_status st;
-  if ((st = dalloc(&pl->tplC, (size_t)pl->HP * pl->WP))) return st;
-  if ((st = dalloc(&pl->tst, 1))) return st;
-  if ((st = dalloc(&pl->keys, (size_t)p.batch))) return st;
-  const int64_t ntiles = (int64_t)pl->tiles_u * pl->tiles_v * p.batch;
+  if ((st = dalloc(&pl->tplC, (size_t)pl->n_tmpl * pl->HP * pl->WP))) return st;
+  if ((st = dalloc(&pl->tst, (size_t)pl->n_tmpl))) return st;
+  if ((st = dalloc(&pl->keys, (size_t)p.batch * pl->n_tmpl))) return st;
+  const int64_t ntiles = (int64_t)pl->tiles_u * pl->tiles_v * p.batch * pl->n_tmpl;
   if (pl->split > 1) {
     if ((st = dalloc(&pl->part, (size_t)ntiles * pl->split * v->rv_nt()))) return st;
     if ((st = dalloc(&pl->cnt, (size_t)ntiles))) return st;
@@ -521,7 +542,7 @@ ncc_status create_tm(ncc_plan pl) {
   if ((st = dalloc(&pl->S1, (size_t)p.batch * pl->s_frame_stride))) return st;
   if ((st = dalloc(&pl->S2, (size_t)p.batch * pl->s_frame_stride))) return st;
   {  // template chunks: 2D map over the zero-padded centred template
-    const uint64_t dims[2] = {(uint64_t)pl->WP, (uint64_t)pl->HP};
+    const uint64_t dims[2] = {(uint64_t)pl->WP, (uint64_t)pl->HP * pl->n_tmpl};
     const uint64_t strides[1] = {(uint64_t)pl->WP * 4};
     const uint32_t box[2] = {(uint32_t)v->CW, (uint32_t)v->CH};
     pl->tma_ok = encode_f32(&pl->map_tpl, pl->tplC, 2, dims, strides, box);
@@ -532,7 +553,8 @@ ncc_status create_tm(ncc_plan pl) {
   in.V = pl->V;
   in.u_begin = pl->u_begin;
   in.u_end = pl->u_end;
-  in.outputs_per_call = (int64_t)pl->Ub * pl->V * p.batch;
+  in.outputs_per_call = pl->roi_mode ? (int64_t)p.roi_h * p.roi_w * p.batch * pl->n_tmpl
+                                     : (int64_t)pl->Ub * pl->V * p.batch;
   in.flops_per_call = 2.0 * h * (double)w * (double)in.outputs_per_call;
   in.specialized = pl->jit_lib ? 2 : (v->TH != 0);
   in.variant_id = pl->jit_lib ? -1 : (int)(v - kTmVariants);
@@ -542,7 +564,7 @@ ncc_status create_tm(ncc_plan pl) {
   {
     const int ct = pl->use_ct ? 1 : 0;
     fill_kernel_info(pl, v->k[1][ct], v->nt, v->smem[1][ct], pl->tiles_u * pl->tiles_v * pl->split,
-                     p.batch, 1);
+                     p.batch * pl->n_tmpl, 1);
     in.split = pl->split;
     in.const_template = pl->use_ct;
     in.slabs = pl->n_slabs;
@@ -700,13 +722,13 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
   box_rows_kernel<kBoxRowsNT><<<g1, kBoxRowsNT, smem, s>>>(frames, p.image_pitch, (int64_t)p.image_h * p.image_pitch,
                                                            p.image_w, row0, w, V, seg, pl->RS1, pl->RS2,
                                                            pl->rs_frame_stride);
-  dim3 g2(ceil_div(V, kBoxColsNT), ceil_div(rows_out, kBoxColsRB), batch);
-  box_cols_kernel<kBoxColsNT, kBoxColsRB><<<g2, kBoxColsNT, 0, s>>>(pl->RS1, pl->RS2, pl->rs_frame_stride, V, h,
-                                                                    rows_out, pl->S1, pl->S2, pl->s_frame_stride);
+  dim3 g2(ceil_div(V, 32), ceil_div(rows_out, kBoxColsNW * kBoxColsL), batch);
+  box_cols_kernel<kBoxColsNW, kBoxColsL><<<g2, kBoxColsNW * 32, 0, s>>>(pl->RS1, pl->RS2, pl->rs_frame_stride, V, h,
+                                                                        rows_out, pl->S1, pl->S2, pl->s_frame_stride);
 }
 
 ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, int64_t tmpl_pitch, float* d_scores,
-                     ncc_peak* d_peaks, cudaStream_t s) {
+                     ncc_peak* d_peaks, cudaStream_t s, const int32_t* d_rois = nullptr) {
   const ncc_problem& p = pl->p;
   const TmVariant* v = pl->tmv;
   if (p.flags & NCC_F_TIMING) {
@@ -718,8 +740,8 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   mark(pl, s, 0);
   NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
   NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
-  tm_template_prep<<<1, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
-                                             pl->tst, pl->keys, p.batch);
+  tm_template_prep<<<pl->n_tmpl, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP,
+                                                       pl->WP, pl->tst, pl->keys, p.batch);
   mark(pl, pl->side, 1);
   NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
   launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
@@ -754,6 +776,13 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   a.cnt = pl->cnt;
   a.S = pl->split;
   a.ssd = p.score == NCC_SCORE_SSD;
+  a.n_tmpl = pl->n_tmpl;
+  a.roi = pl->roi_mode ? d_rois : nullptr;
+  a.roi_h = p.roi_h;
+  a.roi_w = p.roi_w;
+  a.tpl_stride = (int64_t)pl->HP * pl->WP;
+  a.tpl_rows = pl->HP;
+  a.map_u0 = pl->u_begin;
   // TMA needs a 16-B aligned base and a pitch that is a multiple of 16 B; else plain loads.
   CUtensorMap map_img;
   memset(&map_img, 0, sizeof(map_img));
@@ -764,7 +793,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     const uint32_t box[3] = {(uint32_t)v->ip, (uint32_t)v->ir, 1u};
     use_tma = encode_f32(&map_img, d_images, 3, dims, strides, box);
   }
-  dim3 grid(pl->tiles_u * pl->tiles_v * pl->split, p.batch);
+  dim3 grid(pl->tiles_u * pl->tiles_v * pl->split, p.batch * pl->n_tmpl);
   const int t = use_tma ? 1 : 0, ct = pl->use_ct ? 1 : 0;
   const int nCWl = pl->WP / v->CW;
   a.carry = pl->carry;
@@ -777,17 +806,16 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     a.c_row0 = r0;
     a.first = sl == 0;
     a.last = sl == pl->n_slabs - 1;
+    const size_t cbytes = (size_t)(pl->n_tmpl > 1 ? (int64_t)pl->n_tmpl * pl->HP : (r1 - r0)) * pl->WP * 4;
     if (ct && pl->jit_ctpl) {  // the plan's own constant slot (JIT library): stream order suffices
-      NCC_CUDA(cudaMemcpyAsync(pl->jit_ctpl, pl->tplC + (size_t)r0 * pl->WP, (size_t)(r1 - r0) * pl->WP * 4,
-                               cudaMemcpyDeviceToDevice, s));
+      NCC_CUDA(cudaMemcpyAsync(pl->jit_ctpl, pl->tplC + (size_t)r0 * pl->WP, cbytes, cudaMemcpyDeviceToDevice, s));
       NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
     } else if (ct) {  // template rows [r0, r1) into the constant bank (stream-ordered after the prep)
       ConstSlot& cs = g_const_slot[pl->device & 63];
       std::lock_guard<std::mutex> lk(cs.mu);
       if (!cs.done) NCC_CUDA(cudaEventCreateWithFlags(&cs.done, cudaEventDisableTiming));
       else NCC_CUDA(cudaStreamWaitEvent(s, cs.done, 0));
-      NCC_CUDA(cudaMemcpyToSymbolAsync(c_tpl, pl->tplC + (size_t)r0 * pl->WP, (size_t)(r1 - r0) * pl->WP * 4, 0,
-                                       cudaMemcpyDeviceToDevice, s));
+      NCC_CUDA(cudaMemcpyToSymbolAsync(c_tpl, pl->tplC + (size_t)r0 * pl->WP, cbytes, 0, cudaMemcpyDeviceToDevice, s));
       NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
       NCC_CUDA(cudaEventRecord(cs.done, s));
     } else {
@@ -795,8 +823,8 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     }
   }
   mark(pl, s, 3);
-  tm_finalize<<<ceil_div(p.batch, 128), 128, 0, s>>>(pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks),
-                                                     p.batch, p.score == NCC_SCORE_SSD);
+  tm_finalize<<<ceil_div((int64_t)p.batch * pl->n_tmpl, 128), 128, 0, s>>>(
+      pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks), p.batch, p.score == NCC_SCORE_SSD, pl->n_tmpl);
   mark(pl, s, 4);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch");
@@ -1035,11 +1063,21 @@ ncc_status ncc_plan_timing(ncc_plan pl, ncc_timing* out) {
 ncc_status ncc_match(ncc_plan pl, const float* d_images, const float* d_tmpl, int64_t tmpl_pitch, float* d_scores,
                      ncc_peak* d_peaks, void* stream) {
   if (!pl) return NCC_ERR_INVALID_ARGUMENT;
-  if (pl->p.mode != NCC_MODE_MATCH) return NCC_ERR_WRONG_MODE;
+  if (pl->p.mode != NCC_MODE_MATCH || pl->roi_mode) return NCC_ERR_WRONG_MODE;
   if (!d_images || !d_tmpl || !d_peaks || tmpl_pitch < pl->p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
   if ((pl->p.flags & NCC_F_WRITE_SURFACE) && !d_scores) return NCC_ERR_INVALID_ARGUMENT;
   DeviceGuard g(pl->device);
   return run_match(pl, d_images, d_tmpl, tmpl_pitch, d_scores, d_peaks, (cudaStream_t)stream);
+}
+
+ncc_status ncc_match_rois(ncc_plan pl, const float* d_images, const float* d_tmpls, int64_t tmpl_pitch,
+                          const int32_t* d_rois, float* d_scores, ncc_peak* d_peaks, void* stream) {
+  if (!pl) return NCC_ERR_INVALID_ARGUMENT;
+  if (pl->p.mode != NCC_MODE_MATCH || !pl->roi_mode) return NCC_ERR_WRONG_MODE;
+  if (!d_images || !d_tmpls || !d_rois || !d_peaks || tmpl_pitch < pl->p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
+  if ((pl->p.flags & NCC_F_WRITE_SURFACE) && !d_scores) return NCC_ERR_INVALID_ARGUMENT;
+  DeviceGuard g(pl->device);
+  return run_match(pl, d_images, d_tmpls, tmpl_pitch, d_scores, d_peaks, (cudaStream_t)stream, d_rois);
 }
 
 ncc_status piv_correlate_ex(ncc_plan pl, const float* d_a, const float* d_b, float* d_scores, piv_vector* d_vec,
@@ -1058,7 +1096,7 @@ ncc_status piv_correlate(ncc_plan pl, const float* d_a, const float* d_b, piv_ve
 ncc_status ncc_match_host(ncc_plan pl, const float* h_images, const float* h_tmpl, int64_t tmpl_pitch,
                           float* h_scores, ncc_peak* h_peaks, void* stream) {
   if (!pl) return NCC_ERR_INVALID_ARGUMENT;
-  if (pl->p.mode != NCC_MODE_MATCH) return NCC_ERR_WRONG_MODE;
+  if (pl->p.mode != NCC_MODE_MATCH || pl->roi_mode) return NCC_ERR_WRONG_MODE;
   const ncc_problem& p = pl->p;
   if (!h_images || !h_tmpl || !h_peaks || tmpl_pitch < p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
   DeviceGuard g(pl->device);

@@ -276,6 +276,14 @@ struct TmArgs {
   int q_begin, q_end, c_row0, first, last;
   float* carry;
   int ssd;                   // 0: NCC (argmax), 1: SSD = sum (T - W)^2 (argmin; Fig 5.10)
+  // multi-template / ROI mode (TM runtime operation: several templates per frame, each searched
+  // inside its region of interest; Tab 5.1, 5.1.3.4 P:91).  blockIdx.y = frame*n_tmpl + t.
+  int n_tmpl;                // >= 1
+  const int* roi;            // nullable: [batch][n_tmpl][2] offset-space ROI origins (u0, v0)
+  int roi_h, roi_w;          // ROI extent in offsets (ROI mode)
+  int64_t tpl_stride;        // floats between consecutive centred templates (tplC and c_tpl)
+  int tpl_rows;              // padded rows per template (TMA row offset of template t)
+  int map_u0;                // first offset row held in S1/S2 (band start; 0 in ROI mode)
 };
 
 // Template chunks in the constant bank: FFMA takes the template from uniform registers
@@ -357,15 +365,23 @@ __global__ void __launch_bounds__(WX* WY * 32)
   const int ly = lane / LX, lx = lane % LX;
   const int lu = wy * T::LY + ly;         // local output row
   const int lv = (wx * LX + lx) * RV;     // local output col (first of RV)
-  const int f = blockIdx.y;
+  const int ft = blockIdx.y;  // frame * n_tmpl + template
+  const int f = ft / a.n_tmpl, tpl = ft % a.n_tmpl;
   const int S = a.S;
   const int tile = blockIdx.x / S, split = blockIdx.x % S;
   const int ty = tile / a.tiles_v, tx = tile % a.tiles_v;
-  const int u0 = a.u_begin + ty * T::BU;
-  const int v0 = tx * T::BV;
+  int ru0 = a.u_begin, rv0 = 0, u_lim = a.u_end, v_lim = a.V;
+  if (a.roi) {
+    ru0 = a.roi[2 * ft];
+    rv0 = a.roi[2 * ft + 1];
+    u_lim = min(ru0 + a.roi_h, a.U);
+    v_lim = min(rv0 + a.roi_w, a.V);
+  }
+  const int u0 = ru0 + ty * T::BU;
+  const int v0 = rv0 + tx * T::BV;
   const int nq = a.q_end - a.q_begin;
   const int q0 = a.q_begin + (split * nq) / S, q1 = a.q_begin + ((split + 1) * nq) / S;
-  const int64_t tile_lin = (int64_t)f * a.tiles_u * a.tiles_v + tile;
+  const int64_t tile_lin = (int64_t)ft * a.tiles_u * a.tiles_v + tile;
 
   float total[RV];
   if (a.first) {
@@ -386,7 +402,8 @@ __global__ void __launch_bounds__(WX* WY * 32)
 #pragma unroll
       for (int c = 0; c < RV; ++c) part[c] = 0.0f;
       if constexpr (CT)
-        row_dot_c<RV, CW>(irow + i * T::IP, (ic * CH + i - a.c_row0) * tplP + jc * CW, part);
+        row_dot_c<RV, CW>(irow + i * T::IP, (int)(tpl * a.tpl_stride) + (ic * CH + i - a.c_row0) * tplP + jc * CW,
+                          part);
       else
         row_dot<RV, CW>(irow + i * T::IP, Ts + i * CW, part);
 #pragma unroll
@@ -401,7 +418,7 @@ __global__ void __launch_bounds__(WX* WY * 32)
     auto issue = [&](int q, int s) {  // one thread: chunk q -> stage s
       const int ic = q / nCW, jc = q % nCW;
       mbar_expect_tx(&full_bar[s], (uint32_t)((CT ? 0 : T::T_BYTES) + T::I_BYTES));
-      if constexpr (!CT) tma_load_2d(stage_t(s), &map_tpl, jc * CW, ic * CH, &full_bar[s]);
+      if constexpr (!CT) tma_load_2d(stage_t(s), &map_tpl, jc * CW, tpl * a.tpl_rows + ic * CH, &full_bar[s]);
       tma_load_3d(stage_i(s), &map_img, v0 + jc * CW, u0 + ic * CH, f, &full_bar[s]);
     };
     if (tid == 0) {
@@ -431,14 +448,14 @@ __global__ void __launch_bounds__(WX* WY * 32)
       const int ic = q / nCW, jc = q % nCW;
       __syncthreads();
       if constexpr (!CT) {
-        const float* tsrc = a.tplC + (int64_t)(ic * CH) * tplP + jc * CW;
+        const float* tsrc = a.tplC + tpl * a.tpl_stride + (int64_t)(ic * CH) * tplP + jc * CW;
         for (int k = tid; k < CH * CW; k += T::NT) Ts[k] = tsrc[(k / CW) * tplP + (k % CW)];
       }
       const int gr0 = u0 + ic * CH, gc0 = v0 + jc * CW;
       for (int k = tid; k < T::IR * T::IP; k += T::NT) {
         const int r = k / T::IP, c = k % T::IP;
         const int gr = gr0 + r, gc = gc0 + c;
-        Is[k] = (gr < a.H && gc < a.W) ? __ldg(img + (int64_t)gr * a.pitch + gc) : 0.0f;
+        Is[k] = (gr >= 0 && gc >= 0 && gr < a.H && gc < a.W) ? __ldg(img + (int64_t)gr * a.pitch + gc) : 0.0f;
       }
       __syncthreads();
       compute_chunk(q, Ts, Is);
@@ -475,18 +492,20 @@ __global__ void __launch_bounds__(WX* WY * 32)
   }
 
   // ---- fused epilogue: normalise, clamp, optional surface, argmax key
-  const TemplateStats ts = *a.tst;
+  const TemplateStats ts = a.tst[tpl];
   const double n = (double)h * (double)w;
   const int u = u0 + lu;
   unsigned long long best = 0ull;
-  if (u < a.u_end) {
-    const int64_t rowoff = (int64_t)f * a.stat_frame_stride + (int64_t)(u - a.u_begin) * a.V;
-    float* srow = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + (int64_t)(u - a.u_begin) * a.V
-                           : nullptr;
+  if (u >= 0 && u < u_lim) {
+    const int64_t rowoff = (int64_t)f * a.stat_frame_stride + (int64_t)(u - a.map_u0) * a.V;
+    float* srow = nullptr;
+    if (a.scores)
+      srow = a.roi ? a.scores + ((int64_t)ft * a.roi_h + (u - ru0)) * a.roi_w - rv0
+                   : a.scores + (int64_t)f * a.score_frame_stride + (int64_t)(u - a.u_begin) * a.V;
 #pragma unroll
     for (int c = 0; c < RV; ++c) {
       const int v = v0 + lv + c;
-      if (v < a.V) {
+      if (v >= 0 && v < v_lim) {
         const double s1 = a.S1[rowoff + v], s2 = a.S2[rowoff + v];
         float sc;
         if (a.ssd)  // sum T^2 - 2 sum T W + sum W^2, with sum T W = sum A_C W + Tbar S1
@@ -500,7 +519,7 @@ __global__ void __launch_bounds__(WX* WY * 32)
     }
   }
   best = block_max_key(best, red_key);
-  if (tid == 0 && best) atomicMax(a.keys + f, best);
+  if (tid == 0 && best) atomicMax(a.keys + ft, best);
 }
 
 // Template prep (Fig 5.2): Tbar, A_C = T - Tbar (fp32, zero-padded), A_D = sum A_C^2 (fp64),
@@ -508,6 +527,11 @@ __global__ void __launch_bounds__(WX* WY * 32)
 __global__ void tm_template_prep(const float* __restrict__ tmpl, int64_t tpitch, int h, int w,
                                  float* __restrict__ tplC, int HP, int WP, TemplateStats* ts,
                                  unsigned long long* keys, int batch) {
+  // blockIdx.x = template index (multi-template mode): template t at tmpl + t*h*tpitch
+  const int t = blockIdx.x, T = gridDim.x;
+  tmpl += (int64_t)t * h * tpitch;
+  tplC += (int64_t)t * HP * WP;
+  ts += t;
   __shared__ double red[32];
   const int n = h * w;
   double s = 0.0, s2 = 0.0;
@@ -541,13 +565,14 @@ __global__ void tm_template_prep(const float* __restrict__ tmpl, int64_t tpitch,
     ts->flat = (e <= kFlatRel * s2) ? 1 : 0;
     ts->pad = 0;
   }
-  for (int f = threadIdx.x; f < batch; f += blockDim.x) keys[f] = 0ull;
+  for (int f = threadIdx.x; f < batch; f += blockDim.x) keys[(int64_t)f * T + t] = 0ull;
 }
 
 __global__ void tm_finalize(const unsigned long long* __restrict__ keys, const TemplateStats* ts, int V,
-                            PeakOut* __restrict__ peaks, int batch, int ssd) {
-  const int f = blockIdx.x * blockDim.x + threadIdx.x;
-  if (f >= batch) return;
+                            PeakOut* __restrict__ peaks, int batch, int ssd, int n_tmpl) {
+  const int f = blockIdx.x * blockDim.x + threadIdx.x;  // frame * n_tmpl + template
+  if (f >= batch * n_tmpl) return;
+  ts += f % n_tmpl;
   const unsigned long long k = keys[f];
   const uint32_t idx = key_index(k);
   PeakOut p;
@@ -628,36 +653,80 @@ __global__ void __launch_bounds__(NT)
   }
 }
 
-// Vertical pass: S[f][u][v] = sum_{i<h} RS[f][u + i][v] for u < rows_out: direct sum for the
-// first of RB rows, then sliding updates (fp64).  grid = (ceil(V/NT), ceil(rows_out/RB), batch).
-template <int NT, int RB>
-__global__ void __launch_bounds__(NT)
+// Vertical pass: S[f][u][v] = sum_{i<h} RS[f][u + i][v] for u < rows_out (fp64).
+// CTA = 32 columns (lanes) x NW warps, output rows [ub, ub + NW*L).  The first row's sum is
+// formed cooperatively (each warp sums h/NW rows, combined in warp order); the others follow
+// from a block scan of the differences d_k = RS[ub+k+h] - RS[ub+k] (warp-local sequential
+// scan + exclusive scan of the warp totals).  ~3 loads per output, all warps issue
+// independent loads (the sliding form needed h + 2L dependent-latency loads per thread).
+// Exact for 2^-8-quantised inputs.  grid = (ceil(V/32), ceil(rows_out/(NW*L)), batch).
+template <int NW, int L>
+__global__ void __launch_bounds__(NW * 32)
     box_cols_kernel(const double* __restrict__ RS1, const double* __restrict__ RS2, int64_t rs_frame_stride,
                     int V, int h, int rows_out, double* __restrict__ S1, double* __restrict__ S2,
                     int64_t s_frame_stride) {
-  const int v = blockIdx.x * NT + threadIdx.x;
-  if (v >= V) return;
+  __shared__ double part1[NW][32], part2[NW][32], tot1[NW][32], tot2[NW][32];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int v = blockIdx.x * 32 + lane;
+  const bool okv = v < V;
+  const int vv = okv ? v : V - 1;
   const int f = blockIdx.z;
-  const int ub = blockIdx.y * RB;
-  const double* r1 = RS1 + (int64_t)f * rs_frame_stride + v;
-  const double* r2 = RS2 + (int64_t)f * rs_frame_stride + v;
-  double* o1 = S1 + (int64_t)f * s_frame_stride + v;
-  double* o2 = S2 + (int64_t)f * s_frame_stride + v;
+  const int ub = blockIdx.y * (NW * L);
+  const double* r1 = RS1 + (int64_t)f * rs_frame_stride + vv;
+  const double* r2 = RS2 + (int64_t)f * rs_frame_stride + vv;
+  // (1) first output row of the CTA: sum over rows ub .. ub+h-1, split over the warps
   double a1 = 0.0, a2 = 0.0;
-#pragma unroll 8
-  for (int i = 0; i < h; ++i) {
+  for (int i = wid; i < h; i += NW) {
     a1 += __ldg(r1 + (int64_t)(ub + i) * V);
     a2 += __ldg(r2 + (int64_t)(ub + i) * V);
   }
-  const int ue = min(ub + RB, rows_out);
-  o1[(int64_t)ub * V] = a1;
-  o2[(int64_t)ub * V] = a2;
-#pragma unroll 4
-  for (int u = ub + 1; u < ue; ++u) {
-    a1 += __ldg(r1 + (int64_t)(u + h - 1) * V) - __ldg(r1 + (int64_t)(u - 1) * V);
-    a2 += __ldg(r2 + (int64_t)(u + h - 1) * V) - __ldg(r2 + (int64_t)(u - 1) * V);
-    o1[(int64_t)u * V] = a1;
-    o2[(int64_t)u * V] = a2;
+  part1[wid][lane] = a1;
+  part2[wid][lane] = a2;
+  // (2) this warp's differences and their local inclusive scan
+  const int k0 = wid * L;
+  double d1[L], d2[L];
+#pragma unroll
+  for (int k = 0; k < L; ++k) {
+    const int u = ub + k0 + k;  // output row whose difference to the next is d_k
+    const bool ok = (u + 1 < rows_out);
+    d1[k] = ok ? __ldg(r1 + (int64_t)(u + h) * V) - __ldg(r1 + (int64_t)u * V) : 0.0;
+    d2[k] = ok ? __ldg(r2 + (int64_t)(u + h) * V) - __ldg(r2 + (int64_t)u * V) : 0.0;
+  }
+  double c1 = 0.0, c2 = 0.0;
+#pragma unroll
+  for (int k = 0; k < L; ++k) {
+    c1 += d1[k];
+    c2 += d2[k];
+    d1[k] = c1;
+    d2[k] = c2;
+  }
+  tot1[wid][lane] = c1;
+  tot2[wid][lane] = c2;
+  __syncthreads();
+  double b1 = 0.0, b2 = 0.0;
+  for (int q = 0; q < NW; ++q) {
+    b1 += part1[q][lane];
+    b2 += part2[q][lane];
+  }
+  for (int q = 0; q < wid; ++q) {
+    b1 += tot1[q][lane];
+    b2 += tot2[q][lane];
+  }
+  // (3) outputs: row ub+k0 gets the base; row ub+k0+k+1 gets base + prefix d_0..d_k
+  if (!okv) return;
+  double* o1 = S1 + (int64_t)f * s_frame_stride + v;
+  double* o2 = S2 + (int64_t)f * s_frame_stride + v;
+  if (ub + k0 < rows_out) {
+    o1[(int64_t)(ub + k0) * V] = b1;
+    o2[(int64_t)(ub + k0) * V] = b2;
+  }
+#pragma unroll
+  for (int k = 0; k + 1 < L; ++k) {
+    const int u = ub + k0 + k + 1;
+    if (u < rows_out) {
+      o1[(int64_t)u * V] = b1 + d1[k];
+      o2[(int64_t)u * V] = b2 + d2[k];
+    }
   }
 }
 
