@@ -95,3 +95,13 @@ def test_product_package_does_not_import_oracle():
             if f.endswith((".py", ".cu", ".cuh", ".h")):
                 txt = open(os.path.join(dp, f)).read()
                 assert "import oracle" not in txt and "from oracle" not in txt and "ncc_oracle" not in txt, f
+
+
+def test_c_example_compiles_against_the_header(tmp_path):
+    """The C ABI is usable from plain C (gcc, no CUDA headers): examples/ncc_example.c."""
+    import subprocess
+    exe = tmp_path / "ncc_example"
+    r = subprocess.run(["gcc", "-O2", "-I", os.path.join(ROOT, "include"), os.path.join(ROOT, "examples", "ncc_example.c"),
+                        "-o", str(exe), "-L", os.path.dirname(N.LIB_PATH), "-lncc_b200",
+                        "-Wl,-rpath," + os.path.dirname(N.LIB_PATH)], capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr

@@ -238,3 +238,15 @@ def test_concurrent_plans_on_two_streams():
     finally:
         for p in plans:
             p.close()
+
+
+def test_c_example_runs_end_to_end(tmp_path):
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    libdir = os.path.join(root, "paper_conf_ipps_moorelk13_b200")
+    exe = tmp_path / "ncc_example"
+    subprocess.check_call(["gcc", "-O2", "-I", os.path.join(root, "include"), os.path.join(root, "examples", "ncc_example.c"),
+                           "-o", str(exe), "-L", libdir, "-lncc_b200", "-Wl,-rpath," + libdir])
+    r = subprocess.run([str(exe)], capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stdout + r.stderr
