@@ -380,7 +380,10 @@ __global__ void __launch_bounds__(WX* WY * 32)
   const int u0 = ru0 + ty * T::BU;
   const int v0 = rv0 + tx * T::BV;
   const int nq = a.q_end - a.q_begin;
-  const int q0 = a.q_begin + (split * nq) / S, q1 = a.q_begin + ((split + 1) * nq) / S;
+  const int q0 = a.q_begin + (split * nq) / S;
+  // a tile entirely outside its (clipped) ROI computes nothing (a TMA box may not start past
+  // the tensor), but still takes part in the split-K combine
+  const int q1 = (u0 >= u_lim || v0 >= v_lim) ? q0 : a.q_begin + ((split + 1) * nq) / S;
   const int64_t tile_lin = (int64_t)ft * a.tiles_u * a.tiles_v + tile;
 
   float total[RV];
