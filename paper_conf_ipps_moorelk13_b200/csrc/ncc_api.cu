@@ -496,7 +496,7 @@ ncc_status create_tm(ncc_plan pl) {
   // of a problem uses the same S and the same per-offset accumulation order): the smallest
   // S <= chunks whose unit count fills whole "rounds" of resident CTAs to >= 97 %.
   pl->tiles_u = ceil_div(pl->roi_mode ? p.roi_h : pl->Ub, v->bu);
-  pl->tiles_v = ceil_div(pl->roi_mode ? p.roi_w : pl->V, v->bv);
+  pl->tiles_v = ceil_div(pl->roi_mode ? p.roi_w + 3 : pl->V, v->bv);  // ROI tiles start 16-B aligned
   {
     int per_sm = 0;
     const int ct = pl->use_ct ? 1 : 0;
@@ -869,7 +869,9 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   // TMA maps over all frames of the call (3D: cols, rows, pair); plain loads otherwise
   CUtensorMap mB;
   memset(&mB, 0, sizeof(mB));
-  bool use_tma = v->k_tma != nullptr && p.image_pitch % 4 == 0 && reinterpret_cast<uintptr_t>(B) % 16 == 0;
+  // a TMA box must start on a 16-byte boundary of the row: window columns kx * step_x
+  bool use_tma = v->k_tma != nullptr && p.image_pitch % 4 == 0 && p.step_x % 4 == 0 &&
+                 reinterpret_cast<uintptr_t>(B) % 16 == 0;
   if (use_tma) {
     const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
     const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)fs * 4};

@@ -377,8 +377,13 @@ __global__ void __launch_bounds__(WX* WY * 32)
     u_lim = min(ru0 + a.roi_h, a.U);
     v_lim = min(rv0 + a.roi_w, a.V);
   }
+  // tiles start at a multiple of 4 columns: a TMA box must start on a 16-byte boundary of the
+  // row (measured on B200: an unaligned inner coordinate raises an illegal instruction); the
+  // ROI's first columns below rv0 are computed and masked (host: tiles_v covers roi_w + 3)
+  const int v_org = rv0 & ~3;
+  const int v_min = rv0 > 0 ? rv0 : 0;
   const int u0 = ru0 + ty * T::BU;
-  const int v0 = rv0 + tx * T::BV;
+  const int v0 = v_org + tx * T::BV;
   const int nq = a.q_end - a.q_begin;
   const int q0 = a.q_begin + (split * nq) / S;
   // a tile entirely outside its (clipped) ROI computes nothing (a TMA box may not start past
@@ -508,7 +513,7 @@ __global__ void __launch_bounds__(WX* WY * 32)
 #pragma unroll
     for (int c = 0; c < RV; ++c) {
       const int v = v0 + lv + c;
-      if (v >= 0 && v < v_lim) {
+      if (v >= v_min && v < v_lim) {
         const double s1 = a.S1[rowoff + v], s2 = a.S2[rowoff + v];
         float sc;
         if (a.ssd)  // sum T^2 - 2 sum T W + sum W^2, with sum T W = sum A_C W + Tbar S1

@@ -108,12 +108,13 @@ def test_cfg4_two_pairs_sampled():
 @pytest.mark.parametrize("h,w,my,mx,sy,sx", [(24, 20, 5, 7, 9, 11), (16, 16, 4, 4, 8, 8), (32, 32, 16, 16, 16, 16),
                                              (13, 29, 3, 0, 7, 5)])
 @pytest.mark.parametrize("generic", [True, False])
-def test_odd_shapes_generic_and_runtime_specialised(h, w, my, mx, sy, sx, generic):
-    p = synth.particle_pair_integer(150, 170, 2, -3, seed=5000 + h)
+@pytest.mark.parametrize("W", [170, 168])  # 170: plain loads (pitch); 168: TMA when step_x % 4 == 0
+def test_odd_shapes_generic_and_runtime_specialised(h, w, my, mx, sy, sx, generic, W):
+    p = synth.particle_pair_integer(150, W, 2, -3, seed=5000 + h)
     v, sc, info = run_piv([p.A], [p.B], (h, w), None, None, generic=generic, search=(my, mx), step=(sy, sx))
     aot = (h, w, my, mx) == (32, 32, 16, 16)
     assert info["specialized"] == (0 if generic else (1 if aot else 2)), info["variant_name"]
-    Ky, Kx = oracle.piv_grid(150, 170, h, w, my, mx, sy, sx)
+    Ky, Kx = oracle.piv_grid(150, W, h, w, my, mx, sy, sx)
     assert v["iy"].shape == (1, Ky, Kx)
     ref = oracle.piv_pair(p.A, p.B, h, w, my, mx, sy, sx)
     np.testing.assert_array_equal(v["iy"][0], ref["iy"])
