@@ -28,6 +28,7 @@
 
 #include "../../include/ncc.h"
 #include "ncc_kernels.cuh"
+#include "ncc_tc.cuh"
 
 using namespace nccb;
 
@@ -162,6 +163,7 @@ const PivVariant kPivVariants[] = {
 
 constexpr int kBoxRowsNT = 256, kBoxRowsSEG = 2048;  // max segment; actual = min(V, SEG)
 constexpr int kBoxColsNW = 8, kBoxColsL = 16;  // 32 columns x 8 warps x 16 rows per CTA
+constexpr int kBox2dNT = 256, kBoxTV = 128;      // fused window sums: 128-column strips
 
 int ceil_div(int64_t a, int64_t b) { return (int)((a + b - 1) / b); }
 
@@ -292,6 +294,10 @@ struct ncc_plan_s {
   // shared scratch (window sums)
   double *RS1, *RS2, *S1, *S2;
   int64_t rs_frame_stride, s_frame_stride;
+  int box_r, box_iwp, box_smem, nsm;  // fused window-sum kernel (box_smem 0: two-pass fallback)
+  // tensor-core numerator (tm_tc_kernel): 0 = CUDA-core path
+  int tc, tc_wc, tc_nbi, tc_nbj, tc_vtiles, tc_useg, tc_nseg;
+  float *tcB, *tc_part;
   // side stream for work independent of the main chain (template prep || window sums)
   cudaStream_t side;
   cudaEvent_t ev_fork, ev_join;
@@ -327,6 +333,8 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->tst);
   cudaFree(pl->keys);
   cudaFree(pl->RS1);
+  cudaFree(pl->tcB);
+  cudaFree(pl->tc_part);
   cudaFree(pl->RS2);
   cudaFree(pl->S1);
   cudaFree(pl->S2);
@@ -392,6 +400,72 @@ void fill_kernel_info(ncc_plan pl, const void* fn, int nt, int smem, int gx, int
   pl->info.grid_x = gx;
   pl->info.grid_y = gy;
   pl->info.grid_z = gz;
+}
+
+// Fused window-sum kernel geometry: R rows of a (kBoxTV + w - 1)-column strip staged per
+// sub-block; NCC_BOX_TWO_PASS=1 (or a strip too wide for shared memory) keeps the two-pass form.
+ncc_status setup_box(ncc_plan pl, int w) {
+  int maxsm = 0;
+  NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
+  NCC_CUDA(cudaDeviceGetAttribute(&pl->nsm, cudaDevAttrMultiProcessorCount, pl->device));
+  pl->box_iwp = kBoxTV + w - 1;
+  const int64_t r = ((int64_t)maxsm / 8 - 2 * pl->box_iwp) / (2 * pl->box_iwp);
+  pl->box_r = r > 16 ? 16 : (int)r;
+  pl->box_smem = 0;
+  if (pl->box_r >= 1 && !getenv("NCC_BOX_TWO_PASS")) {
+    pl->box_smem = (2 * pl->box_r + 2) * pl->box_iwp * (int)sizeof(double);
+    NCC_CUDA(cudaFuncSetAttribute((const void*)box2d_kernel<kBox2dNT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  pl->box_smem));
+  }
+  return NCC_OK;
+}
+
+// Tensor-core numerator (ncc_tc.cuh) for band-mode TM: template blocks of tc::kHB rows x WC
+// columns, 128-column output tiles, output-row segments.  WC and the segment count minimise
+// waves x (image rows per CTA) x (column chunks per row), the kernel's MMA time model.
+ncc_status setup_tc(ncc_plan pl) {
+  const ncc_problem& p = pl->p;
+  pl->tc = 0;
+  const char* env = getenv("NCC_TC");
+  if (!env || atoi(env) == 0 || pl->roi_mode || pl->n_tmpl != 1) return NCC_OK;
+  const int h = p.tmpl_h, w = p.tmpl_w;
+  pl->tc_vtiles = ceil_div(pl->V, 128);
+  pl->tc_nbi = ceil_div(h, tc::kHB);
+  double best = 1e300;
+  for (int wc = tc::kWB; wc <= 128; wc *= 2) {
+    const int nbj = ceil_div(w, wc);
+    const int64_t per_seg = (int64_t)pl->tc_vtiles * pl->tc_nbi * nbj * p.batch;
+    for (int nseg = 1; nseg <= 64 && nseg <= pl->Ub; ++nseg) {
+      const int useg = ceil_div(pl->Ub, nseg);
+      const int64_t ctas = per_seg * ceil_div(pl->Ub, useg);
+      const int64_t waves = (ctas + pl->nsm - 1) / pl->nsm;
+      const double cost = (double)waves * (double)(ceil_div(useg + tc::kHB - 1, tc::kG) * tc::kG) * (wc / tc::kWB);
+      if (cost < best * 0.999) {
+        best = cost;
+        pl->tc_wc = wc;
+        pl->tc_nbj = nbj;
+        pl->tc_useg = useg;
+        pl->tc_nseg = ceil_div(pl->Ub, useg);
+      }
+    }
+    if (wc >= w) break;
+  }
+  const int nblk = pl->tc_nbi * pl->tc_nbj;
+  ncc_status st;
+  if ((st = dalloc(&pl->tcB, (size_t)nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
+  if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
+  const int smem = tc::smem_bytes(pl->tc_wc);
+  NCC_CUDA(cudaFuncSetAttribute((const void*)tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  pl->tc = 1;
+  ncc_plan_info& in = pl->info;
+  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d", tc::kHB, pl->tc_wc, pl->tc_nseg);
+  fill_kernel_info(pl, (const void*)tm_tc_kernel, tc::kThreads, smem, nblk * pl->tc_vtiles * pl->tc_nseg, p.batch, 1);
+  in.specialized = 1;
+  in.split = nblk;
+  in.const_template = 0;
+  in.slabs = 1;
+  in.launches_per_call = 2 + (pl->box_smem ? 1 : 2) + 3;  // prep, operand prep, sums, numerator, finish, finalize
+  return NCC_OK;
 }
 
 ncc_status create_tm(ncc_plan pl) {
@@ -537,8 +611,11 @@ ncc_status create_tm(ncc_plan pl) {
     if ((st = dalloc(&pl->carry, (size_t)ntiles * v->rv_nt()))) return st;
   pl->rs_frame_stride = (int64_t)pl->Hs * pl->V;
   pl->s_frame_stride = (int64_t)pl->Ub * pl->V;
-  if ((st = dalloc(&pl->RS1, (size_t)p.batch * pl->rs_frame_stride))) return st;
-  if ((st = dalloc(&pl->RS2, (size_t)p.batch * pl->rs_frame_stride))) return st;
+  if ((st = setup_box(pl, w))) return st;
+  if (!pl->box_smem) {  // row-sum intermediate of the two-pass form only
+    if ((st = dalloc(&pl->RS1, (size_t)p.batch * pl->rs_frame_stride))) return st;
+    if ((st = dalloc(&pl->RS2, (size_t)p.batch * pl->rs_frame_stride))) return st;
+  }
   if ((st = dalloc(&pl->S1, (size_t)p.batch * pl->s_frame_stride))) return st;
   if ((st = dalloc(&pl->S2, (size_t)p.batch * pl->s_frame_stride))) return st;
   {  // template chunks: 2D map over the zero-padded centred template
@@ -568,9 +645,9 @@ ncc_status create_tm(ncc_plan pl) {
     in.split = pl->split;
     in.const_template = pl->use_ct;
     in.slabs = pl->n_slabs;
-    in.launches_per_call = 4 + pl->n_slabs;  // prep, 2 window-sum passes, numerator(s), finalize
+    in.launches_per_call = 2 + (pl->box_smem ? 1 : 2) + pl->n_slabs;  // prep, window sums, numerator(s), finalize
   }
-  return NCC_OK;
+  return setup_tc(pl);
 }
 
 ncc_status create_piv(ncc_plan pl) {
@@ -671,14 +748,17 @@ ncc_status create_piv(ncc_plan pl) {
   // window-sum maps of frame B, processed in sub-batches of pairs (scratch budget ~2 GiB)
   pl->rs_frame_stride = (int64_t)p.image_h * pl->map_w;
   pl->s_frame_stride = (int64_t)pl->map_h * pl->map_w;
-  const double per_pair = 16.0 * (double)(pl->rs_frame_stride + pl->s_frame_stride);
+  ncc_status st;
+  if ((st = setup_box(pl, w))) return st;
+  const double per_pair = 16.0 * (double)((pl->box_smem ? 0 : pl->rs_frame_stride) + pl->s_frame_stride);
   int sb = (int)(2.0 * 1024 * 1024 * 1024 / per_pair);
   if (sb < 1) sb = 1;
   if (sb > p.batch) sb = p.batch;
   pl->sub_batch = sb;
-  ncc_status st;
-  if ((st = dalloc(&pl->RS1, (size_t)sb * pl->rs_frame_stride))) return st;
-  if ((st = dalloc(&pl->RS2, (size_t)sb * pl->rs_frame_stride))) return st;
+  if (!pl->box_smem) {
+    if ((st = dalloc(&pl->RS1, (size_t)sb * pl->rs_frame_stride))) return st;
+    if ((st = dalloc(&pl->RS2, (size_t)sb * pl->rs_frame_stride))) return st;
+  }
   if ((st = dalloc(&pl->S1, (size_t)sb * pl->s_frame_stride))) return st;
   if ((st = dalloc(&pl->S2, (size_t)sb * pl->s_frame_stride))) return st;
 
@@ -693,7 +773,7 @@ ncc_status create_piv(ncc_plan pl) {
   in.variant_id = pl->jit_lib ? -1 : (int)(v - kPivVariants);
   snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
   fill_kernel_info(pl, v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
-  in.launches_per_call = 3 * ceil_div(p.batch, sb);  // per sub-batch: 2 window-sum passes + PIV kernel
+  in.launches_per_call = (pl->box_smem ? 2 : 3) * ceil_div(p.batch, sb);  // per sub-batch: window sums + PIV
   return NCC_OK;
 }
 
@@ -715,6 +795,17 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
   const ncc_problem& p = pl->p;
   const int h = p.tmpl_h, w = p.tmpl_w;
   const int V = p.image_w - w + 1;
+  if (pl->box_smem) {  // fused single pass; rows per CTA halved until the grid fills the GPU twice
+    const int gx = ceil_div(V, kBoxTV);
+    int TU = 64;
+    while (TU > pl->box_r && (int64_t)gx * ceil_div(rows_out, TU) * batch < 2 * pl->nsm) TU /= 2;
+    dim3 g(gx, ceil_div(rows_out, TU), batch);
+    box2d_kernel<kBox2dNT><<<g, kBox2dNT, pl->box_smem, s>>>(frames, p.image_pitch,
+                                                            (int64_t)p.image_h * p.image_pitch, row0, h, w, V,
+                                                            rows_out, kBoxTV, TU, pl->box_r, pl->box_iwp, pl->S1,
+                                                            pl->S2, pl->s_frame_stride);
+    return;
+  }
   const int rows_in = rows_out + h - 1;
   const int seg = V < kBoxRowsSEG ? V : kBoxRowsSEG;
   const int smem = (int)((seg + w + 1) * 2 * sizeof(double));
@@ -743,10 +834,57 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   tm_template_prep<<<pl->n_tmpl, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP,
                                                        pl->WP, pl->tst, pl->keys, p.batch);
   mark(pl, pl->side, 1);
+  if (pl->tc) {
+    const int nblk = pl->tc_nbi * pl->tc_nbj;
+    tm_tc_tpl_prep<<<nblk, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj, pl->tcB);
+  }
   NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
   launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
   NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
   mark(pl, s, 2);
+  CUtensorMap map_tc;
+  bool tc_now = false;
+  if (pl->tc && reinterpret_cast<uintptr_t>(d_images) % 16 == 0 && p.image_pitch % 4 == 0) {
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
+    const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)p.image_h * p.image_pitch * 4};
+    const uint32_t box[3] = {(uint32_t)tc::kBoxW, 1u, 1u};
+    tc_now = encode_f32(&map_tc, d_images, 3, dims, strides, box);
+  }
+  if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
+    const int nblk = pl->tc_nbi * pl->tc_nbj;
+    TcArgs t;
+    t.img = d_images;
+    t.pitch = p.image_pitch;
+    t.frame_stride = (int64_t)p.image_h * p.image_pitch;
+    t.H = p.image_h;
+    t.W = p.image_w;
+    t.tcB = pl->tcB;
+    t.WC = pl->tc_wc;
+    t.nbi = pl->tc_nbi;
+    t.nbj = pl->tc_nbj;
+    t.V = pl->V;
+    t.u_begin = pl->u_begin;
+    t.u_end = pl->u_end;
+    t.useg = pl->tc_useg;
+    t.nseg = pl->tc_nseg;
+    t.vtiles = pl->tc_vtiles;
+    t.part = pl->tc_part;
+    t.part_frame_stride = (int64_t)pl->Ub * pl->V;
+    t.part_blk_stride = t.part_frame_stride * p.batch;
+    tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, p.batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
+        t, map_tc);
+    mark(pl, s, 3);
+    tm_tc_finish<<<dim3(pl->Ub, p.batch), 256, 0, s>>>(
+        pl->tc_part, nblk, t.part_blk_stride, t.part_frame_stride, pl->S1, pl->S2, pl->s_frame_stride, pl->tst,
+        p.tmpl_h, p.tmpl_w, pl->V, pl->u_begin, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
+        (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD);
+    tm_finalize<<<ceil_div((int64_t)p.batch, 128), 128, 0, s>>>(
+        pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks), p.batch, p.score == NCC_SCORE_SSD, 1);
+    mark(pl, s, 4);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch (tensor core)");
+    return NCC_OK;
+  }
   TmArgs a;
   a.img = d_images;
   a.pitch = p.image_pitch;

@@ -661,6 +661,104 @@ __global__ void __launch_bounds__(NT)
   }
 }
 
+// Fused window sums (one pass, no row-sum intermediate):
+//   S[f][u][v] = sum_{i<h, j<w} I[f][row0 + u + i][v + j]  (and of squares), fp64.
+// CTA = a strip of TV output columns x TU output rows, processed in sub-blocks of R rows:
+//   (1) vertical: each thread owns input columns c of the strip (TV + w - 1 of them) and keeps
+//       the column sum CS_u(c) = sum_{i<h} I[u + i][c] in shared memory; the CTA's first row is
+//       summed directly (h loads), every later row slides: CS += I[u + h - 1] - I[u - 1];
+//   (2) horizontal: one warp per row turns CS into an inclusive prefix P (warp scans with a
+//       carry) and writes S[u][v] = P[v + w - 1] - P[v - 1].
+// Every partial sum is exact for 2^-8-quantised inputs (any order), so S is exact there.
+// grid = (ceil(V / TV), ceil(rows_out / TU), batch), block = NT,
+// dynamic smem = (2 * R + 2) * IWP doubles (X1, X2 [R][IWP]; C1, C2 [IWP]).
+template <int NT>
+__global__ void __launch_bounds__(NT)
+    box2d_kernel(const float* __restrict__ img, int64_t pitch, int64_t frame_stride, int row0, int h, int w, int V,
+                 int rows_out, int TV, int TU, int R, int IWP, double* __restrict__ S1, double* __restrict__ S2,
+                 int64_t s_frame_stride) {
+  extern __shared__ double sm_box[];
+  double* X1 = sm_box;
+  double* X2 = X1 + (int64_t)R * IWP;
+  double* C1 = X2 + (int64_t)R * IWP;
+  double* C2 = C1 + IWP;
+  const int f = blockIdx.z;
+  const int v0 = blockIdx.x * TV;
+  const int ub = blockIdx.y * TU;
+  const int tv = min(TV, V - v0);
+  const int iw = tv + w - 1;
+  const int nrow = min(TU, rows_out - ub);
+  const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + ub) * pitch + v0;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  constexpr int NW = NT / 32;
+  for (int r0 = 0; r0 < nrow; r0 += R) {
+    const int nr = min(R, nrow - r0);
+    for (int c = threadIdx.x; c < iw; c += NT) {
+      const float* col = src + c;
+      double c1, c2;
+      int r = 0;
+      if (r0 == 0) {  // first output row of the CTA: direct column sum (independent loads)
+        double a[4] = {0.0, 0.0, 0.0, 0.0}, b[4] = {0.0, 0.0, 0.0, 0.0};
+        int i = 0;
+        for (; i + 4 <= h; i += 4) {
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            const double x = __ldg(col + (int64_t)(i + k) * pitch);
+            a[k] += x;
+            b[k] = fma(x, x, b[k]);
+          }
+        }
+        for (; i < h; ++i) {
+          const double x = __ldg(col + (int64_t)i * pitch);
+          a[0] += x;
+          b[0] = fma(x, x, b[0]);
+        }
+        c1 = (a[0] + a[1]) + (a[2] + a[3]);
+        c2 = (b[0] + b[1]) + (b[2] + b[3]);
+        X1[c] = c1;
+        X2[c] = c2;
+        r = 1;
+      } else {
+        c1 = C1[c];
+        c2 = C2[c];
+      }
+      for (; r < nr; ++r) {  // slide down one row: + entering row, - leaving row
+        const int u = r0 + r;
+        const double xi = __ldg(col + (int64_t)(u + h - 1) * pitch);
+        const double xo = __ldg(col + (int64_t)(u - 1) * pitch);
+        c1 = (c1 + xi) - xo;
+        c2 = fma(-xo, xo, fma(xi, xi, c2));
+        X1[(int64_t)r * IWP + c] = c1;
+        X2[(int64_t)r * IWP + c] = c2;
+      }
+      C1[c] = c1;
+      C2[c] = c2;
+    }
+    __syncthreads();
+    for (int r = wid; r < nr; r += NW) {
+      double* x1 = X1 + (int64_t)r * IWP;
+      double* x2 = X2 + (int64_t)r * IWP;
+      double k1 = 0.0, k2 = 0.0;
+      for (int c0 = 0; c0 < iw; c0 += 32) {
+        const int c = c0 + lane;
+        double p1 = c < iw ? x1[c] : 0.0, p2 = c < iw ? x2[c] : 0.0;
+        p1 = warp_incl_scan_d(p1) + k1;
+        p2 = warp_incl_scan_d(p2) + k2;
+        if (c < iw) { x1[c] = p1; x2[c] = p2; }
+        k1 = __shfl_sync(0xffffffffu, p1, 31);
+        k2 = __shfl_sync(0xffffffffu, p2, 31);
+      }
+      __syncwarp();
+      const int64_t o = (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
+      for (int v = lane; v < tv; v += 32) {
+        S1[o + v] = x1[v + w - 1] - (v > 0 ? x1[v - 1] : 0.0);
+        S2[o + v] = x2[v + w - 1] - (v > 0 ? x2[v - 1] : 0.0);
+      }
+    }
+    __syncthreads();
+  }
+}
+
 // Vertical pass: S[f][u][v] = sum_{i<h} RS[f][u + i][v] for u < rows_out (fp64).
 // CTA = 32 columns (lanes) x NW warps, output rows [ub, ub + NW*L).  The first row's sum is
 // formed cooperatively (each warp sums h/NW rows, combined in warp order); the others follow

@@ -1,0 +1,403 @@
+// ncc_tc.cuh -- tensor-core (tcgen05, kind::tf32) numerator of the TM path.
+//
+// What it computes: the numerator stage of Fig 5.3, N[u][v] = sum_{i,j} A_C[i][j] *
+// I[u+i][v+j], for a template block of up to HB x WC template elements; the normalisation
+// (Figs 5.1/5.2) and the argmax stay in fp64 / fp32 exactly as in the CUDA-core path.
+//
+// Mapping onto the 5th-generation tensor cores (sm_100a):
+//   * M = 128 output columns v of a tile (one TMEM lane each);
+//   * K = template columns j, 8 per tcgen05.mma (tf32);
+//   * N = a window of output rows u: for image row r the B operand row c is the template row
+//     r - u(c), i.e. a window into the REVERSED, zero-padded template block held in shared
+//     memory (K-major, no swizzle, 16-byte rows, so a window may start at any row: only the
+//     descriptor start address moves); the accumulator D[v][u] lives in a ring of TMEM columns
+//     indexed by u, and the MMA over image row r adds exactly the terms A_C[r-u][.] * I[r][v+.]
+//     to every output row u of the window -- each output's sum accumulates in D in the same
+//     row-by-row order, whatever band / segment the CTA works on (bitwise band-invariant).
+//   * A operand = the Hankel matrix H_r[v][j] = I[r][v0+v+j] of image row r, written by the
+//     producer warps straight into TMEM (tcgen05.st; lane v = row v), so the MMAs read only
+//     the template window from shared memory.
+//   * fp32 accuracy from tf32 units: x = hi + lo (hi = tf32(x), lo = x - hi exact), and
+//     A.B ~ A_hi.B_hi + A_hi.B_lo + A_lo.B_hi ("3xTF32"; dropped term ~2^-22 relative).
+// Rows are processed in groups of G: the window of group g is the HB + G output rows
+// [G g - HB + 1, G g + G + 1); after the group the first G of them are complete, drained from
+// TMEM (tcgen05.ld) to the partial-numerator buffer and their columns zeroed for reuse.
+// Warp roles: warps 0-3 produce the Hankel operand (and drain the ring: lane quadrant w),
+// warp 4 (one thread) issues the MMAs; TMEM A is double-buffered per (row, column chunk).
+#pragma once
+#include "ncc_kernels.cuh"
+
+namespace nccb {
+namespace tc {
+
+__device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFFu);
+  d |= (uint64_t)((lbo >> 4) & 0x3FFFu) << 16;
+  d |= (uint64_t)((sbo >> 4) & 0x3FFFu) << 32;
+  d |= (uint64_t)1 << 46;  // descriptor version (sm_100); base offset 0; SWIZZLE_NONE
+  return d;
+}
+// kind::tf32 instruction descriptor: D f32, A/B tf32, both K-major, M = 128
+__host__ __device__ constexpr uint32_t idesc_tf32(int N) {
+  return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+}
+__device__ __forceinline__ void mma_ts(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t idesc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, 1, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d),
+      "r"(a_tmem), "l"(b), "r"(idesc)
+      : "memory");
+}
+__device__ __forceinline__ void commit(uint64_t* bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+__device__ __forceinline__ void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void st_wait() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void st8(uint32_t addr, const uint32_t (&v)[8]) {
+  asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(addr), "r"(v[0]),
+               "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7])
+               : "memory");
+}
+__device__ __forceinline__ void ld8(uint32_t addr, uint32_t (&v)[8]) {
+  asm volatile("tcgen05.ld.sync.aligned.32x32b.x8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7])
+               : "r"(addr)
+               : "memory");
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ bool elect_one() {
+  uint32_t pred = 0;
+  asm volatile("{\n\t.reg .pred P;\n\telect.sync _|P, 0xffffffff;\n\tselp.u32 %0, 1, 0, P;\n}" : "=r"(pred));
+  return pred != 0;
+}
+__device__ __forceinline__ uint32_t to_tf32(float x) {
+  uint32_t r;
+  asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+  return r;
+}
+
+constexpr int kHB = 128;   // template rows per block (B window rows N = kHB + kG)
+constexpr int kG = 8;      // image rows per group (ring advance, drain granularity)
+constexpr int kWB = 32;    // template columns per TMEM A chunk (4 MMAs of K = 8)
+constexpr int kRing = 256; // TMEM accumulator ring columns
+constexpr int kNBuf = 4;   // TMEM A stages (columns kRing + b*2*kWB .. ; 256 + 4*64 = 512)
+static_assert(kRing + kNBuf * 2 * kWB <= 512, "TMEM columns");
+constexpr int kNWin = kHB + kG;
+constexpr int kLB = ((kHB + 2 * kG - 1 + 7) / 8) * 8;  // rows of the reversed template block
+constexpr int kGroups = kNBuf;                           // producer groups of 4 warps; group g: stages q = g mod kNBuf
+constexpr int kThreads = kGroups * 128 + 32;             // + 1 MMA warp
+constexpr int kBoxW = 128 + kWB;                         // image-row segment of one stage (TMA box)
+constexpr int kNImg = 8;                                 // image-row ring (TMA issue distance)
+static_assert(kNImg % kNBuf == 0, "a stage and the stage kNImg later belong to the same producer group");
+// shared bytes of the template operand for a column super-block of WC columns (hi + lo)
+__host__ __device__ constexpr uint32_t plane_bytes() { return kLB * 16; }
+__host__ __device__ constexpr int b_bytes(int WC) { return 2 * (WC / 4) * kLB * 16; }
+// dynamic shared memory per CTA: the operand, padded so that one CTA fits per SM (the CTA
+// allocates all 512 TMEM columns)
+__host__ __device__ constexpr int img_off(int WC) { return ((b_bytes(WC) + 127) / 128) * 128; }
+__host__ __device__ constexpr int smem_need(int WC) { return img_off(WC) + kNImg * kBoxW * 4; }
+__host__ __device__ constexpr int smem_bytes(int WC) { return smem_need(WC) > 120 * 1024 ? smem_need(WC) : 120 * 1024; }
+
+}  // namespace tc
+
+#ifdef NCC_TC_TRACE  // tools/microbench/tc_trace.cu: per-stage clock64 stamps of CTA 0
+__device__ long long* g_tc_trace;
+#define TC_STAMP(slot, q) \
+  if (blockIdx.x == 0 && blockIdx.y == 0 && (q) < 1024) g_tc_trace[(slot)*1024 + (q)] = clock64()
+__device__ int g_tc_exp;  // timing experiments (trace builds only): bit0 no A stores, bit1 no wrap, bit2 one product
+#define TC_EXP(bit) (g_tc_exp & (bit))
+#else
+#define TC_EXP(bit) 0
+#define TC_STAMP(slot, q)
+#endif
+
+struct TcArgs {
+  const float* img;
+  int64_t pitch, frame_stride;
+  int H, W;
+  const float* tcB;     // [nblk][2 (hi, lo)][WC/4 planes][kLB rows][4]: reversed template blocks
+  int WC;               // template columns per CTA (multiple of kWB, <= 128)
+  int nbi, nbj;         // template blocks (row blocks of kHB, column super-blocks of WC)
+  int V;                // output columns
+  int u_begin, u_end;   // output rows of the band
+  int useg, nseg;       // output rows per CTA segment, segments
+  int vtiles;
+  float* part;          // [nblk][batch][u_end - u_begin][V] partial numerators
+  int64_t part_blk_stride, part_frame_stride;
+};
+
+// grid = (nblk * vtiles * nseg, batch); block = tc::kThreads; dynamic smem = tc::b_bytes(WC).
+__global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
+                                                                  const __grid_constant__ CUtensorMap map_img) {
+  using namespace tc;
+  extern __shared__ __align__(1024) unsigned char smem_tc[];
+  __shared__ __align__(8) uint64_t a_full[kNBuf], mma_done[kNBuf], img_full[kNImg], img_empty[kNImg];
+  __shared__ uint32_t tmem_base_s;
+
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  const int nblk = a.nbi * a.nbj;
+  const int blk = blockIdx.x % nblk;
+  const int rest = blockIdx.x / nblk;
+  const int vt = rest % a.vtiles, seg = rest / a.vtiles;
+  const int bi = blk / a.nbj, bj = blk % a.nbj;
+  const int f = blockIdx.y;
+  const int v0 = vt * 128;
+  const int ua = a.u_begin + seg * a.useg;
+  const int nu = min(a.useg, a.u_end - ua);  // output rows of this CTA
+  const int i0 = bi * kHB, j0 = bj * a.WC;
+  const int nch = a.WC / kWB;                // TMEM chunks per image row
+  const int R = nu + kHB - 1;                // image rows touching the CTA's outputs
+  const int ngrp = (R + kG - 1) / kG;
+  const int nrow = ngrp * kG;
+  const int nstage = nrow * nch;             // (row, chunk) stages
+  const uint32_t plane = kLB * 16;           // bytes per K plane of the template operand
+  const int npl = a.WC / 4;
+
+  // template operand (precomputed layout) -> shared memory
+  {
+    const float4* src = reinterpret_cast<const float4*>(a.tcB + (int64_t)blk * (b_bytes(a.WC) / 4));
+    float4* dst = reinterpret_cast<float4*>(smem_tc);
+    const int n4 = b_bytes(a.WC) / 16;
+    for (int k = tid; k < n4; k += kThreads) dst[k] = __ldg(src + k);
+  }
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], 512;" ::"r"(smem_u32(&tmem_base_s)));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == 0) {
+    for (int b = 0; b < kNBuf; ++b) {
+      mbar_init(&a_full[b], 128);
+      mbar_init(&mma_done[b], 1);
+    }
+    for (int b = 0; b < kNImg; ++b) {
+      mbar_init(&img_full[b], 1);
+      mbar_init(&img_empty[b], 128);
+    }
+    fence_mbar_init();
+  }
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tbase = tmem_base_s;
+  const uint32_t a_col0 = kRing;  // A buffers: [kRing + b*2*kWB, +kWB) hi, [+kWB, +2kWB) lo
+
+  if (warp < 4 * kGroups) {
+    // ===================== producers (lane v = output column v0 + v) and ring drain.
+    // Group grp (warps 4 grp .. 4 grp + 3, TMEM lane quadrants 0..3) handles the stages
+    // q = grp mod kNBuf, i.e. TMEM A buffer grp: the groups' latencies overlap.
+    const int grp = warp >> 2, wq = warp & 3;
+    const int gtid = tid & 127;  // thread index within the group
+    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
+    const int v = wq * 32 + lane;
+    if (grp == 0) {  // zero the accumulator ring before the first MMA (ordered by group 0's a_full arrival)
+      const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
+#pragma unroll 1
+      for (int c = 0; c < kRing; c += 8) st8(tbase + lane_base + c, z);
+      st_wait();
+      fence_before();
+    }
+    const float* ring = reinterpret_cast<const float*>(smem_tc + img_off(a.WC));
+    // stage q = (image row rr, column chunk ch): row ua + i0 + rr, columns v0 + j0 + 32 ch + [0, kBoxW)
+    auto stage_zero = [&](int q) {  // rows past the image / chunks past its width: zero operand
+      return ua + i0 + q / nch >= a.H || v0 + j0 + (q % nch) * kWB >= a.W;
+    };
+    auto issue = [&](int q) {  // one thread: TMA of stage q into ring slot q % kNImg
+      const int sl = q % kNImg;
+      if (q >= kNImg) mbar_wait_bounded(&img_empty[sl], (uint32_t)(((q - kNImg) / kNImg) & 1));
+      if (stage_zero(q)) {
+        mbar_arrive(&img_full[sl]);
+      } else {
+        mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 4));
+        tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 4, &map_img, v0 + j0 + (q % nch) * kWB, ua + i0 + q / nch,
+                    f, &img_full[sl]);
+      }
+    };
+    if (tid == 0) {
+      tma_prefetch_desc(&map_img);
+      for (int q = 0; q < kNImg && q < nstage; ++q) issue(q);
+    }
+    float* part = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * a.part_frame_stride;
+#pragma unroll 1
+    for (int q = grp; q < nstage + kNBuf; q += kGroups) {
+      const int b = grp;
+      if (q >= kNBuf) {  // MMAs of stage q - kNBuf (same buffer) are done
+        const int qd = q - kNBuf;
+        mbar_wait_bounded(&mma_done[b], (uint32_t)((qd / kNBuf) & 1));
+        fence_after();
+        if (gtid == 0) TC_STAMP(0, qd);
+        if (qd % nch == nch - 1 && (qd / nch) % kG == kG - 1) {  // last stage of group gd
+          const int gd = (qd / nch) / kG;
+          const uint32_t col = (uint32_t)((gd * kG) % kRing);
+          uint32_t d[8];
+          ld8(tbase + lane_base + col, d);
+          const int vv = v0 + v;
+#pragma unroll
+          for (int k = 0; k < kG; ++k) {
+            const int up = gd * kG - kHB + 1 + k;  // output row (CTA-relative)
+            if (up >= 0 && up < nu && vv < a.V)
+              part[(int64_t)(ua - a.u_begin + up) * a.V + vv] = __uint_as_float(d[k]);
+          }
+          const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
+          st8(tbase + lane_base + col, z);
+        }
+      }
+      if (q < nstage) {
+        const int sl = q % kNImg;
+        mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
+        if (gtid == 0) TC_STAMP(5, q);
+        float x[kWB];
+        const bool zero = stage_zero(q);
+#pragma unroll
+        for (int k = 0; k < kWB; ++k) x[k] = zero ? 0.0f : ring[sl * kBoxW + v + k];
+        mbar_arrive(&img_empty[sl]);
+        if (gtid == 0) TC_STAMP(6, q);
+        if (gtid == 0 && q + kNImg < nstage) issue(q + kNImg);
+        if (gtid == 0) TC_STAMP(7, q);
+        uint32_t hi[kWB], lo[kWB];
+#pragma unroll
+        for (int k = 0; k < kWB; ++k) {
+          hi[k] = to_tf32(x[k]);
+          lo[k] = __float_as_uint(x[k] - __uint_as_float(hi[k]));
+        }
+        if (gtid == 0) TC_STAMP(1, q);
+        const uint32_t ab = tbase + lane_base + a_col0 + (uint32_t)(b * 2 * kWB);
+#pragma unroll
+        if (!TC_EXP(1))
+          for (int c = 0; c < kWB; c += 8) {
+            st8(ab + c, *reinterpret_cast<const uint32_t(*)[8]>(hi + c));
+            st8(ab + kWB + c, *reinterpret_cast<const uint32_t(*)[8]>(lo + c));
+          }
+        st_wait();
+        fence_before();
+        mbar_arrive(&a_full[b]);
+        if (gtid == 0) TC_STAMP(2, q);
+      }
+    }
+  } else if (warp == 4 * kGroups) {
+    // ===================== MMA issuer (one thread)
+    // Straight-line issue: the thread's scalar work per MMA is one 64-bit descriptor add and one
+    // TMEM address add (measured: a loop body of ~30 dependent scalar instructions per MMA
+    // throttles issue to ~250 cycles per MMA, ~4x the tensor pipe's time for N = 136).
+    {  // the whole warp runs the loop (warp-uniform operands -> uniform datapath); one lane issues
+      const uint32_t bhi = smem_u32(smem_tc);
+      const uint64_t dlo_off = (uint64_t)(((uint32_t)npl * plane) >> 4);  // hi -> lo operand (descriptor units)
+      constexpr uint64_t kKStep = (uint64_t)((2 * plane_bytes()) >> 4);   // one K-step = two planes
+      int b = 0, ph = 0, ch = 0, s = 0, g = 0;
+#pragma unroll 1
+      for (int q = 0; q < nstage; ++q) {
+        if (!TC_EXP(16)) mbar_wait_bounded(&a_full[b], (uint32_t)ph);
+        if (!TC_EXP(8)) fence_after();
+        if (lane == 0) TC_STAMP(3, q);
+        const uint32_t col = TC_EXP(2) ? 0u : (uint32_t)((g * kG) & (kRing - 1));
+        // B window: planes of chunk ch, starting at row kG - 1 - s of the reversed block
+        const uint64_t dh = sdesc(bhi + (uint32_t)(ch * (kWB / 4)) * plane + (uint32_t)(kG - 1 - s) * 16, plane, 128);
+        const uint64_t dl = dh + dlo_off;
+        const uint32_t ah = tbase + a_col0 + (uint32_t)(b * 2 * kWB), al = ah + kWB;
+        const uint32_t dcol = tbase + col;
+        const bool leader = elect_one();
+        if (!leader) {
+        } else if (col + kNWin <= (uint32_t)kRing) {
+          const uint32_t id = idesc_tf32(kNWin);
+#pragma unroll
+          for (int kk = 0; kk < kWB / 8; ++kk) {
+            mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
+            if (!TC_EXP(4)) {
+              mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
+              mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
+            }
+          }
+        } else {  // window wraps the ring: columns [col, kRing) and [0, kNWin - (kRing - col))
+          const uint32_t n1 = (uint32_t)kRing - col;
+          const uint32_t id1 = idesc_tf32((int)n1), id2 = idesc_tf32(kNWin - (int)n1);
+          const uint64_t o2 = (uint64_t)n1;  // n1 rows of 16 B, in descriptor units
+#pragma unroll
+          for (int kk = 0; kk < kWB / 8; ++kk) {
+            mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id1);
+            mma_ts(tbase, ah + kk * 8, dh + kk * kKStep + o2, id2);
+            if (!TC_EXP(4)) {
+              mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id1);
+              mma_ts(tbase, ah + kk * 8, dl + kk * kKStep + o2, id2);
+              mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id1);
+              mma_ts(tbase, al + kk * 8, dh + kk * kKStep + o2, id2);
+            }
+          }
+        }
+        if (leader) commit(&mma_done[b]);
+        __syncwarp();
+        if (lane == 0) TC_STAMP(4, q);
+        if (++b == kNBuf) { b = 0; ph ^= 1; }
+        if (++ch == nch) {
+          ch = 0;
+          if (++s == kG) { s = 0; ++g; }
+        }
+      }
+    }
+    __syncwarp();
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tbase));
+}
+
+// Template operand: for block (bi, bj) the reversed, zero-padded rows Rv[k] = A_C[i0 + K0 - k]
+// (K0 = kHB + kG - 2, zero outside the block / template), split into tf32 hi and fp32 lo, laid
+// out [2][WC/4 planes][kLB rows][4 floats] (the UMMA K-major no-swizzle canonical layout with
+// 16-byte rows).  grid = nblk, block = 256.
+__global__ void tm_tc_tpl_prep(const float* __restrict__ tplC, int tplP, int h, int w, int WC, int nbj,
+                               float* __restrict__ tcB) {
+  using namespace tc;
+  const int blk = blockIdx.x, bi = blk / nbj, bj = blk % nbj;
+  const int i0 = bi * kHB, j0 = bj * WC;
+  const int npl = WC / 4;
+  float* out = tcB + (int64_t)blk * (b_bytes(WC) / 4);
+  const int n = npl * kLB * 4;
+  for (int e = threadIdx.x; e < n; e += blockDim.x) {
+    const int c = e / (kLB * 4), k = (e / 4) % kLB, t = e % 4;
+    const int row = kHB + kG - 2 - k;
+    const int i = i0 + row, j = j0 + 4 * c + t;
+    const float val = (row >= 0 && row < kHB && i < h && j < w) ? tplC[(int64_t)i * tplP + j] : 0.0f;
+    const float hi = __uint_as_float(to_tf32(val));
+    out[e] = hi;
+    out[n + e] = val - hi;
+  }
+}
+
+// Sum the partial numerators of the template blocks in block order, normalise (or SSD),
+// optional surface store, per-frame argmax key.  grid = (Ub, batch), block = 256.
+__global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ part, int nblk, int64_t blk_stride,
+                                                    int64_t frame_stride, const double* __restrict__ S1,
+                                                    const double* __restrict__ S2, int64_t stat_frame_stride,
+                                                    const TemplateStats* tst, int h, int w, int V, int u_begin,
+                                                    float* scores, int64_t score_frame_stride,
+                                                    unsigned long long* keys, int ssd) {
+  __shared__ unsigned long long red[32];
+  const int ur = blockIdx.x, f = blockIdx.y;
+  const int u = u_begin + ur;
+  const TemplateStats ts = tst[0];
+  const double n = (double)h * (double)w;
+  const float* p = part + (int64_t)f * frame_stride + (int64_t)ur * V;
+  const int64_t so = (int64_t)f * stat_frame_stride + (int64_t)ur * V;
+  float* srow = scores ? scores + (int64_t)f * score_frame_stride + (int64_t)ur * V : nullptr;
+  unsigned long long best = 0ull;
+  for (int v = threadIdx.x; v < V; v += blockDim.x) {
+    float tot = 0.0f;
+    for (int b = 0; b < nblk; ++b) tot += __ldg(p + (int64_t)b * blk_stride + v);
+    const double s1 = S1[so + v], s2 = S2[so + v];
+    float sc;
+    if (ssd)
+      sc = (float)(ts.sumsq - 2.0 * ((double)tot + ts.sum / n * s1) + s2);
+    else
+      sc = ncc_normalize(tot, s1, s2, n, ts);
+    if (srow) srow[v] = sc;
+    const unsigned long long k = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
+    best = k > best ? k : best;
+  }
+  best = block_max_key(best, red);
+  if (threadIdx.x == 0 && best) atomicMax(keys + f, best);
+}
+
+}  // namespace nccb

@@ -250,3 +250,21 @@ def test_c_example_runs_end_to_end(tmp_path):
                            "-o", str(exe), "-L", libdir, "-lncc_b200", "-Wl,-rpath," + libdir])
     r = subprocess.run([str(exe)], capture_output=True, text=True, timeout=300)
     assert r.returncode == 0, r.stdout + r.stderr
+
+
+@pytest.mark.parametrize("h,w", [(128, 128), (37, 300), (9, 5)])
+def test_window_sum_forms_agree(h, w, monkeypatch):
+    """Fused single-pass window sums vs the two-pass (row sums, column scan) form: bitwise equal
+    scores on 2^-8-quantised inputs (every fp64 partial sum is exact there), and both within
+    the oracle tolerance."""
+    g = synth.rng(70 + h)
+    img = synth.quantize(synth.uniform_image(300, 420, 71 + w))
+    u, v = int(g.integers(0, 300 - h + 1)), int(g.integers(0, 420 - w + 1))
+    T = np.ascontiguousarray(img[u:u + h, v:v + w])
+    _, fused, info = run_match(img, T)
+    monkeypatch.setenv("NCC_BOX_TWO_PASS", "1")
+    _, two, info2 = run_match(img, T)
+    assert info2["launches_per_call"] == info["launches_per_call"] + 1
+    np.testing.assert_array_equal(fused, two)
+    ref = oracle.ncc_surface(img, T)
+    assert np.max(np.abs(fused[0] - ref)) <= TOL

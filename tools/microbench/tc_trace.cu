@@ -1,0 +1,77 @@
+// Per-stage timeline of tm_tc_kernel (CTA 0) on a cfg2-shaped problem (1024^2 image, 128^2
+// template, WC = 32, 4 segments): clock64 stamps of the producer (after the mma_done wait,
+// after the tf32 split, after the TMEM stores) and of the MMA issuer (after the a_full wait,
+// after the commit).  nvcc -gencode arch=compute_100a,code=sm_100a -O3 -DNCC_TC_TRACE
+//   -I../../paper_conf_ipps_moorelk13_b200/csrc -o tc_trace tc_trace.cu -lcuda
+#include <cstdio>
+#include <vector>
+#include <cuda.h>
+#include "ncc_tc.cuh"
+
+int main(int argc, char** argv) {
+  using namespace nccb;
+  const int H = 1024, W = 1024, h = 128, w = 128, U = H - h + 1, V = W - w + 1;
+  const int WC = argc > 1 ? atoi(argv[1]) : 32, nseg = argc > 2 ? atoi(argv[2]) : 4;
+  const int exp = argc > 3 ? atoi(argv[3]) : 0;
+  cudaMemcpyToSymbol(g_tc_exp, &exp, sizeof(exp));
+  const int nbi = 1, nbj = (w + WC - 1) / WC, vtiles = (V + 127) / 128;
+  float *img, *tcB, *part;
+  long long* tr;
+  cudaMalloc(&img, (size_t)H * W * 4);
+  cudaMemset(img, 0, (size_t)H * W * 4);
+  cudaMalloc(&tcB, (size_t)nbi * nbj * tc::b_bytes(WC));
+  cudaMemset(tcB, 0, (size_t)nbi * nbj * tc::b_bytes(WC));
+  cudaMalloc(&part, (size_t)nbi * nbj * U * V * 4);
+  cudaMalloc(&tr, 8 * 1024 * 8);
+  cudaMemset(tr, 0, 8 * 1024 * 8);
+  cudaMemcpyToSymbol(g_tc_trace, &tr, sizeof(tr));
+  TcArgs a{};
+  a.img = img; a.pitch = W; a.frame_stride = (int64_t)H * W; a.H = H; a.W = W;
+  a.tcB = tcB; a.WC = WC; a.nbi = nbi; a.nbj = nbj; a.V = V; a.u_begin = 0; a.u_end = U;
+  a.useg = (U + nseg - 1) / nseg; a.nseg = nseg; a.vtiles = vtiles; a.part = part;
+  a.part_frame_stride = (int64_t)U * V; a.part_blk_stride = a.part_frame_stride;
+  const int smem = tc::smem_bytes(WC);
+  cudaFuncSetAttribute(tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  dim3 grid(nbi * nbj * vtiles * nseg, 1);
+  CUtensorMap map;
+  cuuint64_t gd[3] = {(cuuint64_t)W, (cuuint64_t)H, 1}, gs[2] = {(cuuint64_t)W * 4, (cuuint64_t)H * W * 4};
+  cuuint32_t bx[3] = {(cuuint32_t)tc::kBoxW, 1, 1}, es[3] = {1, 1, 1};
+  CUresult cr = cuTensorMapEncodeTiled(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, img, gd, gs, bx, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                                       CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (cr != CUDA_SUCCESS) { printf("encode failed %d\n", (int)cr); return 1; }
+  for (int it = 0; it < 3; ++it) tm_tc_kernel<<<grid, tc::kThreads, smem>>>(a, map);
+  cudaEvent_t e0, e1;
+  cudaEventCreate(&e0); cudaEventCreate(&e1);
+  cudaEventRecord(e0);
+  tm_tc_kernel<<<grid, tc::kThreads, smem>>>(a, map);
+  cudaEventRecord(e1);
+  cudaError_t e = cudaDeviceSynchronize();
+  float ms = 0; cudaEventElapsedTime(&ms, e0, e1);
+  std::vector<long long> t(8 * 1024);
+  cudaMemcpy(t.data(), tr, t.size() * 8, cudaMemcpyDeviceToHost);
+  printf("{\"err\": \"%s\", \"exp\": %d, \"ms\": %.4f, \"grid\": %d}\n", cudaGetErrorString(e), exp, ms, grid.x);
+  const long long t0 = t[3 * 1024];
+  for (int q = 100; q < 104; ++q)
+    printf("q=%3d  img_full_ok=%8lld  lds_done=%8lld  issue_done=%8lld\n", q, t[5 * 1024 + q] - t0, t[6 * 1024 + q] - t0,
+           t[7 * 1024 + q] - t0);
+  for (int q = 100; q < 104; ++q)
+    printf("q=%3d  prod_wait_done(q)=%8lld  prod_split(q)=%8lld  prod_arrive(q)=%8lld  mma_go(q)=%8lld  mma_commit(q)=%8lld\n", q,
+           t[q] - t0, t[1024 + q] - t0, t[2048 + q] - t0, t[3072 + q] - t0, t[4096 + q] - t0);
+  // steady-state averages over stages 40..300
+  double d_go = 0, d_arr = 0, d_done = 0;
+  for (int q = 41; q < 300; ++q) {
+    d_go += t[3072 + q] - t[3072 + q - 1];
+    d_arr += t[2048 + q] - t[2048 + q - 1];
+    d_done += t[q] - t[q - 1];
+  }
+  printf("avg cycles/stage: mma_go %.1f  prod_arrive %.1f  mma_done %.1f\n", d_go / 259, d_arr / 259, d_done / 259);
+  double lag = 0, split = 0, stw = 0;
+  for (int q = 41; q < 300; ++q) {
+    lag += t[3072 + q] - t[2048 + q];       // arrive -> MMA thread sees it
+    split += t[1024 + q] - t[q - 4 >= 0 ? q - 4 : 0];
+    stw += t[2048 + q] - t[1024 + q];       // LDG issue + TMEM stores + wait
+  }
+  printf("avg: arrive->mma_go %.1f  split->arrive %.1f\n", lag / 259, stw / 259);
+  return 0;
+}
