@@ -344,9 +344,26 @@ def main():
     flops = plan.info.flops_per_call
     achieved = flops / (num_avg / 1e3) / 1e12
     max_mhz = clocks.get("sm_max_mhz") or 1965.0
-    peak = sms * 128 * 2 * max_mhz * 1e6 / 1e12
     sm_mhz = clocks.get("sm_mhz")
-    peak_at_clock = sms * 128 * 2 * sm_mhz * 1e6 / 1e12 if sm_mhz else None
+    tensor = plan.info.variant_name.decode().startswith("tm_tc")
+    if tensor:
+        # 3xTF32 on tcgen05: 3 tf32 MMAs per fp32 MAC.  tf32 peak = measured bf16 GEMM peak x the
+        # nominal tf32/bf16 ratio (1.1 / 2.25 PFLOP/s, B200_PROFILING.md); the fp32-equivalent
+        # peak of the method is a third of it.
+        mp = {}
+        try:
+            mp = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+        except Exception:
+            pass
+        bf16 = mp.get("bf16_tflops") or 1590.0
+        peak = bf16 * (1.1 / 2.25) / 3.0
+        peak_note = (f"3xTF32 fp32-equivalent tensor peak = {'measured' if mp else 'fallback'} bf16 GEMM "
+                     f"{bf16:.1f} TFLOP/s x (tf32/bf16 nominal 1.1/2.25) / 3 MMAs per MAC")
+        peak_at_clock = peak * sm_mhz / max_mhz if sm_mhz else None
+    else:
+        peak = sms * 128 * 2 * max_mhz * 1e6 / 1e12
+        peak_note = "FP32 FFMA peak = SMs x 128 lanes x 2 FLOP x max SM clock (derived; MEASURED_PEAKS.json has no FP32 figure)"
+        peak_at_clock = sms * 128 * 2 * sm_mhz * 1e6 / 1e12 if sm_mhz else None
 
     # ---- end-to-end through the host-buffer C-ABI call (H2D + compute + D2H in the region)
     e2e = None
@@ -369,7 +386,7 @@ def main():
     if os.path.exists(prof):
         try:
             tj = json.load(open(prof))
-            traffic = tj.get(f"cfg{cfg}")
+            traffic = tj.get(f"cfg{cfg}_tc" if tensor else f"cfg{cfg}")
             if traffic is None and f"cfg{cfg}_per_pair" in tj:
                 traffic = tj[f"cfg{cfg}_per_pair"] * plan.info.grid_z
         except Exception:
@@ -383,10 +400,8 @@ def main():
                        "units_per_step_per_gpu": units_per_step, "l2": "flushed between steps (512 MiB write)",
                        "variant": plan.info.variant_name.decode(), "regs_per_thread": plan.info.regs_per_thread,
                        "parallelism": f"replicas{ws}" if wl["kind"] == "tm" else f"pairs/{ws}"},
-            "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                         "frac": achieved / peak, "traffic": traffic,
-                         "peak_note": "FP32 FFMA peak = SMs x 128 lanes x 2 FLOP x max SM clock "
-                                      "(derived; MEASURED_PEAKS.json has no FP32 figure)",
+            "roofline": {"bound": "tensor" if tensor else "alu", "achieved": achieved, "peak": peak,
+                         "unit": "TFLOP/s", "frac": achieved / peak, "traffic": traffic, "peak_note": peak_note,
                          "frac_at_sampled_clock": (achieved / peak_at_clock) if peak_at_clock else None,
                          "kernel_ms": num_avg, "kernel_share_of_step": num_avg / (total_ms / args.steps)},
             "clocks": clocks, "e2e": e2e, "gpu_launches": launches_per_step * args.steps,

@@ -65,7 +65,8 @@ enum {
     NCC_F_WRITE_SURFACE = 1u,  /* TM: ncc_match writes the score surface (d_scores required) */
     NCC_F_GENERIC_KERNEL = 2u, /* force the run-time-evaluated (RE) generic kernels         */
     NCC_F_NO_JIT = 4u,         /* reserved: never compile at run time                        */
-    NCC_F_TIMING = 8u          /* record per-stage CUDA-event timings (ncc_plan_timing)     */
+    NCC_F_TIMING = 8u,         /* record per-stage CUDA-event timings (ncc_plan_timing)     */
+    NCC_F_CUDA_CORES = 16u     /* TM: never use the tensor-core (tcgen05 3xTF32) numerator   */
 };
 
 /* Output flag bits (ncc_peak.flags, piv_vector.flags). */

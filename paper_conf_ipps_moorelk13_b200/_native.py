@@ -21,7 +21,7 @@ STATUS = {0: "NCC_OK", 1: "NCC_ERR_INVALID_ARGUMENT", 2: "NCC_ERR_UNSUPPORTED", 
 NCC_MODE_MATCH, NCC_MODE_PIV = 0, 1
 NCC_SCORE_NCC, NCC_SCORE_SSD = 0, 1
 NCC_SUBPIX_GAUSS3, NCC_SUBPIX_PARABOLA3, NCC_SUBPIX_NONE = 0, 1, 2
-NCC_F_WRITE_SURFACE, NCC_F_GENERIC_KERNEL, NCC_F_NO_JIT, NCC_F_TIMING = 1, 2, 4, 8
+NCC_F_WRITE_SURFACE, NCC_F_GENERIC_KERNEL, NCC_F_NO_JIT, NCC_F_TIMING, NCC_F_CUDA_CORES = 1, 2, 4, 8, 16
 FLAG_FLAT_TEMPLATE, FLAG_EDGE_Y, FLAG_EDGE_X, FLAG_PARABOLA_Y, FLAG_PARABOLA_X, FLAG_INVALID = 1, 2, 4, 8, 16, 32
 
 EXPORTS = ["ncc_plan_create", "ncc_match", "ncc_match_rois", "piv_correlate", "piv_correlate_ex", "ncc_match_host",

@@ -60,10 +60,12 @@ class MatchPlan(_Plan):
     """Template matching: corr2 at every valid offset of each frame (Listing 5.1)."""
 
     def __init__(self, H, W, h, w, batch=1, device=0, shard_rank=0, shard_count=1, write_surface=False,
-                 generic=False, timing=False, image_pitch=None, score=N.NCC_SCORE_NCC, n_templates=0, roi=None):
-        """roi=(roi_h, roi_w) with n_templates >= 1 selects ROI mode (match_rois)."""
+                 generic=False, timing=False, image_pitch=None, score=N.NCC_SCORE_NCC, n_templates=0, roi=None,
+                 cuda_cores=False):
+        """roi=(roi_h, roi_w) with n_templates >= 1 selects ROI mode (match_rois); cuda_cores=True never
+        uses the tensor-core numerator (the library picks it by a cost model otherwise)."""
         flags = (N.NCC_F_WRITE_SURFACE if write_surface else 0) | (N.NCC_F_GENERIC_KERNEL if generic else 0) | \
-                (N.NCC_F_TIMING if timing else 0)
+                (N.NCC_F_TIMING if timing else 0) | (N.NCC_F_CUDA_CORES if cuda_cores else 0)
         rh, rw = roi if roi is not None else (0, 0)
         super().__init__(N.make_problem(N.NCC_MODE_MATCH, H, W, image_pitch, h, w, batch=batch,
                                         shard_rank=shard_rank, shard_count=shard_count, flags=flags,

@@ -426,8 +426,12 @@ ncc_status setup_box(ncc_plan pl, int w) {
 ncc_status setup_tc(ncc_plan pl) {
   const ncc_problem& p = pl->p;
   pl->tc = 0;
+  // NCC_TC=0 / NCC_F_CUDA_CORES / generic plans: CUDA-core path; NCC_TC=1: tensor cores whenever
+  // eligible; default: the cost model below (tensor cores when clearly faster).
   const char* env = getenv("NCC_TC");
-  if (!env || atoi(env) == 0 || pl->roi_mode || pl->n_tmpl != 1) return NCC_OK;
+  const int mode = env ? atoi(env) : -1;
+  if (mode == 0 || (p.flags & (NCC_F_CUDA_CORES | NCC_F_GENERIC_KERNEL)) || pl->roi_mode || pl->n_tmpl != 1)
+    return NCC_OK;
   const int h = p.tmpl_h, w = p.tmpl_w;
   pl->tc_vtiles = ceil_div(pl->V, 128);
   pl->tc_nbi = ceil_div(h, tc::kHB);
@@ -450,6 +454,11 @@ ncc_status setup_tc(ncc_plan pl) {
     }
     if (wc >= w) break;
   }
+  // measured B200 rates: ~1170 cycles per tensor-core stage (12 MMAs of 128 x 136 x 8, 3xTF32),
+  // ~95 useful FP32 MACs per cycle per SM on the CUDA-core path
+  const double tc_cycles = best * 1170.0;
+  const double cc_cycles = (double)h * w * (double)pl->Ub * pl->V * p.batch / (95.0 * pl->nsm);
+  if (mode < 0 && !(tc_cycles < 0.8 * cc_cycles)) return NCC_OK;
   const int nblk = pl->tc_nbi * pl->tc_nbj;
   ncc_status st;
   if ((st = dalloc(&pl->tcB, (size_t)nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;

@@ -25,7 +25,17 @@ def _lib():
 
 @pytest.fixture(autouse=True)
 def _tc(monkeypatch):
-    monkeypatch.setenv("NCC_TC", "1")
+    monkeypatch.setenv("NCC_TC", "1")  # tensor cores whenever eligible (the default picks by cost)
+
+
+def test_tc_is_default_for_cfg2_and_not_for_small_templates(monkeypatch):
+    monkeypatch.delenv("NCC_TC")
+    with MatchPlan(1024, 1024, 128, 128) as plan:
+        assert plan.info.variant_name.decode().startswith("tm_tc")
+    with MatchPlan(1024, 1024, 128, 128, cuda_cores=True) as plan:
+        assert not plan.info.variant_name.decode().startswith("tm_tc")
+    with MatchPlan(64, 64, 16, 16) as plan:
+        assert not plan.info.variant_name.decode().startswith("tm_tc")
 
 
 def run(imgs, T, shard=(0, 1), score=N.NCC_SCORE_NCC):

@@ -31,7 +31,7 @@ def run_match(img, T, generic=False, batch_imgs=None, shard=(0, 1)):
     h, w = T.shape
     dev = torch.device("cuda", 0)
     with MatchPlan(H, W, h, w, batch=imgs.shape[0], write_surface=True, generic=generic,
-                   shard_rank=shard[0], shard_count=shard[1]) as plan:
+                   shard_rank=shard[0], shard_count=shard[1], cuda_cores=True) as plan:
         d_img = torch.from_numpy(imgs).to(dev)
         d_t = torch.from_numpy(np.ascontiguousarray(T)).to(dev)
         peaks, scores = plan.match(d_img, d_t)
@@ -119,7 +119,7 @@ def test_batch_frames_and_host_path():
     stack = torch.from_numpy(np.stack(imgs)).pin_memory()
     tt = torch.from_numpy(T).pin_memory()
     hp = torch.empty((3, 4), dtype=torch.int32).pin_memory()
-    with MatchPlan(200, 180, 24, 20, batch=3) as plan:
+    with MatchPlan(200, 180, 24, 20, batch=3, cuda_cores=True) as plan:
         plan.match_host(stack, tt, hp)
         torch.cuda.synchronize()
     d = decode_peaks(hp)
@@ -190,7 +190,7 @@ def test_unaligned_pitch_uses_plain_loads():
     buf = np.zeros((H, P), np.float32)
     buf[:, :W] = img
     dev = torch.device("cuda", 0)
-    with MatchPlan(H, W, 16, 16, write_surface=True, image_pitch=P) as plan:
+    with MatchPlan(H, W, 16, 16, write_surface=True, image_pitch=P, cuda_cores=True) as plan:
         peaks, s = plan.match(torch.from_numpy(buf).to(dev), torch.from_numpy(T).to(dev))
         torch.cuda.synchronize()
     ref, pk = oracle.ncc_match(img, T)
@@ -211,9 +211,11 @@ def test_cfg2_split_k_bands_bitwise():
     np.testing.assert_array_equal(np.concatenate(parts, axis=0), full[0])
 
 
-def test_concurrent_plans_on_two_streams():
+@pytest.mark.parametrize("cuda_cores", [True, False])
+def test_concurrent_plans_on_two_streams(cuda_cores):
     """Two TM plans with different templates on two streams: the shared constant-bank
-    template slot is ordered by the library, both results stay exact."""
+    template slot (CUDA-core path) is ordered by the library; tensor-core plans own their
+    scratch; both results stay exact."""
     dev = torch.device("cuda", 0)
     imgs, Ts, refs = [], [], []
     for k in range(2):
@@ -222,7 +224,7 @@ def test_concurrent_plans_on_two_streams():
         Ts.append(torch.from_numpy(T).to(dev))
         refs.append((u0, v0))
     streams = [torch.cuda.Stream(dev), torch.cuda.Stream(dev)]
-    plans = [MatchPlan(1024, 1024, 128, 128) for _ in range(2)]
+    plans = [MatchPlan(1024, 1024, 128, 128, cuda_cores=cuda_cores) for _ in range(2)]
     try:
         outs = []
         for _ in range(3):

@@ -20,7 +20,10 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "sm__throughput.avg.pct_of_peak_sustained_elapsed", "sm__warps_active.avg.pct_of_peak_sustained_active",
         "smsp__issue_active.avg.pct_of_peak_sustained_active", "sm__cycles_active.avg", "gpc__cycles_elapsed.max",
         "l1tex__data_bank_conflicts_pipe_lsu_mem_shared_op_ld.sum",
-        "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum"]
+        "l1tex__data_pipe_lsu_wavefronts_mem_shared_op_ld.sum",
+        "sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
+        "sm__mem_tensor_cycles_active.avg.pct_of_peak_sustained_active",
+        "sm__inst_executed_pipe_uniform.avg.pct_of_peak_sustained_active"]
 
 
 def full(rep, out):
