@@ -408,7 +408,11 @@ ncc_status setup_box(ncc_plan pl, int w) {
   int maxsm = 0;
   NCC_CUDA(cudaDeviceGetAttribute(&maxsm, cudaDevAttrMaxSharedMemoryPerBlockOptin, pl->device));
   NCC_CUDA(cudaDeviceGetAttribute(&pl->nsm, cudaDevAttrMultiProcessorCount, pl->device));
-  pl->box_iwp = kBoxTV + w - 1;
+  {  // padded row: 32 chunks of L (power of two) columns + one pad double per chunk
+    int L = 1;
+    while (32 * L < kBoxTV + w - 1) L *= 2;
+    pl->box_iwp = 32 * L + 32;
+  }
   const int64_t r = ((int64_t)maxsm / 8 - 2 * pl->box_iwp) / (2 * pl->box_iwp);
   pl->box_r = r > 16 ? 16 : (int)r;
   pl->box_smem = 0;
@@ -804,10 +808,10 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
   const ncc_problem& p = pl->p;
   const int h = p.tmpl_h, w = p.tmpl_w;
   const int V = p.image_w - w + 1;
-  if (pl->box_smem) {  // fused single pass; rows per CTA halved until the grid fills the GPU twice
+  if (pl->box_smem) {  // fused single pass; rows per CTA halved until the grid covers every SM
     const int gx = ceil_div(V, kBoxTV);
     int TU = 64;
-    while (TU > pl->box_r && (int64_t)gx * ceil_div(rows_out, TU) * batch < 2 * pl->nsm) TU /= 2;
+    while (TU > pl->box_r && (int64_t)gx * ceil_div(rows_out, TU) * batch < pl->nsm) TU /= 2;
     dim3 g(gx, ceil_div(rows_out, TU), batch);
     box2d_kernel<kBox2dNT><<<g, kBox2dNT, pl->box_smem, s>>>(frames, p.image_pitch,
                                                             (int64_t)p.image_h * p.image_pitch, row0, h, w, V,

@@ -691,6 +691,12 @@ __global__ void __launch_bounds__(NT)
   const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + ub) * pitch + v0;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   constexpr int NW = NT / 32;
+  // row layout for the blocked scan: lane k owns the L consecutive columns [k L, k L + L), stored
+  // with one pad double per chunk (index c + c / L) so the 32 lanes hit distinct bank pairs
+  int lsh = 0;
+  while ((32 << lsh) < iw) ++lsh;
+  const int L = 1 << lsh;
+  auto pidx = [&](int c) { return c + (c >> lsh); };
   for (int r0 = 0; r0 < nrow; r0 += R) {
     const int nr = min(R, nrow - r0);
     for (int c = threadIdx.x; c < iw; c += NT) {
@@ -700,14 +706,18 @@ __global__ void __launch_bounds__(NT)
       if (r0 == 0) {  // first output row of the CTA: direct column sum (independent loads)
         double a[4] = {0.0, 0.0, 0.0, 0.0}, b[4] = {0.0, 0.0, 0.0, 0.0};
         int i = 0;
-        for (; i + 4 <= h; i += 4) {
+        for (; i + 32 <= h; i += 32) {  // 32 loads in flight, then 4 accumulator chains
+          float xs[32];
 #pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            const double x = __ldg(col + (int64_t)(i + k) * pitch);
-            a[k] += x;
-            b[k] = fma(x, x, b[k]);
+          for (int k = 0; k < 32; ++k) xs[k] = __ldg(col + (int64_t)(i + k) * pitch);
+#pragma unroll
+          for (int k = 0; k < 32; ++k) {
+            const double x = xs[k];
+            a[k & 3] += x;
+            b[k & 3] = fma(x, x, b[k & 3]);
           }
         }
+#pragma unroll 8
         for (; i < h; ++i) {
           const double x = __ldg(col + (int64_t)i * pitch);
           a[0] += x;
@@ -715,21 +725,22 @@ __global__ void __launch_bounds__(NT)
         }
         c1 = (a[0] + a[1]) + (a[2] + a[3]);
         c2 = (b[0] + b[1]) + (b[2] + b[3]);
-        X1[c] = c1;
-        X2[c] = c2;
+        X1[pidx(c)] = c1;
+        X2[pidx(c)] = c2;
         r = 1;
       } else {
         c1 = C1[c];
         c2 = C2[c];
       }
+#pragma unroll 4
       for (; r < nr; ++r) {  // slide down one row: + entering row, - leaving row
         const int u = r0 + r;
         const double xi = __ldg(col + (int64_t)(u + h - 1) * pitch);
         const double xo = __ldg(col + (int64_t)(u - 1) * pitch);
         c1 = (c1 + xi) - xo;
         c2 = fma(-xo, xo, fma(xi, xi, c2));
-        X1[(int64_t)r * IWP + c] = c1;
-        X2[(int64_t)r * IWP + c] = c2;
+        X1[(int64_t)r * IWP + pidx(c)] = c1;
+        X2[(int64_t)r * IWP + pidx(c)] = c2;
       }
       C1[c] = c1;
       C2[c] = c2;
@@ -738,21 +749,25 @@ __global__ void __launch_bounds__(NT)
     for (int r = wid; r < nr; r += NW) {
       double* x1 = X1 + (int64_t)r * IWP;
       double* x2 = X2 + (int64_t)r * IWP;
-      double k1 = 0.0, k2 = 0.0;
-      for (int c0 = 0; c0 < iw; c0 += 32) {
-        const int c = c0 + lane;
-        double p1 = c < iw ? x1[c] : 0.0, p2 = c < iw ? x2[c] : 0.0;
-        p1 = warp_incl_scan_d(p1) + k1;
-        p2 = warp_incl_scan_d(p2) + k2;
-        if (c < iw) { x1[c] = p1; x2[c] = p2; }
-        k1 = __shfl_sync(0xffffffffu, p1, 31);
-        k2 = __shfl_sync(0xffffffffu, p2, 31);
+      // blocked inclusive prefix: chunk totals, warp scan of the totals, chunk prefixes
+      const int cb = lane * L, ce = min(cb + L, iw);
+      double t1 = 0.0, t2 = 0.0;
+      for (int c = cb; c < ce; ++c) {
+        t1 += x1[pidx(c)];
+        t2 += x2[pidx(c)];
+      }
+      double p1 = warp_incl_scan_d(t1) - t1, p2 = warp_incl_scan_d(t2) - t2;
+      for (int c = cb; c < ce; ++c) {
+        p1 += x1[pidx(c)];
+        p2 += x2[pidx(c)];
+        x1[pidx(c)] = p1;
+        x2[pidx(c)] = p2;
       }
       __syncwarp();
       const int64_t o = (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
       for (int v = lane; v < tv; v += 32) {
-        S1[o + v] = x1[v + w - 1] - (v > 0 ? x1[v - 1] : 0.0);
-        S2[o + v] = x2[v + w - 1] - (v > 0 ? x2[v - 1] : 0.0);
+        S1[o + v] = x1[pidx(v + w - 1)] - (v > 0 ? x1[pidx(v - 1)] : 0.0);
+        S2[o + v] = x2[pidx(v + w - 1)] - (v > 0 ? x2[pidx(v - 1)] : 0.0);
       }
     }
     __syncthreads();

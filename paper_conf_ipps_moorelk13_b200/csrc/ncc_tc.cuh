@@ -367,7 +367,9 @@ __global__ void tm_tc_tpl_prep(const float* __restrict__ tplC, int tplP, int h, 
 }
 
 // Sum the partial numerators of the template blocks in block order, normalise (or SSD),
-// optional surface store, per-frame argmax key.  grid = (Ub, batch), block = 256.
+// optional surface store, per-frame argmax key.  grid = (Ub, batch), block = 256; each thread
+// takes kFinV columns with all their loads issued first (the kernel is load-latency bound).
+constexpr int kFinV = 4;
 __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ part, int nblk, int64_t blk_stride,
                                                     int64_t frame_stride, const double* __restrict__ S1,
                                                     const double* __restrict__ S2, int64_t stat_frame_stride,
@@ -378,23 +380,45 @@ __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ pa
   const int ur = blockIdx.x, f = blockIdx.y;
   const int u = u_begin + ur;
   const TemplateStats ts = tst[0];
-  const double n = (double)h * (double)w;
+  const double inv_n = 1.0 / ((double)h * (double)w);
   const float* p = part + (int64_t)f * frame_stride + (int64_t)ur * V;
   const int64_t so = (int64_t)f * stat_frame_stride + (int64_t)ur * V;
   float* srow = scores ? scores + (int64_t)f * score_frame_stride + (int64_t)ur * V : nullptr;
   unsigned long long best = 0ull;
-  for (int v = threadIdx.x; v < V; v += blockDim.x) {
-    float tot = 0.0f;
-    for (int b = 0; b < nblk; ++b) tot += __ldg(p + (int64_t)b * blk_stride + v);
-    const double s1 = S1[so + v], s2 = S2[so + v];
+  for (int v0 = threadIdx.x; v0 < V; v0 += blockDim.x * kFinV) {
+    float tot[kFinV];
+    double s1v[kFinV], s2v[kFinV];
+#pragma unroll
+    for (int k = 0; k < kFinV; ++k) {
+      const int v = v0 + k * blockDim.x;
+      tot[k] = 0.0f;
+      s1v[k] = s2v[k] = 0.0;
+      if (v < V) {
+        s1v[k] = __ldg(S1 + so + v);
+        s2v[k] = __ldg(S2 + so + v);
+      }
+    }
+    for (int b = 0; b < nblk; ++b) {
+#pragma unroll
+      for (int k = 0; k < kFinV; ++k) {
+        const int v = v0 + k * blockDim.x;
+        if (v < V) tot[k] += __ldg(p + (int64_t)b * blk_stride + v);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < kFinV; ++k) {
+    const int v = v0 + k * blockDim.x;
+    if (v >= V) break;
+    const double s1 = s1v[k], s2 = s2v[k];
     float sc;
     if (ssd)
-      sc = (float)(ts.sumsq - 2.0 * ((double)tot + ts.sum / n * s1) + s2);
-    else
-      sc = ncc_normalize(tot, s1, s2, n, ts);
+      sc = (float)(ts.sumsq - 2.0 * ((double)tot[k] + ts.sum * inv_n * s1) + s2);
+    else  // fp64 variance, fp32 rsqrt: |error| <= ~4e-7 (the fp64 divide/sqrt dominated this kernel)
+      sc = ncc_normalize_fast(tot[k], s1, s2, inv_n, ts.csum, ts.energy, ts.flat != 0);
     if (srow) srow[v] = sc;
-    const unsigned long long k = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
-    best = k > best ? k : best;
+    const unsigned long long key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
+    best = key > best ? key : best;
+    }
   }
   best = block_max_key(best, red);
   if (threadIdx.x == 0 && best) atomicMax(keys + f, best);
