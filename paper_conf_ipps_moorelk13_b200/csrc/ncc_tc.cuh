@@ -82,15 +82,26 @@ __device__ __forceinline__ uint32_t to_tf32(float x) {
 constexpr int kHB = 128;   // template rows per block (B window rows N = kHB + kG)
 constexpr int kG = 8;      // image rows per group (ring advance, drain granularity)
 constexpr int kWB = 32;    // template columns per TMEM A chunk (4 MMAs of K = 8)
-constexpr int kRing = 256; // TMEM accumulator ring columns
-constexpr int kNBuf = 4;   // TMEM A stages (columns kRing + b*2*kWB .. ; 256 + 4*64 = 512)
+constexpr int kRing = 320; // TMEM accumulator columns (sliding window of output rows)
+constexpr int kNBuf = 3;   // TMEM A stages (columns kRing + b*2*kWB .. ; 320 + 3*64 = 512)
 static_assert(kRing + kNBuf * 2 * kWB <= 512, "TMEM columns");
 constexpr int kNWin = kHB + kG;
+// The window of group g starts at column (kG g) mod kRelocAt: when it would run past kRing the
+// kHB live columns [kRelocAt, kRelocAt + kHB) are moved to [0, kHB) (relocation warps), so every
+// MMA covers one contiguous run of columns (no ring-wrap split into two MMAs).
+constexpr int kRelocAt = ((kRing - kNWin) / kG + 1) * kG;
+static_assert(kRelocAt + kHB == kRing && kRelocAt >= kNWin, "relocation geometry");
 constexpr int kLB = ((kHB + 2 * kG - 1 + 7) / 8) * 8;  // rows of the reversed template block
 constexpr int kGroups = kNBuf;                           // producer groups of 4 warps; group g: stages q = g mod kNBuf
-constexpr int kThreads = kGroups * 128 + 32;             // + 1 MMA warp
+// warp roles: producers 0 .. 4 kGroups - 1, relocation 4 kGroups .. + 3, TMA, then the MMA warp
+// LAST: the SMSP arbiter issues highest-warp-id-first, and every cycle the MMA warp waits to issue
+// is a cycle the tensor pipe idles (its queue is about one MMA deep).
+constexpr int kRelocWarp0 = 4 * kGroups;
+constexpr int kTmaWarp = kRelocWarp0 + 4;
+constexpr int kMmaWarp = kTmaWarp + 1;
+constexpr int kThreads = kGroups * 128 + 32 + 128 + 32;
 constexpr int kBoxW = 128 + kWB;                         // image-row segment of one stage (TMA box)
-constexpr int kNImg = 8;                                 // image-row ring (TMA issue distance)
+constexpr int kNImg = 9;                                 // image-row ring (TMA issue distance)
 static_assert(kNImg % kNBuf == 0, "a stage and the stage kNImg later belong to the same producer group");
 // shared bytes of the template operand for a column super-block of WC columns (hi + lo)
 __host__ __device__ constexpr uint32_t plane_bytes() { return kLB * 16; }
@@ -134,7 +145,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
                                                                   const __grid_constant__ CUtensorMap map_img) {
   using namespace tc;
   extern __shared__ __align__(1024) unsigned char smem_tc[];
-  __shared__ __align__(8) uint64_t a_full[kNBuf], mma_done[kNBuf], img_full[kNImg], img_empty[kNImg];
+  __shared__ __align__(8) uint64_t a_full[kNBuf], mma_done[kNBuf], img_full[kNImg], img_empty[kNImg], reloc_req,
+      reloc_done;
   __shared__ uint32_t tmem_base_s;
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -177,6 +189,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       mbar_init(&img_full[b], 1);
       mbar_init(&img_empty[b], 128);
     }
+    mbar_init(&reloc_req, 1);
+    mbar_init(&reloc_done, 128);
     fence_mbar_init();
   }
   fence_before();
@@ -185,6 +199,22 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   const uint32_t tbase = tmem_base_s;
   const uint32_t a_col0 = kRing;  // A buffers: [kRing + b*2*kWB, +kWB) hi, [+kWB, +2kWB) lo
 
+  // stage q = (image row rr, column chunk ch): row ua + i0 + rr, columns v0 + j0 + 32 ch + [0, kBoxW)
+  auto stage_zero = [&](int q) {  // rows past the image / chunks past its width: zero operand
+    return ua + i0 + q / nch >= a.H || v0 + j0 + (q % nch) * kWB >= a.W;
+  };
+  auto issue = [&](int q) {  // one thread: TMA of stage q into ring slot q % kNImg
+    const int sl = q % kNImg;
+    if (q >= kNImg) mbar_wait_bounded(&img_empty[sl], (uint32_t)(((q - kNImg) / kNImg) & 1));
+    if (stage_zero(q)) {
+      mbar_arrive(&img_full[sl]);
+    } else {
+      mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 4));
+      tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 4, &map_img, v0 + j0 + (q % nch) * kWB, ua + i0 + q / nch,
+                  f, &img_full[sl]);
+    }
+  };
+  const int nreloc = (ngrp - 1) / (kRelocAt / kG);  // groups g > 0 whose window restarts at column 0
   if (warp < 4 * kGroups) {
     // ===================== producers (lane v = output column v0 + v) and ring drain.
     // Group grp (warps 4 grp .. 4 grp + 3, TMEM lane quadrants 0..3) handles the stages
@@ -201,37 +231,18 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       fence_before();
     }
     const float* ring = reinterpret_cast<const float*>(smem_tc + img_off(a.WC));
-    // stage q = (image row rr, column chunk ch): row ua + i0 + rr, columns v0 + j0 + 32 ch + [0, kBoxW)
-    auto stage_zero = [&](int q) {  // rows past the image / chunks past its width: zero operand
-      return ua + i0 + q / nch >= a.H || v0 + j0 + (q % nch) * kWB >= a.W;
-    };
-    auto issue = [&](int q) {  // one thread: TMA of stage q into ring slot q % kNImg
-      const int sl = q % kNImg;
-      if (q >= kNImg) mbar_wait_bounded(&img_empty[sl], (uint32_t)(((q - kNImg) / kNImg) & 1));
-      if (stage_zero(q)) {
-        mbar_arrive(&img_full[sl]);
-      } else {
-        mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 4));
-        tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 4, &map_img, v0 + j0 + (q % nch) * kWB, ua + i0 + q / nch,
-                    f, &img_full[sl]);
-      }
-    };
-    if (tid == 0) {
-      tma_prefetch_desc(&map_img);
-      for (int q = 0; q < kNImg && q < nstage; ++q) issue(q);
-    }
     float* part = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * a.part_frame_stride;
 #pragma unroll 1
     for (int q = grp; q < nstage + kNBuf; q += kGroups) {
       const int b = grp;
       if (q >= kNBuf) {  // MMAs of stage q - kNBuf (same buffer) are done
         const int qd = q - kNBuf;
-        mbar_wait_bounded(&mma_done[b], (uint32_t)((qd / kNBuf) & 1));
-        fence_after();
+        if (!TC_EXP(256)) mbar_wait_bounded(&mma_done[b], (uint32_t)((qd / kNBuf) & 1));
+        if (!TC_EXP(128)) fence_after();
         if (gtid == 0) TC_STAMP(0, qd);
-        if (qd % nch == nch - 1 && (qd / nch) % kG == kG - 1) {  // last stage of group gd
+        if (!TC_EXP(32) && qd % nch == nch - 1 && (qd / nch) % kG == kG - 1) {  // last stage of group gd
           const int gd = (qd / nch) / kG;
-          const uint32_t col = (uint32_t)((gd * kG) % kRing);
+          const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
           uint32_t d[8];
           ld8(tbase + lane_base + col, d);
           const int vv = v0 + v;
@@ -252,10 +263,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         float x[kWB];
         const bool zero = stage_zero(q);
 #pragma unroll
-        for (int k = 0; k < kWB; ++k) x[k] = zero ? 0.0f : ring[sl * kBoxW + v + k];
+        for (int k = 0; k < kWB; ++k) x[k] = (zero || TC_EXP(64)) ? 0.0f : ring[sl * kBoxW + v + k];
         mbar_arrive(&img_empty[sl]);
         if (gtid == 0) TC_STAMP(6, q);
-        if (gtid == 0 && q + kNImg < nstage) issue(q + kNImg);
         if (gtid == 0) TC_STAMP(7, q);
         uint32_t hi[kWB], lo[kWB];
 #pragma unroll
@@ -271,13 +281,53 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
             st8(ab + c, *reinterpret_cast<const uint32_t(*)[8]>(hi + c));
             st8(ab + kWB + c, *reinterpret_cast<const uint32_t(*)[8]>(lo + c));
           }
-        st_wait();
-        fence_before();
+        if (!TC_EXP(512)) st_wait();
+        if (!TC_EXP(128)) fence_before();
         mbar_arrive(&a_full[b]);
         if (gtid == 0) TC_STAMP(2, q);
       }
     }
-  } else if (warp == 4 * kGroups) {
+  } else if (warp == kTmaWarp) {
+    // ===================== TMA producer: image-row segments, kNImg stages ahead
+    if (lane == 0) {
+      tma_prefetch_desc(&map_img);
+#pragma unroll 1
+      for (int q = 0; q < nstage; ++q) issue(q);
+    }
+    __syncwarp();
+  } else if (warp >= kRelocWarp0 && warp < kRelocWarp0 + 4) {
+    // ===================== relocation warps (lane quadrant warp % 4): move the live window
+    const uint32_t lane_base = (uint32_t)((warp & 3) * 32) << 16;
+    const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
+#pragma unroll 1
+    for (int k = 0; k < nreloc; ++k) {
+      // rare event: poll with back-off so the idle warps do not take issue slots from the
+      // producer and MMA warps sharing their SM sub-partitions
+      for (long long it = 0;; ++it) {
+        uint32_t done = 0;
+        asm volatile(
+            "{\n\t.reg .pred P;\n\tmbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, P;\n}"
+            : "=r"(done)
+            : "r"(smem_u32(&reloc_req)), "r"((uint32_t)(k & 1))
+            : "memory");
+        if (done) break;
+        if (it > (1ll << 26)) __trap();
+        __nanosleep(256);
+      }
+      fence_after();
+#pragma unroll 1
+      for (int c = 0; c < kHB; c += 8) {
+        uint32_t d[8];
+        ld8(tbase + lane_base + kRelocAt + c, d);
+        st8(tbase + lane_base + c, d);
+        st8(tbase + lane_base + kRelocAt + c, z);
+      }
+      st_wait();
+      fence_before();
+      mbar_arrive(&reloc_done);
+    }
+  } else if (warp == kMmaWarp) {
     // ===================== MMA issuer (one thread)
     // Straight-line issue: the thread's scalar work per MMA is one 64-bit descriptor add and one
     // TMEM address add (measured: a loop body of ~30 dependent scalar instructions per MMA
@@ -286,54 +336,60 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       const uint32_t bhi = smem_u32(smem_tc);
       const uint64_t dlo_off = (uint64_t)(((uint32_t)npl * plane) >> 4);  // hi -> lo operand (descriptor units)
       constexpr uint64_t kKStep = (uint64_t)((2 * plane_bytes()) >> 4);   // one K-step = two planes
-      int b = 0, ph = 0, ch = 0, s = 0, g = 0;
+      int b = 0, ph = 0, ch = 0, s = 0, g = 0, nrel_done = 0;
+      // Software-pipelined issue: the wait for stage q+1's operand happens while the last K-step
+      // of stage q is still queued (the tensor pipe's queue is short; a per-stage wait between
+      // the last MMA of q and the first of q+1 left it idle for a few hundred cycles per stage).
+      if (nstage > 0 && !TC_EXP(16)) mbar_wait_bounded(&a_full[0], 0u);
+      fence_after();
 #pragma unroll 1
       for (int q = 0; q < nstage; ++q) {
-        if (!TC_EXP(16)) mbar_wait_bounded(&a_full[b], (uint32_t)ph);
-        if (!TC_EXP(8)) fence_after();
         if (lane == 0) TC_STAMP(3, q);
-        const uint32_t col = TC_EXP(2) ? 0u : (uint32_t)((g * kG) & (kRing - 1));
+        const uint32_t col = (uint32_t)((g * kG) % kRelocAt);
+        if (!TC_EXP(2048) && col == 0 && g > 0 && ch == 0 && s == 0) {  // window restart: relocate the live columns first
+          const int qp = q - 1;  // MMAs complete in order: the last stage's completion covers all
+          mbar_wait_bounded(&mma_done[qp % kNBuf], (uint32_t)((qp / kNBuf) & 1));
+          fence_after();
+          fence_before();
+          if (elect_one()) mbar_arrive(&reloc_req);
+          __syncwarp();
+          mbar_wait_bounded(&reloc_done, (uint32_t)(nrel_done & 1));
+          fence_after();
+          ++nrel_done;
+        }
         // B window: planes of chunk ch, starting at row kG - 1 - s of the reversed block
         const uint64_t dh = sdesc(bhi + (uint32_t)(ch * (kWB / 4)) * plane + (uint32_t)(kG - 1 - s) * 16, plane, 128);
         const uint64_t dl = dh + dlo_off;
         const uint32_t ah = tbase + a_col0 + (uint32_t)(b * 2 * kWB), al = ah + kWB;
         const uint32_t dcol = tbase + col;
-        const bool leader = elect_one();
-        if (!leader) {
-        } else if (col + kNWin <= (uint32_t)kRing) {
-          const uint32_t id = idesc_tf32(kNWin);
+        const uint32_t id = idesc_tf32(kNWin);
+        if (elect_one()) {
 #pragma unroll
-          for (int kk = 0; kk < kWB / 8; ++kk) {
+          for (int kk = 0; kk < kWB / 8 - 1; ++kk) {
             mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
-            if (!TC_EXP(4)) {
-              mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
-              mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
-            }
-          }
-        } else {  // window wraps the ring: columns [col, kRing) and [0, kNWin - (kRing - col))
-          const uint32_t n1 = (uint32_t)kRing - col;
-          const uint32_t id1 = idesc_tf32((int)n1), id2 = idesc_tf32(kNWin - (int)n1);
-          const uint64_t o2 = (uint64_t)n1;  // n1 rows of 16 B, in descriptor units
-#pragma unroll
-          for (int kk = 0; kk < kWB / 8; ++kk) {
-            mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id1);
-            mma_ts(tbase, ah + kk * 8, dh + kk * kKStep + o2, id2);
-            if (!TC_EXP(4)) {
-              mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id1);
-              mma_ts(tbase, ah + kk * 8, dl + kk * kKStep + o2, id2);
-              mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id1);
-              mma_ts(tbase, al + kk * 8, dh + kk * kKStep + o2, id2);
-            }
+            mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
+            mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
           }
         }
-        if (leader) commit(&mma_done[b]);
         __syncwarp();
-        if (lane == 0) TC_STAMP(4, q);
+        // advance the counters and wait for the next stage's operand under the queued MMAs
+        const int bq = b;
         if (++b == kNBuf) { b = 0; ph ^= 1; }
         if (++ch == nch) {
           ch = 0;
           if (++s == kG) { s = 0; ++g; }
         }
+        if (q + 1 < nstage && !TC_EXP(16)) mbar_wait_bounded(&a_full[b], (uint32_t)ph);
+        fence_after();
+        if (elect_one()) {
+          constexpr int kk = kWB / 8 - 1;
+          mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
+          mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
+          mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
+          commit(&mma_done[bq]);
+        }
+        __syncwarp();
+        if (lane == 0) TC_STAMP(4, q);
       }
     }
     __syncwarp();

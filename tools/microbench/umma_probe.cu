@@ -586,7 +586,7 @@ __global__ void rate_mut_kernel(int iters, int mode, int nk_rt, float* sink, lon
   constexpr int K = 64, N = 136, LB = N + 16;
   float* Bs = reinterpret_cast<float*>(sm);
   const int tid = threadIdx.x, warp = tid >> 5;
-  for (int e = tid; e < (K / 4) * LB * 4; e += blockDim.x) Bs[e] = 0.001f * (e % 97);
+  for (int e = tid; e < 2 * (K / 4) * LB * 4; e += blockDim.x) Bs[e] = 0.001f * (e % 97);
   fence_async_smem();
   if (warp == 0) tmem_alloc<512>(&tbase);
   if (tid == 0) { for (int b = 0; b < 5; ++b) mbar_init(&bar[b], 1); asm volatile("fence.mbarrier_init.release.cluster;"); }
@@ -602,7 +602,8 @@ __global__ void rate_mut_kernel(int iters, int mode, int nk_rt, float* sink, lon
   __syncthreads();
   fence_after();
   long long t0 = clock64();
-  if (tid == 0) {
+  const int issuer = (mode & 128) ? 12 * 32 : 0;
+  if (tid == issuer) {
     for (int it = 0; it < iters; ++it) {
       if (mode & 4) {
         for (int kk = 0; kk < nk_rt; ++kk) {
@@ -612,8 +613,12 @@ __global__ void rate_mut_kernel(int iters, int mode, int nk_rt, float* sink, lon
       } else {
 #pragma unroll
         for (int kk = 0; kk < K / 8; ++kk) {
-          const uint64_t b = sdesc(su32(Bs) + kk * 2 * LB * 16, LB * 16, 128);
-          mma_tf32_ts(d, d + 320 + kk * 8, b, idesc_tf32(128, N), (mode & 2) ? 1 : ((it | kk) > 0));
+          const int kb = (mode & 64) ? (kk % 4) : kk;            // 3-product pattern: 4 K-steps x 3
+          const int pp = (mode & 64) ? (kk / 4) % 3 : 0;
+          const uint32_t boff = ((mode & 16) && (kk & 1)) || ((mode & 64) && pp == 1) ? (uint32_t)(8 * LB * 16) : 0u;
+          const uint32_t aoff = ((mode & 32) && (kk & 1)) || ((mode & 64) && pp == 2) ? 32u : 0u;
+          const uint64_t b = sdesc(su32(Bs) + kb * 2 * LB * 16 + boff, LB * 16, 128);
+          mma_tf32_ts(d, d + 320 + kb * 8 + aoff, b, idesc_tf32(128, N), (mode & 2) ? 1 : ((it | kk) > 0));
         }
       }
       if (mode & 1) mma_commit(&bar[it & 3]);
@@ -626,7 +631,7 @@ __global__ void rate_mut_kernel(int iters, int mode, int nk_rt, float* sink, lon
   }
   if (mode & 8) {
     __syncthreads();
-    if (tid == 0) {
+    if (tid == issuer) {
       mbar_wait(&bar[4], 0);
       cycles[blockIdx.x] = clock64() - t0;
     }
@@ -668,10 +673,134 @@ static void rate_mut(int mode, int threads = 256) {
   cudaFree(cyc);
 }
 
+// ---- replica of tm_tc_kernel's MMA stream (no producers): per stage 4 K-steps x 3 products,
+// B window start row 7 - (q % 8), D window start (8 * (q / 8)) % 192, A buffer q % 3; whole warp
+// runs the loop, one elected lane issues.  mode bits: 1 fixed B start, 2 fixed D, 4 fixed A buf.
+__global__ void rate_k_kernel(int stages, int mode, float* sink, long long* cycles) {
+  extern __shared__ __align__(1024) unsigned char sm[];
+  __shared__ uint64_t bar[4];
+  __shared__ uint32_t tbase;
+  constexpr int NW = 136, LB = 144;
+  constexpr uint32_t PL = LB * 16;
+  const int tid = threadIdx.x, warp = tid >> 5;
+  float* Bs = reinterpret_cast<float*>(sm);
+  for (int e = tid; e < 2 * 8 * LB * 4; e += blockDim.x) Bs[e] = (mode & 16) ? 0.0f : 0.001f * (e % 97);
+  fence_async_smem();
+  if (warp == 0) tmem_alloc<512>(&tbase);
+  if (tid == 0) {
+    for (int b = 0; b < 4; ++b) mbar_init(&bar[b], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;");
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(&bar[3])) : "memory");
+  }
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t d = tbase;
+  {
+    float z[8] = {0.5f, 0.25f, 0.125f, 1.f, 2.f, 3.f, 4.f, 5.f};
+    if (mode & 16) for (int k = 0; k < 8; ++k) z[k] = 0.0f;
+    if (warp < 4) for (int c = 0; c < 512; c += 8) tmem_st8(d + ((uint32_t)(warp * 32) << 16) + c, z);
+    tmem_st_wait();
+    fence_before();
+    __syncthreads();
+    fence_after();
+  }
+  long long t0 = clock64();
+  if (tid == 0) sink[4000] = 0.0f;
+  __syncthreads();
+  if (warp == 0) {
+    const uint32_t bhi = su32(Bs);
+    const uint64_t dlo_off = (uint64_t)((8 * PL) >> 4);
+    constexpr uint64_t kKStep = (uint64_t)((2 * PL) >> 4);
+    int b = 0;
+    for (int q = 0; q < stages; ++q) {
+      const int s = (mode & 1) ? 0 : (q & 7), g = (mode & 2) ? 0 : q >> 3;
+      const uint32_t col = (uint32_t)((g * 8) % 192);
+      const uint64_t dh = sdesc(bhi + (uint32_t)(7 - s) * 16, PL, 128);
+      const uint64_t dl = dh + dlo_off;
+      const uint32_t ah = d + 320 + (uint32_t)(((mode & 4) ? 0 : b) * 64), al = ah + 32;
+      const uint32_t dcol = d + col;
+      if (elect_one()) {
+        const uint32_t id = idesc_tf32(128, NW);
+#pragma unroll
+        for (int kk = 0; kk < 4; ++kk) {
+          mma_tf32_ts(dcol, ah + kk * 8, dh + kk * kKStep, id, 1);
+          mma_tf32_ts(dcol, ah + kk * 8, dl + kk * kKStep, id, 1);
+          mma_tf32_ts(dcol, al + kk * 8, dh + kk * kKStep, id, 1);
+        }
+        mma_commit(&bar[b]);
+      }
+      __syncwarp();
+      if ((mode & 8) && (tid & 31) == 0 && q < 1024) { sink[1024 + q] = (float)clock64(); }
+      if (mode & 32) mbar_wait(&bar[3], 0);  // an already-completed barrier phase
+      if (mode & 64) fence_after();
+      if (mode >= 256) {  // per-stage issue gap of (mode >> 8) * 50 cycles
+        const long long t1 = clock64();
+        while (clock64() - t1 < (long long)(mode >> 8) * 50) {
+        }
+      }
+      if (++b == 3) b = 0;
+    }
+    if (tid == 0) {
+      const int ql = stages - 1;
+      mbar_wait(&bar[ql % 3], (ql / 3) & 1);
+      cycles[blockIdx.x] = clock64() - t0;
+      *(volatile int*)&sink[4000] = 1;  // stop flag for the busy warps
+    }
+  } else if ((mode & 128) && warp >= 4) {
+    // busy warps: dependent-free FMA stream with a sleep duty cycle (mode >> 8: sleep ns per 64 FMAs)
+    float a0 = tid, a1 = tid + 1, a2 = tid + 2, a3 = tid + 3;
+    const int sl = mode >> 8;
+    for (int it = 0; it < 200000; ++it) {
+#pragma unroll
+      for (int k = 0; k < 16; ++k) {
+        a0 = fmaf(a0, 1.0001f, 0.5f); a1 = fmaf(a1, 1.0001f, 0.5f); a2 = fmaf(a2, 1.0001f, 0.5f); a3 = fmaf(a3, 1.0001f, 0.5f);
+      }
+      if (sl) __nanosleep(sl);
+      if ((it & 63) == 0 && *(volatile int*)&sink[4000]) break;
+    }
+    if (a0 + a1 + a2 + a3 == 1.2345f) sink[tid] = a0;
+  }
+  __syncthreads();
+  fence_after();
+  float v[8];
+  tmem_ld8(d + ((uint32_t)((warp & 3) * 32) << 16), v);
+  if (v[0] == 12345.f) sink[tid] = v[1];
+  fence_before();
+  __syncthreads();
+  if (warp == 0) tmem_free<512>(d);
+}
+
+static void rate_k(int mode, int threads = 128, int smem = 150000) {
+  CK(cudaFuncSetAttribute(rate_k_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  float* sink;
+  long long* cyc;
+  int nsm = 0;
+  CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0));
+  CK(cudaMalloc(&sink, 65536));
+  CK(cudaMalloc(&cyc, nsm * 8));
+  const int stages = 600;
+  rate_k_kernel<<<nsm, threads, smem>>>(30, mode, sink, cyc);
+  CK(cudaDeviceSynchronize());
+  rate_k_kernel<<<nsm, threads, smem>>>(stages, mode, sink, cyc);
+  CK(cudaDeviceSynchronize());
+  std::vector<long long> c(nsm);
+  CK(cudaMemcpy(c.data(), cyc, nsm * 8, cudaMemcpyDeviceToHost));
+  double avg = 0;
+  for (auto x : c) avg += x;
+  avg /= nsm;
+  printf("{\"probe\": \"rate_k\", \"mode\": %d, \"threads\": %d, \"smem\": %d, \"cycles_per_stage\": %.1f, \"per_mma\": %.1f}\n", mode, threads, smem, avg / stages,
+         avg / stages / 12);
+  cudaFree(sink);
+  cudaFree(cyc);
+}
+
 int main(int argc, char** argv) {
   setvbuf(stdout, nullptr, _IONBF, 0);
-  for (int m : {0, 1, 2, 4, 8, 15}) rate_mut(m);
-  rate_mut(0, 128);
-  rate_mut(8, 128);
+  rate_k(0, 576, 125000);
+  rate_k(128, 576, 125000);
+  rate_k(128 | (64 << 8), 576, 125000);
+  rate_k(128 | (200 << 8), 576, 125000);
+  rate_k(32 | 128 | (64 << 8), 576, 125000);
   return 0;
 }
