@@ -104,3 +104,47 @@ def test_tc_matches_cuda_core_path(monkeypatch):
     _, s_cc, info = run([img], T)
     assert not info["variant_name"].startswith("tm_tc")
     assert np.max(np.abs(s_tc - s_cc)) <= TOL
+
+
+def test_tc_unaligned_pitch_falls_back_at_run_time():
+    """pitch % 4 != 0: no TMA map for the image -> the plan runs its CUDA-core kernel."""
+    img, T, u0, v0 = synth.tm_inputs(2, k=9)
+    H, W = img.shape
+    P = W + 1
+    buf = np.zeros((H, P), np.float32)
+    buf[:, :W] = img
+    dev = torch.device("cuda", 0)
+    with MatchPlan(H, W, 128, 128, write_surface=True, image_pitch=P) as plan:
+        assert plan.info.variant_name.decode().startswith("tm_tc")
+        pk, s = plan.match(torch.from_numpy(buf).to(dev), torch.from_numpy(T).to(dev))
+        torch.cuda.synchronize()
+    d = decode_peaks(pk)
+    assert (int(d["u"][0]), int(d["v"][0])) == (u0, v0)
+    g = synth.rng(96)
+    us, vs = g.integers(0, 897, 100), g.integers(0, 897, 100)
+    assert np.max(np.abs(s[0].cpu().numpy()[us, vs] - oracle.ncc_at(img, T, us, vs))) <= TOL
+
+
+def test_tc_host_path_matches_device_path():
+    img, T, u0, v0 = synth.tm_inputs(2, k=11)
+    peaks, s, _ = run([img], T)
+    hp = torch.empty((1, 4), dtype=torch.int32).pin_memory()
+    with MatchPlan(1024, 1024, 128, 128) as plan:
+        assert plan.info.variant_name.decode().startswith("tm_tc")
+        plan.match_host(torch.from_numpy(img[None].copy()).pin_memory(), torch.from_numpy(T).pin_memory(), hp)
+        torch.cuda.synchronize()
+    d = decode_peaks(hp)
+    assert (int(d["u"][0]), int(d["v"][0])) == (peaks["u"][0], peaks["v"][0]) == (u0, v0)
+    assert float(d["score"][0]) == float(peaks["score"][0])
+
+
+@pytest.mark.parametrize("h,w", [(128, 128), (129, 129), (32, 32), (128, 33), (255, 64)])
+def test_tc_block_boundaries(h, w):
+    """Template sizes at and just past the 128-row block and 32-column chunk boundaries."""
+    img = synth.uniform_image(h + 170, w + 150, 3 * h + w)
+    T, u0, v0 = synth.planted_template(img, h, w, 7 * h + w)
+    ref, pk = oracle.ncc_match(img, T)
+    peaks, s, info = run([img], T)
+    assert info["variant_name"].startswith("tm_tc")
+    assert np.max(np.abs(s[0] - ref)) <= TOL
+    assert (peaks["u"][0], peaks["v"][0]) == (u0, v0)
