@@ -116,8 +116,12 @@ __host__ __device__ constexpr int smem_bytes(int WC) { return smem_need(WC) > 12
 
 #ifdef NCC_TC_TRACE  // tools/microbench/tc_trace.cu: per-stage clock64 stamps of CTA 0
 __device__ long long* g_tc_trace;
+#ifdef NCC_TC_NOSTAMP
+#define TC_STAMP(slot, q)
+#else
 #define TC_STAMP(slot, q) \
   if (blockIdx.x == 0 && blockIdx.y == 0 && (q) < 1024) g_tc_trace[(slot)*1024 + (q)] = clock64()
+#endif
 __device__ int g_tc_exp;  // timing experiments (trace builds only): bit0 no A stores, bit1 no wrap, bit2 one product
 #define TC_EXP(bit) (g_tc_exp & (bit))
 #else
@@ -232,61 +236,71 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     }
     const float* ring = reinterpret_cast<const float*>(smem_tc + img_off(a.WC));
     float* part = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * a.part_frame_stride;
+    // Software-pipelined producer: the operand of the group's next stage is read from the ring
+    // and split while the group waits for its TMEM buffer, so the critical path from "MMAs of
+    // the buffer's previous stage done" to "a_full" is only the TMEM stores (the MMA warp has
+    // kNBuf - 1 stages of slack).  The ring drain of a finished group follows the arrival.
+    uint32_t hi[kWB], lo[kWB];
+    auto load_split = [&](int q) {
+      const int sl = q % kNImg;
+      mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
+      if (gtid == 0) TC_STAMP(5, q);
+      float x[kWB];
+      const bool zero = stage_zero(q);
+#pragma unroll
+      for (int k = 0; k < kWB; ++k) x[k] = (zero || TC_EXP(64)) ? 0.0f : ring[sl * kBoxW + v + k];
+      mbar_arrive(&img_empty[sl]);
+#pragma unroll
+      for (int k = 0; k < kWB; ++k) {
+        hi[k] = to_tf32(x[k]);
+        lo[k] = __float_as_uint(x[k] - __uint_as_float(hi[k]));
+      }
+      if (gtid == 0) TC_STAMP(1, q);
+    };
+    if (grp < nstage) load_split(grp);
+    const int b = grp;
 #pragma unroll 1
     for (int q = grp; q < nstage + kNBuf; q += kGroups) {
-      const int b = grp;
-      if (q >= kNBuf) {  // MMAs of stage q - kNBuf (same buffer) are done
-        const int qd = q - kNBuf;
+      const int qd = q - kNBuf;  // the buffer's previous stage
+      if (qd >= 0) {
         if (!TC_EXP(256)) mbar_wait_bounded(&mma_done[b], (uint32_t)((qd / kNBuf) & 1));
         if (!TC_EXP(128)) fence_after();
         if (gtid == 0) TC_STAMP(0, qd);
-        if (!TC_EXP(32) && qd % nch == nch - 1 && (qd / nch) % kG == kG - 1) {  // last stage of group gd
-          const int gd = (qd / nch) / kG;
-          const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
-          uint32_t d[8];
-          ld8(tbase + lane_base + col, d);
-          const int vv = v0 + v;
-#pragma unroll
-          for (int k = 0; k < kG; ++k) {
-            const int up = gd * kG - kHB + 1 + k;  // output row (CTA-relative)
-            if (up >= 0 && up < nu && vv < a.V)
-              part[(int64_t)(ua - a.u_begin + up) * a.V + vv] = __uint_as_float(d[k]);
-          }
-          const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
-          st8(tbase + lane_base + col, z);
-        }
       }
       if (q < nstage) {
-        const int sl = q % kNImg;
-        mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
-        if (gtid == 0) TC_STAMP(5, q);
-        float x[kWB];
-        const bool zero = stage_zero(q);
-#pragma unroll
-        for (int k = 0; k < kWB; ++k) x[k] = (zero || TC_EXP(64)) ? 0.0f : ring[sl * kBoxW + v + k];
-        mbar_arrive(&img_empty[sl]);
-        if (gtid == 0) TC_STAMP(6, q);
-        if (gtid == 0) TC_STAMP(7, q);
-        uint32_t hi[kWB], lo[kWB];
-#pragma unroll
-        for (int k = 0; k < kWB; ++k) {
-          hi[k] = to_tf32(x[k]);
-          lo[k] = __float_as_uint(x[k] - __uint_as_float(hi[k]));
-        }
-        if (gtid == 0) TC_STAMP(1, q);
         const uint32_t ab = tbase + lane_base + a_col0 + (uint32_t)(b * 2 * kWB);
+        if (!TC_EXP(1)) {
 #pragma unroll
-        if (!TC_EXP(1))
           for (int c = 0; c < kWB; c += 8) {
             st8(ab + c, *reinterpret_cast<const uint32_t(*)[8]>(hi + c));
             st8(ab + kWB + c, *reinterpret_cast<const uint32_t(*)[8]>(lo + c));
           }
+        }
         if (!TC_EXP(512)) st_wait();
         if (!TC_EXP(128)) fence_before();
         mbar_arrive(&a_full[b]);
         if (gtid == 0) TC_STAMP(2, q);
       }
+      // drain the ring columns of a group whose last stage was qd (its MMAs are complete);
+      // the zeroing stores are waited for before this group's next a_full arrival
+      if (qd >= 0 && !TC_EXP(32) && qd % nch == nch - 1 && (qd / nch) % kG == kG - 1) {
+        const int gd = (qd / nch) / kG;
+        const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
+        uint32_t d[8];
+        ld8(tbase + lane_base + col, d);
+        const int vv = v0 + v;
+#pragma unroll
+        for (int k = 0; k < kG; ++k) {
+          const int up = gd * kG - kHB + 1 + k;  // output row (CTA-relative)
+          if (up >= 0 && up < nu && vv < a.V)
+            part[(int64_t)(ua - a.u_begin + up) * a.V + vv] = __uint_as_float(d[k]);
+        }
+        const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
+        st8(tbase + lane_base + col, z);
+      }
+      if (q + kGroups < nstage) load_split(q + kGroups);
     }
+    st_wait();  // last zeroing stores
   } else if (warp == kTmaWarp) {
     // ===================== TMA producer: image-row segments, kNImg stages ahead
     if (lane == 0) {
