@@ -133,7 +133,10 @@ struct PivVariant {
   const void* k_ldg;
   const void* k_ws = nullptr;  // persistent warp-specialised form (TMA only), if instantiated
   int ws_ncw = 0, ws_npw = 0;
+  int ws_bp = 0;     // staged pitch (= TMA box width) of the WS kernel; 0: the plan's piv_bp
+  int ws_bytes = 0;  // dynamic shared memory of the WS kernel; 0: 2 PivShape<12,64> stages + score tile
 };
+using Ws2Cfg4 = PivWs2Shape<64, 64, 32, 32, 16, 64>;
 #define PIV_VARIANT_SK(NAME, TH, TW, MY, MX, RV, CW, NT, WPB, MINB, IPT)                                     \
   PivVariant {                                                                                              \
     NAME, TH, TW, MY, MX, RV, CW, NT, WPB, 1, IPT,                                                          \
@@ -150,6 +153,11 @@ struct PivVariant {
 const PivVariant kPivVariants[] = {
     PIV_VARIANT_RE("piv_re_rv12_cw16_nt256", 12, 16, 256, 1),
     PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt416_w4", 32, 32, 16, 16, 12, 32, 416, 4, 2, 1),
+    PivVariant{"piv_ws2_64x64_m32_rv16_c8p4", 64, 64, 32, 32, 12, 64, 416, 1, 1, 1,
+               reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, true, true, 1>),
+               reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, false, true, 1>),
+               reinterpret_cast<const void*>(&piv_ws2_kernel<64, 64, 32, 32, 16, 64, 8, 4>), 8, 4, Ws2Cfg4::BP,
+               Ws2Cfg4::smem_bytes},
     PivVariant{"piv_ws_64x64_m32_rv12_c13p4", 64, 64, 32, 32, 12, 64, 416, 1, 1, 1,
                reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, true, true, 1>),
                reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, false, true, 1>),
@@ -290,6 +298,7 @@ struct ncc_plan_s {
   // PIV
   int Ky, Kx, OY, OX, sub_batch, piv_bp, piv_smem, map_w, map_h;
   int ws_smem, ws_grid;  // persistent warp-specialised PIV kernel (0: not used)
+  int ws_bp;             // its staged pitch = TMA box width
   const PivVariant* pivv;
   // shared scratch (window sums)
   double *RS1, *RS2, *S1, *S2;
@@ -744,10 +753,11 @@ ncc_status create_piv(ncc_plan pl) {
   NCC_CUDA(cudaFuncSetAttribute(v->k_ldg, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->piv_smem));
   if (v->k_ws && !getenv("NCC_NO_WS")) {  // persistent warp-specialised form: 2 stages + score tile
     PivShape<12, 64> ps(h, w, my, mx, pl->piv_bp, false);
-    const int64_t ws_bytes = (2 * (int64_t)(ps.tp_fl + ps.b_fl) + ps.s_fl) * 4;
+    const int64_t ws_bytes = v->ws_bytes ? v->ws_bytes : (2 * (int64_t)(ps.tp_fl + ps.b_fl) + ps.s_fl) * 4;
     int nsm = 0;
     NCC_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, pl->device));
     if (ws_bytes <= maxsm && v->CW == 64 && v->RV == 12) {
+      pl->ws_bp = v->ws_bp ? v->ws_bp : pl->piv_bp;
       NCC_CUDA(cudaFuncSetAttribute(v->k_ws, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ws_bytes));
       pl->ws_smem = (int)ws_bytes;
       pl->ws_grid = nsm;
@@ -785,7 +795,10 @@ ncc_status create_piv(ncc_plan pl) {
   in.specialized = pl->jit_lib ? 2 : (v->TH != 0);
   in.variant_id = pl->jit_lib ? -1 : (int)(v - kPivVariants);
   snprintf(in.variant_name, sizeof(in.variant_name), "%s", v->name);
-  fill_kernel_info(pl, v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
+  if (pl->ws_smem)  // persistent warp-specialised kernel: one CTA per SM loops over the windows
+    fill_kernel_info(pl, v->k_ws, (v->ws_ncw + v->ws_npw) * 32, pl->ws_smem, pl->ws_grid, 1, sb);  // z: pairs per launch
+  else
+    fill_kernel_info(pl, v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
   in.launches_per_call = (pl->box_smem ? 2 : 3) * ceil_div(p.batch, sb);  // per sub-batch: window sums + PIV
   return NCC_OK;
 }
@@ -1029,6 +1042,14 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
     const uint32_t boxB[3] = {(uint32_t)pl->piv_bp, (uint32_t)(p.tmpl_h + 2 * p.search_y), 1u};
     use_tma = boxB[1] <= 256 && boxB[0] <= 256 && encode_f32(&mB, B, 3, dims, strides, boxB);
   }
+  CUtensorMap mW;  // the WS kernel's own box width
+  memset(&mW, 0, sizeof(mW));
+  if (use_tma && pl->ws_smem) {
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
+    const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)fs * 4};
+    const uint32_t boxB[3] = {(uint32_t)pl->ws_bp, (uint32_t)(p.tmpl_h + 2 * p.search_y), 1u};
+    if (!(boxB[0] <= 256 && encode_f32(&mW, B, 3, dims, strides, boxB))) return NCC_ERR_CUDA;
+  }
   const int groups = ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB);
   mark(pl, s, 0);
   for (int sb = 0; sb < nsub; ++sb) {
@@ -1040,7 +1061,7 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
     dim3 grid(groups, 1, np);
     if (use_tma && pl->ws_smem) {
       int total = (int)((int64_t)np * pl->Ky * pl->Kx);
-      void* wargs[3] = {&a, &mB, &total};
+      void* wargs[3] = {&a, &mW, &total};
       const int g = total < pl->ws_grid ? total : pl->ws_grid;
       NCC_CUDA(cudaLaunchKernel(v->k_ws, dim3(g), dim3((v->ws_ncw + v->ws_npw) * 32), wargs, (size_t)pl->ws_smem, s));
     } else {

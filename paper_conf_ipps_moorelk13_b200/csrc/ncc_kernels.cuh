@@ -170,6 +170,23 @@ __device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity
   }
   __trap();
 }
+// Long waits of otherwise idle warps (a producer waiting for a window's core): back off with
+// nanosleep so the spinning does not take issue slots from the warps doing the work.
+__device__ __forceinline__ void mbar_wait_backoff(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  for (long long it = 0; it < (1ll << 28); ++it) {
+    asm volatile(
+        "{\n\t.reg .pred P;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, P;\n}"
+        : "=r"(done)
+        : "r"(smem_u32(bar)), "r"(parity)
+        : "memory");
+    if (done) return;
+    __nanosleep(200);
+  }
+  __trap();
+}
 __device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
   asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
@@ -913,6 +930,35 @@ __device__ __forceinline__ void row_dot_pairs(const float* __restrict__ img, con
   }
 }
 
+// Same sums, image-major order: for each image value x[c], every (p, q) with p + 2q = c, so
+// consecutive FFMA2 share the scalar operand (reuse cache) and read only the template pair and
+// the accumulator pair.  Per accumulator the products still come in increasing p.
+template <int RV, int CW>
+__device__ __forceinline__ void row_dot_pairs_x(const float* __restrict__ img, const u64* __restrict__ TP,
+                                                u64 (&A2)[RV / 2]) {
+  static_assert(RV % 4 == 0 && CW % 4 == 0, "RV and CW must be multiples of 4");
+  float x[RV + CW + 4];
+  u64 tp[CW + 2];
+#pragma unroll
+  for (int c = 0; c < RV + CW; c += 4) {
+    const float4 v = *reinterpret_cast<const float4*>(img + c);
+    x[c] = v.x; x[c + 1] = v.y; x[c + 2] = v.z; x[c + 3] = v.w;
+  }
+#pragma unroll
+  for (int pp = 0; pp <= CW; pp += 2) {
+    const ulonglong2 t = *reinterpret_cast<const ulonglong2*>(TP + pp);
+    tp[pp] = t.x;
+    tp[pp + 1] = t.y;
+  }
+#pragma unroll
+  for (int c = 0; c < RV + CW; ++c)
+#pragma unroll
+    for (int q = RV / 2 - 1; q >= 0; --q) {
+      const int p = c - 2 * q;
+      if (p >= 0 && p <= CW) ffma2_bcast(A2[q], x[c], tp[p]);
+    }
+}
+
 // Per-window shared-memory geometry (floats); regions rounded to 128 B for TMA destinations.
 // TP: template pairs, per row nCW blocks of PB = CW + 2 pairs.  Sc (score tile) aliases TP
 // when ALIAS (scores are held in registers across the barrier that ends the numerator).
@@ -1545,6 +1591,339 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
 #pragma unroll
         for (int c = 0; c < RV; ++c) sc[c] = out[c];
       }
+      mbar_arrive(&scfull_b);
+    }
+  }
+}
+
+// ================================================================== PIV, persistent + warp-specialised, balanced core
+// piv_ws_kernel spreads (2m+1) x ceil((2m+1)/RV) items over 13 consumer warps: the SMSP that
+// holds 4 of them sets the pace (13/16 of the FMA pipe) and 7 of every 72 columns are padding.
+// Here the consumers own exactly the 2m_y x 2m_x core of the offset grid -- NCW warps, two per
+// SMSP, RV = 16 shifts per lane, no padding -- and the producer warps, otherwise idle while a
+// window is correlated, compute the (2m_x+1) + 2m_y border offsets (last row dy = +m_y, last
+// column dx = +m_x) with scalar FFMA from the same staged stage.  Items of a warp: 8 output rows
+// x 4 column groups, laid out so each 8-lane LDS.128 phase covers 4 rows x 2 groups and the
+// staged pitch (BP = 4 mod 32 floats) puts them on 8 distinct 16-B bank groups.
+__host__ __device__ constexpr int piv_ws2_pitch(int TW, int MX, int CW) {
+  return (((2 * MX + ((TW + CW - 1) / CW) * CW) - 4 + 31) / 32) * 32 + 4;
+}
+template <int TH, int TW, int MY, int MX, int RV, int CW>
+struct PivWs2Shape {
+  static constexpr int OY = 2 * MY + 1, OX = 2 * MX + 1, OYc = 2 * MY, OXc = 2 * MX, NG = OXc / RV;
+  static constexpr int nCW = TW / CW, PB = CW + 2, TPP = nCW * PB, BR = TH + 2 * MY;
+  static constexpr int BP = piv_ws2_pitch(TW, MX, CW);
+  static constexpr int SP = (OX + 3) & ~3;  // score tile pitch
+  static constexpr int tp_fl = ((TH * TPP * 2 + 31) / 32) * 32, b_fl = ((BR * BP + 31) / 32) * 32;
+  static constexpr int s_fl = ((OY * SP + 31) / 32) * 32;
+  static constexpr int NE = OX + OYc;  // border offsets computed by the producers
+  static constexpr int smem_bytes = (2 * (tp_fl + b_fl) + s_fl) * 4;
+};
+template <int TH, int TW, int MY, int MX, int RV, int CW, int NCW, int NPW>
+__global__ void __launch_bounds__((NCW + NPW) * 32, 1)
+    piv_ws2_kernel(const PivArgs a, const __grid_constant__ CUtensorMap mapB, int nwin_total) {
+  using S = PivWs2Shape<TH, TW, MY, MX, RV, CW>;
+  constexpr int NCT = NCW * 32, NPT = NPW * 32;
+  static_assert(RV == 16 && S::NG == 4 && S::OXc % RV == 0, "lane layout: 4 groups of 16 shifts per row");
+  static_assert(S::OYc == 8 * NCW, "one warp per 8 core rows");
+  static_assert(TW % CW == 0 && CW % 4 == 0, "whole column chunks");
+  static_assert((S::BP / 4) % 8 == 1, "conflict-free LDS.128 phases");
+  constexpr int NEW = (S::NE + NPW - 1) / NPW;  // border offsets per producer warp: e = pw + NPW * o
+  static_assert(NEW <= 64 && TW % 32 == 0, "border: <= 2 offsets per lane, whole 32-column lane strips");
+  constexpr int EPT = 2;
+  extern __shared__ __align__(1024) unsigned char smem_raw[];
+  float* smem = reinterpret_cast<float*>(smem_raw);
+  __shared__ __align__(8) uint64_t full_b[2], empty_b[2], scfull_b, scempty_b;
+  __shared__ double st_mean[2], st_sumsq[2], st_energy[2], st_csum[2];
+  __shared__ int st_flat[2];
+  __shared__ double pred[NPW * 4];
+  __shared__ unsigned long long pkey[NPW];
+  auto TPs = [&](int s) { return reinterpret_cast<u64*>(smem + s * (S::tp_fl + S::b_fl)); };
+  auto Bs = [&](int s) { return smem + s * (S::tp_fl + S::b_fl) + S::tp_fl; };
+  float* Sc = smem + 2 * (S::tp_fl + S::b_fl);
+
+  const int tid = threadIdx.x;
+  const int nwin = a.Ky * a.Kx;
+  if (tid == 0) {
+    tma_prefetch_desc(&mapB);
+    mbar_init(&full_b[0], 2);
+    mbar_init(&full_b[1], 2);
+    mbar_init(&empty_b[0], NCT);
+    mbar_init(&empty_b[1], NCT);
+    mbar_init(&scfull_b, NCT);
+    mbar_init(&scempty_b, 1);
+    fence_mbar_init();
+  }
+  __syncthreads();
+  const int nlocal = (nwin_total - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+  auto win_of = [&](int k, int& lz, int& lin) {
+    const int wdx = (int)blockIdx.x + k * (int)gridDim.x;
+    lz = wdx / nwin;
+    lin = wdx % nwin;
+  };
+  const double inv_n = 1.0 / ((double)TH * (double)TW);
+
+  if (tid >= NCT) {
+    // =============================== producers
+    const int pt = tid - NCT, lane = tid & 31, pw = pt >> 5;
+    constexpr int PERT = (TH * TW + NPT - 1) / NPT;
+    auto reduce2 = [&](double& x0, double& x1) {  // deterministic sum over the producer threads
+      x0 = warp_sum_d(x0);
+      x1 = warp_sum_d(x1);
+      named_bar_sync(1, NPT);
+      if (lane == 0) { pred[pw * 2] = x0; pred[pw * 2 + 1] = x1; }
+      named_bar_sync(1, NPT);
+      x0 = 0.0;
+      x1 = 0.0;
+      for (int q = 0; q < NPW; ++q) { x0 += pred[q * 2]; x1 += pred[q * 2 + 1]; }
+    };
+    auto border = [&](int e, int& dy, int& dx) {
+      if (e < S::OX) { dy = S::OYc; dx = e; } else { dy = e - S::OX; dx = S::OXc; }
+    };
+    float ext_prev[EPT];
+    auto owned = [&](int q) { return pw + NPW * (lane + 32 * q); };  // border offset index of slot q
+    auto epilogue = [&](int k) {
+      int lz, lin;
+      win_of(k, lz, lin);
+      const int s = k & 1;
+      mbar_wait_backoff(&scfull_b, (uint32_t)(k & 1));
+#pragma unroll
+      for (int q = 0; q < EPT; ++q) {  // border scores of window k (computed during its core)
+        const int e = owned(q);
+        if (e < S::NE) {
+          int dy, dx;
+          border(e, dy, dx);
+          Sc[dy * S::SP + dx] = ext_prev[q];
+        }
+      }
+      named_bar_sync(1, NPT);
+      constexpr int tile = S::OY * S::OX;
+      unsigned long long best = 0ull;
+      const int pr = a.pair0 + lz;
+      for (int e = pt; e < tile; e += NPT) {
+        const int row = e / S::OX, col = e % S::OX;
+        const float sv = Sc[row * S::SP + col];
+        if (a.scores) a.scores[((int64_t)pr * nwin + lin) * tile + e] = sv;
+        const unsigned long long key = make_key(a.ssd ? -sv : sv, (uint32_t)e);
+        best = key > best ? key : best;
+      }
+      best = warp_max_key(best);
+      if (lane == 0) pkey[pw] = best;
+      named_bar_sync(1, NPT);
+      if (pt == 0) {
+        unsigned long long bk = 0ull;
+        for (int q = 0; q < NPW; ++q) bk = pkey[q] > bk ? pkey[q] : bk;
+        const uint32_t kk = key_index(bk);
+        const int row = (int)(kk / S::OX), col = (int)(kk % S::OX);
+        const int iy = row - MY, ix = col - MX;
+        uint32_t flags = (st_flat[s] && !a.ssd) ? (kFlatTemplate | kInvalid) : 0u;
+        double ddy = 0.0, ddx = 0.0;
+        bool par = false;
+        if (row == 0 || row == S::OY - 1) {
+          flags |= kEdgeY;
+        } else {
+          const double cm = Sc[(row - 1) * S::SP + col], c0 = Sc[row * S::SP + col], cp = Sc[(row + 1) * S::SP + col];
+          ddy = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
+          if (par) flags |= kParabolaY;
+        }
+        par = false;
+        if (col == 0 || col == S::OX - 1) {
+          flags |= kEdgeX;
+        } else {
+          const double cm = Sc[row * S::SP + col - 1], c0 = Sc[row * S::SP + col], cp = Sc[row * S::SP + col + 1];
+          ddx = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
+          if (par) flags |= kParabolaX;
+        }
+        VecOut o;
+        o.iy = iy;
+        o.ix = ix;
+        o.dy = (float)(iy + ddy);
+        o.dx = (float)(ix + ddx);
+        o.score = a.ssd ? -key_score(bk) : key_score(bk);
+        o.flags = flags;
+        a.vec[(int64_t)pr * nwin + lin] = o;
+        mbar_arrive(&scempty_b);  // the score tile may be overwritten
+      }
+      named_bar_sync(1, NPT);  // pkey / stats reuse
+    };
+    for (int k = 0; k < nlocal; ++k) {
+      const int s = k & 1;
+      int lz, lin;
+      win_of(k, lz, lin);
+      const int pr = a.pair0 + lz;
+      const int y = MY + (lin / a.Kx) * a.sy, x = MX + (lin % a.Kx) * a.sx;
+      if (k >= 2) mbar_wait_bounded(&empty_b[s], (uint32_t)(((k >> 1) - 1) & 1));
+      if (pt == 0) {
+        mbar_expect_tx(&full_b[s], (uint32_t)(S::BR * S::BP * 4));
+        tma_load_3d(Bs(s), &mapB, x - MX, y - MY, pr, &full_b[s]);
+      }
+      // mask statistics and template pairs (as piv_ncc_kernel)
+      const float* Af = a.A + (int64_t)pr * a.frame_stride;
+      float mv[PERT];
+#pragma unroll
+      for (int q = 0; q < PERT; ++q) {
+        const int e = pt + q * NPT;
+        mv[q] = e < TH * TW ? __ldg(Af + (int64_t)(y + e / TW) * a.pitch + x + e % TW) : 0.0f;
+      }
+      double s1 = 0.0, s2 = 0.0;
+#pragma unroll
+      for (int q = 0; q < PERT; ++q) { s1 += (double)mv[q]; s2 += (double)mv[q] * (double)mv[q]; }
+      reduce2(s1, s2);
+      const double mean = s1 * inv_n;
+      double e2 = 0.0, cs = 0.0;
+      u64* tpw = TPs(s);
+#pragma unroll
+      for (int q = 0; q < PERT; ++q) {
+        const int e = pt + q * NPT;
+        if (e < TH * TW) {
+          const int i = e / TW, j = e % TW;
+          const double d = (double)mv[q] - mean;
+          const float ac = (float)d;
+          e2 += d * d;
+          cs += (double)ac;
+          float* tp = reinterpret_cast<float*>(tpw + i * S::TPP + (j / CW) * S::PB);
+          const int l = j % CW;
+          tp[2 * l + 1] = ac;
+          tp[2 * (l + 1)] = ac;
+          if (l == 0) tp[0] = 0.0f;
+          if (l == CW - 1) tp[2 * CW + 1] = 0.0f;
+        }
+      }
+      reduce2(e2, cs);
+      const bool flat = e2 <= kFlatRel * s2;
+      if (pt == 0) {
+        st_mean[s] = mean;
+        st_sumsq[s] = s2;
+        st_energy[s] = e2;
+        st_csum[s] = cs;
+        st_flat[s] = flat ? 1 : 0;
+      }
+      named_bar_sync(1, NPT);  // template pairs + stats of all producers written
+      if (pt == 0) mbar_arrive(&full_b[s]);
+      // border offsets of window k: same products and row-blocked partials as the core
+      mbar_wait_bounded(&full_b[s], (uint32_t)((k >> 1) & 1));  // search region landed
+      // Lanes split the template columns (j = lane + 32c), each warp walks its NEW border
+      // offsets per template row: conflict-free scalar loads of the region, the template value
+      // loaded once per row; per-lane fp32 sums over <= 2*TH products, then a butterfly sum.
+      float ext_cur[EPT];
+      {
+        constexpr int JPL = TW / 32;
+        const float* tpf = reinterpret_cast<const float*>(tpw);
+        const float* bs = Bs(s) + lane;
+        int boff[NEW];
+#pragma unroll
+        for (int o = 0; o < NEW; ++o) {
+          const int e = pw + NPW * o;
+          int dy = 0, dx = 0;
+          if (e < S::NE) border(e, dy, dx);
+          boff[o] = dy * S::BP + dx;
+        }
+        float acc[NEW];
+#pragma unroll
+        for (int o = 0; o < NEW; ++o) acc[o] = 0.0f;
+#pragma unroll 1
+        for (int i = 0; i < TH; ++i) {
+          float tv[JPL];
+#pragma unroll
+          for (int c = 0; c < JPL; ++c) {
+            const int j = lane + 32 * c;
+            tv[c] = tpf[(i * S::TPP + (j / CW) * S::PB) * 2 + 1 + 2 * (j % CW)];
+          }
+          const float* br = bs + i * S::BP;
+#pragma unroll
+          for (int o = 0; o < NEW; ++o)
+#pragma unroll
+            for (int c = 0; c < JPL; ++c) acc[o] = fmaf(tv[c], br[boff[o] + 32 * c], acc[o]);
+        }
+        float mine[EPT] = {0.0f, 0.0f};
+#pragma unroll
+        for (int o = 0; o < NEW; ++o) {
+          float v = acc[o];
+#pragma unroll
+          for (int d = 16; d; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
+          if (o == lane) mine[0] = v;
+          if (o == lane + 32) mine[1] = v;
+        }
+        const double* S1f = a.S1 + (int64_t)lz * a.map_frame_stride;
+        const double* S2f = a.S2 + (int64_t)lz * a.map_frame_stride;
+#pragma unroll
+        for (int q = 0; q < EPT; ++q) {
+          const int e = owned(q);
+          float v = 0.0f;
+          if (e < S::NE) {
+            int dy, dx;
+            border(e, dy, dx);
+            const int64_t mi = (int64_t)(y - MY + dy) * a.map_pitch + (x - MX + dx);
+            const double ws1 = __ldg(S1f + mi), ws2 = __ldg(S2f + mi);
+            v = a.ssd ? (float)(s2 - 2.0 * ((double)mine[q] + mean * ws1) + ws2)
+                      : ncc_normalize_fast(mine[q], ws1, ws2, inv_n, cs, e2, flat);
+          }
+          ext_cur[q] = v;
+        }
+      }
+      if (k >= 1) epilogue(k - 1);
+#pragma unroll
+      for (int q = 0; q < EPT; ++q) ext_prev[q] = ext_cur[q];
+    }
+    if (nlocal >= 1) epilogue(nlocal - 1);
+  } else {
+    // =============================== consumers: 8 core rows x 4 groups of RV shifts per warp
+    const int wq = tid >> 5, l = tid & 31, ph = l >> 3, q8 = l & 7;
+    const int row = wq * 8 + 4 * (ph >> 1) + (q8 & 3);
+    const int g = (q8 >> 2) + 2 * (ph & 1);
+    for (int k = 0; k < nlocal; ++k) {
+      const int s = k & 1;
+      int lz, lin;
+      win_of(k, lz, lin);
+      const int y = MY + (lin / a.Kx) * a.sy, x = MX + (lin % a.Kx) * a.sx;
+      mbar_wait_bounded(&full_b[s], (uint32_t)((k >> 1) & 1));
+      float out[RV];
+      {
+        u64 tot2[RV / 2];
+#pragma unroll
+        for (int q = 0; q < RV / 2; ++q) tot2[q] = 0ull;
+        const float* brow = Bs(s) + row * S::BP + g * RV;
+        const u64* tpw = TPs(s);
+#pragma unroll 1
+        for (int i = 0; i < TH; ++i) {
+#pragma unroll
+          for (int jc = 0; jc < S::nCW; ++jc) {
+            u64 part2[RV / 2];
+#pragma unroll
+            for (int q = 0; q < RV / 2; ++q) part2[q] = 0ull;
+#ifdef NCC_WS2_XMAJOR
+            row_dot_pairs_x<RV, CW>(brow + i * S::BP + jc * CW, tpw + i * S::TPP + jc * S::PB, part2);
+#else
+            row_dot_pairs<RV, CW>(brow + i * S::BP + jc * CW, tpw + i * S::TPP + jc * S::PB, part2);
+#endif
+#pragma unroll
+            for (int q = 0; q < RV / 2; ++q) add2(tot2[q], part2[q]);
+          }
+        }
+        const double csum = st_csum[s], energy = st_energy[s], tmean = st_mean[s], tsq = st_sumsq[s];
+        const bool flat = st_flat[s] != 0;
+        const double* S1f = a.S1 + (int64_t)lz * a.map_frame_stride;
+        const double* S2f = a.S2 + (int64_t)lz * a.map_frame_stride;
+        const int64_t mrow = (int64_t)(y - MY + row) * a.map_pitch + (x - MX) + g * RV;
+#pragma unroll
+        for (int q = 0; q < RV / 2; ++q) {
+          const float lo = __uint_as_float((uint32_t)(tot2[q] & 0xFFFFFFFFull));
+          const float hi = __uint_as_float((uint32_t)(tot2[q] >> 32));
+#pragma unroll
+          for (int e = 0; e < 2; ++e) {
+            const int c = 2 * q + 1 - e;
+            const double s1 = __ldg(S1f + mrow + c), s2 = __ldg(S2f + mrow + c);
+            const float num = e == 0 ? lo : hi;
+            out[c] = a.ssd ? (float)(tsq - 2.0 * ((double)num + tmean * s1) + s2)
+                           : ncc_normalize_fast(num, s1, s2, inv_n, csum, energy, flat);
+          }
+        }
+      }
+      mbar_arrive(&empty_b[s]);  // done reading stage s (pairs, region, stats)
+      if (k >= 1) mbar_wait_bounded(&scempty_b, (uint32_t)((k - 1) & 1));
+      float* sc = Sc + row * S::SP + g * RV;
+#pragma unroll
+      for (int c = 0; c < RV; c += 4) *reinterpret_cast<float4*>(sc + c) = make_float4(out[c], out[c + 1], out[c + 2], out[c + 3]);
       mbar_arrive(&scfull_b);
     }
   }

@@ -4,13 +4,13 @@
 register sources that are not served by the operand-reuse cache; uniform registers and
 constants are free).
 
-  cuobjdump -sass lib.so | python tools/sass_banks.py [function-substring]
+  cuobjdump -sass lib.so | python tools/sass_banks.py [function-substring] [opcode-only]
 """
 import re
 import sys
 
 
-def analyze(lines):
+def analyze(lines, only=None):
     n = cyc = 0
     hist = {}
     prev_reuse = [None, None, None]  # register kept in each slot's reuse cache by the previous instruction
@@ -19,6 +19,9 @@ def analyze(lines):
         if not m:
             continue
         op, args = m.group(1), m.group(2)
+        if only and op != only:
+            prev_reuse = [None, None, None]
+            continue
         parts = [p.strip() for p in args.split(",")]
         srcs = parts[1:]
         regs = []
@@ -47,17 +50,18 @@ def analyze(lines):
 
 if __name__ == "__main__":
     key = sys.argv[1] if len(sys.argv) > 1 else ""
+    only = sys.argv[2] if len(sys.argv) > 2 else None  # e.g. FFMA2: model only that opcode
     cur, buf, out = None, [], {}
     for ln in sys.stdin:
         m = re.search(r"Function : (\S+)", ln)
         if m:
             if cur is not None:
-                out[cur] = analyze(buf)
+                out[cur] = analyze(buf, only)
             cur, buf = m.group(1), []
         else:
             buf.append(ln)
     if cur is not None:
-        out[cur] = analyze(buf)
+        out[cur] = analyze(buf, only)
     for f, (n, cyc, hist) in out.items():
         if key in f and n:
             print(f"{f[:90]:90s} fma-lanes={n:6d} est_cycles={cyc:6d} eff={n / cyc:.3f} {dict(sorted(hist.items()))}")
