@@ -135,8 +135,10 @@ struct PivVariant {
   int ws_ncw = 0, ws_npw = 0;
   int ws_bp = 0;     // staged pitch (= TMA box width) of the WS kernel; 0: the plan's piv_bp
   int ws_bytes = 0;  // dynamic shared memory of the WS kernel; 0: 2 PivShape<12,64> stages + score tile
+  int ws_wps = 1;    // windows per pipeline stage of the WS kernel
 };
-using Ws2Cfg4 = PivWs2Shape<64, 64, 32, 32, 16, 64>;
+using Ws2Cfg4 = PivWs2Shape<64, 64, 32, 32, 16, 64, 1>;
+using Ws2Cfg3 = PivWs2Shape<32, 32, 16, 16, 16, 32, 4>;
 #define PIV_VARIANT_SK(NAME, TH, TW, MY, MX, RV, CW, NT, WPB, MINB, IPT)                                     \
   PivVariant {                                                                                              \
     NAME, TH, TW, MY, MX, RV, CW, NT, WPB, 1, IPT,                                                          \
@@ -152,12 +154,17 @@ using Ws2Cfg4 = PivWs2Shape<64, 64, 32, 32, 16, 64>;
 
 const PivVariant kPivVariants[] = {
     PIV_VARIANT_RE("piv_re_rv12_cw16_nt256", 12, 16, 256, 1),
+    PivVariant{"piv_ws2_32x32_m16_rv16_c8p8_w4", 32, 32, 16, 16, 12, 32, 416, 4, 1, 1,
+               reinterpret_cast<const void*>(&piv_ncc_kernel<32, 32, 16, 16, 12, 32, 416, 4, 2, true, true, 1>),
+               reinterpret_cast<const void*>(&piv_ncc_kernel<32, 32, 16, 16, 12, 32, 416, 4, 2, false, true, 1>),
+               reinterpret_cast<const void*>(&piv_ws2_kernel<32, 32, 16, 16, 16, 32, 8, 8, 4>), 8, 8, Ws2Cfg3::BP,
+               Ws2Cfg3::smem_bytes, 4},
     PIV_VARIANT_SK("piv_sk_32x32_m16_rv12_nt416_w4", 32, 32, 16, 16, 12, 32, 416, 4, 2, 1),
-    PivVariant{"piv_ws2_64x64_m32_rv16_c8p4", 64, 64, 32, 32, 12, 64, 416, 1, 1, 1,
+    PivVariant{"piv_ws2_64x64_m32_rv16_c8p8", 64, 64, 32, 32, 12, 64, 416, 1, 1, 1,
                reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, true, true, 1>),
                reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, false, true, 1>),
-               reinterpret_cast<const void*>(&piv_ws2_kernel<64, 64, 32, 32, 16, 64, 8, 4>), 8, 4, Ws2Cfg4::BP,
-               Ws2Cfg4::smem_bytes},
+               reinterpret_cast<const void*>(&piv_ws2_kernel<64, 64, 32, 32, 16, 64, 8, 8, 1>), 8, 8, Ws2Cfg4::BP,
+               Ws2Cfg4::smem_bytes, 1},
     PivVariant{"piv_ws_64x64_m32_rv12_c13p4", 64, 64, 32, 32, 12, 64, 416, 1, 1, 1,
                reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, true, true, 1>),
                reinterpret_cast<const void*>(&piv_ncc_kernel<64, 64, 32, 32, 12, 64, 416, 1, 2, false, true, 1>),
@@ -756,7 +763,7 @@ ncc_status create_piv(ncc_plan pl) {
     const int64_t ws_bytes = v->ws_bytes ? v->ws_bytes : (2 * (int64_t)(ps.tp_fl + ps.b_fl) + ps.s_fl) * 4;
     int nsm = 0;
     NCC_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, pl->device));
-    if (ws_bytes <= maxsm && v->CW == 64 && v->RV == 12) {
+    if (ws_bytes <= maxsm && (v->ws_bytes || (v->CW == 64 && v->RV == 12))) {
       pl->ws_bp = v->ws_bp ? v->ws_bp : pl->piv_bp;
       NCC_CUDA(cudaFuncSetAttribute(v->k_ws, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ws_bytes));
       pl->ws_smem = (int)ws_bytes;
@@ -1062,7 +1069,8 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
     if (use_tma && pl->ws_smem) {
       int total = (int)((int64_t)np * pl->Ky * pl->Kx);
       void* wargs[3] = {&a, &mW, &total};
-      const int g = total < pl->ws_grid ? total : pl->ws_grid;
+      const int ngroups = ceil_div(total, v->ws_wps);
+      const int g = ngroups < pl->ws_grid ? ngroups : pl->ws_grid;
       NCC_CUDA(cudaLaunchKernel(v->k_ws, dim3(g), dim3((v->ws_ncw + v->ws_npw) * 32), wargs, (size_t)pl->ws_smem, s));
     } else {
       void* args[2] = {&a, &mB};

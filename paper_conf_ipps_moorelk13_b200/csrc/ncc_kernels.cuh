@@ -1599,16 +1599,17 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
 // ================================================================== PIV, persistent + warp-specialised, balanced core
 // piv_ws_kernel spreads (2m+1) x ceil((2m+1)/RV) items over 13 consumer warps: the SMSP that
 // holds 4 of them sets the pace (13/16 of the FMA pipe) and 7 of every 72 columns are padding.
-// Here the consumers own exactly the 2m_y x 2m_x core of the offset grid -- NCW warps, two per
-// SMSP, RV = 16 shifts per lane, no padding -- and the producer warps, otherwise idle while a
-// window is correlated, compute the (2m_x+1) + 2m_y border offsets (last row dy = +m_y, last
-// column dx = +m_x) with scalar FFMA from the same staged stage.  Items of a warp: 8 output rows
-// x 4 column groups, laid out so each 8-lane LDS.128 phase covers 4 rows x 2 groups and the
+// Here the consumers own exactly the 2m_y x 2m_x core of each offset grid -- NCW warps, two
+// per SMSP, RV = 16 shifts per lane, no padding -- and the producer warps, otherwise idle while
+// a window is correlated, compute the (2m_x+1) + 2m_y border offsets (last row dy = +m_y, last
+// column dx = +m_x) from the same staged stage.  A stage holds WPS windows (cfg 4: one 64x64
+// window; cfg 3: four 32x32 windows) so that every consumer lane owns RV core offsets.
+// Consumer lane layout: each 8-lane LDS.128 phase covers 4 rows x 2 column groups and the
 // staged pitch (BP = 4 mod 32 floats) puts them on 8 distinct 16-B bank groups.
 __host__ __device__ constexpr int piv_ws2_pitch(int TW, int MX, int CW) {
   return (((2 * MX + ((TW + CW - 1) / CW) * CW) - 4 + 31) / 32) * 32 + 4;
 }
-template <int TH, int TW, int MY, int MX, int RV, int CW>
+template <int TH, int TW, int MY, int MX, int RV, int CW, int WPS>
 struct PivWs2Shape {
   static constexpr int OY = 2 * MY + 1, OX = 2 * MX + 1, OYc = 2 * MY, OXc = 2 * MX, NG = OXc / RV;
   static constexpr int nCW = TW / CW, PB = CW + 2, TPP = nCW * PB, BR = TH + 2 * MY;
@@ -1616,31 +1617,37 @@ struct PivWs2Shape {
   static constexpr int SP = (OX + 3) & ~3;  // score tile pitch
   static constexpr int tp_fl = ((TH * TPP * 2 + 31) / 32) * 32, b_fl = ((BR * BP + 31) / 32) * 32;
   static constexpr int s_fl = ((OY * SP + 31) / 32) * 32;
-  static constexpr int NE = OX + OYc;  // border offsets computed by the producers
-  static constexpr int smem_bytes = (2 * (tp_fl + b_fl) + s_fl) * 4;
+  static constexpr int stage_fl = WPS * (tp_fl + b_fl);
+  static constexpr int NE = OX + OYc;      // border offsets of one window (producers)
+  static constexpr int RPW = 32 / NG;      // core rows per consumer warp
+  static constexpr int WPW = OYc / RPW;    // consumer warps per window
+  static constexpr int smem_bytes = (2 * stage_fl + WPS * s_fl) * 4;
 };
-template <int TH, int TW, int MY, int MX, int RV, int CW, int NCW, int NPW>
+template <int TH, int TW, int MY, int MX, int RV, int CW, int NCW, int NPW, int WPS>
 __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
     piv_ws2_kernel(const PivArgs a, const __grid_constant__ CUtensorMap mapB, int nwin_total) {
-  using S = PivWs2Shape<TH, TW, MY, MX, RV, CW>;
+  using S = PivWs2Shape<TH, TW, MY, MX, RV, CW, WPS>;
   constexpr int NCT = NCW * 32, NPT = NPW * 32;
-  static_assert(RV == 16 && S::NG == 4 && S::OXc % RV == 0, "lane layout: 4 groups of 16 shifts per row");
-  static_assert(S::OYc == 8 * NCW, "one warp per 8 core rows");
-  static_assert(TW % CW == 0 && CW % 4 == 0, "whole column chunks");
+  static_assert(RV == 16 && S::OXc % RV == 0 && (S::NG == 2 || S::NG == 4), "lane layout: 2 or 4 groups per row");
+  static_assert(S::OYc % S::RPW == 0 && S::WPW * WPS == NCW, "consumer warps tile the cores of the stage");
+  static_assert(TW % CW == 0 && CW % 4 == 0 && TW % 32 == 0, "whole column chunks and 32-column lane strips");
   static_assert((S::BP / 4) % 8 == 1, "conflict-free LDS.128 phases");
-  constexpr int NEW = (S::NE + NPW - 1) / NPW;  // border offsets per producer warp: e = pw + NPW * o
-  static_assert(NEW <= 64 && TW % 32 == 0, "border: <= 2 offsets per lane, whole 32-column lane strips");
-  constexpr int EPT = 2;
+  static_assert(WPS <= NPW && NPW % WPS == 0, "producer warps split evenly over the windows of a stage");
+  constexpr int PPW = NPW / WPS;                        // producer warps per window (border offsets)
+  constexpr int NEW = (S::NE + PPW - 1) / PPW;          // border offsets per producer warp
+  constexpr int EPT = (NEW + 31) / 32;                  // ... per lane
+  constexpr int JPL = TW / 32;                          // template columns per lane (border sums)
+  static_assert((TH * TW) % NPT == 0 && NPT % TW == 0, "producer threads tile each mask in whole rows");
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   float* smem = reinterpret_cast<float*>(smem_raw);
   __shared__ __align__(8) uint64_t full_b[2], empty_b[2], scfull_b, scempty_b;
-  __shared__ double st_mean[2], st_sumsq[2], st_energy[2], st_csum[2];
-  __shared__ int st_flat[2];
-  __shared__ double pred[NPW * 4];
-  __shared__ unsigned long long pkey[NPW];
-  auto TPs = [&](int s) { return reinterpret_cast<u64*>(smem + s * (S::tp_fl + S::b_fl)); };
-  auto Bs = [&](int s) { return smem + s * (S::tp_fl + S::b_fl) + S::tp_fl; };
-  float* Sc = smem + 2 * (S::tp_fl + S::b_fl);
+  __shared__ double st_mean[2][WPS], st_sumsq[2][WPS], st_energy[2][WPS], st_csum[2][WPS];
+  __shared__ int st_flat[2][WPS];
+  __shared__ double pred[NPW * 2 * WPS];
+  __shared__ unsigned long long pkey[NPW][WPS];
+  auto TPs = [&](int s, int wi) { return reinterpret_cast<u64*>(smem + s * S::stage_fl + wi * S::tp_fl); };
+  auto Bs = [&](int s, int wi) { return smem + s * S::stage_fl + WPS * S::tp_fl + wi * S::b_fl; };
+  auto Sc = [&](int wi) { return smem + 2 * S::stage_fl + wi * S::s_fl; };
 
   const int tid = threadIdx.x;
   const int nwin = a.Ky * a.Kx;
@@ -1655,210 +1662,288 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
     fence_mbar_init();
   }
   __syncthreads();
-  const int nlocal = (nwin_total - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
-  auto win_of = [&](int k, int& lz, int& lin) {
-    const int wdx = (int)blockIdx.x + k * (int)gridDim.x;
+  const int ngroups = (nwin_total + WPS - 1) / WPS;
+  const int nlocal = (ngroups - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+  // window wi of the k-th stage group of this CTA: pair (relative to pair0) and linear index
+  auto win_of = [&](int k, int wi, int& lz, int& lin) {
+    const int wdx = ((int)blockIdx.x + k * (int)gridDim.x) * WPS + wi;
     lz = wdx / nwin;
     lin = wdx % nwin;
+    return wdx < nwin_total;
   };
   const double inv_n = 1.0 / ((double)TH * (double)TW);
 
   if (tid >= NCT) {
     // =============================== producers
     const int pt = tid - NCT, lane = tid & 31, pw = pt >> 5;
-    constexpr int PERT = (TH * TW + NPT - 1) / NPT;
-    auto reduce2 = [&](double& x0, double& x1) {  // deterministic sum over the producer threads
-      x0 = warp_sum_d(x0);
-      x1 = warp_sum_d(x1);
-      named_bar_sync(1, NPT);
-      if (lane == 0) { pred[pw * 2] = x0; pred[pw * 2 + 1] = x1; }
-      named_bar_sync(1, NPT);
-      x0 = 0.0;
-      x1 = 0.0;
-      for (int q = 0; q < NPW; ++q) { x0 += pred[q * 2]; x1 += pred[q * 2 + 1]; }
-    };
+    const int bwin = pw / PPW, bsub = pw % PPW;  // this warp's border window and its offset stride slot
+    constexpr int PERT = (WPS * TH * TW + NPT - 1) / NPT;
     auto border = [&](int e, int& dy, int& dx) {
       if (e < S::OX) { dy = S::OYc; dx = e; } else { dy = e - S::OX; dx = S::OXc; }
     };
+    auto owned = [&](int q) { return bsub + PPW * (lane + 32 * q); };  // border offset of slot q
     float ext_prev[EPT];
-    auto owned = [&](int q) { return pw + NPW * (lane + 32 * q); };  // border offset index of slot q
     auto epilogue = [&](int k) {
-      int lz, lin;
-      win_of(k, lz, lin);
-      const int s = k & 1;
       mbar_wait_backoff(&scfull_b, (uint32_t)(k & 1));
+      const int s = k & 1;
 #pragma unroll
-      for (int q = 0; q < EPT; ++q) {  // border scores of window k (computed during its core)
+      for (int q = 0; q < EPT; ++q) {  // border scores of group k (computed during its core)
         const int e = owned(q);
         if (e < S::NE) {
           int dy, dx;
           border(e, dy, dx);
-          Sc[dy * S::SP + dx] = ext_prev[q];
+          Sc(bwin)[dy * S::SP + dx] = ext_prev[q];
         }
       }
       named_bar_sync(1, NPT);
+      // normalise every offset of the stage's windows (numerators -> NCC / SSD from the fp64
+      // window sums), write the scores back for the sub-pixel fit, per-window argmax keys
       constexpr int tile = S::OY * S::OX;
-      unsigned long long best = 0ull;
-      const int pr = a.pair0 + lz;
-      for (int e = pt; e < tile; e += NPT) {
-        const int row = e / S::OX, col = e % S::OX;
-        const float sv = Sc[row * S::SP + col];
-        if (a.scores) a.scores[((int64_t)pr * nwin + lin) * tile + e] = sv;
-        const unsigned long long key = make_key(a.ssd ? -sv : sv, (uint32_t)e);
-        best = key > best ? key : best;
+      constexpr int CH = 8;  // window-sum loads in flight per thread
+      unsigned long long best[WPS];
+#pragma unroll
+      for (int wi = 0; wi < WPS; ++wi) {
+        best[wi] = 0ull;
+        int lz, lin;
+        if (!win_of(k, wi, lz, lin)) continue;
+        const int y0 = (lin / a.Kx) * a.sy, x0 = (lin % a.Kx) * a.sx;  // map origin (y - m_y, x - m_x)
+        const double* S1f = a.S1 + (int64_t)lz * a.map_frame_stride + (int64_t)y0 * a.map_pitch + x0;
+        const double* S2f = a.S2 + (int64_t)lz * a.map_frame_stride + (int64_t)y0 * a.map_pitch + x0;
+        const double csum = st_csum[s][wi], energy = st_energy[s][wi], tmean = st_mean[s][wi],
+                     tsq = st_sumsq[s][wi];
+        const bool flat = st_flat[s][wi] != 0;
+        float* T = Sc(wi);
+        float* gsc = a.scores ? a.scores + ((int64_t)(a.pair0 + lz) * nwin + lin) * tile : nullptr;
+        unsigned long long bw = 0ull;
+        for (int e0 = pt; e0 < tile; e0 += CH * NPT) {
+          double w1[CH], w2[CH];
+#pragma unroll
+          for (int c = 0; c < CH; ++c) {
+            const int e = e0 + c * NPT;
+            if (e < tile) {
+              const int64_t mi = (int64_t)(e / S::OX) * a.map_pitch + e % S::OX;
+              w1[c] = __ldg(S1f + mi);
+              w2[c] = __ldg(S2f + mi);
+            }
+          }
+#pragma unroll
+          for (int c = 0; c < CH; ++c) {
+            const int e = e0 + c * NPT;
+            if (e < tile) {
+              float* tp = T + (e / S::OX) * S::SP + e % S::OX;
+              const float num = *tp;
+              const float sv = a.ssd ? (float)(tsq - 2.0 * ((double)num + tmean * w1[c]) + w2[c])
+                                     : ncc_normalize_fast(num, w1[c], w2[c], inv_n, csum, energy, flat);
+              *tp = sv;
+              if (gsc) gsc[e] = sv;
+              const unsigned long long key = make_key(a.ssd ? -sv : sv, (uint32_t)e);
+              bw = key > bw ? key : bw;
+            }
+          }
+        }
+        best[wi] = bw;
       }
-      best = warp_max_key(best);
-      if (lane == 0) pkey[pw] = best;
+#pragma unroll
+      for (int wi = 0; wi < WPS; ++wi) {
+        best[wi] = warp_max_key(best[wi]);
+        if (lane == 0) pkey[pw][wi] = best[wi];
+      }
       named_bar_sync(1, NPT);
-      if (pt == 0) {
-        unsigned long long bk = 0ull;
-        for (int q = 0; q < NPW; ++q) bk = pkey[q] > bk ? pkey[q] : bk;
-        const uint32_t kk = key_index(bk);
-        const int row = (int)(kk / S::OX), col = (int)(kk % S::OX);
-        const int iy = row - MY, ix = col - MX;
-        uint32_t flags = (st_flat[s] && !a.ssd) ? (kFlatTemplate | kInvalid) : 0u;
-        double ddy = 0.0, ddx = 0.0;
-        bool par = false;
-        if (row == 0 || row == S::OY - 1) {
-          flags |= kEdgeY;
-        } else {
-          const double cm = Sc[(row - 1) * S::SP + col], c0 = Sc[row * S::SP + col], cp = Sc[(row + 1) * S::SP + col];
-          ddy = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
-          if (par) flags |= kParabolaY;
+      if (pt < WPS) {
+        const int wi = pt;
+        int lz, lin;
+        if (win_of(k, wi, lz, lin)) {
+          const float* T = Sc(wi);
+          unsigned long long bk = 0ull;
+          for (int q = 0; q < NPW; ++q) bk = pkey[q][wi] > bk ? pkey[q][wi] : bk;
+          const uint32_t kk = key_index(bk);
+          const int row = (int)(kk / S::OX), col = (int)(kk % S::OX);
+          const int iy = row - MY, ix = col - MX;
+          uint32_t flags = (st_flat[s][wi] && !a.ssd) ? (kFlatTemplate | kInvalid) : 0u;
+          double ddy = 0.0, ddx = 0.0;
+          bool par = false;
+          if (row == 0 || row == S::OY - 1) {
+            flags |= kEdgeY;
+          } else {
+            const double cm = T[(row - 1) * S::SP + col], c0 = T[row * S::SP + col], cp = T[(row + 1) * S::SP + col];
+            ddy = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
+            if (par) flags |= kParabolaY;
+          }
+          par = false;
+          if (col == 0 || col == S::OX - 1) {
+            flags |= kEdgeX;
+          } else {
+            const double cm = T[row * S::SP + col - 1], c0 = T[row * S::SP + col], cp = T[row * S::SP + col + 1];
+            ddx = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
+            if (par) flags |= kParabolaX;
+          }
+          VecOut o;
+          o.iy = iy;
+          o.ix = ix;
+          o.dy = (float)(iy + ddy);
+          o.dx = (float)(ix + ddx);
+          o.score = a.ssd ? -key_score(bk) : key_score(bk);
+          o.flags = flags;
+          a.vec[(int64_t)(a.pair0 + lz) * nwin + lin] = o;
         }
-        par = false;
-        if (col == 0 || col == S::OX - 1) {
-          flags |= kEdgeX;
-        } else {
-          const double cm = Sc[row * S::SP + col - 1], c0 = Sc[row * S::SP + col], cp = Sc[row * S::SP + col + 1];
-          ddx = a.ssd ? subpix3_min(cm, c0, cp, a.subpix) : subpix3(cm, c0, cp, a.subpix, &par);
-          if (par) flags |= kParabolaX;
-        }
-        VecOut o;
-        o.iy = iy;
-        o.ix = ix;
-        o.dy = (float)(iy + ddy);
-        o.dx = (float)(ix + ddx);
-        o.score = a.ssd ? -key_score(bk) : key_score(bk);
-        o.flags = flags;
-        a.vec[(int64_t)pr * nwin + lin] = o;
-        mbar_arrive(&scempty_b);  // the score tile may be overwritten
       }
-      named_bar_sync(1, NPT);  // pkey / stats reuse
+      named_bar_sync(1, NPT);  // every score tile read; pkey / stats reusable
+      if (pt == 0) mbar_arrive(&scempty_b);  // the score tiles may be overwritten
     };
     for (int k = 0; k < nlocal; ++k) {
       const int s = k & 1;
-      int lz, lin;
-      win_of(k, lz, lin);
-      const int pr = a.pair0 + lz;
-      const int y = MY + (lin / a.Kx) * a.sy, x = MX + (lin % a.Kx) * a.sx;
+      int wy[WPS], wx[WPS], wz[WPS];
+      bool wv[WPS];
+      int nvalid = 0;
+#pragma unroll
+      for (int wi = 0; wi < WPS; ++wi) {
+        int lz, lin;
+        wv[wi] = win_of(k, wi, lz, lin);
+        wz[wi] = a.pair0 + lz;
+        wy[wi] = MY + (lin / a.Kx) * a.sy;
+        wx[wi] = MX + (lin % a.Kx) * a.sx;
+        nvalid += wv[wi] ? 1 : 0;
+      }
       if (k >= 2) mbar_wait_bounded(&empty_b[s], (uint32_t)(((k >> 1) - 1) & 1));
       if (pt == 0) {
-        mbar_expect_tx(&full_b[s], (uint32_t)(S::BR * S::BP * 4));
-        tma_load_3d(Bs(s), &mapB, x - MX, y - MY, pr, &full_b[s]);
+        mbar_expect_tx(&full_b[s], (uint32_t)(nvalid * S::BR * S::BP * 4));
+#pragma unroll
+        for (int wi = 0; wi < WPS; ++wi)
+          if (wv[wi]) tma_load_3d(Bs(s, wi), &mapB, wx[wi] - MX, wy[wi] - MY, wz[wi], &full_b[s]);
       }
-      // mask statistics and template pairs (as piv_ncc_kernel)
-      const float* Af = a.A + (int64_t)pr * a.frame_stride;
+      // mask statistics (Fig 5.2) and template pairs, all windows of the stage at once; element
+      // pt + q*NPT of the stage = window q / QPW, row pt / TW + (q % QPW) * RPQ, column pt % TW
+      constexpr int QPW = TH * TW / NPT, RPQ = NPT / TW;
+      const int pr0 = pt / TW, pc0 = pt % TW;
       float mv[PERT];
 #pragma unroll
-      for (int q = 0; q < PERT; ++q) {
-        const int e = pt + q * NPT;
-        mv[q] = e < TH * TW ? __ldg(Af + (int64_t)(y + e / TW) * a.pitch + x + e % TW) : 0.0f;
+      for (int wi = 0; wi < WPS; ++wi) {
+        const float* Aw = a.A + (int64_t)wz[wi] * a.frame_stride + (int64_t)(wy[wi] + pr0) * a.pitch + wx[wi] + pc0;
+#pragma unroll
+        for (int q = 0; q < QPW; ++q) mv[wi * QPW + q] = wv[wi] ? __ldg(Aw + (int64_t)(q * RPQ) * a.pitch) : 0.0f;
       }
-      double s1 = 0.0, s2 = 0.0;
+      double v[2 * WPS];
 #pragma unroll
-      for (int q = 0; q < PERT; ++q) { s1 += (double)mv[q]; s2 += (double)mv[q] * (double)mv[q]; }
-      reduce2(s1, s2);
-      const double mean = s1 * inv_n;
-      double e2 = 0.0, cs = 0.0;
-      u64* tpw = TPs(s);
+      for (int wi = 0; wi < 2 * WPS; ++wi) v[wi] = 0.0;
 #pragma unroll
       for (int q = 0; q < PERT; ++q) {
-        const int e = pt + q * NPT;
-        if (e < TH * TW) {
-          const int i = e / TW, j = e % TW;
-          const double d = (double)mv[q] - mean;
-          const float ac = (float)d;
-          e2 += d * d;
-          cs += (double)ac;
-          float* tp = reinterpret_cast<float*>(tpw + i * S::TPP + (j / CW) * S::PB);
-          const int l = j % CW;
-          tp[2 * l + 1] = ac;
-          tp[2 * (l + 1)] = ac;
-          if (l == 0) tp[0] = 0.0f;
-          if (l == CW - 1) tp[2 * CW + 1] = 0.0f;
+        const int wi = q / QPW;
+        const double t = (double)mv[q];
+#pragma unroll
+        for (int w2 = 0; w2 < WPS; ++w2)
+          if (w2 == wi) { v[2 * w2] += t; v[2 * w2 + 1] += t * t; }
+      }
+      auto reduce = [&]() {  // deterministic sums over the producer threads
+#pragma unroll
+        for (int j = 0; j < 2 * WPS; ++j) v[j] = warp_sum_d(v[j]);
+        named_bar_sync(1, NPT);
+        if (lane == 0)
+#pragma unroll
+          for (int j = 0; j < 2 * WPS; ++j) pred[pw * 2 * WPS + j] = v[j];
+        named_bar_sync(1, NPT);
+#pragma unroll
+        for (int j = 0; j < 2 * WPS; ++j) {
+          double r = 0.0;
+          for (int q = 0; q < NPW; ++q) r += pred[q * 2 * WPS + j];
+          v[j] = r;
         }
+      };
+      reduce();
+      double mean[WPS], sumsq[WPS];
+#pragma unroll
+      for (int wi = 0; wi < WPS; ++wi) {
+        mean[wi] = v[2 * wi] * inv_n;
+        sumsq[wi] = v[2 * wi + 1];
+        v[2 * wi] = 0.0;
+        v[2 * wi + 1] = 0.0;
       }
-      reduce2(e2, cs);
-      const bool flat = e2 <= kFlatRel * s2;
-      if (pt == 0) {
-        st_mean[s] = mean;
-        st_sumsq[s] = s2;
-        st_energy[s] = e2;
-        st_csum[s] = cs;
-        st_flat[s] = flat ? 1 : 0;
+#pragma unroll
+      for (int q = 0; q < PERT; ++q) {
+        const int wi = q / QPW, i = pr0 + (q % QPW) * RPQ, j = pc0;
+        double mm = 0.0;
+#pragma unroll
+        for (int w2 = 0; w2 < WPS; ++w2) mm = (w2 == wi) ? mean[w2] : mm;
+        const double d = (double)mv[q] - mm;
+        const float ac = (float)d;
+#pragma unroll
+        for (int w2 = 0; w2 < WPS; ++w2)
+          if (w2 == wi) { v[2 * w2] += d * d; v[2 * w2 + 1] += (double)ac; }
+        float* tp = reinterpret_cast<float*>(TPs(s, wi) + i * S::TPP + (j / CW) * S::PB);
+        const int l = j % CW;
+        tp[2 * l + 1] = ac;
+        tp[2 * (l + 1)] = ac;
+        if (l == 0) tp[0] = 0.0f;
+        if (l == CW - 1) tp[2 * CW + 1] = 0.0f;
+      }
+      reduce();
+      if (pt < WPS) {
+        double mm = 0, ss = 0, ee = 0, cc = 0;
+#pragma unroll
+        for (int w2 = 0; w2 < WPS; ++w2)
+          if (w2 == pt) { mm = mean[w2]; ss = sumsq[w2]; ee = v[2 * w2]; cc = v[2 * w2 + 1]; }
+        st_mean[s][pt] = mm;
+        st_sumsq[s][pt] = ss;
+        st_energy[s][pt] = ee;
+        st_csum[s][pt] = cc;
+        st_flat[s][pt] = (ee <= kFlatRel * ss) ? 1 : 0;
       }
       named_bar_sync(1, NPT);  // template pairs + stats of all producers written
       if (pt == 0) mbar_arrive(&full_b[s]);
-      // border offsets of window k: same products and row-blocked partials as the core
-      mbar_wait_bounded(&full_b[s], (uint32_t)((k >> 1) & 1));  // search region landed
-      // Lanes split the template columns (j = lane + 32c), each warp walks its NEW border
-      // offsets per template row: conflict-free scalar loads of the region, the template value
-      // loaded once per row; per-lane fp32 sums over <= 2*TH products, then a butterfly sum.
+      // Border offsets of this warp's window: lanes split the template columns (j = lane + 32c),
+      // the warp walks up to 32 offsets per pass; conflict-free scalar loads of the region, the
+      // template value loaded once per row; per-lane fp32 sums over <= JPL*TH products, then a
+      // butterfly sum across the lanes.
+      mbar_wait_bounded(&full_b[s], (uint32_t)((k >> 1) & 1));  // search regions landed
       float ext_cur[EPT];
-      {
-        constexpr int JPL = TW / 32;
-        const float* tpf = reinterpret_cast<const float*>(tpw);
-        const float* bs = Bs(s) + lane;
-        int boff[NEW];
 #pragma unroll
-        for (int o = 0; o < NEW; ++o) {
-          const int e = pw + NPW * o;
-          int dy = 0, dx = 0;
-          if (e < S::NE) border(e, dy, dx);
-          boff[o] = dy * S::BP + dx;
-        }
-        float acc[NEW];
+      for (int q = 0; q < EPT; ++q) ext_cur[q] = 0.0f;
+      bool bvalid = false;
 #pragma unroll
-        for (int o = 0; o < NEW; ++o) acc[o] = 0.0f;
-#pragma unroll 1
-        for (int i = 0; i < TH; ++i) {
-          float tv[JPL];
-#pragma unroll
-          for (int c = 0; c < JPL; ++c) {
-            const int j = lane + 32 * c;
-            tv[c] = tpf[(i * S::TPP + (j / CW) * S::PB) * 2 + 1 + 2 * (j % CW)];
-          }
-          const float* br = bs + i * S::BP;
-#pragma unroll
-          for (int o = 0; o < NEW; ++o)
-#pragma unroll
-            for (int c = 0; c < JPL; ++c) acc[o] = fmaf(tv[c], br[boff[o] + 32 * c], acc[o]);
-        }
-        float mine[EPT] = {0.0f, 0.0f};
-#pragma unroll
-        for (int o = 0; o < NEW; ++o) {
-          float v = acc[o];
-#pragma unroll
-          for (int d = 16; d; d >>= 1) v += __shfl_xor_sync(0xffffffffu, v, d);
-          if (o == lane) mine[0] = v;
-          if (o == lane + 32) mine[1] = v;
-        }
-        const double* S1f = a.S1 + (int64_t)lz * a.map_frame_stride;
-        const double* S2f = a.S2 + (int64_t)lz * a.map_frame_stride;
+      for (int w2 = 0; w2 < WPS; ++w2) bvalid = (w2 == bwin) ? wv[w2] : bvalid;
+      if (bvalid) {
+        const float* tpf = reinterpret_cast<const float*>(TPs(s, bwin));
+        const float* bs = Bs(s, bwin) + lane;
 #pragma unroll
         for (int q = 0; q < EPT; ++q) {
-          const int e = owned(q);
-          float v = 0.0f;
-          if (e < S::NE) {
-            int dy, dx;
-            border(e, dy, dx);
-            const int64_t mi = (int64_t)(y - MY + dy) * a.map_pitch + (x - MX + dx);
-            const double ws1 = __ldg(S1f + mi), ws2 = __ldg(S2f + mi);
-            v = a.ssd ? (float)(s2 - 2.0 * ((double)mine[q] + mean * ws1) + ws2)
-                      : ncc_normalize_fast(mine[q], ws1, ws2, inv_n, cs, e2, flat);
+          constexpr int NP = 32;
+          int boff[NP];
+#pragma unroll
+          for (int o = 0; o < NP; ++o) {
+            const int e = bsub + PPW * (32 * q + o);
+            int dy = 0, dx = 0;
+            if (e < S::NE) border(e, dy, dx);
+            boff[o] = dy * S::BP + dx;
           }
-          ext_cur[q] = v;
+          const int nact = min(NP, NEW - 32 * q);  // offsets of this pass (warp-uniform)
+          float acc[NP];
+#pragma unroll
+          for (int o = 0; o < NP; ++o) acc[o] = 0.0f;
+#pragma unroll 1
+          for (int i = 0; i < TH; ++i) {
+            float tv[JPL];
+#pragma unroll
+            for (int c = 0; c < JPL; ++c) {
+              const int j = lane + 32 * c;
+              tv[c] = tpf[(i * S::TPP + (j / CW) * S::PB) * 2 + 1 + 2 * (j % CW)];
+            }
+            const float* br = bs + i * S::BP;
+#pragma unroll
+            for (int o = 0; o < NP; ++o)
+              if (o < nact)
+#pragma unroll
+                for (int c = 0; c < JPL; ++c) acc[o] = fmaf(tv[c], br[boff[o] + 32 * c], acc[o]);
+          }
+          float mine = 0.0f;
+#pragma unroll
+          for (int o = 0; o < NP; ++o) {
+            if (o < nact) {
+              float x = acc[o];
+#pragma unroll
+              for (int d = 16; d; d >>= 1) x += __shfl_xor_sync(0xffffffffu, x, d);
+              if (o == lane) mine = x;
+            }
+          }
+          ext_cur[q] = mine;  // raw numerator; normalised with the core in the epilogue
         }
       }
       if (k >= 1) epilogue(k - 1);
@@ -1867,23 +1952,26 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
     }
     if (nlocal >= 1) epilogue(nlocal - 1);
   } else {
-    // =============================== consumers: 8 core rows x 4 groups of RV shifts per warp
+    // =============================== consumers: RPW core rows x NG groups of RV shifts per warp
     const int wq = tid >> 5, l = tid & 31, ph = l >> 3, q8 = l & 7;
-    const int row = wq * 8 + 4 * (ph >> 1) + (q8 & 3);
-    const int g = (q8 >> 2) + 2 * (ph & 1);
+    constexpr int PHR = S::NG / 2;  // 8-lane phases per 4-row block
+    const int wi = wq / S::WPW;
+    const int row = (wq % S::WPW) * S::RPW + 4 * (ph / PHR) + (q8 & 3);
+    const int g = (q8 >> 2) + 2 * (ph % PHR);
     for (int k = 0; k < nlocal; ++k) {
       const int s = k & 1;
       int lz, lin;
-      win_of(k, lz, lin);
-      const int y = MY + (lin / a.Kx) * a.sy, x = MX + (lin % a.Kx) * a.sx;
+      const bool valid = win_of(k, wi, lz, lin);
       mbar_wait_bounded(&full_b[s], (uint32_t)((k >> 1) & 1));
       float out[RV];
-      {
+#pragma unroll
+      for (int c = 0; c < RV; ++c) out[c] = 0.0f;
+      if (valid) {
         u64 tot2[RV / 2];
 #pragma unroll
         for (int q = 0; q < RV / 2; ++q) tot2[q] = 0ull;
-        const float* brow = Bs(s) + row * S::BP + g * RV;
-        const u64* tpw = TPs(s);
+        const float* brow = Bs(s, wi) + row * S::BP + g * RV;
+        const u64* tpw = TPs(s, wi);
 #pragma unroll 1
         for (int i = 0; i < TH; ++i) {
 #pragma unroll
@@ -1891,37 +1979,20 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
             u64 part2[RV / 2];
 #pragma unroll
             for (int q = 0; q < RV / 2; ++q) part2[q] = 0ull;
-#ifdef NCC_WS2_XMAJOR
-            row_dot_pairs_x<RV, CW>(brow + i * S::BP + jc * CW, tpw + i * S::TPP + jc * S::PB, part2);
-#else
             row_dot_pairs<RV, CW>(brow + i * S::BP + jc * CW, tpw + i * S::TPP + jc * S::PB, part2);
-#endif
 #pragma unroll
             for (int q = 0; q < RV / 2; ++q) add2(tot2[q], part2[q]);
           }
         }
-        const double csum = st_csum[s], energy = st_energy[s], tmean = st_mean[s], tsq = st_sumsq[s];
-        const bool flat = st_flat[s] != 0;
-        const double* S1f = a.S1 + (int64_t)lz * a.map_frame_stride;
-        const double* S2f = a.S2 + (int64_t)lz * a.map_frame_stride;
-        const int64_t mrow = (int64_t)(y - MY + row) * a.map_pitch + (x - MX) + g * RV;
 #pragma unroll
-        for (int q = 0; q < RV / 2; ++q) {
-          const float lo = __uint_as_float((uint32_t)(tot2[q] & 0xFFFFFFFFull));
-          const float hi = __uint_as_float((uint32_t)(tot2[q] >> 32));
-#pragma unroll
-          for (int e = 0; e < 2; ++e) {
-            const int c = 2 * q + 1 - e;
-            const double s1 = __ldg(S1f + mrow + c), s2 = __ldg(S2f + mrow + c);
-            const float num = e == 0 ? lo : hi;
-            out[c] = a.ssd ? (float)(tsq - 2.0 * ((double)num + tmean * s1) + s2)
-                           : ncc_normalize_fast(num, s1, s2, inv_n, csum, energy, flat);
-          }
+        for (int q = 0; q < RV / 2; ++q) {  // raw numerators; the producers normalise
+          out[2 * q + 1] = __uint_as_float((uint32_t)(tot2[q] & 0xFFFFFFFFull));
+          out[2 * q] = __uint_as_float((uint32_t)(tot2[q] >> 32));
         }
       }
-      mbar_arrive(&empty_b[s]);  // done reading stage s (pairs, region, stats)
+      mbar_arrive(&empty_b[s]);  // done reading stage s (pairs, regions, stats)
       if (k >= 1) mbar_wait_bounded(&scempty_b, (uint32_t)((k - 1) & 1));
-      float* sc = Sc + row * S::SP + g * RV;
+      float* sc = Sc(wi) + row * S::SP + g * RV;
 #pragma unroll
       for (int c = 0; c < RV; c += 4) *reinterpret_cast<float4*>(sc + c) = make_float4(out[c], out[c + 1], out[c + 2], out[c + 3]);
       mbar_arrive(&scfull_b);

@@ -41,3 +41,13 @@ for name, rg in list(regions.items()) + [("rest", [k for k in range(len(data)) i
     print(f"== {name}: samples {s}, warp-instructions {ninst}")
     print("   stalls:", ", ".join(f"{h} {v} ({100 * v / max(s, 1):.0f}%)" for h, v in c.most_common(8)))
     print("   ops:", ", ".join(f"{o} {v}" for o, v in opc.most_common(8)))
+
+if len(sys.argv) > 2:  # top instructions by samples outside the core loop
+    top = int(sys.argv[2])
+    rest = [(int(float(data[k][iall] or 0)), k) for k in range(len(data)) if not (lo <= k <= hi)]
+    rest.sort(reverse=True)
+    print(f"== top {top} sampled instructions outside the core loop (index, samples, reasons, source)")
+    for smp, k in rest[:top]:
+        r = data[k]
+        rs = sorted(((int(float(r[i] or 0)), h) for i, h in sc), reverse=True)[:3]
+        print(f"{k:6d} {smp:7d}  {', '.join(f'{h}:{v}' for v, h in rs if v):50s} {r[isrc][:70]}")
