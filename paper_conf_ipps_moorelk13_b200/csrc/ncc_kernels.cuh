@@ -173,8 +173,8 @@ __device__ __forceinline__ void mbar_wait_bounded(uint64_t* bar, uint32_t parity
 // Long waits of otherwise idle warps (a producer waiting for a window's core): back off with
 // nanosleep so the spinning does not take issue slots from the warps doing the work.
 __device__ __forceinline__ void mbar_wait_backoff(uint64_t* bar, uint32_t parity) {
-  uint32_t done = 0;
-  for (long long it = 0; it < (1ll << 28); ++it) {
+  uint32_t done = 0, ns = 64;
+  for (long long it = 0; it < (1ll << 26); ++it) {
     asm volatile(
         "{\n\t.reg .pred P;\n\t"
         "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
@@ -183,7 +183,8 @@ __device__ __forceinline__ void mbar_wait_backoff(uint64_t* bar, uint32_t parity
         : "r"(smem_u32(bar)), "r"(parity)
         : "memory");
     if (done) return;
-    __nanosleep(200);
+    __nanosleep(ns);
+    ns = ns < 2048 ? 2 * ns : ns;
   }
   __trap();
 }
@@ -1596,6 +1597,24 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
   }
 }
 
+// Sum of v[i] over the 32 lanes of a warp, for all 32 i at once: each level keeps half of the
+// values and swaps the other half with the partner lane (16 + 8 + 4 + 2 + 1 shuffles); lane l
+// ends with the total of v[l].
+__device__ __forceinline__ float warp_transpose_sum32(float (&v)[32]) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int d = 16; d >= 1; d >>= 1) {
+    const bool up = (lane & d) != 0;
+#pragma unroll
+    for (int i = 0; i < d; ++i) {
+      const float send = up ? v[i] : v[i + d];
+      const float keep = up ? v[i + d] : v[i];
+      v[i] = keep + __shfl_xor_sync(0xffffffffu, send, d);
+    }
+  }
+  return v[0];
+}
+
 // ================================================================== PIV, persistent + warp-specialised, balanced core
 // piv_ws_kernel spreads (2m+1) x ceil((2m+1)/RV) items over 13 consumer warps: the SMSP that
 // holds 4 of them sets the pace (13/16 of the FMA pipe) and 7 of every 72 columns are padding.
@@ -1903,47 +1922,39 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
       if (bvalid) {
         const float* tpf = reinterpret_cast<const float*>(TPs(s, bwin));
         const float* bs = Bs(s, bwin) + lane;
+        // one pass over the rows for all NEW offsets of the warp (offsets past NE compute
+        // harmless products from the staged region and are dropped)
+        int boff[NEW];
+#pragma unroll
+        for (int o = 0; o < NEW; ++o) {
+          const int e = bsub + PPW * o;
+          int dy = 0, dx = 0;
+          if (e < S::NE) border(e, dy, dx);
+          boff[o] = dy * S::BP + dx;
+        }
+        float acc[EPT * 32];
+#pragma unroll
+        for (int o = 0; o < EPT * 32; ++o) acc[o] = 0.0f;
+#pragma unroll 1
+        for (int i = 0; i < TH; ++i) {
+          float tv[JPL];
+#pragma unroll
+          for (int c = 0; c < JPL; ++c) {
+            const int j = lane + 32 * c;
+            tv[c] = tpf[(i * S::TPP + (j / CW) * S::PB) * 2 + 1 + 2 * (j % CW)];
+          }
+          const float* br = bs + i * S::BP;
+#pragma unroll
+          for (int o = 0; o < NEW; ++o)
+#pragma unroll
+            for (int c = 0; c < JPL; ++c) acc[o] = fmaf(tv[c], br[boff[o] + 32 * c], acc[o]);
+        }
 #pragma unroll
         for (int q = 0; q < EPT; ++q) {
-          constexpr int NP = 32;
-          int boff[NP];
+          float blk[32];
 #pragma unroll
-          for (int o = 0; o < NP; ++o) {
-            const int e = bsub + PPW * (32 * q + o);
-            int dy = 0, dx = 0;
-            if (e < S::NE) border(e, dy, dx);
-            boff[o] = dy * S::BP + dx;
-          }
-          const int nact = min(NP, NEW - 32 * q);  // offsets of this pass (warp-uniform)
-          float acc[NP];
-#pragma unroll
-          for (int o = 0; o < NP; ++o) acc[o] = 0.0f;
-#pragma unroll 1
-          for (int i = 0; i < TH; ++i) {
-            float tv[JPL];
-#pragma unroll
-            for (int c = 0; c < JPL; ++c) {
-              const int j = lane + 32 * c;
-              tv[c] = tpf[(i * S::TPP + (j / CW) * S::PB) * 2 + 1 + 2 * (j % CW)];
-            }
-            const float* br = bs + i * S::BP;
-#pragma unroll
-            for (int o = 0; o < NP; ++o)
-              if (o < nact)
-#pragma unroll
-                for (int c = 0; c < JPL; ++c) acc[o] = fmaf(tv[c], br[boff[o] + 32 * c], acc[o]);
-          }
-          float mine = 0.0f;
-#pragma unroll
-          for (int o = 0; o < NP; ++o) {
-            if (o < nact) {
-              float x = acc[o];
-#pragma unroll
-              for (int d = 16; d; d >>= 1) x += __shfl_xor_sync(0xffffffffu, x, d);
-              if (o == lane) mine = x;
-            }
-          }
-          ext_cur[q] = mine;  // raw numerator; normalised with the core in the epilogue
+          for (int o = 0; o < 32; ++o) blk[o] = acc[32 * q + o];
+          ext_cur[q] = warp_transpose_sum32(blk);  // raw numerator of offset owned(q)
         }
       }
       if (k >= 1) epilogue(k - 1);
