@@ -17,6 +17,7 @@
 #include <fstream>
 #include <sstream>
 
+#include <algorithm>
 #include <chrono>
 #include <cstdio>
 #include <cstdlib>
@@ -108,9 +109,9 @@ EncodeTiledFn encode_fn() {
   return fn;
 }
 
-// fp32 tensor map of `rank` dims (innermost first), strides in bytes for dims 1..rank-1.
+// fp32 (or 8-byte element) tensor map of `rank` dims (innermost first), strides in bytes for dims 1..rank-1.
 bool encode_f32(CUtensorMap* m, const void* base, int rank, const uint64_t* dims, const uint64_t* strides_bytes,
-                const uint32_t* box) {
+                const uint32_t* box, bool u64 = false) {
   EncodeTiledFn fn = encode_fn();
   if (!fn) return false;
   cuuint64_t gd[3], gs[2];
@@ -120,7 +121,8 @@ bool encode_f32(CUtensorMap* m, const void* base, int rank, const uint64_t* dims
     bx[i] = box[i];
   }
   for (int i = 0; i + 1 < rank; ++i) gs[i] = strides_bytes[i];
-  return fn(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (cuuint32_t)rank, const_cast<void*>(base), gd, gs, bx, es,
+  return fn(m, u64 ? CU_TENSOR_MAP_DATA_TYPE_UINT64 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, (cuuint32_t)rank,
+            const_cast<void*>(base), gd, gs, bx, es,
             CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
@@ -311,6 +313,7 @@ struct ncc_plan_s {
   double *RS1, *RS2, *S1, *S2;
   int64_t rs_frame_stride, s_frame_stride;
   int box_r, box_iwp, box_smem, nsm;  // fused window-sum kernel (box_smem 0: two-pass fallback)
+  float* tc_img2 = nullptr;  // band rows as (tf32 hi, lo) pairs for the tensor-core numerator
   // tensor-core numerator (tm_tc_kernel): 0 = CUDA-core path
   int tc, tc_wc, tc_nbi, tc_nbj, tc_vtiles, tc_useg, tc_nseg;
   float *tcB, *tc_part;
@@ -351,6 +354,7 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->RS1);
   cudaFree(pl->tcB);
   cudaFree(pl->tc_part);
+  cudaFree(pl->tc_img2);
   cudaFree(pl->RS2);
   cudaFree(pl->S1);
   cudaFree(pl->S2);
@@ -463,8 +467,19 @@ ncc_status setup_tc(ncc_plan pl) {
       const int useg = ceil_div(pl->Ub, nseg);
       const int64_t ctas = per_seg * ceil_div(pl->Ub, useg);
       const int64_t waves = (ctas + pl->nsm - 1) / pl->nsm;
-      const double cost = (double)waves * (double)(ceil_div(useg + tc::kHB - 1, tc::kG) * tc::kG) * (wc / tc::kWB);
-      if (cost < best * 0.999) {
+      // cycles of a CTA: per stage ~230 cycles of fixed cost + 12 MMAs of 68 x N/136 cycles,
+      // N = the group's trimmed window (tm_tc_kernel: ramp-in / ramp-out rows cover fewer columns)
+      double cta = 0.0;
+      const int ngrp = ceil_div(useg + tc::kHB - 1, tc::kG);
+      for (int g = 0; g < ngrp; ++g) {
+        const int lo = std::max(0, tc::kHB - 1 - tc::kG * g);
+        const int chi = std::min(tc::kNWin, useg + tc::kHB - 1 - tc::kG * g);
+        const int c0 = (lo / 8) * 8;
+        const int n = std::max(16, ((chi - c0 + 7) / 8) * 8);
+        cta += tc::kG * (230.0 + 12.0 * 68.0 * n / tc::kNWin);
+      }
+      const double cost = (double)waves * cta * (wc / tc::kWB);
+      if (cost < best * 0.98) {  // more segments only when clearly cheaper (per-CTA setup is not modelled)
         best = cost;
         pl->tc_wc = wc;
         pl->tc_nbj = nbj;
@@ -474,15 +489,16 @@ ncc_status setup_tc(ncc_plan pl) {
     }
     if (wc >= w) break;
   }
-  // measured B200 rates: ~1170 cycles per tensor-core stage (12 MMAs of 128 x 136 x 8, 3xTF32),
-  // ~95 useful FP32 MACs per cycle per SM on the CUDA-core path
-  const double tc_cycles = best * 1170.0;
+  // measured B200 rates: ~1050-1170 cycles per full tensor-core stage (12 MMAs of 128 x 136 x 8,
+  // 3xTF32; modelled above), ~95 useful FP32 MACs per cycle per SM on the CUDA-core path
+  const double tc_cycles = best;
   const double cc_cycles = (double)h * w * (double)pl->Ub * pl->V * p.batch / (95.0 * pl->nsm);
   if (mode < 0 && !(tc_cycles < 0.8 * cc_cycles)) return NCC_OK;
   const int nblk = pl->tc_nbi * pl->tc_nbj;
   ncc_status st;
   if ((st = dalloc(&pl->tcB, (size_t)nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
   if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
+  if ((st = dalloc(&pl->tc_img2, (size_t)2 * p.batch * pl->Hs * p.image_w))) return st;  // (hi, lo) pairs
   const int smem = tc::smem_bytes(pl->tc_wc);
   NCC_CUDA(cudaFuncSetAttribute((const void*)tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   pl->tc = 1;
@@ -877,18 +893,18 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   mark(pl, s, 2);
   CUtensorMap map_tc;
   bool tc_now = false;
-  if (pl->tc && reinterpret_cast<uintptr_t>(d_images) % 16 == 0 && p.image_pitch % 4 == 0) {
-    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
-    const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)p.image_h * p.image_pitch * 4};
+  if (pl->tc) {  // the band's rows as (hi, lo) pairs: W x Hs x batch 8-byte elements
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)pl->Hs, (uint64_t)p.batch};
+    const uint64_t strides[2] = {(uint64_t)p.image_w * 8, (uint64_t)pl->Hs * p.image_w * 8};
     const uint32_t box[3] = {(uint32_t)tc::kBoxW, 1u, 1u};
-    tc_now = encode_f32(&map_tc, d_images, 3, dims, strides, box);
+    tc_now = encode_f32(&map_tc, pl->tc_img2, 3, dims, strides, box, true);
   }
   if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
     const int nblk = pl->tc_nbi * pl->tc_nbj;
+    tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, p.batch), 128, 0, s>>>(
+        d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
+        reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * p.image_w);
     TcArgs t;
-    t.img = d_images;
-    t.pitch = p.image_pitch;
-    t.frame_stride = (int64_t)p.image_h * p.image_pitch;
     t.H = p.image_h;
     t.W = p.image_w;
     t.tcB = pl->tcB;

@@ -68,6 +68,25 @@ __device__ __forceinline__ void ld8(uint32_t addr, uint32_t (&v)[8]) {
                : "memory");
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
+// shared-window address forms (precomputed once: the generic -> shared conversion reads a
+// special register, which the MMA issuer cannot afford between two MMAs)
+__device__ __forceinline__ void commit_u32(uint32_t bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_wait_u32(uint32_t bar, uint32_t parity) {
+  uint32_t done = 0;
+  for (long long it = 0; it < (1ll << 30); ++it) {
+    asm volatile(
+        "{\n\t.reg .pred P;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+        "selp.u32 %0, 1, 0, P;\n}"
+        : "=r"(done)
+        : "r"(bar), "r"(parity)
+        : "memory");
+    if (done) return;
+  }
+  __trap();
+}
 __device__ __forceinline__ bool elect_one() {
   uint32_t pred = 0;
   asm volatile("{\n\t.reg .pred P;\n\telect.sync _|P, 0xffffffff;\n\tselp.u32 %0, 1, 0, P;\n}" : "=r"(pred));
@@ -109,7 +128,7 @@ __host__ __device__ constexpr int b_bytes(int WC) { return 2 * (WC / 4) * kLB * 
 // dynamic shared memory per CTA: the operand, padded so that one CTA fits per SM (the CTA
 // allocates all 512 TMEM columns)
 __host__ __device__ constexpr int img_off(int WC) { return ((b_bytes(WC) + 127) / 128) * 128; }
-__host__ __device__ constexpr int smem_need(int WC) { return img_off(WC) + kNImg * kBoxW * 4; }
+__host__ __device__ constexpr int smem_need(int WC) { return img_off(WC) + kNImg * kBoxW * 8; }
 __host__ __device__ constexpr int smem_bytes(int WC) { return smem_need(WC) > 120 * 1024 ? smem_need(WC) : 120 * 1024; }
 
 }  // namespace tc
@@ -130,8 +149,8 @@ __device__ int g_tc_exp;  // timing experiments (trace builds only): bit0 no A s
 #endif
 
 struct TcArgs {
-  const float* img;
-  int64_t pitch, frame_stride;
+  // the image as (tf32 hi, fp32 lo) pairs of the band's rows (tm_tc_split), read through the
+  // tensor map; H = absolute image rows (zero rows past it), u_begin = the band's first row
   int H, W;
   const float* tcB;     // [nblk][2 (hi, lo)][WC/4 planes][kLB rows][4]: reversed template blocks
   int WC;               // template columns per CTA (multiple of kWB, <= 128)
@@ -213,13 +232,15 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     if (stage_zero(q)) {
       mbar_arrive(&img_full[sl]);
     } else {
-      mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 4));
-      tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 4, &map_img, v0 + j0 + (q % nch) * kWB, ua + i0 + q / nch,
-                  f, &img_full[sl]);
+      mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 8));
+      tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 8, &map_img, v0 + j0 + (q % nch) * kWB,
+                  ua - a.u_begin + i0 + q / nch, f, &img_full[sl]);
     }
   };
   const int nreloc = (ngrp - 1) / (kRelocAt / kG);  // groups g > 0 whose window restarts at column 0
-  if (warp < 4 * kGroups) {
+  if (TC_EXP(32768) && warp != kMmaWarp) {
+    // trace experiment: the MMA warp alone
+  } else if (warp < 4 * kGroups) {
     // ===================== producers (lane v = output column v0 + v) and ring drain.
     // Group grp (warps 4 grp .. 4 grp + 3, TMEM lane quadrants 0..3) handles the stages
     // q = grp mod kNBuf, i.e. TMEM A buffer grp: the groups' latencies overlap.
@@ -234,7 +255,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       st_wait();
       fence_before();
     }
-    const float* ring = reinterpret_cast<const float*>(smem_tc + img_off(a.WC));
+    const uint2* ring = reinterpret_cast<const uint2*>(smem_tc + img_off(a.WC));
     float* part = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * a.part_frame_stride;
     // Software-pipelined producer: the operand of the group's next stage is read from the ring
     // and split while the group waits for its TMEM buffer, so the critical path from "MMAs of
@@ -245,16 +266,16 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       const int sl = q % kNImg;
       mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
       if (gtid == 0) TC_STAMP(5, q);
-      float x[kWB];
-      const bool zero = stage_zero(q);
-#pragma unroll
-      for (int k = 0; k < kWB; ++k) x[k] = (zero || TC_EXP(64)) ? 0.0f : ring[sl * kBoxW + v + k];
-      mbar_arrive(&img_empty[sl]);
+      // the split x = hi + lo was done once per image element (tm_tc_split): one 8-byte load
+      // per Hankel element, no per-lane conversion work
+      const bool zero = stage_zero(q) || TC_EXP(64);
 #pragma unroll
       for (int k = 0; k < kWB; ++k) {
-        hi[k] = to_tf32(x[k]);
-        lo[k] = __float_as_uint(x[k] - __uint_as_float(hi[k]));
+        const uint2 p = zero ? make_uint2(0u, 0u) : ring[sl * kBoxW + v + k];
+        hi[k] = p.x;
+        lo[k] = p.y;
       }
+      mbar_arrive(&img_empty[sl]);
       if (gtid == 0) TC_STAMP(1, q);
     };
     if (grp < nstage) load_split(grp);
@@ -315,19 +336,23 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
 #pragma unroll 1
     for (int k = 0; k < nreloc; ++k) {
-      // rare event: poll with back-off so the idle warps do not take issue slots from the
-      // producer and MMA warps sharing their SM sub-partitions
-      for (long long it = 0;; ++it) {
-        uint32_t done = 0;
-        asm volatile(
-            "{\n\t.reg .pred P;\n\tmbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
-            "selp.u32 %0, 1, 0, P;\n}"
-            : "=r"(done)
-            : "r"(smem_u32(&reloc_req)), "r"((uint32_t)(k & 1))
-            : "memory");
-        if (done) break;
-        if (it > (1ll << 26)) __trap();
-        __nanosleep(256);
+      // rare event: wait in the mbarrier's own suspend (try_wait), not with nanosleep polling:
+      // sleeping warps on the SM slow the MMA warp's issue (tools/microbench/umma_probe.cu)
+      if (TC_EXP(8192)) {
+        for (long long it = 0;; ++it) {
+          uint32_t done = 0;
+          asm volatile(
+              "{\n\t.reg .pred P;\n\tmbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+              "selp.u32 %0, 1, 0, P;\n}"
+              : "=r"(done)
+              : "r"(smem_u32(&reloc_req)), "r"((uint32_t)(k & 1))
+              : "memory");
+          if (done) break;
+          if (it > (1ll << 26)) __trap();
+          __nanosleep(256);
+        }
+      } else {
+        mbar_wait_bounded(&reloc_req, (uint32_t)(k & 1));
       }
       fence_after();
 #pragma unroll 1
@@ -351,59 +376,86 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       const uint64_t dlo_off = (uint64_t)(((uint32_t)npl * plane) >> 4);  // hi -> lo operand (descriptor units)
       constexpr uint64_t kKStep = (uint64_t)((2 * plane_bytes()) >> 4);   // one K-step = two planes
       int b = 0, ph = 0, ch = 0, s = 0, g = 0, nrel_done = 0;
+      (void)ch;
+      // Window trimming: the window of group g holds output rows u = kG g - kHB + 1 + c
+      // (c < kNWin); only 0 <= u < nu are kept, so during the ramp-in / ramp-out rows of the
+      // CTA (the first and last kHB - 1 image rows) the MMAs cover just the columns [c0, c0+nN)
+      // holding valid rows (8-column granularity, N >= 16).  The skipped columns belong to rows
+      // that are never drained, so the accumulated values of the kept rows are unchanged.
+      int c0 = 0, nN = kNWin;
+      auto trim = [&](int gg) {
+        const int lo = max(0, kHB - 1 - kG * gg);
+        const int chi = min(kNWin, nu + kHB - 1 - kG * gg);
+        c0 = (lo / 8) * 8;
+        nN = ((chi - c0 + 7) / 8) * 8;
+        if (nN < 16) {
+          nN = 16;
+          if (c0 + 16 > kNWin) c0 = kNWin - 16;
+        }
+        if (TC_EXP(4096)) { c0 = 0; nN = kNWin; }
+      };
       // Software-pipelined issue: the wait for stage q+1's operand happens while the last K-step
       // of stage q is still queued (the tensor pipe's queue is short; a per-stage wait between
       // the last MMA of q and the first of q+1 left it idle for a few hundred cycles per stage).
-      if (nstage > 0 && !TC_EXP(16)) mbar_wait_bounded(&a_full[0], 0u);
+      // Per stage the issuer only adds constants to precomputed uniform operands: barrier
+      // addresses are converted once, the B descriptor moves by one 16-byte row per image row,
+      // the accumulator column / instruction descriptor change once per group.
+      const uint32_t full0 = smem_u32(&a_full[0]), done0 = smem_u32(&mma_done[0]);
+      const bool leader = elect_one();
+      if (nstage > 0 && !TC_EXP(16)) mbar_wait_u32(full0, 0u);
       fence_after();
+      int q = 0;
 #pragma unroll 1
-      for (int q = 0; q < nstage; ++q) {
-        if (lane == 0) TC_STAMP(3, q);
+      for (g = 0; q < nstage; ++g) {
         const uint32_t col = (uint32_t)((g * kG) % kRelocAt);
-        if (!TC_EXP(2048) && col == 0 && g > 0 && ch == 0 && s == 0) {  // window restart: relocate the live columns first
+        if (!TC_EXP(2048) && col == 0 && g > 0) {  // window restart: relocate the live columns first
           const int qp = q - 1;  // MMAs complete in order: the last stage's completion covers all
-          mbar_wait_bounded(&mma_done[qp % kNBuf], (uint32_t)((qp / kNBuf) & 1));
+          mbar_wait_u32(done0 + 8 * (qp % kNBuf), (uint32_t)((qp / kNBuf) & 1));
           fence_after();
           fence_before();
-          if (elect_one()) mbar_arrive(&reloc_req);
+          if (leader) mbar_arrive(&reloc_req);
           __syncwarp();
           mbar_wait_bounded(&reloc_done, (uint32_t)(nrel_done & 1));
           fence_after();
           ++nrel_done;
         }
-        // B window: planes of chunk ch, starting at row kG - 1 - s of the reversed block
-        const uint64_t dh = sdesc(bhi + (uint32_t)(ch * (kWB / 4)) * plane + (uint32_t)(kG - 1 - s) * 16, plane, 128);
-        const uint64_t dl = dh + dlo_off;
-        const uint32_t ah = tbase + a_col0 + (uint32_t)(b * 2 * kWB), al = ah + kWB;
-        const uint32_t dcol = tbase + col;
-        const uint32_t id = idesc_tf32(kNWin);
-        if (elect_one()) {
+        trim(g);
+        const uint32_t dcol = tbase + col + (uint32_t)c0;
+        const uint32_t id = idesc_tf32(nN);
+        // B window of (s = 0, ch = 0): row kG - 1 + c0 of the reversed block
+        const uint64_t dg = sdesc(bhi + (uint32_t)(kG - 1 + c0) * 16, plane, 128);
+#pragma unroll 1
+        for (s = 0; s < kG && q < nstage; ++s) {
+#pragma unroll 1
+          for (ch = 0; ch < nch; ++ch, ++q) {
+            if (lane == 0) TC_STAMP(3, q);
+            const uint64_t dh = dg - (uint64_t)s + (uint64_t)(((uint32_t)ch * (kWB / 4) * plane) >> 4);
+            const uint64_t dl = dh + dlo_off;
+            const uint32_t ah = tbase + a_col0 + (uint32_t)(b * 2 * kWB), al = ah + kWB;
+            if (leader) {
 #pragma unroll
-          for (int kk = 0; kk < kWB / 8 - 1; ++kk) {
-            mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
-            mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
-            mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
+              for (int kk = 0; kk < kWB / 8 - 1; ++kk) {
+                mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
+                mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
+                mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
+              }
+            }
+            __syncwarp();
+            const int bq = b;
+            if (++b == kNBuf) { b = 0; ph ^= 1; }
+            if (q + 1 < nstage && !TC_EXP(16)) mbar_wait_u32(full0 + 8 * b, (uint32_t)ph);
+            if (!TC_EXP(16384)) fence_after();
+            if (leader) {
+              constexpr int kk = kWB / 8 - 1;
+              mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
+              mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
+              mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
+              commit_u32(done0 + 8 * bq);
+            }
+            __syncwarp();
+            if (lane == 0) TC_STAMP(4, q);
           }
         }
-        __syncwarp();
-        // advance the counters and wait for the next stage's operand under the queued MMAs
-        const int bq = b;
-        if (++b == kNBuf) { b = 0; ph ^= 1; }
-        if (++ch == nch) {
-          ch = 0;
-          if (++s == kG) { s = 0; ++g; }
-        }
-        if (q + 1 < nstage && !TC_EXP(16)) mbar_wait_bounded(&a_full[b], (uint32_t)ph);
-        fence_after();
-        if (elect_one()) {
-          constexpr int kk = kWB / 8 - 1;
-          mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
-          mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
-          mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
-          commit(&mma_done[bq]);
-        }
-        __syncwarp();
-        if (lane == 0) TC_STAMP(4, q);
       }
     }
     __syncwarp();
@@ -411,6 +463,39 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   fence_before();
   __syncthreads();
   if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, 512;" ::"r"(tbase));
+}
+
+// Image operand of the tensor-core numerator: every element of the band's rows split once into
+// (hi = tf32(x) with round-to-nearest, lo = x - hi, exact in fp32), stored as an 8-byte pair so
+// the producer warps load each Hankel element with one LDS.64.  grid = (ceil(W/4/128), rows,
+// batch), block = 128; out row r = image row row0 + r.
+__global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
+                                                   int W, int row0, uint2* __restrict__ out, int64_t out_frame_stride) {
+  const int c = (blockIdx.x * 128 + threadIdx.x) * 4;
+  if (c >= W) return;
+  const int r = blockIdx.y, f = blockIdx.z;
+  const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch + c;
+  uint2* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * W + c;
+  float x[4];
+  if (c + 4 <= W && (reinterpret_cast<uintptr_t>(src) & 15) == 0) {
+    const float4 v = __ldg(reinterpret_cast<const float4*>(src));
+    x[0] = v.x; x[1] = v.y; x[2] = v.z; x[3] = v.w;
+  } else {
+#pragma unroll
+    for (int k = 0; k < 4; ++k) x[k] = c + k < W ? __ldg(src + k) : 0.0f;
+  }
+  uint2 o[4];
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    o[k].x = tc::to_tf32(x[k]);
+    o[k].y = __float_as_uint(x[k] - __uint_as_float(o[k].x));
+  }
+  if (c + 4 <= W) {
+    reinterpret_cast<uint4*>(dst)[0] = make_uint4(o[0].x, o[0].y, o[1].x, o[1].y);
+    reinterpret_cast<uint4*>(dst)[1] = make_uint4(o[2].x, o[2].y, o[3].x, o[3].y);
+  } else {
+    for (int k = 0; c + k < W; ++k) dst[k] = o[k];
+  }
 }
 
 // Template operand: for block (bi, bj) the reversed, zero-padded rows Rv[k] = A_C[i0 + K0 - k]

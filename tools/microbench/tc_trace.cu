@@ -17,8 +17,8 @@ int main(int argc, char** argv) {
   const int nbi = 1, nbj = (w + WC - 1) / WC, vtiles = (V + 127) / 128;
   float *img, *tcB, *part;
   long long* tr;
-  cudaMalloc(&img, (size_t)H * W * 4);
-  cudaMemset(img, 0, (size_t)H * W * 4);
+  cudaMalloc(&img, (size_t)H * W * 8);  // (hi, lo) pairs, as written by tm_tc_split
+  cudaMemset(img, 0, (size_t)H * W * 8);
   cudaMalloc(&tcB, (size_t)nbi * nbj * tc::b_bytes(WC));
   cudaMemset(tcB, 0, (size_t)nbi * nbj * tc::b_bytes(WC));
   cudaMalloc(&part, (size_t)nbi * nbj * U * V * 4);
@@ -26,7 +26,7 @@ int main(int argc, char** argv) {
   cudaMemset(tr, 0, 8 * 1024 * 8);
   cudaMemcpyToSymbol(g_tc_trace, &tr, sizeof(tr));
   TcArgs a{};
-  a.img = img; a.pitch = W; a.frame_stride = (int64_t)H * W; a.H = H; a.W = W;
+  a.H = H; a.W = W;
   a.tcB = tcB; a.WC = WC; a.nbi = nbi; a.nbj = nbj; a.V = V; a.u_begin = 0; a.u_end = U;
   a.useg = (U + nseg - 1) / nseg; a.nseg = nseg; a.vtiles = vtiles; a.part = part;
   a.part_frame_stride = (int64_t)U * V; a.part_blk_stride = a.part_frame_stride;
@@ -34,9 +34,9 @@ int main(int argc, char** argv) {
   cudaFuncSetAttribute(tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   dim3 grid(nbi * nbj * vtiles * nseg, 1);
   CUtensorMap map;
-  cuuint64_t gd[3] = {(cuuint64_t)W, (cuuint64_t)H, 1}, gs[2] = {(cuuint64_t)W * 4, (cuuint64_t)H * W * 4};
+  cuuint64_t gd[3] = {(cuuint64_t)W, (cuuint64_t)H, 1}, gs[2] = {(cuuint64_t)W * 8, (cuuint64_t)H * W * 8};
   cuuint32_t bx[3] = {(cuuint32_t)tc::kBoxW, 1, 1}, es[3] = {1, 1, 1};
-  CUresult cr = cuTensorMapEncodeTiled(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, img, gd, gs, bx, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+  CUresult cr = cuTensorMapEncodeTiled(&map, CU_TENSOR_MAP_DATA_TYPE_UINT64, 3, img, gd, gs, bx, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
                                        CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
                                        CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   if (cr != CUDA_SUCCESS) { printf("encode failed %d\n", (int)cr); return 1; }
@@ -73,5 +73,23 @@ int main(int argc, char** argv) {
     stw += t[2048 + q] - t[1024 + q];       // LDG issue + TMEM stores + wait
   }
   printf("avg: arrive->mma_go %.1f  split->arrive %.1f\n", lag / 259, stw / 259);
+  // per-region stage times of CTA 0 (mma_go(q+1) - mma_go(q)): ramp-in, middle, ramp-out rows
+  {
+    const int nu = (U + nseg - 1) / nseg, R = nu + tc::kHB - 1;
+    const int nst = ((R + tc::kG - 1) / tc::kG) * tc::kG * (WC / tc::kWB);
+    const int per_row = WC / tc::kWB;
+    double rin = 0, mid = 0, rout = 0;
+    int nin = 0, nmid = 0, nout = 0;
+    for (int q = 1; q < nst && q < 1024; ++q) {
+      const double d = (double)(t[3072 + q] - t[3072 + q - 1]);
+      const int row = q / per_row;
+      if (row < tc::kHB - 1) { rin += d; ++nin; }
+      else if (row < nu) { mid += d; ++nmid; }
+      else { rout += d; ++nout; }
+    }
+    printf("stages %d: ramp-in %.1f (%d)  middle %.1f (%d)  ramp-out %.1f (%d)  total %lld cycles\n", nst,
+           nin ? rin / nin : 0, nin, nmid ? mid / nmid : 0, nmid, nout ? rout / nout : 0, nout,
+           (long long)(t[4096 + (nst < 1024 ? nst : 1024) - 1] - t[3072]));
+  }
   return 0;
 }

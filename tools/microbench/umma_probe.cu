@@ -734,9 +734,9 @@ __global__ void rate_k_kernel(int stages, int mode, float* sink, long long* cycl
       if ((mode & 8) && (tid & 31) == 0 && q < 1024) { sink[1024 + q] = (float)clock64(); }
       if (mode & 32) mbar_wait(&bar[3], 0);  // an already-completed barrier phase
       if (mode & 64) fence_after();
-      if (mode >= 256) {  // per-stage issue gap of (mode >> 8) * 50 cycles
+      if (mode & 512) {  // per-stage issue gap of ((mode >> 20) & 255) * 50 cycles
         const long long t1 = clock64();
-        while (clock64() - t1 < (long long)(mode >> 8) * 50) {
+        while (clock64() - t1 < (long long)((mode >> 20) & 255) * 50) {
         }
       }
       if (++b == 3) b = 0;
@@ -746,11 +746,39 @@ __global__ void rate_k_kernel(int stages, int mode, float* sink, long long* cycl
       mbar_wait(&bar[ql % 3], (ql / 3) & 1);
       cycles[blockIdx.x] = clock64() - t0;
       *(volatile int*)&sink[4000] = 1;  // stop flag for the busy warps
+      if (mode & 32768) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(su32(&bar[2])) : "memory");
     }
-  } else if ((mode & 128) && warp >= 4) {
+    if (mode & 65536) asm volatile("bar.arrive 1, %0;" ::"r"((int)blockDim.x - 128 + 32) : "memory");
+  } else if ((mode & (4096 | 8192)) && warp >= 4 && (((mode & 4096) && (warp & 3) == 0) || ((mode & 8192) && (warp & 3) != 0))) {
+    // spinning waiters: mbarrier try_wait on a phase that completes only at the end (bar[2])
+    for (long long it = 0; it < (1ll << 28); ++it) {
+      uint32_t done = 0;
+      asm volatile(
+          "{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\tselp.u32 %0, 1, 0, P;\n}"
+          : "=r"(done)
+          : "r"(su32(&bar[2])), "r"(0u)
+          : "memory");
+      if (done || *(volatile int*)&sink[4000]) break;
+      if (mode & 16384) __nanosleep(200);
+    }
+  } else if ((mode & 32768) && warp >= 4) {
+    // waiters with a long suspend-time hint (the thread sleeps in the barrier until the phase completes)
+    for (long long it = 0; it < (1ll << 20); ++it) {
+      uint32_t done = 0;
+      asm volatile(
+          "{\n\t.reg .pred P;\n\tmbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2, %3;\n\tselp.u32 %0, 1, 0, P;\n}"
+          : "=r"(done)
+          : "r"(su32(&bar[2])), "r"(0u), "r"(1000000u)
+          : "memory");
+      if (done) break;
+    }
+  } else if ((mode & 65536) && warp >= 4) {
+    // waiters blocked on a named hardware barrier (released by the MMA thread at the end)
+    asm volatile("bar.sync 1, %0;" ::"r"((int)blockDim.x - 128 + 32) : "memory");
+  } else if ((mode & 128) && warp >= 4 && (!(mode & 1024) || (warp & 3) != 0) && (!(mode & 2048) || (warp & 3) == 0)) {
     // busy warps: dependent-free FMA stream with a sleep duty cycle (mode >> 8: sleep ns per 64 FMAs)
     float a0 = tid, a1 = tid + 1, a2 = tid + 2, a3 = tid + 3;
-    const int sl = mode >> 8;
+    const int sl = (mode & (1024 | 2048)) ? 0 : (mode >> 8);
     for (int it = 0; it < 200000; ++it) {
 #pragma unroll
       for (int k = 0; k < 16; ++k) {
@@ -799,8 +827,13 @@ int main(int argc, char** argv) {
   setvbuf(stdout, nullptr, _IONBF, 0);
   rate_k(0, 576, 125000);
   rate_k(128, 576, 125000);
-  rate_k(128 | (64 << 8), 576, 125000);
-  rate_k(128 | (200 << 8), 576, 125000);
-  rate_k(32 | 128 | (64 << 8), 576, 125000);
+  rate_k(128 | 1024, 576, 125000);  // busy warps only on the other three SMSPs
+  rate_k(128 | 2048, 576, 125000);  // busy warps only on the MMA warp's SMSP
+  rate_k(4096, 576, 125000);        // try_wait spinners on the MMA warp's SMSP (warps 4, 8, 12, 16)
+  rate_k(4096, 160, 125000);        // one spinner on the MMA warp's SMSP (warp 4)
+  rate_k(8192, 576, 125000);        // spinners on the other SMSPs
+  rate_k(4096 | 16384, 576, 125000);  // spinners with nanosleep(200) on the MMA warp's SMSP
+  rate_k(32768, 576, 125000);       // waiters with a long try_wait suspend-time hint
+  rate_k(65536, 576, 125000);       // waiters blocked in bar.sync
   return 0;
 }
