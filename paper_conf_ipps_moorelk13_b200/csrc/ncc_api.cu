@@ -127,6 +127,8 @@ bool encode_f32(CUtensorMap* m, const void* base, int rank, const uint64_t* dims
             CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
 }
 
+constexpr int kTcColsMax = 8;  // ragged tensor-core column tiles up to this width run on tm_tc_cols
+
 struct PivVariant {
   const char* name;
   int TH, TW, MY, MX;  // 0 = run-time (RE)
@@ -316,10 +318,11 @@ struct ncc_plan_s {
   float* tc_img2 = nullptr;  // band rows as (tf32 hi, lo) pairs for the tensor-core numerator
   // tensor-core numerator (tm_tc_kernel): 0 = CUDA-core path
   int tc, tc_wc, tc_nbi, tc_nbj, tc_vtiles, tc_useg, tc_nseg;
+  int tc_vcols;  // last output columns computed by tm_tc_cols (0: none)
   float *tcB, *tc_part;
   // side stream for work independent of the main chain (template prep || window sums)
   cudaStream_t side;
-  cudaEvent_t ev_fork, ev_join;
+  cudaEvent_t ev_fork, ev_join, ev_cols;
   // timing (NCC_F_TIMING)
   std::vector<cudaEvent_t> ev;
   int n_ev_used;
@@ -366,6 +369,7 @@ void free_plan(ncc_plan pl) {
   for (cudaEvent_t e : pl->ev) cudaEventDestroy(e);
   if (pl->ev_fork) cudaEventDestroy(pl->ev_fork);
   if (pl->ev_join) cudaEventDestroy(pl->ev_join);
+  if (pl->ev_cols) cudaEventDestroy(pl->ev_cols);
   if (pl->side) cudaStreamDestroy(pl->side);
   if (pl->jit_lib) cudaLibraryUnload(pl->jit_lib);
   delete pl;
@@ -457,17 +461,26 @@ ncc_status setup_tc(ncc_plan pl) {
   if (mode == 0 || (p.flags & (NCC_F_CUDA_CORES | NCC_F_GENERIC_KERNEL)) || pl->roi_mode || pl->n_tmpl != 1)
     return NCC_OK;
   const int h = p.tmpl_h, w = p.tmpl_w;
+  // a ragged last column tile of at most kTcColsMax columns goes to tm_tc_cols instead of a
+  // whole column of tensor-core CTAs
   pl->tc_vtiles = ceil_div(pl->V, 128);
+  pl->tc_vcols = 0;
+  if (pl->V > 128 && pl->V % 128 != 0 && pl->V % 128 <= kTcColsMax && w <= 512 && !getenv("NCC_TC_NO_COLS")) {
+    pl->tc_vtiles = pl->V / 128;
+    pl->tc_vcols = pl->V % 128;
+  }
   pl->tc_nbi = ceil_div(h, tc::kHB);
   double best = 1e300;
   for (int wc = tc::kWB; wc <= 128; wc *= 2) {
     const int nbj = ceil_div(w, wc);
     const int64_t per_seg = (int64_t)pl->tc_vtiles * pl->tc_nbi * nbj * p.batch;
+    const int force_seg = getenv("NCC_TC_NSEG") ? atoi(getenv("NCC_TC_NSEG")) : 0;  // sweeps
     for (int nseg = 1; nseg <= 64 && nseg <= pl->Ub; ++nseg) {
+      if (force_seg > 0 && nseg != force_seg) continue;
       const int useg = ceil_div(pl->Ub, nseg);
       const int64_t ctas = per_seg * ceil_div(pl->Ub, useg);
       const int64_t waves = (ctas + pl->nsm - 1) / pl->nsm;
-      // cycles of a CTA: per stage ~230 cycles of fixed cost + 12 MMAs of 68 x N/136 cycles,
+      // cycles of a CTA: per stage ~320 cycles of fixed cost + 12 MMAs of 68 x N/136 cycles,
       // N = the group's trimmed window (tm_tc_kernel: ramp-in / ramp-out rows cover fewer columns)
       double cta = 0.0;
       const int ngrp = ceil_div(useg + tc::kHB - 1, tc::kG);
@@ -476,7 +489,7 @@ ncc_status setup_tc(ncc_plan pl) {
         const int chi = std::min(tc::kNWin, useg + tc::kHB - 1 - tc::kG * g);
         const int c0 = (lo / 8) * 8;
         const int n = std::max(16, ((chi - c0 + 7) / 8) * 8);
-        cta += tc::kG * (230.0 + 12.0 * 68.0 * n / tc::kNWin);
+        cta += tc::kG * (320.0 + 12.0 * 68.0 * n / tc::kNWin);
       }
       const double cost = (double)waves * cta * (wc / tc::kWB);
       if (cost < best * 0.98) {  // more segments only when clearly cheaper (per-CTA setup is not modelled)
@@ -503,7 +516,8 @@ ncc_status setup_tc(ncc_plan pl) {
   NCC_CUDA(cudaFuncSetAttribute((const void*)tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   pl->tc = 1;
   ncc_plan_info& in = pl->info;
-  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d", tc::kHB, pl->tc_wc, pl->tc_nseg);
+  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d%s", tc::kHB, pl->tc_wc, pl->tc_nseg,
+           pl->tc_vcols ? "_cols" : "");
   fill_kernel_info(pl, (const void*)tm_tc_kernel, tc::kThreads, smem, nblk * pl->tc_vtiles * pl->tc_nseg, p.batch, 1);
   in.specialized = 1;
   in.split = nblk;
@@ -642,6 +656,7 @@ ncc_status create_tm(ncc_plan pl) {
   NCC_CUDA(cudaStreamCreateWithFlags(&pl->side, cudaStreamNonBlocking));
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_fork, cudaEventDisableTiming));
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_join, cudaEventDisableTiming));
+  NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_cols, cudaEventDisableTiming));
   ncc_status st;
   if ((st = dalloc(&pl->tplC, (size_t)pl->n_tmpl * pl->HP * pl->WP))) return st;
   if ((st = dalloc(&pl->tst, (size_t)pl->n_tmpl))) return st;
@@ -888,6 +903,24 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     tm_tc_tpl_prep<<<nblk, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj, pl->tcB);
   }
   NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
+  if (pl->tc && pl->tc_vcols) {
+    const int nblk = pl->tc_nbi * pl->tc_nbj;
+    {  // the ragged last columns: after the join, so they overlap the tensor-core kernel (which
+       // leaves SMs free) rather than delay its start; joined before tm_tc_finish
+      const int64_t items = (int64_t)p.batch * pl->Ub * pl->tc_vcols;
+      const int64_t pfs = (int64_t)pl->Ub * pl->V;
+      auto cols = [&](auto kern) {
+        kern<<<(unsigned)ceil_div(items, 8), 256, 0, pl->side>>>(
+            d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w,
+            pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, p.batch, pl->tc_part, pfs * p.batch, pfs, nblk);
+      };
+      const int jc = ceil_div(p.tmpl_w, 32);
+      if (jc <= 4) cols(tm_tc_cols<4>);
+      else if (jc <= 8) cols(tm_tc_cols<8>);
+      else cols(tm_tc_cols<16>);
+    }
+    NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
+  }
   launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
   NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
   mark(pl, s, 2);
@@ -923,6 +956,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, p.batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
     mark(pl, s, 3);
+    if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
     tm_tc_finish<<<dim3(pl->Ub, p.batch), 256, 0, s>>>(
         pl->tc_part, nblk, t.part_blk_stride, t.part_frame_stride, pl->S1, pl->S2, pl->s_frame_stride, pl->tst,
         p.tmpl_h, p.tmpl_w, pl->V, pl->u_begin, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,

@@ -550,7 +550,7 @@ __global__ void __launch_bounds__(WX* WY * 32)
 
 // Template prep (Fig 5.2): Tbar, A_C = T - Tbar (fp32, zero-padded), A_D = sum A_C^2 (fp64),
 // flat flag; resets the per-frame argmax keys.  One CTA, deterministic reductions.
-__global__ void tm_template_prep(const float* __restrict__ tmpl, int64_t tpitch, int h, int w,
+__global__ void __launch_bounds__(1024) tm_template_prep(const float* __restrict__ tmpl, int64_t tpitch, int h, int w,
                                  float* __restrict__ tplC, int HP, int WP, TemplateStats* ts,
                                  unsigned long long* keys, int batch) {
   // blockIdx.x = template index (multi-template mode): template t at tmpl + t*h*tpitch
@@ -560,26 +560,46 @@ __global__ void tm_template_prep(const float* __restrict__ tmpl, int64_t tpitch,
   ts += t;
   __shared__ double red[32];
   const int n = h * w;
+  // loads in batches of 8 per thread (the single CTA is load-latency bound)
+  constexpr int LB = 8;
   double s = 0.0, s2 = 0.0;
-  for (int k = threadIdx.x; k < n; k += blockDim.x) {
-    const double t = tmpl[(int64_t)(k / w) * tpitch + (k % w)];
-    s += t;
-    s2 += t * t;
+  for (int k0 = threadIdx.x; k0 < n; k0 += LB * blockDim.x) {
+    float x[LB];
+#pragma unroll
+    for (int r = 0; r < LB; ++r) {
+      const int k = k0 + r * blockDim.x;
+      x[r] = k < n ? __ldg(tmpl + (int64_t)(k / w) * tpitch + (k % w)) : 0.0f;
+    }
+#pragma unroll
+    for (int r = 0; r < LB; ++r) {
+      s += (double)x[r];
+      s2 += (double)x[r] * (double)x[r];
+    }
   }
   s = block_sum_d(s, red);
   s2 = block_sum_d(s2, red);
   const double mean = s / (double)n;
   double e = 0.0, cs = 0.0;
-  for (int k = threadIdx.x; k < HP * WP; k += blockDim.x) {
-    const int i = k / WP, j = k % WP;
-    float ac = 0.0f;
-    if (i < h && j < w) {
-      const double a = (double)tmpl[(int64_t)i * tpitch + j] - mean;
-      e += a * a;
-      ac = (float)a;
-      cs += (double)ac;
+  for (int k0 = threadIdx.x; k0 < HP * WP; k0 += LB * blockDim.x) {
+    float x[LB];
+#pragma unroll
+    for (int r = 0; r < LB; ++r) {
+      const int k = k0 + r * blockDim.x, i = k / WP, j = k % WP;
+      x[r] = (k < HP * WP && i < h && j < w) ? __ldg(tmpl + (int64_t)i * tpitch + j) : 0.0f;
     }
-    tplC[k] = ac;
+#pragma unroll
+    for (int r = 0; r < LB; ++r) {
+      const int k = k0 + r * blockDim.x, i = k / WP, j = k % WP;
+      if (k >= HP * WP) break;
+      float ac = 0.0f;
+      if (i < h && j < w) {
+        const double a = (double)x[r] - mean;
+        e += a * a;
+        ac = (float)a;
+        cs += (double)ac;
+      }
+      tplC[k] = ac;
+    }
   }
   e = block_sum_d(e, red);
   cs = block_sum_d(cs, red);

@@ -498,6 +498,53 @@ __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img
   }
 }
 
+// Numerator of the last V - v_lo (< 128) output columns, which would otherwise cost a whole
+// column of tensor-core CTAs (V = W - w + 1 is 1 mod 128 for power-of-two frames and
+// templates): one warp per (frame, output row, column); lanes split the template columns, a
+// fresh fp32 partial per template row, then a warp sum.  Written to block plane 0 (the other
+// planes get zeros), so tm_tc_finish's block sum is the full numerator.  Loads of RB template
+// rows are issued before their products (the kernel is load-latency bound).  grid =
+// ceil(items / 8), block = 256.
+template <int JC>  // JC = ceil(w / 32) template columns per lane
+__global__ void __launch_bounds__(256) tm_tc_cols(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
+                                                  const float* __restrict__ tplC, int tplP, int h, int w, int v_lo,
+                                                  int V, int u_begin, int Ub, int batch, float* __restrict__ part,
+                                                  int64_t blk_stride, int64_t part_frame_stride, int nblk) {
+  const int nc = V - v_lo;
+  const int64_t item = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (item >= (int64_t)batch * Ub * nc) return;
+  const int lane = threadIdx.x & 31;
+  const int c = (int)(item % nc);
+  const int64_t t = item / nc;
+  const int ur = (int)(t % Ub), f = (int)(t / Ub);
+  const float* I = img + (int64_t)f * frame_stride + (int64_t)(u_begin + ur) * pitch + v_lo + c + lane;
+  const float* T = tplC + lane;  // zero-padded to tplP >= 32 * JC columns
+  constexpr int RB = 8;           // template rows per batch of loads (RB * JC * 2 loads in flight)
+  float tot = 0.0f;
+  for (int i0 = 0; i0 < h; i0 += RB) {
+    float tv[RB][JC], xv[RB][JC];
+#pragma unroll
+    for (int r = 0; r < RB; ++r)
+#pragma unroll
+      for (int k = 0; k < JC; ++k) {
+        const bool ok = i0 + r < h && lane + 32 * k < w;
+        tv[r][k] = ok ? __ldg(T + (int64_t)(i0 + r) * tplP + 32 * k) : 0.0f;
+        xv[r][k] = ok ? __ldg(I + (int64_t)(i0 + r) * pitch + 32 * k) : 0.0f;
+      }
+#pragma unroll
+    for (int r = 0; r < RB; ++r) {
+      float pr = 0.0f;  // fresh partial per template row
+#pragma unroll
+      for (int k = 0; k < JC; ++k) pr = fmaf(tv[r][k], xv[r][k], pr);
+      tot += pr;
+    }
+  }
+#pragma unroll
+  for (int d = 16; d; d >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, d);
+  for (int b = lane; b < nblk; b += 32)
+    part[(int64_t)b * blk_stride + (int64_t)f * part_frame_stride + (int64_t)ur * V + v_lo + c] = b == 0 ? tot : 0.0f;
+}
+
 // Template operand: for block (bi, bj) the reversed, zero-padded rows Rv[k] = A_C[i0 + K0 - k]
 // (K0 = kHB + kG - 2, zero outside the block / template), split into tf32 hi and fp32 lo, laid
 // out [2][WC/4 planes][kLB rows][4 floats] (the UMMA K-major no-swizzle canonical layout with
