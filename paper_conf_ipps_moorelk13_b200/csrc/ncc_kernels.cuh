@@ -560,6 +560,50 @@ __global__ void __launch_bounds__(1024) tm_template_prep(const float* __restrict
   ts += t;
   __shared__ double red[32];
   const int n = h * w;
+  if ((w & 3) == 0 && (WP & 3) == 0 && (tpitch & 3) == 0 && (reinterpret_cast<unsigned long long>(tmpl) & 15) == 0 &&
+      (reinterpret_cast<unsigned long long>(tplC) & 15) == 0 && (int)blockDim.x % (w / 4) == 0) {
+    // float4 path: thread -> (row slot, 4-column group); rows strided by blockDim / (w / 4)
+    const int g4 = w / 4, rs = (int)blockDim.x / g4;
+    const int jr = (int)threadIdx.x / g4, jc = ((int)threadIdx.x % g4) * 4;
+    double s = 0.0, s2 = 0.0;
+#pragma unroll 4
+    for (int i = jr; i < h; i += rs) {
+      const float4 x = __ldg(reinterpret_cast<const float4*>(tmpl + (int64_t)i * tpitch + jc));
+      s += ((double)x.x + (double)x.y) + ((double)x.z + (double)x.w);
+      s2 += ((double)x.x * x.x + (double)x.y * x.y) + ((double)x.z * x.z + (double)x.w * x.w);
+    }
+    s = block_sum_d(s, red);
+    s2 = block_sum_d(s2, red);
+    const double mean = s / (double)n;
+    double e = 0.0, cs = 0.0;
+#pragma unroll 4
+    for (int i = jr; i < h; i += rs) {
+      const float4 x = __ldg(reinterpret_cast<const float4*>(tmpl + (int64_t)i * tpitch + jc));
+      const double a0 = (double)x.x - mean, a1 = (double)x.y - mean, a2 = (double)x.z - mean,
+                   a3 = (double)x.w - mean;
+      e += (a0 * a0 + a1 * a1) + (a2 * a2 + a3 * a3);
+      const float4 ac = make_float4((float)a0, (float)a1, (float)a2, (float)a3);
+      cs += ((double)ac.x + (double)ac.y) + ((double)ac.z + (double)ac.w);
+      *reinterpret_cast<float4*>(tplC + (int64_t)i * WP + jc) = ac;
+    }
+    // zero padding (columns w .. WP, rows h .. HP)
+    for (int k = threadIdx.x; k < HP * WP; k += blockDim.x) {
+      const int i = k / WP, j = k % WP;
+      if (i >= h || j >= w) tplC[k] = 0.0f;
+    }
+    e = block_sum_d(e, red);
+    cs = block_sum_d(cs, red);
+    if (threadIdx.x == 0) {
+      ts->sum = s;
+      ts->sumsq = s2;
+      ts->energy = e;
+      ts->csum = cs;
+      ts->flat = (e <= kFlatRel * s2) ? 1 : 0;
+      ts->pad = 0;
+    }
+    for (int f = threadIdx.x; f < batch; f += blockDim.x) keys[(int64_t)f * T + t] = 0ull;
+    return;
+  }
   // loads in batches of 8 per thread (the single CTA is load-latency bound)
   constexpr int LB = 8;
   double s = 0.0, s2 = 0.0;
@@ -770,15 +814,26 @@ __global__ void __launch_bounds__(NT)
         c1 = C1[c];
         c2 = C2[c];
       }
-#pragma unroll 4
-      for (; r < nr; ++r) {  // slide down one row: + entering row, - leaving row
-        const int u = r0 + r;
-        const double xi = __ldg(col + (int64_t)(u + h - 1) * pitch);
-        const double xo = __ldg(col + (int64_t)(u - 1) * pitch);
-        c1 = (c1 + xi) - xo;
-        c2 = fma(-xo, xo, fma(xi, xi, c2));
-        X1[(int64_t)r * IWP + pidx(c)] = c1;
-        X2[(int64_t)r * IWP + pidx(c)] = c2;
+      // slide down one row at a time (+ entering row, - leaving row); the loads of up to 16
+      // rows are issued before the dependent sums (the sums are a serial chain per column)
+      for (; r < nr; r += 16) {
+        float xin[16], xout[16];
+#pragma unroll
+        for (int k = 0; k < 16; ++k) {
+          const int u = r0 + r + k;
+          const bool ok = r + k < nr;
+          xin[k] = ok ? __ldg(col + (int64_t)(u + h - 1) * pitch) : 0.0f;
+          xout[k] = ok ? __ldg(col + (int64_t)(u - 1) * pitch) : 0.0f;
+        }
+#pragma unroll
+        for (int k = 0; k < 16; ++k) {
+          if (r + k >= nr) break;
+          const double xi = xin[k], xo = xout[k];
+          c1 = (c1 + xi) - xo;
+          c2 = fma(-xo, xo, fma(xi, xi, c2));
+          X1[(int64_t)(r + k) * IWP + pidx(c)] = c1;
+          X2[(int64_t)(r + k) * IWP + pidx(c)] = c2;
+        }
       }
       C1[c] = c1;
       C2[c] = c2;

@@ -240,6 +240,16 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   const int nreloc = (ngrp - 1) / (kRelocAt / kG);  // groups g > 0 whose window restarts at column 0
   if (TC_EXP(32768) && warp != kMmaWarp) {
     // trace experiment: the MMA warp alone
+  } else if (TC_EXP(65536) && warp < 4 * kGroups) {
+    // trace experiment: no producers (TMA and relocation warps still run)
+    if (warp == 0) {
+      for (int q = 0; q < nstage; ++q) {  // keep the TMA ring moving
+        const int sl = q % kNImg;
+        mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
+        if (lane == 0) for (int k = 0; k < 128; ++k) mbar_arrive(&img_empty[sl]);
+        __syncwarp();
+      }
+    }
   } else if (warp < 4 * kGroups) {
     // ===================== producers (lane v = output column v0 + v) and ring drain.
     // Group grp (warps 4 grp .. 4 grp + 3, TMEM lane quadrants 0..3) handles the stages
