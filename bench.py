@@ -360,7 +360,15 @@ def main():
         peak_note = (f"3xTF32 fp32-equivalent tensor peak = {'measured' if mp else 'fallback'} bf16 GEMM "
                      f"{bf16:.1f} TFLOP/s x (tf32/bf16 nominal 1.1/2.25) / 3 MMAs per MAC")
         peak_at_clock = peak * sm_mhz / max_mhz if sm_mhz else None
+        # the hardware issue rate, from our own probe (tools/microbench/umma_probe.cu): a
+        # cta_group::1 M=128 tf32 MMA of width N takes N/2 cycles (K=8) = 4096 tf32 FLOP/cycle/SM.
+        # The cuBLAS-measured bf16 figure above is a power-capped GEMM and sits below it, so
+        # frac can approach or pass 1 for a kernel running at full clock; this is the strict one.
+        issue_peak = sms * 4096 * max_mhz * 1e6 / 3.0 / 1e12
+        issue = {"issue_rate_peak": issue_peak, "frac_of_issue_rate": achieved / issue_peak,
+                 "issue_rate_note": "SMs x 4096 tf32 FLOP/cycle (probe: N=136 MMA = 68 cycles) x max SM clock / 3"}
     else:
+        issue = {}
         peak = sms * 128 * 2 * max_mhz * 1e6 / 1e12
         peak_note = "FP32 FFMA peak = SMs x 128 lanes x 2 FLOP x max SM clock (derived; MEASURED_PEAKS.json has no FP32 figure)"
         peak_at_clock = sms * 128 * 2 * sm_mhz * 1e6 / 1e12 if sm_mhz else None
@@ -403,7 +411,8 @@ def main():
             "roofline": {"bound": "tensor" if tensor else "alu", "achieved": achieved, "peak": peak,
                          "unit": "TFLOP/s", "frac": achieved / peak, "traffic": traffic, "peak_note": peak_note,
                          "frac_at_sampled_clock": (achieved / peak_at_clock) if peak_at_clock else None,
-                         "kernel_ms": num_avg, "kernel_share_of_step": num_avg / (total_ms / args.steps)},
+                         "kernel_ms": num_avg, "kernel_share_of_step": num_avg / (total_ms / args.steps),
+                         **issue},
             "clocks": clocks, "e2e": e2e, "gpu_launches": launches_per_step * args.steps,
             "correct": correct, "wall_s": t_wall}
 

@@ -319,7 +319,10 @@ struct ncc_plan_s {
   // tensor-core numerator (tm_tc_kernel): 0 = CUDA-core path
   int tc, tc_wc, tc_nbi, tc_nbj, tc_vtiles, tc_useg, tc_nseg;
   int tc_vcols;  // last output columns computed by tm_tc_cols (0: none)
+  int tc_sched;  // 0: window sums || template prep; 1/2: window sums on the side stream, overlapping the
+                 // numerator; 3 (default): image split, then window sums || template prep + ragged columns
   float *tcB, *tc_part;
+  unsigned int* tc_done;  // per-frame count of finished tm_tc_finish CTAs (self-resetting)
   // side stream for work independent of the main chain (template prep || window sums)
   cudaStream_t side;
   cudaEvent_t ev_fork, ev_join, ev_cols;
@@ -357,6 +360,7 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->RS1);
   cudaFree(pl->tcB);
   cudaFree(pl->tc_part);
+  cudaFree(pl->tc_done);
   cudaFree(pl->tc_img2);
   cudaFree(pl->RS2);
   cudaFree(pl->S1);
@@ -465,6 +469,9 @@ ncc_status setup_tc(ncc_plan pl) {
   // whole column of tensor-core CTAs
   pl->tc_vtiles = ceil_div(pl->V, 128);
   pl->tc_vcols = 0;
+  // launch order (measured on B200, cfg2 step: 0 -> 0.2135 ms, 3 -> 0.2074 ms; 1/2 delay the
+  // tensor-core kernel's start or starve the ragged-column kernel); NCC_TM_SCHED overrides
+  pl->tc_sched = getenv("NCC_TM_SCHED") ? atoi(getenv("NCC_TM_SCHED")) : 3;
   if (pl->V > 128 && pl->V % 128 != 0 && pl->V % 128 <= kTcColsMax && w <= 512 && !getenv("NCC_TC_NO_COLS")) {
     pl->tc_vtiles = pl->V / 128;
     pl->tc_vcols = pl->V % 128;
@@ -512,6 +519,8 @@ ncc_status setup_tc(ncc_plan pl) {
   if ((st = dalloc(&pl->tcB, (size_t)nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
   if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
   if ((st = dalloc(&pl->tc_img2, (size_t)2 * p.batch * pl->Hs * p.image_w))) return st;  // (hi, lo) pairs
+  if ((st = dalloc(&pl->tc_done, (size_t)p.batch))) return st;
+  NCC_CUDA(cudaMemset(pl->tc_done, 0, (size_t)p.batch * sizeof(unsigned int)));
   const int smem = tc::smem_bytes(pl->tc_wc);
   NCC_CUDA(cudaFuncSetAttribute((const void*)tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   pl->tc = 1;
@@ -523,7 +532,8 @@ ncc_status setup_tc(ncc_plan pl) {
   in.split = nblk;
   in.const_template = 0;
   in.slabs = 1;
-  in.launches_per_call = 2 + (pl->box_smem ? 1 : 2) + 3;  // prep, operand prep, sums, numerator, finish, finalize
+  // template prep, operand prep, window sums, image split, numerator, finish (+ peak), ragged columns
+  in.launches_per_call = 2 + (pl->box_smem ? 1 : 2) + 3 + (pl->tc_vcols ? 1 : 0);
   return NCC_OK;
 }
 
@@ -891,39 +901,6 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     if (st) return st;
   }
   pl->timing_kind = 1;
-  // fork: template prep on the side stream, window sums on the main stream, join
-  mark(pl, s, 0);
-  NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
-  NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
-  tm_template_prep<<<pl->n_tmpl, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP,
-                                                       pl->WP, pl->tst, pl->keys, p.batch);
-  mark(pl, pl->side, 1);
-  if (pl->tc) {
-    const int nblk = pl->tc_nbi * pl->tc_nbj;
-    tm_tc_tpl_prep<<<nblk, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj, pl->tcB);
-  }
-  NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
-  if (pl->tc && pl->tc_vcols) {
-    const int nblk = pl->tc_nbi * pl->tc_nbj;
-    {  // the ragged last columns: after the join, so they overlap the tensor-core kernel (which
-       // leaves SMs free) rather than delay its start; joined before tm_tc_finish
-      const int64_t items = (int64_t)p.batch * pl->Ub * pl->tc_vcols;
-      const int64_t pfs = (int64_t)pl->Ub * pl->V;
-      auto cols = [&](auto kern) {
-        kern<<<(unsigned)ceil_div(items, 8), 256, 0, pl->side>>>(
-            d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w,
-            pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, p.batch, pl->tc_part, pfs * p.batch, pfs, nblk);
-      };
-      const int jc = ceil_div(p.tmpl_w, 32);
-      if (jc <= 4) cols(tm_tc_cols<4>);
-      else if (jc <= 8) cols(tm_tc_cols<8>);
-      else cols(tm_tc_cols<16>);
-    }
-    NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
-  }
-  launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
-  NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
-  mark(pl, s, 2);
   CUtensorMap map_tc;
   bool tc_now = false;
   if (pl->tc) {  // the band's rows as (hi, lo) pairs: W x Hs x batch 8-byte elements
@@ -932,11 +909,72 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     const uint32_t box[3] = {(uint32_t)tc::kBoxW, 1u, 1u};
     tc_now = encode_f32(&map_tc, pl->tc_img2, 3, dims, strides, box, true);
   }
-  if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
-    const int nblk = pl->tc_nbi * pl->tc_nbj;
+  const int nblk_tc = pl->tc_nbi * pl->tc_nbj;
+  auto launch_cols = [&]() {  // the ragged last columns (tensor-core path), on the side stream
+    const int64_t items = (int64_t)p.batch * pl->Ub * pl->tc_vcols;
+    const int64_t pfs = (int64_t)pl->Ub * pl->V;
+    auto cols = [&](auto kern) {
+      kern<<<(unsigned)ceil_div(items, 8), 256, 0, pl->side>>>(
+          d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w,
+          pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, p.batch, pl->tc_part, pfs * p.batch, pfs, nblk_tc);
+    };
+    const int jc = ceil_div(p.tmpl_w, 32);
+    if (jc <= 4) cols(tm_tc_cols<4>);
+    else if (jc <= 8) cols(tm_tc_cols<8>);
+    else cols(tm_tc_cols<16>);
+  };
+  auto launch_split = [&]() {
     tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, p.batch), 128, 0, s>>>(
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
         reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * p.image_w);
+  };
+  // fork: template prep on the side stream
+  mark(pl, s, 0);
+  NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
+  NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
+  tm_template_prep<<<pl->n_tmpl, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP,
+                                                       pl->WP, pl->tst, pl->keys, p.batch);
+  mark(pl, pl->side, 1);
+  if (pl->tc)
+    tm_tc_tpl_prep<<<nblk_tc, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj, pl->tcB);
+  NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
+  const bool late_box = tc_now && (pl->tc_sched == 1 || pl->tc_sched == 2);
+  if (tc_now && pl->tc_sched == 3) {
+    // the image split first (small: it leaves room for the template prep, which starts at once
+    // on the side stream), then the window sums on the main stream; the ragged columns follow
+    // the template prep on the side stream and overlap the window sums / tensor-core kernel
+    if (pl->tc_vcols) {
+      launch_cols();
+      NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
+    }
+    launch_split();
+    launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
+    NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
+    mark(pl, s, 2);
+  } else if (late_box) {
+    // window sums are needed only by tm_tc_finish: they run on the side stream after the
+    // template prep, concurrently with the image split and the tensor-core kernel (which
+    // leaves SMs free); the split runs on the main stream concurrently with the template prep
+    if (pl->tc_sched == 1) launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, pl->side);
+    if (pl->tc_vcols) launch_cols();
+    if (pl->tc_sched == 2) launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, pl->side);
+    NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
+    launch_split();
+    NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
+    mark(pl, s, 2);
+  } else {
+    // window sums on the main stream while the template prep runs on the side stream
+    if (pl->tc && pl->tc_vcols) {  // after the join: overlaps the tensor-core kernel rather than delay its start
+      launch_cols();
+      NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
+    }
+    launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
+    NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
+    mark(pl, s, 2);
+  }
+  if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
+    const int nblk = nblk_tc;
+    if (!late_box && pl->tc_sched != 3) launch_split();
     TcArgs t;
     t.H = p.image_h;
     t.W = p.image_w;
@@ -956,13 +994,11 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, p.batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
     mark(pl, s, 3);
-    if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
+    if (pl->tc_vcols || late_box) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
     tm_tc_finish<<<dim3(pl->Ub, p.batch), 256, 0, s>>>(
         pl->tc_part, nblk, t.part_blk_stride, t.part_frame_stride, pl->S1, pl->S2, pl->s_frame_stride, pl->tst,
         p.tmpl_h, p.tmpl_w, pl->V, pl->u_begin, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
-        (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD);
-    tm_finalize<<<ceil_div((int64_t)p.batch, 128), 128, 0, s>>>(
-        pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks), p.batch, p.score == NCC_SCORE_SSD, 1);
+        (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks));
     mark(pl, s, 4);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch (tensor core)");

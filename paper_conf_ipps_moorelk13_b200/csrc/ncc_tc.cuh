@@ -579,7 +579,7 @@ __global__ void tm_tc_tpl_prep(const float* __restrict__ tplC, int tplP, int h, 
 }
 
 // Sum the partial numerators of the template blocks in block order, normalise (or SSD),
-// optional surface store, per-frame argmax key.  grid = (Ub, batch), block = 256; each thread
+// optional surface store, per-frame argmax key; the frame's last CTA writes its peak.  grid = (Ub, batch), block = 256; each thread
 // takes kFinV columns with all their loads issued first (the kernel is load-latency bound).
 constexpr int kFinV = 4;
 __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ part, int nblk, int64_t blk_stride,
@@ -587,8 +587,10 @@ __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ pa
                                                     const double* __restrict__ S2, int64_t stat_frame_stride,
                                                     const TemplateStats* tst, int h, int w, int V, int u_begin,
                                                     float* scores, int64_t score_frame_stride,
-                                                    unsigned long long* keys, int ssd) {
+                                                    unsigned long long* keys, int ssd,
+                                                    unsigned int* __restrict__ done, PeakOut* __restrict__ peaks) {
   __shared__ unsigned long long red[32];
+  __shared__ bool last;
   const int ur = blockIdx.x, f = blockIdx.y;
   const int u = u_begin + ur;
   const TemplateStats ts = tst[0];
@@ -633,7 +635,26 @@ __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ pa
     }
   }
   best = block_max_key(best, red);
-  if (threadIdx.x == 0 && best) atomicMax(keys + f, best);
+  if (threadIdx.x == 0) {
+    if (best) atomicMax(keys + f, best);
+    // the frame's last CTA turns the key into its peak (tm_finalize fused): every CTA's
+    // atomicMax is ordered before its counter increment
+    __threadfence();
+    last = atomicAdd(done + f, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last && threadIdx.x == 0) {
+    __threadfence();
+    const unsigned long long k = atomicOr(keys + f, 0ull);
+    const uint32_t idx = key_index(k);
+    PeakOut pk;
+    pk.score = ssd ? -key_score(k) : key_score(k);
+    pk.u = (int32_t)(idx / (uint32_t)V);
+    pk.v = (int32_t)(idx % (uint32_t)V);
+    pk.flags = (ts.flat && !ssd) ? (kFlatTemplate | kInvalid) : 0u;
+    peaks[f] = pk;
+    done[f] = 0u;  // ready for the next call (stream-ordered)
+  }
 }
 
 }  // namespace nccb
