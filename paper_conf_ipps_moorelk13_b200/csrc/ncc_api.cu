@@ -335,6 +335,9 @@ struct ncc_plan_s {
   float *st_a, *st_b, *st_t, *st_s;
   void* st_out;
   size_t st_a_bytes, st_b_bytes, st_t_bytes, st_s_bytes, st_out_bytes;
+  // PIV host streaming (lazy): copy stream, per-slot "copied" / "slot free" events
+  cudaStream_t copy;
+  cudaEvent_t ev_copied[2], ev_free[2], ev_start;
 };
 
 namespace {
@@ -375,6 +378,12 @@ void free_plan(ncc_plan pl) {
   if (pl->ev_join) cudaEventDestroy(pl->ev_join);
   if (pl->ev_cols) cudaEventDestroy(pl->ev_cols);
   if (pl->side) cudaStreamDestroy(pl->side);
+  for (int k = 0; k < 2; ++k) {
+    if (pl->ev_copied[k]) cudaEventDestroy(pl->ev_copied[k]);
+    if (pl->ev_free[k]) cudaEventDestroy(pl->ev_free[k]);
+  }
+  if (pl->ev_start) cudaEventDestroy(pl->ev_start);
+  if (pl->copy) cudaStreamDestroy(pl->copy);
   if (pl->jit_lib) cudaLibraryUnload(pl->jit_lib);
   delete pl;
 }
@@ -824,6 +833,7 @@ ncc_status create_piv(ncc_plan pl) {
   const double per_pair = 16.0 * (double)((pl->box_smem ? 0 : pl->rs_frame_stride) + pl->s_frame_stride);
   int sb = (int)(2.0 * 1024 * 1024 * 1024 / per_pair);
   if (sb < 1) sb = 1;
+  if (const char* e = getenv("NCC_PIV_SUB_BATCH")) sb = std::min(sb, std::max(1, atoi(e)));  // tests / sweeps
   if (sb > p.batch) sb = p.batch;
   pl->sub_batch = sb;
   if (!pl->box_smem) {
@@ -1088,10 +1098,13 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   return NCC_OK;
 }
 
-ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores, piv_vector* d_vec, cudaStream_t s) {
+// `npairs` pairs (<= the plan's batch) from A / B; vectors (and scores) of pair k at index k.
+ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores, piv_vector* d_vec, cudaStream_t s,
+                   int npairs = -1) {
   const ncc_problem& p = pl->p;
   const PivVariant* v = pl->pivv;
-  const int nsub = ceil_div(p.batch, pl->sub_batch);
+  const int batch = npairs < 0 ? p.batch : npairs;
+  const int nsub = ceil_div(batch, pl->sub_batch);
   if (p.flags & NCC_F_TIMING) {
     ncc_status st = ensure_events(pl, 3 * nsub + 1);
     if (st) return st;
@@ -1130,7 +1143,7 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   bool use_tma = v->k_tma != nullptr && p.image_pitch % 4 == 0 && p.step_x % 4 == 0 &&
                  reinterpret_cast<uintptr_t>(B) % 16 == 0;
   if (use_tma) {
-    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)batch};
     const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)fs * 4};
     const uint32_t boxB[3] = {(uint32_t)pl->piv_bp, (uint32_t)(p.tmpl_h + 2 * p.search_y), 1u};
     use_tma = boxB[1] <= 256 && boxB[0] <= 256 && encode_f32(&mB, B, 3, dims, strides, boxB);
@@ -1138,7 +1151,7 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   CUtensorMap mW;  // the WS kernel's own box width
   memset(&mW, 0, sizeof(mW));
   if (use_tma && pl->ws_smem) {
-    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)batch};
     const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)fs * 4};
     const uint32_t boxB[3] = {(uint32_t)pl->ws_bp, (uint32_t)(p.tmpl_h + 2 * p.search_y), 1u};
     if (!(boxB[0] <= 256 && encode_f32(&mW, B, 3, dims, strides, boxB))) return NCC_ERR_CUDA;
@@ -1147,7 +1160,7 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   mark(pl, s, 0);
   for (int sb = 0; sb < nsub; ++sb) {
     const int p0 = sb * pl->sub_batch;
-    const int np = (p0 + pl->sub_batch <= p.batch) ? pl->sub_batch : p.batch - p0;
+    const int np = (p0 + pl->sub_batch <= batch) ? pl->sub_batch : batch - p0;
     launch_box(pl, B + p0 * fs, np, 0, pl->map_h, s);
     mark(pl, s, 3 * sb + 1);
     a.pair0 = p0;
@@ -1398,14 +1411,56 @@ ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, p
   const size_t fb = (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float);
   const size_t vb = (size_t)p.batch * pl->Ky * pl->Kx * sizeof(piv_vector);
   ncc_status st;
-  if ((st = stage((void**)&pl->st_a, &pl->st_a_bytes, fb))) return st;
-  if ((st = stage((void**)&pl->st_b, &pl->st_b_bytes, fb))) return st;
-  if ((st = stage(&pl->st_out, &pl->st_out_bytes, vb))) return st;
-  NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_a, fb, cudaMemcpyHostToDevice, s));
-  NCC_CUDA(cudaMemcpyAsync(pl->st_b, h_b, fb, cudaMemcpyHostToDevice, s));
-  st = run_piv(pl, pl->st_a, pl->st_b, nullptr, (piv_vector*)pl->st_out, s);
-  if (st) return st;
-  NCC_CUDA(cudaMemcpyAsync(h_vec, pl->st_out, vb, cudaMemcpyDeviceToHost, s));
+  const int chunk = pl->sub_batch;
+  if (p.batch <= chunk) {  // one chunk: copy in, run, copy out
+    if ((st = stage((void**)&pl->st_a, &pl->st_a_bytes, fb))) return st;
+    if ((st = stage((void**)&pl->st_b, &pl->st_b_bytes, fb))) return st;
+    if ((st = stage(&pl->st_out, &pl->st_out_bytes, vb))) return st;
+    NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_a, fb, cudaMemcpyHostToDevice, s));
+    NCC_CUDA(cudaMemcpyAsync(pl->st_b, h_b, fb, cudaMemcpyHostToDevice, s));
+    st = run_piv(pl, pl->st_a, pl->st_b, nullptr, (piv_vector*)pl->st_out, s);
+    if (st) return st;
+    NCC_CUDA(cudaMemcpyAsync(h_vec, pl->st_out, vb, cudaMemcpyDeviceToHost, s));
+    return NCC_OK;
+  }
+  // Streaming: chunks of sub_batch pairs through two device slots.  The host->device copy of
+  // chunk c + 1 runs on the plan's copy stream while chunk c is correlated on `stream`; a slot
+  // is refilled only after the chunk that used it (and its vectors' copy-back) is done.
+  if (!pl->copy) {
+    NCC_CUDA(cudaStreamCreateWithFlags(&pl->copy, cudaStreamNonBlocking));
+    for (int k = 0; k < 2; ++k) {
+      NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_copied[k], cudaEventDisableTiming));
+      NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_free[k], cudaEventDisableTiming));
+    }
+    NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_start, cudaEventDisableTiming));
+  }
+  const size_t pair_b = (size_t)p.image_h * p.image_pitch * sizeof(float);
+  const size_t vpair_b = (size_t)pl->Ky * pl->Kx * sizeof(piv_vector);
+  const size_t slot_b = (size_t)chunk * pair_b, vslot_b = (size_t)chunk * vpair_b;
+  if ((st = stage((void**)&pl->st_a, &pl->st_a_bytes, 2 * slot_b))) return st;
+  if ((st = stage((void**)&pl->st_b, &pl->st_b_bytes, 2 * slot_b))) return st;
+  if ((st = stage(&pl->st_out, &pl->st_out_bytes, 2 * vslot_b))) return st;
+  NCC_CUDA(cudaEventRecord(pl->ev_start, s));  // earlier work on `stream` may still use the slots
+  NCC_CUDA(cudaStreamWaitEvent(pl->copy, pl->ev_start, 0));
+  const int nch = ceil_div(p.batch, chunk);
+  for (int c = 0; c < nch; ++c) {
+    const int k = c & 1, n = std::min(chunk, p.batch - c * chunk);
+    float* sa = pl->st_a + (size_t)k * (slot_b / sizeof(float));
+    float* sb = pl->st_b + (size_t)k * (slot_b / sizeof(float));
+    piv_vector* sv = reinterpret_cast<piv_vector*>(static_cast<char*>(pl->st_out) + (size_t)k * vslot_b);
+    if (c >= 2) NCC_CUDA(cudaStreamWaitEvent(pl->copy, pl->ev_free[k], 0));
+    NCC_CUDA(cudaMemcpyAsync(sa, h_a + (size_t)c * chunk * (pair_b / sizeof(float)), n * pair_b,
+                             cudaMemcpyHostToDevice, pl->copy));
+    NCC_CUDA(cudaMemcpyAsync(sb, h_b + (size_t)c * chunk * (pair_b / sizeof(float)), n * pair_b,
+                             cudaMemcpyHostToDevice, pl->copy));
+    NCC_CUDA(cudaEventRecord(pl->ev_copied[k], pl->copy));
+    NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_copied[k], 0));
+    st = run_piv(pl, sa, sb, nullptr, sv, s, n);
+    if (st) return st;
+    NCC_CUDA(cudaMemcpyAsync(reinterpret_cast<char*>(h_vec) + (size_t)c * chunk * vpair_b, sv, n * vpair_b,
+                             cudaMemcpyDeviceToHost, s));
+    NCC_CUDA(cudaEventRecord(pl->ev_free[k], s));
+  }
   return NCC_OK;
 }
 

@@ -152,6 +152,28 @@ def test_host_path_matches_device_path():
     np.testing.assert_array_equal(d["dy"].numpy(), v["dy"])
 
 
+@pytest.mark.parametrize("sub_batch", [1, 2])
+def test_host_path_streams_chunks(monkeypatch, sub_batch):
+    """Host path with more pairs than one sub-batch: chunks stream through two device slots
+    (copy of chunk c+1 overlapping the correlation of chunk c); vectors equal the device path."""
+    P = 5
+    pairs = [synth.particle_pair_integer(256, 256, 3 - k, k - 2, seed=7100 + k) for k in range(P)]
+    v, _, _ = run_piv([p.A for p in pairs], [p.B for p in pairs], 32, 16, 16, scores=False)
+    monkeypatch.setenv("NCC_PIV_SUB_BATCH", str(sub_batch))
+    hA = torch.from_numpy(np.stack([p.A for p in pairs])).pin_memory()
+    hB = torch.from_numpy(np.stack([p.B for p in pairs])).pin_memory()
+    with PivPlan(256, 256, 32, 16, 16, pairs=P) as plan:
+        hv = torch.full((P,) + plan.grid + (6,), -1, dtype=torch.int32).pin_memory()
+        for _ in range(2):  # the second call reuses the slots after the first call's chunks
+            plan.correlate_host(hA, hB, hv)
+        torch.cuda.synchronize()
+    d = decode_vectors(hv)
+    for k in ("iy", "ix", "dy", "dx", "score", "flags"):
+        np.testing.assert_array_equal(d[k].numpy(), v[k])
+    for k in range(P):
+        assert (d["iy"][k] == 3 - k).all() and (d["ix"][k] == k - 2).all()
+
+
 def test_unaligned_pitch_plain_loads():
     p = synth.particle_pair_integer(256, 256, 5, 2, seed=8000)
     P = 259
