@@ -532,6 +532,8 @@ ncc_status setup_tc(ncc_plan pl) {
   NCC_CUDA(cudaMemset(pl->tc_done, 0, (size_t)p.batch * sizeof(unsigned int)));
   const int smem = tc::smem_bytes(pl->tc_wc);
   NCC_CUDA(cudaFuncSetAttribute((const void*)tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  NCC_CUDA(cudaFuncSetAttribute((const void*)tm_tc_prep, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                kPrepSmemFloats * 4));
   pl->tc = 1;
   ncc_plan_info& in = pl->info;
   snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d%s", tc::kHB, pl->tc_wc, pl->tc_nseg,
@@ -541,8 +543,8 @@ ncc_status setup_tc(ncc_plan pl) {
   in.split = nblk;
   in.const_template = 0;
   in.slabs = 1;
-  // template prep, operand prep, window sums, image split, numerator, finish (+ peak), ragged columns
-  in.launches_per_call = 2 + (pl->box_smem ? 1 : 2) + 3 + (pl->tc_vcols ? 1 : 0);
+  // template prep (+ operand), window sums, image split, numerator, finish (+ peak), ragged columns
+  in.launches_per_call = (h * w <= kPrepSmemFloats ? 1 : 2) + (pl->box_smem ? 1 : 2) + 3 + (pl->tc_vcols ? 1 : 0);
   return NCC_OK;
 }
 
@@ -902,6 +904,11 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
                                                                         rows_out, pl->S1, pl->S2, pl->s_frame_stride);
 }
 
+bool getenv_flag_two_kernel_prep() {  // NCC_TC_TWO_KERNEL_PREP=1: the earlier two-launch template prep
+  static const bool v = getenv("NCC_TC_TWO_KERNEL_PREP") != nullptr;
+  return v;
+}
+
 ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, int64_t tmpl_pitch, float* d_scores,
                      ncc_peak* d_peaks, cudaStream_t s, const int32_t* d_rois = nullptr) {
   const ncc_problem& p = pl->p;
@@ -942,11 +949,19 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   mark(pl, s, 0);
   NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
   NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
-  tm_template_prep<<<pl->n_tmpl, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP,
-                                                       pl->WP, pl->tst, pl->keys, p.batch);
-  mark(pl, pl->side, 1);
-  if (pl->tc)
-    tm_tc_tpl_prep<<<nblk_tc, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj, pl->tcB);
+  if (pl->tc && p.tmpl_h * p.tmpl_w <= kPrepSmemFloats && !getenv_flag_two_kernel_prep()) {
+    // one launch: template stats + centred template + MMA operand, template staged in shared memory
+    tm_tc_prep<<<nblk_tc, 1024, p.tmpl_h * p.tmpl_w * 4, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
+                                               pl->tst, pl->keys, p.batch, pl->tc_wc, pl->tc_nbj, pl->tcB);
+    mark(pl, pl->side, 1);
+  } else {
+    tm_template_prep<<<pl->n_tmpl, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP,
+                                                         pl->WP, pl->tst, pl->keys, p.batch);
+    mark(pl, pl->side, 1);
+    if (pl->tc)
+      tm_tc_tpl_prep<<<nblk_tc, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj,
+                                                    pl->tcB);
+  }
   NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
   const bool late_box = tc_now && (pl->tc_sched == 1 || pl->tc_sched == 2);
   if (tc_now && pl->tc_sched == 3) {

@@ -788,7 +788,18 @@ __global__ void __launch_bounds__(NT)
       if (r0 == 0) {  // first output row of the CTA: direct column sum (independent loads)
         double a[4] = {0.0, 0.0, 0.0, 0.0}, b[4] = {0.0, 0.0, 0.0, 0.0};
         int i = 0;
-        for (; i + 32 <= h; i += 32) {  // 32 loads in flight, then 4 accumulator chains
+        for (; i + 64 <= h; i += 64) {  // 64 loads in flight, then 4 accumulator chains
+          float xs[64];
+#pragma unroll
+          for (int k = 0; k < 64; ++k) xs[k] = __ldg(col + (int64_t)(i + k) * pitch);
+#pragma unroll
+          for (int k = 0; k < 64; ++k) {
+            const double x = xs[k];
+            a[k & 3] += x;
+            b[k & 3] = fma(x, x, b[k & 3]);
+          }
+        }
+        for (; i + 32 <= h; i += 32) {  // 32 loads in flight
           float xs[32];
 #pragma unroll
           for (int k = 0; k < 32; ++k) xs[k] = __ldg(col + (int64_t)(i + k) * pitch);
@@ -1717,6 +1728,13 @@ struct PivWs2Shape {
   static constexpr int WPW = OYc / RPW;    // consumer warps per window
   static constexpr int smem_bytes = (2 * stage_fl + WPS * s_fl) * 4;
 };
+#ifdef NCC_PIV_TRACE  // tools/microbench/piv_trace.cu: clock64 stamps per stage of CTA 0
+__device__ long long* g_piv_trace;
+#define PIV_STAMP(slot, k) \
+  if (blockIdx.x == 0 && (k) < 64) g_piv_trace[(slot)*64 + (k)] = clock64()
+#else
+#define PIV_STAMP(slot, k)
+#endif
 template <int TH, int TW, int MY, int MX, int RV, int CW, int NCW, int NPW, int WPS>
 __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
     piv_ws2_kernel(const PivArgs a, const __grid_constant__ CUtensorMap mapB, int nwin_total) {
@@ -1779,6 +1797,7 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
     float ext_prev[EPT];
     auto epilogue = [&](int k) {
       mbar_wait_backoff(&scfull_b, (uint32_t)(k & 1));
+      if (pt == 0) PIV_STAMP(6, k);
       const int s = k & 1;
 #pragma unroll
       for (int q = 0; q < EPT; ++q) {  // border scores of group k (computed during its core)
@@ -1883,6 +1902,7 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
       }
       named_bar_sync(1, NPT);  // every score tile read; pkey / stats reusable
       if (pt == 0) mbar_arrive(&scempty_b);  // the score tiles may be overwritten
+      if (pt == 0) PIV_STAMP(7, k);
     };
     for (int k = 0; k < nlocal; ++k) {
       const int s = k & 1;
@@ -1898,7 +1918,9 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
         wx[wi] = MX + (lin % a.Kx) * a.sx;
         nvalid += wv[wi] ? 1 : 0;
       }
+      if (pt == 0) PIV_STAMP(0, k);
       if (k >= 2) mbar_wait_bounded(&empty_b[s], (uint32_t)(((k >> 1) - 1) & 1));
+      if (pt == 0) PIV_STAMP(1, k);
       if (pt == 0) {
         mbar_expect_tx(&full_b[s], (uint32_t)(nvalid * S::BR * S::BP * 4));
 #pragma unroll
@@ -1943,6 +1965,7 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
         }
       };
       reduce();
+      if (pt == 0) PIV_STAMP(2, k);
       double mean[WPS], sumsq[WPS];
 #pragma unroll
       for (int wi = 0; wi < WPS; ++wi) {
@@ -1983,11 +2006,13 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
       }
       named_bar_sync(1, NPT);  // template pairs + stats of all producers written
       if (pt == 0) mbar_arrive(&full_b[s]);
+      if (pt == 0) PIV_STAMP(3, k);
       // Border offsets of this warp's window: lanes split the template columns (j = lane + 32c),
       // the warp walks up to 32 offsets per pass; conflict-free scalar loads of the region, the
       // template value loaded once per row; per-lane fp32 sums over <= JPL*TH products, then a
       // butterfly sum across the lanes.
       mbar_wait_bounded(&full_b[s], (uint32_t)((k >> 1) & 1));  // search regions landed
+      if (pt == 0) PIV_STAMP(4, k);
       float ext_cur[EPT];
 #pragma unroll
       for (int q = 0; q < EPT; ++q) ext_cur[q] = 0.0f;
@@ -2032,6 +2057,7 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
           ext_cur[q] = warp_transpose_sum32(blk);  // raw numerator of offset owned(q)
         }
       }
+      if (pt == 0) PIV_STAMP(5, k);
       if (k >= 1) epilogue(k - 1);
 #pragma unroll
       for (int q = 0; q < EPT; ++q) ext_prev[q] = ext_cur[q];
@@ -2049,6 +2075,7 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
       int lz, lin;
       const bool valid = win_of(k, wi, lz, lin);
       mbar_wait_bounded(&full_b[s], (uint32_t)((k >> 1) & 1));
+      if (tid == 0) PIV_STAMP(8, k);
       float out[RV];
 #pragma unroll
       for (int c = 0; c < RV; ++c) out[c] = 0.0f;
@@ -2077,7 +2104,9 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
         }
       }
       mbar_arrive(&empty_b[s]);  // done reading stage s (pairs, regions, stats)
+      if (tid == 0) PIV_STAMP(9, k);
       if (k >= 1) mbar_wait_bounded(&scempty_b, (uint32_t)((k - 1) & 1));
+      if (tid == 0) PIV_STAMP(10, k);
       float* sc = Sc(wi) + row * S::SP + g * RV;
 #pragma unroll
       for (int c = 0; c < RV; c += 4) *reinterpret_cast<float4*>(sc + c) = make_float4(out[c], out[c + 1], out[c + 2], out[c + 3]);

@@ -578,6 +578,104 @@ __global__ void tm_tc_tpl_prep(const float* __restrict__ tplC, int tplP, int h, 
   }
 }
 
+constexpr int kPrepSmemFloats = 48 * 1024;  // tm_tc_prep: templates up to 192 KB (else the two-kernel prep)
+// Template prep of the tensor-core path in one launch (Fig 5.2, a1, + the MMA operand): every
+// CTA forms the template mean (same code, same order: every CTA gets the same value), writes
+// its share of the centred, zero-padded template A_C = (float)(T - mean) (HP x WP, read by
+// tm_tc_cols) and its own template block's reversed, hi/lo-split operand (as tm_tc_tpl_prep,
+// from the same expression); CTA 0 adds A_D = sum (T - mean)^2, the sum of the fp32 A_C values,
+// the flat flag and resets the frame keys.  grid = nblk, block = 1024.
+__global__ void __launch_bounds__(1024) tm_tc_prep(const float* __restrict__ tmpl, int64_t tpitch, int h, int w,
+                                                   float* __restrict__ tplC, int HP, int WP, TemplateStats* ts,
+                                                   unsigned long long* keys, int batch, int WC, int nbj,
+                                                   float* __restrict__ tcB) {
+  using namespace tc;
+  extern __shared__ float tsm[];  // the whole template, dense h x w (n <= kPrepSmemFloats)
+  __shared__ double red[32];
+  const int n = h * w;
+  // one pass over the template, staged in shared memory: float4 loads when rows allow it
+  // (w, pitch and base 16-byte aligned), all of a thread's loads in flight
+  double s = 0.0, s2 = 0.0;
+  const bool v4 = (w & 3) == 0 && (tpitch & 3) == 0 && (reinterpret_cast<uintptr_t>(tmpl) & 15) == 0;
+  if (v4) {
+    const int g4 = w >> 2, n4 = n >> 2;
+    constexpr int LB = 4;
+    for (int k0 = threadIdx.x; k0 < n4; k0 += LB * blockDim.x) {
+      float4 x[LB];
+#pragma unroll
+      for (int r = 0; r < LB; ++r) {
+        const int k = k0 + r * blockDim.x;
+        x[r] = k < n4 ? __ldg(reinterpret_cast<const float4*>(tmpl + (int64_t)(k / g4) * tpitch) + k % g4)
+                      : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+#pragma unroll
+      for (int r = 0; r < LB; ++r) {
+        const int k = k0 + r * blockDim.x;
+        if (k < n4) reinterpret_cast<float4*>(tsm)[k] = x[r];
+        s += ((double)x[r].x + (double)x[r].y) + ((double)x[r].z + (double)x[r].w);
+        s2 += ((double)x[r].x * x[r].x + (double)x[r].y * x[r].y) + ((double)x[r].z * x[r].z + (double)x[r].w * x[r].w);
+      }
+    }
+  } else {
+    constexpr int LB = 8;
+    for (int k0 = threadIdx.x; k0 < n; k0 += LB * blockDim.x) {
+      float x[LB];
+#pragma unroll
+      for (int r = 0; r < LB; ++r) {
+        const int k = k0 + r * blockDim.x;
+        x[r] = k < n ? __ldg(tmpl + (int64_t)(k / w) * tpitch + (k % w)) : 0.0f;
+      }
+#pragma unroll
+      for (int r = 0; r < LB; ++r) {
+        const int k = k0 + r * blockDim.x;
+        if (k < n) tsm[k] = x[r];
+        s += (double)x[r];
+        s2 += (double)x[r] * (double)x[r];
+      }
+    }
+  }
+  s = block_sum_d(s, red);  // (its barriers also publish tsm)
+  s2 = block_sum_d(s2, red);
+  const double mean = s / (double)n;
+  // centred, zero-padded template (HP x WP), row-strided over the CTAs
+  for (int i = blockIdx.x; i < HP; i += gridDim.x)
+    for (int j = threadIdx.x; j < WP; j += blockDim.x)
+      tplC[(int64_t)i * WP + j] = (i < h && j < w) ? (float)((double)tsm[i * w + j] - mean) : 0.0f;
+  {  // this CTA's template block operand (reversed rows, hi / lo planes; as tm_tc_tpl_prep)
+    const int blk = blockIdx.x, bi = blk / nbj, bj = blk % nbj;
+    const int i0 = bi * kHB, j0 = bj * WC;
+    float* out = tcB + (int64_t)blk * (b_bytes(WC) / 4);
+    const int nb = (WC / 4) * kLB * 4;
+    for (int e = threadIdx.x; e < nb; e += blockDim.x) {
+      const int c = e / (kLB * 4), k = (e / 4) % kLB, t = e % 4;
+      const int row = kHB + kG - 2 - k;
+      const int i = i0 + row, j = j0 + 4 * c + t;
+      const float val = (row >= 0 && row < kHB && i < h && j < w) ? (float)((double)tsm[i * w + j] - mean) : 0.0f;
+      const float hi = __uint_as_float(to_tf32(val));
+      out[e] = hi;
+      out[nb + e] = val - hi;
+    }
+  }
+  if (blockIdx.x != 0) return;
+  double e = 0.0, cs = 0.0;
+  for (int k = threadIdx.x; k < n; k += blockDim.x) {
+    const double a = (double)tsm[k] - mean;
+    e += a * a;
+    cs += (double)(float)a;
+  }
+  e = block_sum_d(e, red);
+  cs = block_sum_d(cs, red);
+  if (threadIdx.x == 0) {
+    ts->sum = s;
+    ts->sumsq = s2;
+    ts->energy = e;
+    ts->csum = cs;
+    ts->flat = (e <= kFlatRel * s2) ? 1 : 0;
+    ts->pad = 0;
+  }
+  for (int f = threadIdx.x; f < batch; f += blockDim.x) keys[f] = 0ull;
+}
+
 // Sum the partial numerators of the template blocks in block order, normalise (or SSD),
 // optional surface store, per-frame argmax key; the frame's last CTA writes its peak.  grid = (Ub, batch), block = 256; each thread
 // takes kFinV columns with all their loads issued first (the kernel is load-latency bound).
