@@ -338,6 +338,15 @@ struct ncc_plan_s {
   // PIV host streaming (lazy): copy stream, per-slot "copied" / "slot free" events
   cudaStream_t copy;
   cudaEvent_t ev_copied[2], ev_free[2], ev_start;
+  // CUDA-graph replay of execute calls (lazy): capture stream, a few instantiated graphs keyed
+  // by the call's pointer arguments (the host path alternates two staging slots)
+  cudaStream_t cap;
+  int capturing;
+  struct GraphEntry {
+    uintptr_t key[6];
+    cudaGraphExec_t exec;
+  } graphs[4];
+  int n_graphs, next_graph;
 };
 
 namespace {
@@ -384,6 +393,8 @@ void free_plan(ncc_plan pl) {
   }
   if (pl->ev_start) cudaEventDestroy(pl->ev_start);
   if (pl->copy) cudaStreamDestroy(pl->copy);
+  for (int k = 0; k < pl->n_graphs; ++k) cudaGraphExecDestroy(pl->graphs[k].exec);
+  if (pl->cap) cudaStreamDestroy(pl->cap);
   if (pl->jit_lib) cudaLibraryUnload(pl->jit_lib);
   delete pl;
 }
@@ -873,7 +884,9 @@ ncc_status ensure_events(ncc_plan pl, int n) {
 }
 
 inline void mark(ncc_plan pl, cudaStream_t s, int i) {
-  if (pl->p.flags & NCC_F_TIMING) cudaEventRecord(pl->ev[i], s);
+  // under graph capture an event record is a dependency marker unless recorded as external:
+  // then it becomes an event-record node that the replay executes (timing stays valid)
+  if (pl->p.flags & NCC_F_TIMING) cudaEventRecordWithFlags(pl->ev[i], s, pl->capturing ? cudaEventRecordExternal : 0);
 }
 
 // window sums of `batch` frames over rows [row0, row0 + rows_out + h - 1)
@@ -1093,13 +1106,18 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       NCC_CUDA(cudaMemcpyAsync(pl->jit_ctpl, pl->tplC + (size_t)r0 * pl->WP, cbytes, cudaMemcpyDeviceToDevice, s));
       NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
     } else if (ct) {  // template rows [r0, r1) into the constant bank (stream-ordered after the prep)
-      ConstSlot& cs = g_const_slot[pl->device & 63];
-      std::lock_guard<std::mutex> lk(cs.mu);
-      if (!cs.done) NCC_CUDA(cudaEventCreateWithFlags(&cs.done, cudaEventDisableTiming));
-      else NCC_CUDA(cudaStreamWaitEvent(s, cs.done, 0));
-      NCC_CUDA(cudaMemcpyToSymbolAsync(c_tpl, pl->tplC + (size_t)r0 * pl->WP, cbytes, 0, cudaMemcpyDeviceToDevice, s));
-      NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
-      NCC_CUDA(cudaEventRecord(cs.done, s));
+      if (pl->capturing) {  // graph: the slot's ordering events wrap the graph launch (run_graph)
+        NCC_CUDA(cudaMemcpyToSymbolAsync(c_tpl, pl->tplC + (size_t)r0 * pl->WP, cbytes, 0, cudaMemcpyDeviceToDevice, s));
+        NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
+      } else {
+        ConstSlot& cs = g_const_slot[pl->device & 63];
+        std::lock_guard<std::mutex> lk(cs.mu);
+        if (!cs.done) NCC_CUDA(cudaEventCreateWithFlags(&cs.done, cudaEventDisableTiming));
+        else NCC_CUDA(cudaStreamWaitEvent(s, cs.done, 0));
+        NCC_CUDA(cudaMemcpyToSymbolAsync(c_tpl, pl->tplC + (size_t)r0 * pl->WP, cbytes, 0, cudaMemcpyDeviceToDevice, s));
+        NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
+        NCC_CUDA(cudaEventRecord(cs.done, s));
+      }
     } else {
       NCC_CUDA(cudaLaunchKernel(v->k[t][ct], grid, dim3(v->nt), args, (size_t)v->smem[t][ct], s));
     }
@@ -1195,6 +1213,65 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   }
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "piv_correlate launch");
+  return NCC_OK;
+}
+
+// Execute calls as CUDA graphs: the first call with a given set of pointer arguments captures
+// the launch sequence (side-stream fork / join included) on the plan's capture stream and
+// instantiates it; later calls replay it with one cudaGraphLaunch (no per-kernel launch cost,
+// shorter gaps between dependent kernels).  Plans whose kernels read the device-wide constant
+// template slot order the whole graph against other plans with the slot's event.
+// NCC_NO_GRAPH=1 launches kernel by kernel.
+bool graphs_disabled() {
+  static const bool v = getenv("NCC_NO_GRAPH") != nullptr;
+  return v;
+}
+
+template <class Body>
+ncc_status run_graph(ncc_plan pl, const uintptr_t (&key)[6], cudaStream_t s, Body&& body) {
+  if (graphs_disabled()) return body(s);
+  int hit = -1;
+  for (int k = 0; k < pl->n_graphs; ++k)
+    if (memcmp(pl->graphs[k].key, key, sizeof(key)) == 0) hit = k;
+  if (hit < 0) {
+    if (!pl->cap) NCC_CUDA(cudaStreamCreateWithFlags(&pl->cap, cudaStreamNonBlocking));
+    NCC_CUDA(cudaStreamBeginCapture(pl->cap, cudaStreamCaptureModeThreadLocal));
+    pl->capturing = 1;
+    const ncc_status st = body(pl->cap);
+    pl->capturing = 0;
+    cudaGraph_t g = nullptr;
+    const cudaError_t e = cudaStreamEndCapture(pl->cap, &g);
+    if (st != NCC_OK) {
+      if (g) cudaGraphDestroy(g);
+      cudaGetLastError();
+      return st;
+    }
+    if (e != cudaSuccess) return cuda_fail(e, "graph capture");
+    cudaGraphExec_t ex = nullptr;
+    const cudaError_t ei = cudaGraphInstantiate(&ex, g, 0);
+    cudaGraphDestroy(g);
+    if (ei != cudaSuccess) return cuda_fail(ei, "graph instantiate");
+    if (pl->n_graphs < 4) {
+      hit = pl->n_graphs++;
+    } else {  // replace round robin (the replaced graph may still run: destroy is deferred by CUDA)
+      hit = pl->next_graph;
+      pl->next_graph = (pl->next_graph + 1) % 4;
+      cudaGraphExecDestroy(pl->graphs[hit].exec);
+    }
+    pl->graphs[hit].exec = ex;
+    memcpy(pl->graphs[hit].key, key, sizeof(key));
+  }
+  const bool shared_const = pl->p.mode == NCC_MODE_MATCH && !pl->tc && pl->use_ct && !pl->jit_ctpl;
+  if (shared_const) {
+    ConstSlot& cs = g_const_slot[pl->device & 63];
+    std::lock_guard<std::mutex> lk(cs.mu);
+    if (!cs.done) NCC_CUDA(cudaEventCreateWithFlags(&cs.done, cudaEventDisableTiming));
+    else NCC_CUDA(cudaStreamWaitEvent(s, cs.done, 0));
+    NCC_CUDA(cudaGraphLaunch(pl->graphs[hit].exec, s));
+    NCC_CUDA(cudaEventRecord(cs.done, s));
+  } else {
+    NCC_CUDA(cudaGraphLaunch(pl->graphs[hit].exec, s));
+  }
   return NCC_OK;
 }
 
@@ -1363,7 +1440,11 @@ ncc_status ncc_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   if (!d_images || !d_tmpl || !d_peaks || tmpl_pitch < pl->p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
   if ((pl->p.flags & NCC_F_WRITE_SURFACE) && !d_scores) return NCC_ERR_INVALID_ARGUMENT;
   DeviceGuard g(pl->device);
-  return run_match(pl, d_images, d_tmpl, tmpl_pitch, d_scores, d_peaks, (cudaStream_t)stream);
+  const uintptr_t key[6] = {(uintptr_t)d_images, (uintptr_t)d_tmpl, (uintptr_t)tmpl_pitch, (uintptr_t)d_scores,
+                            (uintptr_t)d_peaks, 0};
+  return run_graph(pl, key, (cudaStream_t)stream, [&](cudaStream_t st) {
+    return run_match(pl, d_images, d_tmpl, tmpl_pitch, d_scores, d_peaks, st);
+  });
 }
 
 ncc_status ncc_match_rois(ncc_plan pl, const float* d_images, const float* d_tmpls, int64_t tmpl_pitch,
@@ -1373,7 +1454,11 @@ ncc_status ncc_match_rois(ncc_plan pl, const float* d_images, const float* d_tmp
   if (!d_images || !d_tmpls || !d_rois || !d_peaks || tmpl_pitch < pl->p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
   if ((pl->p.flags & NCC_F_WRITE_SURFACE) && !d_scores) return NCC_ERR_INVALID_ARGUMENT;
   DeviceGuard g(pl->device);
-  return run_match(pl, d_images, d_tmpls, tmpl_pitch, d_scores, d_peaks, (cudaStream_t)stream, d_rois);
+  const uintptr_t key[6] = {(uintptr_t)d_images, (uintptr_t)d_tmpls, (uintptr_t)tmpl_pitch, (uintptr_t)d_scores,
+                            (uintptr_t)d_peaks, (uintptr_t)d_rois};
+  return run_graph(pl, key, (cudaStream_t)stream, [&](cudaStream_t st) {
+    return run_match(pl, d_images, d_tmpls, tmpl_pitch, d_scores, d_peaks, st, d_rois);
+  });
 }
 
 ncc_status piv_correlate_ex(ncc_plan pl, const float* d_a, const float* d_b, float* d_scores, piv_vector* d_vec,
@@ -1382,7 +1467,11 @@ ncc_status piv_correlate_ex(ncc_plan pl, const float* d_a, const float* d_b, flo
   if (pl->p.mode != NCC_MODE_PIV) return NCC_ERR_WRONG_MODE;
   if (!d_a || !d_b || !d_vec) return NCC_ERR_INVALID_ARGUMENT;
   DeviceGuard g(pl->device);
-  return run_piv(pl, d_a, d_b, d_scores, d_vec, (cudaStream_t)stream);
+  const uintptr_t key[6] = {(uintptr_t)d_a, (uintptr_t)d_b, (uintptr_t)d_scores, (uintptr_t)d_vec,
+                            (uintptr_t)pl->p.batch, 0};
+  return run_graph(pl, key, (cudaStream_t)stream, [&](cudaStream_t st) {
+    return run_piv(pl, d_a, d_b, d_scores, d_vec, st);
+  });
 }
 
 ncc_status piv_correlate(ncc_plan pl, const float* d_a, const float* d_b, piv_vector* d_vec, void* stream) {
@@ -1409,7 +1498,13 @@ ncc_status ncc_match_host(ncc_plan pl, const float* h_images, const float* h_tmp
   NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_images, img_bytes, cudaMemcpyHostToDevice, s));
   NCC_CUDA(cudaMemcpy2DAsync(pl->st_t, p.tmpl_w * sizeof(float), h_tmpl, tmpl_pitch * sizeof(float),
                              p.tmpl_w * sizeof(float), p.tmpl_h, cudaMemcpyHostToDevice, s));
-  st = run_match(pl, pl->st_a, pl->st_t, p.tmpl_w, pl->st_s, (ncc_peak*)pl->st_out, s);
+  {
+    const uintptr_t key[6] = {(uintptr_t)pl->st_a, (uintptr_t)pl->st_t, (uintptr_t)p.tmpl_w, (uintptr_t)pl->st_s,
+                              (uintptr_t)pl->st_out, 0};
+    st = run_graph(pl, key, s, [&](cudaStream_t cs) {
+      return run_match(pl, pl->st_a, pl->st_t, p.tmpl_w, pl->st_s, (ncc_peak*)pl->st_out, cs);
+    });
+  }
   if (st) return st;
   NCC_CUDA(cudaMemcpyAsync(h_peaks, pl->st_out, (size_t)p.batch * sizeof(ncc_peak), cudaMemcpyDeviceToHost, s));
   if (surf && h_scores) NCC_CUDA(cudaMemcpyAsync(h_scores, pl->st_s, s_bytes, cudaMemcpyDeviceToHost, s));
@@ -1433,7 +1528,11 @@ ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, p
     if ((st = stage(&pl->st_out, &pl->st_out_bytes, vb))) return st;
     NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_a, fb, cudaMemcpyHostToDevice, s));
     NCC_CUDA(cudaMemcpyAsync(pl->st_b, h_b, fb, cudaMemcpyHostToDevice, s));
-    st = run_piv(pl, pl->st_a, pl->st_b, nullptr, (piv_vector*)pl->st_out, s);
+    const uintptr_t key[6] = {(uintptr_t)pl->st_a, (uintptr_t)pl->st_b, 0, (uintptr_t)pl->st_out,
+                              (uintptr_t)p.batch, 0};
+    st = run_graph(pl, key, s, [&](cudaStream_t cs) {
+      return run_piv(pl, pl->st_a, pl->st_b, nullptr, (piv_vector*)pl->st_out, cs);
+    });
     if (st) return st;
     NCC_CUDA(cudaMemcpyAsync(h_vec, pl->st_out, vb, cudaMemcpyDeviceToHost, s));
     return NCC_OK;
@@ -1470,7 +1569,8 @@ ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, p
                              cudaMemcpyHostToDevice, pl->copy));
     NCC_CUDA(cudaEventRecord(pl->ev_copied[k], pl->copy));
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_copied[k], 0));
-    st = run_piv(pl, sa, sb, nullptr, sv, s, n);
+    const uintptr_t key[6] = {(uintptr_t)sa, (uintptr_t)sb, 0, (uintptr_t)sv, (uintptr_t)n, 0};
+    st = run_graph(pl, key, s, [&](cudaStream_t cs) { return run_piv(pl, sa, sb, nullptr, sv, cs, n); });
     if (st) return st;
     NCC_CUDA(cudaMemcpyAsync(reinterpret_cast<char*>(h_vec) + (size_t)c * chunk * vpair_b, sv, n * vpair_b,
                              cudaMemcpyDeviceToHost, s));
