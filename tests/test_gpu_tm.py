@@ -270,3 +270,49 @@ def test_window_sum_forms_agree(h, w, monkeypatch):
     np.testing.assert_array_equal(fused, two)
     ref = oracle.ncc_surface(img, T)
     assert np.max(np.abs(fused[0] - ref)) <= TOL
+
+
+@pytest.mark.parametrize("cuda_cores", [True, False])
+def test_graph_replay_rotating_buffers(cuda_cores, tmp_path):
+    """Execute calls replay captured CUDA graphs keyed by their pointer arguments (at most 4 per
+    plan): rotating 6 buffer sets forces captures, replays and evictions; every call's peak is
+    the planted one and the surfaces equal, bit for bit, a run launching kernel by kernel
+    (NCC_NO_GRAPH=1 in a subprocess)."""
+    import subprocess
+    import sys
+    import os
+    dev = torch.device("cuda", 0)
+    H, W, h, w = (256, 256, 32, 32)
+    sets = []
+    for k in range(6):
+        img = synth.uniform_image(H, W, 9000 + k)
+        T, u0, v0 = synth.planted_template(img, h, w, 9500 + k)
+        sets.append((img, np.ascontiguousarray(T), u0, v0))
+    np.save(tmp_path / "imgs.npy", np.stack([s[0] for s in sets]))
+    np.save(tmp_path / "tmpls.npy", np.stack([s[1] for s in sets]))
+    surfaces = {}
+    with MatchPlan(H, W, h, w, write_surface=True, cuda_cores=cuda_cores) as plan:
+        bufs = [(torch.from_numpy(s[0]).to(dev), torch.from_numpy(s[1]).to(dev)) for s in sets]
+        for _ in range(3):
+            for k, (di, dt) in enumerate(bufs):
+                pk, sc = plan.match(di, dt)
+                torch.cuda.synchronize()
+                d = decode_peaks(pk)
+                assert (int(d["u"][0]), int(d["v"][0])) == (sets[k][2], sets[k][3])
+                surfaces[k] = sc[0].cpu().numpy()
+    code = (
+        "import sys, numpy as np, torch\n"
+        f"sys.path.insert(0, {repr(os.getcwd())})\n"
+        "from paper_conf_ipps_moorelk13_b200.api import MatchPlan\n"
+        f"imgs = np.load({repr(str(tmp_path / 'imgs.npy'))}); ts = np.load({repr(str(tmp_path / 'tmpls.npy'))})\n"
+        f"out = []\n"
+        f"with MatchPlan({H}, {W}, {h}, {w}, write_surface=True, cuda_cores={cuda_cores}) as p:\n"
+        "    for k in range(len(imgs)):\n"
+        "        _, sc = p.match(torch.from_numpy(imgs[k]).cuda(), torch.from_numpy(ts[k]).cuda())\n"
+        "        out.append(sc[0].cpu().numpy())\n"
+        f"np.save({repr(str(tmp_path / 'direct.npy'))}, np.stack(out))\n")
+    env = dict(os.environ, NCC_NO_GRAPH="1")
+    subprocess.run([sys.executable, "-c", code], check=True, env=env, timeout=300)
+    direct = np.load(tmp_path / "direct.npy")
+    for k in range(6):
+        np.testing.assert_array_equal(surfaces[k], direct[k])
