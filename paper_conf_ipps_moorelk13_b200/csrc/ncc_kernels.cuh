@@ -1749,6 +1749,14 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
   constexpr int NEW = (S::NE + PPW - 1) / PPW;          // border offsets per producer warp
   constexpr int EPT = (NEW + 31) / 32;                  // ... per lane
   constexpr int JPL = TW / 32;                          // template columns per lane (border sums)
+  // Register-reusing border sums (windows of at most 32 x 32 with 2m <= 32, two producer warps
+  // per window): warp 0 of the window takes the last row (dy = 2m_y; lane = template row i,
+  // sliding along the image row: each staged value feeds up to 2m_x + 1 products), warp 1 the
+  // last column (dx = 2m_x; lane = template column j, sliding down the image column).  One
+  // shared-memory value per ~16-32 products instead of one per product (the scalar form's
+  // loads were half of a stage's shared-memory traffic and stalled the consumers).
+  constexpr bool kRB = PPW == 2 && EPT >= 2 && TH <= 32 && TW <= 32 && S::OXc <= 32 && S::OYc <= 32 && TW % 4 == 0 &&
+                       S::OXc % 4 == 0;
   static_assert((TH * TW) % NPT == 0 && NPT % TW == 0, "producer threads tile each mask in whole rows");
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   float* smem = reinterpret_cast<float*>(smem_raw);
@@ -1799,13 +1807,22 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
       mbar_wait_backoff(&scfull_b, (uint32_t)(k & 1));
       if (pt == 0) PIV_STAMP(6, k);
       const int s = k & 1;
+      if constexpr (kRB) {  // row warp: lane o -> (2m_y, o), lane 0 also (2m_y, 2m_x); column warp: (o, 2m_x)
+        if (bsub == 0) {
+          if (lane < S::OXc) Sc(bwin)[S::OYc * S::SP + lane] = ext_prev[0];
+          if (lane == 0) Sc(bwin)[S::OYc * S::SP + S::OXc] = ext_prev[1];
+        } else if (lane < S::OYc) {
+          Sc(bwin)[lane * S::SP + S::OXc] = ext_prev[0];
+        }
+      } else {
 #pragma unroll
-      for (int q = 0; q < EPT; ++q) {  // border scores of group k (computed during its core)
-        const int e = owned(q);
-        if (e < S::NE) {
-          int dy, dx;
-          border(e, dy, dx);
-          Sc(bwin)[dy * S::SP + dx] = ext_prev[q];
+        for (int q = 0; q < EPT; ++q) {  // border scores of group k (computed during its core)
+          const int e = owned(q);
+          if (e < S::NE) {
+            int dy, dx;
+            border(e, dy, dx);
+            Sc(bwin)[dy * S::SP + dx] = ext_prev[q];
+          }
         }
       }
       named_bar_sync(1, NPT);
@@ -2019,7 +2036,71 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
       bool bvalid = false;
 #pragma unroll
       for (int w2 = 0; w2 < WPS; ++w2) bvalid = (w2 == bwin) ? wv[w2] : bvalid;
-      if (bvalid) {
+      if (kRB && bvalid) {
+        const float* tpf = reinterpret_cast<const float*>(TPs(s, bwin));
+        auto tval = [&](int i, int j) { return tpf[(i * S::TPP + (j / CW) * S::PB) * 2 + 1 + 2 * (j % CW)]; };
+        const float* bsr = Bs(s, bwin);
+        if (bsub == 0) {
+          // last row: lane i (< TH) owns template row i; out[dx] = sum_j T[i][j] B[i + 2m_y][j + dx]
+          constexpr int NC = TW + S::OXc;  // staged columns touched
+          float t[TW], acc[S::OX];
+#pragma unroll
+          for (int d = 0; d < S::OX; ++d) acc[d] = 0.0f;
+          if (lane < TH) {
+#pragma unroll
+            for (int j = 0; j < TW; ++j) t[j] = tval(lane, j);
+            const float* brow = bsr + (lane + S::OYc) * S::BP;
+#pragma unroll
+            for (int c4 = 0; c4 < NC; c4 += 4) {
+              const float4 v = *reinterpret_cast<const float4*>(brow + c4);
+              const float b[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+              for (int e = 0; e < 4; ++e)
+#pragma unroll
+                for (int d = 0; d < S::OX; ++d) {
+                  const int j = c4 + e - d;
+                  if (j >= 0 && j < TW) acc[d] = fmaf(t[j], b[e], acc[d]);
+                }
+            }
+          }
+          float blk[32];
+#pragma unroll
+          for (int d = 0; d < 32; ++d) blk[d] = d < S::OXc ? acc[d] : 0.0f;
+          ext_cur[0] = warp_transpose_sum32(blk);  // lane o: (2m_y, o)
+          float corner = acc[S::OXc];
+#pragma unroll
+          for (int o = 16; o; o >>= 1) corner += __shfl_xor_sync(0xffffffffu, corner, o);
+          ext_cur[1 % EPT] = lane == 0 ? corner : ext_cur[1 % EPT];
+        } else {
+          // last column: lane j (< TW) owns template column j; out[dy] = sum_i T[i][j] B[i + dy][j + 2m_x]
+          constexpr int NR = TH + S::OYc;
+          float t[TH], acc[S::OYc];
+#pragma unroll
+          for (int d = 0; d < S::OYc; ++d) acc[d] = 0.0f;
+          if (lane < TW) {
+#pragma unroll
+            for (int i = 0; i < TH; ++i) t[i] = tval(i, lane);
+            const float* bcol = bsr + S::OXc + lane;
+#pragma unroll
+            for (int r0 = 0; r0 < NR; r0 += 8) {
+              float b[8];
+#pragma unroll
+              for (int e = 0; e < 8; ++e) b[e] = r0 + e < NR ? bcol[(r0 + e) * S::BP] : 0.0f;
+#pragma unroll
+              for (int e = 0; e < 8; ++e)
+#pragma unroll
+                for (int d = 0; d < S::OYc; ++d) {
+                  const int i = r0 + e - d;
+                  if (i >= 0 && i < TH) acc[d] = fmaf(t[i], b[e], acc[d]);
+                }
+            }
+          }
+          float blk[32];
+#pragma unroll
+          for (int d = 0; d < 32; ++d) blk[d] = d < S::OYc ? acc[d] : 0.0f;
+          ext_cur[0] = warp_transpose_sum32(blk);  // lane o: (o, 2m_x)
+        }
+      } else if (bvalid) {
         const float* tpf = reinterpret_cast<const float*>(TPs(s, bwin));
         const float* bs = Bs(s, bwin) + lane;
         // one pass over the rows for all NEW offsets of the warp (offsets past NE compute
