@@ -1749,14 +1749,21 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
   constexpr int NEW = (S::NE + PPW - 1) / PPW;          // border offsets per producer warp
   constexpr int EPT = (NEW + 31) / 32;                  // ... per lane
   constexpr int JPL = TW / 32;                          // template columns per lane (border sums)
-  // Register-reusing border sums (windows of at most 32 x 32 with 2m <= 32, two producer warps
-  // per window): warp 0 of the window takes the last row (dy = 2m_y; lane = template row i,
-  // sliding along the image row: each staged value feeds up to 2m_x + 1 products), warp 1 the
-  // last column (dx = 2m_x; lane = template column j, sliding down the image column).  One
-  // shared-memory value per ~16-32 products instead of one per product (the scalar form's
-  // loads were half of a stage's shared-memory traffic and stalled the consumers).
-  constexpr bool kRB = PPW == 2 && EPT >= 2 && TH <= 32 && TW <= 32 && S::OXc <= 32 && S::OYc <= 32 && TW % 4 == 0 &&
-                       S::OXc % 4 == 0;
+  // Register-reusing border sums: half of a window's producer warps take the last row
+  // (dy = 2m_y), each a 16-offset slice dx0 = 16 w (the last slice up to 2m_x + 1), lane = template
+  // row (mod 32), sliding along the staged image row in chunks of JC template columns; the other
+  // half take the last column (dx = 2m_x) in 16-offset slices of dy, lane = template column (mod
+  // 32), sliding down the staged image column in chunks of IC template rows.  Each staged value
+  // feeds 16-33 products (the scalar form loaded one value per product: half of a stage's
+  // shared-memory traffic, which stalled the consumers' LDS.128 stream).  A transpose-sum over
+  // the lanes leaves offset o of the slice in lane o.
+  constexpr int RWb = PPW / 2, CWb = PPW / 2;                     // row / column border warps
+  constexpr int AX = S::OX - 16 * (RWb - 1), AY = S::OYc - 16 * (CWb - 1);  // last slices' sizes
+  constexpr int RPL = (TH + 31) / 32, CPL = (TW + 31) / 32;        // template rows / columns per lane
+  constexpr int JC = TW <= 32 ? TW : 16, IC = TH <= 32 ? TH : 16;  // chunk of template columns / rows
+  constexpr bool kRB = PPW % 2 == 0 && PPW >= 2 && AX >= 16 && AX <= 33 && (AX < 33 || EPT >= 2) && AY >= 1 &&
+                       AY <= 32 && TW % JC == 0 &&
+                       TH % IC == 0 && JC % 4 == 0 && (TH <= 32 || TH % 32 == 0) && (TW <= 32 || TW % 32 == 0);
   static_assert((TH * TW) % NPT == 0 && NPT % TW == 0, "producer threads tile each mask in whole rows");
   extern __shared__ __align__(1024) unsigned char smem_raw[];
   float* smem = reinterpret_cast<float*>(smem_raw);
@@ -1807,12 +1814,15 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
       mbar_wait_backoff(&scfull_b, (uint32_t)(k & 1));
       if (pt == 0) PIV_STAMP(6, k);
       const int s = k & 1;
-      if constexpr (kRB) {  // row warp: lane o -> (2m_y, o), lane 0 also (2m_y, 2m_x); column warp: (o, 2m_x)
-        if (bsub == 0) {
-          if (lane < S::OXc) Sc(bwin)[S::OYc * S::SP + lane] = ext_prev[0];
-          if (lane == 0) Sc(bwin)[S::OYc * S::SP + S::OXc] = ext_prev[1];
-        } else if (lane < S::OYc) {
-          Sc(bwin)[lane * S::SP + S::OXc] = ext_prev[0];
+      if constexpr (kRB) {  // row warp w: lane o -> (2m_y, 16 w + o) [+ the 33rd in lane 0];
+                            // column warp w: lane o -> (16 w + o, 2m_x)
+        if (bsub < RWb) {
+          const int n = bsub == RWb - 1 ? AX : 16;
+          if (lane < n && lane < 32) Sc(bwin)[S::OYc * S::SP + 16 * bsub + lane] = ext_prev[0];
+          if (n == 33 && lane == 0) Sc(bwin)[S::OYc * S::SP + 16 * bsub + 32] = ext_prev[EPT - 1];
+        } else {
+          const int w = bsub - RWb, n = w == CWb - 1 ? AY : 16;
+          if (lane < n) Sc(bwin)[(16 * w + lane) * S::SP + S::OXc] = ext_prev[0];
         }
       } else {
 #pragma unroll
@@ -2040,65 +2050,82 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
         const float* tpf = reinterpret_cast<const float*>(TPs(s, bwin));
         auto tval = [&](int i, int j) { return tpf[(i * S::TPP + (j / CW) * S::PB) * 2 + 1 + 2 * (j % CW)]; };
         const float* bsr = Bs(s, bwin);
-        if (bsub == 0) {
-          // last row: lane i (< TH) owns template row i; out[dx] = sum_j T[i][j] B[i + 2m_y][j + dx]
-          constexpr int NC = TW + S::OXc;  // staged columns touched
-          float t[TW], acc[S::OX];
+        float blk[32];
+        if (bsub < RWb) {
+          // last row, slice dx in [dx0, dx0 + n): out[dx] = sum_i sum_j T[i][j] B[i + 2m_y][j + dx]
+          const int dx0 = 16 * bsub;
+          float acc[AX];
 #pragma unroll
-          for (int d = 0; d < S::OX; ++d) acc[d] = 0.0f;
-          if (lane < TH) {
+          for (int d = 0; d < AX; ++d) acc[d] = 0.0f;
 #pragma unroll
-            for (int j = 0; j < TW; ++j) t[j] = tval(lane, j);
-            const float* brow = bsr + (lane + S::OYc) * S::BP;
+          for (int ri = 0; ri < RPL; ++ri) {
+            const int i = lane + 32 * ri;
+            if (i < TH) {
+              const float* brow = bsr + (i + S::OYc) * S::BP + dx0;
+#pragma unroll 1
+              for (int j0 = 0; j0 < TW; j0 += JC) {
+                float t[JC];
 #pragma unroll
-            for (int c4 = 0; c4 < NC; c4 += 4) {
-              const float4 v = *reinterpret_cast<const float4*>(brow + c4);
-              const float b[4] = {v.x, v.y, v.z, v.w};
+                for (int j = 0; j < JC; ++j) t[j] = tval(i, j0 + j);
 #pragma unroll
-              for (int e = 0; e < 4; ++e)
+                for (int c4 = 0; c4 < JC + AX - 1; c4 += 4) {
+                  const float4 v = *reinterpret_cast<const float4*>(brow + j0 + c4);
+                  const float b[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
-                for (int d = 0; d < S::OX; ++d) {
-                  const int j = c4 + e - d;
-                  if (j >= 0 && j < TW) acc[d] = fmaf(t[j], b[e], acc[d]);
+                  for (int e = 0; e < 4; ++e)
+#pragma unroll
+                    for (int d = 0; d < AX; ++d) {
+                      const int j = c4 + e - d;
+                      if (j >= 0 && j < JC) acc[d] = fmaf(t[j], b[e], acc[d]);
+                    }
                 }
+              }
             }
           }
-          float blk[32];
 #pragma unroll
-          for (int d = 0; d < 32; ++d) blk[d] = d < S::OXc ? acc[d] : 0.0f;
-          ext_cur[0] = warp_transpose_sum32(blk);  // lane o: (2m_y, o)
-          float corner = acc[S::OXc];
+          for (int d = 0; d < 32; ++d) blk[d] = d < AX ? acc[d] : 0.0f;
+          ext_cur[0] = warp_transpose_sum32(blk);
+          if constexpr (AX == 33) {  // the 33rd offset of the slice: plain warp sum into lane 0
+            float x = acc[AX - 1];
 #pragma unroll
-          for (int o = 16; o; o >>= 1) corner += __shfl_xor_sync(0xffffffffu, corner, o);
-          ext_cur[1 % EPT] = lane == 0 ? corner : ext_cur[1 % EPT];
+            for (int o = 16; o; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
+            ext_cur[EPT - 1] = lane == 0 ? x : ext_cur[EPT - 1];
+          }
         } else {
-          // last column: lane j (< TW) owns template column j; out[dy] = sum_i T[i][j] B[i + dy][j + 2m_x]
-          constexpr int NR = TH + S::OYc;
-          float t[TH], acc[S::OYc];
+          // last column, slice dy in [dy0, dy0 + n): out[dy] = sum_i sum_j T[i][j] B[i + dy][j + 2m_x]
+          const int dy0 = 16 * (bsub - RWb);
+          float acc[AY];
 #pragma unroll
-          for (int d = 0; d < S::OYc; ++d) acc[d] = 0.0f;
-          if (lane < TW) {
+          for (int d = 0; d < AY; ++d) acc[d] = 0.0f;
 #pragma unroll
-            for (int i = 0; i < TH; ++i) t[i] = tval(i, lane);
-            const float* bcol = bsr + S::OXc + lane;
+          for (int cj = 0; cj < CPL; ++cj) {
+            const int j = lane + 32 * cj;
+            if (j < TW) {
+              const float* bcol = bsr + dy0 * S::BP + S::OXc + j;
+#pragma unroll 1
+              for (int i0 = 0; i0 < TH; i0 += IC) {
+                float t[IC];
 #pragma unroll
-            for (int r0 = 0; r0 < NR; r0 += 8) {
-              float b[8];
+                for (int i = 0; i < IC; ++i) t[i] = tval(i0 + i, j);
 #pragma unroll
-              for (int e = 0; e < 8; ++e) b[e] = r0 + e < NR ? bcol[(r0 + e) * S::BP] : 0.0f;
+                for (int r8 = 0; r8 < IC + AY - 1; r8 += 8) {
+                  float b[8];
 #pragma unroll
-              for (int e = 0; e < 8; ++e)
+                  for (int e = 0; e < 8; ++e) b[e] = r8 + e < IC + AY - 1 ? bcol[(i0 + r8 + e) * S::BP] : 0.0f;
 #pragma unroll
-                for (int d = 0; d < S::OYc; ++d) {
-                  const int i = r0 + e - d;
-                  if (i >= 0 && i < TH) acc[d] = fmaf(t[i], b[e], acc[d]);
+                  for (int e = 0; e < 8; ++e)
+#pragma unroll
+                    for (int d = 0; d < AY; ++d) {
+                      const int i = r8 + e - d;
+                      if (i >= 0 && i < IC) acc[d] = fmaf(t[i], b[e], acc[d]);
+                    }
                 }
+              }
             }
           }
-          float blk[32];
 #pragma unroll
-          for (int d = 0; d < 32; ++d) blk[d] = d < S::OYc ? acc[d] : 0.0f;
-          ext_cur[0] = warp_transpose_sum32(blk);  // lane o: (o, 2m_x)
+          for (int d = 0; d < 32; ++d) blk[d] = d < AY ? acc[d] : 0.0f;
+          ext_cur[0] = warp_transpose_sum32(blk);
         }
       } else if (bvalid) {
         const float* tpf = reinterpret_cast<const float*>(TPs(s, bwin));
