@@ -323,6 +323,10 @@ struct ncc_plan_s {
                  // numerator; 3 (default): image split, then window sums || template prep + ragged columns
   float *tcB, *tc_part;
   unsigned int* tc_done;  // per-frame count of finished tm_tc_finish CTAs (self-resetting)
+  // tiny problems: the whole TM path in one launch (tm_tiny_kernel)
+  const void* tiny_fn;
+  int tiny_ctas, tiny_rows, tiny_smem;
+  unsigned int* tiny_done;
   // side stream for work independent of the main chain (template prep || window sums)
   cudaStream_t side;
   cudaEvent_t ev_fork, ev_join, ev_cols;
@@ -373,6 +377,7 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->tcB);
   cudaFree(pl->tc_part);
   cudaFree(pl->tc_done);
+  cudaFree(pl->tiny_done);
   cudaFree(pl->tc_img2);
   cudaFree(pl->RS2);
   cudaFree(pl->S1);
@@ -559,6 +564,51 @@ ncc_status setup_tc(ncc_plan pl) {
   return NCC_OK;
 }
 
+// Tiny problems (far below one wave): one launch does prep, window sums, numerator, normalise,
+// argmax and the peak (tm_tiny_kernel), AOT-specialised for the template sizes below.  Taken when
+// the band has at most kTinyOffsets offsets and a CTA's rows fit in shared memory; not for the
+// generic / ROI / multi-template forms.  NCC_NO_TINY=1 keeps the general launch sequence.
+constexpr int64_t kTinyOffsets = 16384;
+ncc_status setup_tiny(ncc_plan pl) {
+  const ncc_problem& p = pl->p;
+  pl->tiny_fn = nullptr;
+  const int h = p.tmpl_h, w = p.tmpl_w;
+  const char* tc_env = getenv("NCC_TC");
+  if ((p.flags & NCC_F_GENERIC_KERNEL) || pl->roi_mode || pl->n_tmpl != 1 || getenv("NCC_NO_TINY") ||
+      (tc_env && atoi(tc_env) == 1) ||
+      (int64_t)pl->Ub * pl->V > kTinyOffsets)
+    return NCC_OK;
+  const void* fn = nullptr;
+  if (h == 16 && w == 16) fn = (const void*)tm_tiny_kernel<16, 16>;
+  else if (h == 32 && w == 32) fn = (const void*)tm_tiny_kernel<32, 32>;
+  if (!fn) return NCC_OK;
+  // ~64 offsets per CTA (one per thread after the staging), at most one CTA per SM per frame
+  int ctas = (int)std::min<int64_t>(ceil_div((int64_t)pl->Ub * pl->V, 64), pl->Ub);
+  ctas = std::max(1, std::min(ctas, pl->nsm));
+  const int rows = ceil_div(pl->Ub, ctas);
+  ctas = ceil_div(pl->Ub, rows);
+  const int64_t smem = (int64_t)rows * p.image_w * 16 + ((int64_t)h * w + (int64_t)(rows + h - 1) * p.image_w) * 4;
+  if (smem > 96 * 1024) return NCC_OK;
+  NCC_CUDA(cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  ncc_status st;
+  if ((st = dalloc(&pl->tiny_done, (size_t)p.batch))) return st;
+  NCC_CUDA(cudaMemset(pl->tiny_done, 0, (size_t)p.batch * sizeof(unsigned int)));
+  NCC_CUDA(cudaMemset(pl->keys, 0, (size_t)p.batch * sizeof(unsigned long long)));
+  pl->tiny_fn = fn;
+  pl->tiny_ctas = ctas;
+  pl->tiny_rows = rows;
+  pl->tiny_smem = (int)smem;
+  ncc_plan_info& in = pl->info;
+  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tiny_%dx%d_c%d", h, w, ctas);
+  fill_kernel_info(pl, fn, 256, (int)smem, ctas, p.batch, 1);
+  in.specialized = 1;
+  in.split = 1;
+  in.const_template = 0;
+  in.slabs = 1;
+  in.launches_per_call = 1;
+  return NCC_OK;
+}
+
 ncc_status create_tm(ncc_plan pl) {
   const ncc_problem& p = pl->p;
   const int h = p.tmpl_h, w = p.tmpl_w;
@@ -739,6 +789,8 @@ ncc_status create_tm(ncc_plan pl) {
     in.slabs = pl->n_slabs;
     in.launches_per_call = 2 + (pl->box_smem ? 1 : 2) + pl->n_slabs;  // prep, window sums, numerator(s), finalize
   }
+  if ((st = setup_tiny(pl))) return st;
+  if (pl->tiny_fn) return NCC_OK;
   return setup_tc(pl);
 }
 
@@ -931,6 +983,22 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     if (st) return st;
   }
   pl->timing_kind = 1;
+  if (pl->tiny_fn) {  // the whole path in one launch
+    mark(pl, s, 0);
+    mark(pl, s, 1);
+    mark(pl, s, 2);
+    float* scores = (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr;
+    int64_t fs = (int64_t)p.image_h * p.image_pitch, sfs = (int64_t)pl->Ub * pl->V;
+    int W = p.image_w, h = p.tmpl_h, w = p.tmpl_w, ub = pl->u_begin, Ubv = pl->Ub, V = pl->V, rows = pl->tiny_rows;
+    int ssd = p.score == NCC_SCORE_SSD;
+    int64_t pitch = p.image_pitch;
+    void* args[] = {&d_images, &pitch, &fs, &W, &d_tmpl, &tmpl_pitch, &h, &w, &ub, &Ubv, &V, &rows,
+                    &scores, &sfs, &pl->keys, &pl->tiny_done, &d_peaks, &ssd};
+    NCC_CUDA(cudaLaunchKernel(pl->tiny_fn, dim3(pl->tiny_ctas, p.batch), dim3(256), args, (size_t)pl->tiny_smem, s));
+    mark(pl, s, 3);
+    mark(pl, s, 4);
+    return NCC_OK;
+  }
   CUtensorMap map_tc;
   bool tc_now = false;
   if (pl->tc) {  // the band's rows as (hi, lo) pairs: W x Hs x batch 8-byte elements
@@ -1261,7 +1329,7 @@ ncc_status run_graph(ncc_plan pl, const uintptr_t (&key)[6], cudaStream_t s, Bod
     pl->graphs[hit].exec = ex;
     memcpy(pl->graphs[hit].key, key, sizeof(key));
   }
-  const bool shared_const = pl->p.mode == NCC_MODE_MATCH && !pl->tc && pl->use_ct && !pl->jit_ctpl;
+  const bool shared_const = pl->p.mode == NCC_MODE_MATCH && !pl->tc && !pl->tiny_fn && pl->use_ct && !pl->jit_ctpl;
   if (shared_const) {
     ConstSlot& cs = g_const_slot[pl->device & 63];
     std::lock_guard<std::mutex> lk(cs.mu);

@@ -2223,4 +2223,119 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
   }
 }
 
+// ================================================================== TM, tiny problems (one launch)
+// For problems far below one wave (cfg 1: 64^2 frame, 16^2 template, 2,401 offsets) the step is
+// launch- and latency-bound, so the whole path runs in ONE kernel: every CTA stages the template
+// (prep a1: fp64 mean / energy, centred fp32 A_C, flat flag -- redundantly, a few hundred loads)
+// and its band of image rows in shared memory; the window sums (a2) are fp64 column sums of h
+// rows, then w of them per offset (exact for 2^-8-quantised inputs, any order); each thread takes
+// offsets (u, v) and forms the numerator (a3: fp32, a fresh partial per template row, the order
+// of tm_ncc_kernel's row-blocked partials), normalises (a4) and keys the argmax (a5); the frame's last CTA turns
+// the key into its peak and resets the key / counter for the next call.
+// grid = (ctas per frame, batch), block = 256; dynamic smem = 2 rows W doubles + (h w + (rows + h - 1) W)
+// floats.
+template <int TH, int TW>
+__global__ void __launch_bounds__(256) tm_tiny_kernel(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
+                                                      int W, const float* __restrict__ tmpl, int64_t tpitch, int h_rt,
+                                                      int w_rt, int u_begin, int Ub, int V, int rows_per_cta,
+                                                      float* __restrict__ scores, int64_t score_frame_stride,
+                                                      unsigned long long* keys, unsigned int* done, PeakOut* peaks,
+                                                      int ssd) {
+  const int h = TH ? TH : h_rt, w = TW ? TW : w_rt, n = h * w;
+  extern __shared__ double tiny_smd[];
+  double* C1 = tiny_smd;                       // column sums over h rows: [rows][W] (fp64)
+  double* C2 = C1 + (int64_t)rows_per_cta * W; // ... of squares
+  float* T = reinterpret_cast<float*>(C2 + (int64_t)rows_per_cta * W);  // centred template, h x w
+  float* X = T + n;                            // image rows [r0, r0 + rows + h - 1) of the band, W columns
+  __shared__ double red[8];
+  __shared__ unsigned long long redk[8];
+  __shared__ bool last;
+  const int f = blockIdx.y;
+  const int r0 = blockIdx.x * rows_per_cta;
+  const int rows = min(rows_per_cta, Ub - r0);
+  // template: raw values, fp64 sum / sum of squares
+  double s = 0.0, s2 = 0.0;
+  for (int k = threadIdx.x; k < n; k += blockDim.x) {
+    const float x = __ldg(tmpl + (int64_t)(k / w) * tpitch + k % w);
+    T[k] = x;
+    s += (double)x;
+    s2 += (double)x * (double)x;
+  }
+  // image rows of this CTA
+  const float* src = img + (int64_t)f * frame_stride + (int64_t)(u_begin + r0) * pitch;
+  const int nr = rows + h - 1;
+  for (int k = threadIdx.x; k < nr * W; k += blockDim.x) X[k] = __ldg(src + (int64_t)(k / W) * pitch + k % W);
+  s = block_sum_d(s, red);
+  s2 = block_sum_d(s2, red);
+  const double mean = s / (double)n, inv_n = 1.0 / (double)n;
+  double e = 0.0, cs = 0.0;
+  for (int k = threadIdx.x; k < n; k += blockDim.x) {
+    const double a = (double)T[k] - mean;
+    e += a * a;
+    const float ac = (float)a;
+    cs += (double)ac;
+    T[k] = ac;  // each element is read and rewritten by the same thread
+  }
+  // window sums, separable: column sums of h rows, then (below) w of them per offset
+  for (int k = threadIdx.x; k < rows * W; k += blockDim.x) {
+    const int r = k / W, c = k % W;
+    double a = 0.0, b = 0.0;
+    for (int i = 0; i < h; ++i) {
+      const double x = X[(r + i) * W + c];
+      a += x;
+      b = fma(x, x, b);
+    }
+    C1[k] = a;
+    C2[k] = b;
+  }
+  e = block_sum_d(e, red);  // (its barriers also publish T, X, C1, C2)
+  cs = block_sum_d(cs, red);
+  const bool flat = e <= kFlatRel * s2;
+  unsigned long long best = 0ull;
+  for (int o = threadIdx.x; o < rows * V; o += blockDim.x) {
+    const int ur = o / V, v = o % V;
+    float num = 0.0f;
+#pragma unroll 2
+    for (int i = 0; i < h; ++i) {
+      const float* xr = X + (ur + i) * W + v;
+      const float* tr = T + i * w;
+      float part = 0.0f;  // fresh partial per template row
+#pragma unroll 8
+      for (int j = 0; j < w; ++j) part = fmaf(tr[j], xr[j], part);
+      num += part;
+    }
+    double s1 = 0.0, s2w = 0.0;
+#pragma unroll 8
+    for (int j = 0; j < w; ++j) {
+      s1 += C1[ur * W + v + j];
+      s2w += C2[ur * W + v + j];
+    }
+    const float sc = ssd ? (float)(s2 - 2.0 * ((double)num + mean * s1) + s2w)
+                         : ncc_normalize_fast(num, s1, s2w, inv_n, cs, e, flat);
+    const int u = u_begin + r0 + ur;
+    if (scores) scores[(int64_t)f * score_frame_stride + (int64_t)(r0 + ur) * V + v] = sc;
+    const unsigned long long key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
+    best = key > best ? key : best;
+  }
+  best = block_max_key(best, redk);
+  if (threadIdx.x == 0) {
+    if (best) atomicMax(keys + f, best);
+    __threadfence();
+    last = atomicAdd(done + f, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (last && threadIdx.x == 0) {
+    __threadfence();
+    const unsigned long long k = atomicExch(keys + f, 0ull);  // read and reset for the next call
+    const uint32_t idx = key_index(k);
+    PeakOut pk;
+    pk.score = ssd ? -key_score(k) : key_score(k);
+    pk.u = (int32_t)(idx / (uint32_t)V);
+    pk.v = (int32_t)(idx % (uint32_t)V);
+    pk.flags = (flat && !ssd) ? (kFlatTemplate | kInvalid) : 0u;
+    peaks[f] = pk;
+    done[f] = 0u;
+  }
+}
+
 }  // namespace nccb

@@ -316,3 +316,49 @@ def test_graph_replay_rotating_buffers(cuda_cores, tmp_path):
     direct = np.load(tmp_path / "direct.npy")
     for k in range(6):
         np.testing.assert_array_equal(surfaces[k], direct[k])
+
+
+@pytest.mark.parametrize("ssd", [False, True])
+def test_tiny_one_launch_path(monkeypatch, ssd):
+    """cfg1-sized problems run the whole path in one launch (tm_tiny_kernel): surfaces within
+    the tolerance of the fp64 oracle (NCC; SSD relative to the energy scale), planted peaks
+    exact, for a batch of frames, a band shard, and identical peaks with the general launch
+    sequence (NCC_NO_TINY=1)."""
+    dev = torch.device("cuda", 0)
+    frames = [synth.tm_inputs(1, k=40 + k) for k in range(3)]
+    T = frames[0][1]
+    imgs = np.stack([frames[0][0]] + [f[0] for f in frames[1:]])
+    score = 1 if ssd else 0
+    d_img = torch.from_numpy(imgs).to(dev)
+    d_t = torch.from_numpy(np.ascontiguousarray(T)).to(dev)
+    outs = {}
+    for tiny in (True, False):
+        if not tiny:
+            monkeypatch.setenv("NCC_NO_TINY", "1")
+        with MatchPlan(64, 64, 16, 16, batch=3, write_surface=True, score=score) as plan:
+            assert plan.info.variant_name.decode().startswith("tm_tiny") == tiny
+            pk, sc = plan.match(d_img, d_t)
+            pk, sc = plan.match(d_img, d_t)  # second call: keys / counters were reset by the first
+            torch.cuda.synchronize()
+            outs[tiny] = ({k: v.cpu().numpy() for k, v in decode_peaks(pk).items()}, sc.cpu().numpy())
+    pk, sc = outs[True]
+    for f in range(3):
+        if ssd:
+            ref, _ = oracle.ssd_match(imgs[f], T)
+            scale = float((T.astype(np.float64) ** 2).sum() + (imgs[f].astype(np.float64) ** 2).sum() / 16)
+            assert np.max(np.abs(sc[f] - ref)) <= 1e-5 * scale
+        else:
+            ref, _ = oracle.ncc_match(imgs[f], T)
+            assert np.max(np.abs(sc[f] - ref)) <= TOL
+    assert (int(pk["u"][0]), int(pk["v"][0])) == (frames[0][2], frames[0][3])
+    for k in ("u", "v", "flags"):
+        np.testing.assert_array_equal(pk[k], outs[False][0][k])
+    # a band shard: global coordinates, rows of the band only
+    monkeypatch.delenv("NCC_NO_TINY")
+    with MatchPlan(64, 64, 16, 16, write_surface=True, shard_rank=1, shard_count=3) as plan:
+        assert plan.info.variant_name.decode().startswith("tm_tiny")
+        pk1, sc1 = plan.match(d_img[:1], d_t)
+        torch.cuda.synchronize()
+        u0, u1 = plan.info.u_begin, plan.info.u_end
+        ref, _ = oracle.ncc_match(imgs[0], T)
+        assert np.max(np.abs(sc1[0].cpu().numpy() - ref[u0:u1])) <= TOL
