@@ -755,7 +755,7 @@ __global__ void __launch_bounds__(NT)
 // grid = (ceil(V / TV), ceil(rows_out / TU), batch), block = NT,
 // dynamic smem = (2 * R + 2) * IWP doubles (X1, X2 [R][IWP]; C1, C2 [IWP]).
 template <int NT>
-__global__ void __launch_bounds__(NT)
+__global__ void __launch_bounds__(NT, 2)
     box2d_kernel(const float* __restrict__ img, int64_t pitch, int64_t frame_stride, int row0, int h, int w, int V,
                  int rows_out, int TV, int TU, int R, int IWP, double* __restrict__ S1, double* __restrict__ S2,
                  int64_t s_frame_stride) {
@@ -779,19 +779,25 @@ __global__ void __launch_bounds__(NT)
   while ((32 << lsh) < iw) ++lsh;
   const int L = 1 << lsh;
   auto pidx = [&](int c) { return c + (c >> lsh); };
+  // in-frame element offsets and shared-memory indices in 32 bits (a frame's rows x pitch and the
+  // staged strip are far below 2^31): one IMAD per load / store instead of 64-bit products
+  const int P = (int)pitch, iwp = IWP;
   for (int r0 = 0; r0 < nrow; r0 += R) {
     const int nr = min(R, nrow - r0);
     for (int c = threadIdx.x; c < iw; c += NT) {
       const float* col = src + c;
+      double* x1c = X1 + pidx(c);
+      double* x2c = X2 + pidx(c);
       double c1, c2;
       int r = 0;
       if (r0 == 0) {  // first output row of the CTA: direct column sum (independent loads)
         double a[4] = {0.0, 0.0, 0.0, 0.0}, b[4] = {0.0, 0.0, 0.0, 0.0};
         int i = 0;
         for (; i + 64 <= h; i += 64) {  // 64 loads in flight, then 4 accumulator chains
+          const float* ci = col + i * P;
           float xs[64];
 #pragma unroll
-          for (int k = 0; k < 64; ++k) xs[k] = __ldg(col + (int64_t)(i + k) * pitch);
+          for (int k = 0; k < 64; ++k) xs[k] = __ldg(ci + k * P);
 #pragma unroll
           for (int k = 0; k < 64; ++k) {
             const double x = xs[k];
@@ -800,9 +806,10 @@ __global__ void __launch_bounds__(NT)
           }
         }
         for (; i + 32 <= h; i += 32) {  // 32 loads in flight
+          const float* ci = col + i * P;
           float xs[32];
 #pragma unroll
-          for (int k = 0; k < 32; ++k) xs[k] = __ldg(col + (int64_t)(i + k) * pitch);
+          for (int k = 0; k < 32; ++k) xs[k] = __ldg(ci + k * P);
 #pragma unroll
           for (int k = 0; k < 32; ++k) {
             const double x = xs[k];
@@ -812,14 +819,14 @@ __global__ void __launch_bounds__(NT)
         }
 #pragma unroll 8
         for (; i < h; ++i) {
-          const double x = __ldg(col + (int64_t)i * pitch);
+          const double x = __ldg(col + i * P);
           a[0] += x;
           b[0] = fma(x, x, b[0]);
         }
         c1 = (a[0] + a[1]) + (a[2] + a[3]);
         c2 = (b[0] + b[1]) + (b[2] + b[3]);
-        X1[pidx(c)] = c1;
-        X2[pidx(c)] = c2;
+        x1c[0] = c1;
+        x2c[0] = c2;
         r = 1;
       } else {
         c1 = C1[c];
@@ -828,22 +835,25 @@ __global__ void __launch_bounds__(NT)
       // slide down one row at a time (+ entering row, - leaving row); the loads of up to 16
       // rows are issued before the dependent sums (the sums are a serial chain per column)
       for (; r < nr; r += 16) {
+        const float* pin = col + (r0 + r + h - 1) * P;   // entering row of output row r0 + r
+        const float* pout = col + (r0 + r - 1) * P;      // leaving row
         float xin[16], xout[16];
 #pragma unroll
         for (int k = 0; k < 16; ++k) {
-          const int u = r0 + r + k;
           const bool ok = r + k < nr;
-          xin[k] = ok ? __ldg(col + (int64_t)(u + h - 1) * pitch) : 0.0f;
-          xout[k] = ok ? __ldg(col + (int64_t)(u - 1) * pitch) : 0.0f;
+          xin[k] = ok ? __ldg(pin + k * P) : 0.0f;
+          xout[k] = ok ? __ldg(pout + k * P) : 0.0f;
         }
+        double* s1p = x1c + r * iwp;
+        double* s2p = x2c + r * iwp;
 #pragma unroll
         for (int k = 0; k < 16; ++k) {
           if (r + k >= nr) break;
           const double xi = xin[k], xo = xout[k];
           c1 = (c1 + xi) - xo;
           c2 = fma(-xo, xo, fma(xi, xi, c2));
-          X1[(int64_t)(r + k) * IWP + pidx(c)] = c1;
-          X2[(int64_t)(r + k) * IWP + pidx(c)] = c2;
+          s1p[k * iwp] = c1;
+          s2p[k * iwp] = c2;
         }
       }
       C1[c] = c1;
@@ -851,27 +861,31 @@ __global__ void __launch_bounds__(NT)
     }
     __syncthreads();
     for (int r = wid; r < nr; r += NW) {
-      double* x1 = X1 + (int64_t)r * IWP;
-      double* x2 = X2 + (int64_t)r * IWP;
-      // blocked inclusive prefix: chunk totals, warp scan of the totals, chunk prefixes
-      const int cb = lane * L, ce = min(cb + L, iw);
+      double* x1 = X1 + r * iwp;
+      double* x2 = X2 + r * iwp;
+      // blocked inclusive prefix: chunk totals, warp scan of the totals, chunk prefixes; the
+      // lane's chunk [lane L, lane L + L) is contiguous in the padded row, at lane (L + 1)
+      const int cb = lane * L, n = max(0, min(L, iw - cb));
+      double* y1 = x1 + lane * (L + 1);
+      double* y2 = x2 + lane * (L + 1);
       double t1 = 0.0, t2 = 0.0;
-      for (int c = cb; c < ce; ++c) {
-        t1 += x1[pidx(c)];
-        t2 += x2[pidx(c)];
+      for (int k = 0; k < n; ++k) {
+        t1 += y1[k];
+        t2 += y2[k];
       }
       double p1 = warp_incl_scan_d(t1) - t1, p2 = warp_incl_scan_d(t2) - t2;
-      for (int c = cb; c < ce; ++c) {
-        p1 += x1[pidx(c)];
-        p2 += x2[pidx(c)];
-        x1[pidx(c)] = p1;
-        x2[pidx(c)] = p2;
+      for (int k = 0; k < n; ++k) {
+        p1 += y1[k];
+        p2 += y2[k];
+        y1[k] = p1;
+        y2[k] = p2;
       }
       __syncwarp();
-      const int64_t o = (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
+      double* o1 = S1 + (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
+      double* o2 = S2 + (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
       for (int v = lane; v < tv; v += 32) {
-        S1[o + v] = x1[pidx(v + w - 1)] - (v > 0 ? x1[pidx(v - 1)] : 0.0);
-        S2[o + v] = x2[pidx(v + w - 1)] - (v > 0 ? x2[pidx(v - 1)] : 0.0);
+        o1[v] = x1[pidx(v + w - 1)] - (v > 0 ? x1[pidx(v - 1)] : 0.0);
+        o2[v] = x2[pidx(v + w - 1)] - (v > 0 ? x2[pidx(v - 1)] : 0.0);
       }
     }
     __syncthreads();
