@@ -1746,8 +1746,11 @@ struct PivWs2Shape {
 __device__ long long* g_piv_trace;
 #define PIV_STAMP(slot, k) \
   if (blockIdx.x == 0 && (k) < 64) g_piv_trace[(slot)*64 + (k)] = clock64()
+__device__ int g_piv_exp;  // timing experiments (trace builds only): 1 no border sums, 2 no epilogue normalisation
+#define PIV_EXP(bit) (g_piv_exp & (bit))
 #else
 #define PIV_STAMP(slot, k)
+#define PIV_EXP(bit) 0
 #endif
 template <int TH, int TW, int MY, int MX, int RV, int CW, int NCW, int NPW, int WPS>
 __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
@@ -1874,7 +1877,7 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
 #pragma unroll
           for (int c = 0; c < CH; ++c) {
             const int e = e0 + c * NPT;
-            if (e < tile) {
+            if (e < tile && !PIV_EXP(2)) {
               const int64_t mi = (int64_t)(e / S::OX) * a.map_pitch + e % S::OX;
               w1[c] = __ldg(S1f + mi);
               w2[c] = __ldg(S2f + mi);
@@ -1886,8 +1889,9 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
             if (e < tile) {
               float* tp = T + (e / S::OX) * S::SP + e % S::OX;
               const float num = *tp;
-              const float sv = a.ssd ? (float)(tsq - 2.0 * ((double)num + tmean * w1[c]) + w2[c])
-                                     : ncc_normalize_fast(num, w1[c], w2[c], inv_n, csum, energy, flat);
+              const float sv = PIV_EXP(2) ? num
+                               : a.ssd ? (float)(tsq - 2.0 * ((double)num + tmean * w1[c]) + w2[c])
+                                       : ncc_normalize_fast(num, w1[c], w2[c], inv_n, csum, energy, flat);
               *tp = sv;
               if (gsc) gsc[e] = sv;
               const unsigned long long key = make_key(a.ssd ? -sv : sv, (uint32_t)e);
@@ -2060,7 +2064,8 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
       bool bvalid = false;
 #pragma unroll
       for (int w2 = 0; w2 < WPS; ++w2) bvalid = (w2 == bwin) ? wv[w2] : bvalid;
-      if (kRB && bvalid) {
+      if (PIV_EXP(1)) {
+      } else if (kRB && bvalid) {
         const float* tpf = reinterpret_cast<const float*>(TPs(s, bwin));
         auto tval = [&](int i, int j) { return tpf[(i * S::TPP + (j / CW) * S::PB) * 2 + 1 + 2 * (j % CW)]; };
         const float* bsr = Bs(s, bwin);

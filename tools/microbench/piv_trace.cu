@@ -4,7 +4,7 @@
 // core end, after the score-tile wait).  Random frames, constant window sums (timing only).
 //   nvcc -gencode arch=compute_100a,code=sm_100a -O3 -DNCC_PIV_TRACE
 //     -I../../paper_conf_ipps_moorelk13_b200/csrc -o piv_trace piv_trace.cu -lcuda
-// usage: piv_trace <3|4> [pairs]
+// usage: piv_trace <3|4> [pairs] [experiment bits: 1 no border sums, 2 no epilogue normalisation]
 #include <cstdio>
 #include <cstdlib>
 #include <vector>
@@ -90,6 +90,8 @@ int run(int H, int W, int S, int P) {
 int main(int argc, char** argv) {
   const int cfg = argc > 1 ? atoi(argv[1]) : 3;
   const int P = argc > 2 ? atoi(argv[2]) : 1;
+  const int exp = argc > 3 ? atoi(argv[3]) : 0;
+  cudaMemcpyToSymbol(g_piv_exp, &exp, sizeof(exp));
   if (cfg == 3) return run<32, 32, 16, 16, 32, 4>(1024, 1024, 16, P);
   return run<64, 64, 32, 32, 64, 1>(2048, 2048, 32, P);
 }
