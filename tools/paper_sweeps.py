@@ -2,8 +2,9 @@
 """Paper-shaped sweeps: structural analogues of the dissertation's
 experiments whose numbers are lost (PAPER.md captions only):
 
-  * Tab 6.13  TM partial sums, run-time evaluated (RE) vs specialised (SK):
-                          time, TFLOP/s and registers/thread for RE, AOT-SK and NVRTC-SK.
+  * Tab 6.13  TM partial sums, run-time evaluated (RE) vs specialised (SK) CUDA-core
+                          kernels, beside the default tensor-core numerator (TC): time, TFLOP/s
+                          and registers/thread.
   * Tab 6.4/6.16  PIV mask-size set   (masks 16..64, search +-16).
   * Tab 6.5/6.17  PIV search set  (mask 32, m = 4..32).
   * Tab 6.6/6.18  PIV overlap set (mask 32, m = 16, 0..75 % overlap).
@@ -50,8 +51,8 @@ def tm_re_vs_sk():
         c = synth.CONFIGS[cfg]
         img, T, u0, v0 = synth.tm_inputs(cfg)
         d_img, d_t = torch.from_numpy(img).to(DEV), torch.from_numpy(T).to(DEV)
-        for tier, generic in (("SK", False), ("RE", True)):
-            with MatchPlan(c["H"], c["W"], c["h"], c["w"], timing=True, generic=generic) as plan:
+        for tier, generic, cc in (("TC", False, False), ("SK", False, True), ("RE", True, True)):
+            with MatchPlan(c["H"], c["W"], c["h"], c["w"], timing=True, generic=generic, cuda_cores=cc) as plan:
                 pk = None
 
                 def run():
@@ -78,7 +79,9 @@ def tm_odd_template():
                 pk, _ = plan.match(d_img, d_t)
             num, tot = timed(plan, run)
             d = decode_peaks(pk)
-            emit(table="5.2", h=156, w=116, tier="RE" if generic else "JIT", variant=plan.info.variant_name.decode(),
+            name = plan.info.variant_name.decode()
+            emit(table="5.2", h=156, w=116, tier="RE" if generic else ("TC" if name.startswith("tm_tc") else "JIT"),
+                 variant=name,
                  regs=plan.info.regs_per_thread, numerator_ms=num, step_ms=tot,
                  tflops=plan.info.flops_per_call / num / 1e9, correct=(int(d["u"][0]), int(d["v"][0])) == (u0, v0))
 
