@@ -950,6 +950,7 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
     const int gx = ceil_div(V, kBoxTV);
     int TU = 64;
     while (TU > pl->box_r && (int64_t)gx * ceil_div(rows_out, TU) * batch < pl->nsm) TU /= 2;
+    if (const char* e = getenv("NCC_BOX_TU")) TU = std::max(pl->box_r, atoi(e));  // sweeps
     dim3 g(gx, ceil_div(rows_out, TU), batch);
     box2d_kernel<kBox2dNT><<<g, kBox2dNT, pl->box_smem, s>>>(frames, p.image_pitch,
                                                             (int64_t)p.image_h * p.image_pitch, row0, h, w, V,
