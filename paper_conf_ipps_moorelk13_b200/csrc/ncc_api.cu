@@ -346,8 +346,14 @@ struct ncc_plan_s {
   // by the call's pointer arguments (the host path alternates two staging slots)
   cudaStream_t cap;
   int capturing;
+  // host path (ncc_match_host): inputs copied inside the launch sequence -- the template on the
+  // side stream ahead of its prep, the frames on the main stream -- so the prep overlaps the
+  // frames' copy (transient, set around one call)
+  const float* h_img_in;
+  const float* h_tmpl_in;
+  int64_t h_tmpl_pitch;
   struct GraphEntry {
-    uintptr_t key[6];
+    uintptr_t key[8];
     cudaGraphExec_t exec;
   } graphs[4];
   int n_graphs, next_graph;
@@ -986,6 +992,13 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   pl->timing_kind = 1;
   if (pl->tiny_fn) {  // the whole path in one launch
     mark(pl, s, 0);
+    if (pl->h_tmpl_in) {
+      NCC_CUDA(cudaMemcpy2DAsync(const_cast<float*>(d_tmpl), tmpl_pitch * sizeof(float), pl->h_tmpl_in,
+                                 pl->h_tmpl_pitch * sizeof(float), p.tmpl_w * sizeof(float), p.tmpl_h,
+                                 cudaMemcpyHostToDevice, s));
+      NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
+                               (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
+    }
     mark(pl, s, 1);
     mark(pl, s, 2);
     float* scores = (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr;
@@ -1031,6 +1044,13 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   mark(pl, s, 0);
   NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
   NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
+  if (pl->h_tmpl_in) {  // host path: template copy ahead of its prep, frames on the main stream
+    NCC_CUDA(cudaMemcpy2DAsync(const_cast<float*>(d_tmpl), tmpl_pitch * sizeof(float), pl->h_tmpl_in,
+                               pl->h_tmpl_pitch * sizeof(float), p.tmpl_w * sizeof(float), p.tmpl_h,
+                               cudaMemcpyHostToDevice, pl->side));
+    NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
+                             (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
+  }
   if (pl->tc && p.tmpl_h * p.tmpl_w <= kPrepSmemFloats && !getenv_flag_two_kernel_prep()) {
     // one launch: template stats + centred template + MMA operand, template staged in shared memory
     tm_tc_prep<<<nblk_tc, 1024, p.tmpl_h * p.tmpl_w * 4, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
@@ -1291,13 +1311,22 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
 // shorter gaps between dependent kernels).  Plans whose kernels read the device-wide constant
 // template slot order the whole graph against other plans with the slot's event.
 // NCC_NO_GRAPH=1 launches kernel by kernel.
+bool is_pinned(const void* p) {  // page-locked (or device-accessible) host memory
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeHost || a.type == cudaMemoryTypeManaged;
+}
+
 bool graphs_disabled() {
   static const bool v = getenv("NCC_NO_GRAPH") != nullptr;
   return v;
 }
 
 template <class Body>
-ncc_status run_graph(ncc_plan pl, const uintptr_t (&key)[6], cudaStream_t s, Body&& body) {
+ncc_status run_graph(ncc_plan pl, const uintptr_t (&key)[8], cudaStream_t s, Body&& body) {
   if (graphs_disabled()) return body(s);
   int hit = -1;
   for (int k = 0; k < pl->n_graphs; ++k)
@@ -1509,7 +1538,7 @@ ncc_status ncc_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   if (!d_images || !d_tmpl || !d_peaks || tmpl_pitch < pl->p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
   if ((pl->p.flags & NCC_F_WRITE_SURFACE) && !d_scores) return NCC_ERR_INVALID_ARGUMENT;
   DeviceGuard g(pl->device);
-  const uintptr_t key[6] = {(uintptr_t)d_images, (uintptr_t)d_tmpl, (uintptr_t)tmpl_pitch, (uintptr_t)d_scores,
+  const uintptr_t key[8] = {(uintptr_t)d_images, (uintptr_t)d_tmpl, (uintptr_t)tmpl_pitch, (uintptr_t)d_scores,
                             (uintptr_t)d_peaks, 0};
   return run_graph(pl, key, (cudaStream_t)stream, [&](cudaStream_t st) {
     return run_match(pl, d_images, d_tmpl, tmpl_pitch, d_scores, d_peaks, st);
@@ -1523,7 +1552,7 @@ ncc_status ncc_match_rois(ncc_plan pl, const float* d_images, const float* d_tmp
   if (!d_images || !d_tmpls || !d_rois || !d_peaks || tmpl_pitch < pl->p.tmpl_w) return NCC_ERR_INVALID_ARGUMENT;
   if ((pl->p.flags & NCC_F_WRITE_SURFACE) && !d_scores) return NCC_ERR_INVALID_ARGUMENT;
   DeviceGuard g(pl->device);
-  const uintptr_t key[6] = {(uintptr_t)d_images, (uintptr_t)d_tmpls, (uintptr_t)tmpl_pitch, (uintptr_t)d_scores,
+  const uintptr_t key[8] = {(uintptr_t)d_images, (uintptr_t)d_tmpls, (uintptr_t)tmpl_pitch, (uintptr_t)d_scores,
                             (uintptr_t)d_peaks, (uintptr_t)d_rois};
   return run_graph(pl, key, (cudaStream_t)stream, [&](cudaStream_t st) {
     return run_match(pl, d_images, d_tmpls, tmpl_pitch, d_scores, d_peaks, st, d_rois);
@@ -1536,7 +1565,7 @@ ncc_status piv_correlate_ex(ncc_plan pl, const float* d_a, const float* d_b, flo
   if (pl->p.mode != NCC_MODE_PIV) return NCC_ERR_WRONG_MODE;
   if (!d_a || !d_b || !d_vec) return NCC_ERR_INVALID_ARGUMENT;
   DeviceGuard g(pl->device);
-  const uintptr_t key[6] = {(uintptr_t)d_a, (uintptr_t)d_b, (uintptr_t)d_scores, (uintptr_t)d_vec,
+  const uintptr_t key[8] = {(uintptr_t)d_a, (uintptr_t)d_b, (uintptr_t)d_scores, (uintptr_t)d_vec,
                             (uintptr_t)pl->p.batch, 0};
   return run_graph(pl, key, (cudaStream_t)stream, [&](cudaStream_t st) {
     return run_piv(pl, d_a, d_b, d_scores, d_vec, st);
@@ -1564,11 +1593,23 @@ ncc_status ncc_match_host(ncc_plan pl, const float* h_images, const float* h_tmp
   if ((st = stage((void**)&pl->st_t, &pl->st_t_bytes, t_bytes))) return st;
   if (surf && (st = stage((void**)&pl->st_s, &pl->st_s_bytes, s_bytes))) return st;
   if ((st = stage(&pl->st_out, &pl->st_out_bytes, (size_t)p.batch * sizeof(ncc_peak)))) return st;
-  NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_images, img_bytes, cudaMemcpyHostToDevice, s));
-  NCC_CUDA(cudaMemcpy2DAsync(pl->st_t, p.tmpl_w * sizeof(float), h_tmpl, tmpl_pitch * sizeof(float),
-                             p.tmpl_w * sizeof(float), p.tmpl_h, cudaMemcpyHostToDevice, s));
-  {
-    const uintptr_t key[6] = {(uintptr_t)pl->st_a, (uintptr_t)pl->st_t, (uintptr_t)p.tmpl_w, (uintptr_t)pl->st_s,
+  if (is_pinned(h_images) && is_pinned(h_tmpl)) {
+    // pinned inputs: the copies are part of the (captured) launch sequence, the template's
+    // ahead of its prep on the side stream (see run_match)
+    const uintptr_t key[8] = {(uintptr_t)pl->st_a, (uintptr_t)pl->st_t, (uintptr_t)p.tmpl_w, (uintptr_t)pl->st_s,
+                              (uintptr_t)pl->st_out, (uintptr_t)h_images, (uintptr_t)h_tmpl, (uintptr_t)tmpl_pitch};
+    pl->h_img_in = h_images;
+    pl->h_tmpl_in = h_tmpl;
+    pl->h_tmpl_pitch = tmpl_pitch;
+    st = run_graph(pl, key, s, [&](cudaStream_t cs) {
+      return run_match(pl, pl->st_a, pl->st_t, p.tmpl_w, pl->st_s, (ncc_peak*)pl->st_out, cs);
+    });
+    pl->h_img_in = pl->h_tmpl_in = nullptr;
+  } else {  // pageable inputs (staged copies, not capturable): copy, then the device-path graph
+    NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_images, img_bytes, cudaMemcpyHostToDevice, s));
+    NCC_CUDA(cudaMemcpy2DAsync(pl->st_t, p.tmpl_w * sizeof(float), h_tmpl, tmpl_pitch * sizeof(float),
+                               p.tmpl_w * sizeof(float), p.tmpl_h, cudaMemcpyHostToDevice, s));
+    const uintptr_t key[8] = {(uintptr_t)pl->st_a, (uintptr_t)pl->st_t, (uintptr_t)p.tmpl_w, (uintptr_t)pl->st_s,
                               (uintptr_t)pl->st_out, 0};
     st = run_graph(pl, key, s, [&](cudaStream_t cs) {
       return run_match(pl, pl->st_a, pl->st_t, p.tmpl_w, pl->st_s, (ncc_peak*)pl->st_out, cs);
@@ -1597,7 +1638,7 @@ ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, p
     if ((st = stage(&pl->st_out, &pl->st_out_bytes, vb))) return st;
     NCC_CUDA(cudaMemcpyAsync(pl->st_a, h_a, fb, cudaMemcpyHostToDevice, s));
     NCC_CUDA(cudaMemcpyAsync(pl->st_b, h_b, fb, cudaMemcpyHostToDevice, s));
-    const uintptr_t key[6] = {(uintptr_t)pl->st_a, (uintptr_t)pl->st_b, 0, (uintptr_t)pl->st_out,
+    const uintptr_t key[8] = {(uintptr_t)pl->st_a, (uintptr_t)pl->st_b, 0, (uintptr_t)pl->st_out,
                               (uintptr_t)p.batch, 0};
     st = run_graph(pl, key, s, [&](cudaStream_t cs) {
       return run_piv(pl, pl->st_a, pl->st_b, nullptr, (piv_vector*)pl->st_out, cs);
@@ -1638,7 +1679,7 @@ ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, p
                              cudaMemcpyHostToDevice, pl->copy));
     NCC_CUDA(cudaEventRecord(pl->ev_copied[k], pl->copy));
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_copied[k], 0));
-    const uintptr_t key[6] = {(uintptr_t)sa, (uintptr_t)sb, 0, (uintptr_t)sv, (uintptr_t)n, 0};
+    const uintptr_t key[8] = {(uintptr_t)sa, (uintptr_t)sb, 0, (uintptr_t)sv, (uintptr_t)n, 0};
     st = run_graph(pl, key, s, [&](cudaStream_t cs) { return run_piv(pl, sa, sb, nullptr, sv, cs, n); });
     if (st) return st;
     NCC_CUDA(cudaMemcpyAsync(reinterpret_cast<char*>(h_vec) + (size_t)c * chunk * vpair_b, sv, n * vpair_b,

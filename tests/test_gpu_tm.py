@@ -362,3 +362,29 @@ def test_tiny_one_launch_path(monkeypatch, ssd):
         u0, u1 = plan.info.u_begin, plan.info.u_end
         ref, _ = oracle.ncc_match(imgs[0], T)
         assert np.max(np.abs(sc1[0].cpu().numpy() - ref[u0:u1])) <= TOL
+
+
+@pytest.mark.parametrize("shape,pinned", [((1024, 1024, 128, 128), True), ((1024, 1024, 128, 128), False),
+                                          ((64, 64, 16, 16), True), ((200, 180, 24, 20), True)])
+def test_host_path_alternating_buffers(shape, pinned):
+    """Host entry point (the frames' and template's copies inside the captured launch sequence
+    for pinned buffers, staged copies for pageable ones): alternating two input sets over
+    several calls gives each set's planted peak (tensor-core, tiny and CUDA-core plans)."""
+    H, W, h, w = shape
+    sets = []
+    for k in range(2):
+        img = synth.uniform_image(H, W, 9100 + k)
+        T, u0, v0 = synth.planted_template(img, h, w, 9200 + k)
+        hi, ht = torch.from_numpy(img), torch.from_numpy(np.ascontiguousarray(T))
+        if pinned:
+            hi, ht = hi.pin_memory(), ht.pin_memory()
+        sets.append((hi, ht, u0, v0))
+    hp = torch.empty((1, 4), dtype=torch.int32).pin_memory()
+    with MatchPlan(H, W, h, w) as plan:
+        for _ in range(3):
+            for hi, ht, u0, v0 in sets:
+                plan.match_host(hi, ht, hp)
+                torch.cuda.synchronize()
+                d = decode_peaks(hp)
+                assert (int(d["u"][0]), int(d["v"][0])) == (u0, v0)
+                assert abs(float(d["score"][0]) - 1.0) <= TOL
