@@ -475,7 +475,12 @@ ncc_status setup_box(ncc_plan pl, int w) {
   const int64_t r = ((int64_t)maxsm / 8 - 2 * pl->box_iwp) / (2 * pl->box_iwp);
   pl->box_r = r > 16 ? 16 : (int)r;
   pl->box_smem = 0;
-  if (pl->box_r >= 1 && !getenv("NCC_BOX_TWO_PASS")) {
+  // the fused form re-sums h - 1 halo rows and w - 1 halo columns per CTA: for large windows
+  // (cfg 5: 512^2, ~45 loads per output) the two-pass form (row prefix sums, then a column
+  // scan; ~3 loads per output) is 3.3x faster (834 -> 251 us, measured); below 256 the fused
+  // form wins or ties (cfg 2: 18 vs 17.5 us, PIV 32^2: 16 us)
+  const bool large = (pl->p.tmpl_h >= 256 || w >= 256) && !getenv("NCC_BOX_FUSED");  // NCC_BOX_FUSED=1: tests
+  if (pl->box_r >= 1 && !large && !getenv("NCC_BOX_TWO_PASS")) {
     pl->box_smem = (2 * pl->box_r + 2) * pl->box_iwp * (int)sizeof(double);
     NCC_CUDA(cudaFuncSetAttribute((const void*)box2d_kernel<kBox2dNT>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   pl->box_smem));

@@ -710,7 +710,22 @@ __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ pa
         s2v[k] = __ldg(S2 + so + v);
       }
     }
-    for (int b = 0; b < nblk; ++b) {
+    int b = 0;
+    for (; b + 4 <= nblk; b += 4) {  // 16 loads in flight, summed in block order
+      float x[4][kFinV];
+#pragma unroll
+      for (int bb = 0; bb < 4; ++bb)
+#pragma unroll
+        for (int k = 0; k < kFinV; ++k) {
+          const int v = v0 + k * blockDim.x;
+          x[bb][k] = v < V ? __ldg(p + (int64_t)(b + bb) * blk_stride + v) : 0.0f;
+        }
+#pragma unroll
+      for (int bb = 0; bb < 4; ++bb)
+#pragma unroll
+        for (int k = 0; k < kFinV; ++k) tot[k] += x[bb][k];
+    }
+    for (; b < nblk; ++b) {
 #pragma unroll
       for (int k = 0; k < kFinV; ++k) {
         const int v = v0 + k * blockDim.x;

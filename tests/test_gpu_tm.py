@@ -263,7 +263,9 @@ def test_window_sum_forms_agree(h, w, monkeypatch):
     img = synth.quantize(synth.uniform_image(300, 420, 71 + w))
     u, v = int(g.integers(0, 300 - h + 1)), int(g.integers(0, 420 - w + 1))
     T = np.ascontiguousarray(img[u:u + h, v:v + w])
+    monkeypatch.setenv("NCC_BOX_FUSED", "1")  # windows >= 256 wide default to the two-pass form
     _, fused, info = run_match(img, T)
+    monkeypatch.delenv("NCC_BOX_FUSED")
     monkeypatch.setenv("NCC_BOX_TWO_PASS", "1")
     _, two, info2 = run_match(img, T)
     assert info2["launches_per_call"] == info["launches_per_call"] + 1
