@@ -1028,17 +1028,21 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   const int nblk_tc = pl->tc_nbi * pl->tc_nbj;
   auto launch_cols = [&]() {  // the ragged last columns (tensor-core path), on the side stream
-    const int64_t items = (int64_t)p.batch * pl->Ub * pl->tc_vcols;
+    // small templates: one output per warp (short CTAs that finish before the tensor-core grid
+    // needs their SMs, cfg 2); large ones: 4 sliding rows per warp (a quarter of the loads;
+    // cfg 5: 740 -> 329 us, no longer delaying the numerator's start)
+    constexpr int RWN = 4;
+    const int jc = ceil_div(p.tmpl_w, 32);
+    const int64_t items = (int64_t)p.batch * (jc <= 8 ? pl->Ub : ceil_div(pl->Ub, RWN)) * pl->tc_vcols;
     const int64_t pfs = (int64_t)pl->Ub * pl->V;
     auto cols = [&](auto kern) {
       kern<<<(unsigned)ceil_div(items, 8), 256, 0, pl->side>>>(
           d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w,
           pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, p.batch, pl->tc_part, pfs * p.batch, pfs, nblk_tc);
     };
-    const int jc = ceil_div(p.tmpl_w, 32);
     if (jc <= 4) cols(tm_tc_cols<4>);
     else if (jc <= 8) cols(tm_tc_cols<8>);
-    else cols(tm_tc_cols<16>);
+    else cols(tm_tc_cols_rw<16, RWN>);
   };
   auto launch_split = [&]() {
     tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, p.batch), 128, 0, s>>>(

@@ -555,6 +555,74 @@ __global__ void __launch_bounds__(256) tm_tc_cols(const float* __restrict__ img,
     part[(int64_t)b * blk_stride + (int64_t)f * part_frame_stride + (int64_t)ur * V + v_lo + c] = b == 0 ? tot : 0.0f;
 }
 
+// As tm_tc_cols, RWN consecutive output rows per warp: template row i is loaded once for the
+// RWN rows, and the RWN image rows in flight slide down (row ur0 + r + i lives in register slot
+// (r + i) mod RWN), so each step loads one template row and one new image row for RWN x 32 JC
+// products (0.5 loads per product at RWN = 4, was 2).  Per output the products still come
+// row by row with a fresh partial per template row (the tm_tc_cols order).  grid =
+// ceil(items / 8) with items = batch x ceil(Ub / RWN) x columns, block = 256.
+template <int JC, int RWN>
+__global__ void __launch_bounds__(256) tm_tc_cols_rw(const float* __restrict__ img, int64_t pitch,
+                                                     int64_t frame_stride, const float* __restrict__ tplC, int tplP,
+                                                     int h, int w, int v_lo, int V, int u_begin, int Ub, int batch,
+                                                     float* __restrict__ part, int64_t blk_stride,
+                                                     int64_t part_frame_stride, int nblk) {
+  const int nc = V - v_lo, nrb = (Ub + RWN - 1) / RWN;
+  const int64_t item = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
+  if (item >= (int64_t)batch * nrb * nc) return;
+  const int lane = threadIdx.x & 31;
+  const int c = (int)(item % nc);
+  const int64_t t = item / nc;
+  const int ur0 = (int)(t % nrb) * RWN, f = (int)(t / nrb);
+  const int nrows_in = Ub + h - 1;  // band rows + halo (relative to u_begin)
+  const float* I = img + (int64_t)f * frame_stride + (int64_t)(u_begin + ur0) * pitch + v_lo + c + lane;
+  const float* T = tplC + lane;
+  bool okc[JC];
+#pragma unroll
+  for (int k = 0; k < JC; ++k) okc[k] = lane + 32 * k < w;
+  float win[RWN][JC];
+  auto load_row = [&](float (&dst)[JC], int rr) {  // image row ur0 + rr of the band
+    const bool ok = ur0 + rr < nrows_in;
+#pragma unroll
+    for (int k = 0; k < JC; ++k) dst[k] = (ok && okc[k]) ? __ldg(I + (int64_t)rr * pitch + 32 * k) : 0.0f;
+  };
+#pragma unroll
+  for (int r = 0; r < RWN - 1; ++r) load_row(win[r], r);
+  float tot[RWN];
+#pragma unroll
+  for (int r = 0; r < RWN; ++r) tot[r] = 0.0f;
+  for (int i0 = 0; i0 < h; i0 += RWN) {
+#pragma unroll
+    for (int s = 0; s < RWN; ++s) {
+      const int i = i0 + s;
+      if (i < h) {
+        load_row(win[(RWN - 1 + s) % RWN], RWN - 1 + i);
+        float tv[JC];
+#pragma unroll
+        for (int k = 0; k < JC; ++k) tv[k] = okc[k] ? __ldg(T + (int64_t)i * tplP + 32 * k) : 0.0f;
+#pragma unroll
+        for (int r = 0; r < RWN; ++r) {
+          float pr = 0.0f;  // fresh partial per template row
+#pragma unroll
+          for (int k = 0; k < JC; ++k) pr = fmaf(tv[k], win[(r + s) % RWN][k], pr);
+          tot[r] += pr;
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int r = 0; r < RWN; ++r) {
+#pragma unroll
+    for (int d = 16; d; d >>= 1) tot[r] += __shfl_xor_sync(0xffffffffu, tot[r], d);
+  }
+  for (int b = lane; b < nblk; b += 32)
+#pragma unroll
+    for (int r = 0; r < RWN; ++r)
+      if (ur0 + r < Ub)
+        part[(int64_t)b * blk_stride + (int64_t)f * part_frame_stride + (int64_t)(ur0 + r) * V + v_lo + c] =
+            b == 0 ? tot[r] : 0.0f;
+}
+
 // Template operand: for block (bi, bj) the reversed, zero-padded rows Rv[k] = A_C[i0 + K0 - k]
 // (K0 = kHB + kG - 2, zero outside the block / template), split into tf32 hi and fp32 lo, laid
 // out [2][WC/4 planes][kLB rows][4 floats] (the UMMA K-major no-swizzle canonical layout with
