@@ -1100,7 +1100,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     mark(pl, s, 2);
   } else {
     // window sums on the main stream while the template prep runs on the side stream
-    if (pl->tc && pl->tc_vcols) {  // after the join: overlaps the tensor-core kernel rather than delay its start
+    if (tc_now && pl->tc_vcols) {  // after the join: overlaps the tensor-core kernel rather than delay its start
       launch_cols();
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }

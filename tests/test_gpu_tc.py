@@ -148,3 +148,38 @@ def test_tc_block_boundaries(h, w):
     assert info["variant_name"].startswith("tm_tc")
     assert np.max(np.abs(s[0] - ref)) <= TOL
     assert (peaks["u"][0], peaks["v"][0]) == (u0, v0)
+
+
+@pytest.mark.parametrize("H,W,h,w", [(400, 556, 300, 300), (380, 555, 260, 299)])
+def test_tc_large_template_ragged_columns(H, W, h, w):
+    """Templates wider than 256 with a ragged last output column (V = 1 mod 128): the ragged
+    column comes from tm_tc_cols_rw (4 sliding output rows per warp) and the window sums from the
+    two-pass form; full surface vs the fp64 oracle, planted peak exact.  W = 555 has a row of
+    (hi, lo) pairs that is not a 16-byte multiple: the plan falls back to the CUDA-core kernel at
+    run time (and its captured graph must not leave the ragged-column launch unjoined)."""
+    img = synth.uniform_image(H, W, h + w + 1)
+    T, u0, v0 = synth.planted_template(img, h, w, 3 * h + 1)
+    ref, pk = oracle.ncc_match(img, T)
+    peaks, s, info = run([img], T)
+    assert info["variant_name"].startswith("tm_tc") and info["variant_name"].endswith("_cols"), info["variant_name"]
+    assert np.max(np.abs(s[0] - ref)) <= TOL
+    assert np.max(np.abs(s[0][:, -2:] - ref[:, -2:])) <= TOL
+    assert (int(peaks["u"][0]), int(peaks["v"][0])) == (pk.u, pk.v) == (u0, v0)
+
+
+def test_tc_cfg5_full_surface_fft():
+    """cfg5 (4096^2 frame, 512^2 template) on the default tensor-core plan: full surface vs the
+    independent fp64 FFT route (pinned to brute force in test_oracle.py), brute-force samples
+    including the ragged last column, planted peak exact."""
+    from oracle.ncc_fft import ncc_surface_fft
+    img, T, u0, v0 = synth.tm_inputs(5, k=3)
+    peaks, s, info = run([img], T)
+    assert info["variant_name"].startswith("tm_tc"), info["variant_name"]
+    f = ncc_surface_fft(img, T)
+    assert np.max(np.abs(s[0] - f)) <= TOL
+    g = synth.rng(99)
+    us = np.concatenate([g.integers(0, 3585, 24), [u0, 3584, 0, 1792]])
+    vs = np.concatenate([g.integers(0, 3585, 24), [v0, 3584, 3584, 3584]])
+    bf = oracle.ncc_at(img, T, us, vs)
+    assert np.max(np.abs(s[0][us, vs] - bf)) <= TOL
+    assert (int(peaks["u"][0]), int(peaks["v"][0])) == (u0, v0)
