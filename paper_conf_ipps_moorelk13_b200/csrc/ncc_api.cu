@@ -554,7 +554,8 @@ ncc_status setup_tc(ncc_plan pl) {
   ncc_status st;
   if ((st = dalloc(&pl->tcB, (size_t)nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
   if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
-  if ((st = dalloc(&pl->tc_img2, (size_t)2 * p.batch * pl->Hs * p.image_w))) return st;  // (hi, lo) pairs
+  // (hi, lo) pairs, rows padded to an even count of pairs: a 16-byte multiple for the TMA map
+  if ((st = dalloc(&pl->tc_img2, (size_t)2 * p.batch * pl->Hs * ((p.image_w + 1) & ~1)))) return st;
   if ((st = dalloc(&pl->tc_done, (size_t)p.batch))) return st;
   NCC_CUDA(cudaMemset(pl->tc_done, 0, (size_t)p.batch * sizeof(unsigned int)));
   const int smem = tc::smem_bytes(pl->tc_wc);
@@ -1022,7 +1023,8 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   bool tc_now = false;
   if (pl->tc) {  // the band's rows as (hi, lo) pairs: W x Hs x batch 8-byte elements
     const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)pl->Hs, (uint64_t)p.batch};
-    const uint64_t strides[2] = {(uint64_t)p.image_w * 8, (uint64_t)pl->Hs * p.image_w * 8};
+    const int wp = (p.image_w + 1) & ~1;  // pairs per staged row (even)
+    const uint64_t strides[2] = {(uint64_t)wp * 8, (uint64_t)pl->Hs * wp * 8};
     const uint32_t box[3] = {(uint32_t)tc::kBoxW, 1u, 1u};
     tc_now = encode_f32(&map_tc, pl->tc_img2, 3, dims, strides, box, true);
   }
@@ -1047,7 +1049,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   auto launch_split = [&]() {
     tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, p.batch), 128, 0, s>>>(
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
-        reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * p.image_w);
+        reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 1) & ~1), (p.image_w + 1) & ~1);
   };
   // fork: template prep on the side stream
   mark(pl, s, 0);

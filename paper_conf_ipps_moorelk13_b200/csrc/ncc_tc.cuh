@@ -478,14 +478,16 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 // Image operand of the tensor-core numerator: every element of the band's rows split once into
 // (hi = tf32(x) with round-to-nearest, lo = x - hi, exact in fp32), stored as an 8-byte pair so
 // the producer warps load each Hankel element with one LDS.64.  grid = (ceil(W/4/128), rows,
-// batch), block = 128; out row r = image row row0 + r.
+// batch), block = 128; out row r = image row row0 + r, rows out_pitch (even: 16-byte TMA stride)
+// pairs apart.
 __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
-                                                   int W, int row0, uint2* __restrict__ out, int64_t out_frame_stride) {
+                                                   int W, int row0, uint2* __restrict__ out, int64_t out_frame_stride,
+                                                   int out_pitch) {
   const int c = (blockIdx.x * 128 + threadIdx.x) * 4;
   if (c >= W) return;
   const int r = blockIdx.y, f = blockIdx.z;
   const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch + c;
-  uint2* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * W + c;
+  uint2* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * out_pitch + c;
   float x[4];
   if (c + 4 <= W && (reinterpret_cast<uintptr_t>(src) & 15) == 0) {
     const float4 v = __ldg(reinterpret_cast<const float4*>(src));

@@ -107,7 +107,8 @@ def test_tc_matches_cuda_core_path(monkeypatch):
 
 
 def test_tc_unaligned_pitch_falls_back_at_run_time():
-    """pitch % 4 != 0: no TMA map for the image -> the plan runs its CUDA-core kernel."""
+    """pitch % 4 != 0: the image split (tm_tc_split) reads rows with scalar loads; the
+    tensor-core kernel reads its own (hi, lo) copy through TMA; results stay exact."""
     img, T, u0, v0 = synth.tm_inputs(2, k=9)
     H, W = img.shape
     P = W + 1
@@ -154,9 +155,8 @@ def test_tc_block_boundaries(h, w):
 def test_tc_large_template_ragged_columns(H, W, h, w):
     """Templates wider than 256 with a ragged last output column (V = 1 mod 128): the ragged
     column comes from tm_tc_cols_rw (4 sliding output rows per warp) and the window sums from the
-    two-pass form; full surface vs the fp64 oracle, planted peak exact.  W = 555 has a row of
-    (hi, lo) pairs that is not a 16-byte multiple: the plan falls back to the CUDA-core kernel at
-    run time (and its captured graph must not leave the ragged-column launch unjoined)."""
+    two-pass form; full surface vs the fp64 oracle, planted peak exact.  W = 555: the staged
+    (hi, lo) rows are padded to an even number of pairs (16-byte TMA stride)."""
     img = synth.uniform_image(H, W, h + w + 1)
     T, u0, v0 = synth.planted_template(img, h, w, 3 * h + 1)
     ref, pk = oracle.ncc_match(img, T)
