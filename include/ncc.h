@@ -25,6 +25,11 @@
  *    staging buffers.  One plan is used by one stream at a time.
  *  - Execute calls are asynchronous on `stream` (cudaStream_t passed as void*; NULL = the
  *    legacy default stream).  Results are valid after the stream is synchronised.
+ *  - Execute calls replay CUDA graphs: the first call with a given set of pointer arguments
+ *    captures the plan's launch sequence (on a plan-owned capture stream) and later calls with
+ *    the same pointers launch it as one graph; a plan keeps up to 4 such graphs.  Buffers may
+ *    be reused or replaced freely between calls (a new pointer set is captured on first use);
+ *    NCC_NO_GRAPH=1 in the environment launches kernel by kernel.
  *  - Errors: shape/argument errors are returned by ncc_plan_create
  *    (NCC_ERR_INVALID_ARGUMENT); launch failures by the execute call (NCC_ERR_CUDA).
  *    Data-dependent conditions are never status codes: they are flag bits in the outputs.
@@ -193,8 +198,12 @@ ncc_status piv_correlate_ex(ncc_plan plan, const float* d_frames_a, const float*
 
 /* Host-buffer variants (end-to-end path): copy inputs host->device into plan-owned
  * staging buffers on `stream`, run, and copy results device->host.  Pinned host memory
- * gives asynchronous copies; results are valid after the stream is synchronised.
- * h_scores may be NULL (not copied back). */
+ * gives asynchronous copies (and, for ncc_match_host, copies captured into the launch
+ * sequence: the template's copy overlaps the frames'); results are valid after the stream is
+ * synchronised.  h_scores may be NULL (not copied back).  piv_correlate_host streams batches
+ * larger than one sub-batch through two device slots (the copy of chunk c+1 overlaps the
+ * correlation of chunk c on a plan-owned copy stream); the host buffers must stay valid until
+ * the stream is synchronised. */
 ncc_status ncc_match_host(ncc_plan plan, const float* h_images, const float* h_tmpl,
                           int64_t tmpl_pitch, float* h_scores, ncc_peak* h_peaks, void* stream);
 ncc_status piv_correlate_host(ncc_plan plan, const float* h_frames_a, const float* h_frames_b,
