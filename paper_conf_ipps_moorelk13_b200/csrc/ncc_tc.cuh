@@ -279,11 +279,23 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       // the split x = hi + lo was done once per image element (tm_tc_split): one 8-byte load
       // per Hankel element, no per-lane conversion work
       const bool zero = stage_zero(q) || TC_EXP(64);
+      // 16-byte loads from the even element at or below v (lanes 2i and 2i+1 share them: half
+      // the shared-memory wavefronts of one 8-byte load per element), odd lanes shift by one
+      const uint4* r4 = reinterpret_cast<const uint4*>(ring + sl * kBoxW + (v & ~1));
+      const bool odd = (v & 1) != 0;
+      uint32_t eh[kWB + 2], el[kWB + 2];
+#pragma unroll
+      for (int m = 0; m < kWB / 2 + 1; ++m) {
+        const uint4 t = zero ? make_uint4(0u, 0u, 0u, 0u) : r4[m];
+        eh[2 * m] = t.x;
+        el[2 * m] = t.y;
+        eh[2 * m + 1] = t.z;
+        el[2 * m + 1] = t.w;
+      }
 #pragma unroll
       for (int k = 0; k < kWB; ++k) {
-        const uint2 p = zero ? make_uint2(0u, 0u) : ring[sl * kBoxW + v + k];
-        hi[k] = p.x;
-        lo[k] = p.y;
+        hi[k] = odd ? eh[k + 1] : eh[k];
+        lo[k] = odd ? el[k + 1] : el[k];
       }
       mbar_arrive(&img_empty[sl]);
       if (gtid == 0) TC_STAMP(1, q);
