@@ -489,7 +489,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 
 // Image operand of the tensor-core numerator: every element of the band's rows split once into
 // (hi = tf32(x) with round-to-nearest, lo = x - hi, exact in fp32), stored as an 8-byte pair so
-// the producer warps load each Hankel element with one LDS.64.  grid = (ceil(W/4/128), rows,
+// the producer warps load the Hankel elements directly (16-byte loads).  grid = (ceil(W/4/128), rows,
 // batch), block = 128; out row r = image row row0 + r, rows out_pitch (even: 16-byte TMA stride)
 // pairs apart.
 __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
