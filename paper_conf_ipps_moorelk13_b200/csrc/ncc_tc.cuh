@@ -831,7 +831,9 @@ __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ pa
   }
   best = block_max_key(best, red);
   if (threadIdx.x == 0) {
-    if (best) atomicMax(keys + f, best);
+    // keys only grow: a CTA whose best is not above the (possibly stale) current key skips
+    // its atomic -- most do, which halves the same-address atomics of the grid
+    if (best && best > __ldcg(keys + f)) atomicMax(keys + f, best);
     // the frame's last CTA turns the key into its peak (tm_finalize fused): every CTA's
     // atomicMax is ordered before its counter increment
     __threadfence();
