@@ -301,6 +301,17 @@ def main():
         hv = torch.empty(vec.shape, dtype=torch.int32).pin_memory()
         e2e_step = lambda: plan.correlate_host(hA, hB, hv, stream=stream)  # noqa: E731
 
+    # ---- multi-GPU: every timed step ends with the path's only collective, the gather of the
+    # 16-B peaks / 24-B vectors to all ranks (NCCL over NVLink, ordered on the compute stream)
+    if ws > 1:
+        res_t = peaks if wl["kind"] == "tm" else vec.reshape(-1, 6)
+        gathered_t = torch.empty((ws,) + tuple(res_t.shape), dtype=res_t.dtype, device=dev)
+        compute_step = step
+
+        def step():
+            compute_step()
+            dist.all_gather_into_tensor(gathered_t, res_t)
+
     # ---- warmup, then the timed region (barrier + sync on both sides)
     run_steps(step, args.warmup, plan)
     sampler = ClockSampler(physical_gpu_index(local))
