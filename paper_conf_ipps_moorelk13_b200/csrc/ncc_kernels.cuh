@@ -2283,7 +2283,23 @@ __global__ void __launch_bounds__(256) tm_tiny_kernel(const float* __restrict__ 
   // image rows of this CTA
   const float* src = img + (int64_t)f * frame_stride + (int64_t)(u_begin + r0) * pitch;
   const int nr = rows + h - 1;
-  for (int k = threadIdx.x; k < nr * W; k += blockDim.x) X[k] = __ldg(src + (int64_t)(k / W) * pitch + k % W);
+  {  // all of a thread's loads in flight before its stores (one memory round trip, not one per element)
+    constexpr int LB = 8;
+    const int ne = nr * W;
+    for (int k0 = threadIdx.x; k0 < ne; k0 += LB * blockDim.x) {
+      float v[LB];
+#pragma unroll
+      for (int r = 0; r < LB; ++r) {
+        const int k = k0 + r * blockDim.x;
+        v[r] = k < ne ? __ldg(src + (int64_t)(k / W) * pitch + k % W) : 0.0f;
+      }
+#pragma unroll
+      for (int r = 0; r < LB; ++r) {
+        const int k = k0 + r * blockDim.x;
+        if (k < ne) X[k] = v[r];
+      }
+    }
+  }
   s = block_sum_d(s, red);
   s2 = block_sum_d(s2, red);
   const double mean = s / (double)n, inv_n = 1.0 / (double)n;
