@@ -105,3 +105,21 @@ def test_c_example_compiles_against_the_header(tmp_path):
                         "-o", str(exe), "-L", os.path.dirname(N.LIB_PATH), "-lncc_b200",
                         "-Wl,-rpath," + os.path.dirname(N.LIB_PATH)], capture_output=True, text=True)
     assert r.returncode == 0, r.stderr
+
+
+def test_experiments_tables_match_the_committed_sweep(tmp_path):
+    """EXPERIMENTS.md's tables are generated from profiles/r01_paper_sweeps.jsonl
+    (tools/experiments_md.py): regenerating them from the committed measurements changes
+    nothing, and every sweep run was correct against its planted input."""
+    import json
+    import shutil
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    src = os.path.join(root, "profiles", "r01_paper_sweeps.jsonl")
+    md = tmp_path / "EXPERIMENTS.md"
+    shutil.copy(os.path.join(root, "EXPERIMENTS.md"), md)
+    subprocess.run([sys.executable, os.path.join(root, "tools", "experiments_md.py"), src, str(md)], check=True)
+    assert md.read_text() == open(os.path.join(root, "EXPERIMENTS.md")).read()
+    rows = [json.loads(l) for l in open(src) if l.strip().startswith("{")]
+    assert rows and all(r["correct"] in (True, None) for r in rows)
