@@ -2212,7 +2212,7 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
         for (int q = 0; q < RV / 2; ++q) tot2[q] = 0ull;
         const float* brow = Bs(s, wi) + row * S::BP + g * RV;
         const u64* tpw = TPs(s, wi);
-#pragma unroll 1
+#pragma unroll 2
         for (int i = 0; i < TH; ++i) {
 #pragma unroll
           for (int jc = 0; jc < S::nCW; ++jc) {
