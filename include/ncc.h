@@ -69,7 +69,7 @@ enum { NCC_SUBPIX_GAUSS3 = 0, NCC_SUBPIX_PARABOLA3 = 1, NCC_SUBPIX_NONE = 2 };
 enum {
     NCC_F_WRITE_SURFACE = 1u,  /* TM: ncc_match writes the score surface (d_scores required) */
     NCC_F_GENERIC_KERNEL = 2u, /* force the run-time-evaluated (RE) generic kernels         */
-    NCC_F_NO_JIT = 4u,         /* reserved: never compile at run time                        */
+    NCC_F_NO_JIT = 4u,         /* never compile at run time (NVRTC): AOT instance or generic */
     NCC_F_TIMING = 8u,         /* record per-stage CUDA-event timings (ncc_plan_timing)     */
     NCC_F_CUDA_CORES = 16u     /* TM: never use the tensor-core (tcgen05 3xTF32) numerator   */
 };
@@ -141,7 +141,10 @@ typedef struct {
     int32_t batch;
     int64_t outputs_per_call;  /* TM: band offsets x batch; PIV: Ky*Kx*batch vectors        */
     double flops_per_call;     /* algorithmic numerator FLOP per call (2hw per offset)      */
-    int32_t specialized;       /* 1 = compile-time specialised (SK) kernel, 0 = generic (RE) */
+    int32_t specialized;       /* numerator tier: 1 = ahead-of-time specialised (SK) instance,
+                                  2 = run-time specialised (NVRTC) kernel, 0 = generic run-time-
+                                  evaluated (RE) kernel, 3 = tensor-core kernel (tcgen05 3xTF32;
+                                  one kernel for every shape, h and w run-time evaluated)       */
     int32_t variant_id;        /* index into the variant table                              */
     int32_t regs_per_thread;   /* numerator kernel registers/thread                         */
     int32_t threads_per_block; /* numerator kernel block size                               */

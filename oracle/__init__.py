@@ -70,11 +70,14 @@ def lib():
         _lib.oracle_template_is_flat.argtypes = [P, i64, i32, i32]
         _lib.oracle_subpixel3.argtypes = [ctypes.c_double] * 3 + [ctypes.POINTER(ctypes.c_int)]
         _lib.oracle_subpixel3.restype = ctypes.c_double
+        _lib.oracle_subpixel3_min.argtypes = [ctypes.c_double] * 3
+        _lib.oracle_subpixel3_min.restype = ctypes.c_double
         _lib.oracle_piv_grid.argtypes = [i32] * 8 + [ctypes.POINTER(ctypes.c_int)] * 2
         _lib.oracle_piv_pair.argtypes = [P, P, i32, i32, i64] + [i32] * 6 + [P, P]
         _lib.oracle_piv_windows.argtypes = [P, P, i32, i32, i64] + [i32] * 6 + [P, P, i32, P, P]
         _lib.oracle_piv_window_scores.argtypes = [P, P, i32, i32, i64] + [i32] * 8 + [P]
         _lib.oracle_num_threads.restype = i32
+        _lib.oracle_set_num_threads.argtypes = [i32]
         _lib.oracle_ssd_surface.argtypes = [P, i32, i32, i64, P, i32, i32, i64, i32, i32, P]
         _lib.oracle_argmin.argtypes = [P, i64]
         _lib.oracle_argmin.restype = i64
@@ -93,6 +96,11 @@ def _ptr(a: np.ndarray):
 
 def num_threads() -> int:
     return int(lib().oracle_num_threads())
+
+
+def set_num_threads(n: int) -> None:
+    """OpenMP threads for later oracle calls (bench.py times a 1-thread rate beside the full one)."""
+    lib().oracle_set_num_threads(int(n))
 
 
 def ncc_surface(img: np.ndarray, tmpl: np.ndarray, u_begin: int = 0, u_end: int | None = None) -> np.ndarray:
@@ -154,6 +162,11 @@ def subpixel3(cm: float, c0: float, cp: float) -> tuple[float, bool]:
     par = ctypes.c_int(0)
     d = lib().oracle_subpixel3(float(cm), float(c0), float(cp), ctypes.byref(par))
     return float(d), bool(par.value)
+
+
+def subpixel3_min(cm: float, c0: float, cp: float) -> float:
+    """3-point parabolic fit of a minimum (SSD sub-pixel, Fig 5.10): 0 if not a minimum."""
+    return float(lib().oracle_subpixel3_min(float(cm), float(c0), float(cp)))
 
 
 def piv_grid(H, W, h, w, my, mx, sy, sx) -> tuple[int, int]:

@@ -203,6 +203,19 @@ double oracle_subpixel3(double cm, double c0, double cp, int *parabola)
     return num / den;
 }
 
+/* ---------------------------------------------------------------------------
+ * Sub-pixel 3-point fit of a MINIMUM along one axis (SSD, the paper's PIV score: Fig 5.10
+ * caption P:167-168 "offset sum of squared differences"; S8c reading 6): the parabola
+ * through (-1, cm), (0, c0), (+1, cp) has its vertex at delta = (c- - c+) / (2 (c- - 2 c0 + c+));
+ * it is a minimum only when that denominator is > 0, otherwise no fit (delta = 0).
+ * ------------------------------------------------------------------------- */
+double oracle_subpixel3_min(double cm, double c0, double cp)
+{
+    const double den = 2.0 * (cm - 2.0 * c0 + cp);
+    if (den <= 0.0) return 0.0; /* not a minimum (or flat): no fit */
+    return (cm - cp) / den;
+}
+
 typedef struct {
     int32_t iy, ix;  /* integer displacement of the peak (dy*, dx*)         */
     double dy, dx;   /* sub-pixel displacement dy* + delta_y, dx* + delta_x */
@@ -272,18 +285,14 @@ static void piv_one_window_ssd(const float *A, const float *B, int64_t pitch,
     if (iy == -my || iy == my) {
         flags |= OF_EDGE_Y;
     } else {
-        const double cm = scratch[(iy + my - 1) * OX + (ix + mx)], c0 = scratch[(iy + my) * OX + (ix + mx)],
-                     cp = scratch[(iy + my + 1) * OX + (ix + mx)];
-        const double den = 2.0 * (cm - 2.0 * c0 + cp);
-        if (den > 0.0) ddy = (cm - cp) / den;
+        ddy = oracle_subpixel3_min(scratch[(iy + my - 1) * OX + (ix + mx)], scratch[(iy + my) * OX + (ix + mx)],
+                                   scratch[(iy + my + 1) * OX + (ix + mx)]);
     }
     if (ix == -mx || ix == mx) {
         flags |= OF_EDGE_X;
     } else {
-        const double cm = scratch[(iy + my) * OX + (ix + mx - 1)], c0 = scratch[(iy + my) * OX + (ix + mx)],
-                     cp = scratch[(iy + my) * OX + (ix + mx + 1)];
-        const double den = 2.0 * (cm - 2.0 * c0 + cp);
-        if (den > 0.0) ddx = (cm - cp) / den;
+        ddx = oracle_subpixel3_min(scratch[(iy + my) * OX + (ix + mx - 1)], scratch[(iy + my) * OX + (ix + mx)],
+                                   scratch[(iy + my) * OX + (ix + mx + 1)]);
     }
     out->iy = iy;
     out->ix = ix;
@@ -375,6 +384,17 @@ int oracle_piv_windows_ssd(const float *A, const float *B, int H, int W, int64_t
         piv_one_window_ssd(A, B, pitch, h, w, my, mx, my + kys[i] * sy, mx + kxs[i] * sx,
                            scratch + (int64_t)i * per, &out[i]);
     return 0;
+}
+
+/* Set the OpenMP thread count of later calls (bench.py's 1-thread oracle rate). */
+void oracle_set_num_threads(int n)
+{
+#ifdef _OPENMP
+    extern void omp_set_num_threads(int);
+    if (n > 0) omp_set_num_threads(n);
+#else
+    (void)n;
+#endif
 }
 
 int oracle_num_threads(void)

@@ -25,6 +25,45 @@ def decode_vectors(raw: torch.Tensor) -> dict:
             "dx": raw[..., 3].view(torch.float32), "score": raw[..., 4].view(torch.float32), "flags": raw[..., 5]}
 
 
+def _check_tensor(t, name: str, dtype, device, min_numel: int, last_dims=None, contiguous=True):
+    """Raise ValueError unless `t` can be handed to the C ABI as a flat buffer of `min_numel`
+    elements: dtype, device (a torch.device, or None for host memory), contiguity (or unit
+    stride in the last dimension when contiguous=False), size and the trailing dimensions."""
+    import torch as _t
+    if not isinstance(t, _t.Tensor):
+        raise ValueError(f"{name}: expected a torch.Tensor, got {type(t).__name__}")
+    if t.dtype != dtype:
+        raise ValueError(f"{name}: dtype {t.dtype}, expected {dtype}")
+    if device is None:
+        if t.is_cuda:
+            raise ValueError(f"{name}: expected a host tensor, got {t.device}")
+    elif t.device != device:
+        raise ValueError(f"{name}: on {t.device}, expected {device}")
+    if contiguous and not t.is_contiguous():
+        raise ValueError(f"{name}: must be contiguous")
+    if not contiguous and t.dim() and t.stride(-1) != 1:
+        raise ValueError(f"{name}: the last dimension must have unit stride")
+    if last_dims is not None:
+        got = tuple(t.shape[-len(last_dims):]) if t.dim() >= len(last_dims) else tuple(t.shape)
+        if got != tuple(last_dims):
+            raise ValueError(f"{name}: trailing shape {got}, expected {tuple(last_dims)}")
+    span = t.numel() if contiguous else (1 + sum((d - 1) * st for d, st in zip(t.shape, t.stride())) if t.numel() else 0)
+    if span < min_numel:
+        raise ValueError(f"{name}: {span} elements, need at least {min_numel}")
+
+
+def _check_template(t, name: str, h: int, w: int, device, count: int = 1):
+    """Template(s): (h, >= w) or (count, h, >= w) fp32 with unit column stride; the row stride
+    is passed to the C ABI as the template pitch."""
+    import torch as _t
+    _check_tensor(t, name, _t.float32, device, 0, contiguous=False)
+    want_dim = 2 if count == 1 and t.dim() == 2 else 3
+    if t.dim() != want_dim or t.shape[-2] < h or t.shape[-1] < w or (want_dim == 3 and t.shape[0] < count):
+        raise ValueError(f"{name}: shape {tuple(t.shape)}, expected ({'%d, ' % count if want_dim == 3 else ''}{h}, >={w})")
+    if want_dim == 3 and t.stride(0) != t.stride(1) * h:
+        raise ValueError(f"{name}: templates must be {h} rows of one pitch apart (stride(0) == h * stride(1))")
+
+
 class _Plan:
     def __init__(self, problem: N.NccProblem, device: int):
         self.problem = problem
@@ -76,14 +115,30 @@ class MatchPlan(_Plan):
     def band_rows(self):
         return self.info.u_end - self.info.u_begin
 
+    def _frames_numel(self):
+        p = self.problem
+        return p.batch * p.image_h * p.image_pitch
+
+    def _check_match_io(self, images, tmpl, peaks, scores, device, count=1):
+        p = self.problem
+        _check_tensor(images, "images", torch.float32, device, self._frames_numel(),
+                      last_dims=(p.image_h, p.image_pitch))
+        _check_template(tmpl, "tmpl" if count == 1 else "tmpls", p.tmpl_h, p.tmpl_w, device, count)
+        _check_tensor(peaks, "peaks", torch.int32, device, p.batch * count * 4)
+        if self.write_surface and scores is not None:
+            rows, cols = (p.roi_h, p.roi_w) if count > 1 or p.roi_h else (self.band_rows, self.info.V)
+            _check_tensor(scores, "scores", torch.float32, device, p.batch * count * rows * cols)
+
     def match(self, images: torch.Tensor, tmpl: torch.Tensor, stream=None, peaks=None, scores=None):
+        """images: (batch, H, pitch) or (H, pitch) fp32 on the plan's device; tmpl (h, >= w) with
+        unit column stride.  Shapes, dtypes, devices and output sizes are checked (ValueError)."""
         p = self.problem
         dev = torch.device("cuda", self.device)
-        assert images.is_cuda and images.dtype == torch.float32 and tmpl.dtype == torch.float32
         if peaks is None:
             peaks = torch.empty((p.batch, 4), dtype=torch.int32, device=dev)
         if self.write_surface and scores is None:
             scores = torch.empty((p.batch, self.band_rows, self.info.V), dtype=torch.float32, device=dev)
+        self._check_match_io(images, tmpl, peaks, scores, dev)
         N.ncc_match(self.handle, images, tmpl, tmpl.stride(0), scores, peaks, self._stream(stream))
         return peaks, scores
 
@@ -97,11 +152,15 @@ class MatchPlan(_Plan):
             peaks = torch.empty((p.batch, T, 4), dtype=torch.int32, device=dev)
         if self.write_surface and scores is None:
             scores = torch.empty((p.batch, T, p.roi_h, p.roi_w), dtype=torch.float32, device=dev)
+        self._check_match_io(images, tmpls, peaks, scores, dev, count=T)
+        _check_tensor(rois, "rois", torch.int32, dev, p.batch * T * 2)
         N.ncc_match_rois(self.handle, images, tmpls, tmpls.stride(1), rois, scores, peaks, self._stream(stream))
         return peaks, scores
 
     def match_host(self, h_images: torch.Tensor, h_tmpl: torch.Tensor, h_peaks: torch.Tensor, h_scores=None,
                    stream=None):
+        """Host tensors (pinned for asynchronous, captured copies); same layouts as match()."""
+        self._check_match_io(h_images, h_tmpl, h_peaks, h_scores, None)
         N.ncc_match_host(self.handle, h_images, h_tmpl, h_tmpl.stride(0), h_scores, h_peaks, self._stream(stream))
         return h_peaks
 
@@ -132,9 +191,19 @@ class PivPlan(_Plan):
         if scores:
             sc = torch.empty((p.batch, Ky, Kx, 2 * p.search_y + 1, 2 * p.search_x + 1), dtype=torch.float32,
                              device=dev)
+        self._check_piv_io(A, B, vectors, dev)
         N.piv_correlate_ex(self.handle, A, B, sc, vectors, self._stream(stream))
         return vectors, sc
 
+    def _check_piv_io(self, A, B, vectors, device):
+        p = self.problem
+        n = p.batch * p.image_h * p.image_pitch
+        _check_tensor(A, "frames_a", torch.float32, device, n, last_dims=(p.image_h, p.image_pitch))
+        _check_tensor(B, "frames_b", torch.float32, device, n, last_dims=(p.image_h, p.image_pitch))
+        Ky, Kx = self.grid
+        _check_tensor(vectors, "vectors", torch.int32, device, p.batch * Ky * Kx * 6)
+
     def correlate_host(self, h_A, h_B, h_vectors, stream=None):
+        self._check_piv_io(h_A, h_B, h_vectors, None)
         N.piv_correlate_host(self.handle, h_A, h_B, h_vectors, self._stream(stream))
         return h_vectors

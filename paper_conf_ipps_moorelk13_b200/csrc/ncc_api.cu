@@ -355,6 +355,7 @@ struct ncc_plan_s {
   struct GraphEntry {
     uintptr_t key[8];
     cudaGraphExec_t exec;
+    int timing_kind, piv_nsub;  // host-side facts of the captured sequence, restored on replay
   } graphs[4];
   int n_graphs, next_graph;
 };
@@ -404,7 +405,8 @@ void free_plan(ncc_plan pl) {
   }
   if (pl->ev_start) cudaEventDestroy(pl->ev_start);
   if (pl->copy) cudaStreamDestroy(pl->copy);
-  for (int k = 0; k < pl->n_graphs; ++k) cudaGraphExecDestroy(pl->graphs[k].exec);
+  for (int k = 0; k < pl->n_graphs; ++k)
+    if (pl->graphs[k].exec) cudaGraphExecDestroy(pl->graphs[k].exec);
   if (pl->cap) cudaStreamDestroy(pl->cap);
   if (pl->jit_lib) cudaLibraryUnload(pl->jit_lib);
   delete pl;
@@ -567,7 +569,7 @@ ncc_status setup_tc(ncc_plan pl) {
   snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d%s", tc::kHB, pl->tc_wc, pl->tc_nseg,
            pl->tc_vcols ? "_cols" : "");
   fill_kernel_info(pl, (const void*)tm_tc_kernel, tc::kThreads, smem, nblk * pl->tc_vtiles * pl->tc_nseg, p.batch, 1);
-  in.specialized = 1;
+  in.specialized = 3;  // tensor-core tier: one kernel for every shape (h, w run-time evaluated), not an SK
   in.split = nblk;
   in.const_template = 0;
   in.slabs = 1;
@@ -1051,17 +1053,20 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
         reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 1) & ~1), (p.image_w + 1) & ~1);
   };
-  // fork: template prep on the side stream
+  // fork: template prep on the side stream.  Host path: the frames' copy is issued on the main
+  // stream BEFORE the fork event, so everything on the side stream that reads the frames (the
+  // ragged-column kernel, the late window sums) is ordered after it; the template's copy runs on
+  // the side stream ahead of its prep, concurrently with the frames' copy.
   mark(pl, s, 0);
+  if (pl->h_img_in)
+    NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
+                             (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
   NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
   NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
-  if (pl->h_tmpl_in) {  // host path: template copy ahead of its prep, frames on the main stream
+  if (pl->h_tmpl_in)
     NCC_CUDA(cudaMemcpy2DAsync(const_cast<float*>(d_tmpl), tmpl_pitch * sizeof(float), pl->h_tmpl_in,
                                pl->h_tmpl_pitch * sizeof(float), p.tmpl_w * sizeof(float), p.tmpl_h,
                                cudaMemcpyHostToDevice, pl->side));
-    NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
-                             (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
-  }
   if (pl->tc && p.tmpl_h * p.tmpl_w <= kPrepSmemFloats && !getenv_flag_two_kernel_prep()) {
     // one launch: template stats + centred template + MMA operand, template staged in shared memory
     tm_tc_prep<<<nblk_tc, 1024, p.tmpl_h * p.tmpl_w * 4, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
@@ -1357,18 +1362,43 @@ ncc_status run_graph(ncc_plan pl, const uintptr_t (&key)[8], cudaStream_t s, Bod
     }
     if (e != cudaSuccess) return cuda_fail(e, "graph capture");
     cudaGraphExec_t ex = nullptr;
-    const cudaError_t ei = cudaGraphInstantiate(&ex, g, 0);
-    cudaGraphDestroy(g);
-    if (ei != cudaSuccess) return cuda_fail(ei, "graph instantiate");
-    if (pl->n_graphs < 4) {
+    const bool fresh_slot = pl->n_graphs < 4;
+    if (fresh_slot) {
       hit = pl->n_graphs++;
-    } else {  // replace round robin (the replaced graph may still run: destroy is deferred by CUDA)
+      pl->graphs[hit].exec = nullptr;
+    } else {
+      // evict round robin.  Callers rotating more than 4 buffer sets would otherwise pay a full
+      // instantiation per call: the evicted executable is updated in place with the new graph
+      // (same topology, new pointer arguments) when CUDA allows it; else re-instantiated.  (A
+      // replay still in flight keeps the parameters it was launched with.)
       hit = pl->next_graph;
       pl->next_graph = (pl->next_graph + 1) % 4;
-      cudaGraphExecDestroy(pl->graphs[hit].exec);
+      cudaGraphExecUpdateResultInfo ui;
+      if (cudaGraphExecUpdate(pl->graphs[hit].exec, g, &ui) == cudaSuccess) {
+        ex = pl->graphs[hit].exec;
+      } else {
+        cudaGetLastError();
+        cudaGraphExecDestroy(pl->graphs[hit].exec);
+      }
+      pl->graphs[hit].exec = nullptr;
     }
+    if (!ex) {
+      const cudaError_t ei = cudaGraphInstantiate(&ex, g, 0);
+      if (ei != cudaSuccess) {
+        cudaGraphDestroy(g);
+        if (fresh_slot) --pl->n_graphs;                                   // slot unused again
+        else memset(pl->graphs[hit].key, 0xFF, sizeof(pl->graphs[hit].key));  // never matches; exec null
+        return cuda_fail(ei, "graph instantiate");
+      }
+    }
+    cudaGraphDestroy(g);
     pl->graphs[hit].exec = ex;
     memcpy(pl->graphs[hit].key, key, sizeof(key));
+    pl->graphs[hit].timing_kind = pl->timing_kind;
+    pl->graphs[hit].piv_nsub = pl->piv_nsub;
+  } else {
+    pl->timing_kind = pl->graphs[hit].timing_kind;  // the replayed sequence's, not the last capture's
+    pl->piv_nsub = pl->graphs[hit].piv_nsub;
   }
   const bool shared_const = pl->p.mode == NCC_MODE_MATCH && !pl->tc && !pl->tiny_fn && pl->use_ct && !pl->jit_ctpl;
   if (shared_const) {

@@ -27,23 +27,32 @@ def pair_range(P: int, rank: int, world: int) -> tuple[int, int]:
     return (rank * P) // world, ((rank + 1) * P) // world
 
 
-def merge_peaks(peaks: torch.Tensor, V: int) -> torch.Tensor:
+def peak_keys(peaks: torch.Tensor, V: int, ssd: bool = False) -> torch.Tensor:
+    """int32 (..., 4) ncc_peak records -> int64 keys ordered like the kernels' packed 64-bit key
+    (csrc make_key): high 32 bits = order-preserving image of the fp32 score (of -score for SSD,
+    whose peak is the minimum), low 32 bits = 0xFFFFFFFF - (u*V + v), so the largest key is the
+    best score with ties going to the smallest global linear offset index.  Shifted by -2^63
+    so the unsigned key order is the signed int64 order."""
+    p = peaks.reshape(-1, 4) if peaks.dim() == 1 else peaks
+    score = p[..., 0].view(torch.float32)
+    if ssd:
+        score = -score
+    b = score.view(torch.int32).to(torch.int64) & 0xFFFFFFFF
+    o = torch.where(b >= 0x80000000, (~b) & 0xFFFFFFFF, b | 0x80000000)
+    lin = p[..., 1].to(torch.int64) * V + p[..., 2].to(torch.int64)
+    return (o - 0x80000000) * (1 << 32) + (0xFFFFFFFF - lin)
+
+
+def merge_peaks(peaks: torch.Tensor, V: int, ssd: bool = False) -> torch.Tensor:
     """peaks: int32 (world, batch, 4) ncc_peak records -> (batch, 4) merged records.
 
-    Per frame: max score; tie -> smallest u*V+v.  Records are selected, never recomputed.
+    One max over the packed keys per frame (the kernels' own tie rule: best score -- max for
+    NCC, min for SSD -- then the smallest u*V+v).  Records are selected, never recomputed; no
+    host synchronisation (works on the device for NCCL-gathered records).
     """
     p = peaks.reshape(peaks.shape[0], -1, 4)
-    score = p[..., 0].view(torch.float32).to(torch.float64)
-    lin = p[..., 1].to(torch.int64) * V + p[..., 2].to(torch.int64)
-    # lexicographic (score desc, lin asc): pick via sort on a combined float64 key per frame
-    best = []
-    for f in range(p.shape[1]):
-        s, l = score[:, f], lin[:, f]
-        m = s.max()
-        cand = torch.nonzero(s == m).flatten()
-        r = cand[torch.argmin(l[cand])]
-        best.append(p[r, f])
-    return torch.stack(best)
+    best = torch.argmax(peak_keys(p, V, ssd), dim=0)  # (batch,) rank holding each frame's peak
+    return p[best, torch.arange(p.shape[1], device=p.device)]
 
 
 def gather_results(local: torch.Tensor, group=None) -> torch.Tensor:
@@ -53,9 +62,11 @@ def gather_results(local: torch.Tensor, group=None) -> torch.Tensor:
         out = torch.empty((world,) + tuple(local.shape), dtype=local.dtype, device=local.device)
         dist.all_gather_into_tensor(out, local.contiguous(), group=group)
         return out
-    parts = [torch.empty_like(local) for _ in range(world)]
-    dist.all_gather(parts, local.contiguous(), group=group)
-    return torch.stack(parts)
+    # gloo (CPU tests, or several ranks sharing one GPU): host tensors
+    src = local.detach().cpu().contiguous()
+    parts = [torch.empty_like(src) for _ in range(world)]
+    dist.all_gather(parts, src, group=group)
+    return torch.stack(parts).to(local.device)
 
 
 def gather_vectors(local: torch.Tensor, counts: list[int], group=None) -> torch.Tensor:
@@ -68,7 +79,8 @@ def gather_vectors(local: torch.Tensor, counts: list[int], group=None) -> torch.
     return torch.cat([allv[r, : counts[r]] for r in range(world)], dim=0)
 
 
-def sharded_match(images: torch.Tensor, tmpl: torch.Tensor, device: int, group=None, write_surface=False):
+def sharded_match(images: torch.Tensor, tmpl: torch.Tensor, device: int, group=None, write_surface=False,
+                  score: int = 0):
     """Single large match split by offset-row bands over the process group.
 
     Every rank holds the full frame(s) (it reads only rows [u0, u1+h-1)); returns the merged
@@ -79,11 +91,11 @@ def sharded_match(images: torch.Tensor, tmpl: torch.Tensor, device: int, group=N
     B, H, W = images.shape
     h, w = tmpl.shape
     with MatchPlan(H, W, h, w, batch=B, device=device, shard_rank=rank, shard_count=world,
-                   write_surface=write_surface) as plan:
+                   write_surface=write_surface, score=score) as plan:
         peaks, scores = plan.match(images, tmpl)
         V = plan.info.V
     allp = gather_results(peaks, group)
-    return merge_peaks(allp, V), scores
+    return merge_peaks(allp, V, ssd=score == 1), scores
 
 
 def sharded_piv(frames_a: torch.Tensor, frames_b: torch.Tensor, win, search, step, total_pairs: int, device: int,

@@ -123,3 +123,32 @@ def test_experiments_tables_match_the_committed_sweep(tmp_path):
     assert md.read_text() == open(os.path.join(root, "EXPERIMENTS.md")).read()
     rows = [json.loads(l) for l in open(src) if l.strip().startswith("{")]
     assert rows and all(r["correct"] in (True, None) for r in rows)
+
+
+def test_python_binding_validates_buffers_before_the_c_abi():
+    """wrong dtype / device / shape / contiguity / size raise ValueError
+    in the binding instead of reaching the C ABI as raw pointers (checked on host tensors)."""
+    import torch
+    from paper_conf_ipps_moorelk13_b200.api import _check_tensor, _check_template
+    ok = torch.zeros((2, 8, 10), dtype=torch.float32)
+    _check_tensor(ok, "images", torch.float32, None, 2 * 8 * 10, last_dims=(8, 10))
+    bad = [
+        (ok.double(), dict(dtype=torch.float32)),                          # dtype
+        (ok[:, :, :5], dict(last_dims=(8, 10))),                            # trailing shape
+        (ok.transpose(1, 2), dict()),                                       # not contiguous
+        (ok[:1], dict()),                                                   # too small
+    ]
+    for t, kw in bad:
+        args = dict(dtype=torch.float32, device=None, min_numel=2 * 8 * 10, last_dims=None)
+        args.update(kw)
+        with pytest.raises(ValueError):
+            _check_tensor(t, "x", args["dtype"], args["device"], args["min_numel"], last_dims=args["last_dims"])
+    with pytest.raises(ValueError):  # a device tensor where host memory is required is caught too
+        _check_tensor(ok, "x", torch.float32, torch.device("cuda", 0), 1)
+    # templates: (h, >= w) with unit column stride; a padded row pitch is fine
+    big = torch.zeros((6, 12), dtype=torch.float32)
+    _check_template(big[:, :7], "tmpl", 6, 7, None)
+    with pytest.raises(ValueError):
+        _check_template(big[:, ::2], "tmpl", 6, 6, None)  # column stride 2
+    with pytest.raises(ValueError):
+        _check_template(big, "tmpl", 7, 7, None)  # too few rows

@@ -102,7 +102,9 @@ def test_cfg4_two_pairs_sampled():
             rs = oracle.piv_window_scores(As[pi], Bs[pi], 64, 64, 32, 32, 32, 32, ky, kx)
             assert np.max(np.abs(sc[pi, ky, kx] - rs)) <= TOL
             assert v["flags"][pi, ky, kx] == ref["flags"][i]
+            assert v["iy"][pi, ky, kx] == ref["iy"][i] and v["ix"][pi, ky, kx] == ref["ix"][i]
             assert abs(v["dy"][pi, ky, kx] - ref["dy"][i]) <= 2e-3
+            assert abs(v["dx"][pi, ky, kx] - ref["dx"][i]) <= 2e-3
 
 
 @pytest.mark.parametrize("h,w,my,mx,sy,sx", [(24, 20, 5, 7, 9, 11), (16, 16, 4, 4, 8, 8), (32, 32, 16, 16, 16, 16),

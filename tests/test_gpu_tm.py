@@ -15,6 +15,7 @@ import synth
 from paper_conf_ipps_moorelk13_b200 import build as B
 from paper_conf_ipps_moorelk13_b200 import shard
 from paper_conf_ipps_moorelk13_b200.api import MatchPlan, decode_peaks
+from _peaks import assert_peak_ok
 
 pytestmark = pytest.mark.gpu
 TOL = 1e-4
@@ -50,6 +51,52 @@ def test_cfg1_full_surface(generic):
     assert (peaks["u"][0], peaks["v"][0]) == (u0, v0) == (pk.u, pk.v)
     assert peaks["flags"][0] == 0
     assert abs(peaks["score"][0] - 1.0) <= TOL
+
+
+@pytest.mark.parametrize("smooth", [False, True])
+def test_cfg1_default_plan_full_surface(smooth):
+    """cfg1 (64^2 / 16^2) on the DEFAULT plan (the one-launch tm_tiny_kernel), uniform and the
+    smooth cancellation-stress variant of SURVEY 8(d): full surface vs the fp64 oracle, planted
+    peak exact."""
+    img, T, u0, v0 = synth.tm_inputs(1, smooth=smooth)
+    ref, pk = oracle.ncc_match(img, T)
+    dev = torch.device("cuda", 0)
+    with MatchPlan(64, 64, 16, 16, write_surface=True) as plan:
+        assert plan.info.variant_name.decode().startswith("tm_tiny"), plan.info.variant_name
+        peaks, s = plan.match(torch.from_numpy(img).to(dev), torch.from_numpy(T).to(dev))
+        torch.cuda.synchronize()
+    d = decode_peaks(peaks)
+    assert np.max(np.abs(s[0].cpu().numpy() - ref)) <= TOL
+    assert (int(d["u"][0]), int(d["v"][0])) == (u0, v0) == (pk.u, pk.v)
+
+
+@pytest.mark.parametrize("base,delta,flat", [(4.0, 2.0 ** -15, True), (4.0, 2.0 ** -13, False)])
+@pytest.mark.parametrize("cuda_cores", [True, False])
+def test_flat_threshold_straddle(base, delta, flat, cuda_cores):
+    """SURVEY 8(c) reading 4 on the GPU: checkerboard templates whose centred / raw energy ratio
+    straddles 1e-10 (pinned in test_oracle.py::test_flat_threshold_relative_to_raw_energy) get
+    the oracle's flat decision -- FLAT_TEMPLATE|INVALID and an all-zero surface for the flat one,
+    a valid peak and oracle-equal scores for the other (CUDA-core and tensor-core templates)."""
+    h = w = 4 if cuda_cores else 144
+    sgn = np.where((np.add.outer(np.arange(h), np.arange(w)) % 2) == 0, 1.0, -1.0)
+    T = (base + delta * sgn).astype(np.float32)
+    assert oracle.template_is_flat(T) == flat
+    img = synth.uniform_image(h + 60, w + 70, 41)
+    dev = torch.device("cuda", 0)
+    with MatchPlan(h + 60, w + 70, h, w, write_surface=True, cuda_cores=cuda_cores) as plan:
+        if not cuda_cores:
+            assert plan.info.variant_name.decode().startswith("tm_tc"), plan.info.variant_name
+        peaks, s = plan.match(torch.from_numpy(img).to(dev), torch.from_numpy(T).to(dev))
+        torch.cuda.synchronize()
+    d = decode_peaks(peaks)
+    s = s[0].cpu().numpy()
+    if flat:
+        assert int(d["flags"][0]) & 1 and int(d["flags"][0]) & 32
+        assert np.all(s == 0.0)
+    else:
+        assert int(d["flags"][0]) == 0
+        ref = oracle.ncc_surface(img, T)
+        assert np.max(np.abs(s - ref)) <= TOL
 
 
 @pytest.mark.parametrize("H,W,h,w,smooth", [(100, 137, 23, 17, False), (157, 123, 33, 41, True),
@@ -114,7 +161,10 @@ def test_batch_frames_and_host_path():
     for k in range(3):
         ref, pk = oracle.ncc_match(imgs[k], T)
         assert np.max(np.abs(s[k] - ref)) <= TOL
-        assert (peaks["u"][k], peaks["v"][k]) == (pk.u, pk.v)
+        if k == 1:  # planted: exact
+            assert (peaks["u"][k], peaks["v"][k]) == (pk.u, pk.v)
+        else:  # no planted match: SURVEY 8(c) reading 5 (near-tie rule)
+            assert_peak_ok(int(peaks["u"][k]), int(peaks["v"][k]), ref)
     # host-buffer entry point gives the same peaks
     stack = torch.from_numpy(np.stack(imgs)).pin_memory()
     tt = torch.from_numpy(T).pin_memory()

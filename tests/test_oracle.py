@@ -7,7 +7,9 @@ The oracle (oracle/ncc_oracle.c) is checked against things other than itself:
     symmetry, flat -> 0),
   * an independent algebra (oracle/ncc_fft.py: FFT numerator + fp64 SAT denominator),
   * PIV: planted integer shifts, the window-grid count by enumeration, sub-pixel closed
-    forms (Gaussian / parabola triples are recovered exactly).
+    forms (Gaussian / parabola triples are recovered exactly), the SSD minimum fit
+    (exact parabolas, mirrored triples, a fractional-shift particle pair), and the flat
+    threshold (templates straddling 1e-10 of the raw energy).
 Citations: PAPER.md Fig 5.1 caption P:132-137 (definition), Listing 5.1 caption
 P:250-251 (corr2 per shift), PIV Figs 5.9-5.12 captions P:165-171; SURVEY.md 8(c).
 """
@@ -291,8 +293,67 @@ def test_piv_ssd_planted_shift_and_parabola():
     p = synth.particle_pair_integer(160, 176, -2, 4, seed=45)
     v = oracle.piv_windows_ssd(p.A, p.B, 32, 32, 8, 8, 16, 16, [1, 2, 3], [1, 4, 2])
     assert np.all(v["iy"] == -2) and np.all(v["ix"] == 4) and np.all(v["score"] < 1e-9)
-    # parabola fit of an exact parabola minimum recovers delta
-    for d in (0.3, -0.2):
-        c = [1.0 + 2.0 * (k - d) ** 2 for k in (-1, 0, 1)]
-        den = 2 * (c[0] - 2 * c[1] + c[2])
-        assert abs((c[0] - c[2]) / den - d) < 1e-12
+
+
+# ---------------------------------------------------------------- SSD sub-pixel (Fig 5.10: argmin + parabola)
+@pytest.mark.parametrize("delta,a,b", [(0.3, 1.0, 2.0), (-0.2, 0.0, 0.5), (0.49, 7.5, 0.01), (-0.45, 3.0, 40.0)])
+def test_subpixel3_min_exact_parabola(delta, a, b):
+    """Closed form: c_k = a + b (k - delta)^2 (b > 0) is a parabola with its minimum at delta;
+    the oracle's 3-point minimum fit must return delta exactly (to rounding)."""
+    c = [a + b * (k - delta) ** 2 for k in (-1, 0, 1)]
+    assert abs(oracle.subpixel3_min(*c) - delta) < 1e-12
+
+
+def test_subpixel3_min_special_cases():
+    assert oracle.subpixel3_min(2.0, 1.0, 2.0) == 0.0     # symmetric -> 0
+    assert oracle.subpixel3_min(1.0, 2.0, 1.0) == 0.0     # a maximum, not a minimum -> no fit
+    assert oracle.subpixel3_min(1.0, 1.0, 1.0) == 0.0     # flat -> no fit
+    # sign: the lower neighbour pulls the vertex towards it
+    assert oracle.subpixel3_min(1.0, 0.5, 2.0) < 0.0 < oracle.subpixel3_min(2.0, 0.5, 1.0)
+    # the maximum fit (NCC) and the minimum fit (SSD) agree on mirrored triples: delta of
+    # (c-, c0, c+) as a minimum == delta of (-c-, -c0, -c+) as a maximum (parabolic branch)
+    for tri in [(3.0, 1.0, 2.0), (5.0, 0.2, 0.9)]:
+        d_min = oracle.subpixel3_min(*tri)
+        d_max, par = oracle.subpixel3(*[-x for x in tri])
+        assert par and abs(d_min - d_max) < 1e-15
+
+
+def test_piv_ssd_fractional_shift_sign_and_magnitude():
+    """SSD PIV on a particle pair re-rendered at a known fractional shift (2.3, -1.6): the
+    integer argmin is the nearest integer shift and the oracle's parabolic sub-pixel estimate
+    moves towards the planted value with the right sign on both axes (bias of the 3-point
+    parabola on 2.6-px particles is well under 0.25 px)."""
+    p = synth.particle_pair_subpixel(160, 160, 2.3, -1.6, seed=37)
+    v = oracle.piv_windows_ssd(p.A, p.B, 32, 32, 6, 6, 16, 16, [1, 2, 3, 4, 2], [1, 3, 2, 4, 4])
+    assert np.all(v["iy"] == 2) and np.all(v["ix"] == -2)
+    assert np.all(v["flags"] & (oracle.EDGE_Y | oracle.EDGE_X) == 0)
+    fy, fx = v["dy"] - v["iy"], v["dx"] - v["ix"]
+    assert np.all(fy > 0) and np.all(fx > 0)  # 2 -> 2.3 (up), -2 -> -1.6 (up)
+    assert np.median(np.abs(v["dy"] - 2.3)) < 0.25 and np.median(np.abs(v["dx"] + 1.6)) < 0.25
+
+
+# ---------------------------------------------------------------- flat threshold (S8c reading 4)
+def _checker(n: int, base: float, delta: float) -> np.ndarray:
+    s = np.where((np.add.outer(np.arange(n), np.arange(n)) % 2) == 0, 1.0, -1.0)
+    return (base + delta * s).astype(np.float32)
+
+
+def test_flat_threshold_relative_to_raw_energy():
+    """Flat <=> sum (T - Tbar)^2 <= 1e-10 * sum T^2.  A 4x4 checkerboard 4 +- d has centred
+    energy 16 d^2 and raw energy ~256, ratio d^2 / 16 (all values exact in fp32):
+      d = 2^-15: ratio 5.8e-11 -> flat;  d = 2^-13: ratio 9.3e-10 -> not flat.
+    The d = 2^-15 case is NOT flat under an absolute threshold (16 d^2 = 1.5e-8 > 1e-10) nor
+    under a threshold based on sum T (1e-10 * 64 = 6.4e-9 < 1.5e-8), so either mistake fails.
+    Tiny-valued templates (2^-20 scale, centred energy ~1e-13) are flat under an absolute
+    threshold but not under the relative one.  Scaling by a power of two never changes it."""
+    assert oracle.template_is_flat(_checker(4, 4.0, 2.0 ** -15))
+    assert not oracle.template_is_flat(_checker(4, 4.0, 2.0 ** -13))
+    for k in (-6, 0, 10):
+        assert oracle.template_is_flat(_checker(4, 4.0, 2.0 ** -15) * np.float32(2.0 ** k))
+        assert not oracle.template_is_flat(_checker(4, 4.0, 2.0 ** -13) * np.float32(2.0 ** k))
+    tiny = (synth.uniform_image(6, 5, 38) * np.float32(2.0 ** -20)).astype(np.float32)
+    assert not oracle.template_is_flat(tiny)
+    # and corr2 returns 0 for the flat one / a finite score for the other
+    img = synth.uniform_image(12, 12, 39)
+    assert np.all(oracle.ncc_surface(img, _checker(4, 4.0, 2.0 ** -15)) == 0.0)
+    assert np.all(oracle.ncc_surface(img, _checker(4, 4.0, 2.0 ** -13)) != 0.0)

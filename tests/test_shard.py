@@ -53,6 +53,33 @@ def test_merge_equals_global_argmax_with_ties(seed):
         assert (int(merged[0, 1]), int(merged[0, 2])) == (k // 23, k % 23) == (5, 7)
 
 
+def test_merge_ssd_takes_minimum_and_ties_smallest_index():
+    """SSD peaks (argmin): the band merge must keep the smallest SSD, ties -> smallest u*V+v."""
+    V = 10
+    recs = torch.tensor(np.array([[np.float32(3.5).view(np.int32), 0, 4, 0],
+                                  [np.float32(0.25).view(np.int32), 7, 1, 0],
+                                  [np.float32(0.25).view(np.int32), 5, 9, 0],
+                                  [np.float32(9.0).view(np.int32), 9, 0, 0]], dtype=np.int32))
+    m = shard.merge_peaks(recs[:, None, :], V, ssd=True)
+    assert (int(m[0, 1]), int(m[0, 2])) == (5, 9)
+    m = shard.merge_peaks(recs[:, None, :], V, ssd=False)
+    assert (int(m[0, 1]), int(m[0, 2])) == (9, 0)
+
+
+def test_peak_keys_order_matches_score_then_index():
+    """Packed keys sort like (score desc, index asc) over negative, zero and positive scores."""
+    g = np.random.default_rng(3)
+    sc = np.concatenate([g.standard_normal(200).astype(np.float32), [0.0, 0.0, 1.0, 1.0, -1.0]]).astype(np.float32)
+    us = g.integers(0, 50, sc.size)
+    vs = g.integers(0, 30, sc.size)
+    recs = torch.tensor(np.stack([sc.view(np.int32), us, vs, np.zeros_like(us)], 1).astype(np.int32))
+    k = shard.peak_keys(recs, 30).numpy()
+    order = np.argsort(-k, kind="stable")
+    ref = sorted(range(sc.size), key=lambda i: (-float(sc[i]), us[i] * 30 + vs[i]))
+    # equal (score, index) pairs are interchangeable; compare the sorted tuples
+    assert [(float(sc[i]), us[i] * 30 + vs[i]) for i in order] == [(float(sc[i]), us[i] * 30 + vs[i]) for i in ref]
+
+
 def _free_port():
     s = socket.socket()
     s.bind(("127.0.0.1", 0))

@@ -100,8 +100,7 @@ def piv_case(table, win, m, step, dy=5, dx=-3):
             num, tot = timed(plan, run)
             d = decode_vectors(vec)
             ok = bool(((d["iy"] == dy) & (d["ix"] == dx)).float().mean() > 0.99) if max(abs(dy), abs(dx)) < m else None
-            emit(table=table, win=win, m=m, step=step, tier=["AOT", "JIT"][plan.info.specialized - 1]
-                 if plan.info.specialized else "RE", variant=plan.info.variant_name.decode(),
+            emit(table=table, win=win, m=m, step=step, tier=["RE", "AOT", "JIT", "TC"][plan.info.specialized], variant=plan.info.variant_name.decode(),
                  regs=plan.info.regs_per_thread, vectors=plan.info.outputs_per_call, numerator_ms=num, step_ms=tot,
                  vectors_per_s=plan.info.outputs_per_call / (tot / 1e3),
                  tflops=plan.info.flops_per_call / num / 1e9, correct=ok)
