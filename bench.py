@@ -489,6 +489,8 @@ def main():
     import torch.distributed as dist
     from paper_conf_ipps_moorelk13_b200 import build as B
 
+    if args.backend == "gloo":  # dry run: ranks may share the GPUs there are
+        local = local % max(1, torch.cuda.device_count())
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if ws > 1:
