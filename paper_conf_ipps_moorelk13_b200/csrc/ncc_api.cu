@@ -319,17 +319,20 @@ struct ncc_plan_s {
   // tensor-core numerator (tm_tc_kernel): 0 = CUDA-core path
   int tc, tc_wc, tc_nbi, tc_nbj, tc_vtiles, tc_useg, tc_nseg;
   int tc_vcols;  // last output columns computed by tm_tc_cols (0: none)
-  int tc_sched;  // 0: window sums || template prep; 1/2: window sums on the side stream, overlapping the
-                 // numerator; 3 (default): image split, then window sums || template prep + ragged columns
-  float *tcB, *tc_part;
-  unsigned int* tc_done;  // per-frame count of finished tm_tc_finish CTAs (self-resetting)
+  int tc_sched;  // 0: window sums || template prep, image split after them; 3 (default): image split,
+                 // then window sums || template prep + ragged columns
+  float *tcB, *tc_acc;     // reversed template-block operands; running numerator (one plane)
+  unsigned int* tc_done;   // finished tm_tc_tail CTAs (self-resetting)
+  unsigned int* tc_flags;  // chain flags [batch][vtiles * nseg][ngrp_max][4] (self-resetting)
+  unsigned long long* tc_ticket;  // CTA start tickets (monotonic)
+  int tc_ngrp;
   // tiny problems: the whole TM path in one launch (tm_tiny_kernel)
   const void* tiny_fn;
   int tiny_ctas, tiny_rows, tiny_smem;
   unsigned int* tiny_done;
   // side stream for work independent of the main chain (template prep || window sums)
   cudaStream_t side;
-  cudaEvent_t ev_fork, ev_join, ev_cols;
+  cudaEvent_t ev_fork, ev_join, ev_cols, ev_img;
   // timing (NCC_F_TIMING)
   std::vector<cudaEvent_t> ev;
   int n_ev_used;
@@ -382,8 +385,10 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->keys);
   cudaFree(pl->RS1);
   cudaFree(pl->tcB);
-  cudaFree(pl->tc_part);
+  cudaFree(pl->tc_acc);
   cudaFree(pl->tc_done);
+  cudaFree(pl->tc_flags);
+  cudaFree(pl->tc_ticket);
   cudaFree(pl->tiny_done);
   cudaFree(pl->tc_img2);
   cudaFree(pl->RS2);
@@ -398,6 +403,7 @@ void free_plan(ncc_plan pl) {
   if (pl->ev_fork) cudaEventDestroy(pl->ev_fork);
   if (pl->ev_join) cudaEventDestroy(pl->ev_join);
   if (pl->ev_cols) cudaEventDestroy(pl->ev_cols);
+  if (pl->ev_img) cudaEventDestroy(pl->ev_img);
   if (pl->side) cudaStreamDestroy(pl->side);
   for (int k = 0; k < 2; ++k) {
     if (pl->ev_copied[k]) cudaEventDestroy(pl->ev_copied[k]);
@@ -510,6 +516,7 @@ ncc_status setup_tc(ncc_plan pl) {
   // launch order (measured on B200, cfg2 step: 0 -> 0.2135 ms, 3 -> 0.2074 ms; 1/2 delay the
   // tensor-core kernel's start or starve the ragged-column kernel); NCC_TM_SCHED overrides
   pl->tc_sched = getenv("NCC_TM_SCHED") ? atoi(getenv("NCC_TM_SCHED")) : 3;
+  if (pl->tc_sched != 0) pl->tc_sched = 3;  // (the earlier 1/2: window sums after the numerator's start)
   if (pl->V > 128 && pl->V % 128 != 0 && pl->V % 128 <= kTcColsMax && w <= 512 && !getenv("NCC_TC_NO_COLS")) {
     pl->tc_vtiles = pl->V / 128;
     pl->tc_vcols = pl->V % 128;
@@ -555,11 +562,19 @@ ncc_status setup_tc(ncc_plan pl) {
   const int nblk = pl->tc_nbi * pl->tc_nbj;
   ncc_status st;
   if ((st = dalloc(&pl->tcB, (size_t)nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
-  if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
+  // one running-numerator plane whatever the number of template blocks (they accumulate in a
+  // chain inside tm_tc_kernel), chain flags, the CTA ticket counter
+  if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) return st;
+  pl->tc_ngrp = ceil_div(pl->tc_useg + tc::kHB - 1, tc::kG);
+  const size_t nflags = (size_t)p.batch * pl->tc_vtiles * pl->tc_nseg * pl->tc_ngrp * 4;
+  if ((st = dalloc(&pl->tc_flags, nflags))) return st;
+  NCC_CUDA(cudaMemset(pl->tc_flags, 0, nflags * sizeof(unsigned int)));
+  if ((st = dalloc(&pl->tc_ticket, (size_t)1))) return st;
+  NCC_CUDA(cudaMemset(pl->tc_ticket, 0, sizeof(unsigned long long)));
   // (hi, lo) pairs, rows padded to an even count of pairs: a 16-byte multiple for the TMA map
   if ((st = dalloc(&pl->tc_img2, (size_t)2 * p.batch * pl->Hs * ((p.image_w + 1) & ~1)))) return st;
-  if ((st = dalloc(&pl->tc_done, (size_t)p.batch))) return st;
-  NCC_CUDA(cudaMemset(pl->tc_done, 0, (size_t)p.batch * sizeof(unsigned int)));
+  if ((st = dalloc(&pl->tc_done, (size_t)1))) return st;
+  NCC_CUDA(cudaMemset(pl->tc_done, 0, sizeof(unsigned int)));
   const int smem = tc::smem_bytes(pl->tc_wc);
   NCC_CUDA(cudaFuncSetAttribute((const void*)tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   NCC_CUDA(cudaFuncSetAttribute((const void*)tm_tc_prep, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -573,7 +588,8 @@ ncc_status setup_tc(ncc_plan pl) {
   in.split = nblk;
   in.const_template = 0;
   in.slabs = 1;
-  // template prep (+ operand), window sums, image split, numerator, finish (+ peak), ragged columns
+  // template prep (+ operand), window sums, image split, numerator (+ chained block sum,
+  // normalisation, argmax keys), tail (ragged columns' normalisation + peak), ragged columns
   in.launches_per_call = (h * w <= kPrepSmemFloats ? 1 : 2) + (pl->box_smem ? 1 : 2) + 3 + (pl->tc_vcols ? 1 : 0);
   return NCC_OK;
 }
@@ -753,6 +769,7 @@ ncc_status create_tm(ncc_plan pl) {
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_fork, cudaEventDisableTiming));
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_join, cudaEventDisableTiming));
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_cols, cudaEventDisableTiming));
+  NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_img, cudaEventDisableTiming));
   ncc_status st;
   if ((st = dalloc(&pl->tplC, (size_t)pl->n_tmpl * pl->HP * pl->WP))) return st;
   if ((st = dalloc(&pl->tst, (size_t)pl->n_tmpl))) return st;
@@ -1032,6 +1049,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   const int nblk_tc = pl->tc_nbi * pl->tc_nbj;
   auto launch_cols = [&]() {  // the ragged last columns (tensor-core path), on the side stream
+    if (pl->h_img_in) cudaStreamWaitEvent(pl->side, pl->ev_img, 0);  // host path: frames copied (errors: cudaGetLastError below)
     // small templates: one output per warp (short CTAs that finish before the tensor-core grid
     // needs their SMs, cfg 2); large ones: 4 sliding rows per warp (a quarter of the loads;
     // cfg 5: 740 -> 329 us, no longer delaying the numerator's start)
@@ -1042,7 +1060,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     auto cols = [&](auto kern) {
       kern<<<(unsigned)ceil_div(items, 8), 256, 0, pl->side>>>(
           d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w,
-          pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, p.batch, pl->tc_part, pfs * p.batch, pfs, nblk_tc);
+          pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, p.batch, pl->tc_acc, pfs);
     };
     if (jc <= 4) cols(tm_tc_cols<4>);
     else if (jc <= 8) cols(tm_tc_cols<8>);
@@ -1053,20 +1071,22 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
         reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 1) & ~1), (p.image_w + 1) & ~1);
   };
-  // fork: template prep on the side stream.  Host path: the frames' copy is issued on the main
-  // stream BEFORE the fork event, so everything on the side stream that reads the frames (the
-  // ragged-column kernel, the late window sums) is ordered after it; the template's copy runs on
-  // the side stream ahead of its prep, concurrently with the frames' copy.
+  // fork: template prep on the side stream.  Host path: the template's copy runs on the side
+  // stream ahead of its prep, concurrently with the frames' copy on the main stream; the side
+  // stream's only reader of the frames (the ragged-column kernel) waits for the frames' copy
+  // (ev_img) -- the main stream's kernels are ordered after it anyway.
   mark(pl, s, 0);
-  if (pl->h_img_in)
-    NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
-                             (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
   NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
   NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
   if (pl->h_tmpl_in)
     NCC_CUDA(cudaMemcpy2DAsync(const_cast<float*>(d_tmpl), tmpl_pitch * sizeof(float), pl->h_tmpl_in,
                                pl->h_tmpl_pitch * sizeof(float), p.tmpl_w * sizeof(float), p.tmpl_h,
                                cudaMemcpyHostToDevice, pl->side));
+  if (pl->h_img_in) {
+    NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
+                             (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
+    NCC_CUDA(cudaEventRecord(pl->ev_img, s));
+  }
   if (pl->tc && p.tmpl_h * p.tmpl_w <= kPrepSmemFloats && !getenv_flag_two_kernel_prep()) {
     // one launch: template stats + centred template + MMA operand, template staged in shared memory
     tm_tc_prep<<<nblk_tc, 1024, p.tmpl_h * p.tmpl_w * 4, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
@@ -1081,7 +1101,6 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
                                                     pl->tcB);
   }
   NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
-  const bool late_box = tc_now && (pl->tc_sched == 1 || pl->tc_sched == 2);
   if (tc_now && pl->tc_sched == 3) {
     // the image split first (small: it leaves room for the template prep, which starts at once
     // on the side stream), then the window sums on the main stream; the ragged columns follow
@@ -1094,19 +1113,9 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
-  } else if (late_box) {
-    // window sums are needed only by tm_tc_finish: they run on the side stream after the
-    // template prep, concurrently with the image split and the tensor-core kernel (which
-    // leaves SMs free); the split runs on the main stream concurrently with the template prep
-    if (pl->tc_sched == 1) launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, pl->side);
-    if (pl->tc_vcols) launch_cols();
-    if (pl->tc_sched == 2) launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, pl->side);
-    NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
-    launch_split();
-    NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
-    mark(pl, s, 2);
   } else {
-    // window sums on the main stream while the template prep runs on the side stream
+    // window sums on the main stream while the template prep runs on the side stream (the
+    // tensor-core kernel normalises in its drains, so the window sums always precede it)
     if (tc_now && pl->tc_vcols) {  // after the join: overlaps the tensor-core kernel rather than delay its start
       launch_cols();
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
@@ -1117,7 +1126,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
     const int nblk = nblk_tc;
-    if (!late_box && pl->tc_sched != 3) launch_split();
+    if (pl->tc_sched != 3) launch_split();
     TcArgs t;
     t.H = p.image_h;
     t.W = p.image_w;
@@ -1131,16 +1140,29 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.useg = pl->tc_useg;
     t.nseg = pl->tc_nseg;
     t.vtiles = pl->tc_vtiles;
-    t.part = pl->tc_part;
-    t.part_frame_stride = (int64_t)pl->Ub * pl->V;
-    t.part_blk_stride = t.part_frame_stride * p.batch;
+    t.acc = pl->tc_acc;
+    t.acc_frame_stride = (int64_t)pl->Ub * pl->V;
+    t.flags = pl->tc_flags;
+    t.ngrp_max = pl->tc_ngrp;
+    t.ticket = pl->tc_ticket;
+    t.S1 = pl->S1;
+    t.S2 = pl->S2;
+    t.stat_frame_stride = pl->s_frame_stride;
+    t.tst = pl->tst;
+    t.h = p.tmpl_h;
+    t.w = p.tmpl_w;
+    t.scores = (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr;
+    t.score_frame_stride = (int64_t)pl->Ub * pl->V;
+    t.keys = pl->keys;
+    t.ssd = p.score == NCC_SCORE_SSD;
     tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, p.batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
     mark(pl, s, 3);
-    if (pl->tc_vcols || late_box) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
-    tm_tc_finish<<<dim3(pl->Ub, p.batch), 256, 0, s>>>(
-        pl->tc_part, nblk, t.part_blk_stride, t.part_frame_stride, pl->S1, pl->S2, pl->s_frame_stride, pl->tst,
-        p.tmpl_h, p.tmpl_w, pl->V, pl->u_begin, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
+    if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
+    const int64_t tail_items = (int64_t)p.batch * pl->Ub * pl->tc_vcols;
+    tm_tc_tail<<<(unsigned)std::max<int64_t>(1, ceil_div(tail_items, 256)), 256, 0, s>>>(
+        pl->tc_acc, (int64_t)pl->Ub * pl->V, pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V,
+        pl->V - pl->tc_vcols, pl->u_begin, pl->Ub, p.batch, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
         (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks));
     mark(pl, s, 4);
     cudaError_t e = cudaGetLastError();

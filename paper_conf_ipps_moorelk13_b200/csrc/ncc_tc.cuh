@@ -159,9 +159,33 @@ struct TcArgs {
   int u_begin, u_end;   // output rows of the band
   int useg, nseg;       // output rows per CTA segment, segments
   int vtiles;
-  float* part;          // [nblk][batch][u_end - u_begin][V] partial numerators
-  int64_t part_blk_stride, part_frame_stride;
+  // Template blocks of one output tile accumulate in a fixed chain, block 0 -> nblk - 1 (no
+  // partial planes, no summation kernel -- the paper's K2 global round trip, Figs 5.4-5.6, is
+  // gone): block b > 0 adds its drained rows to the running numerator block b - 1 left in `acc`
+  // (per-row-group, per-warp flags), the last block normalises them in the same drain.
+  float* acc;              // [batch][u_end - u_begin][V] running numerator (one plane)
+  int64_t acc_frame_stride;
+  unsigned int* flags;     // [batch][vtiles * nseg][ngrp_max][4]: blocks done with a row group
+  int ngrp_max;
+  unsigned long long* ticket;  // monotonically increasing CTA ticket (start order -> chain order)
+  const double *S1, *S2;   // fp64 window sums [batch][u_end - u_begin][V] (box2d)
+  int64_t stat_frame_stride;
+  const TemplateStats* tst;
+  int h, w;
+  float* scores;           // optional surface [batch][u_end - u_begin][V]
+  int64_t score_frame_stride;
+  unsigned long long* keys;  // per-frame packed argmax keys
+  int ssd;
 };
+
+__device__ __forceinline__ unsigned int ld_acquire_u32(const unsigned int* p) {
+  unsigned int v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release_u32(unsigned int* p, unsigned int v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
 
 // grid = (nblk * vtiles * nseg, batch); block = tc::kThreads; dynamic smem = tc::b_bytes(WC).
 __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
@@ -171,14 +195,23 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   __shared__ __align__(8) uint64_t a_full[kNBuf], mma_done[kNBuf], img_full[kNImg], img_empty[kNImg], reloc_req,
       reloc_done;
   __shared__ uint32_t tmem_base_s;
+  __shared__ unsigned long long ticket_s;
 
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int nblk = a.nbi * a.nbj;
-  const int blk = blockIdx.x % nblk;
-  const int rest = blockIdx.x / nblk;
-  const int vt = rest % a.vtiles, seg = rest / a.vtiles;
+  // The CTA's work comes from a ticket taken when it starts, template block fastest: the CTA of
+  // block b of a tile always started after the one of block b - 1 (which it may wait for), so
+  // the chain never waits on a CTA that is not resident or finished, whatever the hardware's
+  // dispatch order.  The counter only grows: a launch of this plan always has the same grid.
+  if (tid == 0) ticket_s = atomicAdd(a.ticket, 1ull) % ((unsigned long long)gridDim.x * gridDim.y);
+  __syncthreads();
+  const int64_t tk = (int64_t)ticket_s;
+  const int blk = (int)(tk % nblk);
+  const int64_t rest = tk / nblk;
+  const int tile = (int)(rest % ((int64_t)a.vtiles * a.nseg));  // = seg * vtiles + vt
+  const int vt = tile % a.vtiles, seg = tile / a.vtiles;
   const int bi = blk / a.nbj, bj = blk % a.nbj;
-  const int f = blockIdx.y;
+  const int f = (int)(rest / ((int64_t)a.vtiles * a.nseg));
   const int v0 = vt * 128;
   const int ua = a.u_begin + seg * a.useg;
   const int nu = min(a.useg, a.u_end - ua);  // output rows of this CTA
@@ -266,7 +299,73 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       fence_before();
     }
     const uint2* ring = reinterpret_cast<const uint2*>(smem_tc + img_off(a.WC));
-    float* part = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * a.part_frame_stride;
+    const int vv = v0 + v;
+    // (pointers are formed inside the drain from the kernel parameters: the producers run at
+    // the 96-register cap -- 5 warps of this SMSP-bound CTA share one SMSP's register file)
+    // Drain of row group gd (its MMAs are complete): output rows up = kG gd - kHB + 1 + k.
+    // Chain: block b > 0 waits until block b - 1 published the group's running numerator (this
+    // warp's 32 columns), adds its own; blocks b < nblk - 1 publish; the last block normalises
+    // (fp64 variance, fp32 rsqrt, as the CUDA-core path), writes the surface and folds the keys.
+    // Per output the order is ((p_0 + p_1) + p_2) + ... in block order: deterministic and
+    // independent of bands and segments.
+    auto drain = [&](int gd, const uint32_t (&d)[8]) {
+      const int up0 = gd * kG - kHB + 1;
+      if (up0 + kG <= 0 || up0 >= nu) return;  // ramp groups hold no output row of this CTA
+      const bool colok = vv < a.V;
+      const bool last_blk = blk == nblk - 1;
+      const int64_t rowbase = (int64_t)(ua - a.u_begin) * a.V + vv;  // CTA's first output row, this column
+      float* accf = a.acc + (int64_t)f * a.acc_frame_stride + rowbase;
+      float x[kG];
+#pragma unroll
+      for (int k = 0; k < kG; ++k) x[k] = __uint_as_float(d[k]);
+      unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + wq;
+      if (blk > 0) {
+        if (lane == 0) {
+          for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
+            if (it > (1ll << 28)) __trap();
+        }
+        __syncwarp();
+#pragma unroll
+        for (int k = 0; k < kG; ++k) {
+          const int up = up0 + k;
+          if (up >= 0 && up < nu && colok) x[k] = __ldcg(accf + (int64_t)up * a.V) + x[k];
+        }
+      }
+      if (!last_blk) {
+#pragma unroll
+        for (int k = 0; k < kG; ++k) {
+          const int up = up0 + k;
+          if (up >= 0 && up < nu && colok) __stcg(accf + (int64_t)up * a.V, x[k]);
+        }
+        __threadfence();
+        __syncwarp();
+        if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
+        return;
+      }
+      const TemplateStats ts = a.tst[0];
+      const double inv_n = 1.0 / ((double)a.h * (double)a.w);
+      const double* s1p = a.S1 + (int64_t)f * a.stat_frame_stride + rowbase;
+      const double* s2p = a.S2 + (int64_t)f * a.stat_frame_stride + rowbase;
+      float* scp = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + rowbase : nullptr;
+      unsigned long long best = 0ull;
+#pragma unroll
+      for (int k = 0; k < kG; ++k) {
+        const int up = up0 + k;
+        if (up >= 0 && up < nu && colok) {
+          const double s1 = __ldcg(s1p + (int64_t)up * a.V), s2 = __ldcg(s2p + (int64_t)up * a.V);
+          const float sc = a.ssd ? (float)(ts.sumsq - 2.0 * ((double)x[k] + ts.sum * inv_n * s1) + s2)
+                                 : ncc_normalize_fast(x[k], s1, s2, inv_n, ts.csum, ts.energy, ts.flat != 0);
+          if (scp) scp[(int64_t)up * a.V] = sc;
+          const unsigned long long key = make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)(ua + up) * a.V + vv));
+          best = key > best ? key : best;
+        }
+      }
+      best = warp_max_key(best);
+      if (lane == 0) {
+        if (best && best > __ldcg(a.keys + f)) atomicMax(a.keys + f, best);
+        if (blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
+      }
+    };
     // Software-pipelined producer: the operand of the group's next stage is read from the ring
     // and split while the group waits for its TMEM buffer, so the critical path from "MMAs of
     // the buffer's previous stage done" to "a_full" is only the TMEM stores (the MMA warp has
@@ -331,15 +430,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
         uint32_t d[8];
         ld8(tbase + lane_base + col, d);
-        const int vv = v0 + v;
-#pragma unroll
-        for (int k = 0; k < kG; ++k) {
-          const int up = gd * kG - kHB + 1 + k;  // output row (CTA-relative)
-          if (up >= 0 && up < nu && vv < a.V)
-            part[(int64_t)(ua - a.u_begin + up) * a.V + vv] = __uint_as_float(d[k]);
-        }
         const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
-        st8(tbase + lane_base + col, z);
+        st8(tbase + lane_base + col, z);  // the columns are free again once read
+        drain(gd, d);
       }
       if (q + kGroups < nstage) load_split(q + kGroups);
     }
@@ -525,15 +618,15 @@ __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img
 // Numerator of the last V - v_lo (< 128) output columns, which would otherwise cost a whole
 // column of tensor-core CTAs (V = W - w + 1 is 1 mod 128 for power-of-two frames and
 // templates): one warp per (frame, output row, column); lanes split the template columns, a
-// fresh fp32 partial per template row, then a warp sum.  Written to block plane 0 (the other
-// planes get zeros), so tm_tc_finish's block sum is the full numerator.  Loads of RB template
+// fresh fp32 partial per template row, then a warp sum: the full numerator, written to the
+// running-numerator plane (normalised by tm_tc_tail).  Loads of RB template
 // rows are issued before their products (the kernel is load-latency bound).  grid =
 // ceil(items / 8), block = 256.
 template <int JC>  // JC = ceil(w / 32) template columns per lane
 __global__ void __launch_bounds__(256) tm_tc_cols(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
                                                   const float* __restrict__ tplC, int tplP, int h, int w, int v_lo,
-                                                  int V, int u_begin, int Ub, int batch, float* __restrict__ part,
-                                                  int64_t blk_stride, int64_t part_frame_stride, int nblk) {
+                                                  int V, int u_begin, int Ub, int batch, float* __restrict__ acc,
+                                                  int64_t acc_frame_stride) {
   const int nc = V - v_lo;
   const int64_t item = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (item >= (int64_t)batch * Ub * nc) return;
@@ -565,8 +658,7 @@ __global__ void __launch_bounds__(256) tm_tc_cols(const float* __restrict__ img,
   }
 #pragma unroll
   for (int d = 16; d; d >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, d);
-  for (int b = lane; b < nblk; b += 32)
-    part[(int64_t)b * blk_stride + (int64_t)f * part_frame_stride + (int64_t)ur * V + v_lo + c] = b == 0 ? tot : 0.0f;
+  if (lane == 0) acc[(int64_t)f * acc_frame_stride + (int64_t)ur * V + v_lo + c] = tot;
 }
 
 // As tm_tc_cols, RWN consecutive output rows per warp: template row i is loaded once for the
@@ -579,8 +671,7 @@ template <int JC, int RWN>
 __global__ void __launch_bounds__(256) tm_tc_cols_rw(const float* __restrict__ img, int64_t pitch,
                                                      int64_t frame_stride, const float* __restrict__ tplC, int tplP,
                                                      int h, int w, int v_lo, int V, int u_begin, int Ub, int batch,
-                                                     float* __restrict__ part, int64_t blk_stride,
-                                                     int64_t part_frame_stride, int nblk) {
+                                                     float* __restrict__ acc, int64_t acc_frame_stride) {
   const int nc = V - v_lo, nrb = (Ub + RWN - 1) / RWN;
   const int64_t item = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (item >= (int64_t)batch * nrb * nc) return;
@@ -629,12 +720,10 @@ __global__ void __launch_bounds__(256) tm_tc_cols_rw(const float* __restrict__ i
 #pragma unroll
     for (int d = 16; d; d >>= 1) tot[r] += __shfl_xor_sync(0xffffffffu, tot[r], d);
   }
-  for (int b = lane; b < nblk; b += 32)
+  if (lane == 0)
 #pragma unroll
     for (int r = 0; r < RWN; ++r)
-      if (ur0 + r < Ub)
-        part[(int64_t)b * blk_stride + (int64_t)f * part_frame_stride + (int64_t)(ur0 + r) * V + v_lo + c] =
-            b == 0 ? tot[r] : 0.0f;
+      if (ur0 + r < Ub) acc[(int64_t)f * acc_frame_stride + (int64_t)(ur0 + r) * V + v_lo + c] = tot[r];
 }
 
 // Template operand: for block (bi, bj) the reversed, zero-padded rows Rv[k] = A_C[i0 + K0 - k]
@@ -758,100 +847,66 @@ __global__ void __launch_bounds__(1024) tm_tc_prep(const float* __restrict__ tmp
   for (int f = threadIdx.x; f < batch; f += blockDim.x) keys[f] = 0ull;
 }
 
-// Sum the partial numerators of the template blocks in block order, normalise (or SSD),
-// optional surface store, per-frame argmax key; the frame's last CTA writes its peak.  grid = (Ub, batch), block = 256; each thread
-// takes kFinV columns with all their loads issued first (the kernel is load-latency bound).
-constexpr int kFinV = 4;
-__global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ part, int nblk, int64_t blk_stride,
-                                                    int64_t frame_stride, const double* __restrict__ S1,
-                                                    const double* __restrict__ S2, int64_t stat_frame_stride,
-                                                    const TemplateStats* tst, int h, int w, int V, int u_begin,
-                                                    float* scores, int64_t score_frame_stride,
-                                                    unsigned long long* keys, int ssd,
-                                                    unsigned int* __restrict__ done, PeakOut* __restrict__ peaks) {
-  __shared__ unsigned long long red[32];
+// Ragged last columns [v_lo, V) (computed by tm_tc_cols into the running-numerator plane):
+// normalise (or SSD), optional surface store, fold into the per-frame argmax keys; the last CTA
+// to finish turns every frame's key into its peak (tm_finalize fused) -- the tensor-core kernel
+// folded its own columns' keys before this launch (stream order).  grid = max(1, ceil(items /
+// 256)), items = batch x Ub x (V - v_lo); block = 256.
+__global__ void __launch_bounds__(256) tm_tc_tail(const float* __restrict__ acc, int64_t acc_frame_stride,
+                                                  const double* __restrict__ S1, const double* __restrict__ S2,
+                                                  int64_t stat_frame_stride, const TemplateStats* tst, int h, int w,
+                                                  int V, int v_lo, int u_begin, int Ub, int batch, float* scores,
+                                                  int64_t score_frame_stride, unsigned long long* keys, int ssd,
+                                                  unsigned int* __restrict__ done, PeakOut* __restrict__ peaks) {
   __shared__ bool last;
-  const int ur = blockIdx.x, f = blockIdx.y;
-  const int u = u_begin + ur;
   const TemplateStats ts = tst[0];
+  const int nc = V - v_lo;
+  const int64_t items = (int64_t)batch * Ub * nc;
+  const int64_t it = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const double inv_n = 1.0 / ((double)h * (double)w);
-  const float* p = part + (int64_t)f * frame_stride + (int64_t)ur * V;
-  const int64_t so = (int64_t)f * stat_frame_stride + (int64_t)ur * V;
-  float* srow = scores ? scores + (int64_t)f * score_frame_stride + (int64_t)ur * V : nullptr;
-  unsigned long long best = 0ull;
-  for (int v0 = threadIdx.x; v0 < V; v0 += blockDim.x * kFinV) {
-    float tot[kFinV];
-    double s1v[kFinV], s2v[kFinV];
-#pragma unroll
-    for (int k = 0; k < kFinV; ++k) {
-      const int v = v0 + k * blockDim.x;
-      tot[k] = 0.0f;
-      s1v[k] = s2v[k] = 0.0;
-      if (v < V) {
-        s1v[k] = __ldg(S1 + so + v);
-        s2v[k] = __ldg(S2 + so + v);
-      }
-    }
-    int b = 0;
-    for (; b + 4 <= nblk; b += 4) {  // 16 loads in flight, summed in block order
-      float x[4][kFinV];
-#pragma unroll
-      for (int bb = 0; bb < 4; ++bb)
-#pragma unroll
-        for (int k = 0; k < kFinV; ++k) {
-          const int v = v0 + k * blockDim.x;
-          x[bb][k] = v < V ? __ldg(p + (int64_t)(b + bb) * blk_stride + v) : 0.0f;
-        }
-#pragma unroll
-      for (int bb = 0; bb < 4; ++bb)
-#pragma unroll
-        for (int k = 0; k < kFinV; ++k) tot[k] += x[bb][k];
-    }
-    for (; b < nblk; ++b) {
-#pragma unroll
-      for (int k = 0; k < kFinV; ++k) {
-        const int v = v0 + k * blockDim.x;
-        if (v < V) tot[k] += __ldg(p + (int64_t)b * blk_stride + v);
-      }
-    }
-#pragma unroll
-    for (int k = 0; k < kFinV; ++k) {
-    const int v = v0 + k * blockDim.x;
-    if (v >= V) break;
-    const double s1 = s1v[k], s2 = s2v[k];
-    float sc;
-    if (ssd)
-      sc = (float)(ts.sumsq - 2.0 * ((double)tot[k] + ts.sum * inv_n * s1) + s2);
-    else  // fp64 variance, fp32 rsqrt: |error| <= ~4e-7 (the fp64 divide/sqrt dominated this kernel)
-      sc = ncc_normalize_fast(tot[k], s1, s2, inv_n, ts.csum, ts.energy, ts.flat != 0);
-    if (srow) srow[v] = sc;
-    const unsigned long long key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
-    best = key > best ? key : best;
-    }
+  int f = -1;
+  unsigned long long key = 0ull;
+  if (it < items) {
+    const int c = (int)(it % nc);
+    const int64_t t = it / nc;
+    const int ur = (int)(t % Ub);
+    f = (int)(t / Ub);
+    const int v = v_lo + c;
+    const int64_t o = (int64_t)ur * V + v;
+    const float num = acc[(int64_t)f * acc_frame_stride + o];
+    const double s1 = S1[(int64_t)f * stat_frame_stride + o], s2 = S2[(int64_t)f * stat_frame_stride + o];
+    const float sc = ssd ? (float)(ts.sumsq - 2.0 * ((double)num + ts.sum * inv_n * s1) + s2)
+                         : ncc_normalize_fast(num, s1, s2, inv_n, ts.csum, ts.energy, ts.flat != 0);
+    if (scores) scores[(int64_t)f * score_frame_stride + o] = sc;
+    key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)(u_begin + ur) * V + v));
   }
-  best = block_max_key(best, red);
-  if (threadIdx.x == 0) {
-    // keys only grow: a CTA whose best is not above the (possibly stale) current key skips
-    // its atomic -- most do, which halves the same-address atomics of the grid
-    if (best && best > __ldcg(keys + f)) atomicMax(keys + f, best);
-    // the frame's last CTA turns the key into its peak (tm_finalize fused): every CTA's
-    // atomicMax is ordered before its counter increment
-    __threadfence();
-    last = atomicAdd(done + f, 1u) == gridDim.x - 1;
+  // a warp whose items all belong to one frame folds them first (the usual case)
+  const int f0 = __shfl_sync(0xffffffffu, f, 0);
+  if (__all_sync(0xffffffffu, f == f0)) {
+    key = warp_max_key(key);
+    if ((threadIdx.x & 31) == 0 && f0 >= 0 && key > __ldcg(keys + f0)) atomicMax(keys + f0, key);
+  } else if (f >= 0 && key > __ldcg(keys + f)) {
+    atomicMax(keys + f, key);
   }
   __syncthreads();
-  if (last && threadIdx.x == 0) {
+  if (threadIdx.x == 0) {
     __threadfence();
-    const unsigned long long k = atomicOr(keys + f, 0ull);
+    last = atomicAdd(done, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  for (int fr = threadIdx.x; fr < batch; fr += blockDim.x) {
+    const unsigned long long k = atomicOr(keys + fr, 0ull);
     const uint32_t idx = key_index(k);
     PeakOut pk;
     pk.score = ssd ? -key_score(k) : key_score(k);
     pk.u = (int32_t)(idx / (uint32_t)V);
     pk.v = (int32_t)(idx % (uint32_t)V);
     pk.flags = (ts.flat && !ssd) ? (kFlatTemplate | kInvalid) : 0u;
-    peaks[f] = pk;
-    done[f] = 0u;  // ready for the next call (stream-ordered)
+    peaks[fr] = pk;
   }
+  if (threadIdx.x == 0) *done = 0u;  // ready for the next call (stream-ordered)
 }
 
 }  // namespace nccb

@@ -72,12 +72,14 @@ def test_cfg1_default_plan_full_surface(smooth):
 
 @pytest.mark.parametrize("base,delta,flat", [(4.0, 2.0 ** -15, True), (4.0, 2.0 ** -13, False)])
 @pytest.mark.parametrize("cuda_cores", [True, False])
-def test_flat_threshold_straddle(base, delta, flat, cuda_cores):
+def test_flat_threshold_straddle(base, delta, flat, cuda_cores, monkeypatch):
     """SURVEY 8(c) reading 4 on the GPU: checkerboard templates whose centred / raw energy ratio
     straddles 1e-10 (pinned in test_oracle.py::test_flat_threshold_relative_to_raw_energy) get
     the oracle's flat decision -- FLAT_TEMPLATE|INVALID and an all-zero surface for the flat one,
     a valid peak and oracle-equal scores for the other (CUDA-core and tensor-core templates)."""
     h = w = 4 if cuda_cores else 144
+    if not cuda_cores:
+        monkeypatch.setenv("NCC_TC", "1")  # tensor cores whenever eligible (small problem)
     sgn = np.where((np.add.outer(np.arange(h), np.arange(w)) % 2) == 0, 1.0, -1.0)
     T = (base + delta * sgn).astype(np.float32)
     assert oracle.template_is_flat(T) == flat

@@ -27,6 +27,10 @@ def main():
         d_img, d_t = torch.from_numpy(img).to(DEV), torch.from_numpy(T).to(DEV)
         plan = MatchPlan(c["H"], c["W"], c["h"], c["w"])
         call = lambda: plan.match(d_img, d_t)  # noqa: E731
+        if os.environ.get("TL_HOST"):  # the host-buffer entry point (copies in the timeline)
+            h_img, h_t = torch.from_numpy(img).pin_memory(), torch.from_numpy(T).pin_memory()
+            h_pk = torch.empty((1, 4), dtype=torch.int32).pin_memory()
+            call = lambda: plan.match_host(h_img, h_t, h_pk)  # noqa: E731
     else:
         P = 1 if cfg == 3 else 8
         A = torch.rand((P, c["H"], c["W"]), device=DEV)
@@ -37,12 +41,12 @@ def main():
         flush.fill_(1.0)
         call()
     torch.cuda.synchronize()
-    with profile(activities=[ProfilerActivity.CUDA]) as prof:
+    with profile(activities=[ProfilerActivity.CUDA, ProfilerActivity.CPU]) as prof:
         for _ in range(reps):
             flush.fill_(1.0)
             call()
         torch.cuda.synchronize()
-    evs = [e for e in prof.events() if e.device_type.name == "CUDA"]
+    evs = [e for e in prof.events() if e.device_type.name == "CUDA" or "Memcpy" in e.name]
     evs.sort(key=lambda e: e.time_range.start)
     # split into steps at each flush kernel
     steps, cur = [], None
