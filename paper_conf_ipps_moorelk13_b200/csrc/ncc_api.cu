@@ -1006,9 +1006,12 @@ bool getenv_flag_two_kernel_prep() {  // NCC_TC_TWO_KERNEL_PREP=1: the earlier t
   return v;
 }
 
+// `nframes` frames (<= the plan's batch; -1 = all) from d_images; peaks / surfaces of frame k at
+// index k (the host path streams chunks of frames through this).
 ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, int64_t tmpl_pitch, float* d_scores,
-                     ncc_peak* d_peaks, cudaStream_t s, const int32_t* d_rois = nullptr) {
+                     ncc_peak* d_peaks, cudaStream_t s, const int32_t* d_rois = nullptr, int nframes = -1) {
   const ncc_problem& p = pl->p;
+  const int batch = nframes < 0 ? p.batch : nframes;
   const TmVariant* v = pl->tmv;
   if (p.flags & NCC_F_TIMING) {
     ncc_status st = ensure_events(pl, 5);
@@ -1022,7 +1025,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
                                  pl->h_tmpl_pitch * sizeof(float), p.tmpl_w * sizeof(float), p.tmpl_h,
                                  cudaMemcpyHostToDevice, s));
       NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
-                               (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
+                               (size_t)batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
     }
     mark(pl, s, 1);
     mark(pl, s, 2);
@@ -1033,7 +1036,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     int64_t pitch = p.image_pitch;
     void* args[] = {&d_images, &pitch, &fs, &W, &d_tmpl, &tmpl_pitch, &h, &w, &ub, &Ubv, &V, &rows,
                     &scores, &sfs, &pl->keys, &pl->tiny_done, &d_peaks, &ssd};
-    NCC_CUDA(cudaLaunchKernel(pl->tiny_fn, dim3(pl->tiny_ctas, p.batch), dim3(256), args, (size_t)pl->tiny_smem, s));
+    NCC_CUDA(cudaLaunchKernel(pl->tiny_fn, dim3(pl->tiny_ctas, batch), dim3(256), args, (size_t)pl->tiny_smem, s));
     mark(pl, s, 3);
     mark(pl, s, 4);
     return NCC_OK;
@@ -1041,7 +1044,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   CUtensorMap map_tc;
   bool tc_now = false;
   if (pl->tc) {  // the band's rows as (hi, lo) pairs: W x Hs x batch 8-byte elements
-    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)pl->Hs, (uint64_t)p.batch};
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)pl->Hs, (uint64_t)batch};
     const int wp = (p.image_w + 1) & ~1;  // pairs per staged row (even)
     const uint64_t strides[2] = {(uint64_t)wp * 8, (uint64_t)pl->Hs * wp * 8};
     const uint32_t box[3] = {(uint32_t)tc::kBoxW, 1u, 1u};
@@ -1055,19 +1058,19 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     // cfg 5: 740 -> 329 us, no longer delaying the numerator's start)
     constexpr int RWN = 4;
     const int jc = ceil_div(p.tmpl_w, 32);
-    const int64_t items = (int64_t)p.batch * (jc <= 8 ? pl->Ub : ceil_div(pl->Ub, RWN)) * pl->tc_vcols;
+    const int64_t items = (int64_t)batch * (jc <= 8 ? pl->Ub : ceil_div(pl->Ub, RWN)) * pl->tc_vcols;
     const int64_t pfs = (int64_t)pl->Ub * pl->V;
     auto cols = [&](auto kern) {
       kern<<<(unsigned)ceil_div(items, 8), 256, 0, pl->side>>>(
           d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w,
-          pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, p.batch, pl->tc_acc, pfs);
+          pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, batch, pl->tc_acc, pfs);
     };
     if (jc <= 4) cols(tm_tc_cols<4>);
     else if (jc <= 8) cols(tm_tc_cols<8>);
     else cols(tm_tc_cols_rw<16, RWN>);
   };
   auto launch_split = [&]() {
-    tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, p.batch), 128, 0, s>>>(
+    tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, batch), 128, 0, s>>>(
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
         reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 1) & ~1), (p.image_w + 1) & ~1);
   };
@@ -1084,17 +1087,17 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
                                cudaMemcpyHostToDevice, pl->side));
   if (pl->h_img_in) {
     NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
-                             (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
+                             (size_t)batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
     NCC_CUDA(cudaEventRecord(pl->ev_img, s));
   }
   if (pl->tc && p.tmpl_h * p.tmpl_w <= kPrepSmemFloats && !getenv_flag_two_kernel_prep()) {
     // one launch: template stats + centred template + MMA operand, template staged in shared memory
     tm_tc_prep<<<nblk_tc, 1024, p.tmpl_h * p.tmpl_w * 4, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
-                                               pl->tst, pl->keys, p.batch, pl->tc_wc, pl->tc_nbj, pl->tcB);
+                                               pl->tst, pl->keys, batch, pl->tc_wc, pl->tc_nbj, pl->tcB);
     mark(pl, pl->side, 1);
   } else {
     tm_template_prep<<<pl->n_tmpl, 1024, 0, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP,
-                                                         pl->WP, pl->tst, pl->keys, p.batch);
+                                                         pl->WP, pl->tst, pl->keys, batch);
     mark(pl, pl->side, 1);
     if (pl->tc)
       tm_tc_tpl_prep<<<nblk_tc, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj,
@@ -1110,7 +1113,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }
     launch_split();
-    launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
+    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
   } else {
@@ -1120,7 +1123,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       launch_cols();
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }
-    launch_box(pl, d_images, p.batch, pl->u_begin, pl->Ub, s);
+    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
   }
@@ -1155,14 +1158,14 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.score_frame_stride = (int64_t)pl->Ub * pl->V;
     t.keys = pl->keys;
     t.ssd = p.score == NCC_SCORE_SSD;
-    tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, p.batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
+    tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
     mark(pl, s, 3);
     if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
-    const int64_t tail_items = (int64_t)p.batch * pl->Ub * pl->tc_vcols;
+    const int64_t tail_items = (int64_t)batch * pl->Ub * pl->tc_vcols;
     tm_tc_tail<<<(unsigned)std::max<int64_t>(1, ceil_div(tail_items, 256)), 256, 0, s>>>(
         pl->tc_acc, (int64_t)pl->Ub * pl->V, pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V,
-        pl->V - pl->tc_vcols, pl->u_begin, pl->Ub, p.batch, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
+        pl->V - pl->tc_vcols, pl->u_begin, pl->Ub, batch, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
         (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks));
     mark(pl, s, 4);
     cudaError_t e = cudaGetLastError();
@@ -1210,12 +1213,12 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   memset(&map_img, 0, sizeof(map_img));
   bool use_tma = pl->tma_ok && (reinterpret_cast<uintptr_t>(d_images) % 16 == 0) && (p.image_pitch % 4 == 0);
   if (use_tma) {
-    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)p.batch};
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)batch};
     const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)p.image_h * p.image_pitch * 4};
     const uint32_t box[3] = {(uint32_t)v->ip, (uint32_t)v->ir, 1u};
     use_tma = encode_f32(&map_img, d_images, 3, dims, strides, box);
   }
-  dim3 grid(pl->tiles_u * pl->tiles_v * pl->split, p.batch * pl->n_tmpl);
+  dim3 grid(pl->tiles_u * pl->tiles_v * pl->split, batch * pl->n_tmpl);
   const int t = use_tma ? 1 : 0, ct = pl->use_ct ? 1 : 0;
   const int nCWl = pl->WP / v->CW;
   a.carry = pl->carry;
@@ -1250,8 +1253,8 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     }
   }
   mark(pl, s, 3);
-  tm_finalize<<<ceil_div((int64_t)p.batch * pl->n_tmpl, 128), 128, 0, s>>>(
-      pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks), p.batch, p.score == NCC_SCORE_SSD, pl->n_tmpl);
+  tm_finalize<<<ceil_div((int64_t)batch * pl->n_tmpl, 128), 128, 0, s>>>(
+      pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks), batch, p.score == NCC_SCORE_SSD, pl->n_tmpl);
   mark(pl, s, 4);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch");
@@ -1433,6 +1436,18 @@ ncc_status run_graph(ncc_plan pl, const uintptr_t (&key)[8], cudaStream_t s, Bod
   } else {
     NCC_CUDA(cudaGraphLaunch(pl->graphs[hit].exec, s));
   }
+  return NCC_OK;
+}
+
+// The host paths' copy stream and slot events (lazy).
+ncc_status ensure_copy_stream(ncc_plan pl) {
+  if (pl->copy) return NCC_OK;
+  NCC_CUDA(cudaStreamCreateWithFlags(&pl->copy, cudaStreamNonBlocking));
+  for (int k = 0; k < 2; ++k) {
+    NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_copied[k], cudaEventDisableTiming));
+    NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_free[k], cudaEventDisableTiming));
+  }
+  NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_start, cudaEventDisableTiming));
   return NCC_OK;
 }
 
@@ -1652,11 +1667,58 @@ ncc_status ncc_match_host(ncc_plan pl, const float* h_images, const float* h_tmp
   const bool surf = (p.flags & NCC_F_WRITE_SURFACE) != 0;
   const size_t s_bytes = surf ? (size_t)p.batch * pl->Ub * pl->V * sizeof(float) : 0;
   ncc_status st;
+  const bool pinned = is_pinned(h_images) && is_pinned(h_tmpl);
+  // frames per streamed chunk: ~8 MB of frames (NCC_TM_CHUNK overrides)
+  const size_t frame_b = (size_t)p.image_h * p.image_pitch * sizeof(float);
+  int chunk = (int)std::max<size_t>(1, ((size_t)8 << 20) / frame_b);
+  if (const char* e = getenv("NCC_TM_CHUNK")) chunk = std::max(1, atoi(e));
+  if (pinned && p.batch > chunk) {
+    // Streaming (the paper's per-frame runtime operation, 5.1.3.4 P:91): chunks of
+    // frames through two device slots -- the host->device copy of chunk c + 1 runs on the plan's
+    // copy stream while chunk c is matched on `stream`; a slot is refilled only after its chunk's
+    // peaks (and surfaces) were copied back.  The template is copied once per call.
+    if ((st = ensure_copy_stream(pl))) return st;
+    const size_t sframe_b = (size_t)pl->Ub * pl->V * sizeof(float);
+    const size_t slot_b = (size_t)chunk * frame_b, sslot_b = surf ? (size_t)chunk * sframe_b : 0;
+    const size_t pslot_b = (size_t)chunk * sizeof(ncc_peak);
+    if ((st = stage((void**)&pl->st_a, &pl->st_a_bytes, 2 * slot_b))) return st;
+    if ((st = stage((void**)&pl->st_t, &pl->st_t_bytes, t_bytes))) return st;
+    if (surf && (st = stage((void**)&pl->st_s, &pl->st_s_bytes, 2 * sslot_b))) return st;
+    if ((st = stage(&pl->st_out, &pl->st_out_bytes, 2 * pslot_b))) return st;
+    NCC_CUDA(cudaMemcpy2DAsync(pl->st_t, p.tmpl_w * sizeof(float), h_tmpl, tmpl_pitch * sizeof(float),
+                               p.tmpl_w * sizeof(float), p.tmpl_h, cudaMemcpyHostToDevice, s));
+    NCC_CUDA(cudaEventRecord(pl->ev_start, s));  // earlier work on `stream` may still use the slots
+    NCC_CUDA(cudaStreamWaitEvent(pl->copy, pl->ev_start, 0));
+    const int nch = ceil_div(p.batch, chunk);
+    for (int c = 0; c < nch; ++c) {
+      const int k = c & 1, n = std::min(chunk, p.batch - c * chunk);
+      float* sa = pl->st_a + (size_t)k * (slot_b / sizeof(float));
+      float* ss = surf ? pl->st_s + (size_t)k * (sslot_b / sizeof(float)) : nullptr;
+      ncc_peak* so = reinterpret_cast<ncc_peak*>(static_cast<char*>(pl->st_out) + (size_t)k * pslot_b);
+      if (c >= 2) NCC_CUDA(cudaStreamWaitEvent(pl->copy, pl->ev_free[k], 0));
+      NCC_CUDA(cudaMemcpyAsync(sa, reinterpret_cast<const char*>(h_images) + (size_t)c * slot_b, n * frame_b,
+                               cudaMemcpyHostToDevice, pl->copy));
+      NCC_CUDA(cudaEventRecord(pl->ev_copied[k], pl->copy));
+      NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_copied[k], 0));
+      const uintptr_t key[8] = {(uintptr_t)sa, (uintptr_t)pl->st_t, (uintptr_t)p.tmpl_w, (uintptr_t)ss,
+                                (uintptr_t)so, (uintptr_t)n, 0, 1};
+      st = run_graph(pl, key, s, [&](cudaStream_t cs) {
+        return run_match(pl, sa, pl->st_t, p.tmpl_w, ss, so, cs, nullptr, n);
+      });
+      if (st) return st;
+      NCC_CUDA(cudaMemcpyAsync(h_peaks + (size_t)c * chunk, so, n * sizeof(ncc_peak), cudaMemcpyDeviceToHost, s));
+      if (surf && h_scores)
+        NCC_CUDA(cudaMemcpyAsync(reinterpret_cast<char*>(h_scores) + (size_t)c * chunk * sframe_b, ss,
+                                 n * sframe_b, cudaMemcpyDeviceToHost, s));
+      NCC_CUDA(cudaEventRecord(pl->ev_free[k], s));
+    }
+    return NCC_OK;
+  }
   if ((st = stage((void**)&pl->st_a, &pl->st_a_bytes, img_bytes))) return st;
   if ((st = stage((void**)&pl->st_t, &pl->st_t_bytes, t_bytes))) return st;
   if (surf && (st = stage((void**)&pl->st_s, &pl->st_s_bytes, s_bytes))) return st;
   if ((st = stage(&pl->st_out, &pl->st_out_bytes, (size_t)p.batch * sizeof(ncc_peak)))) return st;
-  if (is_pinned(h_images) && is_pinned(h_tmpl)) {
+  if (pinned) {
     // pinned inputs: the copies are part of the (captured) launch sequence, the template's
     // ahead of its prep on the side stream (see run_match)
     const uintptr_t key[8] = {(uintptr_t)pl->st_a, (uintptr_t)pl->st_t, (uintptr_t)p.tmpl_w, (uintptr_t)pl->st_s,
@@ -1713,14 +1775,7 @@ ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, p
   // Streaming: chunks of sub_batch pairs through two device slots.  The host->device copy of
   // chunk c + 1 runs on the plan's copy stream while chunk c is correlated on `stream`; a slot
   // is refilled only after the chunk that used it (and its vectors' copy-back) is done.
-  if (!pl->copy) {
-    NCC_CUDA(cudaStreamCreateWithFlags(&pl->copy, cudaStreamNonBlocking));
-    for (int k = 0; k < 2; ++k) {
-      NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_copied[k], cudaEventDisableTiming));
-      NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_free[k], cudaEventDisableTiming));
-    }
-    NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_start, cudaEventDisableTiming));
-  }
+  if ((st = ensure_copy_stream(pl))) return st;
   const size_t pair_b = (size_t)p.image_h * p.image_pitch * sizeof(float);
   const size_t vpair_b = (size_t)pl->Ky * pl->Kx * sizeof(piv_vector);
   const size_t slot_b = (size_t)chunk * pair_b, vslot_b = (size_t)chunk * vpair_b;
