@@ -424,6 +424,30 @@ def measure(ctx, cfg, steps, warmup, headline=True, cpu_budget=10.0):
     e2e = {"value": units_all * steps / (et / 1e3), "unit": unit, "h2d_bytes_per_step": h2d,
            "d2h_bytes_per_step": d2h, "ms_per_step": et / steps,
            "api": "ncc_match_host" if kind == "tm" else "piv_correlate_host"}
+    if kind == "tm" and not multi:
+        # a stream of frames through the same public call: 8 frames per call, the host->device
+        # copy of the next chunk overlapping the match of the current one, beside the
+        # device-resident rate of the same 8-frame batch
+        F = 8
+        p8 = MatchPlan(wl["H"], wl["W"], wl["h"], wl["w"], batch=F, device=local)
+        hs = torch.from_numpy(np.ascontiguousarray(np.broadcast_to(wl["img"], (F,) + wl["img"].shape))).pin_memory()
+        hp8 = torch.empty((F, 4), dtype=torch.int32).pin_memory()
+        ds = hs.to(dev)
+        dp8 = torch.empty((F, 4), dtype=torch.int32, device=dev)
+        st8 = min(steps, 10)
+        run_steps(ctx, lambda: p8.match_host(hs, h_t, hp8, stream=stream), 3)
+        s_ms, _ = run_steps(ctx, lambda: p8.match_host(hs, h_t, hp8, stream=stream), st8)
+        run_steps(ctx, lambda: p8.match(ds, d_t, stream=stream, peaks=dp8), 3)
+        d_ms, _ = run_steps(ctx, lambda: p8.match(ds, d_t, stream=stream, peaks=dp8), st8)
+        u8 = p8.info.outputs_per_call
+        ok8 = bool((decode_peaks(hp8)["u"] == wl["planted"][0]).all() and (decode_peaks(hp8)["v"] == wl["planted"][1]).all())
+        e2e["stream8"] = {"value": u8 * st8 / (sum(s_ms) / 1e3), "unit": unit, "frames_per_call": F,
+                          "h2d_bytes_per_step": F * wl["img"].nbytes + wl["T"].nbytes,
+                          "d2h_bytes_per_step": F * 16, "ms_per_step": sum(s_ms) / st8,
+                          "device_value_same_batch": u8 * st8 / (sum(d_ms) / 1e3),
+                          "frac_of_device_same_batch": sum(d_ms) / sum(s_ms), "correct": ok8}
+        p8.close()
+        del hs, ds
 
     c = synth.CONFIGS[cfg]
     line = {"metric": metric, "value": value, "unit": unit, "n_gpus": ws if multi else 1, "steps": steps,

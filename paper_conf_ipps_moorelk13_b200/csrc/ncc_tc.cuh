@@ -110,6 +110,12 @@ constexpr int kNWin = kHB + kG;
 // MMA covers one contiguous run of columns (no ring-wrap split into two MMAs).
 constexpr int kRelocAt = ((kRing - kNWin) / kG + 1) * kG;
 static_assert(kRelocAt + kHB == kRing && kRelocAt >= kNWin, "relocation geometry");
+// Row groups in flight between the MMA warp and the drain (epilogue) warps: the columns drained
+// after group g are next written by the window of group g + kGRing (they enter it as its newest
+// kG output rows: (kG g + kHB) mod kRelocAt == kG (g - kGRing)), so the MMA warp waits for the
+// drain of group g - kGRing before group g; group-completion barriers form a ring of as many.
+constexpr int kGRing = (kRelocAt - kHB) / kG;
+static_assert(kGRing == 8 && ((kGRing * kG + kHB) % kRelocAt) == 0, "drain ring geometry");
 constexpr int kLB = ((kHB + 2 * kG - 1 + 7) / 8) * 8;  // rows of the reversed template block
 constexpr int kGroups = kNBuf;                           // producer groups of 4 warps; group g: stages q = g mod kNBuf
 // warp roles: producers 0 .. 4 kGroups - 1, relocation 4 kGroups .. + 3, TMA, then the MMA warp
@@ -193,7 +199,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   using namespace tc;
   extern __shared__ __align__(1024) unsigned char smem_tc[];
   __shared__ __align__(8) uint64_t a_full[kNBuf], mma_done[kNBuf], img_full[kNImg], img_empty[kNImg], reloc_req,
-      reloc_done;
+      reloc_done, grp_done[kGRing], drained[kGRing];
   __shared__ uint32_t tmem_base_s;
   __shared__ unsigned long long ticket_s;
 
@@ -247,6 +253,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     }
     mbar_init(&reloc_req, 1);
     mbar_init(&reloc_done, 128);
+    for (int b = 0; b < kGRing; ++b) {
+      mbar_init(&grp_done[b], 1);   // tcgen05.commit after a row group's last MMA
+      mbar_init(&drained[b], 128);  // the group's accumulator columns read and zeroed
+    }
     fence_mbar_init();
   }
   fence_before();
@@ -270,7 +280,6 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
                   ua - a.u_begin + i0 + q / nch, f, &img_full[sl]);
     }
   };
-  const int nreloc = (ngrp - 1) / (kRelocAt / kG);  // groups g > 0 whose window restarts at column 0
   if (TC_EXP(32768) && warp != kMmaWarp) {
     // trace experiment: the MMA warp alone
   } else if (TC_EXP(65536) && warp < 4 * kGroups) {
@@ -284,7 +293,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       }
     }
   } else if (warp < 4 * kGroups) {
-    // ===================== producers (lane v = output column v0 + v) and ring drain.
+    // ===================== producers (lane v = output column v0 + v).
     // Group grp (warps 4 grp .. 4 grp + 3, TMEM lane quadrants 0..3) handles the stages
     // q = grp mod kNBuf, i.e. TMEM A buffer grp: the groups' latencies overlap.
     const int grp = warp >> 2, wq = warp & 3;
@@ -299,9 +308,83 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       fence_before();
     }
     const uint2* ring = reinterpret_cast<const uint2*>(smem_tc + img_off(a.WC));
-    const int vv = v0 + v;
-    // (pointers are formed inside the drain from the kernel parameters: the producers run at
-    // the 96-register cap -- 5 warps of this SMSP-bound CTA share one SMSP's register file)
+    // Software-pipelined producer: the operand of the group's next stage is read from the ring
+    // and split while the group waits for its TMEM buffer, so the critical path from "MMAs of
+    // the buffer's previous stage done" to "a_full" is only the TMEM stores (the MMA warp has
+    // kNBuf - 1 stages of slack).  (Finished row groups are drained by the epilogue warps.)
+    uint32_t hi[kWB], lo[kWB];
+    auto load_split = [&](int q) {
+      const int sl = q % kNImg;
+      mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
+      if (gtid == 0) TC_STAMP(5, q);
+      // the split x = hi + lo was done once per image element (tm_tc_split): one 8-byte load
+      // per Hankel element, no per-lane conversion work
+      const bool zero = stage_zero(q) || TC_EXP(64);
+      // 16-byte loads from the even element at or below v (lanes 2i and 2i+1 share them: half
+      // the shared-memory wavefronts of one 8-byte load per element), odd lanes shift by one
+      const uint4* r4 = reinterpret_cast<const uint4*>(ring + sl * kBoxW + (v & ~1));
+      const bool odd = (v & 1) != 0;
+      uint32_t eh[kWB + 2], el[kWB + 2];
+#pragma unroll
+      for (int m = 0; m < kWB / 2 + 1; ++m) {
+        const uint4 t = zero ? make_uint4(0u, 0u, 0u, 0u) : r4[m];
+        eh[2 * m] = t.x;
+        el[2 * m] = t.y;
+        eh[2 * m + 1] = t.z;
+        el[2 * m + 1] = t.w;
+      }
+#pragma unroll
+      for (int k = 0; k < kWB; ++k) {
+        hi[k] = odd ? eh[k + 1] : eh[k];
+        lo[k] = odd ? el[k + 1] : el[k];
+      }
+      mbar_arrive(&img_empty[sl]);
+      if (gtid == 0) TC_STAMP(1, q);
+    };
+    if (grp < nstage) load_split(grp);
+    const int b = grp;
+#pragma unroll 1
+    for (int q = grp; q < nstage + kNBuf; q += kGroups) {
+      const int qd = q - kNBuf;  // the buffer's previous stage
+      if (qd >= 0) {
+        if (!TC_EXP(256)) mbar_wait_bounded(&mma_done[b], (uint32_t)((qd / kNBuf) & 1));
+        if (!TC_EXP(128)) fence_after();
+        if (gtid == 0) TC_STAMP(0, qd);
+      }
+      if (q < nstage) {
+        const uint32_t ab = tbase + lane_base + a_col0 + (uint32_t)(b * 2 * kWB);
+        if (!TC_EXP(1)) {
+#pragma unroll
+          for (int c = 0; c < kWB; c += 8) {
+            st8(ab + c, *reinterpret_cast<const uint32_t(*)[8]>(hi + c));
+            st8(ab + kWB + c, *reinterpret_cast<const uint32_t(*)[8]>(lo + c));
+          }
+        }
+        if (!TC_EXP(512)) st_wait();
+        if (!TC_EXP(128)) fence_before();
+        mbar_arrive(&a_full[b]);
+        if (gtid == 0) TC_STAMP(2, q);
+      }
+      if (q + kGroups < nstage) load_split(q + kGroups);
+    }
+  } else if (warp == kTmaWarp) {
+    // ===================== TMA producer: image-row segments, kNImg stages ahead
+    if (lane == 0) {
+      tma_prefetch_desc(&map_img);
+#pragma unroll 1
+      for (int q = 0; q < nstage; ++q) issue(q);
+    }
+    __syncwarp();
+  } else if (warp >= kRelocWarp0 && warp < kRelocWarp0 + 4) {
+    // ===================== epilogue warps (lane quadrant wq = warp % 4, lane v = column v0 + v):
+    // drain every finished row group -- read its kG accumulator columns from TMEM, zero them,
+    // release them to the MMA warp (drained ring) -- then do the group's global work (block
+    // chain, normalisation, keys) off the producers' and the MMA warp's critical path; between
+    // groups, the rare relocation of the live window.
+    const int wq = warp & 3;
+    const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
+    const int vv = v0 + wq * 32 + lane;
+    const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
     // Drain of row group gd (its MMAs are complete): output rows up = kG gd - kHB + 1 + k.
     // Chain: block b > 0 waits until block b - 1 published the group's running numerator (this
     // warp's 32 columns), adds its own; blocks b < nblk - 1 publish; the last block normalises
@@ -366,120 +449,36 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         if (blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
       }
     };
-    // Software-pipelined producer: the operand of the group's next stage is read from the ring
-    // and split while the group waits for its TMEM buffer, so the critical path from "MMAs of
-    // the buffer's previous stage done" to "a_full" is only the TMEM stores (the MMA warp has
-    // kNBuf - 1 stages of slack).  The ring drain of a finished group follows the arrival.
-    uint32_t hi[kWB], lo[kWB];
-    auto load_split = [&](int q) {
-      const int sl = q % kNImg;
-      mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
-      if (gtid == 0) TC_STAMP(5, q);
-      // the split x = hi + lo was done once per image element (tm_tc_split): one 8-byte load
-      // per Hankel element, no per-lane conversion work
-      const bool zero = stage_zero(q) || TC_EXP(64);
-      // 16-byte loads from the even element at or below v (lanes 2i and 2i+1 share them: half
-      // the shared-memory wavefronts of one 8-byte load per element), odd lanes shift by one
-      const uint4* r4 = reinterpret_cast<const uint4*>(ring + sl * kBoxW + (v & ~1));
-      const bool odd = (v & 1) != 0;
-      uint32_t eh[kWB + 2], el[kWB + 2];
-#pragma unroll
-      for (int m = 0; m < kWB / 2 + 1; ++m) {
-        const uint4 t = zero ? make_uint4(0u, 0u, 0u, 0u) : r4[m];
-        eh[2 * m] = t.x;
-        el[2 * m] = t.y;
-        eh[2 * m + 1] = t.z;
-        el[2 * m + 1] = t.w;
-      }
-#pragma unroll
-      for (int k = 0; k < kWB; ++k) {
-        hi[k] = odd ? eh[k + 1] : eh[k];
-        lo[k] = odd ? el[k + 1] : el[k];
-      }
-      mbar_arrive(&img_empty[sl]);
-      if (gtid == 0) TC_STAMP(1, q);
-    };
-    if (grp < nstage) load_split(grp);
-    const int b = grp;
+    int nrel = 0;
 #pragma unroll 1
-    for (int q = grp; q < nstage + kNBuf; q += kGroups) {
-      const int qd = q - kNBuf;  // the buffer's previous stage
-      if (qd >= 0) {
-        if (!TC_EXP(256)) mbar_wait_bounded(&mma_done[b], (uint32_t)((qd / kNBuf) & 1));
-        if (!TC_EXP(128)) fence_after();
-        if (gtid == 0) TC_STAMP(0, qd);
-      }
-      if (q < nstage) {
-        const uint32_t ab = tbase + lane_base + a_col0 + (uint32_t)(b * 2 * kWB);
-        if (!TC_EXP(1)) {
-#pragma unroll
-          for (int c = 0; c < kWB; c += 8) {
-            st8(ab + c, *reinterpret_cast<const uint32_t(*)[8]>(hi + c));
-            st8(ab + kWB + c, *reinterpret_cast<const uint32_t(*)[8]>(lo + c));
-          }
+    for (int gd = 0; gd < ngrp; ++gd) {
+      if (gd > 0 && (gd * kG) % kRelocAt == 0) {
+        // the MMA warp requests the relocation before group gd (all earlier MMAs complete, all
+        // earlier groups drained by this warp): move the live columns to the front
+        mbar_wait_bounded(&reloc_req, (uint32_t)(nrel & 1));
+        fence_after();
+#pragma unroll 1
+        for (int c = 0; c < kHB; c += 8) {
+          uint32_t d[8];
+          ld8(tbase + lane_base + kRelocAt + c, d);
+          st8(tbase + lane_base + c, d);
+          st8(tbase + lane_base + kRelocAt + c, z);
         }
-        if (!TC_EXP(512)) st_wait();
-        if (!TC_EXP(128)) fence_before();
-        mbar_arrive(&a_full[b]);
-        if (gtid == 0) TC_STAMP(2, q);
+        st_wait();
+        fence_before();
+        mbar_arrive(&reloc_done);
+        ++nrel;
       }
-      // drain the ring columns of a group whose last stage was qd (its MMAs are complete);
-      // the zeroing stores are waited for before this group's next a_full arrival
-      if (qd >= 0 && !TC_EXP(32) && qd % nch == nch - 1 && (qd / nch) % kG == kG - 1) {
-        const int gd = (qd / nch) / kG;
-        const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
-        uint32_t d[8];
-        ld8(tbase + lane_base + col, d);
-        const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
-        st8(tbase + lane_base + col, z);  // the columns are free again once read
-        drain(gd, d);
-      }
-      if (q + kGroups < nstage) load_split(q + kGroups);
-    }
-    st_wait();  // last zeroing stores
-  } else if (warp == kTmaWarp) {
-    // ===================== TMA producer: image-row segments, kNImg stages ahead
-    if (lane == 0) {
-      tma_prefetch_desc(&map_img);
-#pragma unroll 1
-      for (int q = 0; q < nstage; ++q) issue(q);
-    }
-    __syncwarp();
-  } else if (warp >= kRelocWarp0 && warp < kRelocWarp0 + 4) {
-    // ===================== relocation warps (lane quadrant warp % 4): move the live window
-    const uint32_t lane_base = (uint32_t)((warp & 3) * 32) << 16;
-    const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
-#pragma unroll 1
-    for (int k = 0; k < nreloc; ++k) {
-      // rare event: wait in the mbarrier's own suspend (try_wait), not with nanosleep polling:
-      // sleeping warps on the SM slow the MMA warp's issue (tools/microbench/umma_probe.cu)
-      if (TC_EXP(8192)) {
-        for (long long it = 0;; ++it) {
-          uint32_t done = 0;
-          asm volatile(
-              "{\n\t.reg .pred P;\n\tmbarrier.test_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
-              "selp.u32 %0, 1, 0, P;\n}"
-              : "=r"(done)
-              : "r"(smem_u32(&reloc_req)), "r"((uint32_t)(k & 1))
-              : "memory");
-          if (done) break;
-          if (it > (1ll << 26)) __trap();
-          __nanosleep(256);
-        }
-      } else {
-        mbar_wait_bounded(&reloc_req, (uint32_t)(k & 1));
-      }
+      mbar_wait_bounded(&grp_done[gd % kGRing], (uint32_t)((gd / kGRing) & 1));
       fence_after();
-#pragma unroll 1
-      for (int c = 0; c < kHB; c += 8) {
-        uint32_t d[8];
-        ld8(tbase + lane_base + kRelocAt + c, d);
-        st8(tbase + lane_base + c, d);
-        st8(tbase + lane_base + kRelocAt + c, z);
-      }
+      const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
+      uint32_t d[8];
+      ld8(tbase + lane_base + col, d);
+      st8(tbase + lane_base + col, z);  // the columns are free again once read
       st_wait();
       fence_before();
-      mbar_arrive(&reloc_done);
+      mbar_arrive(&drained[gd % kGRing]);
+      if (!TC_EXP(32)) drain(gd, d);
     }
   } else if (warp == kMmaWarp) {
     // ===================== MMA issuer (one thread)
@@ -516,6 +515,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       // addresses are converted once, the B descriptor moves by one 16-byte row per image row,
       // the accumulator column / instruction descriptor change once per group.
       const uint32_t full0 = smem_u32(&a_full[0]), done0 = smem_u32(&mma_done[0]);
+      const uint32_t gdone0 = smem_u32(&grp_done[0]), drained0 = smem_u32(&drained[0]);
       const bool leader = elect_one();
       if (nstage > 0 && !TC_EXP(16)) mbar_wait_u32(full0, 0u);
       fence_after();
@@ -533,6 +533,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           mbar_wait_bounded(&reloc_done, (uint32_t)(nrel_done & 1));
           fence_after();
           ++nrel_done;
+        }
+        if (g >= kGRing) {  // the window's newest columns were drained (and zeroed) after group g - kGRing
+          mbar_wait_u32(drained0 + 8 * ((g - kGRing) % kGRing), (uint32_t)(((g - kGRing) / kGRing) & 1));
+          fence_after();
         }
         trim(g);
         const uint32_t dcol = tbase + col + (uint32_t)c0;
@@ -571,6 +575,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
             if (lane == 0) TC_STAMP(4, q);
           }
         }
+        if (leader) commit_u32(gdone0 + 8 * (g % kGRing));  // group g's MMAs complete -> epilogue drains it
+        __syncwarp();
       }
     }
     __syncwarp();
