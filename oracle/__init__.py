@@ -82,6 +82,8 @@ def lib():
         _lib.oracle_argmin.argtypes = [P, i64]
         _lib.oracle_argmin.restype = i64
         _lib.oracle_piv_windows_ssd.argtypes = [P, P, i32, i32, i64] + [i32] * 6 + [P, P, i32, P, P]
+        _lib.oracle_sad_surface.argtypes = [P, i32, i32, i64, P, i32, i32, i64, i32, i32, P]
+        _lib.oracle_piv_windows_sad.argtypes = [P, P, i32, i32, i64] + [i32] * 6 + [P, P, i32, P, P]
     return _lib
 
 
@@ -256,4 +258,39 @@ def piv_windows_ssd(A, B, h, w, my, mx, sy, sx, kys, kxs) -> np.ndarray:
     if lib().oracle_piv_windows_ssd(_ptr(A), _ptr(B), H, W, W, h, w, my, mx, sy, sx,
                                     _ptr(kys), _ptr(kxs), n, _ptr(scratch), _ptr(out)):
         raise ValueError("oracle_piv_windows_ssd: invalid arguments")
+    return out
+
+
+# ---------------------------------------------------------------- SAD (Ch. 4 specialisation example)
+def sad_surface(img: np.ndarray, tmpl: np.ndarray, u_begin: int = 0, u_end: int | None = None) -> np.ndarray:
+    img, tmpl = _f32(img), _f32(tmpl)
+    H, W = img.shape
+    h, w = tmpl.shape
+    U, V = H - h + 1, W - w + 1
+    if u_end is None:
+        u_end = U
+    out = np.empty((u_end - u_begin, V), dtype=np.float64)
+    if lib().oracle_sad_surface(_ptr(img), H, W, W, _ptr(tmpl), h, w, w, u_begin, u_end, _ptr(out)):
+        raise ValueError("oracle_sad_surface: invalid arguments")
+    return out
+
+
+def sad_match(img, tmpl):
+    s = sad_surface(img, tmpl)
+    k = argmin(s)
+    V = s.shape[1]
+    return s, Peak(float(s.ravel()[k]), k // V, k % V, True)
+
+
+def piv_windows_sad(A, B, h, w, my, mx, sy, sx, kys, kxs) -> np.ndarray:
+    A, B = _f32(A), _f32(B)
+    H, W = A.shape
+    kys = np.ascontiguousarray(kys, dtype=np.int32)
+    kxs = np.ascontiguousarray(kxs, dtype=np.int32)
+    n = len(kys)
+    scratch = np.empty(n * (2 * my + 1) * (2 * mx + 1), dtype=np.float64)
+    out = np.zeros(n, dtype=_PIV_DTYPE)
+    if lib().oracle_piv_windows_sad(_ptr(A), _ptr(B), H, W, W, h, w, my, mx, sy, sx,
+                                    _ptr(kys), _ptr(kxs), n, _ptr(scratch), _ptr(out)):
+        raise ValueError("oracle_piv_windows_sad: invalid arguments")
     return out

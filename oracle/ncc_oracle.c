@@ -93,6 +93,34 @@ static double ssd_window(const float *img, int64_t pitch, int r0, int c0,
     return s;
 }
 
+/* Sum of absolute differences of the template against one window: the specialisation example
+ * of the paper's Ch. 4 ("sum of absolute differences to sum of squared differences")
+ * -- the other classic block-matching score.  Plain definition, fp64, row-major serial sum. */
+static double sad_window(const float *img, int64_t pitch, int r0, int c0,
+                         const float *tmpl, int64_t tpitch, int h, int w)
+{
+    double s = 0.0;
+    for (int i = 0; i < h; ++i)
+        for (int j = 0; j < w; ++j)
+            s += fabs((double)tmpl[(int64_t)i * tpitch + j] - (double)img[(int64_t)(r0 + i) * pitch + (c0 + j)]);
+    return s;
+}
+
+/* SAD surface for offset rows [u_begin, u_end) (valid offsets, as oracle_ncc_surface). */
+int oracle_sad_surface(const float *img, int H, int W, int64_t pitch,
+                       const float *tmpl, int h, int w, int64_t tpitch,
+                       int u_begin, int u_end, double *scores)
+{
+    if (h <= 0 || w <= 0 || h > H || w > W) return -1;
+    const int U = H - h + 1, V = W - w + 1;
+    if (u_begin < 0 || u_end > U || u_begin > u_end) return -1;
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int u = u_begin; u < u_end; ++u)
+        for (int v = 0; v < V; ++v)
+            scores[(int64_t)(u - u_begin) * V + v] = sad_window(img, pitch, u, v, tmpl, tpitch, h, w);
+    return 0;
+}
+
 /* SSD surface for offset rows [u_begin, u_end) (valid offsets, as oracle_ncc_surface). */
 int oracle_ssd_surface(const float *img, int H, int W, int64_t pitch,
                        const float *tmpl, int h, int w, int64_t tpitch,
@@ -265,10 +293,12 @@ static void piv_one_window(const float *A, const float *B, int64_t pitch,
     out->flags = flags;
 }
 
-/* PIV with the SSD score (the paper's metric, Fig 5.10): argmin over the search range
+/* PIV with a distance score -- SSD (the paper's metric, Fig 5.10) or SAD: argmin over the search range
  * (tie -> smallest row-major index), 3-point parabolic sub-pixel fit of the minimum per axis
  * (delta = (c- - c+) / (2 (c- - 2 c0 + c+)), 0 if that denominator <= 0), no fit on the border. */
-static void piv_one_window_ssd(const float *A, const float *B, int64_t pitch,
+typedef double (*window_score_fn)(const float *, int64_t, int, int, const float *, int64_t, int, int);
+
+static void piv_one_window_min(window_score_fn score, const float *A, const float *B, int64_t pitch,
                                int h, int w, int my, int mx, int y, int x,
                                double *scratch, oracle_piv_vector *out)
 {
@@ -277,7 +307,7 @@ static void piv_one_window_ssd(const float *A, const float *B, int64_t pitch,
     for (int dy = -my; dy <= my; ++dy)
         for (int dx = -mx; dx <= mx; ++dx)
             scratch[(dy + my) * OX + (dx + mx)] =
-                ssd_window(B, pitch, y + dy, x + dx, tmpl, pitch, h, w);
+                score(B, pitch, y + dy, x + dx, tmpl, pitch, h, w);
     const int64_t k = oracle_argmin(scratch, (int64_t)OY * OX);
     const int iy = (int)(k / OX) - my, ix = (int)(k % OX) - mx;
     uint32_t flags = 0;
@@ -381,7 +411,24 @@ int oracle_piv_windows_ssd(const float *A, const float *B, int H, int W, int64_t
     const int64_t per = (int64_t)(2 * my + 1) * (2 * mx + 1);
 #pragma omp parallel for schedule(dynamic, 1)
     for (int i = 0; i < count; ++i)
-        piv_one_window_ssd(A, B, pitch, h, w, my, mx, my + kys[i] * sy, mx + kxs[i] * sx,
+        piv_one_window_min(ssd_window, A, B, pitch, h, w, my, mx, my + kys[i] * sy, mx + kxs[i] * sx,
+                           scratch + (int64_t)i * per, &out[i]);
+    return 0;
+}
+
+int oracle_piv_windows_sad(const float *A, const float *B, int H, int W, int64_t pitch,
+                           int h, int w, int my, int mx, int sy, int sx,
+                           const int *kys, const int *kxs, int count,
+                           double *scratch, oracle_piv_vector *out)
+{
+    int Ky, Kx;
+    if (oracle_piv_grid(H, W, h, w, my, mx, sy, sx, &Ky, &Kx)) return -1;
+    for (int i = 0; i < count; ++i)
+        if (kys[i] < 0 || kys[i] >= Ky || kxs[i] < 0 || kxs[i] >= Kx) return -1;
+    const int64_t per = (int64_t)(2 * my + 1) * (2 * mx + 1);
+#pragma omp parallel for schedule(dynamic, 1)
+    for (int i = 0; i < count; ++i)
+        piv_one_window_min(sad_window, A, B, pitch, h, w, my, mx, my + kys[i] * sy, mx + kxs[i] * sx,
                            scratch + (int64_t)i * per, &out[i]);
     return 0;
 }

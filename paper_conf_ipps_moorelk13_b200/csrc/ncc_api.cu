@@ -326,6 +326,7 @@ struct ncc_plan_s {
   unsigned int* tc_flags;  // chain flags [batch][vtiles * nseg][ngrp_max][4] (self-resetting)
   unsigned long long* tc_ticket;  // CTA start tickets (monotonic)
   int tc_ngrp;
+  int tc_exp;  // NCC_TC_EXP timing experiments (0 in normal use; results are wrong with bits set)
   // tiny problems: the whole TM path in one launch (tm_tiny_kernel)
   const void* tiny_fn;
   int tiny_ctas, tiny_rows, tiny_smem;
@@ -523,7 +524,12 @@ ncc_status setup_tc(ncc_plan pl) {
   }
   pl->tc_nbi = ceil_div(h, tc::kHB);
   double best = 1e300;
+  const int force_wc = getenv("NCC_TC_WC") ? atoi(getenv("NCC_TC_WC")) : 0;  // sweeps / experiments
   for (int wc = tc::kWB; wc <= 128; wc *= 2) {
+    if (force_wc && wc != force_wc) {
+      if (wc >= w) break;
+      continue;
+    }
     const int nbj = ceil_div(w, wc);
     const int64_t per_seg = (int64_t)pl->tc_vtiles * pl->tc_nbi * nbj * p.batch;
     const int force_seg = getenv("NCC_TC_NSEG") ? atoi(getenv("NCC_TC_NSEG")) : 0;  // sweeps
@@ -566,6 +572,7 @@ ncc_status setup_tc(ncc_plan pl) {
   // chain inside tm_tc_kernel), chain flags, the CTA ticket counter
   if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) return st;
   pl->tc_ngrp = ceil_div(pl->tc_useg + tc::kHB - 1, tc::kG);
+  pl->tc_exp = getenv("NCC_TC_EXP") ? atoi(getenv("NCC_TC_EXP")) : 0;
   const size_t nflags = (size_t)p.batch * pl->tc_vtiles * pl->tc_nseg * pl->tc_ngrp * 4;
   if ((st = dalloc(&pl->tc_flags, nflags))) return st;
   NCC_CUDA(cudaMemset(pl->tc_flags, 0, nflags * sizeof(unsigned int)));
@@ -1074,17 +1081,17 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
         reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 1) & ~1), (p.image_w + 1) & ~1);
   };
-  // fork: template prep on the side stream.  Host path: the template's copy runs on the side
-  // stream ahead of its prep, concurrently with the frames' copy on the main stream; the side
-  // stream's only reader of the frames (the ragged-column kernel) waits for the frames' copy
-  // (ev_img) -- the main stream's kernels are ordered after it anyway.
+  // fork: template prep on the side stream.  Host path: the template's copy (small) goes first,
+  // then the frames' copy on the main stream runs beside the template prep; the side stream's
+  // only reader of the frames (the ragged-column kernel) waits for the frames' copy (ev_img) --
+  // the main stream's kernels are ordered after it anyway.
   mark(pl, s, 0);
-  NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
-  NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
-  if (pl->h_tmpl_in)
+  if (pl->h_tmpl_in)  // small: first on the copy engine, so the prep overlaps the frames' copy
     NCC_CUDA(cudaMemcpy2DAsync(const_cast<float*>(d_tmpl), tmpl_pitch * sizeof(float), pl->h_tmpl_in,
                                pl->h_tmpl_pitch * sizeof(float), p.tmpl_w * sizeof(float), p.tmpl_h,
-                               cudaMemcpyHostToDevice, pl->side));
+                               cudaMemcpyHostToDevice, s));
+  NCC_CUDA(cudaEventRecord(pl->ev_fork, s));
+  NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_fork, 0));
   if (pl->h_img_in) {
     NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
                              (size_t)batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
@@ -1158,6 +1165,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.score_frame_stride = (int64_t)pl->Ub * pl->V;
     t.keys = pl->keys;
     t.ssd = p.score == NCC_SCORE_SSD;
+    t.exp = pl->tc_exp;
     tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
     mark(pl, s, 3);

@@ -182,6 +182,7 @@ struct TcArgs {
   int64_t score_frame_stride;
   unsigned long long* keys;  // per-frame packed argmax keys
   int ssd;
+  int exp;  // timing experiments (NCC_TC_EXP; 0 in normal use): 1 no chain waits, 2 no drain work
 };
 
 __device__ __forceinline__ unsigned int ld_acquire_u32(const unsigned int* p) {
@@ -403,7 +404,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       for (int k = 0; k < kG; ++k) x[k] = __uint_as_float(d[k]);
       unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + wq;
       if (blk > 0) {
-        if (lane == 0) {
+        if (lane == 0 && !(a.exp & 1)) {
           for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
             if (it > (1ll << 28)) __trap();
         }
@@ -478,7 +479,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       st_wait();
       fence_before();
       mbar_arrive(&drained[gd % kGRing]);
-      if (!TC_EXP(32)) drain(gd, d);
+      if (!TC_EXP(32) && !(a.exp & 2)) drain(gd, d);
     }
   } else if (warp == kMmaWarp) {
     // ===================== MMA issuer (one thread)

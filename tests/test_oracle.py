@@ -357,3 +357,43 @@ def test_flat_threshold_relative_to_raw_energy():
     img = synth.uniform_image(12, 12, 39)
     assert np.all(oracle.ncc_surface(img, _checker(4, 4.0, 2.0 ** -15)) == 0.0)
     assert np.all(oracle.ncc_surface(img, _checker(4, 4.0, 2.0 ** -13)) != 0.0)
+
+
+# ---------------------------------------------------------------- SAD (Ch. 4 specialisation example)
+def test_sad_hand_case():
+    # case A windows are [[a,a+1],[a+3,a+4]] (a = 1,2,4,5) vs T = [[1,2],[3,4]]:
+    # T - W = [[1-a, 1-a], [-a, -a]] -> SAD = 2|1-a| + 2|a| = 2, 6, 14, 18
+    c = _cases()["case_A"]
+    s = oracle.sad_surface(np.array(c["image"], np.float32), np.array(c["template"], np.float32))
+    np.testing.assert_array_equal(s, np.array([[2.0, 6.0], [14.0, 18.0]]))
+
+
+def test_sad_invariants_and_bounds():
+    """SAD >= 0, = 0 at the plant, symmetric, invariant to a common shift, and bounded by the
+    SSD through Cauchy-Schwarz: SSD / max|T - W| <= SAD <= sqrt(n * SSD) (n = h w)."""
+    img, T, u0, v0 = synth.tm_inputs(1)
+    s, pk = oracle.sad_match(img, T)
+    assert s[u0, v0] == 0.0 and (pk.u, pk.v) == (u0, v0)
+    assert np.all(s >= 0.0)
+    g = synth.rng(46)
+    A = g.random((5, 7), dtype=np.float32)
+    B = g.random((5, 7), dtype=np.float32)
+    assert oracle.sad_surface(A, B)[0, 0] == oracle.sad_surface(B, A)[0, 0]
+    q = synth.quantize(img)
+    tq = synth.quantize(T)
+    np.testing.assert_array_equal(oracle.sad_surface(q + 2, tq + 2), oracle.sad_surface(q, tq))
+    sad = oracle.sad_surface(img, T)
+    ssd = oracle.ssd_surface(img, T)
+    n = T.size
+    assert np.all(sad <= np.sqrt(n * ssd) * (1 + 1e-12) + 1e-12)
+    d = np.abs(T.astype(np.float64) - img[3:19, 5:21].astype(np.float64))
+    assert ssd[3, 5] / d.max() <= sad[3, 5] * (1 + 1e-12)
+
+
+def test_piv_sad_planted_shift():
+    p = synth.particle_pair_integer(160, 176, 3, -4, seed=47)
+    v = oracle.piv_windows_sad(p.A, p.B, 32, 32, 8, 8, 16, 16, [1, 2, 3], [1, 4, 2])
+    assert np.all(v["iy"] == 3) and np.all(v["ix"] == -4) and np.all(v["score"] == 0.0)
+    # the sub-pixel step is the same minimum fit as SSD's (pinned above): at an exact integer
+    # shift the SAD surface is V-shaped around 0, the parabola's vertex stays within (-0.5, 0.5)
+    assert np.all(np.abs(v["dy"] - 3) < 0.5) and np.all(np.abs(v["dx"] + 4) < 0.5)
