@@ -61,8 +61,12 @@ enum { NCC_MODE_MATCH = 0, NCC_MODE_PIV = 1 };
 /* Score.  NCC: corr2 (Fig 5.1), peak = argmax.  SSD: sum (T - W)^2, the paper's own PIV
  * similarity score (Fig 5.10 caption), peak = argmin (tie -> smallest index);
  * computed from the same numerator as sum T^2 - 2 (sum A_C W + Tbar S1) + S2; PIV sub-pixel
- * for SSD is the 3-point parabola through the minimum; no flat-template flags for SSD. */
-enum { NCC_SCORE_NCC = 0, NCC_SCORE_SSD = 1 };
+ * for SSD is the 3-point parabola through the minimum; no flat-template flags for SSD.
+ * SAD: sum |T - W|, the metric the paper's specialisation example swaps for SSD (Ch. 4,
+ * P:1176-1179); peak = argmin, PIV sub-pixel as SSD; computed directly (no numerator /
+ * window-sum decomposition exists for |.|): CUDA-core kernels only, no ROI mode
+ * (NCC_ERR_UNSUPPORTED), no flat-template flags. */
+enum { NCC_SCORE_NCC = 0, NCC_SCORE_SSD = 1, NCC_SCORE_SAD = 2 };
 enum { NCC_SUBPIX_GAUSS3 = 0, NCC_SUBPIX_PARABOLA3 = 1, NCC_SUBPIX_NONE = 2 };
 
 /* ncc_problem.flags */

@@ -19,7 +19,7 @@ NCC_OK = 0
 STATUS = {0: "NCC_OK", 1: "NCC_ERR_INVALID_ARGUMENT", 2: "NCC_ERR_UNSUPPORTED", 3: "NCC_ERR_OUT_OF_MEMORY",
           4: "NCC_ERR_CUDA", 5: "NCC_ERR_COMPILE", 6: "NCC_ERR_WRONG_MODE"}
 NCC_MODE_MATCH, NCC_MODE_PIV = 0, 1
-NCC_SCORE_NCC, NCC_SCORE_SSD = 0, 1
+NCC_SCORE_NCC, NCC_SCORE_SSD, NCC_SCORE_SAD = 0, 1, 2
 NCC_SUBPIX_GAUSS3, NCC_SUBPIX_PARABOLA3, NCC_SUBPIX_NONE = 0, 1, 2
 NCC_F_WRITE_SURFACE, NCC_F_GENERIC_KERNEL, NCC_F_NO_JIT, NCC_F_TIMING, NCC_F_CUDA_CORES = 1, 2, 4, 8, 16
 FLAG_FLAT_TEMPLATE, FLAG_EDGE_Y, FLAG_EDGE_X, FLAG_PARABOLA_Y, FLAG_PARABOLA_X, FLAG_INVALID = 1, 2, 4, 8, 16, 32

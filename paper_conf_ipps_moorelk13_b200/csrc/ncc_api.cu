@@ -30,6 +30,7 @@
 #include "../../include/ncc.h"
 #include "ncc_kernels.cuh"
 #include "ncc_tc.cuh"
+#include "ncc_sad.cuh"
 
 using namespace nccb;
 
@@ -327,6 +328,7 @@ struct ncc_plan_s {
   unsigned long long* tc_ticket;  // CTA start tickets (monotonic)
   int tc_ngrp;
   int tc_exp;  // NCC_TC_EXP timing experiments (0 in normal use; results are wrong with bits set)
+  int sad, sad_smem;  // NCC_SCORE_SAD: the direct |t - b| kernels (ncc_sad.cuh), their dynamic smem
   // tiny problems: the whole TM path in one launch (tm_tiny_kernel)
   const void* tiny_fn;
   int tiny_ctas, tiny_rows, tiny_smem;
@@ -420,7 +422,7 @@ void free_plan(ncc_plan pl) {
 }
 
 ncc_status validate(const ncc_problem& p) {
-  if (p.score != NCC_SCORE_NCC && p.score != NCC_SCORE_SSD) return NCC_ERR_INVALID_ARGUMENT;
+  if (p.score != NCC_SCORE_NCC && p.score != NCC_SCORE_SSD && p.score != NCC_SCORE_SAD) return NCC_ERR_INVALID_ARGUMENT;
   if (p.mode != NCC_MODE_MATCH && p.mode != NCC_MODE_PIV) return NCC_ERR_INVALID_ARGUMENT;
   if (p.image_h <= 0 || p.image_w <= 0 || p.tmpl_h <= 0 || p.tmpl_w <= 0) return NCC_ERR_INVALID_ARGUMENT;
   if (p.image_pitch < p.image_w) return NCC_ERR_INVALID_ARGUMENT;
@@ -646,6 +648,30 @@ ncc_status setup_tiny(ncc_plan pl) {
   return NCC_OK;
 }
 
+// SAD (ncc_sad.cuh): no numerator / window-sum decomposition; one direct kernel (+ key reset and
+// peak).  Plain band matching only (no ROI / multi-template form).
+ncc_status setup_sad_tm(ncc_plan pl, int maxsm) {
+  const ncc_problem& p = pl->p;
+  if (pl->roi_mode || pl->n_tmpl != 1) return NCC_ERR_UNSUPPORTED;
+  const int w = p.tmpl_w;
+  const int64_t smem = ((int64_t)kSadCH * w + (int64_t)(kSadCH + kSadTU - 1) * (kSadTV + w - 1 + 3)) * 4;
+  if (smem > maxsm) return NCC_ERR_UNSUPPORTED;
+  NCC_CUDA(cudaFuncSetAttribute((const void*)tm_sad_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  pl->sad = 1;
+  pl->sad_smem = (int)smem;
+  ncc_plan_info& in = pl->info;
+  snprintf(in.variant_name, sizeof(in.variant_name), "tm_sad_%dx%d_rv%d", kSadTU, kSadTV, kSadRV);
+  fill_kernel_info(pl, (const void*)tm_sad_kernel, 256, (int)smem, ceil_div(pl->V, kSadTV), ceil_div(pl->Ub, kSadTU),
+                   p.batch);
+  in.specialized = 0;
+  in.variant_id = -1;
+  in.split = 1;
+  in.const_template = 0;
+  in.slabs = 1;
+  in.launches_per_call = 3;  // key reset, SAD, peak
+  return NCC_OK;
+}
+
 ncc_status create_tm(ncc_plan pl) {
   const ncc_problem& p = pl->p;
   const int h = p.tmpl_h, w = p.tmpl_w;
@@ -827,6 +853,7 @@ ncc_status create_tm(ncc_plan pl) {
     in.slabs = pl->n_slabs;
     in.launches_per_call = 2 + (pl->box_smem ? 1 : 2) + pl->n_slabs;  // prep, window sums, numerator(s), finalize
   }
+  if (p.score == NCC_SCORE_SAD) return setup_sad_tm(pl, maxsm);
   if ((st = setup_tiny(pl))) return st;
   if (pl->tiny_fn) return NCC_OK;
   return setup_tc(pl);
@@ -961,6 +988,19 @@ ncc_status create_piv(ncc_plan pl) {
   else
     fill_kernel_info(pl, v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
   in.launches_per_call = (pl->box_smem ? 2 : 3) * ceil_div(p.batch, sb);  // per sub-batch: window sums + PIV
+  if (p.score == NCC_SCORE_SAD) {  // direct |t - b| kernel, one CTA per (window, pair); no window sums
+    const int OY = 2 * my + 1, OX = 2 * mx + 1, OXP = ((OX + 3) / 4) * 4;
+    const int64_t smem = ((int64_t)h * w + (int64_t)(h + 2 * my) * (w + 2 * mx + 3) + (int64_t)OY * OXP) * 4;
+    if (smem > maxsm) return NCC_ERR_UNSUPPORTED;
+    NCC_CUDA(cudaFuncSetAttribute((const void*)piv_sad_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+    pl->sad = 1;
+    pl->sad_smem = (int)smem;
+    snprintf(in.variant_name, sizeof(in.variant_name), "piv_sad_%dx%d_m%dx%d", h, w, my, mx);
+    fill_kernel_info(pl, (const void*)piv_sad_kernel, 256, (int)smem, pl->Ky * pl->Kx, sb, 1);
+    in.specialized = 0;
+    in.variant_id = -1;
+    in.launches_per_call = ceil_div(p.batch, sb);
+  }
   return NCC_OK;
 }
 
@@ -1025,6 +1065,30 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     if (st) return st;
   }
   pl->timing_kind = 1;
+  if (pl->sad) {  // SAD: key reset, the direct kernel, peak (argmin)
+    mark(pl, s, 0);
+    if (pl->h_tmpl_in) {
+      NCC_CUDA(cudaMemcpy2DAsync(const_cast<float*>(d_tmpl), tmpl_pitch * sizeof(float), pl->h_tmpl_in,
+                                 pl->h_tmpl_pitch * sizeof(float), p.tmpl_w * sizeof(float), p.tmpl_h,
+                                 cudaMemcpyHostToDevice, s));
+      NCC_CUDA(cudaMemcpyAsync(const_cast<float*>(d_images), pl->h_img_in,
+                               (size_t)batch * p.image_h * p.image_pitch * sizeof(float), cudaMemcpyHostToDevice, s));
+    }
+    tm_keys_reset<<<ceil_div(batch, 128), 128, 0, s>>>(pl->keys, batch);
+    mark(pl, s, 1);
+    mark(pl, s, 2);
+    tm_sad_kernel<<<dim3(ceil_div(pl->V, kSadTV), ceil_div(pl->Ub, kSadTU), batch), 256, pl->sad_smem, s>>>(
+        d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_h, p.image_w, d_tmpl, tmpl_pitch,
+        p.tmpl_h, p.tmpl_w, pl->u_begin, pl->Ub, pl->V, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
+        (int64_t)pl->Ub * pl->V, pl->keys);
+    mark(pl, s, 3);
+    tm_finalize<<<ceil_div(batch, 128), 128, 0, s>>>(pl->keys, pl->tst, pl->V, reinterpret_cast<PeakOut*>(d_peaks),
+                                                     batch, 1, 1);
+    mark(pl, s, 4);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch (SAD)");
+    return NCC_OK;
+  }
   if (pl->tiny_fn) {  // the whole path in one launch
     mark(pl, s, 0);
     if (pl->h_tmpl_in) {
@@ -1332,6 +1396,17 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   for (int sb = 0; sb < nsub; ++sb) {
     const int p0 = sb * pl->sub_batch;
     const int np = (p0 + pl->sub_batch <= batch) ? pl->sub_batch : batch - p0;
+    if (pl->sad) {  // SAD: no window sums; frames of the sub-batch addressed from pair p0
+      PivArgs as = a;
+      as.A = A + p0 * fs;
+      as.B = B + p0 * fs;
+      as.pair0 = p0;
+      mark(pl, s, 3 * sb + 1);
+      piv_sad_kernel<<<dim3(pl->Ky * pl->Kx, np), 256, pl->sad_smem, s>>>(as);
+      mark(pl, s, 3 * sb + 2);
+      mark(pl, s, 3 * sb + 3);
+      continue;
+    }
     launch_box(pl, B + p0 * fs, np, 0, pl->map_h, s);
     mark(pl, s, 3 * sb + 1);
     a.pair0 = p0;

@@ -386,70 +386,22 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
     const int vv = v0 + wq * 32 + lane;
     const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
-    // Drain of row group gd (its MMAs are complete): output rows up = kG gd - kHB + 1 + k.
-    // Chain: block b > 0 waits until block b - 1 published the group's running numerator (this
-    // warp's 32 columns), adds its own; blocks b < nblk - 1 publish; the last block normalises
-    // (fp64 variance, fp32 rsqrt, as the CUDA-core path), writes the surface and folds the keys.
-    // Per output the order is ((p_0 + p_1) + p_2) + ... in block order: deterministic and
-    // independent of bands and segments.
-    auto drain = [&](int gd, const uint32_t (&d)[8]) {
-      const int up0 = gd * kG - kHB + 1;
-      if (up0 + kG <= 0 || up0 >= nu) return;  // ramp groups hold no output row of this CTA
-      const bool colok = vv < a.V;
-      const bool last_blk = blk == nblk - 1;
-      const int64_t rowbase = (int64_t)(ua - a.u_begin) * a.V + vv;  // CTA's first output row, this column
-      float* accf = a.acc + (int64_t)f * a.acc_frame_stride + rowbase;
-      float x[kG];
-#pragma unroll
-      for (int k = 0; k < kG; ++k) x[k] = __uint_as_float(d[k]);
-      unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + wq;
-      if (blk > 0) {
-        if (lane == 0 && !(a.exp & 1)) {
-          for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
-            if (it > (1ll << 28)) __trap();
-        }
-        __syncwarp();
-#pragma unroll
-        for (int k = 0; k < kG; ++k) {
-          const int up = up0 + k;
-          if (up >= 0 && up < nu && colok) x[k] = __ldcg(accf + (int64_t)up * a.V) + x[k];
-        }
-      }
-      if (!last_blk) {
-#pragma unroll
-        for (int k = 0; k < kG; ++k) {
-          const int up = up0 + k;
-          if (up >= 0 && up < nu && colok) __stcg(accf + (int64_t)up * a.V, x[k]);
-        }
-        __threadfence();
-        __syncwarp();
-        if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
-        return;
-      }
-      const TemplateStats ts = a.tst[0];
-      const double inv_n = 1.0 / ((double)a.h * (double)a.w);
-      const double* s1p = a.S1 + (int64_t)f * a.stat_frame_stride + rowbase;
-      const double* s2p = a.S2 + (int64_t)f * a.stat_frame_stride + rowbase;
-      float* scp = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + rowbase : nullptr;
-      unsigned long long best = 0ull;
-#pragma unroll
-      for (int k = 0; k < kG; ++k) {
-        const int up = up0 + k;
-        if (up >= 0 && up < nu && colok) {
-          const double s1 = __ldcg(s1p + (int64_t)up * a.V), s2 = __ldcg(s2p + (int64_t)up * a.V);
-          const float sc = a.ssd ? (float)(ts.sumsq - 2.0 * ((double)x[k] + ts.sum * inv_n * s1) + s2)
-                                 : ncc_normalize_fast(x[k], s1, s2, inv_n, ts.csum, ts.energy, ts.flat != 0);
-          if (scp) scp[(int64_t)up * a.V] = sc;
-          const unsigned long long key = make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)(ua + up) * a.V + vv));
-          best = key > best ? key : best;
-        }
-      }
-      best = warp_max_key(best);
-      if (lane == 0) {
-        if (best && best > __ldcg(a.keys + f)) atomicMax(a.keys + f, best);
-        if (blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
-      }
-    };
+    // Row group gd (its MMAs complete) holds output rows up = kG gd - kHB + 1 + k, k < kG.
+    // Chain: block b > 0 adds its values to the running numerator block b - 1 published for the
+    // group (this warp's 32 columns, per-warp flag); blocks b < nblk - 1 publish the new running
+    // value; the last block normalises (fp64 variance, fp32 rsqrt, as the CUDA-core path), writes
+    // the surface and folds the argmax keys.  Per output the order is ((p_0 + p_1) + p_2) + ...
+    // in block order: deterministic, independent of bands and segments.  The group's global
+    // inputs (the predecessor's running values, or the window sums) are loaded BEFORE waiting for
+    // its MMAs, all kG rows at once (clamped addresses), so their latency hides behind the MMAs.
+    const bool last_blk = blk == nblk - 1;
+    const bool colok = vv < a.V;
+    const int vc = colok ? vv : a.V - 1;
+    const int64_t colbase = (int64_t)(ua - a.u_begin) * a.V + vc;  // CTA's first output row, this column
+    float* accf = a.acc + (int64_t)f * a.acc_frame_stride + colbase;
+    const double* s1p = a.S1 + (int64_t)f * a.stat_frame_stride + colbase;
+    const double* s2p = a.S2 + (int64_t)f * a.stat_frame_stride + colbase;
+    const double inv_n = 1.0 / ((double)a.h * (double)a.w);
     int nrel = 0;
 #pragma unroll 1
     for (int gd = 0; gd < ngrp; ++gd) {
@@ -470,6 +422,30 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         mbar_arrive(&reloc_done);
         ++nrel;
       }
+      const int up0 = gd * kG - kHB + 1;
+      const bool has_rows = up0 + kG > 0 && up0 < nu && !TC_EXP(32) && !(a.exp & 2);
+      unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + wq;
+      float prev[kG];
+      double s1v[kG], s2v[kG];
+      if (has_rows) {
+        if (blk > 0) {
+          if (lane == 0 && !(a.exp & 1)) {
+            for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
+              if (it > (1ll << 28)) __trap();
+          }
+          __syncwarp();
+#pragma unroll
+          for (int k = 0; k < kG; ++k) prev[k] = __ldcg(accf + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V);
+        }
+        if (last_blk) {
+#pragma unroll
+          for (int k = 0; k < kG; ++k) {
+            const int64_t o = (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
+            s1v[k] = __ldcg(s1p + o);
+            s2v[k] = __ldcg(s2p + o);
+          }
+        }
+      }
       mbar_wait_bounded(&grp_done[gd % kGRing], (uint32_t)((gd / kGRing) & 1));
       fence_after();
       const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
@@ -479,7 +455,40 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       st_wait();
       fence_before();
       mbar_arrive(&drained[gd % kGRing]);
-      if (!TC_EXP(32) && !(a.exp & 2)) drain(gd, d);
+      if (!has_rows) continue;
+      float x[kG];
+#pragma unroll
+      for (int k = 0; k < kG; ++k) x[k] = blk > 0 ? prev[k] + __uint_as_float(d[k]) : __uint_as_float(d[k]);
+      if (!last_blk) {
+#pragma unroll
+        for (int k = 0; k < kG; ++k) {
+          const int up = up0 + k;
+          if (up >= 0 && up < nu && colok) __stcg(accf + (int64_t)up * a.V, x[k]);
+        }
+        __threadfence();
+        __syncwarp();
+        if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
+        continue;
+      }
+      const TemplateStats ts = a.tst[0];
+      float* scp = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + colbase : nullptr;
+      unsigned long long best = 0ull;
+#pragma unroll
+      for (int k = 0; k < kG; ++k) {
+        const int up = up0 + k;
+        const float sc = a.ssd ? (float)(ts.sumsq - 2.0 * ((double)x[k] + ts.sum * inv_n * s1v[k]) + s2v[k])
+                               : ncc_normalize_fast(x[k], s1v[k], s2v[k], inv_n, ts.csum, ts.energy, ts.flat != 0);
+        if (up >= 0 && up < nu && colok) {
+          if (scp) scp[(int64_t)up * a.V] = sc;
+          const unsigned long long key = make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)(ua + up) * a.V + vv));
+          best = key > best ? key : best;
+        }
+      }
+      best = warp_max_key(best);
+      if (lane == 0) {
+        if (best && best > __ldcg(a.keys + f)) atomicMax(a.keys + f, best);
+        if (blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
+      }
     }
   } else if (warp == kMmaWarp) {
     // ===================== MMA issuer (one thread)
