@@ -228,9 +228,20 @@ struct TmJitChoice {
   int RV, LX, WX, WY, CH, CW;
   bool ct;
 };
+// NCC_TM_JIT="RV,LX,WX,WY,CH,CW" forces a run-time specialised tile (the Tab 6.21 sensitivity
+// sweep, tools/sensitivity.py); the AOT instance for (h, w) is then skipped too.
+bool tm_jit_forced(TmJitChoice* c) {
+  const char* e = getenv("NCC_TM_JIT");
+  if (!e) return false;
+  int v[6];
+  if (sscanf(e, "%d,%d,%d,%d,%d,%d", &v[0], &v[1], &v[2], &v[3], &v[4], &v[5]) != 6) return false;
+  if (c) *c = TmJitChoice{v[0], v[1], v[2], v[3], v[4], v[5], false};
+  return true;
+}
 TmJitChoice tm_jit_choice(int h, int w) {
   static const int cw[] = {64, 32, 16}, ch[] = {32, 16};
   TmJitChoice c{12, 4, 1, 4, pick_chunk(h, ch, 2), pick_chunk(w, cw, 3), false};
+  tm_jit_forced(&c);
   const int WP = ((w + c.CW - 1) / c.CW) * c.CW;
   c.ct = (kConstTplFloats / WP) / c.CH * c.CH >= c.CH;
   return c;
@@ -241,25 +252,43 @@ struct PivJitChoice {
   int64_t win_fl;
   bool ok;
 };
-template <int CW>
-PivShape<12, CW> piv_shape(int h, int w, int my, int mx, int BP) { return PivShape<12, CW>(h, w, my, mx, BP, true); }
+// Run-time mirror of PivShape<RV, CW> (same formulas): items and per-window floats.
+struct PivShapeRT {
+  int items;
+  int64_t win_fl;
+};
+PivShapeRT piv_shape_rt(int RV, int CW, int h, int w, int my, int mx, int BP, bool alias) {
+  const int OY = 2 * my + 1, OX = 2 * mx + 1, OXP = ((OX + RV - 1) / RV) * RV;
+  const int TPP = ((w + CW - 1) / CW) * (CW + 2), BR = h + 2 * my;
+  const int64_t tp_fl = (((int64_t)h * TPP * 2 + 31) / 32) * 32, b_fl = (((int64_t)BR * BP + 31) / 32) * 32;
+  const int64_t s_fl = (((int64_t)OY * OXP + 31) / 32) * 32;
+  return PivShapeRT{OY * ((OX + RV - 1) / RV), (alias ? std::max(tp_fl, s_fl) : tp_fl + s_fl) + b_fl};
+}
 PivJitChoice piv_jit_choice(int h, int w, int my, int mx) {
   static const int cw[] = {64, 32, 16};
   PivJitChoice c{};
   c.RV = 12;
+  int force_wpb = 0;  // NCC_PIV_JIT="RV,WPB": the Tab 6.22 sensitivity sweep (data registers x threads)
+  if (const char* e = getenv("NCC_PIV_JIT")) {
+    int rv = 0, wpb = 0;
+    if (sscanf(e, "%d,%d", &rv, &wpb) == 2 && rv >= 4 && rv % 4 == 0 && wpb >= 1) {
+      c.RV = rv;
+      force_wpb = wpb;
+    }
+  }
   c.CW = pick_chunk(w, cw, 3);
-  const int OX = 2 * mx + 1, NG = (OX + 11) / 12;
-  c.BP = piv_pick_pitch(NG * 12 + ((w + c.CW - 1) / c.CW) * c.CW, 12, NG);
-  int items;
-  if (c.CW == 64) { auto ps = piv_shape<64>(h, w, my, mx, c.BP); items = ps.items; c.win_fl = ps.win_fl; }
-  else if (c.CW == 32) { auto ps = piv_shape<32>(h, w, my, mx, c.BP); items = ps.items; c.win_fl = ps.win_fl; }
-  else { auto ps = piv_shape<16>(h, w, my, mx, c.BP); items = ps.items; c.win_fl = ps.win_fl; }
+  const int OX = 2 * mx + 1, NG = (OX + c.RV - 1) / c.RV;
+  c.BP = piv_pick_pitch(NG * c.RV + ((w + c.CW - 1) / c.CW) * c.CW, c.RV, NG);
+  const PivShapeRT ps = piv_shape_rt(c.RV, c.CW, h, w, my, mx, c.BP, true);
+  const int items = ps.items;
+  c.win_fl = ps.win_fl;
   c.items = items;
   c.ok = false;
   if (items > 1024) return c;  // one item per thread (score tile aliased on the template pairs)
   const int64_t kTwoPerSm = 113 * 1024, kOnePerSm = 227 * 1024;
   double best = -1.0;
   for (int k = 1; k <= 4; ++k) {  // more windows per CTA blow up the per-window register arrays
+    if (force_wpb && k != force_wpb) continue;
     const int nt = ((k * items + 31) / 32) * 32;
     const int64_t smem = (int64_t)k * c.win_fl * 4;
     if (nt > 1024 || smem > kOnePerSm) break;
@@ -689,7 +718,7 @@ ncc_status create_tm(ncc_plan pl) {
   // variant selection (a8): AOT specialised instance > run-time specialised (NVRTC) > generic RE
   const TmVariant* v = &kTmVariants[0];
   bool aot = false;
-  if (!(p.flags & NCC_F_GENERIC_KERNEL))
+  if (!(p.flags & NCC_F_GENERIC_KERNEL) && !tm_jit_forced(nullptr))
     for (const TmVariant& c : kTmVariants)
       if (c.TH == h && c.TW == w) {
         v = &c;
@@ -872,7 +901,7 @@ ncc_status create_piv(ncc_plan pl) {
   // variant selection (a8): AOT specialised instance > run-time specialised (NVRTC) > generic RE
   const PivVariant* v = &kPivVariants[0];
   bool aot = false;
-  if (!(p.flags & NCC_F_GENERIC_KERNEL))
+  if (!(p.flags & NCC_F_GENERIC_KERNEL) && !getenv("NCC_PIV_JIT"))
     for (const PivVariant& c : kPivVariants)
       if (c.TH == h && c.TW == w && c.MY == my && c.MX == mx && !aot) {
         v = &c;  // first matching specialised instance is the default
@@ -916,21 +945,9 @@ ncc_status create_piv(ncc_plan pl) {
   (void)NG;
   const bool alias = v->ALIAS != 0;
   int items = 0;
-  const int64_t win_fl = [&] {
-    if (RV == 12 && CW == 16) {
-      PivShape<12, 16> ps(h, w, my, mx, pl->piv_bp, alias);
-      items = ps.items;
-      return (int64_t)ps.win_fl;
-    }
-    if (RV == 12 && CW == 32) {
-      PivShape<12, 32> ps(h, w, my, mx, pl->piv_bp, alias);
-      items = ps.items;
-      return (int64_t)ps.win_fl;
-    }
-    PivShape<12, 64> ps(h, w, my, mx, pl->piv_bp, alias);
-    items = ps.items;
-    return (int64_t)ps.win_fl;
-  }();
+  const PivShapeRT psr = piv_shape_rt(RV, CW, h, w, my, mx, pl->piv_bp, alias);
+  const int64_t win_fl = psr.win_fl;
+  items = psr.items;
   if (alias && (int64_t)items * v->WPB > (int64_t)v->NT * v->IPT) return NCC_ERR_UNSUPPORTED;
   pl->piv_smem = (int)(win_fl * 4 * v->WPB);
   int maxsm = 0;
