@@ -182,7 +182,8 @@ struct TcArgs {
   int64_t score_frame_stride;
   unsigned long long* keys;  // per-frame packed argmax keys
   int ssd;
-  int exp;  // timing experiments (NCC_TC_EXP; 0 in normal use): 1 no chain waits, 2 no drain work
+  int exp;  // timing experiments (NCC_TC_EXP; 0 in normal use): 1 no chain waits, 2 no drain work,
+            // 4 per-lane fence before the flag, 16 prefetch only (no chain / normalisation work)
 };
 
 __device__ __forceinline__ unsigned int ld_acquire_u32(const unsigned int* p) {
@@ -459,13 +460,16 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       float x[kG];
 #pragma unroll
       for (int k = 0; k < kG; ++k) x[k] = blk > 0 ? prev[k] + __uint_as_float(d[k]) : __uint_as_float(d[k]);
+      if (a.exp & 16) continue;  // experiment: no chain / normalisation work after the drain
       if (!last_blk) {
 #pragma unroll
         for (int k = 0; k < kG; ++k) {
           const int up = up0 + k;
           if (up >= 0 && up < nu && colok) __stcg(accf + (int64_t)up * a.V, x[k]);
         }
-        __threadfence();
+        // __syncwarp orders the lanes' stores before lane 0's release store of the flag
+        // (cumulativity); no per-lane fence needed
+        if (a.exp & 4) __threadfence();
         __syncwarp();
         if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
         continue;

@@ -10,10 +10,9 @@ run() {  # name, workload, env...
 run def2 cfg2
 run nowait2 cfg2 NCC_TC_EXP=1
 run nodrain2 cfg2 NCC_TC_EXP=2
-run wc64 cfg2 NCC_TC_WC=64
-run wc128 cfg2 NCC_TC_WC=128
+run fence2 cfg2 NCC_TC_EXP=4
+run prefonly2 cfg2 NCC_TC_EXP=16
 run def5 cfg5
-run nowait5 cfg5 NCC_TC_EXP=1
 run nodrain5 cfg5 NCC_TC_EXP=2
 python tools/timeline.py 2 > gpurun_out/timeline_cfg2.txt 2>&1
 for f in gpurun_out/exp_*.json; do python -c "
