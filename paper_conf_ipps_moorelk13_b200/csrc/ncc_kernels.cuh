@@ -1806,14 +1806,19 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
     fence_mbar_init();
   }
   __syncthreads();
-  const int ngroups = (nwin_total + WPS - 1) / WPS;
-  const int nlocal = (ngroups - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
-  // window wi of the k-th stage group of this CTA: pair (relative to pair0) and linear index
+  // Windows are dealt to the CTAs one at a time (CTA c: windows c, c + G, c + 2G, ...), so the
+  // CTAs' window counts differ by at most one and only their LAST stage is partly filled: at
+  // cfg 3 (3,721 windows, 148 CTAs, 4 per stage) every CTA runs 6 full stages + one of 1-2
+  // windows, instead of 43 CTAs running a 7th full stage while the others idle.
+  const int nmine = (nwin_total - (int)blockIdx.x + (int)gridDim.x - 1) / (int)gridDim.x;
+  const int nlocal = (nmine + WPS - 1) / WPS;
+  // window wi of the k-th stage of this CTA: pair (relative to pair0) and linear index
   auto win_of = [&](int k, int wi, int& lz, int& lin) {
-    const int wdx = ((int)blockIdx.x + k * (int)gridDim.x) * WPS + wi;
+    const int j = k * WPS + wi;
+    const int wdx = (int)blockIdx.x + j * (int)gridDim.x;
     lz = wdx / nwin;
     lin = wdx % nwin;
-    return wdx < nwin_total;
+    return j < nmine;
   };
   const double inv_n = 1.0 / ((double)TH * (double)TW);
 
