@@ -357,6 +357,7 @@ struct ncc_plan_s {
   unsigned long long* tc_ticket;  // CTA start tickets (monotonic)
   int tc_ngrp;
   int tc_exp;  // NCC_TC_EXP timing experiments (0 in normal use; results are wrong with bits set)
+  int tc_center;  // image operand centred on the template mean (NCC_TC_CENTER=0/1)
   int sad, sad_smem;  // NCC_SCORE_SAD: the direct |t - b| kernels (ncc_sad.cuh), their dynamic smem
   // tiny problems: the whole TM path in one launch (tm_tiny_kernel)
   const void* tiny_fn;
@@ -604,6 +605,7 @@ ncc_status setup_tc(ncc_plan pl) {
   if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) return st;
   pl->tc_ngrp = ceil_div(pl->tc_useg + tc::kHB - 1, tc::kG);
   pl->tc_exp = getenv("NCC_TC_EXP") ? atoi(getenv("NCC_TC_EXP")) : 0;
+  pl->tc_center = getenv("NCC_TC_CENTER") ? atoi(getenv("NCC_TC_CENTER")) : 0;
   const size_t nflags = (size_t)p.batch * pl->tc_vtiles * pl->tc_nseg * pl->tc_ngrp * 4;
   if ((st = dalloc(&pl->tc_flags, nflags))) return st;
   NCC_CUDA(cudaMemset(pl->tc_flags, 0, nflags * sizeof(unsigned int)));
@@ -1157,10 +1159,11 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     else if (jc <= 8) cols(tm_tc_cols<8>);
     else cols(tm_tc_cols_rw<16, RWN>);
   };
-  auto launch_split = [&]() {
-    tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, batch), 128, 0, s>>>(
+  auto launch_split = [&](cudaStream_t st) {
+    tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, batch), 128, 0, st>>>(
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
-        reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 1) & ~1), (p.image_w + 1) & ~1);
+        reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 1) & ~1), (p.image_w + 1) & ~1,
+        pl->tc_center ? pl->tst : nullptr, (double)p.tmpl_h * p.tmpl_w);
   };
   // fork: template prep on the side stream.  Host path: the template's copy (small) goes first,
   // then the frames' copy on the main stream runs beside the template prep; the side stream's
@@ -1191,6 +1194,10 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       tm_tc_tpl_prep<<<nblk_tc, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj,
                                                     pl->tcB);
   }
+  if (tc_now && pl->tc_center) {  // the centred split needs the template mean: after the prep
+    if (pl->h_img_in) NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_img, 0));
+    launch_split(pl->side);
+  }
   NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
   if (tc_now && pl->tc_sched == 3) {
     // the image split first (small: it leaves room for the template prep, which starts at once
@@ -1200,7 +1207,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       launch_cols();
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }
-    launch_split();
+    if (!pl->tc_center) launch_split(s);
     launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
@@ -1217,7 +1224,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
     const int nblk = nblk_tc;
-    if (pl->tc_sched != 3) launch_split();
+    if (pl->tc_sched != 3 && !pl->tc_center) launch_split(s);
     TcArgs t;
     t.H = p.image_h;
     t.W = p.image_w;
@@ -1247,6 +1254,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.keys = pl->keys;
     t.ssd = p.score == NCC_SCORE_SSD;
     t.exp = pl->tc_exp;
+    t.center = pl->tc_center;
     tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
     mark(pl, s, 3);

@@ -182,6 +182,7 @@ struct TcArgs {
   int64_t score_frame_stride;
   unsigned long long* keys;  // per-frame packed argmax keys
   int ssd;
+  int center;  // the image operand is centred on the template mean (tm_tc_split with ts)
   int exp;  // timing experiments (NCC_TC_EXP; 0 in normal use): 1 no chain waits, 2 no drain work,
             // 4 per-lane fence before the flag, 16 prefetch only (no chain / normalisation work)
 };
@@ -475,13 +476,26 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         continue;
       }
       const TemplateStats ts = a.tst[0];
+      // centred operand: sum A_C I = sum A_C (I - c) + c sum A_C
+      const double dc = a.center ? (double)tc_center(&ts, (double)a.h * (double)a.w) * ts.csum : 0.0;
       float* scp = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + colbase : nullptr;
       unsigned long long best = 0ull;
 #pragma unroll
       for (int k = 0; k < kG; ++k) {
         const int up = up0 + k;
-        const float sc = a.ssd ? (float)(ts.sumsq - 2.0 * ((double)x[k] + ts.sum * inv_n * s1v[k]) + s2v[k])
-                               : ncc_normalize_fast(x[k], s1v[k], s2v[k], inv_n, ts.csum, ts.energy, ts.flat != 0);
+        const double num = (double)x[k] + dc;
+        float sc;
+        if (a.ssd) {
+          sc = (float)(ts.sumsq - 2.0 * (num + ts.sum * inv_n * s1v[k]) + s2v[k]);
+        } else {  // as ncc_normalize_fast, from the fp64 numerator
+          const double var = s2v[k] - s1v[k] * s1v[k] * inv_n;
+          if (ts.flat || !(var > kFlatRel * s2v[k])) {
+            sc = 0.0f;
+          } else {
+            const float r = (float)(num - ts.csum * s1v[k] * inv_n) * rsqrtf((float)(ts.energy * var));
+            sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+          }
+        }
         if (up >= 0 && up < nu && colok) {
           if (scp) scp[(int64_t)up * a.V] = sc;
           const unsigned long long key = make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)(ua + up) * a.V + vv));
@@ -605,11 +619,19 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 // the producer warps load the Hankel elements directly (16-byte loads).  grid = (ceil(W/4/128), rows,
 // batch), block = 128; out row r = image row row0 + r, rows out_pitch (even: 16-byte TMA stride)
 // pairs apart.
+// With `ts` (centred operand): every element is first shifted by the template mean,
+// x = I - tc_center(ts, n) (fp32), so the accumulators hold sum A_C (I - c) -- sums without the
+// image's DC level -- and the epilogue adds c * sum A_C back (exact: tc_center is the same fp32
+// value there).  ts = nullptr: the raw image.
+__host__ __device__ __forceinline__ float tc_center(const TemplateStats* ts, double n) {
+  return ts ? (float)(ts->sum / n) : 0.0f;
+}
 __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
                                                    int W, int row0, uint2* __restrict__ out, int64_t out_frame_stride,
-                                                   int out_pitch) {
+                                                   int out_pitch, const TemplateStats* ts, double n) {
   const int c = (blockIdx.x * 128 + threadIdx.x) * 4;
   if (c >= W) return;
+  const float cen = tc_center(ts, n);
   const int r = blockIdx.y, f = blockIdx.z;
   const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch + c;
   uint2* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * out_pitch + c;
@@ -621,6 +643,8 @@ __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img
 #pragma unroll
     for (int k = 0; k < 4; ++k) x[k] = c + k < W ? __ldg(src + k) : 0.0f;
   }
+#pragma unroll
+  for (int k = 0; k < 4; ++k) x[k] = c + k < W ? x[k] - cen : 0.0f;
   uint2 o[4];
 #pragma unroll
   for (int k = 0; k < 4; ++k) {
