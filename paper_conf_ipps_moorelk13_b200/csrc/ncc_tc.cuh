@@ -187,6 +187,11 @@ struct TcArgs {
             // 4 per-lane fence before the flag, 16 prefetch only (no chain / normalisation work)
 };
 
+// Centring constant of the image operand: the template mean as an fp32 value (the same value in
+// tm_tc_split and in the epilogue's correction).
+__host__ __device__ __forceinline__ float tc_center(const TemplateStats* ts, double n) {
+  return ts ? (float)(ts->sum / n) : 0.0f;
+}
 __device__ __forceinline__ unsigned int ld_acquire_u32(const unsigned int* p) {
   unsigned int v;
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -623,9 +628,6 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 // x = I - tc_center(ts, n) (fp32), so the accumulators hold sum A_C (I - c) -- sums without the
 // image's DC level -- and the epilogue adds c * sum A_C back (exact: tc_center is the same fp32
 // value there).  ts = nullptr: the raw image.
-__host__ __device__ __forceinline__ float tc_center(const TemplateStats* ts, double n) {
-  return ts ? (float)(ts->sum / n) : 0.0f;
-}
 __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
                                                    int W, int row0, uint2* __restrict__ out, int64_t out_frame_stride,
                                                    int out_pitch, const TemplateStats* ts, double n) {
