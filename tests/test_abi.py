@@ -152,3 +152,22 @@ def test_python_binding_validates_buffers_before_the_c_abi():
         _check_template(big[:, ::2], "tmpl", 6, 6, None)  # column stride 2
     with pytest.raises(ValueError):
         _check_template(big, "tmpl", 7, 7, None)  # too few rows
+
+
+def test_sensitivity_surfaces_match_the_committed_sweep(tmp_path):
+    """EXPERIMENTS.md's Tab 6.21 / 6.22 surfaces are generated from profiles/r02_sensitivity.jsonl
+    (tools/sensitivity_md.py): regenerating them changes nothing; every built point was correct."""
+    import json
+    import shutil
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    src = os.path.join(root, "profiles", "r02_sensitivity.jsonl")
+    md = tmp_path / "EXPERIMENTS.md"
+    shutil.copy(os.path.join(root, "EXPERIMENTS.md"), md)
+    subprocess.run([sys.executable, os.path.join(root, "tools", "sensitivity_md.py"), src, str(md)], check=True)
+    assert md.read_text() == open(os.path.join(root, "EXPERIMENTS.md")).read()
+    rows = [json.loads(l) for l in open(src) if l.strip().startswith("{")]
+    built = [r for r in rows if "tflops" in r]
+    assert len(built) >= 40 and all(r["correct"] for r in built)
+    assert {r["table"] for r in built} == {"6.21", "6.22"}
