@@ -184,7 +184,7 @@ struct TcArgs {
   int ssd;
   int center;  // the image operand is centred on the template mean (tm_tc_split with ts)
   int exp;  // timing experiments (NCC_TC_EXP; 0 in normal use): 1 no chain waits, 2 no drain work,
-            // 4 per-lane fence before the flag, 16 prefetch only (no chain / normalisation work)
+            // 16 prefetch only (no chain / normalisation work)
 };
 
 // Centring constant of the image operand: the template mean as an fp32 value (the same value in
@@ -436,7 +436,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       double s1v[kG], s2v[kG];
       if (has_rows) {
         if (blk > 0) {
-          if (lane == 0 && !(a.exp & 1)) {
+          if (!(a.exp & 1)) {  // every lane acquires the flag itself (one broadcast load per poll)
             for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
               if (it > (1ll << 28)) __trap();
           }
@@ -473,9 +473,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           const int up = up0 + k;
           if (up >= 0 && up < nu && colok) __stcg(accf + (int64_t)up * a.V, x[k]);
         }
-        // __syncwarp orders the lanes' stores before lane 0's release store of the flag
-        // (cumulativity); no per-lane fence needed
-        if (a.exp & 4) __threadfence();
+        __threadfence();  // each lane's stores before the flag (the threadFenceReduction pattern)
         __syncwarp();
         if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
         continue;
