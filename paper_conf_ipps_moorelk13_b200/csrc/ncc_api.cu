@@ -358,6 +358,7 @@ struct ncc_plan_s {
   int tc_ngrp;
   int tc_exp;  // NCC_TC_EXP timing experiments (0 in normal use; results are wrong with bits set)
   int tc_center;  // image operand centred on the template mean (NCC_TC_CENTER=0/1)
+  unsigned long long* tc_prof;  // NCC_TC_EXP bit 32: per-CTA wait accounting (tools/tc_prof.py)
   int sad, sad_smem;  // NCC_SCORE_SAD: the direct |t - b| kernels (ncc_sad.cuh), their dynamic smem
   // tiny problems: the whole TM path in one launch (tm_tiny_kernel)
   const void* tiny_fn;
@@ -410,6 +411,17 @@ struct DeviceGuard {
 };
 
 void free_plan(ncc_plan pl) {
+  if (pl->tc_prof) {  // NCC_TC_EXP bit 32: the per-CTA accounting of the last call to NCC_TC_PROF_DUMP
+    if (const char* path = getenv("NCC_TC_PROF_DUMP")) {
+      const size_t n = (size_t)pl->tc_nbi * pl->tc_nbj * pl->tc_vtiles * pl->tc_nseg * pl->p.batch * 8;
+      std::vector<unsigned long long> h(n);
+      if (cudaMemcpy(h.data(), pl->tc_prof, n * 8, cudaMemcpyDeviceToHost) == cudaSuccess)
+        if (FILE* fp = fopen(path, "wb")) {
+          fwrite(h.data(), 8, n, fp);
+          fclose(fp);
+        }
+    }
+  }
   cudaFree(pl->tplC);
   cudaFree(pl->part);
   cudaFree(pl->cnt);
@@ -422,6 +434,7 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->tc_done);
   cudaFree(pl->tc_flags);
   cudaFree(pl->tc_ticket);
+  cudaFree(pl->tc_prof);
   cudaFree(pl->tiny_done);
   cudaFree(pl->tc_img2);
   cudaFree(pl->RS2);
@@ -606,6 +619,11 @@ ncc_status setup_tc(ncc_plan pl) {
   pl->tc_ngrp = ceil_div(pl->tc_useg + tc::kHB - 1, tc::kG);
   pl->tc_exp = getenv("NCC_TC_EXP") ? atoi(getenv("NCC_TC_EXP")) : 0;
   pl->tc_center = getenv("NCC_TC_CENTER") ? atoi(getenv("NCC_TC_CENTER")) : 0;
+  if (pl->tc_exp & 32) {
+    const size_t n = (size_t)nblk * pl->tc_vtiles * pl->tc_nseg * p.batch * 8;
+    if ((st = dalloc(&pl->tc_prof, n))) return st;
+    NCC_CUDA(cudaMemset(pl->tc_prof, 0, n * 8));
+  }
   const size_t nflags = (size_t)p.batch * pl->tc_vtiles * pl->tc_nseg * pl->tc_ngrp * 4;
   if ((st = dalloc(&pl->tc_flags, nflags))) return st;
   NCC_CUDA(cudaMemset(pl->tc_flags, 0, nflags * sizeof(unsigned int)));
@@ -1254,6 +1272,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.keys = pl->keys;
     t.ssd = p.score == NCC_SCORE_SSD;
     t.exp = pl->tc_exp;
+    t.prof = pl->tc_prof;
     t.center = pl->tc_center;
     tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);

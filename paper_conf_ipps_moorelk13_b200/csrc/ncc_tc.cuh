@@ -183,6 +183,7 @@ struct TcArgs {
   unsigned long long* keys;  // per-frame packed argmax keys
   int ssd;
   int center;  // the image operand is centred on the template mean (tm_tc_split with ts)
+  unsigned long long* prof;  // NCC_TC_EXP bit 32: per-CTA wait accounting [ticket][8] (globaltimer ns)
   int exp;  // timing experiments (NCC_TC_EXP; 0 in normal use): 1 no chain waits, 2 no drain work,
             // 16 prefetch only (no chain / normalisation work)
 };
@@ -191,6 +192,11 @@ struct TcArgs {
 // tm_tc_split and in the epilogue's correction).
 __host__ __device__ __forceinline__ float tc_center(const TemplateStats* ts, double n) {
   return ts ? (float)(ts->sum / n) : 0.0f;
+}
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
 }
 __device__ __forceinline__ unsigned int ld_acquire_u32(const unsigned int* p) {
   unsigned int v;
@@ -409,9 +415,13 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     const double* s1p = a.S1 + (int64_t)f * a.stat_frame_stride + colbase;
     const double* s2p = a.S2 + (int64_t)f * a.stat_frame_stride + colbase;
     const double inv_n = 1.0 / ((double)a.h * (double)a.w);
+    unsigned long long* prof = (a.exp & 32) && lane == 0 && wq == 1 ? a.prof + (int64_t)tk * 8 : nullptr;
+    unsigned long long p_flag = 0, p_grp = 0, p_work = 0, p_last = 0;
     int nrel = 0;
+    unsigned long long p_chain = 0;
 #pragma unroll 1
     for (int gd = 0; gd < ngrp; ++gd) {
+      if (prof && p_last) p_chain += gtimer() - p_last;
       if (gd > 0 && (gd * kG) % kRelocAt == 0) {
         // the MMA warp requests the relocation before group gd (all earlier MMAs complete, all
         // earlier groups drained by this warp): move the live columns to the front
@@ -434,12 +444,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + wq;
       float prev[kG];
       double s1v[kG], s2v[kG];
+      unsigned long long pt0 = prof ? gtimer() : 0ull;
       if (has_rows) {
         if (blk > 0) {
           if (!(a.exp & 1)) {  // every lane acquires the flag itself (one broadcast load per poll)
             for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
               if (it > (1ll << 28)) __trap();
           }
+          if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt0; pt0 = t; }
           __syncwarp();
 #pragma unroll
           for (int k = 0; k < kG; ++k) prev[k] = __ldcg(accf + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V);
@@ -453,7 +465,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           }
         }
       }
+      if (prof) pt0 = gtimer();
       mbar_wait_bounded(&grp_done[gd % kGRing], (uint32_t)((gd / kGRing) & 1));
+      if (prof) { const unsigned long long t = gtimer(); p_grp += t - pt0; pt0 = t; }
       fence_after();
       const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
       uint32_t d[8];
@@ -462,6 +476,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       st_wait();
       fence_before();
       mbar_arrive(&drained[gd % kGRing]);
+      if (prof) { const unsigned long long t = gtimer(); p_work += t - pt0; pt0 = t; p_last = t; }
       if (!has_rows) continue;
       float x[kG];
 #pragma unroll
@@ -511,6 +526,13 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         if (blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
       }
     }
+    if (prof) {
+      if (p_last) p_chain += gtimer() - p_last;
+      prof[2] = p_flag;
+      prof[3] = p_grp;
+      prof[4] = p_work;
+      prof[5] = p_chain;
+    }
   } else if (warp == kMmaWarp) {
     // ===================== MMA issuer (one thread)
     // Straight-line issue: the thread's scalar work per MMA is one 64-bit descriptor add and one
@@ -547,6 +569,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       // the accumulator column / instruction descriptor change once per group.
       const uint32_t full0 = smem_u32(&a_full[0]), done0 = smem_u32(&mma_done[0]);
       const uint32_t gdone0 = smem_u32(&grp_done[0]), drained0 = smem_u32(&drained[0]);
+      unsigned long long* mprof = (a.exp & 32) && lane == 0 ? a.prof + (int64_t)tk * 8 : nullptr;
+      unsigned long long m_drained = 0, m_afull = 0;
+      if (mprof) mprof[0] = gtimer();
       const bool leader = elect_one();
       if (nstage > 0 && !TC_EXP(16)) mbar_wait_u32(full0, 0u);
       fence_after();
@@ -566,7 +591,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           ++nrel_done;
         }
         if (g >= kGRing) {  // the window's newest columns were drained (and zeroed) after group g - kGRing
+          const unsigned long long t0 = mprof ? gtimer() : 0ull;
           mbar_wait_u32(drained0 + 8 * ((g - kGRing) % kGRing), (uint32_t)(((g - kGRing) / kGRing) & 1));
+          if (mprof) m_drained += gtimer() - t0;
           fence_after();
         }
         trim(g);
@@ -593,7 +620,11 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
             __syncwarp();
             const int bq = b;
             if (++b == kNBuf) { b = 0; ph ^= 1; }
-            if (q + 1 < nstage && !TC_EXP(16)) mbar_wait_u32(full0 + 8 * b, (uint32_t)ph);
+            if (q + 1 < nstage && !TC_EXP(16)) {
+              const unsigned long long t0 = mprof ? gtimer() : 0ull;
+              mbar_wait_u32(full0 + 8 * b, (uint32_t)ph);
+              if (mprof) m_afull += gtimer() - t0;
+            }
             if (!TC_EXP(16384)) fence_after();
             if (leader) {
               constexpr int kk = kWB / 8 - 1;
@@ -608,6 +639,11 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         }
         if (leader) commit_u32(gdone0 + 8 * (g % kGRing));  // group g's MMAs complete -> epilogue drains it
         __syncwarp();
+      }
+      if (mprof) {
+        mprof[1] = gtimer();
+        mprof[6] = m_drained;
+        mprof[7] = m_afull;
       }
     }
     __syncwarp();
