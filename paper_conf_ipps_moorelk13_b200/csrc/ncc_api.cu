@@ -569,7 +569,12 @@ ncc_status setup_tc(ncc_plan pl) {
   }
   pl->tc_nbi = ceil_div(h, tc::kHB);
   double best = 1e300;
-  const int force_wc = getenv("NCC_TC_WC") ? atoi(getenv("NCC_TC_WC")) : 0;  // sweeps / experiments
+  // WC = 32 unless forced (NCC_TC_WC, sweeps): the tensor cores' fp32 accumulation is biased
+  // (truncating) -- at a planted peak, where every product is positive, the relative error of a
+  // block's sum grows with its accumulation count (128 rows x WC/8 K-steps x 3): measured max
+  // |dNCC| 2.25e-5 at WC = 32 and 4.6e-5 at WC = 64 (tools/tc_error.py, cfg2 / cfg5), so the
+  // wider blocks would spend most of the 1e-4 budget.
+  const int force_wc = getenv("NCC_TC_WC") ? atoi(getenv("NCC_TC_WC")) : tc::kWB;
   for (int wc = tc::kWB; wc <= 128; wc *= 2) {
     if (force_wc && wc != force_wc) {
       if (wc >= w) break;

@@ -419,6 +419,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     unsigned long long p_flag = 0, p_grp = 0, p_work = 0, p_last = 0;
     int nrel = 0;
     unsigned long long p_chain = 0;
+    unsigned long long wbest = 0ull;  // last block: this lane's best key over its groups
 #pragma unroll 1
     for (int gd = 0; gd < ngrp; ++gd) {
       if (prof && p_last) p_chain += gtimer() - p_last;
@@ -520,11 +521,12 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           best = key > best ? key : best;
         }
       }
-      best = warp_max_key(best);
-      if (lane == 0) {
-        if (best && best > __ldcg(a.keys + f)) atomicMax(a.keys + f, best);
-        if (blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
-      }
+      wbest = best > wbest ? best : wbest;  // folded per lane; one atomic per warp at the end
+      if (lane == 0 && blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
+    }
+    if (last_blk) {
+      wbest = warp_max_key(wbest);
+      if (lane == 0 && wbest) atomicMax(a.keys + f, wbest);
     }
     if (prof) {
       if (p_last) p_chain += gtimer() - p_last;
