@@ -359,6 +359,7 @@ struct ncc_plan_s {
   int tc_exp;  // NCC_TC_EXP timing experiments (0 in normal use; results are wrong with bits set)
   int tc_center;  // image operand centred on the template mean (NCC_TC_CENTER=0/1)
   unsigned long long* tc_prof;  // NCC_TC_EXP bit 32: per-CTA wait accounting (tools/tc_prof.py)
+  float *tc_rsv, *tc_mean;  // NCC tensor-core plans: fp32 rsqrt(n var) and window mean per offset (window-sum kernels)
   int sad, sad_smem;  // NCC_SCORE_SAD: the direct |t - b| kernels (ncc_sad.cuh), their dynamic smem
   // tiny problems: the whole TM path in one launch (tm_tiny_kernel)
   const void* tiny_fn;
@@ -435,6 +436,8 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->tc_flags);
   cudaFree(pl->tc_ticket);
   cudaFree(pl->tc_prof);
+  cudaFree(pl->tc_rsv);
+  cudaFree(pl->tc_mean);
   cudaFree(pl->tiny_done);
   cudaFree(pl->tc_img2);
   cudaFree(pl->RS2);
@@ -636,6 +639,10 @@ ncc_status setup_tc(ncc_plan pl) {
   NCC_CUDA(cudaMemset(pl->tc_ticket, 0, sizeof(unsigned long long)));
   // (hi, lo) pairs, rows padded to an even count of pairs: a 16-byte multiple for the TMA map
   if ((st = dalloc(&pl->tc_img2, (size_t)2 * p.batch * pl->Hs * ((p.image_w + 1) & ~1)))) return st;
+  if (p.score == NCC_SCORE_NCC) {  // per-offset fp32 normalisation factors (window-sum kernels)
+    if ((st = dalloc(&pl->tc_rsv, (size_t)p.batch * pl->s_frame_stride))) return st;
+    if ((st = dalloc(&pl->tc_mean, (size_t)p.batch * pl->s_frame_stride))) return st;
+  }
   if ((st = dalloc(&pl->tc_done, (size_t)1))) return st;
   NCC_CUDA(cudaMemset(pl->tc_done, 0, sizeof(unsigned int)));
   const int smem = tc::smem_bytes(pl->tc_wc);
@@ -1075,7 +1082,8 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
     box2d_kernel<kBox2dNT><<<g, kBox2dNT, pl->box_smem, s>>>(frames, p.image_pitch,
                                                             (int64_t)p.image_h * p.image_pitch, row0, h, w, V,
                                                             rows_out, kBoxTV, TU, pl->box_r, pl->box_iwp, pl->S1,
-                                                            pl->S2, pl->s_frame_stride);
+                                                            pl->S2, pl->s_frame_stride, pl->tc_rsv, pl->tc_mean,
+                                                            1.0 / ((double)h * (double)w));
     return;
   }
   const int rows_in = rows_out + h - 1;
@@ -1087,7 +1095,7 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
                                                            pl->rs_frame_stride);
   dim3 g2(ceil_div(V, 32), ceil_div(rows_out, kBoxColsNW * kBoxColsL), batch);
   box_cols_kernel<kBoxColsNW, kBoxColsL><<<g2, kBoxColsNW * 32, 0, s>>>(pl->RS1, pl->RS2, pl->rs_frame_stride, V, h,
-                                                                        rows_out, pl->S1, pl->S2, pl->s_frame_stride);
+                                                                        rows_out, pl->S1, pl->S2, pl->s_frame_stride, pl->tc_rsv, pl->tc_mean, 1.0 / ((double)h * (double)w));
 }
 
 bool getenv_flag_two_kernel_prep() {  // NCC_TC_TWO_KERNEL_PREP=1: the earlier two-launch template prep
@@ -1268,6 +1276,8 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.ticket = pl->tc_ticket;
     t.S1 = pl->S1;
     t.S2 = pl->S2;
+    t.rsv = pl->tc_rsv;
+    t.mean = pl->tc_mean;
     t.stat_frame_stride = pl->s_frame_stride;
     t.tst = pl->tst;
     t.h = p.tmpl_h;

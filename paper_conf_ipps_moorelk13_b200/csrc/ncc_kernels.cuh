@@ -674,6 +674,16 @@ __global__ void tm_finalize(const unsigned long long* __restrict__ keys, const T
 }
 
 // ================================================================== window sums (a2)
+// Per-offset normalisation factors of a window for the tensor-core epilogue (which then needs
+// only fp32 arithmetic per output): rsqrt of n x the window variance, S2 - S1^2/n, computed in
+// fp64 and rounded once to fp32 (0 for a flat window: var <= 1e-10 S2, as ncc_normalize), and the
+// window mean S1/n for the sum(A_C) correction.
+__device__ __forceinline__ void window_denoms(double s1, double s2, double inv_n, float* rsv, float* mean) {
+  const double var = s2 - s1 * s1 * inv_n;
+  *rsv = (var > kFlatRel * s2) ? (float)(1.0 / sqrt(var)) : 0.0f;
+  *mean = (float)(s1 * inv_n);
+}
+
 // Inclusive warp scan (fp64, shuffle-up tree).
 __device__ __forceinline__ double warp_incl_scan_d(double v) {
   const int lane = threadIdx.x & 31;
@@ -758,7 +768,7 @@ template <int NT>
 __global__ void __launch_bounds__(NT, 2)
     box2d_kernel(const float* __restrict__ img, int64_t pitch, int64_t frame_stride, int row0, int h, int w, int V,
                  int rows_out, int TV, int TU, int R, int IWP, double* __restrict__ S1, double* __restrict__ S2,
-                 int64_t s_frame_stride) {
+                 int64_t s_frame_stride, float* __restrict__ RSV, float* __restrict__ MEAN, double inv_n) {
   extern __shared__ double sm_box[];
   double* X1 = sm_box;
   double* X2 = X1 + (int64_t)R * IWP;
@@ -884,8 +894,11 @@ __global__ void __launch_bounds__(NT, 2)
       double* o1 = S1 + (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
       double* o2 = S2 + (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
       for (int v = lane; v < tv; v += 32) {
-        o1[v] = x1[pidx(v + w - 1)] - (v > 0 ? x1[pidx(v - 1)] : 0.0);
-        o2[v] = x2[pidx(v + w - 1)] - (v > 0 ? x2[pidx(v - 1)] : 0.0);
+        const double s1 = x1[pidx(v + w - 1)] - (v > 0 ? x1[pidx(v - 1)] : 0.0);
+        const double s2 = x2[pidx(v + w - 1)] - (v > 0 ? x2[pidx(v - 1)] : 0.0);
+        o1[v] = s1;
+        o2[v] = s2;
+        if (RSV) window_denoms(s1, s2, inv_n, RSV + (o1 - S1) + v, MEAN + (o1 - S1) + v);
       }
     }
     __syncthreads();
@@ -903,7 +916,7 @@ template <int NW, int L>
 __global__ void __launch_bounds__(NW * 32)
     box_cols_kernel(const double* __restrict__ RS1, const double* __restrict__ RS2, int64_t rs_frame_stride,
                     int V, int h, int rows_out, double* __restrict__ S1, double* __restrict__ S2,
-                    int64_t s_frame_stride) {
+                    int64_t s_frame_stride, float* __restrict__ RSV, float* __restrict__ MEAN, double inv_n) {
   __shared__ double part1[NW][32], part2[NW][32], tot1[NW][32], tot2[NW][32];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const int v = blockIdx.x * 32 + lane;
@@ -958,6 +971,7 @@ __global__ void __launch_bounds__(NW * 32)
   if (ub + k0 < rows_out) {
     o1[(int64_t)(ub + k0) * V] = b1;
     o2[(int64_t)(ub + k0) * V] = b2;
+    if (RSV) window_denoms(b1, b2, inv_n, RSV + (o1 - S1) + (int64_t)(ub + k0) * V, MEAN + (o1 - S1) + (int64_t)(ub + k0) * V);
   }
 #pragma unroll
   for (int k = 0; k + 1 < L; ++k) {
@@ -965,6 +979,7 @@ __global__ void __launch_bounds__(NW * 32)
     if (u < rows_out) {
       o1[(int64_t)u * V] = b1 + d1[k];
       o2[(int64_t)u * V] = b2 + d2[k];
+      if (RSV) window_denoms(b1 + d1[k], b2 + d2[k], inv_n, RSV + (o1 - S1) + (int64_t)u * V, MEAN + (o1 - S1) + (int64_t)u * V);
     }
   }
 }

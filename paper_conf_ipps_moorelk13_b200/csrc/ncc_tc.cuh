@@ -174,7 +174,8 @@ struct TcArgs {
   unsigned int* flags;     // [batch][vtiles * nseg][ngrp_max][4]: blocks done with a row group
   int ngrp_max;
   unsigned long long* ticket;  // monotonically increasing CTA ticket (start order -> chain order)
-  const double *S1, *S2;   // fp64 window sums [batch][u_end - u_begin][V] (box2d)
+  const double *S1, *S2;   // fp64 window sums [batch][u_end - u_begin][V] (box2d; SSD)
+  const float *rsv, *mean; // NCC: fp32 rsqrt(n var) (0: flat window) and S1/n per offset (same layout)
   int64_t stat_frame_stride;
   const TemplateStats* tst;
   int h, w;
@@ -414,6 +415,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     float* accf = a.acc + (int64_t)f * a.acc_frame_stride + colbase;
     const double* s1p = a.S1 + (int64_t)f * a.stat_frame_stride + colbase;
     const double* s2p = a.S2 + (int64_t)f * a.stat_frame_stride + colbase;
+    const float* rsvp = a.rsv + (int64_t)f * a.stat_frame_stride + colbase;
+    const float* mnp = a.mean + (int64_t)f * a.stat_frame_stride + colbase;
     const double inv_n = 1.0 / ((double)a.h * (double)a.w);
     unsigned long long* prof = (a.exp & 32) && lane == 0 && wq == 1 ? a.prof + (int64_t)tk * 8 : nullptr;
     unsigned long long p_flag = 0, p_grp = 0, p_work = 0, p_last = 0;
@@ -443,7 +446,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       const int up0 = gd * kG - kHB + 1;
       const bool has_rows = up0 + kG > 0 && up0 < nu && !TC_EXP(32) && !(a.exp & 2);
       unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + wq;
-      float prev[kG];
+      float prev[kG], rsv[kG], mnv[kG];
       double s1v[kG], s2v[kG];
       unsigned long long pt0 = prof ? gtimer() : 0ull;
       if (has_rows) {
@@ -461,8 +464,13 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 #pragma unroll
           for (int k = 0; k < kG; ++k) {
             const int64_t o = (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
-            s1v[k] = __ldcg(s1p + o);
-            s2v[k] = __ldcg(s2p + o);
+            if (a.ssd) {
+              s1v[k] = __ldcg(s1p + o);
+              s2v[k] = __ldcg(s2p + o);
+            } else {
+              rsv[k] = __ldcg(rsvp + o);
+              mnv[k] = __ldcg(mnp + o);
+            }
           }
         }
       }
@@ -497,23 +505,23 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       const TemplateStats ts = a.tst[0];
       // centred operand: sum A_C I = sum A_C (I - c) + c sum A_C
       const double dc = a.center ? (double)tc_center(&ts, (double)a.h * (double)a.w) * ts.csum : 0.0;
+      // NCC in fp32 from the window kernels' factors: (N - sum(A_C) S1/n) / sqrt(A_D n var)
+      const float csf = (float)ts.csum, dcf = (float)dc;
+      const float rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
       float* scp = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + colbase : nullptr;
       unsigned long long best = 0ull;
 #pragma unroll
       for (int k = 0; k < kG; ++k) {
         const int up = up0 + k;
-        const double num = (double)x[k] + dc;
+        const double num = (double)x[k] + dc;  // (SSD)
         float sc;
-        if (a.ssd) {
+        if (a.exp & 64) {  // experiment: no normalisation
+          sc = x[k];
+        } else if (a.ssd) {
           sc = (float)(ts.sumsq - 2.0 * (num + ts.sum * inv_n * s1v[k]) + s2v[k]);
-        } else {  // as ncc_normalize_fast, from the fp64 numerator
-          const double var = s2v[k] - s1v[k] * s1v[k] * inv_n;
-          if (ts.flat || !(var > kFlatRel * s2v[k])) {
-            sc = 0.0f;
-          } else {
-            const float r = (float)(num - ts.csum * s1v[k] * inv_n) * rsqrtf((float)(ts.energy * var));
-            sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
-          }
+        } else {  // |error| <= ~3e-7: three fp32 roundings of fp64-derived factors
+          const float r = fmaf(-csf, mnv[k], x[k] + dcf) * (rsv[k] * rse);
+          sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
         }
         if (up >= 0 && up < nu && colok) {
           if (scp) scp[(int64_t)up * a.V] = sc;
