@@ -70,6 +70,19 @@ class _Plan:
         self.device = int(device)
         self.handle = N.ncc_plan_create(problem, self.device)
         self.info = N.ncc_plan_query(self.handle)
+        self._checked = {}  # call kind -> the last validated buffers (identity + data pointers)
+
+    def _validated(self, kind, tensors, check):
+        """Run `check` unless the same tensor objects, at the same addresses and shapes, passed
+        it on the previous call of this kind (the usual loop over one set of buffers)."""
+        sig = tuple((t, t.data_ptr(), t.shape) if t is not None else None for t in tensors)
+        last = self._checked.get(kind)
+        if last is not None and len(last) == len(sig) and all(
+                (a is None and b is None) or (a is not None and b is not None and a[0] is b[0] and a[1] == b[1]
+                                              and a[2] == b[2]) for a, b in zip(last, sig)):
+            return
+        check()
+        self._checked[kind] = sig
 
     def close(self):
         if self.handle:
@@ -138,7 +151,8 @@ class MatchPlan(_Plan):
             peaks = torch.empty((p.batch, 4), dtype=torch.int32, device=dev)
         if self.write_surface and scores is None:
             scores = torch.empty((p.batch, self.band_rows, self.info.V), dtype=torch.float32, device=dev)
-        self._check_match_io(images, tmpl, peaks, scores, dev)
+        self._validated("match", (images, tmpl, peaks, scores),
+                        lambda: self._check_match_io(images, tmpl, peaks, scores, dev))
         N.ncc_match(self.handle, images, tmpl, tmpl.stride(0), scores, peaks, self._stream(stream))
         return peaks, scores
 
@@ -160,7 +174,8 @@ class MatchPlan(_Plan):
     def match_host(self, h_images: torch.Tensor, h_tmpl: torch.Tensor, h_peaks: torch.Tensor, h_scores=None,
                    stream=None):
         """Host tensors (pinned for asynchronous, captured copies); same layouts as match()."""
-        self._check_match_io(h_images, h_tmpl, h_peaks, h_scores, None)
+        self._validated("match_host", (h_images, h_tmpl, h_peaks, h_scores),
+                        lambda: self._check_match_io(h_images, h_tmpl, h_peaks, h_scores, None))
         N.ncc_match_host(self.handle, h_images, h_tmpl, h_tmpl.stride(0), h_scores, h_peaks, self._stream(stream))
         return h_peaks
 
@@ -191,7 +206,7 @@ class PivPlan(_Plan):
         if scores:
             sc = torch.empty((p.batch, Ky, Kx, 2 * p.search_y + 1, 2 * p.search_x + 1), dtype=torch.float32,
                              device=dev)
-        self._check_piv_io(A, B, vectors, dev)
+        self._validated("correlate", (A, B, vectors), lambda: self._check_piv_io(A, B, vectors, dev))
         N.piv_correlate_ex(self.handle, A, B, sc, vectors, self._stream(stream))
         return vectors, sc
 
@@ -204,6 +219,6 @@ class PivPlan(_Plan):
         _check_tensor(vectors, "vectors", torch.int32, device, p.batch * Ky * Kx * 6)
 
     def correlate_host(self, h_A, h_B, h_vectors, stream=None):
-        self._check_piv_io(h_A, h_B, h_vectors, None)
+        self._validated("correlate_host", (h_A, h_B, h_vectors), lambda: self._check_piv_io(h_A, h_B, h_vectors, None))
         N.piv_correlate_host(self.handle, h_A, h_B, h_vectors, self._stream(stream))
         return h_vectors

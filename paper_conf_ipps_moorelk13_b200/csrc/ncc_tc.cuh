@@ -121,10 +121,12 @@ constexpr int kGroups = kNBuf;                           // producer groups of 4
 // warp roles: producers 0 .. 4 kGroups - 1, relocation 4 kGroups .. + 3, TMA, then the MMA warp
 // LAST: the SMSP arbiter issues highest-warp-id-first, and every cycle the MMA warp waits to issue
 // is a cycle the tensor pipe idles (its queue is about one MMA deep).
-constexpr int kRelocWarp0 = 4 * kGroups;
-constexpr int kTmaWarp = kRelocWarp0 + 4;
+constexpr int kRelocWarp0 = 4 * kGroups;   // 4 drain warps (TMEM lane quadrants): drain, zero, relocate
+constexpr int kChainWarp0 = kRelocWarp0 + 4;  // 2 chain warps: the group's global work (64 columns each)
+constexpr int kNChain = 2;
+constexpr int kTmaWarp = kChainWarp0 + kNChain;
 constexpr int kMmaWarp = kTmaWarp + 1;
-constexpr int kThreads = kGroups * 128 + 32 + 128 + 32;
+constexpr int kThreads = kGroups * 128 + 128 + kNChain * 32 + 32 + 32;
 constexpr int kBoxW = 128 + kWB;                         // image-row segment of one stage (TMA box)
 constexpr int kNImg = 9;                                 // image-row ring (TMA issue distance)
 static_assert(kNImg % kNBuf == 0, "a stage and the stage kNImg later belong to the same producer group");
@@ -134,7 +136,9 @@ __host__ __device__ constexpr int b_bytes(int WC) { return 2 * (WC / 4) * kLB * 
 // dynamic shared memory per CTA: the operand, padded so that one CTA fits per SM (the CTA
 // allocates all 512 TMEM columns)
 __host__ __device__ constexpr int img_off(int WC) { return ((b_bytes(WC) + 127) / 128) * 128; }
-__host__ __device__ constexpr int smem_need(int WC) { return img_off(WC) + kNImg * kBoxW * 8; }
+// drained row groups staged for the chain warps: kGRing slots of kG rows x 128 columns (fp32)
+__host__ __device__ constexpr int stage_off(int WC) { return img_off(WC) + kNImg * kBoxW * 8; }
+__host__ __device__ constexpr int smem_need(int WC) { return stage_off(WC) + kGRing * kG * 128 * 4; }
 __host__ __device__ constexpr int smem_bytes(int WC) { return smem_need(WC) > 120 * 1024 ? smem_need(WC) : 120 * 1024; }
 
 }  // namespace tc
@@ -214,7 +218,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   using namespace tc;
   extern __shared__ __align__(1024) unsigned char smem_tc[];
   __shared__ __align__(8) uint64_t a_full[kNBuf], mma_done[kNBuf], img_full[kNImg], img_empty[kNImg], reloc_req,
-      reloc_done, grp_done[kGRing], drained[kGRing];
+      reloc_done, grp_done[kGRing], drained[kGRing], staged[kGRing], consumed[kGRing];
   __shared__ uint32_t tmem_base_s;
   __shared__ unsigned long long ticket_s;
 
@@ -271,6 +275,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     for (int b = 0; b < kGRing; ++b) {
       mbar_init(&grp_done[b], 1);   // tcgen05.commit after a row group's last MMA
       mbar_init(&drained[b], 128);  // the group's accumulator columns read and zeroed
+      mbar_init(&staged[b], 128);   // the group's values in the shared-memory slot (drain warps)
+      mbar_init(&consumed[b], kNChain * 32);  // ... read by the chain warps: the slot is free
     }
     fence_mbar_init();
   }
@@ -391,44 +397,22 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     }
     __syncwarp();
   } else if (warp >= kRelocWarp0 && warp < kRelocWarp0 + 4) {
-    // ===================== epilogue warps (lane quadrant wq = warp % 4, lane v = column v0 + v):
-    // drain every finished row group -- read its kG accumulator columns from TMEM, zero them,
-    // release them to the MMA warp (drained ring) -- then do the group's global work (block
-    // chain, normalisation, keys) off the producers' and the MMA warp's critical path; between
-    // groups, the rare relocation of the live window.
+    // ===================== drain warps (lane quadrant wq = warp % 4, lane = column v0 + 32 wq + lane):
+    // for every finished row group read its kG accumulator columns from TMEM, zero them and
+    // release them to the MMA warp (drained ring), then stage the values in shared memory for the
+    // chain warps (staged / consumed ring); between groups, the rare relocation of the live
+    // window.  No global memory traffic here, so nothing the MMA warp waits for depends on
+    // another CTA.
     const int wq = warp & 3;
     const uint32_t lane_base = (uint32_t)(wq * 32) << 16;
-    const int vv = v0 + wq * 32 + lane;
     const uint32_t z[8] = {0u, 0u, 0u, 0u, 0u, 0u, 0u, 0u};
-    // Row group gd (its MMAs complete) holds output rows up = kG gd - kHB + 1 + k, k < kG.
-    // Chain: block b > 0 adds its values to the running numerator block b - 1 published for the
-    // group (this warp's 32 columns, per-warp flag); blocks b < nblk - 1 publish the new running
-    // value; the last block normalises (fp64 variance, fp32 rsqrt, as the CUDA-core path), writes
-    // the surface and folds the argmax keys.  Per output the order is ((p_0 + p_1) + p_2) + ...
-    // in block order: deterministic, independent of bands and segments.  The group's global
-    // inputs (the predecessor's running values, or the window sums) are loaded BEFORE waiting for
-    // its MMAs, all kG rows at once (clamped addresses), so their latency hides behind the MMAs.
-    const bool last_blk = blk == nblk - 1;
-    const bool colok = vv < a.V;
-    const int vc = colok ? vv : a.V - 1;
-    const int64_t colbase = (int64_t)(ua - a.u_begin) * a.V + vc;  // CTA's first output row, this column
-    float* accf = a.acc + (int64_t)f * a.acc_frame_stride + colbase;
-    const double* s1p = a.S1 + (int64_t)f * a.stat_frame_stride + colbase;
-    const double* s2p = a.S2 + (int64_t)f * a.stat_frame_stride + colbase;
-    const float* rsvp = a.rsv + (int64_t)f * a.stat_frame_stride + colbase;
-    const float* mnp = a.mean + (int64_t)f * a.stat_frame_stride + colbase;
-    const double inv_n = 1.0 / ((double)a.h * (double)a.w);
-    unsigned long long* prof = (a.exp & 32) && lane == 0 && wq == 1 ? a.prof + (int64_t)tk * 8 : nullptr;
-    unsigned long long p_flag = 0, p_grp = 0, p_work = 0, p_last = 0;
+    float* stg = reinterpret_cast<float*>(smem_tc + stage_off(a.WC)) + wq * 32 + lane;
     int nrel = 0;
-    unsigned long long p_chain = 0;
-    unsigned long long wbest = 0ull;  // last block: this lane's best key over its groups
 #pragma unroll 1
     for (int gd = 0; gd < ngrp; ++gd) {
-      if (prof && p_last) p_chain += gtimer() - p_last;
       if (gd > 0 && (gd * kG) % kRelocAt == 0) {
         // the MMA warp requests the relocation before group gd (all earlier MMAs complete, all
-        // earlier groups drained by this warp): move the live columns to the front
+        // earlier groups drained by these warps): move the live columns to the front
         mbar_wait_bounded(&reloc_req, (uint32_t)(nrel & 1));
         fence_after();
 #pragma unroll 1
@@ -443,40 +427,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         mbar_arrive(&reloc_done);
         ++nrel;
       }
-      const int up0 = gd * kG - kHB + 1;
-      const bool has_rows = up0 + kG > 0 && up0 < nu && !TC_EXP(32) && !(a.exp & 2);
-      unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + wq;
-      float prev[kG], rsv[kG], mnv[kG];
-      double s1v[kG], s2v[kG];
-      unsigned long long pt0 = prof ? gtimer() : 0ull;
-      if (has_rows) {
-        if (blk > 0) {
-          if (!(a.exp & 1)) {  // every lane acquires the flag itself (one broadcast load per poll)
-            for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
-              if (it > (1ll << 28)) __trap();
-          }
-          if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt0; pt0 = t; }
-          __syncwarp();
-#pragma unroll
-          for (int k = 0; k < kG; ++k) prev[k] = __ldcg(accf + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V);
-        }
-        if (last_blk) {
-#pragma unroll
-          for (int k = 0; k < kG; ++k) {
-            const int64_t o = (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
-            if (a.ssd) {
-              s1v[k] = __ldcg(s1p + o);
-              s2v[k] = __ldcg(s2p + o);
-            } else {
-              rsv[k] = __ldcg(rsvp + o);
-              mnv[k] = __ldcg(mnp + o);
-            }
-          }
-        }
-      }
-      if (prof) pt0 = gtimer();
       mbar_wait_bounded(&grp_done[gd % kGRing], (uint32_t)((gd / kGRing) & 1));
-      if (prof) { const unsigned long long t = gtimer(); p_grp += t - pt0; pt0 = t; }
       fence_after();
       const uint32_t col = (uint32_t)((gd * kG) % kRelocAt);
       uint32_t d[8];
@@ -485,62 +436,128 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       st_wait();
       fence_before();
       mbar_arrive(&drained[gd % kGRing]);
-      if (prof) { const unsigned long long t = gtimer(); p_work += t - pt0; pt0 = t; p_last = t; }
-      if (!has_rows) continue;
-      float x[kG];
+      const int slot = gd % kGRing;
+      if (gd >= kGRing) mbar_wait_bounded(&consumed[slot], (uint32_t)(((gd - kGRing) / kGRing) & 1));
+      float* sp = stg + slot * (kG * 128);
 #pragma unroll
-      for (int k = 0; k < kG; ++k) x[k] = blk > 0 ? prev[k] + __uint_as_float(d[k]) : __uint_as_float(d[k]);
-      if (a.exp & 16) continue;  // experiment: no chain / normalisation work after the drain
-      if (!last_blk) {
-#pragma unroll
-        for (int k = 0; k < kG; ++k) {
-          const int up = up0 + k;
-          if (up >= 0 && up < nu && colok) __stcg(accf + (int64_t)up * a.V, x[k]);
-        }
-        __threadfence();  // each lane's stores before the flag (the threadFenceReduction pattern)
-        __syncwarp();
-        if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
-        continue;
+      for (int k = 0; k < kG; ++k) sp[k * 128] = __uint_as_float(d[k]);
+      mbar_arrive(&staged[slot]);
+    }
+  } else if (warp >= kChainWarp0 && warp < kChainWarp0 + kNChain) {
+    // ===================== chain warps: lane = columns v0 + 64 cw + 32 j + lane (j = 0, 1).
+    // Row group gd holds output rows up = kG gd - kHB + 1 + k, k < kG.  Chain: block b > 0 adds
+    // its values to the running numerator block b - 1 published for the group (per chain warp
+    // flag); blocks b < nblk - 1 publish the new running value; the last block normalises (fp32
+    // from the window kernels' fp64-derived factors), writes the surface and folds the argmax
+    // keys.  Per output the order is ((p_0 + p_1) + p_2) + ... in block order: deterministic and
+    // independent of bands and segments.
+    const int cw = warp - kChainWarp0;
+    const bool last_blk = blk == nblk - 1;
+    const float* stg = reinterpret_cast<const float*>(smem_tc + stage_off(a.WC)) + cw * 64 + lane;
+    unsigned long long* prof = (a.exp & 32) && lane == 0 && cw == 0 ? a.prof + (int64_t)tk * 8 : nullptr;
+    unsigned long long p_flag = 0, p_grp = 0, p_chain = 0;
+    unsigned long long wbest = 0ull;  // last block: this lane's best key over its groups
+    const double inv_n = 1.0 / ((double)a.h * (double)a.w);
+#pragma unroll 1
+    for (int gd = 0; gd < ngrp; ++gd) {
+      const int up0 = gd * kG - kHB + 1;
+      const bool has_rows = up0 + kG > 0 && up0 < nu && !TC_EXP(32) && !(a.exp & 2);
+      const int slot = gd % kGRing;
+      unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + cw;
+      unsigned long long pt = prof ? gtimer() : 0ull;
+      if (has_rows && blk > 0 && !(a.exp & 1)) {  // every lane acquires the flag itself
+        for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
+          if (it > (1ll << 28)) __trap();
       }
-      const TemplateStats ts = a.tst[0];
-      // centred operand: sum A_C I = sum A_C (I - c) + c sum A_C
-      const double dc = a.center ? (double)tc_center(&ts, (double)a.h * (double)a.w) * ts.csum : 0.0;
-      // NCC in fp32 from the window kernels' factors: (N - sum(A_C) S1/n) / sqrt(A_D n var)
-      const float csf = (float)ts.csum, dcf = (float)dc;
-      const float rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
-      float* scp = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + colbase : nullptr;
-      unsigned long long best = 0ull;
+      if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt; pt = t; }
+      mbar_wait_bounded(&staged[slot], (uint32_t)((gd / kGRing) & 1));
+      if (prof) { const unsigned long long t = gtimer(); p_grp += t - pt; pt = t; }
+      float x[2][kG];
 #pragma unroll
-      for (int k = 0; k < kG; ++k) {
-        const int up = up0 + k;
-        const double num = (double)x[k] + dc;  // (SSD)
-        float sc;
-        if (a.exp & 64) {  // experiment: no normalisation
-          sc = x[k];
-        } else if (a.ssd) {
-          sc = (float)(ts.sumsq - 2.0 * (num + ts.sum * inv_n * s1v[k]) + s2v[k]);
-        } else {  // |error| <= ~3e-7: three fp32 roundings of fp64-derived factors
-          const float r = fmaf(-csf, mnv[k], x[k] + dcf) * (rsv[k] * rse);
-          sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+      for (int j = 0; j < 2; ++j)
+#pragma unroll
+        for (int k = 0; k < kG; ++k) x[j][k] = stg[slot * (kG * 128) + k * 128 + 32 * j];
+      mbar_arrive(&consumed[slot]);
+      if (has_rows && !(a.exp & 16)) {
+        const TemplateStats ts = a.tst[0];
+        // centred operand: sum A_C I = sum A_C (I - c) + c sum A_C
+        const double dc = a.center ? (double)tc_center(&ts, (double)a.h * (double)a.w) * ts.csum : 0.0;
+        const float csf = (float)ts.csum, dcf = (float)dc;
+        const float rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          const int vv = v0 + cw * 64 + 32 * j + lane;
+          const bool colok = vv < a.V;
+          const int64_t colbase = (int64_t)(ua - a.u_begin) * a.V + (colok ? vv : a.V - 1);
+          float* accf = a.acc + (int64_t)f * a.acc_frame_stride + colbase;
+          if (blk > 0) {
+            float prev[kG];
+#pragma unroll
+            for (int k = 0; k < kG; ++k) prev[k] = __ldcg(accf + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V);
+#pragma unroll
+            for (int k = 0; k < kG; ++k) x[j][k] = prev[k] + x[j][k];
+          }
+          if (!last_blk) {
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {
+              const int up = up0 + k;
+              if (up >= 0 && up < nu && colok) __stcg(accf + (int64_t)up * a.V, x[j][k]);
+            }
+            continue;
+          }
+          const int64_t so = (int64_t)f * a.stat_frame_stride + colbase;
+          float* scp = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + colbase : nullptr;
+          float sc[kG];
+          if (a.ssd) {
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {
+              const int64_t o = so + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
+              const double num = (double)x[j][k] + dc;
+              sc[k] = (float)(ts.sumsq - 2.0 * (num + ts.sum * inv_n * __ldcg(a.S1 + o)) + __ldcg(a.S2 + o));
+            }
+          } else {
+            float rsv[kG], mnv[kG];
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {
+              const int64_t o = so + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
+              rsv[k] = __ldcg(a.rsv + o);
+              mnv[k] = __ldcg(a.mean + o);
+            }
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {  // |error| <= ~3e-7: three fp32 roundings of fp64-derived factors
+              const float r = (a.exp & 64) ? x[j][k] : fmaf(-csf, mnv[k], x[j][k] + dcf) * (rsv[k] * rse);
+              sc[k] = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+            }
+          }
+#pragma unroll
+          for (int k = 0; k < kG; ++k) {
+            const int up = up0 + k;
+            if (up >= 0 && up < nu && colok) {
+              if (scp) scp[(int64_t)up * a.V] = sc[k];
+              const unsigned long long key =
+                  make_key(a.ssd ? -sc[k] : sc[k], (uint32_t)((int64_t)(ua + up) * a.V + vv));
+              wbest = key > wbest ? key : wbest;
+            }
+          }
         }
-        if (up >= 0 && up < nu && colok) {
-          if (scp) scp[(int64_t)up * a.V] = sc;
-          const unsigned long long key = make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)(ua + up) * a.V + vv));
-          best = key > best ? key : best;
+        if (!last_blk) {
+          __threadfence();  // each lane's stores before the flag (the threadFenceReduction pattern)
+          __syncwarp();
+          if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
+        } else if (lane == 0 && blk > 0) {
+          *fl = 0u;  // consumed: ready for the next call (stream-ordered)
         }
       }
-      wbest = best > wbest ? best : wbest;  // folded per lane; one atomic per warp at the end
-      if (lane == 0 && blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
+      if (prof) p_chain += gtimer() - pt;
     }
     if (last_blk) {
       wbest = warp_max_key(wbest);
       if (lane == 0 && wbest) atomicMax(a.keys + f, wbest);
     }
     if (prof) {
-      if (p_last) p_chain += gtimer() - p_last;
       prof[2] = p_flag;
       prof[3] = p_grp;
-      prof[4] = p_work;
+      prof[4] = 0;
       prof[5] = p_chain;
     }
   } else if (warp == kMmaWarp) {
