@@ -458,6 +458,17 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     unsigned long long p_flag = 0, p_grp = 0, p_chain = 0;
     unsigned long long wbest = 0ull;  // last block: this lane's best key over its groups
     const double inv_n = 1.0 / ((double)a.h * (double)a.w);
+    int vcol[2];
+    bool colok[2];
+    int64_t cb[2];  // offset of (the CTA's first output row, this column) in a frame's [Ub][V] planes
+#pragma unroll
+    for (int j = 0; j < 2; ++j) {
+      vcol[j] = v0 + cw * 64 + 32 * j + lane;
+      colok[j] = vcol[j] < a.V;
+      cb[j] = (int64_t)(ua - a.u_begin) * a.V + (colok[j] ? vcol[j] : a.V - 1);
+    }
+    float* accb = a.acc + (int64_t)f * a.acc_frame_stride;
+    const int64_t sfo = (int64_t)f * a.stat_frame_stride;
 #pragma unroll 1
     for (int gd = 0; gd < ngrp; ++gd) {
       const int up0 = gd * kG - kHB + 1;
@@ -470,6 +481,28 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           if (it > (1ll << 28)) __trap();
       }
       if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt; pt = t; }
+      // every global input of the group is requested before waiting for its staged values: the
+      // predecessor's running sums (both columns) and, in the last block, the normalisation factors
+      int64_t rowoff[kG];
+#pragma unroll
+      for (int k = 0; k < kG; ++k) rowoff[k] = (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
+      float prev[2][kG], fa[2][kG], fb[2][kG];
+      if (has_rows) {
+#pragma unroll
+        for (int j = 0; j < 2; ++j) {
+          if (blk > 0) {
+#pragma unroll
+            for (int k = 0; k < kG; ++k) prev[j][k] = __ldcg(accb + cb[j] + rowoff[k]);
+          }
+          if (last_blk && !a.ssd) {
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {
+              fa[j][k] = __ldcg(a.rsv + sfo + cb[j] + rowoff[k]);
+              fb[j][k] = __ldcg(a.mean + sfo + cb[j] + rowoff[k]);
+            }
+          }
+        }
+      }
       mbar_wait_bounded(&staged[slot], (uint32_t)((gd / kGRing) & 1));
       if (prof) { const unsigned long long t = gtimer(); p_grp += t - pt; pt = t; }
       float x[2][kG];
@@ -479,73 +512,51 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         for (int k = 0; k < kG; ++k) x[j][k] = stg[slot * (kG * 128) + k * 128 + 32 * j];
       mbar_arrive(&consumed[slot]);
       if (has_rows && !(a.exp & 16)) {
-        const TemplateStats ts = a.tst[0];
-        // centred operand: sum A_C I = sum A_C (I - c) + c sum A_C
-        const double dc = a.center ? (double)tc_center(&ts, (double)a.h * (double)a.w) * ts.csum : 0.0;
-        const float csf = (float)ts.csum, dcf = (float)dc;
-        const float rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
+        if (blk > 0) {
 #pragma unroll
-        for (int j = 0; j < 2; ++j) {
-          const int vv = v0 + cw * 64 + 32 * j + lane;
-          const bool colok = vv < a.V;
-          const int64_t colbase = (int64_t)(ua - a.u_begin) * a.V + (colok ? vv : a.V - 1);
-          float* accf = a.acc + (int64_t)f * a.acc_frame_stride + colbase;
-          if (blk > 0) {
-            float prev[kG];
+          for (int j = 0; j < 2; ++j)
 #pragma unroll
-            for (int k = 0; k < kG; ++k) prev[k] = __ldcg(accf + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V);
+            for (int k = 0; k < kG; ++k) x[j][k] = prev[j][k] + x[j][k];
+        }
+        if (!last_blk) {
 #pragma unroll
-            for (int k = 0; k < kG; ++k) x[j][k] = prev[k] + x[j][k];
-          }
-          if (!last_blk) {
+          for (int j = 0; j < 2; ++j)
 #pragma unroll
             for (int k = 0; k < kG; ++k) {
               const int up = up0 + k;
-              if (up >= 0 && up < nu && colok) __stcg(accf + (int64_t)up * a.V, x[j][k]);
+              if (up >= 0 && up < nu && colok[j]) __stcg(accb + cb[j] + (int64_t)up * a.V, x[j][k]);
             }
-            continue;
-          }
-          const int64_t so = (int64_t)f * a.stat_frame_stride + colbase;
-          float* scp = a.scores ? a.scores + (int64_t)f * a.score_frame_stride + colbase : nullptr;
-          float sc[kG];
-          if (a.ssd) {
-#pragma unroll
-            for (int k = 0; k < kG; ++k) {
-              const int64_t o = so + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
-              const double num = (double)x[j][k] + dc;
-              sc[k] = (float)(ts.sumsq - 2.0 * (num + ts.sum * inv_n * __ldcg(a.S1 + o)) + __ldcg(a.S2 + o));
-            }
-          } else {
-            float rsv[kG], mnv[kG];
-#pragma unroll
-            for (int k = 0; k < kG; ++k) {
-              const int64_t o = so + (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
-              rsv[k] = __ldcg(a.rsv + o);
-              mnv[k] = __ldcg(a.mean + o);
-            }
-#pragma unroll
-            for (int k = 0; k < kG; ++k) {  // |error| <= ~3e-7: three fp32 roundings of fp64-derived factors
-              const float r = (a.exp & 64) ? x[j][k] : fmaf(-csf, mnv[k], x[j][k] + dcf) * (rsv[k] * rse);
-              sc[k] = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
-            }
-          }
-#pragma unroll
-          for (int k = 0; k < kG; ++k) {
-            const int up = up0 + k;
-            if (up >= 0 && up < nu && colok) {
-              if (scp) scp[(int64_t)up * a.V] = sc[k];
-              const unsigned long long key =
-                  make_key(a.ssd ? -sc[k] : sc[k], (uint32_t)((int64_t)(ua + up) * a.V + vv));
-              wbest = key > wbest ? key : wbest;
-            }
-          }
-        }
-        if (!last_blk) {
           __threadfence();  // each lane's stores before the flag (the threadFenceReduction pattern)
           __syncwarp();
           if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
-        } else if (lane == 0 && blk > 0) {
-          *fl = 0u;  // consumed: ready for the next call (stream-ordered)
+        } else {
+          const TemplateStats ts = a.tst[0];
+          // centred operand: sum A_C I = sum A_C (I - c) + c sum A_C
+          const double dc = a.center ? (double)tc_center(&ts, (double)a.h * (double)a.w) * ts.csum : 0.0;
+          const float csf = (float)ts.csum, dcf = (float)dc;
+          const float rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            const int vv = vcol[j];
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {
+              float sc;
+              if (a.ssd) {
+                const double num = (double)x[j][k] + dc;
+                sc = (float)(ts.sumsq - 2.0 * (num + ts.sum * inv_n * __ldcg(a.S1 + sfo + cb[j] + rowoff[k])) + __ldcg(a.S2 + sfo + cb[j] + rowoff[k]));
+              } else {  // |error| <= ~3e-7: three fp32 roundings of fp64-derived factors
+                const float r = (a.exp & 64) ? x[j][k] : fmaf(-csf, fb[j][k], x[j][k] + dcf) * (fa[j][k] * rse);
+                sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+              }
+              const int up = up0 + k;
+              if (up >= 0 && up < nu && colok[j]) {
+                if (a.scores) a.scores[(int64_t)f * a.score_frame_stride + cb[j] + (int64_t)up * a.V] = sc;
+                const unsigned long long key = make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)(ua + up) * a.V + vv));
+                wbest = key > wbest ? key : wbest;
+              }
+            }
+          }
+          if (lane == 0 && blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
         }
       }
       if (prof) p_chain += gtimer() - pt;
