@@ -414,7 +414,7 @@ struct DeviceGuard {
 void free_plan(ncc_plan pl) {
   if (pl->tc_prof) {  // NCC_TC_EXP bit 32: the per-CTA accounting of the last call to NCC_TC_PROF_DUMP
     if (const char* path = getenv("NCC_TC_PROF_DUMP")) {
-      const size_t n = (size_t)pl->tc_nbi * pl->tc_nbj * pl->tc_vtiles * pl->tc_nseg * pl->p.batch * 8;
+      const size_t n = (size_t)pl->tc_nbi * pl->tc_nbj * pl->tc_vtiles * pl->tc_nseg * pl->p.batch * 8 + 512;
       std::vector<unsigned long long> h(n);
       if (cudaMemcpy(h.data(), pl->tc_prof, n * 8, cudaMemcpyDeviceToHost) == cudaSuccess)
         if (FILE* fp = fopen(path, "wb")) {
@@ -628,7 +628,7 @@ ncc_status setup_tc(ncc_plan pl) {
   pl->tc_exp = getenv("NCC_TC_EXP") ? atoi(getenv("NCC_TC_EXP")) : 0;
   pl->tc_center = getenv("NCC_TC_CENTER") ? atoi(getenv("NCC_TC_CENTER")) : 0;
   if (pl->tc_exp & 32) {
-    const size_t n = (size_t)nblk * pl->tc_vtiles * pl->tc_nseg * p.batch * 8;
+    const size_t n = (size_t)nblk * pl->tc_vtiles * pl->tc_nseg * p.batch * 8 + 512;  // + group traces
     if ((st = dalloc(&pl->tc_prof, n))) return st;
     NCC_CUDA(cudaMemset(pl->tc_prof, 0, n * 8));
   }
@@ -1021,6 +1021,10 @@ ncc_status create_piv(ncc_plan pl) {
   }
   if ((st = dalloc(&pl->S1, (size_t)sb * pl->s_frame_stride))) return st;
   if ((st = dalloc(&pl->S2, (size_t)sb * pl->s_frame_stride))) return st;
+  if (p.score == NCC_SCORE_NCC && pl->ws_smem) {  // fp32 normalisation factors for the WS kernels
+    if ((st = dalloc(&pl->tc_rsv, (size_t)sb * pl->s_frame_stride))) return st;
+    if ((st = dalloc(&pl->tc_mean, (size_t)sb * pl->s_frame_stride))) return st;
+  }
 
   ncc_plan_info& in = pl->info;
   in.U = pl->OY;
@@ -1430,6 +1434,8 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
   a.subpix = p.subpix;
   a.BP = pl->piv_bp;
   a.ssd = p.score == NCC_SCORE_SSD;
+  a.rsv = pl->tc_rsv;  // (only the warp-specialised kernels read them)
+  a.mean = pl->tc_mean;
   // TMA maps over all frames of the call (3D: cols, rows, pair); plain loads otherwise
   CUtensorMap mB;
   memset(&mB, 0, sizeof(mB));

@@ -999,6 +999,8 @@ struct PivArgs {
   int subpix;        // 0 Gauss3 (parabolic fallback), 1 parabola, 2 none
   int BP;            // RE: staged B pitch (floats), chosen on the host
   int ssd;           // 0: NCC (argmax), 1: SSD (argmin, parabolic fit of the minimum)
+  const float* rsv;  // NCC (nullable): fp32 rsqrt(n var) of frame B's windows (0: flat), S1/map layout
+  const float* mean; // ... and the window means S1/n
 };
 
 // FFMA2 numerator core with template PAIRS (sm_100a fma.rn.f32x2):
@@ -1892,15 +1894,27 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
         float* T = Sc(wi);
         float* gsc = a.scores ? a.scores + ((int64_t)(a.pair0 + lz) * nwin + lin) * tile : nullptr;
         unsigned long long bw = 0ull;
+        // NCC from the window kernel's fp32 factors (rsqrt(n var), S1/n; fp64-derived, rounded
+        // once): three fp32 roundings per score instead of fp64 loads and arithmetic
+        const bool fac = a.rsv != nullptr && !a.ssd;
+        const float* RVf = fac ? a.rsv + (S1f - a.S1) : nullptr;
+        const float* MNf = fac ? a.mean + (S1f - a.S1) : nullptr;
+        const float csf = (float)csum, rse = flat ? 0.0f : (float)(1.0 / sqrt(energy));
         for (int e0 = pt; e0 < tile; e0 += CH * NPT) {
           double w1[CH], w2[CH];
+          float f1[CH], f2[CH];
 #pragma unroll
           for (int c = 0; c < CH; ++c) {
             const int e = e0 + c * NPT;
             if (e < tile && !PIV_EXP(2)) {
               const int64_t mi = (int64_t)(e / S::OX) * a.map_pitch + e % S::OX;
-              w1[c] = __ldg(S1f + mi);
-              w2[c] = __ldg(S2f + mi);
+              if (fac) {
+                f1[c] = __ldg(RVf + mi);
+                f2[c] = __ldg(MNf + mi);
+              } else {
+                w1[c] = __ldg(S1f + mi);
+                w2[c] = __ldg(S2f + mi);
+              }
             }
           }
 #pragma unroll
@@ -1909,9 +1923,16 @@ __global__ void __launch_bounds__((NCW + NPW) * 32, 1)
             if (e < tile) {
               float* tp = T + (e / S::OX) * S::SP + e % S::OX;
               const float num = *tp;
-              const float sv = PIV_EXP(2) ? num
-                               : a.ssd ? (float)(tsq - 2.0 * ((double)num + tmean * w1[c]) + w2[c])
-                                       : ncc_normalize_fast(num, w1[c], w2[c], inv_n, csum, energy, flat);
+              float sv;
+              if (PIV_EXP(2)) {
+                sv = num;
+              } else if (fac) {
+                const float r = fmaf(-csf, f2[c], num) * (f1[c] * rse);
+                sv = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+              } else {
+                sv = a.ssd ? (float)(tsq - 2.0 * ((double)num + tmean * w1[c]) + w2[c])
+                           : ncc_normalize_fast(num, w1[c], w2[c], inv_n, csum, energy, flat);
+              }
               *tp = sv;
               if (gsc) gsc[e] = sv;
               const unsigned long long key = make_key(a.ssd ? -sv : sv, (uint32_t)e);

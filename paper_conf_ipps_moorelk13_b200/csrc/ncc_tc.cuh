@@ -559,7 +559,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           if (lane == 0 && blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
         }
       }
-      if (prof) p_chain += gtimer() - pt;
+      if (prof) {
+        const unsigned long long t = gtimer();
+        p_chain += t - pt;
+        if (tk < 4 && gd < 64) {  // per-group trace of the first tile's CTAs: [ticket][gd] chain done
+          unsigned long long* tr = a.prof + (int64_t)gridDim.x * gridDim.y * 8;
+          tr[tk * 64 + gd] = t;
+        }
+      }
     }
     if (last_blk) {
       wbest = warp_max_key(wbest);
@@ -568,7 +575,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     if (prof) {
       prof[2] = p_flag;
       prof[3] = p_grp;
-      prof[4] = 0;
+      prof[4] = gtimer();  // chain warps done (the CTA's end)
       prof[5] = p_chain;
     }
   } else if (warp == kMmaWarp) {
@@ -677,6 +684,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         }
         if (leader) commit_u32(gdone0 + 8 * (g % kGRing));  // group g's MMAs complete -> epilogue drains it
         __syncwarp();
+        if (mprof && tk < 4 && g < 64) a.prof[(int64_t)gridDim.x * gridDim.y * 8 + 256 + tk * 64 + g] = gtimer();
       }
       if (mprof) {
         mprof[1] = gtimer();

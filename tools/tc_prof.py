@@ -30,10 +30,12 @@ with MatchPlan(c["H"], c["W"], c["h"], c["w"]) as plan:
     torch.cuda.synchronize()
     name = plan.info.variant_name.decode()
     nblk = plan.info.split
-r = np.fromfile(dump, dtype=np.uint64).astype(np.int64).reshape(-1, 8)
+raw = np.fromfile(dump, dtype=np.uint64).astype(np.int64)
+trace = raw[-512:].reshape(2, 4, 64)  # [chain done | MMA group commit][ticket][group]
+r = raw[:-512].reshape(-1, 8)
 t0 = r[:, 0].min()
 out = {"variant": name, "ctas": len(r), "kernel_us": float((r[:, 1].max() - t0) / 1e3)}
-fields = ["start", "end", "epi_flag_wait", "epi_group_wait", "epi_drain", "epi_chain_work", "mma_drained_wait",
+fields = ["start", "end", "chain_flag_wait", "chain_staged_wait", "cta_end", "chain_work", "mma_drained_wait",
           "mma_afull_wait"]
 per = {}
 for b in range(nblk):
@@ -41,8 +43,11 @@ for b in range(nblk):
     d = {"start_us": float((rb[:, 0] - t0).mean() / 1e3), "end_us": float((rb[:, 1] - t0).mean() / 1e3),
          "end_max_us": float((rb[:, 1] - t0).max() / 1e3)}
     for i, f in enumerate(fields[2:], 2):
-        d[f + "_us"] = float(rb[:, i].mean() / 1e3)
+        d[f + "_us"] = float(((rb[:, i] - t0) if f == "cta_end" else rb[:, i]).mean() / 1e3)
     per[f"blk{b}"] = d
 out["per_block"] = per
+out["trace_tile0"] = {f"blk{b}": {"mma_commit_us": [round((x - t0) / 1e3, 1) if x else None for x in trace[1, b]],
+                                  "chain_done_us": [round((x - t0) / 1e3, 1) if x else None for x in trace[0, b]]}
+                      for b in range(min(4, nblk))}
 print(json.dumps(out, indent=1))
 os.remove(dump)
