@@ -457,6 +457,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     unsigned long long* prof = (a.exp & 32) && lane == 0 && cw == 0 ? a.prof + (int64_t)tk * 8 : nullptr;
     unsigned long long p_flag = 0, p_grp = 0, p_chain = 0;
     unsigned long long wbest = 0ull;  // last block: this lane's best key over its groups
+    int pending = -1;                 // group whose running sums are stored but not yet flagged
     const double inv_n = 1.0 / ((double)a.h * (double)a.w);
     int vcol[2];
     bool colok[2];
@@ -476,32 +477,48 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       const int slot = gd % kGRing;
       unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + cw;
       unsigned long long pt = prof ? gtimer() : 0ull;
-      if (has_rows && blk > 0 && !(a.exp & 1)) {  // every lane acquires the flag itself
-        for (long long it = 0; ld_acquire_u32(fl) < (unsigned)blk; ++it)
-          if (it > (1ll << 28)) __trap();
-      }
-      if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt; pt = t; }
-      // every global input of the group is requested before waiting for its staged values: the
-      // predecessor's running sums (both columns) and, in the last block, the normalisation factors
       int64_t rowoff[kG];
 #pragma unroll
       for (int k = 0; k < kG; ++k) rowoff[k] = (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
       float prev[2][kG], fa[2][kG], fb[2][kG];
-      if (has_rows) {
+      if (has_rows && last_blk && !a.ssd) {  // normalisation factors: no dependency, requested first
 #pragma unroll
-        for (int j = 0; j < 2; ++j) {
-          if (blk > 0) {
+        for (int j = 0; j < 2; ++j)
 #pragma unroll
-            for (int k = 0; k < kG; ++k) prev[j][k] = __ldcg(accb + cb[j] + rowoff[k]);
+          for (int k = 0; k < kG; ++k) {
+            fa[j][k] = __ldcg(a.rsv + sfo + cb[j] + rowoff[k]);
+            fb[j][k] = __ldcg(a.mean + sfo + cb[j] + rowoff[k]);
           }
-          if (last_blk && !a.ssd) {
-#pragma unroll
-            for (int k = 0; k < kG; ++k) {
-              fa[j][k] = __ldcg(a.rsv + sfo + cb[j] + rowoff[k]);
-              fb[j][k] = __ldcg(a.mean + sfo + cb[j] + rowoff[k]);
-            }
-          }
+      }
+      // Software-pipelined chain: the running sums of group gd - 1 were stored at the end of the
+      // previous iteration; their flag is published here, its fence overlapping the first poll of
+      // this group's predecessor flag (two L2 round trips per group instead of three).
+      auto publish_pending = [&]() {
+        if (pending >= 0) {
+          __threadfence();  // each lane's stores before the flag (the threadFenceReduction pattern)
+          __syncwarp();
+          if (lane == 0)
+            st_release_u32(a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + pending) * 4 + cw,
+                           (unsigned)(blk + 1));
+          pending = -1;
         }
+      };
+      if (has_rows && blk > 0 && !(a.exp & 1)) {  // every lane acquires the flag itself
+        unsigned int fv = ld_acquire_u32(fl);
+        publish_pending();
+        for (long long it = 0; fv < (unsigned)blk; ++it) {
+          if (it > (1ll << 28)) __trap();
+          fv = ld_acquire_u32(fl);
+        }
+      } else {
+        publish_pending();
+      }
+      if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt; pt = t; }
+      if (has_rows && blk > 0) {
+#pragma unroll
+        for (int j = 0; j < 2; ++j)
+#pragma unroll
+          for (int k = 0; k < kG; ++k) prev[j][k] = __ldcg(accb + cb[j] + rowoff[k]);
       }
       mbar_wait_bounded(&staged[slot], (uint32_t)((gd / kGRing) & 1));
       if (prof) { const unsigned long long t = gtimer(); p_grp += t - pt; pt = t; }
@@ -526,9 +543,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
               const int up = up0 + k;
               if (up >= 0 && up < nu && colok[j]) __stcg(accb + cb[j] + (int64_t)up * a.V, x[j][k]);
             }
-          __threadfence();  // each lane's stores before the flag (the threadFenceReduction pattern)
-          __syncwarp();
-          if (lane == 0) st_release_u32(fl, (unsigned)(blk + 1));
+          pending = gd;  // published at the start of the next iteration (or after the loop)
         } else {
           const TemplateStats ts = a.tst[0];
           // centred operand: sum A_C I = sum A_C (I - c) + c sum A_C
@@ -567,6 +582,13 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           tr[tk * 64 + gd] = t;
         }
       }
+    }
+    if (pending >= 0) {  // the last group's running sums
+      __threadfence();
+      __syncwarp();
+      if (lane == 0)
+        st_release_u32(a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + pending) * 4 + cw,
+                       (unsigned)(blk + 1));
     }
     if (last_blk) {
       wbest = warp_max_key(wbest);
