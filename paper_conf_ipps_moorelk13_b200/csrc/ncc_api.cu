@@ -351,10 +351,9 @@ struct ncc_plan_s {
   int tc_vcols;  // last output columns computed by tm_tc_cols (0: none)
   int tc_sched;  // 0: window sums || template prep, image split after them; 3 (default): image split,
                  // then window sums || template prep + ragged columns
-  float* tcB;              // reversed template-block operands
-  unsigned long long* tc_acc;  // running numerator {value, tag} (one plane)
-  unsigned int* tc_seq;    // call sequence number of the chain tags
+  float *tcB, *tc_acc;     // reversed template-block operands; running numerator (one plane)
   unsigned int* tc_done;   // finished tm_tc_tail CTAs (self-resetting)
+  unsigned int* tc_flags;  // chain flags [batch][vtiles * nseg][ngrp_max][4] (self-resetting)
   unsigned long long* tc_ticket;  // CTA start tickets (monotonic)
   int tc_ngrp;
   int tc_exp;  // NCC_TC_EXP timing experiments (0 in normal use; results are wrong with bits set)
@@ -434,7 +433,7 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->tcB);
   cudaFree(pl->tc_acc);
   cudaFree(pl->tc_done);
-  cudaFree(pl->tc_seq);
+  cudaFree(pl->tc_flags);
   cudaFree(pl->tc_ticket);
   cudaFree(pl->tc_prof);
   cudaFree(pl->tc_rsv);
@@ -625,12 +624,6 @@ ncc_status setup_tc(ncc_plan pl) {
   // one running-numerator plane whatever the number of template blocks (they accumulate in a
   // chain inside tm_tc_kernel), chain flags, the CTA ticket counter
   if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) return st;
-  NCC_CUDA(cudaMemset(pl->tc_acc, 0, (size_t)p.batch * pl->Ub * pl->V * 8));  // tag 0 = never valid (seq starts at 1)
-  if ((st = dalloc(&pl->tc_seq, (size_t)1))) return st;
-  {
-    const unsigned int one = 1u;
-    NCC_CUDA(cudaMemcpy(pl->tc_seq, &one, sizeof(one), cudaMemcpyHostToDevice));
-  }
   pl->tc_ngrp = ceil_div(pl->tc_useg + tc::kHB - 1, tc::kG);
   pl->tc_exp = getenv("NCC_TC_EXP") ? atoi(getenv("NCC_TC_EXP")) : 0;
   pl->tc_center = getenv("NCC_TC_CENTER") ? atoi(getenv("NCC_TC_CENTER")) : 0;
@@ -639,6 +632,9 @@ ncc_status setup_tc(ncc_plan pl) {
     if ((st = dalloc(&pl->tc_prof, n))) return st;
     NCC_CUDA(cudaMemset(pl->tc_prof, 0, n * 8));
   }
+  const size_t nflags = (size_t)p.batch * pl->tc_vtiles * pl->tc_nseg * pl->tc_ngrp * 4;
+  if ((st = dalloc(&pl->tc_flags, nflags))) return st;
+  NCC_CUDA(cudaMemset(pl->tc_flags, 0, nflags * sizeof(unsigned int)));
   if ((st = dalloc(&pl->tc_ticket, (size_t)1))) return st;
   NCC_CUDA(cudaMemset(pl->tc_ticket, 0, sizeof(unsigned long long)));
   // (hi, lo) pairs, rows padded to an even count of pairs: a 16-byte multiple for the TMA map
@@ -1279,7 +1275,8 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.vtiles = pl->tc_vtiles;
     t.acc = pl->tc_acc;
     t.acc_frame_stride = (int64_t)pl->Ub * pl->V;
-    t.seq = pl->tc_seq;
+    t.flags = pl->tc_flags;
+    t.ngrp_max = pl->tc_ngrp;
     t.ticket = pl->tc_ticket;
     t.S1 = pl->S1;
     t.S2 = pl->S2;
@@ -1304,8 +1301,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     tm_tc_tail<<<(unsigned)std::max<int64_t>(1, ceil_div(tail_items, 256)), 256, 0, s>>>(
         pl->tc_acc, (int64_t)pl->Ub * pl->V, pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V,
         pl->V - pl->tc_vcols, pl->u_begin, pl->Ub, batch, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
-        (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks),
-        pl->tc_seq);
+        (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks));
     mark(pl, s, 4);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch (tensor core)");

@@ -173,9 +173,10 @@ struct TcArgs {
   // partial planes, no summation kernel -- the paper's K2 global round trip, Figs 5.4-5.6, is
   // gone): block b > 0 adds its drained rows to the running numerator block b - 1 left in `acc`
   // (per-row-group, per-warp flags), the last block normalises them in the same drain.
-  unsigned long long* acc; // [batch][u_end - u_begin][V] running numerator {fp32 value, tag} (one plane)
+  float* acc;              // [batch][u_end - u_begin][V] running numerator (one plane)
   int64_t acc_frame_stride;
-  const unsigned int* seq; // call sequence number (incremented by tm_tc_tail after every call)
+  unsigned int* flags;     // [batch][vtiles * nseg][ngrp_max][4]: blocks done with a row group
+  int ngrp_max;
   unsigned long long* ticket;  // monotonically increasing CTA ticket (start order -> chain order)
   const double *S1, *S2;   // fp64 window sums [batch][u_end - u_begin][V] (box2d; SSD)
   const float *rsv, *mean; // NCC: fp32 rsqrt(n var) (0: flat window) and S1/n per offset (same layout)
@@ -201,19 +202,6 @@ __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
   return t;
-}
-__device__ __forceinline__ unsigned int ld_relaxed_u32(const unsigned int* p) {
-  unsigned int v;
-  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
-  unsigned long long v;
-  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-  return v;
-}
-__device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned long long v) {
-  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ unsigned int ld_acquire_u32(const unsigned int* p) {
   unsigned int v;
@@ -458,23 +446,19 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   } else if (warp >= kChainWarp0 && warp < kChainWarp0 + kNChain) {
     // ===================== chain warps: lane = columns v0 + 64 cw + 32 j + lane (j = 0, 1).
     // Row group gd holds output rows up = kG gd - kHB + 1 + k, k < kG.  Chain: block b > 0 adds
-    // its values to the running numerator block b - 1 published for the group; blocks
-    // b < nblk - 1 publish the new running value; the last block normalises (fp32 from the window
-    // kernels' fp64-derived factors), writes the surface and folds the argmax keys.  Per output the
-    // order is ((p_0 + p_1) + p_2) + ... in block order: deterministic and independent of bands
-    // and segments.  Protocol: every running value is one 64-bit word {fp32 value, tag = (call
-    // sequence << 8) | block}, stored and loaded relaxed at gpu scope (single-copy atomic), so the
-    // consumer's polling load IS the data load -- one L2 round trip per group, no flags, fences or
-    // resets (a word left by another call or block never carries the expected tag).
+    // its values to the running numerator block b - 1 published for the group (per chain warp
+    // flag); blocks b < nblk - 1 publish the new running value; the last block normalises (fp32
+    // from the window kernels' fp64-derived factors), writes the surface and folds the argmax
+    // keys.  Per output the order is ((p_0 + p_1) + p_2) + ... in block order: deterministic and
+    // independent of bands and segments.
     const int cw = warp - kChainWarp0;
     const bool last_blk = blk == nblk - 1;
     const float* stg = reinterpret_cast<const float*>(smem_tc + stage_off(a.WC)) + cw * 64 + lane;
     unsigned long long* prof = (a.exp & 32) && lane == 0 && cw == 0 ? a.prof + (int64_t)tk * 8 : nullptr;
     unsigned long long p_flag = 0, p_grp = 0, p_chain = 0;
     unsigned long long wbest = 0ull;  // last block: this lane's best key over its groups
+    int pending = -1;                 // group whose running sums are stored but not yet flagged
     const double inv_n = 1.0 / ((double)a.h * (double)a.w);
-    const uint32_t seq = ld_relaxed_u32(a.seq);
-    const uint32_t tag_in = (seq << 8) | (uint32_t)((blk - 1) & 0xFF), tag_out = (seq << 8) | (uint32_t)(blk & 0xFF);
     int vcol[2];
     bool colok[2];
     int64_t cb[2];  // offset of (the CTA's first output row, this column) in a frame's [Ub][V] planes
@@ -484,21 +468,18 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       colok[j] = vcol[j] < a.V;
       cb[j] = (int64_t)(ua - a.u_begin) * a.V + (colok[j] ? vcol[j] : a.V - 1);
     }
-    unsigned long long* accb = a.acc + (int64_t)f * a.acc_frame_stride;
+    float* accb = a.acc + (int64_t)f * a.acc_frame_stride;
     const int64_t sfo = (int64_t)f * a.stat_frame_stride;
 #pragma unroll 1
     for (int gd = 0; gd < ngrp; ++gd) {
       const int up0 = gd * kG - kHB + 1;
       const bool has_rows = up0 + kG > 0 && up0 < nu && !TC_EXP(32) && !(a.exp & 2);
       const int slot = gd % kGRing;
+      unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + cw;
       unsigned long long pt = prof ? gtimer() : 0ull;
       int64_t rowoff[kG];
-      bool rowok[kG];
 #pragma unroll
-      for (int k = 0; k < kG; ++k) {
-        rowoff[k] = (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
-        rowok[k] = up0 + k >= 0 && up0 + k < nu;
-      }
+      for (int k = 0; k < kG; ++k) rowoff[k] = (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
       float prev[2][kG], fa[2][kG], fb[2][kG];
       if (has_rows && last_blk && !a.ssd) {  // normalisation factors: no dependency, requested first
 #pragma unroll
@@ -509,29 +490,36 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
             fb[j][k] = __ldcg(a.mean + sfo + cb[j] + rowoff[k]);
           }
       }
-      if (has_rows && blk > 0) {  // the predecessor's running values: poll until every word carries its tag
+      // Software-pipelined chain: the running sums of group gd - 1 were stored at the end of the
+      // previous iteration; their flag is published here, its fence overlapping the first poll of
+      // this group's predecessor flag (two L2 round trips per group instead of three).
+      auto publish_pending = [&]() {
+        if (pending >= 0) {
+          __threadfence();  // each lane's stores before the flag (the threadFenceReduction pattern)
+          __syncwarp();
+          if (lane == 0)
+            st_release_u32(a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + pending) * 4 + cw,
+                           (unsigned)(blk + 1));
+          pending = -1;
+        }
+      };
+      if (has_rows && blk > 0 && !(a.exp & 1)) {  // every lane acquires the flag itself
+        unsigned int fv = ld_acquire_u32(fl);
+        publish_pending();
+        for (long long it = 0; fv < (unsigned)blk; ++it) {
+          if (it > (1ll << 28)) __trap();
+          fv = ld_acquire_u32(fl);
+        }
+      } else {
+        publish_pending();
+      }
+      if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt; pt = t; }
+      if (has_rows && blk > 0) {
 #pragma unroll
         for (int j = 0; j < 2; ++j)
 #pragma unroll
-          for (int k = 0; k < kG; ++k) prev[j][k] = 0.0f;
-        bool ready = false;
-        for (long long it = 0; !ready; ++it) {
-          if (it > (1ll << 26)) __trap();
-          ready = true;
-#pragma unroll
-          for (int j = 0; j < 2; ++j)
-#pragma unroll
-            for (int k = 0; k < kG; ++k) {
-              if (rowok[k] && colok[j]) {
-                const unsigned long long wv = ld_relaxed_u64(accb + cb[j] + rowoff[k]);
-                if ((uint32_t)(wv >> 32) == tag_in || (a.exp & 1)) prev[j][k] = __uint_as_float((uint32_t)wv);
-                else ready = false;
-              }
-            }
-          ready = __all_sync(0xffffffffu, ready);
-        }
+          for (int k = 0; k < kG; ++k) prev[j][k] = __ldcg(accb + cb[j] + rowoff[k]);
       }
-      if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt; pt = t; }
       mbar_wait_bounded(&staged[slot], (uint32_t)((gd / kGRing) & 1));
       if (prof) { const unsigned long long t = gtimer(); p_grp += t - pt; pt = t; }
       float x[2][kG];
@@ -551,10 +539,11 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 #pragma unroll
           for (int j = 0; j < 2; ++j)
 #pragma unroll
-            for (int k = 0; k < kG; ++k)
-              if (rowok[k] && colok[j])
-                st_relaxed_u64(accb + cb[j] + rowoff[k],
-                               ((unsigned long long)tag_out << 32) | __float_as_uint(x[j][k]));
+            for (int k = 0; k < kG; ++k) {
+              const int up = up0 + k;
+              if (up >= 0 && up < nu && colok[j]) __stcg(accb + cb[j] + (int64_t)up * a.V, x[j][k]);
+            }
+          pending = gd;  // published at the start of the next iteration (or after the loop)
         } else {
           const TemplateStats ts = a.tst[0];
           // centred operand: sum A_C I = sum A_C (I - c) + c sum A_C
@@ -569,20 +558,20 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
               float sc;
               if (a.ssd) {
                 const double num = (double)x[j][k] + dc;
-                sc = (float)(ts.sumsq - 2.0 * (num + ts.sum * inv_n * __ldcg(a.S1 + sfo + cb[j] + rowoff[k])) +
-                             __ldcg(a.S2 + sfo + cb[j] + rowoff[k]));
+                sc = (float)(ts.sumsq - 2.0 * (num + ts.sum * inv_n * __ldcg(a.S1 + sfo + cb[j] + rowoff[k])) + __ldcg(a.S2 + sfo + cb[j] + rowoff[k]));
               } else {  // |error| <= ~3e-7: three fp32 roundings of fp64-derived factors
                 const float r = (a.exp & 64) ? x[j][k] : fmaf(-csf, fb[j][k], x[j][k] + dcf) * (fa[j][k] * rse);
                 sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
               }
-              if (rowok[k] && colok[j]) {
-                if (a.scores) a.scores[(int64_t)f * a.score_frame_stride + cb[j] + rowoff[k]] = sc;
-                const unsigned long long key =
-                    make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)(ua + up0 + k) * a.V + vv));
+              const int up = up0 + k;
+              if (up >= 0 && up < nu && colok[j]) {
+                if (a.scores) a.scores[(int64_t)f * a.score_frame_stride + cb[j] + (int64_t)up * a.V] = sc;
+                const unsigned long long key = make_key(a.ssd ? -sc : sc, (uint32_t)((int64_t)(ua + up) * a.V + vv));
                 wbest = key > wbest ? key : wbest;
               }
             }
           }
+          if (lane == 0 && blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
         }
       }
       if (prof) {
@@ -593,6 +582,13 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           tr[tk * 64 + gd] = t;
         }
       }
+    }
+    if (pending >= 0) {  // the last group's running sums
+      __threadfence();
+      __syncwarp();
+      if (lane == 0)
+        st_release_u32(a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + pending) * 4 + cw,
+                       (unsigned)(blk + 1));
     }
     if (last_blk) {
       wbest = warp_max_key(wbest);
@@ -777,8 +773,8 @@ __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img
 template <int JC>  // JC = ceil(w / 32) template columns per lane
 __global__ void __launch_bounds__(256) tm_tc_cols(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
                                                   const float* __restrict__ tplC, int tplP, int h, int w, int v_lo,
-                                                  int V, int u_begin, int Ub, int batch,
-                                                  unsigned long long* __restrict__ acc, int64_t acc_frame_stride) {
+                                                  int V, int u_begin, int Ub, int batch, float* __restrict__ acc,
+                                                  int64_t acc_frame_stride) {
   const int nc = V - v_lo;
   const int64_t item = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (item >= (int64_t)batch * Ub * nc) return;
@@ -810,7 +806,7 @@ __global__ void __launch_bounds__(256) tm_tc_cols(const float* __restrict__ img,
   }
 #pragma unroll
   for (int d = 16; d; d >>= 1) tot += __shfl_xor_sync(0xffffffffu, tot, d);
-  if (lane == 0) acc[(int64_t)f * acc_frame_stride + (int64_t)ur * V + v_lo + c] = __float_as_uint(tot);
+  if (lane == 0) acc[(int64_t)f * acc_frame_stride + (int64_t)ur * V + v_lo + c] = tot;
 }
 
 // As tm_tc_cols, RWN consecutive output rows per warp: template row i is loaded once for the
@@ -823,8 +819,7 @@ template <int JC, int RWN>
 __global__ void __launch_bounds__(256) tm_tc_cols_rw(const float* __restrict__ img, int64_t pitch,
                                                      int64_t frame_stride, const float* __restrict__ tplC, int tplP,
                                                      int h, int w, int v_lo, int V, int u_begin, int Ub, int batch,
-                                                     unsigned long long* __restrict__ acc,
-                                                     int64_t acc_frame_stride) {
+                                                     float* __restrict__ acc, int64_t acc_frame_stride) {
   const int nc = V - v_lo, nrb = (Ub + RWN - 1) / RWN;
   const int64_t item = (int64_t)blockIdx.x * 8 + (threadIdx.x >> 5);
   if (item >= (int64_t)batch * nrb * nc) return;
@@ -876,7 +871,7 @@ __global__ void __launch_bounds__(256) tm_tc_cols_rw(const float* __restrict__ i
   if (lane == 0)
 #pragma unroll
     for (int r = 0; r < RWN; ++r)
-      if (ur0 + r < Ub) acc[(int64_t)f * acc_frame_stride + (int64_t)(ur0 + r) * V + v_lo + c] = __float_as_uint(tot[r]);
+      if (ur0 + r < Ub) acc[(int64_t)f * acc_frame_stride + (int64_t)(ur0 + r) * V + v_lo + c] = tot[r];
 }
 
 // Template operand: for block (bi, bj) the reversed, zero-padded rows Rv[k] = A_C[i0 + K0 - k]
@@ -1005,13 +1000,12 @@ __global__ void __launch_bounds__(1024) tm_tc_prep(const float* __restrict__ tmp
 // to finish turns every frame's key into its peak (tm_finalize fused) -- the tensor-core kernel
 // folded its own columns' keys before this launch (stream order).  grid = max(1, ceil(items /
 // 256)), items = batch x Ub x (V - v_lo); block = 256.
-__global__ void __launch_bounds__(256) tm_tc_tail(const unsigned long long* __restrict__ acc, int64_t acc_frame_stride,
+__global__ void __launch_bounds__(256) tm_tc_tail(const float* __restrict__ acc, int64_t acc_frame_stride,
                                                   const double* __restrict__ S1, const double* __restrict__ S2,
                                                   int64_t stat_frame_stride, const TemplateStats* tst, int h, int w,
                                                   int V, int v_lo, int u_begin, int Ub, int batch, float* scores,
                                                   int64_t score_frame_stride, unsigned long long* keys, int ssd,
-                                                  unsigned int* __restrict__ done, PeakOut* __restrict__ peaks,
-                                                  unsigned int* __restrict__ seq) {
+                                                  unsigned int* __restrict__ done, PeakOut* __restrict__ peaks) {
   __shared__ bool last;
   const TemplateStats ts = tst[0];
   const int nc = V - v_lo;
@@ -1027,7 +1021,7 @@ __global__ void __launch_bounds__(256) tm_tc_tail(const unsigned long long* __re
     f = (int)(t / Ub);
     const int v = v_lo + c;
     const int64_t o = (int64_t)ur * V + v;
-    const float num = __uint_as_float((uint32_t)acc[(int64_t)f * acc_frame_stride + o]);
+    const float num = acc[(int64_t)f * acc_frame_stride + o];
     const double s1 = S1[(int64_t)f * stat_frame_stride + o], s2 = S2[(int64_t)f * stat_frame_stride + o];
     const float sc = ssd ? (float)(ts.sumsq - 2.0 * ((double)num + ts.sum * inv_n * s1) + s2)
                          : ncc_normalize_fast(num, s1, s2, inv_n, ts.csum, ts.energy, ts.flat != 0);
@@ -1060,10 +1054,7 @@ __global__ void __launch_bounds__(256) tm_tc_tail(const unsigned long long* __re
     pk.flags = (ts.flat && !ssd) ? (kFlatTemplate | kInvalid) : 0u;
     peaks[fr] = pk;
   }
-  if (threadIdx.x == 0) {
-    *done = 0u;  // ready for the next call (stream-ordered)
-    *seq += 1u;  // the next call's chain tags
-  }
+  if (threadIdx.x == 0) *done = 0u;  // ready for the next call (stream-ordered)
 }
 
 }  // namespace nccb

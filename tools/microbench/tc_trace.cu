@@ -21,14 +21,14 @@ int main(int argc, char** argv) {
   cudaMemset(img, 0, (size_t)H * W * 8);
   cudaMalloc(&tcB, (size_t)nbi * nbj * tc::b_bytes(WC));
   cudaMemset(tcB, 0, (size_t)nbi * nbj * tc::b_bytes(WC));
-  cudaMalloc(&part, (size_t)U * V * 8);
+  cudaMalloc(&part, (size_t)U * V * 4);
   cudaMalloc(&tr, 8 * 1024 * 8);
   cudaMemset(tr, 0, 8 * 1024 * 8);
   cudaMemcpyToSymbol(g_tc_trace, &tr, sizeof(tr));
   TcArgs a{};
   a.H = H; a.W = W;
   a.tcB = tcB; a.WC = WC; a.nbi = nbi; a.nbj = nbj; a.V = V; a.u_begin = 0; a.u_end = U;
-  a.useg = (U + nseg - 1) / nseg; a.nseg = nseg; a.vtiles = vtiles; a.acc = reinterpret_cast<unsigned long long*>(part);
+  a.useg = (U + nseg - 1) / nseg; a.nseg = nseg; a.vtiles = vtiles; a.acc = part;
   a.acc_frame_stride = (int64_t)U * V;
   // chain / epilogue scratch (zero statistics: the normalised values are not inspected here)
   const int ngrp = (a.useg + tc::kHB - 1 + tc::kG - 1) / tc::kG;
@@ -38,7 +38,7 @@ int main(int argc, char** argv) {
   cudaMalloc(&keys, 8); cudaMemset(keys, 0, 8);
   cudaMalloc(&S, (size_t)U * V * 8); cudaMemset(S, 0, (size_t)U * V * 8);
   cudaMalloc(&ts, sizeof(TemplateStats)); cudaMemset(ts, 0, sizeof(TemplateStats));
-  a.seq = (const unsigned int*)flags; a.ticket = ticket; a.rsv = (const float*)S; a.mean = (const float*)S; a.S1 = S; a.S2 = S; a.stat_frame_stride = (int64_t)U * V;
+  a.flags = flags; a.ngrp_max = ngrp; a.ticket = ticket; a.S1 = S; a.S2 = S; a.stat_frame_stride = (int64_t)U * V;
   a.tst = ts; a.h = h; a.w = w; a.scores = nullptr; a.score_frame_stride = 0; a.keys = keys; a.ssd = 0;
   const int smem = tc::smem_bytes(WC);
   cudaFuncSetAttribute(tm_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);

@@ -8,7 +8,6 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
-import numpy as np  # noqa: E402
 import torch  # noqa: E402
 from torch.profiler import ProfilerActivity, profile  # noqa: E402
 
@@ -25,14 +24,12 @@ def main():
     flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device=DEV)
     if c["kind"] == "tm":
         img, T, _, _ = synth.tm_inputs(cfg)
-        F = int(os.environ.get("TL_BATCH", "1"))  # frames per call
-        imgs = np.ascontiguousarray(np.broadcast_to(img, (F,) + img.shape))
-        d_img, d_t = torch.from_numpy(imgs).to(DEV), torch.from_numpy(T).to(DEV)
-        plan = MatchPlan(c["H"], c["W"], c["h"], c["w"], batch=F)
+        d_img, d_t = torch.from_numpy(img).to(DEV), torch.from_numpy(T).to(DEV)
+        plan = MatchPlan(c["H"], c["W"], c["h"], c["w"])
         call = lambda: plan.match(d_img, d_t)  # noqa: E731
         if os.environ.get("TL_HOST"):  # the host-buffer entry point (copies in the timeline)
-            h_img, h_t = torch.from_numpy(imgs).pin_memory(), torch.from_numpy(T).pin_memory()
-            h_pk = torch.empty((F, 4), dtype=torch.int32).pin_memory()
+            h_img, h_t = torch.from_numpy(img).pin_memory(), torch.from_numpy(T).pin_memory()
+            h_pk = torch.empty((1, 4), dtype=torch.int32).pin_memory()
             call = lambda: plan.match_host(h_img, h_t, h_pk)  # noqa: E731
     else:
         P = 1 if cfg == 3 else 8
