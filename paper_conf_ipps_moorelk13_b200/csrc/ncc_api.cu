@@ -351,7 +351,9 @@ struct ncc_plan_s {
   int tc_vcols;  // last output columns computed by tm_tc_cols (0: none)
   int tc_sched;  // 0: window sums || template prep, image split after them; 3 (default): image split,
                  // then window sums || template prep + ragged columns
-  float *tcB, *tc_acc;     // reversed template-block operands; running numerator (one plane)
+  float *tcB, *tc_acc;     // reversed template-block operands; running numerator (one plane, chain mode)
+  int tc_planes;           // planes mode (few template blocks): per-block partial planes + tm_tc_finish
+  float* tc_part;          // [nblk][batch][Ub][V] partial numerators (planes mode)
   unsigned int* tc_done;   // finished tm_tc_tail CTAs (self-resetting)
   unsigned int* tc_flags;  // chain flags [batch][vtiles * nseg][ngrp_max][4] (self-resetting)
   unsigned long long* tc_ticket;  // CTA start tickets (monotonic)
@@ -432,6 +434,7 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->RS1);
   cudaFree(pl->tcB);
   cudaFree(pl->tc_acc);
+  cudaFree(pl->tc_part);
   cudaFree(pl->tc_done);
   cudaFree(pl->tc_flags);
   cudaFree(pl->tc_ticket);
@@ -623,7 +626,17 @@ ncc_status setup_tc(ncc_plan pl) {
   if ((st = dalloc(&pl->tcB, (size_t)nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
   // one running-numerator plane whatever the number of template blocks (they accumulate in a
   // chain inside tm_tc_kernel), chain flags, the CTA ticket counter
-  if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) return st;
+  // Few template blocks (cfg2: 4): each block writes its own partial plane (no waiting between
+  // CTAs) and tm_tc_finish sums them in block order; many (cfg5: 64): the in-kernel chain, one
+  // plane whatever the block count (64 planes were 3.4 GB of writes per cfg5 call).
+  // NCC_TC_PLANES=0/1 overrides.
+  pl->tc_planes = nblk <= 8;
+  if (const char* e = getenv("NCC_TC_PLANES")) pl->tc_planes = atoi(e) != 0;
+  if (pl->tc_planes) {
+    if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
+  } else if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) {
+    return st;
+  }
   pl->tc_ngrp = ceil_div(pl->tc_useg + tc::kHB - 1, tc::kG);
   pl->tc_exp = getenv("NCC_TC_EXP") ? atoi(getenv("NCC_TC_EXP")) : 0;
   pl->tc_center = getenv("NCC_TC_CENTER") ? atoi(getenv("NCC_TC_CENTER")) : 0;
@@ -651,8 +664,8 @@ ncc_status setup_tc(ncc_plan pl) {
                                 kPrepSmemFloats * 4));
   pl->tc = 1;
   ncc_plan_info& in = pl->info;
-  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d%s", tc::kHB, pl->tc_wc, pl->tc_nseg,
-           pl->tc_vcols ? "_cols" : "");
+  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d_%s%s", tc::kHB, pl->tc_wc,
+           pl->tc_nseg, pl->tc_planes ? "planes" : "chain", pl->tc_vcols ? "_cols" : "");
   fill_kernel_info(pl, (const void*)tm_tc_kernel, tc::kThreads, smem, nblk * pl->tc_vtiles * pl->tc_nseg, p.batch, 1);
   in.specialized = 3;  // tensor-core tier: one kernel for every shape (h, w run-time evaluated), not an SK
   in.split = nblk;
@@ -1188,7 +1201,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     auto cols = [&](auto kern) {
       kern<<<(unsigned)ceil_div(items, 8), 256, 0, pl->side>>>(
           d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w,
-          pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, batch, pl->tc_acc, pfs);
+          pl->V - pl->tc_vcols, pl->V, pl->u_begin, pl->Ub, batch, pl->tc_planes ? pl->tc_part : pl->tc_acc, pfs);
     };
     if (jc <= 4) cols(tm_tc_cols<4>);
     else if (jc <= 8) cols(tm_tc_cols<8>);
@@ -1274,6 +1287,9 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.nseg = pl->tc_nseg;
     t.vtiles = pl->tc_vtiles;
     t.acc = pl->tc_acc;
+    t.planes = pl->tc_planes;
+    t.part = pl->tc_part;
+    t.part_blk_stride = (int64_t)p.batch * pl->Ub * pl->V;
     t.acc_frame_stride = (int64_t)pl->Ub * pl->V;
     t.flags = pl->tc_flags;
     t.ngrp_max = pl->tc_ngrp;
@@ -1297,11 +1313,19 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
         t, map_tc);
     mark(pl, s, 3);
     if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
-    const int64_t tail_items = (int64_t)batch * pl->Ub * pl->tc_vcols;
-    tm_tc_tail<<<(unsigned)std::max<int64_t>(1, ceil_div(tail_items, 256)), 256, 0, s>>>(
-        pl->tc_acc, (int64_t)pl->Ub * pl->V, pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V,
-        pl->V - pl->tc_vcols, pl->u_begin, pl->Ub, batch, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
-        (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks));
+    if (pl->tc_planes) {
+      tm_tc_finish<<<dim3(ceil_div(pl->V, 256 * kFinV), pl->Ub, batch), 256, 0, s>>>(
+          pl->tc_part, nblk, (int64_t)p.batch * pl->Ub * pl->V, (int64_t)pl->Ub * pl->V, pl->tc_rsv, pl->tc_mean,
+          pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V, pl->V - pl->tc_vcols, pl->u_begin,
+          (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr, (int64_t)pl->Ub * pl->V, pl->keys,
+          p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks), batch);
+    } else {
+      const int64_t tail_items = (int64_t)batch * pl->Ub * pl->tc_vcols;
+      tm_tc_tail<<<(unsigned)std::max<int64_t>(1, ceil_div(tail_items, 256)), 256, 0, s>>>(
+          pl->tc_acc, (int64_t)pl->Ub * pl->V, pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V,
+          pl->V - pl->tc_vcols, pl->u_begin, pl->Ub, batch, (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr,
+          (int64_t)pl->Ub * pl->V, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks));
+    }
     mark(pl, s, 4);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess) return cuda_fail(e, "ncc_match launch (tensor core)");

@@ -173,7 +173,10 @@ struct TcArgs {
   // partial planes, no summation kernel -- the paper's K2 global round trip, Figs 5.4-5.6, is
   // gone): block b > 0 adds its drained rows to the running numerator block b - 1 left in `acc`
   // (per-row-group, per-warp flags), the last block normalises them in the same drain.
-  float* acc;              // [batch][u_end - u_begin][V] running numerator (one plane)
+  float* acc;              // [batch][u_end - u_begin][V] running numerator (one plane; chain mode)
+  int planes;              // 1: planes mode -- block b writes its partial sums to part + b part_blk_stride
+  float* part;             //    (summed in block order by tm_tc_finish); 0: the chain
+  int64_t part_blk_stride;
   int64_t acc_frame_stride;
   unsigned int* flags;     // [batch][vtiles * nseg][ngrp_max][4]: blocks done with a row group
   int ngrp_max;
@@ -481,7 +484,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 #pragma unroll
       for (int k = 0; k < kG; ++k) rowoff[k] = (int64_t)min(max(up0 + k, 0), nu - 1) * a.V;
       float prev[2][kG], fa[2][kG], fb[2][kG];
-      if (has_rows && last_blk && !a.ssd) {  // normalisation factors: no dependency, requested first
+      if (has_rows && last_blk && !a.ssd && !a.planes) {  // normalisation factors: requested first
 #pragma unroll
         for (int j = 0; j < 2; ++j)
 #pragma unroll
@@ -503,7 +506,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           pending = -1;
         }
       };
-      if (has_rows && blk > 0 && !(a.exp & 1)) {  // every lane acquires the flag itself
+      if (has_rows && blk > 0 && !(a.exp & 1) && !a.planes) {  // every lane acquires the flag itself
         unsigned int fv = ld_acquire_u32(fl);
         publish_pending();
         for (long long it = 0; fv < (unsigned)blk; ++it) {
@@ -514,7 +517,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         publish_pending();
       }
       if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt; pt = t; }
-      if (has_rows && blk > 0) {
+      if (has_rows && blk > 0 && !a.planes) {
 #pragma unroll
         for (int j = 0; j < 2; ++j)
 #pragma unroll
@@ -528,7 +531,16 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 #pragma unroll
         for (int k = 0; k < kG; ++k) x[j][k] = stg[slot * (kG * 128) + k * 128 + 32 * j];
       mbar_arrive(&consumed[slot]);
-      if (has_rows && !(a.exp & 16)) {
+      if (has_rows && a.planes) {  // planes mode: this block's partial sums to its own plane (no waiting)
+        float* pb = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * a.acc_frame_stride;
+#pragma unroll
+        for (int j = 0; j < 2; ++j)
+#pragma unroll
+          for (int k = 0; k < kG; ++k) {
+            const int up = up0 + k;
+            if (up >= 0 && up < nu && colok[j]) __stcg(pb + cb[j] + (int64_t)up * a.V, x[j][k]);
+          }
+      } else if (has_rows && !(a.exp & 16)) {
         if (blk > 0) {
 #pragma unroll
           for (int j = 0; j < 2; ++j)
@@ -583,14 +595,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         }
       }
     }
-    if (pending >= 0) {  // the last group's running sums
+    if (pending >= 0 && !a.planes) {  // the last group's running sums
       __threadfence();
       __syncwarp();
       if (lane == 0)
         st_release_u32(a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + pending) * 4 + cw,
                        (unsigned)(blk + 1));
     }
-    if (last_blk) {
+    if (last_blk && !a.planes) {
       wbest = warp_max_key(wbest);
       if (lane == 0 && wbest) atomicMax(a.keys + f, wbest);
     }
@@ -1040,6 +1052,89 @@ __global__ void __launch_bounds__(256) tm_tc_tail(const float* __restrict__ acc,
   if (threadIdx.x == 0) {
     __threadfence();
     last = atomicAdd(done, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  for (int fr = threadIdx.x; fr < batch; fr += blockDim.x) {
+    const unsigned long long k = atomicOr(keys + fr, 0ull);
+    const uint32_t idx = key_index(k);
+    PeakOut pk;
+    pk.score = ssd ? -key_score(k) : key_score(k);
+    pk.u = (int32_t)(idx / (uint32_t)V);
+    pk.v = (int32_t)(idx % (uint32_t)V);
+    pk.flags = (ts.flat && !ssd) ? (kFlatTemplate | kInvalid) : 0u;
+    peaks[fr] = pk;
+  }
+  if (threadIdx.x == 0) *done = 0u;  // ready for the next call (stream-ordered)
+}
+
+// Planes mode (few template blocks): sum the blocks' partial numerators in block order, normalise
+// (NCC from the window kernels' fp32 factors, |error| <= ~3e-7; SSD from the fp64 sums), optional
+// surface store, per-frame argmax keys; the last CTA writes every frame's peak.  Columns >= v_cols
+// (the ragged last columns, tm_tc_cols) hold their full numerator in block 0's plane.
+// grid = (ceil(V / (256 kFinV)), Ub, batch), block = 256.
+constexpr int kFinV = 4;
+__global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ part, int nblk, int64_t blk_stride,
+                                                    int64_t frame_stride, const float* __restrict__ rsv,
+                                                    const float* __restrict__ mean, const double* __restrict__ S1,
+                                                    const double* __restrict__ S2, int64_t stat_frame_stride,
+                                                    const TemplateStats* tst, int h, int w, int V, int v_cols,
+                                                    int u_begin, float* scores, int64_t score_frame_stride,
+                                                    unsigned long long* keys, int ssd, unsigned int* __restrict__ done,
+                                                    PeakOut* __restrict__ peaks, int batch) {
+  __shared__ unsigned long long red[32];
+  __shared__ bool last;
+  const int ur = blockIdx.y, f = blockIdx.z;
+  const int u = u_begin + ur;
+  const TemplateStats ts = tst[0];
+  const double inv_n = 1.0 / ((double)h * (double)w);
+  const float csf = (float)ts.csum, rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
+  const int64_t ro = (int64_t)f * frame_stride + (int64_t)ur * V;
+  const int64_t so = (int64_t)f * stat_frame_stride + (int64_t)ur * V;
+  unsigned long long best = 0ull;
+  const int vb = blockIdx.x * 256 * kFinV + threadIdx.x;
+  float tot[kFinV], fa[kFinV], fb[kFinV];
+#pragma unroll
+  for (int k = 0; k < kFinV; ++k) {
+    const int v = vb + k * 256;
+    tot[k] = 0.0f;
+    fa[k] = fb[k] = 0.0f;
+    if (v < V && !ssd) {
+      fa[k] = __ldg(rsv + so + v);
+      fb[k] = __ldg(mean + so + v);
+    }
+  }
+  for (int b = 0; b < nblk; ++b) {  // block order: ((p0 + p1) + p2) + ...
+    float x[kFinV];
+#pragma unroll
+    for (int k = 0; k < kFinV; ++k) {
+      const int v = vb + k * 256;
+      x[k] = (v < V && (b == 0 || v < v_cols)) ? __ldcg(part + (int64_t)b * blk_stride + ro + v) : 0.0f;
+    }
+#pragma unroll
+    for (int k = 0; k < kFinV; ++k) tot[k] = b == 0 ? x[k] : tot[k] + x[k];
+  }
+#pragma unroll
+  for (int k = 0; k < kFinV; ++k) {
+    const int v = vb + k * 256;
+    if (v >= V) break;
+    float sc;
+    if (ssd) {
+      sc = (float)(ts.sumsq - 2.0 * ((double)tot[k] + ts.sum * inv_n * __ldg(S1 + so + v)) + __ldg(S2 + so + v));
+    } else {
+      const float r = fmaf(-csf, fb[k], tot[k]) * (fa[k] * rse);
+      sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+    }
+    if (scores) scores[(int64_t)f * score_frame_stride + (int64_t)ur * V + v] = sc;
+    const unsigned long long key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
+    best = key > best ? key : best;
+  }
+  best = block_max_key(best, red);
+  if (threadIdx.x == 0) {
+    if (best && best > __ldcg(keys + f)) atomicMax(keys + f, best);
+    __threadfence();
+    last = atomicAdd(done, 1u) == gridDim.x * gridDim.y * gridDim.z - 1;
   }
   __syncthreads();
   if (!last) return;
