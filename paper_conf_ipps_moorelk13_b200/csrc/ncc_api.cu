@@ -353,6 +353,7 @@ struct ncc_plan_s {
                  // then window sums || template prep + ragged columns
   float *tcB, *tc_acc;     // reversed template-block operands; running numerator (one plane, chain mode)
   int tc_planes;           // planes mode (few template blocks): per-block partial planes + tm_tc_finish
+  int tc_box_late;         // planes mode: window sums after the numerator, as its programmatic dependent
   float* tc_part;          // [nblk][batch][Ub][V] partial numerators (planes mode)
   unsigned int* tc_done;   // finished tm_tc_tail CTAs (self-resetting)
   unsigned int* tc_flags;  // chain flags [batch][vtiles * nseg][ngrp_max][4] (self-resetting)
@@ -632,6 +633,7 @@ ncc_status setup_tc(ncc_plan pl) {
   // NCC_TC_PLANES=0/1 overrides.
   pl->tc_planes = nblk <= 8;
   if (const char* e = getenv("NCC_TC_PLANES")) pl->tc_planes = atoi(e) != 0;
+  pl->tc_box_late = getenv("NCC_TC_BOX_LATE") ? atoi(getenv("NCC_TC_BOX_LATE")) : 1;
   if (pl->tc_planes) {
     if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
   } else if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) {
@@ -1086,7 +1088,10 @@ inline void mark(ncc_plan pl, cudaStream_t s, int i) {
 }
 
 // window sums of `batch` frames over rows [row0, row0 + rows_out + h - 1)
-void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_out, cudaStream_t s) {
+// pdl: launched as a programmatic dependent of the preceding kernel in `s` (the tensor-core
+// numerator, which triggers it at its start): the window sums then run on the SMs the numerator
+// leaves free, instead of in front of it.
+void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_out, cudaStream_t s, bool pdl = false) {
   const ncc_problem& p = pl->p;
   const int h = p.tmpl_h, w = p.tmpl_w;
   const int V = p.image_w - w + 1;
@@ -1096,6 +1101,24 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
     while (TU > pl->box_r && (int64_t)gx * ceil_div(rows_out, TU) * batch < pl->nsm) TU /= 2;
     if (const char* e = getenv("NCC_BOX_TU")) TU = std::max(pl->box_r, atoi(e));  // sweeps
     dim3 g(gx, ceil_div(rows_out, TU), batch);
+    if (pdl) {
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = g;
+      cfg.blockDim = dim3(kBox2dNT);
+      cfg.dynamicSmemBytes = (size_t)pl->box_smem;
+      cfg.stream = s;
+      cudaLaunchAttribute at[1];
+      at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      at[0].val.programmaticStreamSerializationAllowed = 1;
+      cfg.attrs = at;
+      cfg.numAttrs = 1;
+      const int64_t fs = (int64_t)p.image_h * p.image_pitch, sfs = pl->s_frame_stride;
+      const int tv = kBoxTV;
+      cudaLaunchKernelEx(&cfg, box2d_kernel<kBox2dNT>, frames, p.image_pitch, fs, row0, h, w, V, rows_out, tv, TU,
+                         pl->box_r, pl->box_iwp, pl->S1, pl->S2, sfs, pl->tc_rsv, pl->tc_mean,
+                         1.0 / ((double)h * (double)w));
+      return;
+    }
     box2d_kernel<kBox2dNT><<<g, kBox2dNT, pl->box_smem, s>>>(frames, p.image_pitch,
                                                             (int64_t)p.image_h * p.image_pitch, row0, h, w, V,
                                                             rows_out, kBoxTV, TU, pl->box_r, pl->box_iwp, pl->S1,
@@ -1256,7 +1279,9 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }
     if (!pl->tc_center) launch_split(s);
-    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
+    // planes mode: the numerator does not read the window sums (tm_tc_finish does), so they run
+    // after it as its programmatic dependent, on the SMs it leaves free (cfg2: 8 of 148)
+    if (!(pl->tc_planes && pl->box_smem && pl->tc_box_late)) launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
   } else {
@@ -1311,6 +1336,8 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.center = pl->tc_center;
     tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
+    if (pl->tc_sched == 3 && pl->tc_planes && pl->box_smem && pl->tc_box_late)
+      launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, /*pdl=*/true);
     mark(pl, s, 3);
     if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
     if (pl->tc_planes) {

@@ -232,6 +232,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   // the chain never waits on a CTA that is not resident or finished, whatever the hardware's
   // dispatch order.  The counter only grows: a launch of this plan always has the same grid.
   if (tid == 0) ticket_s = atomicAdd(a.ticket, 1ull) % ((unsigned long long)gridDim.x * gridDim.y);
+  // a kernel launched after this one as its programmatic dependent (planes mode: the window sums,
+  // which read only the frames) may start now, on the SMs this grid leaves free
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
   __syncthreads();
   const int64_t tk = (int64_t)ticket_s;
   const int blk = (int)(tk % nblk);
