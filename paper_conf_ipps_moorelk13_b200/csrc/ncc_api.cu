@@ -286,8 +286,24 @@ PivJitChoice piv_jit_choice(int h, int w, int my, int mx) {
   c.ok = false;
   if (items > 1024) return c;  // one item per thread (score tile aliased on the template pairs)
   const int64_t kTwoPerSm = 113 * 1024, kOnePerSm = 227 * 1024;
+  if (force_wpb) {  // sweeps: exactly the requested windows per CTA
+    const int nt = ((force_wpb * items + 31) / 32) * 32;
+    const int64_t smem = (int64_t)force_wpb * c.win_fl * 4;
+    if (nt > 1024 || smem > kOnePerSm) return c;
+    c.WPB = force_wpb;
+    c.NT = nt;
+    c.MINB = smem <= kTwoPerSm ? 2 : 1;
+    c.ok = true;
+    return c;
+  }
   double best = -1.0;
-  for (int k = 1; k <= 4; ++k) {  // more windows per CTA blow up the per-window register arrays
+  // One window per CTA unless its items fill under 60 % of the warps: the Tab 6.22 surface
+  // (EXPERIMENTS.md, cfg3 shape) puts WPB = 1 first at every RV (k = 3 / 4: 86-90 %) -- more
+  // windows per CTA blow up the per-window register arrays (48^2 / 64^2 masks: 128-138 registers,
+  // slower than the generic kernel).
+  const double util1 = (double)items / (((items + 31) / 32) * 32);
+  const int kmax = util1 >= 0.6 ? 1 : 4;
+  for (int k = 1; k <= kmax; ++k) {
     if (force_wpb && k != force_wpb) continue;
     const int nt = ((k * items + 31) / 32) * 32;
     const int64_t smem = (int64_t)k * c.win_fl * 4;
@@ -569,7 +585,7 @@ ncc_status setup_tc(ncc_plan pl) {
   // launch order (measured on B200, cfg2 step: 0 -> 0.2135 ms, 3 -> 0.2074 ms; 1/2 delay the
   // tensor-core kernel's start or starve the ragged-column kernel); NCC_TM_SCHED overrides
   pl->tc_sched = getenv("NCC_TM_SCHED") ? atoi(getenv("NCC_TM_SCHED")) : 3;
-  if (pl->tc_sched != 0) pl->tc_sched = 3;  // (the earlier 1/2: window sums after the numerator's start)
+  if (pl->tc_sched != 0 && pl->tc_sched != 4) pl->tc_sched = 3;  // (1/2: window sums after the numerator's start)
   if (pl->V > 128 && pl->V % 128 != 0 && pl->V % 128 <= kTcColsMax && w <= 512 && !getenv("NCC_TC_NO_COLS")) {
     pl->tc_vtiles = pl->V / 128;
     pl->tc_vcols = pl->V % 128;
@@ -633,7 +649,7 @@ ncc_status setup_tc(ncc_plan pl) {
   // NCC_TC_PLANES=0/1 overrides.
   pl->tc_planes = nblk <= 8;
   if (const char* e = getenv("NCC_TC_PLANES")) pl->tc_planes = atoi(e) != 0;
-  pl->tc_box_late = getenv("NCC_TC_BOX_LATE") ? atoi(getenv("NCC_TC_BOX_LATE")) : 1;
+  pl->tc_box_late = getenv("NCC_TC_BOX_LATE") ? atoi(getenv("NCC_TC_BOX_LATE")) : 0;  // measured: slower
   if (pl->tc_planes) {
     if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
   } else if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) {
@@ -1265,12 +1281,25 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       tm_tc_tpl_prep<<<nblk_tc, 256, 0, pl->side>>>(pl->tplC, pl->WP, p.tmpl_h, p.tmpl_w, pl->tc_wc, pl->tc_nbj,
                                                     pl->tcB);
   }
-  if (tc_now && pl->tc_center) {  // the centred split needs the template mean: after the prep
+  // the image split on the side stream after the template prep: for the centred operand (it needs
+  // the template mean), and in schedule 4 (window sums first on the main stream, alone)
+  const bool split_side = tc_now && (pl->tc_center || pl->tc_sched == 4);
+  if (split_side) {
     if (pl->h_img_in) NCC_CUDA(cudaStreamWaitEvent(pl->side, pl->ev_img, 0));
     launch_split(pl->side);
   }
   NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
-  if (tc_now && pl->tc_sched == 3) {
+  if (tc_now && pl->tc_sched == 4) {
+    // window sums first, alone on the main stream (232 CTAs at 2 per SM leave room for the
+    // template prep's few CTAs); prep -> image split -> ragged columns on the side stream
+    if (pl->tc_vcols) {
+      launch_cols();
+      NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
+    }
+    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
+    NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
+    mark(pl, s, 2);
+  } else if (tc_now && pl->tc_sched == 3) {
     // the image split first (small: it leaves room for the template prep, which starts at once
     // on the side stream), then the window sums on the main stream; the ragged columns follow
     // the template prep on the side stream and overlap the window sums / tensor-core kernel
@@ -1278,7 +1307,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       launch_cols();
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }
-    if (!pl->tc_center) launch_split(s);
+    if (!split_side) launch_split(s);
     // planes mode: the numerator does not read the window sums (tm_tc_finish does), so they run
     // after it as its programmatic dependent, on the SMs it leaves free (cfg2: 8 of 148)
     if (!(pl->tc_planes && pl->box_smem && pl->tc_box_late)) launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
@@ -1297,7 +1326,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
     const int nblk = nblk_tc;
-    if (pl->tc_sched != 3 && !pl->tc_center) launch_split(s);
+    if (pl->tc_sched != 3 && !split_side) launch_split(s);
     TcArgs t;
     t.H = p.image_h;
     t.W = p.image_w;
