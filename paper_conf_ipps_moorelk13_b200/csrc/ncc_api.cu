@@ -575,18 +575,23 @@ ncc_status setup_tc(ncc_plan pl) {
   // eligible; default: the cost model below (tensor cores when clearly faster).
   const char* env = getenv("NCC_TC");
   const int mode = env ? atoi(env) : -1;
-  if (mode == 0 || (p.flags & (NCC_F_CUDA_CORES | NCC_F_GENERIC_KERNEL)) || pl->roi_mode || pl->n_tmpl != 1)
+  if (mode == 0 || (p.flags & (NCC_F_CUDA_CORES | NCC_F_GENERIC_KERNEL)) || (!pl->roi_mode && pl->n_tmpl != 1))
     return NCC_OK;
   const int h = p.tmpl_h, w = p.tmpl_w;
+  // ROI / multi-template mode: every (frame, template) pair is a sub-problem of roi_h x
+  // roi_w offsets whose origin the kernel reads at run time; planes mode only, no ragged-column kernel
+  const bool roi = pl->roi_mode;
+  const int rows = roi ? p.roi_h : pl->Ub, cols = roi ? p.roi_w : pl->V;
+  const int nsub = p.batch * (roi ? pl->n_tmpl : 1);
   // a ragged last column tile of at most kTcColsMax columns goes to tm_tc_cols instead of a
   // whole column of tensor-core CTAs
-  pl->tc_vtiles = ceil_div(pl->V, 128);
+  pl->tc_vtiles = ceil_div(cols, 128);
   pl->tc_vcols = 0;
   // launch order (measured on B200, cfg2 step: 0 -> 0.2135 ms, 3 -> 0.2074 ms; 1/2 delay the
   // tensor-core kernel's start or starve the ragged-column kernel); NCC_TM_SCHED overrides
   pl->tc_sched = getenv("NCC_TM_SCHED") ? atoi(getenv("NCC_TM_SCHED")) : 3;
   if (pl->tc_sched != 0 && pl->tc_sched != 4) pl->tc_sched = 3;  // (1/2: window sums after the numerator's start)
-  if (pl->V > 128 && pl->V % 128 != 0 && pl->V % 128 <= kTcColsMax && w <= 512 && !getenv("NCC_TC_NO_COLS")) {
+  if (!roi && pl->V > 128 && pl->V % 128 != 0 && pl->V % 128 <= kTcColsMax && w <= 512 && !getenv("NCC_TC_NO_COLS")) {
     pl->tc_vtiles = pl->V / 128;
     pl->tc_vcols = pl->V % 128;
   }
@@ -604,12 +609,12 @@ ncc_status setup_tc(ncc_plan pl) {
       continue;
     }
     const int nbj = ceil_div(w, wc);
-    const int64_t per_seg = (int64_t)pl->tc_vtiles * pl->tc_nbi * nbj * p.batch;
+    const int64_t per_seg = (int64_t)pl->tc_vtiles * pl->tc_nbi * nbj * nsub;
     const int force_seg = getenv("NCC_TC_NSEG") ? atoi(getenv("NCC_TC_NSEG")) : 0;  // sweeps
-    for (int nseg = 1; nseg <= 64 && nseg <= pl->Ub; ++nseg) {
+    for (int nseg = 1; nseg <= 64 && nseg <= rows; ++nseg) {
       if (force_seg > 0 && nseg != force_seg) continue;
-      const int useg = ceil_div(pl->Ub, nseg);
-      const int64_t ctas = per_seg * ceil_div(pl->Ub, useg);
+      const int useg = ceil_div(rows, nseg);
+      const int64_t ctas = per_seg * ceil_div(rows, useg);
       const int64_t waves = (ctas + pl->nsm - 1) / pl->nsm;
       // cycles of a CTA: per stage ~320 cycles of fixed cost + 12 MMAs of 68 x N/136 cycles,
       // N = the group's trimmed window (tm_tc_kernel: ramp-in / ramp-out rows cover fewer columns)
@@ -628,7 +633,7 @@ ncc_status setup_tc(ncc_plan pl) {
         pl->tc_wc = wc;
         pl->tc_nbj = nbj;
         pl->tc_useg = useg;
-        pl->tc_nseg = ceil_div(pl->Ub, useg);
+        pl->tc_nseg = ceil_div(rows, useg);
       }
     }
     if (wc >= w) break;
@@ -636,22 +641,22 @@ ncc_status setup_tc(ncc_plan pl) {
   // measured B200 rates: ~1050-1170 cycles per full tensor-core stage (12 MMAs of 128 x 136 x 8,
   // 3xTF32; modelled above), ~95 useful FP32 MACs per cycle per SM on the CUDA-core path
   const double tc_cycles = best;
-  const double cc_cycles = (double)h * w * (double)pl->Ub * pl->V * p.batch / (95.0 * pl->nsm);
+  const double cc_cycles = (double)h * w * (double)rows * cols * nsub / (95.0 * pl->nsm);
   if (mode < 0 && !(tc_cycles < 0.8 * cc_cycles)) return NCC_OK;
   const int nblk = pl->tc_nbi * pl->tc_nbj;
   ncc_status st;
-  if ((st = dalloc(&pl->tcB, (size_t)nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
-  // one running-numerator plane whatever the number of template blocks (they accumulate in a
-  // chain inside tm_tc_kernel), chain flags, the CTA ticket counter
+  if (roi && nblk > 8) return NCC_OK;  // ROI mode runs in planes mode only
+  if ((st = dalloc(&pl->tcB, (size_t)pl->n_tmpl * nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
   // Few template blocks (cfg2: 4): each block writes its own partial plane (no waiting between
   // CTAs) and tm_tc_finish sums them in block order; many (cfg5: 64): the in-kernel chain, one
   // plane whatever the block count (64 planes were 3.4 GB of writes per cfg5 call).
   // NCC_TC_PLANES=0/1 overrides.
   pl->tc_planes = nblk <= 8;
   if (const char* e = getenv("NCC_TC_PLANES")) pl->tc_planes = atoi(e) != 0;
+  if (roi) pl->tc_planes = 1;
   pl->tc_box_late = getenv("NCC_TC_BOX_LATE") ? atoi(getenv("NCC_TC_BOX_LATE")) : 0;  // measured: slower
   if (pl->tc_planes) {
-    if ((st = dalloc(&pl->tc_part, (size_t)nblk * p.batch * pl->Ub * pl->V))) return st;
+    if ((st = dalloc(&pl->tc_part, (size_t)nblk * nsub * rows * cols))) return st;
   } else if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) {
     return st;
   }
@@ -659,7 +664,7 @@ ncc_status setup_tc(ncc_plan pl) {
   pl->tc_exp = getenv("NCC_TC_EXP") ? atoi(getenv("NCC_TC_EXP")) : 0;
   pl->tc_center = getenv("NCC_TC_CENTER") ? atoi(getenv("NCC_TC_CENTER")) : 0;
   if (pl->tc_exp & 32) {
-    const size_t n = (size_t)nblk * pl->tc_vtiles * pl->tc_nseg * p.batch * 8 + 512;  // + group traces
+    const size_t n = (size_t)nblk * pl->tc_vtiles * pl->tc_nseg * nsub * 8 + 512;  // + group traces
     if ((st = dalloc(&pl->tc_prof, n))) return st;
     NCC_CUDA(cudaMemset(pl->tc_prof, 0, n * 8));
   }
@@ -682,9 +687,9 @@ ncc_status setup_tc(ncc_plan pl) {
                                 kPrepSmemFloats * 4));
   pl->tc = 1;
   ncc_plan_info& in = pl->info;
-  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d_%s%s", tc::kHB, pl->tc_wc,
-           pl->tc_nseg, pl->tc_planes ? "planes" : "chain", pl->tc_vcols ? "_cols" : "");
-  fill_kernel_info(pl, (const void*)tm_tc_kernel, tc::kThreads, smem, nblk * pl->tc_vtiles * pl->tc_nseg, p.batch, 1);
+  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d_%s%s%s", tc::kHB, pl->tc_wc,
+           pl->tc_nseg, pl->tc_planes ? "planes" : "chain", pl->tc_vcols ? "_cols" : "", roi ? "_roi" : "");
+  fill_kernel_info(pl, (const void*)tm_tc_kernel, tc::kThreads, smem, nblk * pl->tc_vtiles * pl->tc_nseg, nsub, 1);
   in.specialized = 3;  // tensor-core tier: one kernel for every shape (h, w run-time evaluated), not an SK
   in.split = nblk;
   in.const_template = 0;
@@ -1270,7 +1275,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   if (pl->tc && p.tmpl_h * p.tmpl_w <= kPrepSmemFloats && !getenv_flag_two_kernel_prep()) {
     // one launch: template stats + centred template + MMA operand, template staged in shared memory
-    tm_tc_prep<<<nblk_tc, 1024, p.tmpl_h * p.tmpl_w * 4, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
+    tm_tc_prep<<<dim3(nblk_tc, pl->n_tmpl), 1024, p.tmpl_h * p.tmpl_w * 4, pl->side>>>(d_tmpl, tmpl_pitch, p.tmpl_h, p.tmpl_w, pl->tplC, pl->HP, pl->WP,
                                                pl->tst, pl->keys, batch, pl->tc_wc, pl->tc_nbj, pl->tcB);
     mark(pl, pl->side, 1);
   } else {
@@ -1342,8 +1347,14 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.vtiles = pl->tc_vtiles;
     t.acc = pl->tc_acc;
     t.planes = pl->tc_planes;
+    t.rois = pl->roi_mode ? d_rois : nullptr;
+    t.n_tmpl = pl->n_tmpl;
+    t.roi_h = p.roi_h;
+    t.roi_w = p.roi_w;
+    t.U = pl->U;
     t.part = pl->tc_part;
-    t.part_blk_stride = (int64_t)p.batch * pl->Ub * pl->V;
+    t.part_blk_stride = pl->roi_mode ? (int64_t)p.batch * pl->n_tmpl * p.roi_h * p.roi_w
+                                     : (int64_t)p.batch * pl->Ub * pl->V;
     t.acc_frame_stride = (int64_t)pl->Ub * pl->V;
     t.flags = pl->tc_flags;
     t.ngrp_max = pl->tc_ngrp;
@@ -1363,13 +1374,21 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.exp = pl->tc_exp;
     t.prof = pl->tc_prof;
     t.center = pl->tc_center;
-    tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, batch), tc::kThreads, tc::smem_bytes(pl->tc_wc), s>>>(
+    tm_tc_kernel<<<dim3(nblk * pl->tc_vtiles * pl->tc_nseg, batch * pl->n_tmpl), tc::kThreads,
+                   tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
     if (pl->tc_sched == 3 && pl->tc_planes && pl->box_smem && pl->tc_box_late)
       launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, /*pdl=*/true);
     mark(pl, s, 3);
     if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
-    if (pl->tc_planes) {
+    if (pl->roi_mode) {
+      const int nsub = batch * pl->n_tmpl;
+      tm_tc_finish_roi<<<dim3(ceil_div(p.roi_w, 256 * kFinV), p.roi_h, nsub), 256, 0, s>>>(
+          pl->tc_part, nblk, (int64_t)p.batch * pl->n_tmpl * p.roi_h * p.roi_w, d_rois, pl->n_tmpl, p.roi_h, p.roi_w,
+          pl->U, pl->V, pl->tc_rsv, pl->tc_mean, pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w,
+          (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done,
+          reinterpret_cast<PeakOut*>(d_peaks), nsub);
+    } else if (pl->tc_planes) {
       tm_tc_finish<<<dim3(ceil_div(pl->V, 256 * kFinV), pl->Ub, batch), 256, 0, s>>>(
           pl->tc_part, nblk, (int64_t)p.batch * pl->Ub * pl->V, (int64_t)pl->Ub * pl->V, pl->tc_rsv, pl->tc_mean,
           pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V, pl->V - pl->tc_vcols, pl->u_begin,

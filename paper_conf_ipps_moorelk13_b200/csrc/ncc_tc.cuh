@@ -192,6 +192,8 @@ struct TcArgs {
   int ssd;
   int center;  // the image operand is centred on the template mean (tm_tc_split with ts)
   unsigned long long* prof;  // NCC_TC_EXP bit 32: per-CTA wait accounting [ticket][8] (globaltimer ns)
+  const int32_t* rois;     // ROI mode (planes): [frame][template][2] offset-space origins; else nullptr
+  int n_tmpl, roi_h, roi_w, U;
   int exp;  // timing experiments (NCC_TC_EXP; 0 in normal use): 1 no chain waits, 2 no drain work,
             // 16 prefetch only (no chain / normalisation work)
 };
@@ -242,14 +244,27 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   const int tile = (int)(rest % ((int64_t)a.vtiles * a.nseg));  // = seg * vtiles + vt
   const int vt = tile % a.vtiles, seg = tile / a.vtiles;
   const int bi = blk / a.nbj, bj = blk % a.nbj;
-  const int f = (int)(rest / ((int64_t)a.vtiles * a.nseg));
-  const int v0 = vt * 128;
-  const int ua = a.u_begin + seg * a.useg;
-  const int nu = min(a.useg, a.u_end - ua);  // output rows of this CTA
+  // sub-problem: a frame (plain band matching) or a (frame, template) pair with its ROI
+  const int f = (int)(rest / ((int64_t)a.vtiles * a.nseg));  // sub-problem index
+  int frm = f, tt = 0, ru0 = a.u_begin, uend = a.u_end, rv0 = 0, vend = a.V, opitch = a.V;
+  int64_t osub = a.acc_frame_stride;
+  if (a.rois) {  // ROI mode (planes): the ROI origin of (frame, template) from device memory
+    frm = f / a.n_tmpl;
+    tt = f % a.n_tmpl;
+    ru0 = min(max(a.rois[2 * f], 0), a.U - 1);
+    rv0 = min(max(a.rois[2 * f + 1], 0), a.V - 1);
+    uend = min(ru0 + a.roi_h, a.U);
+    vend = min(rv0 + a.roi_w, a.V);
+    opitch = a.roi_w;
+    osub = (int64_t)a.roi_h * a.roi_w;
+  }
+  const int v0 = rv0 + vt * 128;
+  const int ua = ru0 + seg * a.useg;
+  const int nu = max(0, min(a.useg, uend - ua));  // output rows of this CTA
   const int i0 = bi * kHB, j0 = bj * a.WC;
   const int nch = a.WC / kWB;                // TMEM chunks per image row
   const int R = nu + kHB - 1;                // image rows touching the CTA's outputs
-  const int ngrp = (R + kG - 1) / kG;
+  const int ngrp = nu > 0 ? (R + kG - 1) / kG : 0;
   const int nrow = ngrp * kG;
   const int nstage = nrow * nch;             // (row, chunk) stages
   const uint32_t plane = kLB * 16;           // bytes per K plane of the template operand
@@ -257,7 +272,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 
   // template operand (precomputed layout) -> shared memory
   {
-    const float4* src = reinterpret_cast<const float4*>(a.tcB + (int64_t)blk * (b_bytes(a.WC) / 4));
+    const float4* src = reinterpret_cast<const float4*>(a.tcB + ((int64_t)tt * nblk + blk) * (b_bytes(a.WC) / 4));
     float4* dst = reinterpret_cast<float4*>(smem_tc);
     const int n4 = b_bytes(a.WC) / 16;
     for (int k = tid; k < n4; k += kThreads) dst[k] = __ldg(src + k);
@@ -304,7 +319,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     } else {
       mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 8));
       tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 8, &map_img, v0 + j0 + (q % nch) * kWB,
-                  ua - a.u_begin + i0 + q / nch, f, &img_full[sl]);
+                  ua - a.u_begin + i0 + q / nch, frm, &img_full[sl]);
     }
   };
   if (TC_EXP(32768) && warp != kMmaWarp) {
@@ -471,8 +486,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 #pragma unroll
     for (int j = 0; j < 2; ++j) {
       vcol[j] = v0 + cw * 64 + 32 * j + lane;
-      colok[j] = vcol[j] < a.V;
-      cb[j] = (int64_t)(ua - a.u_begin) * a.V + (colok[j] ? vcol[j] : a.V - 1);
+      colok[j] = vcol[j] < vend;
+      cb[j] = (int64_t)(ua - ru0) * opitch + ((colok[j] ? vcol[j] : vend - 1) - rv0);
     }
     float* accb = a.acc + (int64_t)f * a.acc_frame_stride;
     const int64_t sfo = (int64_t)f * a.stat_frame_stride;
@@ -535,13 +550,13 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         for (int k = 0; k < kG; ++k) x[j][k] = stg[slot * (kG * 128) + k * 128 + 32 * j];
       mbar_arrive(&consumed[slot]);
       if (has_rows && a.planes) {  // planes mode: this block's partial sums to its own plane (no waiting)
-        float* pb = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * a.acc_frame_stride;
+        float* pb = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * osub;
 #pragma unroll
         for (int j = 0; j < 2; ++j)
 #pragma unroll
           for (int k = 0; k < kG; ++k) {
             const int up = up0 + k;
-            if (up >= 0 && up < nu && colok[j]) __stcg(pb + cb[j] + (int64_t)up * a.V, x[j][k]);
+            if (up >= 0 && up < nu && colok[j]) __stcg(pb + cb[j] + (int64_t)up * opitch, x[j][k]);
           }
       } else if (has_rows && !(a.exp & 16)) {
         if (blk > 0) {
@@ -926,6 +941,13 @@ __global__ void __launch_bounds__(1024) tm_tc_prep(const float* __restrict__ tmp
   using namespace tc;
   extern __shared__ float tsm[];  // the whole template, dense h x w (n <= kPrepSmemFloats)
   __shared__ double red[32];
+  {  // several templates (ROI mode): blockIdx.y = template t, rows of the stacked templates
+    const int t = blockIdx.y;
+    tmpl += (int64_t)t * h * tpitch;
+    tplC += (int64_t)t * HP * WP;
+    ts += t;
+    tcB += (int64_t)t * gridDim.x * (b_bytes(WC) / 4);
+  }
   const int n = h * w;
   // one pass over the template, staged in shared memory: float4 loads when rows allow it
   // (w, pitch and base 16-byte aligned), all of a thread's loads in flight
@@ -1007,7 +1029,7 @@ __global__ void __launch_bounds__(1024) tm_tc_prep(const float* __restrict__ tmp
     ts->flat = (e <= kFlatRel * s2) ? 1 : 0;
     ts->pad = 0;
   }
-  for (int f = threadIdx.x; f < batch; f += blockDim.x) keys[f] = 0ull;
+  for (int f = threadIdx.x; f < batch; f += blockDim.x) keys[(int64_t)f * gridDim.y + blockIdx.y] = 0ull;
 }
 
 // Ragged last columns [v_lo, V) (computed by tm_tc_cols into the running-numerator plane):
@@ -1153,6 +1175,78 @@ __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ pa
     peaks[fr] = pk;
   }
   if (threadIdx.x == 0) *done = 0u;  // ready for the next call (stream-ordered)
+}
+
+// ROI mode (planes): per (frame, template) sub-problem sp, sum the blocks' partial numerators of
+// its clipped ROI in block order, normalise with the template's statistics and the frame's window
+// factors, surface [sp][roi_h][roi_w] (clipped positions 0), keys[sp]; the last CTA writes every
+// sub-problem's peak.  grid = (ceil(roi_w / (256 kFinV)), roi_h, F T), block = 256.
+__global__ void __launch_bounds__(256) tm_tc_finish_roi(const float* __restrict__ part, int nblk,
+                                                        int64_t blk_stride, const int32_t* __restrict__ rois,
+                                                        int n_tmpl, int roi_h, int roi_w, int U, int V,
+                                                        const float* __restrict__ rsv, const float* __restrict__ mean,
+                                                        const double* __restrict__ S1, const double* __restrict__ S2,
+                                                        int64_t stat_frame_stride, const TemplateStats* tst, int h,
+                                                        int w, float* scores, unsigned long long* keys, int ssd,
+                                                        unsigned int* __restrict__ done, PeakOut* __restrict__ peaks,
+                                                        int nsub) {
+  __shared__ unsigned long long red[32];
+  __shared__ bool last;
+  const int r = blockIdx.y, sp = blockIdx.z;
+  const int frm = sp / n_tmpl, tt = sp % n_tmpl;
+  const int ru0 = min(max(rois[2 * sp], 0), U - 1), rv0 = min(max(rois[2 * sp + 1], 0), V - 1);
+  const int uend = min(ru0 + roi_h, U), vend = min(rv0 + roi_w, V);
+  const int u = ru0 + r;
+  const TemplateStats ts = tst[tt];
+  const double inv_n = 1.0 / ((double)h * (double)w);
+  const float csf = (float)ts.csum, rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
+  const int64_t ro = (int64_t)sp * roi_h * roi_w + (int64_t)r * roi_w;
+  unsigned long long best = 0ull;
+#pragma unroll
+  for (int k = 0; k < kFinV; ++k) {
+    const int c = blockIdx.x * 256 * kFinV + threadIdx.x + k * 256;
+    if (c >= roi_w) break;
+    const int v = rv0 + c;
+    float sc = 0.0f;
+    if (u < uend && v < vend) {
+      float tot = 0.0f;
+      for (int b = 0; b < nblk; ++b) {  // block order: ((p0 + p1) + p2) + ...
+        const float x = __ldcg(part + (int64_t)b * blk_stride + ro + c);
+        tot = b == 0 ? x : tot + x;
+      }
+      const int64_t so = (int64_t)frm * stat_frame_stride + (int64_t)u * V + v;
+      if (ssd) {
+        sc = (float)(ts.sumsq - 2.0 * ((double)tot + ts.sum * inv_n * __ldg(S1 + so)) + __ldg(S2 + so));
+      } else {
+        const float q = fmaf(-csf, __ldg(mean + so), tot) * (__ldg(rsv + so) * rse);
+        sc = q > 1.0f ? 1.0f : (q < -1.0f ? -1.0f : q);
+      }
+      const unsigned long long key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
+      best = key > best ? key : best;
+    }
+    if (scores) scores[ro + c] = sc;
+  }
+  best = block_max_key(best, red);
+  if (threadIdx.x == 0) {
+    if (best && best > __ldcg(keys + sp)) atomicMax(keys + sp, best);
+    __threadfence();
+    last = atomicAdd(done, 1u) == gridDim.x * gridDim.y * gridDim.z - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  for (int q = threadIdx.x; q < nsub; q += blockDim.x) {
+    const unsigned long long k = atomicOr(keys + q, 0ull);
+    const uint32_t idx = key_index(k);
+    const TemplateStats tq = tst[q % n_tmpl];
+    PeakOut pk;
+    pk.score = ssd ? -key_score(k) : key_score(k);
+    pk.u = (int32_t)(idx / (uint32_t)V);
+    pk.v = (int32_t)(idx % (uint32_t)V);
+    pk.flags = (tq.flat && !ssd) ? (kFlatTemplate | kInvalid) : 0u;
+    peaks[q] = pk;
+  }
+  if (threadIdx.x == 0) *done = 0u;
 }
 
 }  // namespace nccb

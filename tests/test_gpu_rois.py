@@ -81,3 +81,21 @@ def test_roi_plan_rejects_plain_match_and_bad_rois():
             plan.match(torch.zeros((1, 128, 128), device="cuda"), torch.zeros((16, 16), device="cuda"))
     with pytest.raises(N.NccError):
         MatchPlan(128, 128, 16, 16, n_templates=2, roi=(200, 8))
+
+
+@pytest.mark.parametrize("H,W,h,w,T,F,rh,rw,score", [
+    (200, 180, 16, 16, 5, 2, 40, 56, N.NCC_SCORE_NCC),
+    (260, 240, 33, 27, 3, 2, 48, 37, N.NCC_SCORE_NCC),
+    (300, 300, 64, 64, 6, 1, 64, 96, N.NCC_SCORE_NCC),
+    (420, 400, 150, 140, 3, 2, 150, 260, N.NCC_SCORE_NCC),  # 2 x 5 template blocks, 3 column tiles
+    (200, 180, 16, 16, 4, 2, 40, 56, N.NCC_SCORE_SSD),
+])
+def test_rois_on_tensor_cores_vs_oracle(H, W, h, w, T, F, rh, rw, score, monkeypatch):
+    """ROI / multi-template matching on the tensor-core numerator (tcgen05 3xTF32, planes mode):
+    every (frame, template) pair is a sub-problem whose ROI origin the kernel reads at run time;
+    same checks as the CUDA-core path (clipped ROI surfaces within 1e-4, planted peaks exact)."""
+    monkeypatch.setenv("NCC_TC", "1")
+    with MatchPlan(H, W, h, w, batch=F, n_templates=T, roi=(rh, rw)) as plan:
+        name = plan.info.variant_name.decode()
+        assert name.startswith("tm_tc") and name.endswith("_roi"), name
+    test_rois_vs_oracle(H, W, h, w, T, F, rh, rw, score)
