@@ -1130,15 +1130,23 @@ __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ pa
       fb[k] = __ldg(mean + so + v);
     }
   }
-  for (int b = 0; b < nblk; ++b) {  // block order: ((p0 + p1) + p2) + ...
-    float x[kFinV];
+  // all planes' loads in flight at once (planes mode has at most 8 blocks), then the block-order sum
+  // ((p0 + p1) + p2) + ...  (the kernel is load-latency bound)
+  for (int b0 = 0; b0 < nblk; b0 += 8) {
+    float x[8][kFinV];
 #pragma unroll
-    for (int k = 0; k < kFinV; ++k) {
-      const int v = vb + k * 256;
-      x[k] = (v < V && (b == 0 || v < v_cols)) ? __ldcg(part + (int64_t)b * blk_stride + ro + v) : 0.0f;
-    }
+    for (int bb = 0; bb < 8; ++bb)
 #pragma unroll
-    for (int k = 0; k < kFinV; ++k) tot[k] = b == 0 ? x[k] : tot[k] + x[k];
+      for (int k = 0; k < kFinV; ++k) {
+        const int v = vb + k * 256, b = b0 + bb;
+        x[bb][k] = (b < nblk && v < V && (b == 0 || v < v_cols)) ? __ldcg(part + (int64_t)b * blk_stride + ro + v)
+                                                                 : 0.0f;
+      }
+#pragma unroll
+    for (int bb = 0; bb < 8; ++bb)
+#pragma unroll
+      for (int k = 0; k < kFinV; ++k)
+        if (b0 + bb < nblk) tot[k] = (b0 + bb == 0) ? x[bb][k] : tot[k] + x[bb][k];
   }
 #pragma unroll
   for (int k = 0; k < kFinV; ++k) {
