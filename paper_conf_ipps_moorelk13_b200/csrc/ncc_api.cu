@@ -1915,9 +1915,11 @@ ncc_status ncc_match_host(ncc_plan pl, const float* h_images, const float* h_tmp
   const size_t s_bytes = surf ? (size_t)p.batch * pl->Ub * pl->V * sizeof(float) : 0;
   ncc_status st;
   const bool pinned = is_pinned(h_images) && is_pinned(h_tmpl);
-  // frames per streamed chunk: ~8 MB of frames (NCC_TM_CHUNK overrides)
+  // frames per streamed chunk: ~17 MB of frames (NCC_TM_CHUNK overrides; measured at cfg2, 8 frames
+  // per call: chunks of 1 / 2 / 4 / 8 frames reach 57 / 60 / 70 / 65 % of the device-resident rate --
+  // small chunks lose the batched numerator's efficiency, one chunk loses the overlap)
   const size_t frame_b = (size_t)p.image_h * p.image_pitch * sizeof(float);
-  int chunk = (int)std::max<size_t>(1, ((size_t)8 << 20) / frame_b);
+  int chunk = (int)std::max<size_t>(1, ((size_t)17 << 20) / frame_b);
   if (const char* e = getenv("NCC_TM_CHUNK")) chunk = std::max(1, atoi(e));
   if (pinned && p.batch > chunk) {
     // Streaming (the paper's per-frame runtime operation, 5.1.3.4 P:91): chunks of
