@@ -585,7 +585,7 @@ ncc_status setup_tc(ncc_plan pl) {
   const int nsub = p.batch * (roi ? pl->n_tmpl : 1);
   // a ragged last column tile of at most kTcColsMax columns goes to tm_tc_cols instead of a
   // whole column of tensor-core CTAs
-  pl->tc_vtiles = ceil_div(cols, 128);
+  pl->tc_vtiles = ceil_div(roi ? cols + 1 : cols, 128);  // ROI tiles start at the even column <= the origin
   pl->tc_vcols = 0;
   // launch order (measured on B200, cfg2 step: 0 -> 0.2135 ms, 3 -> 0.2074 ms; 1/2 delay the
   // tensor-core kernel's start or starve the ragged-column kernel); NCC_TM_SCHED overrides

@@ -258,7 +258,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     opitch = a.roi_w;
     osub = (int64_t)a.roi_h * a.roi_w;
   }
-  const int v0 = rv0 + vt * 128;
+  // (a TMA box of 8-byte (hi, lo) elements must start 16-byte aligned: ROI tiles start at the even
+  // column at or below the ROI origin, one more tile covers the shift, the extra column is masked)
+  const int v0 = (rv0 & ~1) + vt * 128;
   const int ua = ru0 + seg * a.useg;
   const int nu = max(0, min(a.useg, uend - ua));  // output rows of this CTA
   const int i0 = bi * kHB, j0 = bj * a.WC;
@@ -486,8 +488,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 #pragma unroll
     for (int j = 0; j < 2; ++j) {
       vcol[j] = v0 + cw * 64 + 32 * j + lane;
-      colok[j] = vcol[j] < vend;
-      cb[j] = (int64_t)(ua - ru0) * opitch + ((colok[j] ? vcol[j] : vend - 1) - rv0);
+      colok[j] = vcol[j] >= rv0 && vcol[j] < vend;
+      cb[j] = (int64_t)(ua - ru0) * opitch + ((colok[j] ? vcol[j] : rv0) - rv0);
     }
     float* accb = a.acc + (int64_t)f * a.acc_frame_stride;
     const int64_t sfo = (int64_t)f * a.stat_frame_stride;
