@@ -645,7 +645,6 @@ ncc_status setup_tc(ncc_plan pl) {
   if (mode < 0 && !(tc_cycles < 0.8 * cc_cycles)) return NCC_OK;
   const int nblk = pl->tc_nbi * pl->tc_nbj;
   ncc_status st;
-  if (roi && nblk > 8) return NCC_OK;  // ROI mode runs in planes mode only
   if ((st = dalloc(&pl->tcB, (size_t)pl->n_tmpl * nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
   // Few template blocks (cfg2: 4): each block writes its own partial plane (no waiting between
   // CTAs) and tm_tc_finish sums them in block order; many (cfg5: 64): the in-kernel chain, one
@@ -653,7 +652,7 @@ ncc_status setup_tc(ncc_plan pl) {
   // NCC_TC_PLANES=0/1 overrides.
   pl->tc_planes = nblk <= 8;
   if (const char* e = getenv("NCC_TC_PLANES")) pl->tc_planes = atoi(e) != 0;
-  if (roi) pl->tc_planes = 1;
+  if (roi) pl->tc_planes = 1;  // ROI mode: planes (small per-ROI planes, any block count)
   pl->tc_box_late = getenv("NCC_TC_BOX_LATE") ? atoi(getenv("NCC_TC_BOX_LATE")) : 0;  // measured: slower
   if (pl->tc_planes) {
     if ((st = dalloc(&pl->tc_part, (size_t)nblk * nsub * rows * cols))) return st;
