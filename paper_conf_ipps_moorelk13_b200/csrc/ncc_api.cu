@@ -385,7 +385,8 @@ struct ncc_plan_s {
   int tiny_ctas, tiny_rows, tiny_smem;
   unsigned int* tiny_done;
   // side stream for work independent of the main chain (template prep || window sums)
-  cudaStream_t side;
+  cudaStream_t side, side2;  // side2: the window sums beside the numerator (TM schedule 5)
+  cudaEvent_t ev_box;
   cudaEvent_t ev_fork, ev_join, ev_cols, ev_img;
   // timing (NCC_F_TIMING)
   std::vector<cudaEvent_t> ev;
@@ -474,6 +475,8 @@ void free_plan(ncc_plan pl) {
   if (pl->ev_cols) cudaEventDestroy(pl->ev_cols);
   if (pl->ev_img) cudaEventDestroy(pl->ev_img);
   if (pl->side) cudaStreamDestroy(pl->side);
+  if (pl->side2) cudaStreamDestroy(pl->side2);
+  if (pl->ev_box) cudaEventDestroy(pl->ev_box);
   for (int k = 0; k < 2; ++k) {
     if (pl->ev_copied[k]) cudaEventDestroy(pl->ev_copied[k]);
     if (pl->ev_free[k]) cudaEventDestroy(pl->ev_free[k]);
@@ -590,7 +593,7 @@ ncc_status setup_tc(ncc_plan pl) {
   // launch order (measured on B200, cfg2 step: 0 -> 0.2135 ms, 3 -> 0.2074 ms; 1/2 delay the
   // tensor-core kernel's start or starve the ragged-column kernel); NCC_TM_SCHED overrides
   pl->tc_sched = getenv("NCC_TM_SCHED") ? atoi(getenv("NCC_TM_SCHED")) : 3;
-  if (pl->tc_sched != 0 && pl->tc_sched != 4) pl->tc_sched = 3;  // (1/2: window sums after the numerator's start)
+  if (pl->tc_sched != 0 && pl->tc_sched != 4 && pl->tc_sched != 5) pl->tc_sched = 3;  // (1/2: retired)
   if (!roi && pl->V > 128 && pl->V % 128 != 0 && pl->V % 128 <= kTcColsMax && w <= 512 && !getenv("NCC_TC_NO_COLS")) {
     pl->tc_vtiles = pl->V / 128;
     pl->tc_vcols = pl->V % 128;
@@ -895,6 +898,8 @@ ncc_status create_tm(ncc_plan pl) {
   }
 
   NCC_CUDA(cudaStreamCreateWithFlags(&pl->side, cudaStreamNonBlocking));
+  NCC_CUDA(cudaStreamCreateWithFlags(&pl->side2, cudaStreamNonBlocking));
+  NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_box, cudaEventDisableTiming));
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_fork, cudaEventDisableTiming));
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_join, cudaEventDisableTiming));
   NCC_CUDA(cudaEventCreateWithFlags(&pl->ev_cols, cudaEventDisableTiming));
@@ -1293,7 +1298,23 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     launch_split(pl->side);
   }
   NCC_CUDA(cudaEventRecord(pl->ev_join, pl->side));
-  if (tc_now && pl->tc_sched == 4) {
+  const bool box_beside = tc_now && pl->tc_sched == 5 && pl->tc_planes;
+  if (box_beside) {
+    // planes mode: the numerator does not read the window sums (tm_tc_finish does), so they run on
+    // a second side stream from the start, beside the template prep and the image split; the
+    // numerator waits only for those two and starts on the SMs the window sums leave free
+    NCC_CUDA(cudaStreamWaitEvent(pl->side2, pl->ev_fork, 0));
+    if (pl->h_img_in) NCC_CUDA(cudaStreamWaitEvent(pl->side2, pl->ev_img, 0));
+    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, pl->side2);
+    NCC_CUDA(cudaEventRecord(pl->ev_box, pl->side2));
+    if (pl->tc_vcols) {
+      launch_cols();
+      NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
+    }
+    if (!split_side) launch_split(s);
+    NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
+    mark(pl, s, 2);
+  } else if (tc_now && pl->tc_sched == 4) {
     // window sums first, alone on the main stream (232 CTAs at 2 per SM leave room for the
     // template prep's few CTAs); prep -> image split -> ragged columns on the side stream
     if (pl->tc_vcols) {
@@ -1380,6 +1401,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, /*pdl=*/true);
     mark(pl, s, 3);
     if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
+    if (box_beside) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_box, 0));
     if (pl->roi_mode) {
       const int nsub = batch * pl->n_tmpl;
       tm_tc_finish_roi<<<dim3(ceil_div(p.roi_w, 256 * kFinV), p.roi_h, nsub), 256, 0, s>>>(
