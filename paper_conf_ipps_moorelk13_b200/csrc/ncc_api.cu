@@ -1351,7 +1351,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
     const int nblk = nblk_tc;
-    if (pl->tc_sched != 3 && !split_side) launch_split(s);
+    if (!split_side && !box_beside && pl->tc_sched != 3) launch_split(s);  // schedules 0 / 5-chain
     TcArgs t;
     t.H = p.image_h;
     t.W = p.image_w;
