@@ -1040,6 +1040,7 @@ __global__ void __launch_bounds__(1024) tm_tc_prep(const float* __restrict__ tmp
 // folded its own columns' keys before this launch (stream order).  grid = max(1, ceil(items /
 // 256)), items = batch x Ub x (V - v_lo); block = 256.
 __global__ void __launch_bounds__(256) tm_tc_tail(const float* __restrict__ acc, int64_t acc_frame_stride,
+                                                  const float* __restrict__ rsv, const float* __restrict__ mean,
                                                   const double* __restrict__ S1, const double* __restrict__ S2,
                                                   int64_t stat_frame_stride, const TemplateStats* tst, int h, int w,
                                                   int V, int v_lo, int u_begin, int Ub, int batch, float* scores,
@@ -1061,9 +1062,16 @@ __global__ void __launch_bounds__(256) tm_tc_tail(const float* __restrict__ acc,
     const int v = v_lo + c;
     const int64_t o = (int64_t)ur * V + v;
     const float num = acc[(int64_t)f * acc_frame_stride + o];
-    const double s1 = S1[(int64_t)f * stat_frame_stride + o], s2 = S2[(int64_t)f * stat_frame_stride + o];
-    const float sc = ssd ? (float)(ts.sumsq - 2.0 * ((double)num + ts.sum * inv_n * s1) + s2)
-                         : ncc_normalize_fast(num, s1, s2, inv_n, ts.csum, ts.energy, ts.flat != 0);
+    float sc;
+    if (ssd) {
+      const double s1 = S1[(int64_t)f * stat_frame_stride + o], s2 = S2[(int64_t)f * stat_frame_stride + o];
+      sc = (float)(ts.sumsq - 2.0 * ((double)num + ts.sum * inv_n * s1) + s2);
+    } else {  // the fp32-factor form of tm_tc_finish / the chain epilogue (bitwise the same scores)
+      const float rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
+      const float r = fmaf(-(float)ts.csum, mean[(int64_t)f * stat_frame_stride + o], num) *
+                      (rsv[(int64_t)f * stat_frame_stride + o] * rse);
+      sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+    }
     if (scores) scores[(int64_t)f * score_frame_stride + o] = sc;
     key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)(u_begin + ur) * V + v));
   }
