@@ -10,6 +10,8 @@ import synth  # noqa: E402
 from paper_conf_ipps_moorelk13_b200.api import PivPlan  # noqa: E402
 
 cfg, P = int(sys.argv[1]), int(sys.argv[2])
+if cfg == 3:
+    P = 1  # cfg3 is one 1024 x 1024 pair (the repeats below are the launches)
 c = synth.CONFIGS[cfg]
 wl = dict(cfg=cfg, H=c["H"], W=c["W"], h=c["h"], w=c["w"], m=c["m"], step=c["step"], pairs=P, rank=0)
 dev = torch.device("cuda", 0)
