@@ -16,8 +16,9 @@ LIB = os.path.join(PKG, "libncc_b200.so")
 SOURCES = [os.path.join(CSRC, "ncc_api.cu")]
 KERNELS = os.path.join(CSRC, "ncc_kernels.cuh")
 SRC_INC = os.path.join(CSRC, "ncc_kernels_src.inc")  # generated: the kernel source for NVRTC
-DEPS = SOURCES + [KERNELS, os.path.join(CSRC, "ncc_tc.cuh"), os.path.join(CSRC, "ncc_jit.inc"),
-                  os.path.join(ROOT, "include", "ncc.h")]
+# every source the library is compiled from: all of csrc/ (kernels, headers, includes) + the ABI header
+DEPS = sorted(os.path.join(CSRC, f) for f in os.listdir(CSRC) if f.endswith((".cu", ".cuh", ".inc"))) + \
+    [os.path.join(ROOT, "include", "ncc.h")]
 
 NVCC_FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-std=c++17",
               "--shared", "-Xcompiler", "-fPIC", "-Xptxas", "-v", "-ldl"]

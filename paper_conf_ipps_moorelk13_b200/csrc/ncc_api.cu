@@ -31,6 +31,7 @@
 #include "ncc_kernels.cuh"
 #include "ncc_tc.cuh"
 #include "ncc_sad.cuh"
+#include "ncc_piv_tc.cuh"
 
 using namespace nccb;
 
@@ -357,6 +358,10 @@ struct ncc_plan_s {
   int ws_smem, ws_grid;  // persistent warp-specialised PIV kernel (0: not used)
   int ws_bp;             // its staged pitch = TMA box width
   const PivVariant* pivv;
+  // tensor-core PIV numerator (piv_tc_kernel; 0: CUDA cores): rows per MMA, smem, grid, strip segments
+  int ptc, ptc_R, ptc_smem, ptc_border_smem, ptc_nseg, ptc_segw;
+  float* ptc_border;     // [sub_batch][Ky Kx][OY] numerators of the last column (piv_tc_border_kernel)
+  unsigned long long* ptc_prof;  // NCC_PIV_TC_PROF=<file>: per-CTA wait accounting, dumped at destroy
   // shared scratch (window sums)
   double *RS1, *RS2, *S1, *S2;
   int64_t rs_frame_stride, s_frame_stride;
@@ -432,6 +437,17 @@ struct DeviceGuard {
 };
 
 void free_plan(ncc_plan pl) {
+  if (pl->ptc_prof) {
+    if (const char* path = getenv("NCC_PIV_TC_PROF")) {
+      std::vector<unsigned long long> h((size_t)pl->nsm * 32 + 3 * 2048);
+      if (cudaMemcpy(h.data(), pl->ptc_prof, h.size() * 8, cudaMemcpyDeviceToHost) == cudaSuccess)
+        if (FILE* fp = fopen(path, "wb")) {
+          fwrite(h.data(), 8, h.size(), fp);
+          fclose(fp);
+        }
+    }
+  }
+  cudaFree(pl->ptc_prof);
   if (pl->tc_prof) {  // NCC_TC_EXP bit 32: the per-CTA accounting of the last call to NCC_TC_PROF_DUMP
     if (const char* path = getenv("NCC_TC_PROF_DUMP")) {
       const size_t n = (size_t)pl->tc_nbi * pl->tc_nbj * pl->tc_vtiles * pl->tc_nseg * pl->p.batch * 8 + 512;
@@ -459,6 +475,7 @@ void free_plan(ncc_plan pl) {
   cudaFree(pl->tc_prof);
   cudaFree(pl->tc_rsv);
   cudaFree(pl->tc_mean);
+  cudaFree(pl->ptc_border);
   cudaFree(pl->tiny_done);
   cudaFree(pl->tc_img2);
   cudaFree(pl->RS2);
@@ -1061,7 +1078,40 @@ ncc_status create_piv(ncc_plan pl) {
   }
   if ((st = dalloc(&pl->S1, (size_t)sb * pl->s_frame_stride))) return st;
   if ((st = dalloc(&pl->S2, (size_t)sb * pl->s_frame_stride))) return st;
-  if (p.score == NCC_SCORE_NCC && pl->ws_smem) {  // fp32 normalisation factors for the WS kernels
+  // tensor-core numerator (f3 on the PIV path, ncc_piv_tc.cuh): NCC score, D_x = 2 m_x in {32, 64}
+  // (R = 128 / D_x image rows per MMA), whole 16-column template chunks, and the overlapping windows
+  // of a column strip fit the accumulator / operand slots.  NCC_PIV_TC=0 (or NCC_F_CUDA_CORES) keeps
+  // the CUDA-core kernels.
+  {
+    const char* e = getenv("NCC_PIV_TC");
+    const int Dx = 2 * mx, R = (Dx == 32 || Dx == 64) ? 128 / Dx : 1, span = h + 2 * my;
+    const bool ok = p.score == NCC_SCORE_NCC && !(p.flags & NCC_F_CUDA_CORES) && !(e && atoi(e) == 0) &&
+                    (Dx == 32 || Dx == 64) && w % ptc::kKc == 0 && (h * w) % 128 == 0 &&
+                    h * w <= 128 * ptc::kPrepMax && p.step_y % R == 0 && p.step_y <= span &&
+                    (span + p.step_y - 1) / p.step_y <= ptc::kNSlot - 1 && p.step_x % 4 == 0 &&
+                    p.image_pitch % 4 == 0 && Dx + w <= 256 && ptc::tmem_cols(my, R) <= 512 &&
+                    ptc::smem_bytes(h, w, my, mx) <= maxsm && (2 * my + 1) * (2 * mx + 1) <= 128 * ptc::kEpiMax &&
+                    2 * my + 1 <= 8 * kBorderDY;
+    // default: the tensor cores where they measured faster (R = 2, +-32 search: cfg 4, 1.6x);
+    // at R = 4 (+-16, cfg 3) the CUDA-core kernel wins (EXPERIMENTS.md); NCC_PIV_TC=1 forces them
+    const bool worth = R == 2 || (e && atoi(e) == 1);
+    if (ok && worth) {
+      pl->ptc = 1;
+      pl->ptc_R = R;
+      pl->ptc_smem = ptc::smem_bytes(h, w, my, mx);
+      pl->ptc_border_smem = (h * w + (span + kBorderDY - 1) * w) * 4;
+      if (pl->ptc_border_smem > maxsm) return NCC_ERR_UNSUPPORTED;
+      NCC_CUDA(cudaFuncSetAttribute((const void*)piv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->ptc_smem));
+      NCC_CUDA(cudaFuncSetAttribute((const void*)piv_tc_border_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    pl->ptc_border_smem));
+      if ((st = dalloc(&pl->ptc_border, (size_t)sb * pl->Ky * pl->Kx * pl->OY))) return st;
+      if (getenv("NCC_PIV_TC_PROF")) {
+        if ((st = dalloc(&pl->ptc_prof, (size_t)pl->nsm * 32 + 3 * 2048))) return st;
+        NCC_CUDA(cudaMemset(pl->ptc_prof, 0, ((size_t)pl->nsm * 32 + 3 * 2048) * 8));
+      }
+    }
+  }
+  if (p.score == NCC_SCORE_NCC && (pl->ws_smem || pl->ptc)) {  // fp32 normalisation factors (WS / TC kernels)
     if ((st = dalloc(&pl->tc_rsv, (size_t)sb * pl->s_frame_stride))) return st;
     if ((st = dalloc(&pl->tc_mean, (size_t)sb * pl->s_frame_stride))) return st;
   }
@@ -1081,6 +1131,15 @@ ncc_status create_piv(ncc_plan pl) {
   else
     fill_kernel_info(pl, v->k_ldg, v->NT, pl->piv_smem, ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB), 1, sb);
   in.launches_per_call = (pl->box_smem ? 2 : 3) * ceil_div(p.batch, sb);  // per sub-batch: window sums + PIV
+  if (pl->ptc) {  // per sub-batch: window sums, last-column kernel, tensor-core kernel
+    int nsm = 0;
+    NCC_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, pl->device));
+    snprintf(in.variant_name, sizeof(in.variant_name), "piv_tc_tf32x3_%dx%d_m%dx%d_r%d", h, w, my, mx, pl->ptc_R);
+    fill_kernel_info(pl, (const void*)piv_tc_kernel, ptc::kThreads, pl->ptc_smem, nsm, 1, 1);
+    in.specialized = 3;
+    in.variant_id = -1;
+    in.launches_per_call = (pl->box_smem ? 3 : 4) * ceil_div(p.batch, sb);
+  }
   if (p.score == NCC_SCORE_SAD) {  // direct |t - b| kernel, one CTA per (window, pair); no window sums
     const int OY = 2 * my + 1, OX = 2 * mx + 1, OXP = ((OX + 3) / 4) * 4;
     const int64_t smem = ((int64_t)h * w + (int64_t)(h + 2 * my) * (w + 2 * mx + 3) + (int64_t)OY * OXP) * 4;
@@ -1576,6 +1635,15 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
     const uint32_t boxB[3] = {(uint32_t)pl->ws_bp, (uint32_t)(p.tmpl_h + 2 * p.search_y), 1u};
     if (!(boxB[0] <= 256 && encode_f32(&mW, B, 3, dims, strides, boxB))) return NCC_ERR_CUDA;
   }
+  CUtensorMap mT;  // tensor-core kernel: search-region rows, box (2 m_x + w, 1, 1)
+  memset(&mT, 0, sizeof(mT));
+  if (pl->ptc) {
+    if (reinterpret_cast<uintptr_t>(B) % 16 != 0) return NCC_ERR_INVALID_ARGUMENT;  // (torch allocations are 256-B aligned)
+    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)p.image_h, (uint64_t)batch};
+    const uint64_t strides[2] = {(uint64_t)p.image_pitch * 4, (uint64_t)fs * 4};
+    const uint32_t box[3] = {(uint32_t)(2 * p.search_x + p.tmpl_w), 1u, 1u};
+    if (!encode_f32(&mT, B, 3, dims, strides, box)) return NCC_ERR_CUDA;
+  }
   const int groups = ceil_div((int64_t)pl->Ky * pl->Kx, v->WPB);
   mark(pl, s, 0);
   for (int sb = 0; sb < nsub; ++sb) {
@@ -1596,7 +1664,46 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
     mark(pl, s, 3 * sb + 1);
     a.pair0 = p0;
     dim3 grid(groups, 1, np);
-    if (use_tma && pl->ws_smem) {
+    if (pl->ptc) {
+      PivTcArgs t;
+      t.A = A;
+      t.pitch = p.image_pitch;
+      t.frame_stride = fs;
+      t.h = p.tmpl_h;
+      t.w = p.tmpl_w;
+      t.my = p.search_y;
+      t.mx = p.search_x;
+      t.sy = p.step_y;
+      t.sx = p.step_x;
+      t.Ky = pl->Ky;
+      t.Kx = pl->Kx;
+      t.pair0 = p0;
+      t.Dx = 2 * p.search_x;
+      t.R = pl->ptc_R;
+      // column strips split into segments so that the launch has ~4 units per SM
+      int nseg = (int)std::min<int64_t>(pl->Ky, std::max<int64_t>(1, ceil_div((int64_t)4 * pl->nsm, (int64_t)np * pl->Kx)));
+      if (const char* e = getenv("NCC_PIV_TC_SEGW")) nseg = ceil_div(pl->Ky, std::max(1, atoi(e)));
+      t.segw = ceil_div(pl->Ky, nseg);
+      t.nseg = ceil_div(pl->Ky, t.segw);
+      t.nunits = np * pl->Kx * t.nseg;
+      t.rsv = pl->tc_rsv;
+      t.mean = pl->tc_mean;
+      t.map_pitch = pl->map_w;
+      t.map_frame_stride = pl->s_frame_stride;
+      t.border = pl->ptc_border;
+      t.vec = reinterpret_cast<VecOut*>(d_vec);
+      t.scores = d_scores;
+      t.subpix = p.subpix;
+      t.prof = pl->ptc_prof;
+      t.nab = std::min(ptc::kNABMax, (512 - ptc::kNSlot * ptc::slot_cols(p.search_y, t.R)) / (2 * ptc::kKc));
+      if (const char* e = getenv("NCC_PIV_TC_NAB")) t.nab = std::max(ptc::kNAB, std::min(t.nab, atoi(e)));
+      t.exp = 0;
+      if (const char* e = getenv("NCC_PIV_TC_EXP")) t.exp = atoi(e);
+      piv_tc_border_kernel<<<dim3(pl->Ky * pl->Kx, np), 256, pl->ptc_border_smem, s>>>(t, B);
+      void* targs[2] = {&t, &mT};
+      const int g = std::min(t.nunits, pl->nsm);
+      NCC_CUDA(cudaLaunchKernel((const void*)piv_tc_kernel, dim3(g), dim3(ptc::kThreads), targs, (size_t)pl->ptc_smem, s));
+    } else if (use_tma && pl->ws_smem) {
       int total = (int)((int64_t)np * pl->Ky * pl->Kx);
       void* wargs[3] = {&a, &mW, &total};
       const int ngroups = ceil_div(total, v->ws_wps);

@@ -85,7 +85,8 @@ def test_cfg3_noisy_subpixel_pair_vs_oracle():
     assert d.max() <= 2e-3 and e.max() <= 2e-3
 
 
-def test_cfg4_two_pairs_sampled():
+def test_cfg4_two_pairs_sampled(monkeypatch):
+    monkeypatch.setenv("NCC_PIV_TC", "0")  # the CUDA-core kernel (tensor cores: test_gpu_piv_tc.py)
     cv, specs = synth.piv_batch_from_canvases(4, 2, canvases=2)
     As, Bs = [], []
     for (ci, ay, ax, by, bx, _) in specs:

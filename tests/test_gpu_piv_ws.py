@@ -23,9 +23,10 @@ from paper_conf_ipps_moorelk13_b200.api import PivPlan, decode_vectors
 pytestmark = pytest.mark.gpu
 TOL = 1e-4
 H, W, h, m, s = 384, 448, 64, 32, 32
-KERNELS = {"ws2": ({}, "piv_ws2_64x64_m32_rv16_c8p8"),
-           "ws": ({"NCC_FORCE_VARIANT": "piv_ws_64x64_m32_rv12_c13p4"}, "piv_ws_64x64_m32_rv12_c13p4"),
-           "ncc": ({"NCC_NO_WS": "1"}, "piv_ws2_64x64_m32_rv16_c8p8")}
+# (NCC_PIV_TC=0: these are the CUDA-core kernels; the tensor-core path has test_gpu_piv_tc.py)
+KERNELS = {"ws2": ({"NCC_PIV_TC": "0"}, "piv_ws2_64x64_m32_rv16_c8p8"),
+           "ws": ({"NCC_PIV_TC": "0", "NCC_FORCE_VARIANT": "piv_ws_64x64_m32_rv12_c13p4"}, "piv_ws_64x64_m32_rv12_c13p4"),
+           "ncc": ({"NCC_PIV_TC": "0", "NCC_NO_WS": "1"}, "piv_ws2_64x64_m32_rv16_c8p8")}
 
 
 @pytest.fixture(scope="module", autouse=True)
