@@ -263,30 +263,44 @@ def max_over_ranks(ctx, x):
     return float(t.item())
 
 
-def roofline(ctx, plan, flops, num_avg, step_ms, clocks, cfg):
+def roofline(ctx, plan, flops, num_avg, step_ms, clocks, cfg, pairs=None):
     """Roofline object of the dominant (numerator) kernel."""
     sms = ctx.sms
     achieved = flops / (num_avg / 1e3) / 1e12
     max_mhz = clocks.get("sm_max_mhz") or 1965.0
     sm_mhz = clocks.get("sm_mhz")
     fp32_peak = sms * 128 * 2 * max_mhz * 1e6 / 1e12
-    tensor = plan.info.variant_name.decode().startswith("tm_tc")
+    vname = plan.info.variant_name.decode()
+    tensor = vname.startswith(("tm_tc", "piv_tc"))
+    kname = ("tm_tc_kernel" if vname.startswith("tm_tc") else
+             "piv_tc_kernel + piv_tc_border_kernel (numerator: tensor cores + its last column)"
+             if vname.startswith("piv_tc") else vname)
     extra = {"fp32_peak": fp32_peak, "frac_of_fp32_peak": achieved / fp32_peak,
              "fp32_peak_note": "SMs x 128 FP32 lanes x 2 FLOP x max SM clock (B200_PROFILING.md unit counts)"}
     if tensor:
-        # 3xTF32 on tcgen05: 3 tf32 MMAs per fp32 MAC.  tf32 peak = measured bf16 GEMM peak x the
-        # nominal tf32/bf16 ratio (1.1 / 2.25 PFLOP/s); the fp32-equivalent peak is a third of it.
         mp = measured_peaks()
         bf16 = mp.get("bf16_tflops") or 1590.0
-        peak = bf16 * (1.1 / 2.25) / 3.0
-        peak_note = (f"3xTF32 fp32-equivalent tensor peak = {'measured' if mp else 'fallback'} bf16 GEMM "
-                     f"{bf16:.1f} TFLOP/s x (tf32/bf16 nominal 1.1/2.25) / 3 MMAs per MAC")
+        if vname.startswith("piv_tc"):
+            # 3xBF16 on tcgen05 (kind::f16): 3 bf16 MMAs per fp32-equivalent MAC
+            peak = bf16 / 3.0
+            peak_note = (f"3xBF16 fp32-equivalent tensor peak = {'measured' if mp else 'fallback'} bf16 GEMM "
+                         f"{bf16:.1f} TFLOP/s / 3 MMAs per MAC")
+            issue_peak = sms * 8192 * max_mhz * 1e6 / 3.0 / 1e12
+            issue_note = ("SMs x 8192 bf16 FLOP/cycle (probe: M=128 K=16 MMA of width N >= 90 takes N/2 cycles; "
+                          "narrower ones 45 cycles) x max SM clock / 3")
+        else:
+            # 3xTF32 on tcgen05: 3 tf32 MMAs per fp32 MAC.  tf32 peak = measured bf16 GEMM peak x the
+            # nominal tf32/bf16 ratio (1.1 / 2.25 PFLOP/s); the fp32-equivalent peak is a third of it.
+            peak = bf16 * (1.1 / 2.25) / 3.0
+            peak_note = (f"3xTF32 fp32-equivalent tensor peak = {'measured' if mp else 'fallback'} bf16 GEMM "
+                         f"{bf16:.1f} TFLOP/s x (tf32/bf16 nominal 1.1/2.25) / 3 MMAs per MAC")
+            # our own issue-rate probe (tools/microbench/umma_probe.cu): a cta_group::1 M=128 tf32
+            # MMA of width N takes N/2 cycles (K=8) = 4096 tf32 FLOP/cycle/SM -- the strict one
+            issue_peak = sms * 4096 * max_mhz * 1e6 / 3.0 / 1e12
+            issue_note = "SMs x 4096 tf32 FLOP/cycle (probe: N=136 MMA = 68 cycles) x max SM clock / 3"
         peak_at_clock = peak * sm_mhz / max_mhz if sm_mhz else None
-        # our own issue-rate probe (tools/microbench/umma_probe.cu): a cta_group::1 M=128 tf32
-        # MMA of width N takes N/2 cycles (K=8) = 4096 tf32 FLOP/cycle/SM -- the strict one
-        issue_peak = sms * 4096 * max_mhz * 1e6 / 3.0 / 1e12
         extra.update({"issue_rate_peak": issue_peak, "frac_of_issue_rate": achieved / issue_peak,
-                      "issue_rate_note": "SMs x 4096 tf32 FLOP/cycle (probe: N=136 MMA = 68 cycles) x max SM clock / 3"})
+                      "issue_rate_note": issue_note})
         bound = "tensor"
     else:
         peak = fp32_peak
@@ -299,14 +313,15 @@ def roofline(ctx, plan, flops, num_avg, step_ms, clocks, cfg):
         try:
             tj = json.load(open(prof))
             traffic = tj.get(f"cfg{cfg}_tc" if tensor else f"cfg{cfg}")
-            if traffic is None and f"cfg{cfg}_per_pair" in tj:
-                traffic = tj[f"cfg{cfg}_per_pair"] * plan.info.grid_z
+            pp = f"cfg{cfg}_tc_per_pair" if tensor else f"cfg{cfg}_per_pair"
+            if traffic is None and pp in tj and pairs:  # per call, like `achieved`
+                traffic = tj[pp] * pairs
         except Exception:
             traffic = None
     return {"bound": bound, "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
             "traffic": traffic, "peak_note": peak_note,
             "frac_at_sampled_clock": (achieved / peak_at_clock) if peak_at_clock else None,
-            "kernel": "tm_tc_kernel" if tensor else plan.info.variant_name.decode(),
+            "kernel": kname,
             "kernel_ms": num_avg, "kernel_share_of_step": num_avg / step_ms, **extra}
 
 
@@ -412,7 +427,8 @@ def measure(ctx, cfg, steps, warmup, headline=True, cpu_budget=10.0):
     sec = total_ms / 1e3
     value = units_all * steps / sec
     num_avg = sum(num_ms) / len(num_ms)
-    rl = roofline(ctx, plan, plan.info.flops_per_call, num_avg, total_ms / steps, clocks, cfg)
+    rl = roofline(ctx, plan, plan.info.flops_per_call, num_avg, total_ms / steps, clocks, cfg,
+                  pairs=wl.get("pairs") if kind == "piv" else None)
     tensor = rl["bound"] == "tensor"
 
     # end to end through the host-buffer C-ABI call (H2D + compute + D2H in the region)
@@ -453,8 +469,11 @@ def measure(ctx, cfg, steps, warmup, headline=True, cpu_budget=10.0):
     line = {"metric": metric, "value": value, "unit": unit, "n_gpus": ws if multi else 1, "steps": steps,
             "warmup": warmup, "ms_per_step": total_ms / steps, "higher_is_better": True,
             "scaling": "strong" if (multi and (cfg == 4 or bands)) else "weak", "vs_baseline": None,
-            "dtype": "tf32x3" if tensor else "f32",
-            "arith": ("3xTF32 on tcgen05 tensor cores (fp32-emulated: hi*hi + hi*lo + lo*hi, fp32 accumulate); "
+            "dtype": ("bf16x3" if rl["kernel"].startswith("piv_tc") else "tf32x3") if tensor else "f32",
+            "arith": (("3xBF16 on tcgen05 tensor cores (kind::f16, fp32-emulated: hi*hi + hi*lo + lo*hi with "
+                       "hi = bf16(x), lo = bf16(x - hi), fp32 accumulate); last output column on FFMA; "
+                       "fp64 window sums, fp64 variance") if rl["kernel"].startswith("piv_tc") else
+                      "3xTF32 on tcgen05 tensor cores (fp32-emulated: hi*hi + hi*lo + lo*hi, fp32 accumulate); "
                       "fp64 window sums, fp64 variance") if tensor else
                      "fp32 FFMA numerator; fp64 window sums, fp64 variance",
             "data": "synthetic",

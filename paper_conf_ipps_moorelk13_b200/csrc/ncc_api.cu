@@ -1086,10 +1086,10 @@ ncc_status create_piv(ncc_plan pl) {
     const char* e = getenv("NCC_PIV_TC");
     const int Dx = 2 * mx, R = (Dx == 32 || Dx == 64) ? 128 / Dx : 1, span = h + 2 * my;
     const bool ok = p.score == NCC_SCORE_NCC && !(p.flags & NCC_F_CUDA_CORES) && !(e && atoi(e) == 0) &&
-                    (Dx == 32 || Dx == 64) && w % ptc::kKc == 0 && (h * w) % 128 == 0 &&
+                    (Dx == 32 || Dx == 64) && w % ptc::kKs == 0 && (h * w) % 128 == 0 &&
                     h * w <= 128 * ptc::kPrepMax && p.step_y % R == 0 && p.step_y <= span &&
                     (span + p.step_y - 1) / p.step_y <= ptc::kNSlot - 1 && p.step_x % 4 == 0 &&
-                    p.image_pitch % 4 == 0 && Dx + w <= 256 && ptc::tmem_cols(my, R) <= 512 &&
+                    p.image_pitch % 4 == 0 && Dx + w <= 256 && ptc::tmem_cols(my, R, w) <= 512 &&
                     ptc::smem_bytes(h, w, my, mx) <= maxsm && (2 * my + 1) * (2 * mx + 1) <= 128 * ptc::kEpiMax &&
                     2 * my + 1 <= 8 * kBorderDY;
     // default: the tensor cores where they measured faster (R = 2, +-32 search: cfg 4, 1.6x);
@@ -1134,7 +1134,7 @@ ncc_status create_piv(ncc_plan pl) {
   if (pl->ptc) {  // per sub-batch: window sums, last-column kernel, tensor-core kernel
     int nsm = 0;
     NCC_CUDA(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, pl->device));
-    snprintf(in.variant_name, sizeof(in.variant_name), "piv_tc_tf32x3_%dx%d_m%dx%d_r%d", h, w, my, mx, pl->ptc_R);
+    snprintf(in.variant_name, sizeof(in.variant_name), "piv_tc_bf16x3_%dx%d_m%dx%d_r%d", h, w, my, mx, pl->ptc_R);
     fill_kernel_info(pl, (const void*)piv_tc_kernel, ptc::kThreads, pl->ptc_smem, nsm, 1, 1);
     in.specialized = 3;
     in.variant_id = -1;
@@ -1695,7 +1695,7 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
       t.scores = d_scores;
       t.subpix = p.subpix;
       t.prof = pl->ptc_prof;
-      t.nab = std::min(ptc::kNABMax, (512 - ptc::kNSlot * ptc::slot_cols(p.search_y, t.R)) / (2 * ptc::kKc));
+      t.nab = std::min(ptc::kNABMax, (512 - ptc::kNSlot * ptc::slot_cols(p.search_y, t.R)) / ptc::chunk_cols(p.tmpl_w));
       if (const char* e = getenv("NCC_PIV_TC_NAB")) t.nab = std::max(ptc::kNAB, std::min(t.nab, atoi(e)));
       t.exp = 0;
       if (const char* e = getenv("NCC_PIV_TC_EXP")) t.exp = atoi(e);

@@ -1,4 +1,4 @@
-// ncc_piv_tc.cuh -- tensor-core (tcgen05, kind::tf32, 3xTF32) numerator of the PIV path
+// ncc_piv_tc.cuh -- tensor-core (tcgen05, kind::f16, 3xBF16) numerator of the PIV path
 // (SURVEY 8(f) row f3 extended to the batched PIV correlation of Figs 5.9-5.12).
 //
 // What it computes: for every interrogation window (mask T = frame A at (y, x), h x w) the
@@ -22,41 +22,60 @@
 //     ceil((h + 2 m_y) / s_y) = 4 at cfg 3 / 4), each into its own accumulator slot (kNSlot
 //     slots: the live windows + one being drained); the operand is built once per image row,
 //     not once per window.
-//   * 3xTF32: x = hi + lo (hi = tf32(x), lo = x - hi exact); A.B ~ A_hi.B_hi + A_hi.B_lo + A_lo.B_hi.
+//   * 3xBF16 (kind::f16, K = 16 per MMA): x = hi + lo + r with hi = bf16(x), lo = bf16(x - hi),
+//     |r| <= 2^-17 |x|; A.B ~ A_hi.B_hi + A_hi.B_lo + A_lo.B_hi (each bf16 product exact in the fp32
+//     accumulator).  Per-product error ~2^-16 relative, random in sign: over the h w products of a
+//     window ~2^-16 / sqrt(h w) of the normalisation (1e-7 at 64 x 64) -- and a bf16 MMA does K = 16
+//     in the time a tf32 MMA does K = 8 (an M = 128 MMA takes max(45, N / 2) cycles either way,
+//     tools/microbench/umma_probe.cu rates; this kernel's N is <= 80), so half the MMAs of 3xTF32.
 //   * The last output column dx = 2 m_x (D_x + 1 columns do not fit R D_x = 128 lanes) comes from
 //     a CUDA-core kernel (piv_tc_border_kernel) that runs before this one.
 // Warp roles: 0-3 producers (Hankel operand -> TMEM, lane quadrant w), 4-7 drain / epilogue
-// (accumulators -> shared surface, normalisation, argmax, sub-pixel), 8-11 mask prep (statistics,
-// centred hi/lo reversed operand), 12 TMA (search-region rows), 13 MMA issuer.
+// (accumulators -> shared surface, normalisation, argmax, sub-pixel), 8, 10, 11, 12 mask prep
+// (statistics, centred hi/lo reversed operand), 9 TMA (search-region rows), 13-14 MMA issuers.
 #pragma once
+#include <cuda_bf16.h>
 #include "ncc_tc.cuh"
 
 namespace nccb {
 namespace ptc {
 constexpr int kNSlot = 5;   // accumulator + mask-operand slots (live windows + 1)
-constexpr int kKc = 16;     // template columns per TMEM A chunk (hi 16 + lo 16 columns)
+constexpr int kKs = 16;     // template columns per MMA K-step (bf16); a TMEM A chunk holds kc = 16 or 32
+                            // of them (kc / 2 columns hi + kc / 2 lo: two bf16 per 32-bit column)
 constexpr int kNAB = 3;     // TMEM A buffers (minimum; up to kNABMax when the accumulators leave room)
 constexpr int kNABMax = 8;
 constexpr int kNRing = 4;   // search-region row groups in flight (TMA)
 constexpr int kNStat = 8;   // mask-statistics slots (prep -> epilogue), deeper than the operand slots
-constexpr int kEpiWarp0 = 4, kTmaWarp = 9, kMmaWarp = 13;
+constexpr int kEpiWarp0 = 4, kTmaWarp = 9, kMmaWarp = 13, kNMma = 3;  // MMA warps 13 .. 12 + kNMma
 // mask-prep warps 8, 10, 11, 12: none on the MMA warp's SMSP (warp % 4 == 1), whose issue slots
 // the tensor pipe waits for; the TMA warp (nearly idle) takes warp 9
 __host__ __device__ constexpr bool is_prep_warp(int w) { return w == 8 || w == 10 || w == 11 || w == 12; }
 __host__ __device__ constexpr int prep_index(int w) { return w == 8 ? 0 : w - 9; }
-constexpr int kThreads = 14 * 32;
+constexpr int kThreads = (kMmaWarp + kNMma) * 32;
 constexpr int kPrepMax = 32;  // mask elements per prep thread (h w <= 4096)
 constexpr int kEpiB = 12, kEpiNB = 3, kEpiMax = kEpiB * kEpiNB;  // outputs per epilogue thread, in batches of kEpiB
 __host__ __device__ constexpr int slot_cols(int my, int R) { return ((2 * my + R + 8) + 7) / 8 * 8; }
 __host__ __device__ constexpr int b_rows(int h) { return h + 8; }  // 1 zero row + h + 7 zero rows
-__host__ __device__ constexpr int b_slot_bytes(int h, int w) { return 2 * (w / 4) * b_rows(h) * 16; }
+__host__ __device__ constexpr int b_slot_bytes(int h, int w) { return 2 * (w / 8) * b_rows(h) * 16; }  // bf16 hi + lo
 __host__ __device__ constexpr int ring_pitch(int Dx, int w) { return ((Dx + w + 31) / 32) * 32; }  // floats (128 B rows)
 __host__ __device__ constexpr int surf_pitch(int mx) { return ((2 * mx + 1) + 3) / 4 * 4; }
 __host__ __device__ constexpr int smem_bytes(int h, int w, int my, int mx) {
   return kNSlot * b_slot_bytes(h, w) + kNRing * (128 / (2 * mx)) * ring_pitch(2 * mx, w) * 4 +
          (2 * my + 1) * surf_pitch(mx) * 4;
 }
-__host__ __device__ constexpr int tmem_cols(int my, int R) { return kNSlot * slot_cols(my, R) + kNAB * 2 * kKc; }
+__host__ __device__ constexpr int chunk_cols(int w) { return w % 32 == 0 ? 32 : 16; }  // kc: TMEM columns = elements
+__host__ __device__ constexpr int tmem_cols(int my, int R, int w) { return kNSlot * slot_cols(my, R) + kNAB * chunk_cols(w); }
+// kind::f16 instruction descriptor: D f32, A/B bf16, both K-major, M = 128
+__host__ __device__ constexpr uint32_t idesc_bf16(int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+}
+__device__ __forceinline__ void mma_bf16_ts(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t idesc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, 1, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d),
+      "r"(a_tmem), "l"(b), "r"(idesc)
+      : "memory");
+}
 }  // namespace ptc
 
 struct PivTcArgs {
@@ -110,7 +129,7 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
   const int h = a.h, w = a.w, R = a.R, Dx = a.Dx;
   const int OY = 2 * a.my + 1, OX = 2 * a.mx + 1, OXP = surf_pitch(a.mx);
-  const int SW = slot_cols(a.my, R), LB = b_rows(h), npl = w / 4, nkc = w / kKc;
+  const int SW = slot_cols(a.my, R), LB = b_rows(h), npl = w / 8, kc = chunk_cols(w), nkc = w / kc;
   const int bslot = b_slot_bytes(h, w);
   const int BPr = ring_pitch(Dx, w);
   const int span = h + 2 * a.my;  // search-region rows of one window
@@ -135,7 +154,7 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
     }
     for (int b = 0; b < kNABMax; ++b) {
       mbar_init(&a_full[b], 128);
-      mbar_init(&a_free[b], 1);
+      mbar_init(&a_free[b], kNMma);  // one commit per MMA warp
     }
     for (int b = 0; b < kNSlot; ++b) {
       mbar_init(&b_full[b], 128);
@@ -198,25 +217,41 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
       for (int g = 0; g < ng; ++g, ++gq) {
         const int rs = gq & (kNRing - 1);
         twait(&img_full[rs], (uint32_t)((gq / kNRing) & 1), 0);
-        const float* row = ring + (rs * R + s) * BPr + dx;
+        const float* row0 = ring + (rs * R + s) * BPr + (dx & ~1);
+        const bool odd = (dx & 1) != 0;
         for (int q = 0; q < nkc; ++q, ++cq) {
-          uint32_t hi[kKc], lo[kKc];
+          // kc elements -> kc / 2 columns of (bf16 hi) pairs and kc / 2 of (bf16 lo) pairs, the even
+          // element in the low half of each 32-bit cell
+          // 8-byte loads from the even column at or below dx + j (lanes 2i and 2i+1 share them),
+          // odd lanes take the pair shifted by one; packed conversions (cvt.rn.bf16x2.f32)
+          uint32_t hi[16], lo[16];
+          const float2* r2 = reinterpret_cast<const float2*>(row0 + q * kc);
+          float2 cur = (a.exp & 1) ? make_float2(0.f, 0.f) : r2[0];
 #pragma unroll
-          for (int jj = 0; jj < kKc; ++jj) {
-            const float x = (a.exp & 1) ? 0.0f : row[q * kKc + jj];
-            hi[jj] = tc::to_tf32(x);
-            lo[jj] = __float_as_uint(x - __uint_as_float(hi[jj]));
+          for (int p = 0; p < 16; ++p) {
+            if (2 * p < kc) {
+              const float2 nxt = (a.exp & 1) ? make_float2(0.f, 0.f) : r2[p + 1];
+              const float x0 = odd ? cur.y : cur.x, x1 = odd ? nxt.x : cur.y;
+              cur = nxt;
+              const __nv_bfloat162 hv = __floats2bfloat162_rn(x0, x1);
+              const uint32_t hu = *reinterpret_cast<const uint32_t*>(&hv);
+              const __nv_bfloat162 lv =
+                  __floats2bfloat162_rn(x0 - __uint_as_float(hu << 16), x1 - __uint_as_float(hu & 0xffff0000u));
+              hi[p] = hu;
+              lo[p] = *reinterpret_cast<const uint32_t*>(&lv);
+            }
           }
           if (cq >= nab) {  // the buffer's previous chunk (one round back) consumed
             twait(&a_free[b], (uint32_t)(ph ^ 1), 1);
             tc::fence_after();
           }
-          const uint32_t ab = tbase + lane_base + acol0 + (uint32_t)(b * 2 * kKc);
+          const uint32_t ab = tbase + lane_base + acol0 + (uint32_t)(b * kc);
           if (!(a.exp & 1)) {
-#pragma unroll
-            for (int c = 0; c < kKc; c += 8) {
-              tc::st8(ab + c, *reinterpret_cast<const uint32_t(*)[8]>(hi + c));
-              tc::st8(ab + kKc + c, *reinterpret_cast<const uint32_t(*)[8]>(lo + c));
+            tc::st8(ab, *reinterpret_cast<const uint32_t(*)[8]>(hi));
+            tc::st8(ab + kc / 2, *reinterpret_cast<const uint32_t(*)[8]>(lo));
+            if (kc == 32) {
+              tc::st8(ab + 8, *reinterpret_cast<const uint32_t(*)[8]>(hi + 8));
+              tc::st8(ab + 24, *reinterpret_cast<const uint32_t(*)[8]>(lo + 8));
             }
           }
           tc::st_wait();
@@ -293,8 +328,8 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
         const int st = wseq % kNStat, su = wseq / kNStat;
         if (use >= 1) twait(&win_done[sl], (uint32_t)((use - 1) & 1), 0);
         if (su >= 1) twait(&epi_done[st], (uint32_t)((su - 1) & 1), 1);
-        float* bh = reinterpret_cast<float*>(smem_pt + sl * bslot);
-        float* bl = bh + npl * LB * 4;
+        uint16_t* bh = reinterpret_cast<uint16_t*>(smem_pt + sl * bslot);
+        uint16_t* bl = bh + npl * LB * 8;
         double en = 0.0, cs = 0.0;
 #pragma unroll
         for (int k = 0; k < kPrepMax; ++k) {
@@ -304,10 +339,10 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
             const float ac = (float)d;
             en += d * d;
             cs += (double)ac;
-            const uint32_t hb = tc::to_tf32(ac);
-            const int off = ((j >> 2) * LB + (h - ii)) * 4 + (j & 3);  // row q = h - 1 - i, +1 pre-pad row
-            bh[off] = __uint_as_float(hb);
-            bl[off] = ac - __uint_as_float(hb);
+            const __nv_bfloat16 hb = __float2bfloat16_rn(ac);
+            const int off = ((j >> 3) * LB + (h - ii)) * 8 + (j & 7);  // row q = h - 1 - i, +1 pre-pad row
+            bh[off] = __bfloat16_as_ushort(hb);
+            bl[off] = __bfloat16_as_ushort(__float2bfloat16_rn(ac - __bfloat162float(hb)));
           }
         }
         reduce2(en, cs);
@@ -466,7 +501,7 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
         if (et == 0) mbar_arrive(&epi_done[st]);
       }
     }
-  } else if (warp == kMmaWarp) {
+  } else if (warp >= kMmaWarp) {
     // ===================== MMA issuer.  The whole warp walks the schedule (warp-uniform values
     // stay in uniform registers), one elected lane issues.  Per row group each live window's
     // operands follow from its row offset t = R k alone (a few integer operations); per K chunk
@@ -477,19 +512,24 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
     const uint32_t plane = (uint32_t)LB * 16;
     const uint64_t dconst = tc::sdesc(0u, plane, 128);
     const uint64_t lo_off = (uint64_t)(((uint32_t)npl * LB * 16) >> 4);  // hi -> lo operand (descriptor units)
-    const uint64_t kstep = (uint64_t)((2u * plane) >> 4);                 // one K-step of 8 = two planes
-    const uint64_t qstep = (uint64_t)(((uint32_t)(kKc / 4) * plane) >> 4);  // one K chunk
+    const uint64_t kstep = (uint64_t)((2u * plane) >> 4);                 // one K-step of 16 = two planes of 8
+    const uint64_t qstep = (uint64_t)(((uint32_t)(kc / 8) * plane) >> 4);   // one K chunk
     const int gpw = a.sy / R;  // row groups between two window starts
+    // kNMma issuing warps share the live windows by sequence parity: every accumulator is written
+    // by one warp only, in its fixed order (deterministic); each warp releases the A buffers
+    const int mpar = warp - kMmaWarp;
     int b = 0, ph = 0, wseq = 0, ntr = 0;
     for (int u = blockIdx.x; u < a.nunits; u += gridDim.x) {
       const PivTcUnit un = piv_tc_unit(a, u);
       const int ng = ((un.nw - 1) * a.sy + span + R - 1) / R;
       // live windows, oldest first: slot, slot use, accumulator base, operand base, first group
       int wsl[kNSlot - 1], wuse[kNSlot - 1], wg0[kNSlot - 1];
+      bool wmine[kNSlot - 1];
       uint32_t wdb[kNSlot - 1], wbb[kNSlot - 1];
 #pragma unroll
       for (int li = 0; li < kNSlot - 1; ++li) {
         wsl[li] = wuse[li] = wg0[li] = 0;
+        wmine[li] = false;
         wdb[li] = wbb[li] = 0u;
       }
       int nlive = 0, inext = 0;
@@ -501,6 +541,7 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
               const int sl = wseq % kNSlot;
               wsl[li] = sl;
               wuse[li] = wseq / kNSlot;
+              wmine[li] = (wseq % kNMma) == mpar;
               wg0[li] = g;
               wdb[li] = tbase + (uint32_t)(sl * SW);
               wbb[li] = bsm + (uint32_t)(sl * bslot);
@@ -518,7 +559,7 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
           const int c_lo = c_a - ((c_a + R) & 1);  // even accumulator column
           const int N = ((c_b - c_lo + 1) + 7) & ~7;
           dcol[li] = wdb[li] + (uint32_t)(c_lo + R);
-          idd[li] = tc::idesc_tf32(N);
+          idd[li] = idesc_bf16(N);
           // B row of column c_lo: template row t - c_lo (+1 pre-pad row)
           dh0[li] = dconst + (uint64_t)((wbb[li] + (uint32_t)(h - t + c_lo) * 16u) >> 4);
         }
@@ -528,10 +569,10 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
           twait(&a_full[b], (uint32_t)ph, 0);
           const unsigned long long tq = prof ? pclock() : 0ull;
           tc::fence_after();
-          const uint32_t ah0 = tbase + acol0 + (uint32_t)(b * 2 * kKc);
+          const uint32_t ah0 = tbase + acol0 + (uint32_t)(b * kc);
 #pragma unroll
           for (int li = 0; li < kNSlot - 1; ++li) {
-            if (li >= nlive) continue;
+            if (li >= nlive || !wmine[li]) continue;
             if (q == 0 && g == wg0[li]) {  // the window's first MMA: operand prepared, accumulator slot drained
               twait(&b_full[wsl[li]], (uint32_t)(wuse[li] & 1), 1);
               if (wuse[li] >= 1) twait(&d_free[wsl[li]], (uint32_t)((wuse[li] - 1) & 1), 2);
@@ -540,23 +581,23 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
             if (leader && !(a.exp & 8)) {
               uint64_t dh = dh0[li] + qoff;
 #pragma unroll
-              for (int kk = 0; kk < kKc / 8; ++kk, dh += kstep) {
+              for (int kk = 0; kk < kc / kKs; ++kk, dh += kstep) {
                 const uint32_t ah = ah0 + (uint32_t)(kk * 8);
-                tc::mma_ts(dcol[li], ah, dh, idd[li]);
-                tc::mma_ts(dcol[li], ah, dh + lo_off, idd[li]);
-                tc::mma_ts(dcol[li], ah + kKc, dh, idd[li]);
+                mma_bf16_ts(dcol[li], ah, dh, idd[li]);
+                mma_bf16_ts(dcol[li], ah, dh + lo_off, idd[li]);
+                mma_bf16_ts(dcol[li], ah + kc / 2, dh, idd[li]);
               }
             }
           }
           if (leader) {
             tc::commit(&a_free[b]);
-            if (q == nkc - 1 && nlive > 0 && g - wg0[0] == KT - 1) tc::commit(&win_done[wsl[0]]);
+            if (q == nkc - 1 && nlive > 0 && wmine[0] && g - wg0[0] == KT - 1) tc::commit(&win_done[wsl[0]]);
           }
           __syncwarp();
           if (prof) {
             const unsigned long long te = pclock();
             pacc[3] += te - tq;
-            if (blockIdx.x == 0 && lane == 0 && ntr < 2048) {  // trace of CTA 0's first chunks
+            if (blockIdx.x == 0 && lane == 0 && warp == kMmaWarp && ntr < 2048) {  // trace of CTA 0's first chunks
               prof[gridDim.x * 32 + 3 * ntr] = tw;
               prof[gridDim.x * 32 + 3 * ntr + 1] = tq;
               prof[gridDim.x * 32 + 3 * ntr + 2] = te;
@@ -573,6 +614,7 @@ __global__ void __launch_bounds__(ptc::kThreads, 1) piv_tc_kernel(const PivTcArg
           for (int li = 0; li < kNSlot - 2; ++li) {
             wsl[li] = wsl[li + 1];
             wuse[li] = wuse[li + 1];
+            wmine[li] = wmine[li + 1];
             wg0[li] = wg0[li + 1];
             wdb[li] = wdb[li + 1];
             wbb[li] = wbb[li + 1];

@@ -1,4 +1,4 @@
-"""GPU parity: the tensor-core PIV numerator (piv_tc_kernel, tcgen05 kind::tf32 3xTF32, R image
+"""GPU parity: the tensor-core PIV numerator (piv_tc_kernel, tcgen05 kind::f16 3xBF16, R image
 rows per MMA) through the C ABI vs the fp64 oracle.
 
 Same bar as the CUDA-core PIV tests: window score surfaces within 1e-4 element by
@@ -65,7 +65,7 @@ def test_cfg3_planted_all_windows_on_tensor_cores():
     dy, dx = synth.piv_shift_for_pair(3, 0)
     p = synth.particle_pair_integer(c["H"], c["W"], dy, dx, seed=3000)
     v, sc, info = run([p.A], [p.B], 32, 16, 16)
-    assert info["variant_name"].startswith("piv_tc_tf32x3_32x32_m16x16_r4"), info["variant_name"]
+    assert info["variant_name"].startswith("piv_tc_bf16x3_32x32_m16x16_r4"), info["variant_name"]
     assert info["specialized"] == 3
     assert np.all(v["iy"] == dy) and np.all(v["ix"] == dx)
     assert np.all(np.abs(v["score"] - 1.0) <= TOL)
@@ -84,7 +84,7 @@ def test_cfg4_geometry_all_windows_two_pairs():
         As.append(cv[ci][ay:ay + 384, ax:ax + 384])
         Bs.append(cv[ci][by:by + 384, bx:bx + 384])
     v, sc, info = run(As, Bs, 64, 32, 32)
-    assert info["variant_name"].startswith("piv_tc_tf32x3_64x64_m32x32_r2"), info["variant_name"]
+    assert info["variant_name"].startswith("piv_tc_bf16x3_64x64_m32x32_r2"), info["variant_name"]
     Ky, Kx = oracle.piv_grid(384, 384, 64, 64, 32, 32, 32, 32)
     assert v["iy"].shape == (2, Ky, Kx)
     for pi, (_, _, _, _, _, (dy, dx)) in enumerate(specs):
@@ -192,6 +192,6 @@ def test_default_selection(monkeypatch):
     faster) and the CUDA-core kernel at +-16."""
     monkeypatch.delenv("NCC_PIV_TC", raising=False)
     with PivPlan(512, 512, 64, 32, 32, pairs=1) as plan:
-        assert plan.info.variant_name.decode().startswith("piv_tc_tf32x3_64x64_m32x32_r2")
+        assert plan.info.variant_name.decode().startswith("piv_tc_bf16x3_64x64_m32x32_r2")
     with PivPlan(512, 512, 32, 16, 16, pairs=1) as plan:
         assert plan.info.variant_name.decode().startswith("piv_ws2")

@@ -823,8 +823,96 @@ static void rate_k(int mode, int threads = 128, int smem = 150000) {
   cudaFree(cyc);
 }
 
+
+// ---- bf16 (kind::f16) M=128 K=16 MMA rate with A in TMEM: 2 bf16 per 32-bit TMEM column
+__host__ __device__ constexpr uint32_t idesc_bf16(int M, int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+__device__ __forceinline__ void mma_f16_ts(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}\n" ::"r"(d),
+      "r"(a_tmem), "l"(b), "r"(idesc), "r"(acc));
+}
+template <int N>
+__global__ void rate_bf16_ts_kernel(int iters, float* sink, long long* cycles) {
+  extern __shared__ __align__(1024) unsigned char sm[];
+  __shared__ uint64_t bar;
+  __shared__ uint32_t tbase;
+  constexpr int K = 64;  // bf16 elements
+  uint16_t* Bs = reinterpret_cast<uint16_t*>(sm);
+  const int tid = threadIdx.x, warp = tid >> 5;
+  for (int e = tid; e < (K / 8) * N * 8; e += blockDim.x) Bs[e] = (uint16_t)(0x3c00 + (e % 97));
+  fence_async_smem();
+  if (warp == 0) tmem_alloc<512>(&tbase);
+  if (tid == 0) { mbar_init(&bar, 1); asm volatile("fence.mbarrier_init.release.cluster;"); }
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t d = tbase;
+  const uint32_t lane_base = (uint32_t)(warp * 32) << 16;
+  float z[8] = {0.5f, 0.25f, 0.125f, 1.f, 2.f, 3.f, 4.f, 5.f};
+  for (int c = 0; c < K / 2; c += 8) tmem_st8(d + lane_base + 256 + c, z);
+  tmem_st_wait();
+  fence_before();
+  __syncthreads();
+  fence_after();
+  long long t0 = clock64();
+  if (tid == 0) {
+    for (int it = 0; it < iters; ++it)
+      for (int kk = 0; kk < K / 16; ++kk) {
+        const uint64_t b = sdesc(su32(Bs) + kk * 2 * N * 16, N * 16, 128);
+        mma_f16_ts(d, d + 256 + kk * 8, b, idesc_bf16(128, N), (it | kk) > 0);
+      }
+    mma_commit(&bar);
+  }
+  mbar_wait(&bar, 0);
+  long long t1 = clock64();
+  fence_after();
+  if (tid == 0) cycles[blockIdx.x] = t1 - t0;
+  float v[8];
+  tmem_ld8(d + lane_base, v);
+  if (v[0] == 12345.f) sink[tid] = v[1];
+  fence_before();
+  __syncthreads();
+  if (warp == 0) tmem_free<512>(d);
+}
+template <int N>
+static void rate_bf16_ts() {
+  constexpr int K = 64;
+  const int smem = N * K * 2;
+  CK(cudaFuncSetAttribute(rate_bf16_ts_kernel<N>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  float* sink;
+  long long* cyc;
+  int nsm = 0;
+  CK(cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, 0));
+  CK(cudaMalloc(&sink, 4096));
+  CK(cudaMalloc(&cyc, nsm * 8));
+  const int iters = 2000;
+  rate_bf16_ts_kernel<N><<<nsm, 128, smem>>>(10, sink, cyc);
+  CK(cudaDeviceSynchronize());
+  rate_bf16_ts_kernel<N><<<nsm, 128, smem>>>(iters, sink, cyc);
+  CK(cudaDeviceSynchronize());
+  std::vector<long long> c(nsm);
+  CK(cudaMemcpy(c.data(), cyc, nsm * 8, cudaMemcpyDeviceToHost));
+  double avg = 0;
+  for (auto x : c) avg += x;
+  avg /= nsm;
+  printf("{\"probe\": \"rate_bf16_ts\", \"N\": %d, \"cycles_per_mma\": %.2f, \"floor_cycles\": %.1f}\n", N,
+         avg / ((double)iters * (K / 16)), 128.0 * N / 256.0);
+  cudaFree(sink);
+  cudaFree(cyc);
+}
+
 int main(int argc, char** argv) {
   setvbuf(stdout, nullptr, _IONBF, 0);
+  if (argc > 1 && strcmp(argv[1], "rates") == 0) {  // cycles per M=128 K=8 tf32 MMA vs N, A from smem / TMEM
+    rate<16>(0); rate<32>(0); rate<48>(0); rate<64>(0); rate<80>(0); rate<136>(0); rate<256>(0);
+    rate_ts<16>(); rate_ts<32>(); rate_ts<48>(); rate_ts<64>(); rate_ts<80>(); rate_ts<136>(); rate_ts<256>();
+    rate_bf16_ts<16>(); rate_bf16_ts<32>(); rate_bf16_ts<48>(); rate_bf16_ts<64>(); rate_bf16_ts<80>();
+    rate_bf16_ts<136>(); rate_bf16_ts<256>();
+    return 0;
+  }
   rate_k(0, 576, 125000);
   rate_k(128, 576, 125000);
   rate_k(128 | 1024, 576, 125000);  // busy warps only on the other three SMSPs
