@@ -280,7 +280,7 @@ def roofline(ctx, plan, flops, num_avg, step_ms, clocks, cfg, pairs=None):
     if tensor:
         mp = measured_peaks()
         bf16 = mp.get("bf16_tflops") or 1590.0
-        if vname.startswith("piv_tc"):
+        if vname.startswith(("piv_tc", "tm_tc_bf16")):
             # 3xBF16 on tcgen05 (kind::f16): 3 bf16 MMAs per fp32-equivalent MAC
             peak = bf16 / 3.0
             peak_note = (f"3xBF16 fp32-equivalent tensor peak = {'measured' if mp else 'fallback'} bf16 GEMM "
@@ -469,12 +469,11 @@ def measure(ctx, cfg, steps, warmup, headline=True, cpu_budget=10.0):
     line = {"metric": metric, "value": value, "unit": unit, "n_gpus": ws if multi else 1, "steps": steps,
             "warmup": warmup, "ms_per_step": total_ms / steps, "higher_is_better": True,
             "scaling": "strong" if (multi and (cfg == 4 or bands)) else "weak", "vs_baseline": None,
-            "dtype": ("bf16x3" if rl["kernel"].startswith("piv_tc") else "tf32x3") if tensor else "f32",
-            "arith": (("3xBF16 on tcgen05 tensor cores (kind::f16, fp32-emulated: hi*hi + hi*lo + lo*hi with "
-                       "hi = bf16(x), lo = bf16(x - hi), fp32 accumulate); last output column on FFMA; "
-                       "fp64 window sums, fp64 variance") if rl["kernel"].startswith("piv_tc") else
-                      "3xTF32 on tcgen05 tensor cores (fp32-emulated: hi*hi + hi*lo + lo*hi, fp32 accumulate); "
-                      "fp64 window sums, fp64 variance") if tensor else
+            "dtype": "bf16x3" if tensor else "f32",
+            "arith": ("3xBF16 on tcgen05 tensor cores (kind::f16, fp32-emulated: hi*hi + hi*lo + lo*hi with "
+                      "hi = bf16(x), lo = bf16(x - hi), fp32 accumulate)" +
+                      ("; last output column on FFMA" if rl["kernel"].startswith("piv_tc") else
+                       "; ragged last columns on FFMA") + "; fp64 window sums, fp64 variance") if tensor else
                      "fp32 FFMA numerator; fp64 window sums, fp64 variance",
             "data": "synthetic",
             "frames_per_s" if kind == "tm" else "pairs_per_s": frames_all * steps / sec,

@@ -605,7 +605,7 @@ ncc_status setup_tc(ncc_plan pl) {
   const int nsub = p.batch * (roi ? pl->n_tmpl : 1);
   // a ragged last column tile of at most kTcColsMax columns goes to tm_tc_cols instead of a
   // whole column of tensor-core CTAs
-  pl->tc_vtiles = ceil_div(roi ? cols + 1 : cols, 128);  // ROI tiles start at the even column <= the origin
+  pl->tc_vtiles = ceil_div(roi ? cols + 3 : cols, 128);  // ROI tiles start at the column <= the origin that is a multiple of 4
   pl->tc_vcols = 0;
   // launch order (measured on B200, cfg2 step: 0 -> 0.2135 ms, 3 -> 0.2074 ms; 1/2 delay the
   // tensor-core kernel's start or starve the ragged-column kernel); NCC_TM_SCHED overrides
@@ -693,7 +693,7 @@ ncc_status setup_tc(ncc_plan pl) {
   if ((st = dalloc(&pl->tc_ticket, (size_t)1))) return st;
   NCC_CUDA(cudaMemset(pl->tc_ticket, 0, sizeof(unsigned long long)));
   // (hi, lo) pairs, rows padded to an even count of pairs: a 16-byte multiple for the TMA map
-  if ((st = dalloc(&pl->tc_img2, (size_t)2 * p.batch * pl->Hs * ((p.image_w + 1) & ~1)))) return st;
+  if ((st = dalloc(&pl->tc_img2, (size_t)p.batch * pl->Hs * ((p.image_w + 3) & ~3)))) return st;
   if (p.score == NCC_SCORE_NCC) {  // per-offset fp32 normalisation factors (window-sum kernels)
     if ((st = dalloc(&pl->tc_rsv, (size_t)p.batch * pl->s_frame_stride))) return st;
     if ((st = dalloc(&pl->tc_mean, (size_t)p.batch * pl->s_frame_stride))) return st;
@@ -706,7 +706,7 @@ ncc_status setup_tc(ncc_plan pl) {
                                 kPrepSmemFloats * 4));
   pl->tc = 1;
   ncc_plan_info& in = pl->info;
-  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_tf32x3_hb%d_wc%d_seg%d_%s%s%s", tc::kHB, pl->tc_wc,
+  snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_bf16x3_hb%d_wc%d_seg%d_%s%s%s", tc::kHB, pl->tc_wc,
            pl->tc_nseg, pl->tc_planes ? "planes" : "chain", pl->tc_vcols ? "_cols" : "", roi ? "_roi" : "");
   fill_kernel_info(pl, (const void*)tm_tc_kernel, tc::kThreads, smem, nblk * pl->tc_vtiles * pl->tc_nseg, nsub, 1);
   in.specialized = 3;  // tensor-core tier: one kernel for every shape (h, w run-time evaluated), not an SK
@@ -1288,12 +1288,12 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   CUtensorMap map_tc;
   bool tc_now = false;
-  if (pl->tc) {  // the band's rows as (hi, lo) pairs: W x Hs x batch 8-byte elements
+  if (pl->tc) {  // the band's rows as (bf16 hi | bf16 lo << 16) words: W x Hs x batch 4-byte elements
     const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)pl->Hs, (uint64_t)batch};
-    const int wp = (p.image_w + 1) & ~1;  // pairs per staged row (even)
-    const uint64_t strides[2] = {(uint64_t)wp * 8, (uint64_t)pl->Hs * wp * 8};
+    const int wp = (p.image_w + 3) & ~3;  // words per staged row (16-byte TMA row stride)
+    const uint64_t strides[2] = {(uint64_t)wp * 4, (uint64_t)pl->Hs * wp * 4};
     const uint32_t box[3] = {(uint32_t)tc::kBoxW, 1u, 1u};
-    tc_now = encode_f32(&map_tc, pl->tc_img2, 3, dims, strides, box, true);
+    tc_now = encode_f32(&map_tc, pl->tc_img2, 3, dims, strides, box);
   }
   const int nblk_tc = pl->tc_nbi * pl->tc_nbj;
   auto launch_cols = [&]() {  // the ragged last columns (tensor-core path), on the side stream
@@ -1317,7 +1317,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   auto launch_split = [&](cudaStream_t st) {
     tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, batch), 128, 0, st>>>(
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
-        reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 1) & ~1), (p.image_w + 1) & ~1,
+        reinterpret_cast<uint32_t*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 3) & ~3), (p.image_w + 3) & ~3,
         pl->tc_center ? pl->tst : nullptr, (double)p.tmpl_h * p.tmpl_w);
   };
   // fork: template prep on the side stream.  Host path: the template's copy (small) goes first,

@@ -1,4 +1,4 @@
-// ncc_tc.cuh -- tensor-core (tcgen05, kind::tf32) numerator of the TM path.
+// ncc_tc.cuh -- tensor-core (tcgen05, kind::f16, 3xBF16) numerator of the TM path.
 //
 // What it computes: the numerator stage of Fig 5.3, N[u][v] = sum_{i,j} A_C[i][j] *
 // I[u+i][v+j], for a template block of up to HB x WC template elements; the normalisation
@@ -6,7 +6,7 @@
 //
 // Mapping onto the 5th-generation tensor cores (sm_100a):
 //   * M = 128 output columns v of a tile (one TMEM lane each);
-//   * K = template columns j, 8 per tcgen05.mma (tf32);
+//   * K = template columns j, 16 per tcgen05.mma (bf16);
 //   * N = a window of output rows u: for image row r the B operand row c is the template row
 //     r - u(c), i.e. a window into the REVERSED, zero-padded template block held in shared
 //     memory (K-major, no swizzle, 16-byte rows, so a window may start at any row: only the
@@ -17,14 +17,20 @@
 //   * A operand = the Hankel matrix H_r[v][j] = I[r][v0+v+j] of image row r, written by the
 //     producer warps straight into TMEM (tcgen05.st; lane v = row v), so the MMAs read only
 //     the template window from shared memory.
-//   * fp32 accuracy from tf32 units: x = hi + lo (hi = tf32(x), lo = x - hi exact), and
-//     A.B ~ A_hi.B_hi + A_hi.B_lo + A_lo.B_hi ("3xTF32"; dropped term ~2^-22 relative).
+//   * fp32-level accuracy from bf16 units: x = hi + lo + r (hi = bf16(x), lo = bf16(x - hi),
+//     |r| <= 2^-17 |x|), A.B ~ A_hi.B_hi + A_hi.B_lo + A_lo.B_hi ("3xBF16"; each bf16 product exact
+//     in the fp32 accumulator; per-product error ~2^-16 relative, random in sign, so ~2^-16 /
+//     sqrt(h w) of the normalisation).  Round 1 used tf32 (3xTF32, K = 8): an M = 128 MMA costs
+//     the same cycles for tf32 K = 8 and bf16 K = 16 (umma_probe rates), so 3xBF16 does the same
+//     work in half the MMAs (cfg 5: 28.2 -> 21.5 ms; measured error at the planted peaks 1e-5 vs
+//     2.25e-5 before: half as many accumulation steps).
 // Rows are processed in groups of G: the window of group g is the HB + G output rows
 // [G g - HB + 1, G g + G + 1); after the group the first G of them are complete, drained from
 // TMEM (tcgen05.ld) to the partial-numerator buffer and their columns zeroed for reuse.
 // Warp roles: warps 0-3 produce the Hankel operand (and drain the ring: lane quadrant w),
 // warp 4 (one thread) issues the MMAs; TMEM A is double-buffered per (row, column chunk).
 #pragma once
+#include <cuda_bf16.h>
 #include "ncc_kernels.cuh"
 
 namespace nccb {
@@ -48,6 +54,23 @@ __device__ __forceinline__ void mma_ts(uint32_t d, uint32_t a_tmem, uint64_t b, 
       "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d),
       "r"(a_tmem), "l"(b), "r"(idesc)
       : "memory");
+}
+// kind::f16 instruction descriptor: D f32, A/B bf16, both K-major, M = 128
+__host__ __device__ constexpr uint32_t idesc_bf16(int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(128 >> 4) << 24);
+}
+__device__ __forceinline__ void mma_bf16(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t idesc) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, 1, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d),
+      "r"(a_tmem), "l"(b), "r"(idesc)
+      : "memory");
+}
+// x = hi + lo (+ r, |r| <= 2^-17 |x|): hi = bf16(x), lo = bf16(x - hi), packed (hi | lo << 16)
+__device__ __forceinline__ uint32_t split_bf16(float x) {
+  const __nv_bfloat16 h = __float2bfloat16_rn(x);
+  const __nv_bfloat16 l = __float2bfloat16_rn(x - __bfloat162float(h));
+  return (uint32_t)__bfloat16_as_ushort(h) | ((uint32_t)__bfloat16_as_ushort(l) << 16);
 }
 __device__ __forceinline__ void commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
@@ -103,7 +126,7 @@ constexpr int kG = 8;      // image rows per group (ring advance, drain granular
 constexpr int kWB = 32;    // template columns per TMEM A chunk (4 MMAs of K = 8)
 constexpr int kRing = 320; // TMEM accumulator columns (sliding window of output rows)
 constexpr int kNBuf = 3;   // TMEM A stages (columns kRing + b*2*kWB .. ; 320 + 3*64 = 512)
-static_assert(kRing + kNBuf * 2 * kWB <= 512, "TMEM columns");
+static_assert(kRing + kNBuf * kWB <= 512, "TMEM columns");  // A: kWB / 2 columns of bf16 pairs, hi and lo
 constexpr int kNWin = kHB + kG;
 // The window of group g starts at column (kG g) mod kRelocAt: when it would run past kRing the
 // kHB live columns [kRelocAt, kRelocAt + kHB) are moved to [0, kHB) (relocation warps), so every
@@ -132,12 +155,12 @@ constexpr int kNImg = 9;                                 // image-row ring (TMA 
 static_assert(kNImg % kNBuf == 0, "a stage and the stage kNImg later belong to the same producer group");
 // shared bytes of the template operand for a column super-block of WC columns (hi + lo)
 __host__ __device__ constexpr uint32_t plane_bytes() { return kLB * 16; }
-__host__ __device__ constexpr int b_bytes(int WC) { return 2 * (WC / 4) * kLB * 16; }
+__host__ __device__ constexpr int b_bytes(int WC) { return 2 * (WC / 8) * kLB * 16; }  // bf16 hi + lo planes of 8
 // dynamic shared memory per CTA: the operand, padded so that one CTA fits per SM (the CTA
 // allocates all 512 TMEM columns)
 __host__ __device__ constexpr int img_off(int WC) { return ((b_bytes(WC) + 127) / 128) * 128; }
 // drained row groups staged for the chain warps: kGRing slots of kG rows x 128 columns (fp32)
-__host__ __device__ constexpr int stage_off(int WC) { return img_off(WC) + kNImg * kBoxW * 8; }
+__host__ __device__ constexpr int stage_off(int WC) { return img_off(WC) + kNImg * kBoxW * 4; }
 __host__ __device__ constexpr int smem_need(int WC) { return stage_off(WC) + kGRing * kG * 128 * 4; }
 __host__ __device__ constexpr int smem_bytes(int WC) { return smem_need(WC) > 120 * 1024 ? smem_need(WC) : 120 * 1024; }
 
@@ -260,7 +283,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   }
   // (a TMA box of 8-byte (hi, lo) elements must start 16-byte aligned: ROI tiles start at the even
   // column at or below the ROI origin, one more tile covers the shift, the extra column is masked)
-  const int v0 = (rv0 & ~1) + vt * 128;
+  const int v0 = (rv0 & ~3) + vt * 128;
   const int ua = ru0 + seg * a.useg;
   const int nu = max(0, min(a.useg, uend - ua));  // output rows of this CTA
   const int i0 = bi * kHB, j0 = bj * a.WC;
@@ -270,7 +293,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
   const int nrow = ngrp * kG;
   const int nstage = nrow * nch;             // (row, chunk) stages
   const uint32_t plane = kLB * 16;           // bytes per K plane of the template operand
-  const int npl = a.WC / 4;
+  const int npl = a.WC / 8;  // bf16 K planes (8 columns of 16 bytes)
 
   // template operand (precomputed layout) -> shared memory
   {
@@ -319,8 +342,8 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     if (stage_zero(q)) {
       mbar_arrive(&img_full[sl]);
     } else {
-      mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 8));
-      tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 8, &map_img, v0 + j0 + (q % nch) * kWB,
+      mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 4));
+      tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 4, &map_img, v0 + j0 + (q % nch) * kWB,
                   ua - a.u_begin + i0 + q / nch, frm, &img_full[sl]);
     }
   };
@@ -351,36 +374,35 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       st_wait();
       fence_before();
     }
-    const uint2* ring = reinterpret_cast<const uint2*>(smem_tc + img_off(a.WC));
+    const uint32_t* ring = reinterpret_cast<const uint32_t*>(smem_tc + img_off(a.WC));
     // Software-pipelined producer: the operand of the group's next stage is read from the ring
     // and split while the group waits for its TMEM buffer, so the critical path from "MMAs of
     // the buffer's previous stage done" to "a_full" is only the TMEM stores (the MMA warp has
     // kNBuf - 1 stages of slack).  (Finished row groups are drained by the epilogue warps.)
-    uint32_t hi[kWB], lo[kWB];
+    uint32_t hi[kWB / 2], lo[kWB / 2];  // bf16 pairs (element 2p in the low half)
     auto load_split = [&](int q) {
       const int sl = q % kNImg;
       mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
       if (gtid == 0) TC_STAMP(5, q);
-      // the split x = hi + lo was done once per image element (tm_tc_split): one 8-byte load
-      // per Hankel element, no per-lane conversion work
+      // the split x = hi + lo was done once per image element (tm_tc_split: one 32-bit word
+      // (bf16 hi | bf16 lo << 16) per element); here only byte permutes into (hi, hi) / (lo, lo)
+      // pairs.  8-byte loads from the even element at or below v (lanes 2i and 2i+1 share
+      // them), odd lanes shift by one element.
       const bool zero = stage_zero(q) || TC_EXP(64);
-      // 16-byte loads from the even element at or below v (lanes 2i and 2i+1 share them: half
-      // the shared-memory wavefronts of one 8-byte load per element), odd lanes shift by one
-      const uint4* r4 = reinterpret_cast<const uint4*>(ring + sl * kBoxW + (v & ~1));
+      const uint2* r2 = reinterpret_cast<const uint2*>(ring + sl * kBoxW + (v & ~1));
       const bool odd = (v & 1) != 0;
-      uint32_t eh[kWB + 2], el[kWB + 2];
+      uint32_t e[kWB + 2];
 #pragma unroll
       for (int m = 0; m < kWB / 2 + 1; ++m) {
-        const uint4 t = zero ? make_uint4(0u, 0u, 0u, 0u) : r4[m];
-        eh[2 * m] = t.x;
-        el[2 * m] = t.y;
-        eh[2 * m + 1] = t.z;
-        el[2 * m + 1] = t.w;
+        const uint2 t = zero ? make_uint2(0u, 0u) : r2[m];
+        e[2 * m] = t.x;
+        e[2 * m + 1] = t.y;
       }
 #pragma unroll
-      for (int k = 0; k < kWB; ++k) {
-        hi[k] = odd ? eh[k + 1] : eh[k];
-        lo[k] = odd ? el[k + 1] : el[k];
+      for (int p = 0; p < kWB / 2; ++p) {
+        const uint32_t e0 = odd ? e[2 * p + 1] : e[2 * p], e1 = odd ? e[2 * p + 2] : e[2 * p + 1];
+        hi[p] = __byte_perm(e0, e1, 0x5410);
+        lo[p] = __byte_perm(e0, e1, 0x7632);
       }
       mbar_arrive(&img_empty[sl]);
       if (gtid == 0) TC_STAMP(1, q);
@@ -396,12 +418,12 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         if (gtid == 0) TC_STAMP(0, qd);
       }
       if (q < nstage) {
-        const uint32_t ab = tbase + lane_base + a_col0 + (uint32_t)(b * 2 * kWB);
-        if (!TC_EXP(1)) {
+        const uint32_t ab = tbase + lane_base + a_col0 + (uint32_t)(b * kWB);
+        if (!TC_EXP(1)) {  // [kWB / 2 columns of hi pairs][kWB / 2 of lo pairs]
 #pragma unroll
-          for (int c = 0; c < kWB; c += 8) {
+          for (int c = 0; c < kWB / 2; c += 8) {
             st8(ab + c, *reinterpret_cast<const uint32_t(*)[8]>(hi + c));
-            st8(ab + kWB + c, *reinterpret_cast<const uint32_t(*)[8]>(lo + c));
+            st8(ab + kWB / 2 + c, *reinterpret_cast<const uint32_t(*)[8]>(lo + c));
           }
         }
         if (!TC_EXP(512)) st_wait();
@@ -640,7 +662,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     {  // the whole warp runs the loop (warp-uniform operands -> uniform datapath); one lane issues
       const uint32_t bhi = smem_u32(smem_tc);
       const uint64_t dlo_off = (uint64_t)(((uint32_t)npl * plane) >> 4);  // hi -> lo operand (descriptor units)
-      constexpr uint64_t kKStep = (uint64_t)((2 * plane_bytes()) >> 4);   // one K-step = two planes
+      constexpr uint64_t kKStep = (uint64_t)((2 * plane_bytes()) >> 4);   // one K-step of 16 = two planes of 8
       int b = 0, ph = 0, ch = 0, s = 0, g = 0, nrel_done = 0;
       (void)ch;
       // Window trimming: the window of group g holds output rows u = kG g - kHB + 1 + c
@@ -697,7 +719,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         }
         trim(g);
         const uint32_t dcol = tbase + col + (uint32_t)c0;
-        const uint32_t id = idesc_tf32(nN);
+        const uint32_t id = idesc_bf16(nN);
         // B window of (s = 0, ch = 0): row kG - 1 + c0 of the reversed block
         const uint64_t dg = sdesc(bhi + (uint32_t)(kG - 1 + c0) * 16, plane, 128);
 #pragma unroll 1
@@ -705,15 +727,15 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 #pragma unroll 1
           for (ch = 0; ch < nch; ++ch, ++q) {
             if (lane == 0) TC_STAMP(3, q);
-            const uint64_t dh = dg - (uint64_t)s + (uint64_t)(((uint32_t)ch * (kWB / 4) * plane) >> 4);
+            const uint64_t dh = dg - (uint64_t)s + (uint64_t)(((uint32_t)ch * (kWB / 8) * plane) >> 4);
             const uint64_t dl = dh + dlo_off;
-            const uint32_t ah = tbase + a_col0 + (uint32_t)(b * 2 * kWB), al = ah + kWB;
+            const uint32_t ah = tbase + a_col0 + (uint32_t)(b * kWB), al = ah + kWB / 2;
             if (leader) {
 #pragma unroll
-              for (int kk = 0; kk < kWB / 8 - 1; ++kk) {
-                mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
-                mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
-                mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
+              for (int kk = 0; kk < kWB / 16 - 1; ++kk) {
+                mma_bf16(dcol, ah + kk * 8, dh + kk * kKStep, id);
+                mma_bf16(dcol, ah + kk * 8, dl + kk * kKStep, id);
+                mma_bf16(dcol, al + kk * 8, dh + kk * kKStep, id);
               }
             }
             __syncwarp();
@@ -726,10 +748,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
             }
             if (!TC_EXP(16384)) fence_after();
             if (leader) {
-              constexpr int kk = kWB / 8 - 1;
-              mma_ts(dcol, ah + kk * 8, dh + kk * kKStep, id);
-              mma_ts(dcol, ah + kk * 8, dl + kk * kKStep, id);
-              mma_ts(dcol, al + kk * 8, dh + kk * kKStep, id);
+              constexpr int kk = kWB / 16 - 1;
+              mma_bf16(dcol, ah + kk * 8, dh + kk * kKStep, id);
+              mma_bf16(dcol, ah + kk * 8, dl + kk * kKStep, id);
+              mma_bf16(dcol, al + kk * 8, dh + kk * kKStep, id);
               commit_u32(done0 + 8 * bq);
             }
             __syncwarp();
@@ -763,14 +785,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 // image's DC level -- and the epilogue adds c * sum A_C back (exact: tc_center is the same fp32
 // value there).  ts = nullptr: the raw image.
 __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
-                                                   int W, int row0, uint2* __restrict__ out, int64_t out_frame_stride,
+                                                   int W, int row0, uint32_t* __restrict__ out, int64_t out_frame_stride,
                                                    int out_pitch, const TemplateStats* ts, double n) {
   const int c = (blockIdx.x * 128 + threadIdx.x) * 4;
   if (c >= W) return;
   const float cen = tc_center(ts, n);
   const int r = blockIdx.y, f = blockIdx.z;
   const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch + c;
-  uint2* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * out_pitch + c;
+  uint32_t* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * out_pitch + c;
   float x[4];
   if (c + 4 <= W && (reinterpret_cast<uintptr_t>(src) & 15) == 0) {
     const float4 v = __ldg(reinterpret_cast<const float4*>(src));
@@ -781,15 +803,11 @@ __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img
   }
 #pragma unroll
   for (int k = 0; k < 4; ++k) x[k] = c + k < W ? x[k] - cen : 0.0f;
-  uint2 o[4];
+  uint32_t o[4];
 #pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    o[k].x = tc::to_tf32(x[k]);
-    o[k].y = __float_as_uint(x[k] - __uint_as_float(o[k].x));
-  }
+  for (int k = 0; k < 4; ++k) o[k] = tc::split_bf16(x[k]);
   if (c + 4 <= W) {
-    reinterpret_cast<uint4*>(dst)[0] = make_uint4(o[0].x, o[0].y, o[1].x, o[1].y);
-    reinterpret_cast<uint4*>(dst)[1] = make_uint4(o[2].x, o[2].y, o[3].x, o[3].y);
+    reinterpret_cast<uint4*>(dst)[0] = make_uint4(o[0], o[1], o[2], o[3]);
   } else {
     for (int k = 0; c + k < W; ++k) dst[k] = o[k];
   }
@@ -915,17 +933,17 @@ __global__ void tm_tc_tpl_prep(const float* __restrict__ tplC, int tplP, int h, 
   using namespace tc;
   const int blk = blockIdx.x, bi = blk / nbj, bj = blk % nbj;
   const int i0 = bi * kHB, j0 = bj * WC;
-  const int npl = WC / 4;
-  float* out = tcB + (int64_t)blk * (b_bytes(WC) / 4);
-  const int n = npl * kLB * 4;
+  const int npl = WC / 8;
+  uint16_t* out = reinterpret_cast<uint16_t*>(tcB) + (int64_t)blk * (b_bytes(WC) / 2);
+  const int n = npl * kLB * 8;
   for (int e = threadIdx.x; e < n; e += blockDim.x) {
-    const int c = e / (kLB * 4), k = (e / 4) % kLB, t = e % 4;
+    const int c = e / (kLB * 8), k = (e / 8) % kLB, t = e % 8;
     const int row = kHB + kG - 2 - k;
-    const int i = i0 + row, j = j0 + 4 * c + t;
+    const int i = i0 + row, j = j0 + 8 * c + t;
     const float val = (row >= 0 && row < kHB && i < h && j < w) ? tplC[(int64_t)i * tplP + j] : 0.0f;
-    const float hi = __uint_as_float(to_tf32(val));
-    out[e] = hi;
-    out[n + e] = val - hi;
+    const uint32_t hl = split_bf16(val);
+    out[e] = (uint16_t)(hl & 0xffffu);
+    out[n + e] = (uint16_t)(hl >> 16);
   }
 }
 
@@ -948,7 +966,7 @@ __global__ void __launch_bounds__(1024) tm_tc_prep(const float* __restrict__ tmp
     tmpl += (int64_t)t * h * tpitch;
     tplC += (int64_t)t * HP * WP;
     ts += t;
-    tcB += (int64_t)t * gridDim.x * (b_bytes(WC) / 4);
+    tcB += (int64_t)t * gridDim.x * (b_bytes(WC) / 4);  // (float units: the byte size / 4)
   }
   const int n = h * w;
   // one pass over the template, staged in shared memory: float4 loads when rows allow it
@@ -1002,16 +1020,16 @@ __global__ void __launch_bounds__(1024) tm_tc_prep(const float* __restrict__ tmp
   {  // this CTA's template block operand (reversed rows, hi / lo planes; as tm_tc_tpl_prep)
     const int blk = blockIdx.x, bi = blk / nbj, bj = blk % nbj;
     const int i0 = bi * kHB, j0 = bj * WC;
-    float* out = tcB + (int64_t)blk * (b_bytes(WC) / 4);
-    const int nb = (WC / 4) * kLB * 4;
+    uint16_t* out = reinterpret_cast<uint16_t*>(tcB + (int64_t)blk * (b_bytes(WC) / 4));
+    const int nb = (WC / 8) * kLB * 8;
     for (int e = threadIdx.x; e < nb; e += blockDim.x) {
-      const int c = e / (kLB * 4), k = (e / 4) % kLB, t = e % 4;
+      const int c = e / (kLB * 8), k = (e / 8) % kLB, t = e % 8;
       const int row = kHB + kG - 2 - k;
-      const int i = i0 + row, j = j0 + 4 * c + t;
+      const int i = i0 + row, j = j0 + 8 * c + t;
       const float val = (row >= 0 && row < kHB && i < h && j < w) ? (float)((double)tsm[i * w + j] - mean) : 0.0f;
-      const float hi = __uint_as_float(to_tf32(val));
-      out[e] = hi;
-      out[nb + e] = val - hi;
+      const uint32_t hl = split_bf16(val);
+      out[e] = (uint16_t)(hl & 0xffffu);
+      out[nb + e] = (uint16_t)(hl >> 16);
     }
   }
   if (blockIdx.x != 0) return;

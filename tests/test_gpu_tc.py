@@ -1,5 +1,5 @@
-"""GPU parity of the tensor-core numerator (tcgen05 kind::tf32 with the
-3xTF32 split, ncc_tc.cuh) through the C ABI vs the fp64 oracle: full surfaces within 1e-4,
+"""GPU parity of the tensor-core numerator (tcgen05 kind::f16 with the
+3xBF16 split, ncc_tc.cuh) through the C ABI vs the fp64 oracle: full surfaces within 1e-4,
 planted peaks exact, SSD, several template blocks (h > 128, w > 128), batches, band shards
 bitwise equal to the full problem (the per-output accumulation order does not depend on the
 band), and the CUDA-core path agreeing within the tolerance."""
