@@ -359,7 +359,7 @@ struct ncc_plan_s {
   int ws_bp;             // its staged pitch = TMA box width
   const PivVariant* pivv;
   // tensor-core PIV numerator (piv_tc_kernel; 0: CUDA cores): rows per MMA, smem, grid, strip segments
-  int ptc, ptc_R, ptc_smem, ptc_border_smem, ptc_nseg, ptc_segw;
+  int ptc, ptc_R, ptc_smem, ptc_border_smem, ptc_nseg, ptc_segw, ptc_border_rb;
   float* ptc_border;     // [sub_batch][Ky Kx][OY] numerators of the last column (piv_tc_border_kernel)
   unsigned long long* ptc_prof;  // NCC_PIV_TC_PROF=<file>: per-CTA wait accounting, dumped at destroy
   // shared scratch (window sums)
@@ -1100,6 +1100,13 @@ ncc_status create_piv(ncc_plan pl) {
       pl->ptc_R = R;
       pl->ptc_smem = ptc::smem_bytes(h, w, my, mx);
       pl->ptc_border_smem = (h * w + (span + kBorderDY - 1) * w) * 4;
+      // register-blocked last-column kernel for 32- / 64-row masks of 32 / 64 columns
+      pl->ptc_border_rb = ((h == 32 || h == 64) && (w == 32 || w == 64) && !getenv("NCC_PIV_TC_BORDER_GENERIC")) ? h : 0;
+      if (pl->ptc_border_rb) {
+        pl->ptc_border_smem += 8 * (w / 32) * kBorderDY * 4;
+        const void* f = pl->ptc_border_rb == 64 ? (const void*)piv_tc_border_rb<64> : (const void*)piv_tc_border_rb<32>;
+        NCC_CUDA(cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->ptc_border_smem));
+      }
       if (pl->ptc_border_smem > maxsm) return NCC_ERR_UNSUPPORTED;
       NCC_CUDA(cudaFuncSetAttribute((const void*)piv_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, pl->ptc_smem));
       NCC_CUDA(cudaFuncSetAttribute((const void*)piv_tc_border_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -1699,7 +1706,12 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
       if (const char* e = getenv("NCC_PIV_TC_NAB")) t.nab = std::max(ptc::kNAB, std::min(t.nab, atoi(e)));
       t.exp = 0;
       if (const char* e = getenv("NCC_PIV_TC_EXP")) t.exp = atoi(e);
-      piv_tc_border_kernel<<<dim3(pl->Ky * pl->Kx, np), 256, pl->ptc_border_smem, s>>>(t, B);
+      if (pl->ptc_border_rb == 64)
+        piv_tc_border_rb<64><<<dim3(pl->Ky * pl->Kx, np), 256 * (p.tmpl_w / 32), pl->ptc_border_smem, s>>>(t, B);
+      else if (pl->ptc_border_rb == 32)
+        piv_tc_border_rb<32><<<dim3(pl->Ky * pl->Kx, np), 256 * (p.tmpl_w / 32), pl->ptc_border_smem, s>>>(t, B);
+      else
+        piv_tc_border_kernel<<<dim3(pl->Ky * pl->Kx, np), 256, pl->ptc_border_smem, s>>>(t, B);
       void* targs[2] = {&t, &mT};
       const int g = std::min(t.nunits, pl->nsm);
       NCC_CUDA(cudaLaunchKernel((const void*)piv_tc_kernel, dim3(g), dim3(ptc::kThreads), targs, (size_t)pl->ptc_smem, s));

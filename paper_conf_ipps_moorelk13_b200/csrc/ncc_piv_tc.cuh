@@ -653,20 +653,23 @@ __global__ void __launch_bounds__(256) piv_tc_border_kernel(const PivTcArgs a, c
   const float* Bw = Bf + (int64_t)(a.pair0 + z) * a.frame_stride + (int64_t)(y - a.my) * a.pitch + x + a.mx;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   double s1 = 0.0;
-  for (int e = tid; e < h * w; e += 256) {
-    const float v = __ldg(Aw + (int64_t)(e / w) * a.pitch + e % w);
-    T[e] = v;
-    s1 += (double)v;
-  }
-  for (int e = tid; e < (span + kBorderDY - 1) * w; e += 256)
-    Bc[e] = e < span * w ? __ldg(Bw + (int64_t)(e / w) * a.pitch + e % w) : 0.0f;
+  // staging: one row per warp pass, lanes along the row (no per-element division)
+  for (int i = warp; i < h; i += 8)
+    for (int j = lane; j < w; j += 32) {
+      const float v = __ldg(Aw + (int64_t)i * a.pitch + j);
+      T[i * w + j] = v;
+      s1 += (double)v;
+    }
+  for (int i = warp; i < span + kBorderDY - 1; i += 8)
+    for (int j = lane; j < w; j += 32) Bc[i * w + j] = i < span ? __ldg(Bw + (int64_t)i * a.pitch + j) : 0.0f;
   s1 = warp_sum_d(s1);
   if (lane == 0) red[warp] = s1;
   __syncthreads();
   double tot = 0.0;
   for (int q = 0; q < 8; ++q) tot += red[q];
   const double mean = tot / ((double)h * (double)w);
-  for (int e = tid; e < h * w; e += 256) T[e] = (float)((double)T[e] - mean);
+  for (int i = warp; i < h; i += 8)
+    for (int j = lane; j < w; j += 32) T[i * w + j] = (float)((double)T[i * w + j] - mean);
   __syncthreads();
   const int dy0 = warp * kBorderDY;
   if (dy0 >= OY) return;
@@ -692,6 +695,77 @@ __global__ void __launch_bounds__(256) piv_tc_border_kernel(const PivTcArgs a, c
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
     if (lane == 0 && dy0 + d < OY) const_cast<float*>(a.border)[((int64_t)z * a.Ky * a.Kx + lin) * OY + dy0 + d] = v;
+  }
+}
+
+
+// Register-blocked form for TH = h in {32, 64} and w a multiple of 32: warp (b, c) takes the 9
+// output rows dy = 9 b + d and the template columns j = 32 c + lane; each thread keeps its
+// template column in registers and streams the image column once (row r' of the block meets
+// template rows r' - d: compile-time after unrolling), ~9 FMAs per shared load.  grid = (Ky Kx,
+// pairs), block = 8 (w / 32) warps; dynamic smem as piv_tc_border_kernel + 8 (w / 32) 9 floats.
+template <int TH>
+__global__ void __launch_bounds__(512) piv_tc_border_rb(const PivTcArgs a, const float* __restrict__ Bf) {
+  extern __shared__ __align__(16) float sm_rb[];
+  __shared__ double red[16];
+  const int w = a.w, OY = 2 * a.my + 1, span = TH + 2 * a.my, ncw = w / 32, nth = 256 * ncw;
+  float* T = sm_rb;
+  float* Bc = sm_rb + TH * w;
+  float* part = Bc + (span + kBorderDY - 1) * w;  // [ncw][8][9]
+  const int lin = blockIdx.x, z = blockIdx.y;
+  const int ky = lin / a.Kx, kx = lin % a.Kx;
+  const int y = a.my + ky * a.sy, x = a.mx + kx * a.sx;
+  const float* Aw = a.A + (int64_t)(a.pair0 + z) * a.frame_stride + (int64_t)y * a.pitch + x;
+  const float* Bw = Bf + (int64_t)(a.pair0 + z) * a.frame_stride + (int64_t)(y - a.my) * a.pitch + x + a.mx;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarp = nth / 32;
+  double s1 = 0.0;
+  for (int i = warp; i < TH; i += nwarp)
+    for (int j = lane; j < w; j += 32) {
+      const float v = __ldg(Aw + (int64_t)i * a.pitch + j);
+      T[i * w + j] = v;
+      s1 += (double)v;
+    }
+  for (int i = warp; i < span + kBorderDY - 1; i += nwarp)
+    for (int j = lane; j < w; j += 32) Bc[i * w + j] = i < span ? __ldg(Bw + (int64_t)i * a.pitch + j) : 0.0f;
+  s1 = warp_sum_d(s1);
+  if (lane == 0) red[warp] = s1;
+  __syncthreads();
+  double tot = 0.0;
+  for (int q = 0; q < nwarp; ++q) tot += red[q];
+  const double mean = tot / ((double)TH * (double)w);
+  for (int i = warp; i < TH; i += nwarp)
+    for (int jj = lane; jj < w; jj += 32) T[i * w + jj] = (float)((double)T[i * w + jj] - mean);
+  __syncthreads();
+  const int b = warp & 7, c = warp >> 3, j = 32 * c + lane, dy0 = kBorderDY * b;
+  float tr[TH];  // the thread's template column, pinned in registers (volatile loads: not re-read per use)
+#pragma unroll
+  for (int i = 0; i < TH; ++i)
+    asm volatile("ld.shared.f32 %0, [%1];" : "=f"(tr[i]) : "r"(smem_u32(T + i * w + j)));
+  float acc[kBorderDY];
+#pragma unroll
+  for (int d = 0; d < kBorderDY; ++d) acc[d] = 0.0f;
+  if (dy0 < OY) {
+    const float* bcol = Bc + dy0 * w + j;
+#pragma unroll
+    for (int r = 0; r < TH + kBorderDY - 1; ++r) {
+      const float xv = bcol[r * w];
+#pragma unroll
+      for (int d = 0; d < kBorderDY; ++d)
+        if (r - d >= 0 && r - d < TH) acc[d] = fmaf(tr[r - d], xv, acc[d]);
+    }
+  }
+#pragma unroll
+  for (int d = 0; d < kBorderDY; ++d) {
+    float v = acc[d];
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    if (lane == 0) part[(c * 8 + b) * kBorderDY + d] = v;
+  }
+  __syncthreads();
+  for (int dy = tid; dy < OY; dy += nth) {
+    float v = 0.0f;
+    for (int cc = 0; cc < ncw; ++cc) v += part[(cc * 8 + dy / kBorderDY) * kBorderDY + dy % kBorderDY];
+    const_cast<float*>(a.border)[((int64_t)z * a.Ky * a.Kx + lin) * OY + dy] = v;
   }
 }
 
