@@ -25,7 +25,8 @@ def main():
                    f"cfg4 is per pair (capture: 8-pair launch); bench.py multiplies by the pairs of its launches; "
                    f"'source' names the round each figure was captured in")
     for key, name, per in (("cfg2_tc", "prof_cfg2.json", 1), ("cfg5_tc", "prof_cfg5.json", 1),
-                           ("cfg3", "prof_piv3.json", 1), ("cfg4_per_pair", "prof_piv4.json", 8)):
+                           ("cfg3", "prof_piv3.json", 1), ("cfg4_tc_per_pair", "prof_piv4.json", 8),
+                           ("cfg4_per_pair", "prof_piv4cc.json", 8)):
         p = os.path.join(d, name)
         if not os.path.exists(p):
             continue
