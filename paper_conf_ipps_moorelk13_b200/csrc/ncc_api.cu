@@ -116,8 +116,8 @@ bool encode_f32(CUtensorMap* m, const void* base, int rank, const uint64_t* dims
                 const uint32_t* box, bool u64 = false) {
   EncodeTiledFn fn = encode_fn();
   if (!fn) return false;
-  cuuint64_t gd[3], gs[2];
-  cuuint32_t bx[3], es[3] = {1, 1, 1};
+  cuuint64_t gd[5], gs[4];
+  cuuint32_t bx[5], es[5] = {1, 1, 1, 1, 1};
   for (int i = 0; i < rank; ++i) {
     gd[i] = dims[i];
     bx[i] = box[i];
@@ -366,7 +366,7 @@ struct ncc_plan_s {
   double *RS1, *RS2, *S1, *S2;
   int64_t rs_frame_stride, s_frame_stride;
   int box_r, box_iwp, box_smem, nsm;  // fused window-sum kernel (box_smem 0: two-pass fallback)
-  float* tc_img2 = nullptr;  // band rows as (tf32 hi, lo) pairs for the tensor-core numerator
+  float* tc_img2 = nullptr;  // band rows as the tensor-core numerator's image operand (tm_tc_split)
   // tensor-core numerator (tm_tc_kernel): 0 = CUDA-core path
   int tc, tc_wc, tc_nbi, tc_nbj, tc_vtiles, tc_useg, tc_nseg;
   int tc_vcols;  // last output columns computed by tm_tc_cols (0: none)
@@ -692,8 +692,8 @@ ncc_status setup_tc(ncc_plan pl) {
   NCC_CUDA(cudaMemset(pl->tc_flags, 0, nflags * sizeof(unsigned int)));
   if ((st = dalloc(&pl->tc_ticket, (size_t)1))) return st;
   NCC_CUDA(cudaMemset(pl->tc_ticket, 0, sizeof(unsigned long long)));
-  // (hi, lo) pairs, rows padded to an even count of pairs: a 16-byte multiple for the TMA map
-  if ((st = dalloc(&pl->tc_img2, (size_t)p.batch * pl->Hs * ((p.image_w + 3) & ~3)))) return st;
+  // image operand (tm_tc_split): per band row two planes of ((W + 1) & ~1) 8-byte elements
+  if ((st = dalloc(&pl->tc_img2, (size_t)p.batch * pl->Hs * 4 * ((p.image_w + 1) & ~1)))) return st;
   if (p.score == NCC_SCORE_NCC) {  // per-offset fp32 normalisation factors (window-sum kernels)
     if ((st = dalloc(&pl->tc_rsv, (size_t)p.batch * pl->s_frame_stride))) return st;
     if ((st = dalloc(&pl->tc_mean, (size_t)p.batch * pl->s_frame_stride))) return st;
@@ -1295,12 +1295,12 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   CUtensorMap map_tc;
   bool tc_now = false;
-  if (pl->tc) {  // the band's rows as (bf16 hi | bf16 lo << 16) words: W x Hs x batch 4-byte elements
-    const uint64_t dims[3] = {(uint64_t)p.image_w, (uint64_t)pl->Hs, (uint64_t)batch};
-    const int wp = (p.image_w + 3) & ~3;  // words per staged row (16-byte TMA row stride)
-    const uint64_t strides[2] = {(uint64_t)wp * 4, (uint64_t)pl->Hs * wp * 4};
-    const uint32_t box[3] = {(uint32_t)tc::kBoxW, 1u, 1u};
-    tc_now = encode_f32(&map_tc, pl->tc_img2, 3, dims, strides, box);
+  if (pl->tc) {  // the band's image operand (tm_tc_split): wp x 2 planes x Hs x batch 8-byte elements
+    const int wp = (p.image_w + 1) & ~1;  // elements per plane row (16-byte TMA strides)
+    const uint64_t dims[4] = {(uint64_t)wp, 2u, (uint64_t)pl->Hs, (uint64_t)batch};
+    const uint64_t strides[3] = {(uint64_t)wp * 8, (uint64_t)wp * 16, (uint64_t)pl->Hs * wp * 16};
+    const uint32_t box[4] = {(uint32_t)tc::kBoxW, 2u, 1u, 1u};
+    tc_now = encode_f32(&map_tc, pl->tc_img2, 4, dims, strides, box, true);
   }
   const int nblk_tc = pl->tc_nbi * pl->tc_nbj;
   auto launch_cols = [&]() {  // the ragged last columns (tensor-core path), on the side stream
@@ -1322,9 +1322,10 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     else cols(tm_tc_cols_rw<16, RWN>);
   };
   auto launch_split = [&](cudaStream_t st) {
-    tm_tc_split<<<dim3(ceil_div(ceil_div(p.image_w, 4), 128), pl->Hs, batch), 128, 0, st>>>(
+    const int wp = (p.image_w + 1) & ~1;
+    tm_tc_split<<<dim3(ceil_div(ceil_div(wp, 4), 128), pl->Hs, batch), 128, 0, st>>>(
         d_images, p.image_pitch, (int64_t)p.image_h * p.image_pitch, p.image_w, pl->u_begin,
-        reinterpret_cast<uint32_t*>(pl->tc_img2), (int64_t)pl->Hs * ((p.image_w + 3) & ~3), (p.image_w + 3) & ~3,
+        reinterpret_cast<uint2*>(pl->tc_img2), (int64_t)pl->Hs * 2 * wp, wp,
         pl->tc_center ? pl->tst : nullptr, (double)p.tmpl_h * p.tmpl_w);
   };
   // fork: template prep on the side stream.  Host path: the template's copy (small) goes first,

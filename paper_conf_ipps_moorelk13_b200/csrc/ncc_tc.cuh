@@ -66,6 +66,25 @@ __device__ __forceinline__ void mma_bf16(uint32_t d, uint32_t a_tmem, uint64_t b
       "r"(a_tmem), "l"(b), "r"(idesc)
       : "memory");
 }
+// Warp-wide forms for an issue loop run by all 32 lanes (warp-uniform operands stay on the uniform
+// datapath): the instruction is issued once, by the lane elect.sync picks inside the asm -- no
+// divergent C++ branch around it.
+__device__ __forceinline__ void mma_bf16_warp(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t idesc) {
+  asm volatile(
+      "{\n\t.reg .pred E, A;\n\t"
+      "elect.sync _|E, 0xffffffff;\n\t"
+      "setp.ne.b32 A, 1, 0;\n\t"
+      "@E tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, A;\n\t}" ::"r"(d),
+      "r"(a_tmem), "l"(b), "r"(idesc)
+      : "memory");
+}
+__device__ __forceinline__ void commit_warp(uint32_t bar) {
+  asm volatile(
+      "{\n\t.reg .pred E;\n\t"
+      "elect.sync _|E, 0xffffffff;\n\t"
+      "@E tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(bar)
+      : "memory");
+}
 // x = hi + lo (+ r, |r| <= 2^-17 |x|): hi = bf16(x), lo = bf16(x - hi), packed (hi | lo << 16)
 __device__ __forceinline__ uint32_t split_bf16(float x) {
   const __nv_bfloat16 h = __float2bfloat16_rn(x);
@@ -110,6 +129,34 @@ __device__ __forceinline__ void mbar_wait_u32(uint32_t bar, uint32_t parity) {
   }
   __trap();
 }
+__device__ __forceinline__ bool mbar_try_u32(uint32_t bar, uint32_t parity) {
+  uint32_t done;
+  asm volatile(
+      "{\n\t.reg .pred P;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2;\n\t"
+      "selp.u32 %0, 1, 0, P;\n}"
+      : "=r"(done)
+      : "r"(bar), "r"(parity)
+      : "memory");
+  return done != 0;
+}
+// mbarrier wait as ONE asm block: a non-blocking test_wait, and only on failure loop back (the
+// success path falls through: no taken branch, no call between two MMAs of the issue loop; a
+// satisfied try_wait measured ~350 cycles here).  Traps after ~2^30 failed polls (a hang guard, as
+// mbar_wait_bounded).
+__device__ __forceinline__ void mbar_wait_fall(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred P, Q;\n\t.reg .u32 n;\n\t"
+      "mov.u32 n, 0;\n"
+      "LAB_WAIT:\n\t"
+      "mbarrier.test_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "@!P add.u32 n, n, 1;\n\t"
+      "setp.gt.u32 Q, n, 1073741824;\n\t"
+      "@Q trap;\n\t"
+      "@!P bra LAB_WAIT;\n}"
+      ::"r"(bar), "r"(parity)
+      : "memory");
+}
 __device__ __forceinline__ bool elect_one() {
   uint32_t pred = 0;
   asm volatile("{\n\t.reg .pred P;\n\telect.sync _|P, 0xffffffff;\n\tselp.u32 %0, 1, 0, P;\n}" : "=r"(pred));
@@ -152,7 +199,9 @@ constexpr int kTmaWarp = kChainWarp0 + kNChain;
 constexpr int kMmaWarp = kTmaWarp + 1;
 constexpr int kThreads = kGroups * 128 + 128 + kNChain * 32 + 32 + 32;
 constexpr int kBoxW = 128 + kWB;                         // image-row segment of one stage (TMA box)
-constexpr int kNImg = 9;                                 // image-row ring (TMA issue distance)
+constexpr int kNImg = 24;  // image-row ring (TMA issue distance: ~5 us of lookahead at cfg 2; 9 left the producers
+                           // waiting ~760 cycles per stage for the data)
+static_assert(kWB == 32, "the unrolled issue loop does two K-steps of 16 per stage");
 static_assert(kNImg % kGroups == 0 && kNBuf % kGroups == 0, "a stage and the stage kNImg later belong to the same producer group");
 // shared bytes of the template operand for a column super-block of WC columns (hi + lo)
 __host__ __device__ constexpr uint32_t plane_bytes() { return kLB * 16; }
@@ -161,7 +210,10 @@ __host__ __device__ constexpr int b_bytes(int WC) { return 2 * (WC / 8) * kLB * 
 // allocates all 512 TMEM columns)
 __host__ __device__ constexpr int img_off(int WC) { return ((b_bytes(WC) + 127) / 128) * 128; }
 // drained row groups staged for the chain warps: kGRing slots of kG rows x 128 columns (fp32)
-__host__ __device__ constexpr int stage_off(int WC) { return img_off(WC) + kNImg * kBoxW * 4; }
+// one ring slot: the stage's segment of the image operand as two planes of 8-byte elements (E, F),
+// see tm_tc_split
+constexpr int kSlotBytes = 2 * kBoxW * 8;
+__host__ __device__ constexpr int stage_off(int WC) { return img_off(WC) + kNImg * kSlotBytes; }
 __host__ __device__ constexpr int smem_need(int WC) { return stage_off(WC) + kGRing * kG * 128 * 4; }
 __host__ __device__ constexpr int smem_bytes(int WC) { return smem_need(WC) > 120 * 1024 ? smem_need(WC) : 120 * 1024; }
 
@@ -183,8 +235,8 @@ __device__ int g_tc_exp;  // timing experiments (trace builds only): bit0 no A s
 #endif
 
 struct TcArgs {
-  // the image as (tf32 hi, fp32 lo) pairs of the band's rows (tm_tc_split), read through the
-  // tensor map; H = absolute image rows (zero rows past it), u_begin = the band's first row
+  // the image operand of the band's rows (tm_tc_split: two planes of 8-byte pair elements per row),
+  // read through the tensor map; H = absolute image rows (zero rows past it), u_begin = the band's first row
   int H, W;
   const float* tcB;     // [nblk][2 (hi, lo)][WC/4 planes][kLB rows][4]: reversed template blocks
   int WC;               // template columns per CTA (multiple of kWB, <= 128)
@@ -335,6 +387,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 
   // stage q = (image row rr, column chunk ch): row ua + i0 + rr, columns v0 + j0 + 32 ch + [0, kBoxW)
   auto stage_zero = [&](int q) {  // rows past the image / chunks past its width: zero operand
+    if (nch == 1) return ua + i0 + q >= a.H || v0 + j0 >= a.W;
     return ua + i0 + q / nch >= a.H || v0 + j0 + (q % nch) * kWB >= a.W;
   };
   auto issue = [&](int q) {  // one thread: TMA of stage q into ring slot q % kNImg
@@ -343,9 +396,9 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     if (stage_zero(q)) {
       mbar_arrive(&img_full[sl]);
     } else {
-      mbar_expect_tx(&img_full[sl], (uint32_t)(kBoxW * 4));
-      tma_load_3d(smem_tc + img_off(a.WC) + sl * kBoxW * 4, &map_img, v0 + j0 + (q % nch) * kWB,
-                  ua - a.u_begin + i0 + q / nch, frm, &img_full[sl]);
+      mbar_expect_tx(&img_full[sl], (uint32_t)kSlotBytes);
+      tma_load_4d(smem_tc + img_off(a.WC) + sl * kSlotBytes, &map_img, v0 + j0 + (nch == 1 ? 0 : q % nch) * kWB, 0,
+                  ua - a.u_begin + i0 + (nch == 1 ? q : q / nch), frm, &img_full[sl]);
     }
   };
   if (TC_EXP(32768) && warp != kMmaWarp) {
@@ -375,35 +428,32 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       st_wait();
       fence_before();
     }
-    const uint32_t* ring = reinterpret_cast<const uint32_t*>(smem_tc + img_off(a.WC));
+    const uint2* ring = reinterpret_cast<const uint2*>(smem_tc + img_off(a.WC));
     // Software-pipelined producer: the operand of the group's next stage is read from the ring
-    // and split while the group waits for its TMEM buffer, so the critical path from "MMAs of
-    // the buffer's previous stage done" to "a_full" is only the TMEM stores (the MMA warp has
-    // kNBuf - 1 stages of slack).  (Finished row groups are drained by the epilogue warps.)
+    // while the group waits for its TMEM buffer, so the critical path from "MMAs of the buffer's
+    // previous stage done" to "a_full" is only the TMEM stores (the MMA warp has kNBuf - 1 stages
+    // of slack).  (Finished row groups are drained by the epilogue warps.)
     uint32_t hi[kWB / 2], lo[kWB / 2];  // bf16 pairs (element 2p in the low half)
     auto load_split = [&](int q) {
       const int sl = q % kNImg;
       mbar_wait_bounded(&img_full[sl], (uint32_t)((q / kNImg) & 1));
       if (gtid == 0) TC_STAMP(5, q);
-      // the split x = hi + lo was done once per image element (tm_tc_split: one 32-bit word
-      // (bf16 hi | bf16 lo << 16) per element); here only byte permutes into (hi, hi) / (lo, lo)
-      // pairs.  8-byte loads from the even element at or below v (lanes 2i and 2i+1 share
-      // them), odd lanes shift by one element.
+      // tm_tc_split stored, per image element k, E_k = (P_k, P_{k+2}) and F_k = (Q_k, Q_{k+2}) with
+      // P_k = (bf16 hi_k | hi_{k+1} << 16), Q_k the same of lo: the lane's Hankel row is 8 loads of 8
+      // bytes from each plane (elements v, v + 4, ..., v + 28), already in MMA operand order -- no
+      // shifts, selects or permutes (the producers' instruction count sets the stage time: their
+      // warps share the SMSPs with the MMA issuer).  A warp's load covers 32 consecutive 8-byte
+      // elements: 2 wavefronts, no conflicts.
       const bool zero = stage_zero(q) || TC_EXP(64);
-      const uint2* r2 = reinterpret_cast<const uint2*>(ring + sl * kBoxW + (v & ~1));
-      const bool odd = (v & 1) != 0;
-      uint32_t e[kWB + 2];
+      const uint2* e = ring + sl * 2 * kBoxW + v;
 #pragma unroll
-      for (int m = 0; m < kWB / 2 + 1; ++m) {
-        const uint2 t = zero ? make_uint2(0u, 0u) : r2[m];
-        e[2 * m] = t.x;
-        e[2 * m + 1] = t.y;
-      }
-#pragma unroll
-      for (int p = 0; p < kWB / 2; ++p) {
-        const uint32_t e0 = odd ? e[2 * p + 1] : e[2 * p], e1 = odd ? e[2 * p + 2] : e[2 * p + 1];
-        hi[p] = __byte_perm(e0, e1, 0x5410);
-        lo[p] = __byte_perm(e0, e1, 0x7632);
+      for (int m = 0; m < kWB / 4; ++m) {
+        const uint2 th = zero ? make_uint2(0u, 0u) : e[4 * m];
+        const uint2 tl = zero ? make_uint2(0u, 0u) : e[kBoxW + 4 * m];
+        hi[2 * m] = th.x;
+        hi[2 * m + 1] = th.y;
+        lo[2 * m] = tl.x;
+        lo[2 * m + 1] = tl.y;
       }
       mbar_arrive(&img_empty[sl]);
       if (gtid == 0) TC_STAMP(1, q);
@@ -695,9 +745,98 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       unsigned long long m_drained = 0, m_afull = 0;
       if (mprof) mprof[0] = gtimer();
       const bool leader = elect_one();
-      if (nstage > 0 && !TC_EXP(16)) mbar_wait_u32(full0, 0u);
-      fence_after();
       int q = 0;
+      if (nch == 1 && !TC_EXP(262144) && !TC_EXP(1048576)) {
+        // One template column chunk per image row (WC = 32, the default): per stage the warp waits
+        // for its operand (one try_wait that falls through when the producers are ahead, as they
+        // normally are), then the elected lane issues the stage's 6 MMAs and the commit with
+        // nothing in between.  The tensor pipe queues only about one MMA, so the scalar work between
+        // two MMAs must stay short: the earlier form (the operand wait between the two K-steps, the
+        // unrolled 30-try wait loops whose success path was a taken branch) ran at ~135 cycles per
+        // N = 136 MMA; the pipe's rate is 68 (tools/microbench/issue_probe.cu, tc_trace.cu).
+        uint32_t phs = 0;
+#pragma unroll 1
+        for (g = 0; q < nstage; ++g) {
+          const uint32_t col = (uint32_t)((g * kG) % kRelocAt);
+          if (col == 0 && g > 0) {  // window restart: relocate the live columns first
+            const int qp = q - 1;   // MMAs complete in order: the last stage's completion covers all
+            mbar_wait_u32(done0 + 8 * (qp % kNBuf), (uint32_t)((qp / kNBuf) & 1));
+            fence_after();
+            fence_before();
+            if (leader) mbar_arrive(&reloc_req);
+            __syncwarp();
+            mbar_wait_bounded(&reloc_done, (uint32_t)(nrel_done & 1));
+            fence_after();
+            ++nrel_done;
+          }
+          if (lane == 0) TC_STAMP(6, g);
+          if (g >= kGRing) {  // the window's newest columns were drained (and zeroed) after group g - kGRing
+            const unsigned long long t0 = mprof ? gtimer() : 0ull;
+            mbar_wait_fall(drained0 + 8 * ((g - kGRing) % kGRing), (uint32_t)(((g - kGRing) / kGRing) & 1));
+            if (mprof) m_drained += gtimer() - t0;
+            fence_after();
+          }
+          if (lane == 0) TC_STAMP(7, g);
+          trim(g);
+          const uint32_t dcol = tbase + col + (uint32_t)c0;
+          const uint32_t id = idesc_bf16(nN);
+          const uint64_t dg = sdesc(bhi + (uint32_t)(kG - 1 + c0) * 16, plane, 128);
+#pragma unroll 1
+          for (int st = 0; st < kG; ++st, ++q) {
+            mbar_wait_fall(full0 + 8 * b, phs);
+            fence_after();
+            if (lane == 0) TC_STAMP(3, q);
+            const uint32_t ah = tbase + a_col0 + (uint32_t)(b * kWB);
+            const uint64_t dh = dg - (uint64_t)st;
+            if (leader) {
+              mma_bf16(dcol, ah, dh, id);
+              mma_bf16(dcol, ah, dh + dlo_off, id);
+              mma_bf16(dcol, ah + kWB / 2, dh, id);
+              mma_bf16(dcol, ah + 8, dh + kKStep, id);
+              mma_bf16(dcol, ah + 8, dh + dlo_off + kKStep, id);
+              mma_bf16(dcol, ah + kWB / 2 + 8, dh + kKStep, id);
+              commit_u32(done0 + 8 * b);
+            }
+            __syncwarp();
+            if (lane == 0) TC_STAMP(4, q);
+            if (++b == kNBuf) {
+              b = 0;
+              phs ^= 1u;
+            }
+          }
+          if (leader) commit_u32(gdone0 + 8 * (g % kGRing));  // group g's MMAs complete -> epilogue drains it
+          __syncwarp();
+          if (mprof && tk < 4 && g < 64) a.prof[(int64_t)gridDim.x * gridDim.y * 8 + 256 + tk * 64 + g] = gtimer();
+        }
+        q = nstage;
+      }
+      if (TC_EXP(262144)) {  // trace experiment: the issue_probe loop (fixed operands) inside this kernel
+        for (int it = 0; it < nstage; ++it) {
+          const int ss = it & 7, bb = it % 6;
+          uint32_t dc = tbase + (uint32_t)(((it >> 3) * 8) % 176);
+          uint32_t id = idesc_bf16(kNWin);
+          uint64_t dg = sdesc(bhi + (uint32_t)(kG - 1) * 16, plane, 128);
+          if (TC_EXP(524288)) {  // + the real window trimming and D column of the stage's group
+            trim(it >> 3);
+            dc = tbase + (uint32_t)(((it >> 3) * kG) % kRelocAt) + (uint32_t)c0;
+            id = idesc_bf16(nN);
+            dg = sdesc(bhi + (uint32_t)(kG - 1 + c0) * 16, plane, 128);
+          }
+          const uint32_t ah = tbase + a_col0 + (uint32_t)(bb * kWB);
+          if (lane == 0) TC_STAMP(3, it);
+          if (leader) {
+#pragma unroll
+            for (int kk = 0; kk < 2; ++kk) {
+              mma_bf16(dc, ah + kk * 8, dg - (uint64_t)ss + kk * kKStep, id);
+              mma_bf16(dc, ah + kk * 8, dg - (uint64_t)ss + dlo_off + kk * kKStep, id);
+              mma_bf16(dc, ah + kWB / 2 + kk * 8, dg - (uint64_t)ss + kk * kKStep, id);
+            }
+            commit_u32(done0 + 8 * bb);
+          }
+          __syncwarp();
+        }
+        q = nstage;
+      }
 #pragma unroll 1
       for (g = 0; q < nstage; ++g) {
         const uint32_t col = (uint32_t)((g * kG) % kRelocAt);
@@ -712,9 +851,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
           fence_after();
           ++nrel_done;
         }
-        if (g >= kGRing) {  // the window's newest columns were drained (and zeroed) after group g - kGRing
+        if (g >= kGRing && !TC_EXP(16)) {  // the window's newest columns were drained (and zeroed) after group g - kGRing
           const unsigned long long t0 = mprof ? gtimer() : 0ull;
-          mbar_wait_u32(drained0 + 8 * ((g - kGRing) % kGRing), (uint32_t)(((g - kGRing) / kGRing) & 1));
+          const uint32_t dr = drained0 + 8 * ((g - kGRing) % kGRing), dp = (uint32_t)(((g - kGRing) / kGRing) & 1);
+          if (!mbar_try_u32(dr, dp)) mbar_wait_u32(dr, dp);
           if (mprof) m_drained += gtimer() - t0;
           fence_after();
         }
@@ -723,41 +863,60 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         const uint32_t id = idesc_bf16(nN);
         // B window of (s = 0, ch = 0): row kG - 1 + c0 of the reversed block
         const uint64_t dg = sdesc(bhi + (uint32_t)(kG - 1 + c0) * 16, plane, 128);
+        // Stages in pairs: both operands' waits first (the producers run several stages ahead, so
+        // both normally succeed at the first try and fall through), then 12 MMAs in straight-line
+        // code.  The tensor pipe queues about one MMA: any branch or dependent scalar latency
+        // between two MMAs is lost tensor time (tools/microbench/issue_probe.cu: 6 MMAs per stage
+        // with a wait and the loop's branches between them cost ~135 cycles per MMA; straight-line
+        // MMAs run at the pipe's rate, 68 cycles at N = 136).
+        const int qend = q + kG * nch;  // nstage is a whole number of groups; kG * nch is even
+        int s0 = 0, c0h = 0;            // (image row in group, column chunk) of stage q
 #pragma unroll 1
-        for (s = 0; s < kG && q < nstage; ++s) {
-#pragma unroll 1
-          for (ch = 0; ch < nch; ++ch, ++q) {
-            if (lane == 0) TC_STAMP(3, q);
-            const uint64_t dh = dg - (uint64_t)s + (uint64_t)(((uint32_t)ch * (kWB / 8) * plane) >> 4);
-            const uint64_t dl = dh + dlo_off;
-            const uint32_t ah = tbase + a_col0 + (uint32_t)(b * kWB), al = ah + kWB / 2;
-            if (leader) {
-#pragma unroll
-              for (int kk = 0; kk < kWB / 16 - 1; ++kk) {
-                mma_bf16(dcol, ah + kk * 8, dh + kk * kKStep, id);
-                mma_bf16(dcol, ah + kk * 8, dl + kk * kKStep, id);
-                mma_bf16(dcol, al + kk * 8, dh + kk * kKStep, id);
-              }
-            }
-            __syncwarp();
-            const int bq = b;
-            if (++b == kNBuf) { b = 0; ph ^= 1; }
-            if (q + 1 < nstage && !TC_EXP(16)) {
-              const unsigned long long t0 = mprof ? gtimer() : 0ull;
-              mbar_wait_u32(full0 + 8 * b, (uint32_t)ph);
-              if (mprof) m_afull += gtimer() - t0;
-            }
-            if (!TC_EXP(16384)) fence_after();
-            if (leader) {
-              constexpr int kk = kWB / 16 - 1;
-              mma_bf16(dcol, ah + kk * 8, dh + kk * kKStep, id);
-              mma_bf16(dcol, ah + kk * 8, dl + kk * kKStep, id);
-              mma_bf16(dcol, al + kk * 8, dh + kk * kKStep, id);
-              commit_u32(done0 + 8 * bq);
-            }
-            __syncwarp();
-            if (lane == 0) TC_STAMP(4, q);
+        for (; q < qend; q += 2) {
+          const int s1 = c0h + 1 < nch ? s0 : s0 + 1, c1 = c0h + 1 < nch ? c0h + 1 : 0;
+          const int b1 = b + 1;  // b is even: the pair shares the phase
+          if (!TC_EXP(16)) {
+            const unsigned long long t0 = mprof ? gtimer() : 0ull;
+            if (!mbar_try_u32(full0 + 8 * b, (uint32_t)ph)) mbar_wait_u32(full0 + 8 * b, (uint32_t)ph);
+            if (!mbar_try_u32(full0 + 8 * b1, (uint32_t)ph)) mbar_wait_u32(full0 + 8 * b1, (uint32_t)ph);
+            if (mprof) m_afull += gtimer() - t0;
           }
+          if (!TC_EXP(16384)) fence_after();
+          if (lane == 0) {
+            TC_STAMP(3, q);
+            TC_STAMP(3, q + 1);
+          }
+          const uint64_t dh0 = dg - (uint64_t)s0 + (uint64_t)(((uint32_t)c0h * (kWB / 8) * plane) >> 4);
+          const uint64_t dh1 = dg - (uint64_t)s1 + (uint64_t)(((uint32_t)c1 * (kWB / 8) * plane) >> 4);
+          const uint32_t ah0 = tbase + a_col0 + (uint32_t)(b * kWB), ah1 = ah0 + kWB;
+          if (leader) {
+#pragma unroll
+            for (int kk = 0; kk < kWB / 16; ++kk) {
+              mma_bf16(dcol, ah0 + kk * 8, dh0 + kk * kKStep, id);
+              mma_bf16(dcol, ah0 + kk * 8, dh0 + dlo_off + kk * kKStep, id);
+              mma_bf16(dcol, ah0 + kWB / 2 + kk * 8, dh0 + kk * kKStep, id);
+            }
+            commit_u32(done0 + 8 * b);
+#pragma unroll
+            for (int kk = 0; kk < kWB / 16; ++kk) {
+              mma_bf16(dcol, ah1 + kk * 8, dh1 + kk * kKStep, id);
+              mma_bf16(dcol, ah1 + kk * 8, dh1 + dlo_off + kk * kKStep, id);
+              mma_bf16(dcol, ah1 + kWB / 2 + kk * 8, dh1 + kk * kKStep, id);
+            }
+            commit_u32(done0 + 8 * b1);
+          }
+          __syncwarp();
+          if (lane == 0) {
+            TC_STAMP(4, q);
+            TC_STAMP(4, q + 1);
+          }
+          b += 2;
+          if (b == kNBuf) {
+            b = 0;
+            ph ^= 1;
+          }
+          s0 = c1 + 1 < nch ? s1 : s1 + 1;
+          c0h = c1 + 1 < nch ? c1 + 1 : 0;
         }
         if (leader) commit_u32(gdone0 + 8 * (g % kGRing));  // group g's MMAs complete -> epilogue drains it
         __syncwarp();
@@ -777,40 +936,46 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 }
 
 // Image operand of the tensor-core numerator: every element of the band's rows split once into
-// (hi = tf32(x) with round-to-nearest, lo = x - hi, exact in fp32), stored as an 8-byte pair so
-// the producer warps load the Hankel elements directly (16-byte loads).  grid = (ceil(W/4/128), rows,
-// batch), block = 128; out row r = image row row0 + r, rows out_pitch (even: 16-byte TMA stride)
-// pairs apart.
+// x = hi + lo (hi = bf16(x), lo = bf16(x - hi), both round-to-nearest), then stored in the layout the
+// producer warps copy into TMEM without any per-element work: with P_k = (hi_k | hi_{k+1} << 16) and
+// Q_k = (lo_k | lo_{k+1} << 16) (zero past the row end), row r holds two planes of 8-byte elements,
+// E_k = (P_k, P_{k+2}) then F_k = (Q_k, Q_{k+2}), k < wp = W rounded up to even (16-byte TMA
+// strides): [batch][rows][2][wp] x 8 bytes (16 bytes per image element).  grid = (ceil(wp/4/128),
+// rows, batch), block = 128, 4 elements per thread.  out row r = image row row0 + r.
 // With `ts` (centred operand): every element is first shifted by the template mean,
 // x = I - tc_center(ts, n) (fp32), so the accumulators hold sum A_C (I - c) -- sums without the
 // image's DC level -- and the epilogue adds c * sum A_C back (exact: tc_center is the same fp32
 // value there).  ts = nullptr: the raw image.
 __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img, int64_t pitch, int64_t frame_stride,
-                                                   int W, int row0, uint32_t* __restrict__ out, int64_t out_frame_stride,
-                                                   int out_pitch, const TemplateStats* ts, double n) {
+                                                   int W, int row0, uint2* __restrict__ out, int64_t out_frame_stride,
+                                                   int wp, const TemplateStats* ts, double n) {
   const int c = (blockIdx.x * 128 + threadIdx.x) * 4;
-  if (c >= W) return;
+  if (c >= wp) return;
   const float cen = tc_center(ts, n);
   const int r = blockIdx.y, f = blockIdx.z;
-  const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch + c;
-  uint32_t* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * out_pitch + c;
-  float x[4];
-  if (c + 4 <= W && (reinterpret_cast<uintptr_t>(src) & 15) == 0) {
-    const float4 v = __ldg(reinterpret_cast<const float4*>(src));
-    x[0] = v.x; x[1] = v.y; x[2] = v.z; x[3] = v.w;
-  } else {
+  const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch;
+  uint2* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * 2 * wp + c;
+  // hi / lo of elements c .. c + 6 (P_{c+3+2} needs element c + 6)
+  uint32_t h[7], l[7];
 #pragma unroll
-    for (int k = 0; k < 4; ++k) x[k] = c + k < W ? __ldg(src + k) : 0.0f;
+  for (int k = 0; k < 7; ++k) {
+    const float x = c + k < W ? __ldg(src + c + k) - cen : 0.0f;
+    const uint32_t s2 = tc::split_bf16(x);
+    h[k] = s2 & 0xffffu;
+    l[k] = s2 >> 16;
+  }
+  uint32_t P[6], Q[6];
+#pragma unroll
+  for (int k = 0; k < 6; ++k) {
+    P[k] = h[k] | (h[k + 1] << 16);
+    Q[k] = l[k] | (l[k + 1] << 16);
   }
 #pragma unroll
-  for (int k = 0; k < 4; ++k) x[k] = c + k < W ? x[k] - cen : 0.0f;
-  uint32_t o[4];
-#pragma unroll
-  for (int k = 0; k < 4; ++k) o[k] = tc::split_bf16(x[k]);
-  if (c + 4 <= W) {
-    reinterpret_cast<uint4*>(dst)[0] = make_uint4(o[0], o[1], o[2], o[3]);
-  } else {
-    for (int k = 0; c + k < W; ++k) dst[k] = o[k];
+  for (int k = 0; k < 4; ++k) {
+    if (c + k < wp) {
+      dst[k] = make_uint2(P[k], P[k + 2]);
+      dst[wp + k] = make_uint2(Q[k], Q[k + 2]);
+    }
   }
 }
 
