@@ -969,31 +969,57 @@ __global__ void __launch_bounds__(128) tm_tc_split(const float* __restrict__ img
                                                    int W, int row0, uint2* __restrict__ out, int64_t out_frame_stride,
                                                    int wp, const TemplateStats* ts, double n) {
   const int c = (blockIdx.x * 128 + threadIdx.x) * 4;
-  if (c >= wp) return;
   const float cen = tc_center(ts, n);
   const int r = blockIdx.y, f = blockIdx.z;
   const float* src = img + (int64_t)f * frame_stride + (int64_t)(row0 + r) * pitch;
-  uint2* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * 2 * wp + c;
-  // hi / lo of elements c .. c + 6 (P_{c+3+2} needs element c + 6)
+  // elements c .. c + 3 (one 16-byte load when aligned); c + 4 .. c + 6 from the next lane
+  float x[4];
+  if (c + 4 <= W && ((reinterpret_cast<uintptr_t>(src + c) & 15) == 0)) {
+    const float4 v = __ldg(reinterpret_cast<const float4*>(src + c));
+    x[0] = v.x; x[1] = v.y; x[2] = v.z; x[3] = v.w;
+  } else {
+#pragma unroll
+    for (int k = 0; k < 4; ++k) x[k] = c + k < W ? __ldg(src + c + k) : 0.0f;
+  }
   uint32_t h[7], l[7];
 #pragma unroll
-  for (int k = 0; k < 7; ++k) {
-    const float x = c + k < W ? __ldg(src + c + k) - cen : 0.0f;
-    const uint32_t s2 = tc::split_bf16(x);
+  for (int k = 0; k < 4; ++k) {
+    const uint32_t s2 = tc::split_bf16(c + k < W ? x[k] - cen : 0.0f);
     h[k] = s2 & 0xffffu;
     l[k] = s2 >> 16;
   }
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int k = 0; k < 3; ++k) {
+    uint32_t hn = __shfl_down_sync(0xffffffffu, h[k], 1), ln = __shfl_down_sync(0xffffffffu, l[k], 1);
+    if (lane == 31) {  // the warp's last lane: its neighbour's elements directly
+      const uint32_t s2 = tc::split_bf16(c + 4 + k < W ? __ldg(src + c + 4 + k) - cen : 0.0f);
+      hn = s2 & 0xffffu;
+      ln = s2 >> 16;
+    }
+    h[4 + k] = hn;
+    l[4 + k] = ln;
+  }
+  if (c >= wp) return;
   uint32_t P[6], Q[6];
 #pragma unroll
   for (int k = 0; k < 6; ++k) {
     P[k] = h[k] | (h[k + 1] << 16);
     Q[k] = l[k] | (l[k + 1] << 16);
   }
+  uint2* dst = out + (int64_t)f * out_frame_stride + (int64_t)r * 2 * wp + c;
+  if (c + 4 <= wp) {  // wp is even and c a multiple of 4: 16-byte aligned pairs of elements
+    reinterpret_cast<uint4*>(dst)[0] = make_uint4(P[0], P[2], P[1], P[3]);
+    reinterpret_cast<uint4*>(dst)[1] = make_uint4(P[2], P[4], P[3], P[5]);
+    reinterpret_cast<uint4*>(dst + wp)[0] = make_uint4(Q[0], Q[2], Q[1], Q[3]);
+    reinterpret_cast<uint4*>(dst + wp)[1] = make_uint4(Q[2], Q[4], Q[3], Q[5]);
+  } else {
 #pragma unroll
-  for (int k = 0; k < 4; ++k) {
-    if (c + k < wp) {
-      dst[k] = make_uint2(P[k], P[k + 2]);
-      dst[wp + k] = make_uint2(Q[k], Q[k + 2]);
+    for (int k = 0; k < 4; ++k) {
+      if (c + k < wp) {
+        dst[k] = make_uint2(P[k], P[k + 2]);
+        dst[wp + k] = make_uint2(Q[k], Q[k + 2]);
+      }
     }
   }
 }
