@@ -719,14 +719,49 @@ __global__ void __launch_bounds__(512) piv_tc_border_rb(const PivTcArgs a, const
   const float* Bw = Bf + (int64_t)(a.pair0 + z) * a.frame_stride + (int64_t)(y - a.my) * a.pitch + x + a.mx;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5, nwarp = nth / 32;
   double s1 = 0.0;
-  for (int i = warp; i < TH; i += nwarp)
-    for (int j = lane; j < w; j += 32) {
-      const float v = __ldg(Aw + (int64_t)i * a.pitch + j);
-      T[i * w + j] = v;
-      s1 += (double)v;
+  // The CTA is load-latency bound (one window's 64-wide strips, ~51 KB): with 16-byte aligned rows
+  // every thread issues all its loads (mask, then search strip) before the first use -- one L2 round
+  // trip instead of a dependent one per row batch (cfg 4: 1.15 ms -> see DESIGN 6.2c per 8 pairs).
+  const bool vec = (a.pitch & 3) == 0 && (x & 3) == 0 && ((x + a.mx) & 3) == 0 && (w & 3) == 0 &&
+                   (reinterpret_cast<uintptr_t>(a.A) & 15) == 0 && (reinterpret_cast<uintptr_t>(Bf) & 15) == 0;
+  if (vec) {
+    constexpr int kTV = (TH * 16 + 511) / 512 + 1, kBV = ((TH + 72) * 16 + 511) / 512 + 1;
+    const int w4 = w >> 2, nT = TH * w4, nB = span * w4;
+    float4 tv[kTV], bv[kBV];
+#pragma unroll
+    for (int k = 0; k < kTV; ++k) {
+      const int e = tid + k * nth;
+      if (e < nT) tv[k] = __ldg(reinterpret_cast<const float4*>(Aw + (int64_t)(e / w4) * a.pitch) + e % w4);
     }
-  for (int i = warp; i < span + kBorderDY - 1; i += nwarp)
-    for (int j = lane; j < w; j += 32) Bc[i * w + j] = i < span ? __ldg(Bw + (int64_t)i * a.pitch + j) : 0.0f;
+#pragma unroll
+    for (int k = 0; k < kBV; ++k) {
+      const int e = tid + k * nth;
+      if (e < nB) bv[k] = __ldg(reinterpret_cast<const float4*>(Bw + (int64_t)(e / w4) * a.pitch) + e % w4);
+    }
+#pragma unroll
+    for (int k = 0; k < kTV; ++k) {
+      const int e = tid + k * nth;
+      if (e < nT) {
+        reinterpret_cast<float4*>(T)[e] = tv[k];
+        s1 += ((double)tv[k].x + (double)tv[k].y) + ((double)tv[k].z + (double)tv[k].w);
+      }
+    }
+#pragma unroll
+    for (int k = 0; k < kBV; ++k) {
+      const int e = tid + k * nth;
+      if (e < nB) reinterpret_cast<float4*>(Bc)[e] = bv[k];
+    }
+    for (int e = nB * 4 + tid; e < (span + kBorderDY - 1) * w; e += nth) Bc[e] = 0.0f;
+  } else {
+    for (int i = warp; i < TH; i += nwarp)
+      for (int j = lane; j < w; j += 32) {
+        const float v = __ldg(Aw + (int64_t)i * a.pitch + j);
+        T[i * w + j] = v;
+        s1 += (double)v;
+      }
+    for (int i = warp; i < span + kBorderDY - 1; i += nwarp)
+      for (int j = lane; j < w; j += 32) Bc[i * w + j] = i < span ? __ldg(Bw + (int64_t)i * a.pitch + j) : 0.0f;
+  }
   s1 = warp_sum_d(s1);
   if (lane == 0) red[warp] = s1;
   __syncthreads();
