@@ -1477,11 +1477,11 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
           (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr, pl->keys, p.score == NCC_SCORE_SSD, pl->tc_done,
           reinterpret_cast<PeakOut*>(d_peaks), nsub);
     } else if (pl->tc_planes) {
-      tm_tc_finish<<<dim3(ceil_div(pl->V, 256 * kFinV), pl->Ub, batch), 256, 0, s>>>(
+      tm_tc_finish<<<dim3(ceil_div(pl->V, 256 * kFinV), ceil_div(pl->Ub, kFinR), batch), 256, 0, s>>>(
           pl->tc_part, nblk, (int64_t)p.batch * pl->Ub * pl->V, (int64_t)pl->Ub * pl->V, pl->tc_rsv, pl->tc_mean,
           pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V, pl->V - pl->tc_vcols, pl->u_begin,
           (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr, (int64_t)pl->Ub * pl->V, pl->keys,
-          p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks), batch);
+          p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks), batch, pl->Ub);
     } else {
       const int64_t tail_items = (int64_t)batch * pl->Ub * pl->tc_vcols;
       tm_tc_tail<<<(unsigned)std::max<int64_t>(1, ceil_div(tail_items, 256)), 256, 0, s>>>(

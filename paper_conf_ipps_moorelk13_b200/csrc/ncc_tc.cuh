@@ -1337,8 +1337,9 @@ __global__ void __launch_bounds__(256) tm_tc_tail(const float* __restrict__ acc,
 // (NCC from the window kernels' fp32 factors, |error| <= ~3e-7; SSD from the fp64 sums), optional
 // surface store, per-frame argmax keys; the last CTA writes every frame's peak.  Columns >= v_cols
 // (the ragged last columns, tm_tc_cols) hold their full numerator in block 0's plane.
-// grid = (ceil(V / (256 kFinV)), Ub, batch), block = 256.
+// grid = (ceil(V / (256 kFinV)), ceil(Ub / kFinR), batch), block = 256.
 constexpr int kFinV = 4;
+constexpr int kFinR = 2;  // output rows per CTA (half the CTAs, and half the same-address atomics, of one row each)
 __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ part, int nblk, int64_t blk_stride,
                                                     int64_t frame_stride, const float* __restrict__ rsv,
                                                     const float* __restrict__ mean, const double* __restrict__ S1,
@@ -1346,61 +1347,78 @@ __global__ void __launch_bounds__(256) tm_tc_finish(const float* __restrict__ pa
                                                     const TemplateStats* tst, int h, int w, int V, int v_cols,
                                                     int u_begin, float* scores, int64_t score_frame_stride,
                                                     unsigned long long* keys, int ssd, unsigned int* __restrict__ done,
-                                                    PeakOut* __restrict__ peaks, int batch) {
+                                                    PeakOut* __restrict__ peaks, int batch, int Ub) {
   __shared__ unsigned long long red[32];
   __shared__ bool last;
-  const int ur = blockIdx.y, f = blockIdx.z;
-  const int u = u_begin + ur;
+  const int f = blockIdx.z;
   const TemplateStats ts = tst[0];
   const double inv_n = 1.0 / ((double)h * (double)w);
   const float csf = (float)ts.csum, rse = ts.flat ? 0.0f : (float)(1.0 / sqrt(ts.energy));
-  const int64_t ro = (int64_t)f * frame_stride + (int64_t)ur * V;
-  const int64_t so = (int64_t)f * stat_frame_stride + (int64_t)ur * V;
   unsigned long long best = 0ull;
   const int vb = blockIdx.x * 256 * kFinV + threadIdx.x;
-  float tot[kFinV], fa[kFinV], fb[kFinV];
+  // every row's loads in flight at once (planes mode has at most 8 blocks), then the block-order
+  // sum ((p0 + p1) + p2) + ... per output (the kernel is load-latency bound)
+  float tot[kFinR][kFinV], fa[kFinR][kFinV], fb[kFinR][kFinV];
 #pragma unroll
-  for (int k = 0; k < kFinV; ++k) {
-    const int v = vb + k * 256;
-    tot[k] = 0.0f;
-    fa[k] = fb[k] = 0.0f;
-    if (v < V && !ssd) {
-      fa[k] = __ldg(rsv + so + v);
-      fb[k] = __ldg(mean + so + v);
-    }
-  }
-  // all planes' loads in flight at once (planes mode has at most 8 blocks), then the block-order sum
-  // ((p0 + p1) + p2) + ...  (the kernel is load-latency bound)
-  for (int b0 = 0; b0 < nblk; b0 += 8) {
-    float x[8][kFinV];
+  for (int rr = 0; rr < kFinR; ++rr) {
+    const int ur = blockIdx.y * kFinR + rr;
+    const int64_t so = (int64_t)f * stat_frame_stride + (int64_t)ur * V;
 #pragma unroll
-    for (int bb = 0; bb < 8; ++bb)
-#pragma unroll
-      for (int k = 0; k < kFinV; ++k) {
-        const int v = vb + k * 256, b = b0 + bb;
-        x[bb][k] = (b < nblk && v < V && (b == 0 || v < v_cols)) ? __ldcg(part + (int64_t)b * blk_stride + ro + v)
-                                                                 : 0.0f;
+    for (int k = 0; k < kFinV; ++k) {
+      const int v = vb + k * 256;
+      tot[rr][k] = 0.0f;
+      fa[rr][k] = fb[rr][k] = 0.0f;
+      if (ur < Ub && v < V && !ssd) {
+        fa[rr][k] = __ldg(rsv + so + v);
+        fb[rr][k] = __ldg(mean + so + v);
       }
+    }
+  }
+  for (int b0 = 0; b0 < nblk; b0 += 4) {
+    float x[kFinR][4][kFinV];
 #pragma unroll
-    for (int bb = 0; bb < 8; ++bb)
+    for (int rr = 0; rr < kFinR; ++rr) {
+      const int ur = blockIdx.y * kFinR + rr;
+      const int64_t ro = (int64_t)f * frame_stride + (int64_t)ur * V;
 #pragma unroll
-      for (int k = 0; k < kFinV; ++k)
-        if (b0 + bb < nblk) tot[k] = (b0 + bb == 0) ? x[bb][k] : tot[k] + x[bb][k];
+      for (int bb = 0; bb < 4; ++bb)
+#pragma unroll
+        for (int k = 0; k < kFinV; ++k) {
+          const int v = vb + k * 256, b = b0 + bb;
+          x[rr][bb][k] = (ur < Ub && b < nblk && v < V && (b == 0 || v < v_cols))
+                             ? __ldcg(part + (int64_t)b * blk_stride + ro + v)
+                             : 0.0f;
+        }
+    }
+#pragma unroll
+    for (int rr = 0; rr < kFinR; ++rr)
+#pragma unroll
+      for (int bb = 0; bb < 4; ++bb)
+#pragma unroll
+        for (int k = 0; k < kFinV; ++k)
+          if (b0 + bb < nblk) tot[rr][k] = (b0 + bb == 0) ? x[rr][bb][k] : tot[rr][k] + x[rr][bb][k];
   }
 #pragma unroll
-  for (int k = 0; k < kFinV; ++k) {
-    const int v = vb + k * 256;
-    if (v >= V) break;
-    float sc;
-    if (ssd) {
-      sc = (float)(ts.sumsq - 2.0 * ((double)tot[k] + ts.sum * inv_n * __ldg(S1 + so + v)) + __ldg(S2 + so + v));
-    } else {
-      const float r = fmaf(-csf, fb[k], tot[k]) * (fa[k] * rse);
-      sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+  for (int rr = 0; rr < kFinR; ++rr) {
+    const int ur = blockIdx.y * kFinR + rr;
+    if (ur >= Ub) break;
+    const int u = u_begin + ur;
+    const int64_t so = (int64_t)f * stat_frame_stride + (int64_t)ur * V;
+#pragma unroll
+    for (int k = 0; k < kFinV; ++k) {
+      const int v = vb + k * 256;
+      if (v >= V) break;
+      float sc;
+      if (ssd) {
+        sc = (float)(ts.sumsq - 2.0 * ((double)tot[rr][k] + ts.sum * inv_n * __ldg(S1 + so + v)) + __ldg(S2 + so + v));
+      } else {
+        const float r = fmaf(-csf, fb[rr][k], tot[rr][k]) * (fa[rr][k] * rse);
+        sc = r > 1.0f ? 1.0f : (r < -1.0f ? -1.0f : r);
+      }
+      if (scores) scores[(int64_t)f * score_frame_stride + (int64_t)ur * V + v] = sc;
+      const unsigned long long key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
+      best = key > best ? key : best;
     }
-    if (scores) scores[(int64_t)f * score_frame_stride + (int64_t)ur * V + v] = sc;
-    const unsigned long long key = make_key(ssd ? -sc : sc, (uint32_t)((int64_t)u * V + v));
-    best = key > best ? key : best;
   }
   best = block_max_key(best, red);
   if (threadIdx.x == 0) {
