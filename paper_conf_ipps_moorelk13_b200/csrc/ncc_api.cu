@@ -1182,8 +1182,13 @@ inline void mark(ncc_plan pl, cudaStream_t s, int i) {
 // pdl: launched as a programmatic dependent of the preceding kernel in `s` (the tensor-core
 // numerator, which triggers it at its start): the window sums then run on the SMs the numerator
 // leaves free, instead of in front of it.
-void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_out, cudaStream_t s, bool pdl = false) {
+void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_out, cudaStream_t s, bool pdl = false,
+                bool factors_only = false) {
   const ncc_problem& p = pl->p;
+  // factors_only: the tensor-core NCC path reads only the fp32 factors (rsqrt(n var), S1/n), not
+  // the fp64 sums (12.9 MB of stores at cfg 2)
+  double* const S1o = factors_only && pl->box_smem ? nullptr : pl->S1;
+  double* const S2o = factors_only && pl->box_smem ? nullptr : pl->S2;
   const int h = p.tmpl_h, w = p.tmpl_w;
   const int V = p.image_w - w + 1;
   if (pl->box_smem) {  // fused single pass; rows per CTA halved until the grid covers every SM
@@ -1206,14 +1211,14 @@ void launch_box(ncc_plan pl, const float* frames, int batch, int row0, int rows_
       const int64_t fs = (int64_t)p.image_h * p.image_pitch, sfs = pl->s_frame_stride;
       const int tv = kBoxTV;
       cudaLaunchKernelEx(&cfg, box2d_kernel<kBox2dNT>, frames, p.image_pitch, fs, row0, h, w, V, rows_out, tv, TU,
-                         pl->box_r, pl->box_iwp, pl->S1, pl->S2, sfs, pl->tc_rsv, pl->tc_mean,
+                         pl->box_r, pl->box_iwp, S1o, S2o, sfs, pl->tc_rsv, pl->tc_mean,
                          1.0 / ((double)h * (double)w));
       return;
     }
     box2d_kernel<kBox2dNT><<<g, kBox2dNT, pl->box_smem, s>>>(frames, p.image_pitch,
                                                             (int64_t)p.image_h * p.image_pitch, row0, h, w, V,
-                                                            rows_out, kBoxTV, TU, pl->box_r, pl->box_iwp, pl->S1,
-                                                            pl->S2, pl->s_frame_stride, pl->tc_rsv, pl->tc_mean,
+                                                            rows_out, kBoxTV, TU, pl->box_r, pl->box_iwp, S1o,
+                                                            S2o, pl->s_frame_stride, pl->tc_rsv, pl->tc_mean,
                                                             1.0 / ((double)h * (double)w));
     return;
   }
@@ -1303,6 +1308,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     tc_now = encode_f32(&map_tc, pl->tc_img2, 4, dims, strides, box, true);
   }
   const int nblk_tc = pl->tc_nbi * pl->tc_nbj;
+  const bool tc_factors_only = tc_now && p.score == NCC_SCORE_NCC;  // no fp64 window-sum stores needed
   auto launch_cols = [&]() {  // the ragged last columns (tensor-core path), on the side stream
     if (pl->h_img_in) cudaStreamWaitEvent(pl->side, pl->ev_img, 0);  // host path: frames copied (errors: cudaGetLastError below)
     // small templates: one output per warp (short CTAs that finish before the tensor-core grid
@@ -1372,7 +1378,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     // numerator waits only for those two and starts on the SMs the window sums leave free
     NCC_CUDA(cudaStreamWaitEvent(pl->side2, pl->ev_fork, 0));
     if (pl->h_img_in) NCC_CUDA(cudaStreamWaitEvent(pl->side2, pl->ev_img, 0));
-    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, pl->side2);
+    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, pl->side2, false, tc_factors_only);
     NCC_CUDA(cudaEventRecord(pl->ev_box, pl->side2));
     if (pl->tc_vcols) {
       launch_cols();
@@ -1388,7 +1394,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       launch_cols();
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }
-    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
+    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, false, tc_factors_only);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
   } else if (tc_now && pl->tc_sched == 3) {
@@ -1402,7 +1408,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     if (!split_side) launch_split(s);
     // planes mode: the numerator does not read the window sums (tm_tc_finish does), so they run
     // after it as its programmatic dependent, on the SMs it leaves free (cfg2: 8 of 148)
-    if (!(pl->tc_planes && pl->box_smem && pl->tc_box_late)) launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
+    if (!(pl->tc_planes && pl->box_smem && pl->tc_box_late)) launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, false, tc_factors_only);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
   } else {
@@ -1412,7 +1418,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       launch_cols();
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }
-    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s);
+    launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, false, tc_factors_only);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
   }
@@ -1465,7 +1471,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
                    tc::smem_bytes(pl->tc_wc), s>>>(
         t, map_tc);
     if (pl->tc_sched == 3 && pl->tc_planes && pl->box_smem && pl->tc_box_late)
-      launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, /*pdl=*/true);
+      launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, /*pdl=*/true, tc_factors_only);
     mark(pl, s, 3);
     if (pl->tc_vcols) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_cols, 0));
     if (box_beside) NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_box, 0));

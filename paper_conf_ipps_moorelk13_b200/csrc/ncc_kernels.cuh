@@ -898,14 +898,16 @@ __global__ void __launch_bounds__(NT, 2)
         y2[k] = p2;
       }
       __syncwarp();
-      double* o1 = S1 + (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
-      double* o2 = S2 + (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
+      // S1 == nullptr: only the fp32 normalisation factors are wanted (tensor-core NCC paths)
+      const int64_t oo = (int64_t)f * s_frame_stride + (int64_t)(ub + r0 + r) * V + v0;
       for (int v = lane; v < tv; v += 32) {
         const double s1 = x1[pidx(v + w - 1)] - (v > 0 ? x1[pidx(v - 1)] : 0.0);
         const double s2 = x2[pidx(v + w - 1)] - (v > 0 ? x2[pidx(v - 1)] : 0.0);
-        o1[v] = s1;
-        o2[v] = s2;
-        if (RSV) window_denoms(s1, s2, inv_n, RSV + (o1 - S1) + v, MEAN + (o1 - S1) + v);
+        if (S1) {
+          S1[oo + v] = s1;
+          S2[oo + v] = s2;
+        }
+        if (RSV) window_denoms(s1, s2, inv_n, RSV + oo + v, MEAN + oo + v);
       }
     }
     __syncthreads();
