@@ -610,7 +610,7 @@ ncc_status setup_tc(ncc_plan pl) {
   // launch order (measured on B200, cfg2 step: 0 -> 0.2135 ms, 3 -> 0.2074 ms; 1/2 delay the
   // tensor-core kernel's start or starve the ragged-column kernel); NCC_TM_SCHED overrides
   pl->tc_sched = getenv("NCC_TM_SCHED") ? atoi(getenv("NCC_TM_SCHED")) : 3;
-  if (pl->tc_sched != 0 && pl->tc_sched != 4 && pl->tc_sched != 5) pl->tc_sched = 3;  // (1/2: retired)
+  if (pl->tc_sched != 0 && pl->tc_sched != 4 && pl->tc_sched != 5 && pl->tc_sched != 6) pl->tc_sched = 3;  // (1/2: retired)
   if (!roi && pl->V > 128 && pl->V % 128 != 0 && pl->V % 128 <= kTcColsMax && w <= 512 && !getenv("NCC_TC_NO_COLS")) {
     pl->tc_vtiles = pl->V / 128;
     pl->tc_vcols = pl->V % 128;
@@ -1397,7 +1397,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, false, tc_factors_only);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
-  } else if (tc_now && pl->tc_sched == 3) {
+  } else if (tc_now && (pl->tc_sched == 3 || pl->tc_sched == 6)) {
     // the image split first (small: it leaves room for the template prep, which starts at once
     // on the side stream), then the window sums on the main stream; the ragged columns follow
     // the template prep on the side stream and overlap the window sums / tensor-core kernel
@@ -1405,10 +1405,21 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
       launch_cols();
       NCC_CUDA(cudaEventRecord(pl->ev_cols, pl->side));
     }
+    if (pl->tc_sched == 6) {
+      // schedule 6: the window sums on a second side stream from the start, beside the image split
+      // (neither reads the other's output); the numerator waits for both
+      NCC_CUDA(cudaStreamWaitEvent(pl->side2, pl->ev_fork, 0));
+      if (pl->h_img_in) NCC_CUDA(cudaStreamWaitEvent(pl->side2, pl->ev_img, 0));
+      launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, pl->side2, false, tc_factors_only);
+      NCC_CUDA(cudaEventRecord(pl->ev_box, pl->side2));
+    }
     if (!split_side) launch_split(s);
     // planes mode: the numerator does not read the window sums (tm_tc_finish does), so they run
     // after it as its programmatic dependent, on the SMs it leaves free (cfg2: 8 of 148)
-    if (!(pl->tc_planes && pl->box_smem && pl->tc_box_late)) launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, false, tc_factors_only);
+    if (pl->tc_sched == 6)
+      NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_box, 0));
+    else if (!(pl->tc_planes && pl->box_smem && pl->tc_box_late))
+      launch_box(pl, d_images, batch, pl->u_begin, pl->Ub, s, false, tc_factors_only);
     NCC_CUDA(cudaStreamWaitEvent(s, pl->ev_join, 0));
     mark(pl, s, 2);
   } else {
@@ -1424,7 +1435,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
   }
   if (tc_now) {  // tensor-core numerator, then block sum + normalisation + argmax
     const int nblk = nblk_tc;
-    if (!split_side && !box_beside && pl->tc_sched != 3) launch_split(s);  // schedules 0 / 5-chain
+    if (!split_side && !box_beside && pl->tc_sched != 3 && pl->tc_sched != 6) launch_split(s);  // schedules 0 / 5-chain
     TcArgs t;
     t.H = p.image_h;
     t.W = p.image_w;

@@ -3,7 +3,7 @@
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > gpurun_out/build.log 2>&1
-for v in "NCC_TM_SCHED=3" "NCC_TM_SCHED=5" "NCC_TM_SCHED=4" "NCC_TM_SCHED=0" "NCC_TC_BOX_LATE=1" "NCC_TM_SCHED=3"; do
+for v in ${SCHEDS:-"NCC_TM_SCHED=3" "NCC_TM_SCHED=5" "NCC_TM_SCHED=4" "NCC_TM_SCHED=0" "NCC_TC_BOX_LATE=1" "NCC_TM_SCHED=3"}; do
   env $v timeout 300 python bench.py --workload cfg2 --no-secondary --no-cpu-baseline --steps 40 > gpurun_out/ab.json 2>/dev/null
   python -c "
 import json,sys
