@@ -286,8 +286,8 @@ def roofline(ctx, plan, flops, num_avg, step_ms, clocks, cfg, pairs=None):
             peak_note = (f"3xBF16 fp32-equivalent tensor peak = {'measured' if mp else 'fallback'} bf16 GEMM "
                          f"{bf16:.1f} TFLOP/s / 3 MMAs per MAC")
             issue_peak = sms * 8192 * max_mhz * 1e6 / 3.0 / 1e12
-            issue_note = ("SMs x 8192 bf16 FLOP/cycle (probe: M=128 K=16 MMA of width N >= 90 takes N/2 cycles; "
-                          "narrower ones 45 cycles) x max SM clock / 3")
+            issue_note = ("SMs x 8192 bf16 FLOP/cycle (probe: an M=128 K=16 MMA of width N takes N/2 cycles when "
+                          "issued back to back, tools/microbench/issue_probe.cu) x max SM clock / 3")
         else:
             # 3xTF32 on tcgen05: 3 tf32 MMAs per fp32 MAC.  tf32 peak = measured bf16 GEMM peak x the
             # nominal tf32/bf16 ratio (1.1 / 2.25 PFLOP/s); the fp32-equivalent peak is a third of it.
