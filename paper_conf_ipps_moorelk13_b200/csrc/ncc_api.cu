@@ -1685,7 +1685,7 @@ ncc_status run_piv(ncc_plan pl, const float* A, const float* B, float* d_scores,
       mark(pl, s, 3 * sb + 3);
       continue;
     }
-    launch_box(pl, B + p0 * fs, np, 0, pl->map_h, s);
+    launch_box(pl, B + p0 * fs, np, 0, pl->map_h, s, false, pl->ptc && p.score == NCC_SCORE_NCC);  // the tensor-core PIV path reads only the fp32 factors
     mark(pl, s, 3 * sb + 1);
     a.pair0 = p0;
     dim3 grid(groups, 1, np);
