@@ -108,7 +108,7 @@ def test_c_example_compiles_against_the_header(tmp_path):
 
 
 def test_experiments_tables_match_the_committed_sweep(tmp_path):
-    """EXPERIMENTS.md's tables are generated from profiles/r01_paper_sweeps.jsonl
+    """EXPERIMENTS.md's tables are generated from profiles/r02_paper_sweeps.jsonl
     (tools/experiments_md.py): regenerating them from the committed measurements changes
     nothing, and every sweep run was correct against its planted input."""
     import json
@@ -116,7 +116,7 @@ def test_experiments_tables_match_the_committed_sweep(tmp_path):
     import subprocess
     import sys
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    src = os.path.join(root, "profiles", "r01_paper_sweeps.jsonl")
+    src = os.path.join(root, "profiles", "r02_paper_sweeps.jsonl")
     md = tmp_path / "EXPERIMENTS.md"
     shutil.copy(os.path.join(root, "EXPERIMENTS.md"), md)
     subprocess.run([sys.executable, os.path.join(root, "tools", "experiments_md.py"), src, str(md)], check=True)

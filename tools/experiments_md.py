@@ -1,5 +1,5 @@
 #!/usr/bin/env python
-"""Regenerate the tables of EXPERIMENTS.md from profiles/r01_paper_sweeps.jsonl (the output of
+"""Regenerate the tables of EXPERIMENTS.md from profiles/r02_paper_sweeps.jsonl (the output of
 tools/paper_sweeps.py): every '| ... |' table block that follows a '## Tab ...' heading is
 replaced; headings and prose stay.  Usage: python tools/experiments_md.py [jsonl] [md]"""
 import json
@@ -39,7 +39,7 @@ def tables(rows):
 
 
 def main():
-    src = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "r01_paper_sweeps.jsonl")
+    src = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "profiles", "r02_paper_sweeps.jsonl")
     md = sys.argv[2] if len(sys.argv) > 2 else os.path.join(ROOT, "EXPERIMENTS.md")
     rows = [json.loads(l) for l in open(src) if l.strip().startswith("{")]
     tabs = tables(rows)
