@@ -726,32 +726,43 @@ __global__ void __launch_bounds__(512) piv_tc_border_rb(const PivTcArgs a, const
                    (reinterpret_cast<uintptr_t>(a.A) & 15) == 0 && (reinterpret_cast<uintptr_t>(Bf) & 15) == 0;
   if (vec) {
     constexpr int kTV = (TH * 16 + 511) / 512 + 1, kBV = ((TH + 72) * 16 + 511) / 512 + 1;
-    const int w4 = w >> 2, nT = TH * w4, nB = span * w4;
+    const int w4 = w >> 2, lw4 = __ffs(w4) - 1, nT = TH * w4, nB = span * w4;  // w4 = 8 or 16
     float4 tv[kTV], bv[kBV];
 #pragma unroll
     for (int k = 0; k < kTV; ++k) {
       const int e = tid + k * nth;
-      if (e < nT) tv[k] = __ldg(reinterpret_cast<const float4*>(Aw + (int64_t)(e / w4) * a.pitch) + e % w4);
+      if (e < nT) tv[k] = __ldg(reinterpret_cast<const float4*>(Aw + (int64_t)(e >> lw4) * a.pitch) + (e & (w4 - 1)));
     }
 #pragma unroll
     for (int k = 0; k < kBV; ++k) {
       const int e = tid + k * nth;
-      if (e < nB) bv[k] = __ldg(reinterpret_cast<const float4*>(Bw + (int64_t)(e / w4) * a.pitch) + e % w4);
+      if (e < nB) bv[k] = __ldg(reinterpret_cast<const float4*>(Bw + (int64_t)(e >> lw4) * a.pitch) + (e & (w4 - 1)));
     }
 #pragma unroll
-    for (int k = 0; k < kTV; ++k) {
-      const int e = tid + k * nth;
-      if (e < nT) {
-        reinterpret_cast<float4*>(T)[e] = tv[k];
-        s1 += ((double)tv[k].x + (double)tv[k].y) + ((double)tv[k].z + (double)tv[k].w);
-      }
-    }
+    for (int k = 0; k < kTV; ++k)
+      if (tid + k * nth < nT) s1 += ((double)tv[k].x + (double)tv[k].y) + ((double)tv[k].z + (double)tv[k].w);
 #pragma unroll
     for (int k = 0; k < kBV; ++k) {
       const int e = tid + k * nth;
       if (e < nB) reinterpret_cast<float4*>(Bc)[e] = bv[k];
     }
     for (int e = nB * 4 + tid; e < (span + kBorderDY - 1) * w; e += nth) Bc[e] = 0.0f;
+    // mean over the mask, then the centred mask stored straight from the registers (no second
+    // pass over shared memory)
+    s1 = warp_sum_d(s1);
+    if (lane == 0) red[warp] = s1;
+    __syncthreads();
+    double tot = 0.0;
+    for (int q = 0; q < nwarp; ++q) tot += red[q];
+    const double mean = tot / ((double)TH * (double)w);
+#pragma unroll
+    for (int k = 0; k < kTV; ++k) {
+      const int e = tid + k * nth;
+      if (e < nT)
+        reinterpret_cast<float4*>(T)[e] = make_float4((float)((double)tv[k].x - mean), (float)((double)tv[k].y - mean),
+                                                      (float)((double)tv[k].z - mean), (float)((double)tv[k].w - mean));
+    }
+    __syncthreads();
   } else {
     for (int i = warp; i < TH; i += nwarp)
       for (int j = lane; j < w; j += 32) {
@@ -761,16 +772,16 @@ __global__ void __launch_bounds__(512) piv_tc_border_rb(const PivTcArgs a, const
       }
     for (int i = warp; i < span + kBorderDY - 1; i += nwarp)
       for (int j = lane; j < w; j += 32) Bc[i * w + j] = i < span ? __ldg(Bw + (int64_t)i * a.pitch + j) : 0.0f;
+    s1 = warp_sum_d(s1);
+    if (lane == 0) red[warp] = s1;
+    __syncthreads();
+    double tot = 0.0;
+    for (int q = 0; q < nwarp; ++q) tot += red[q];
+    const double mean = tot / ((double)TH * (double)w);
+    for (int i = warp; i < TH; i += nwarp)
+      for (int jj = lane; jj < w; jj += 32) T[i * w + jj] = (float)((double)T[i * w + jj] - mean);
+    __syncthreads();
   }
-  s1 = warp_sum_d(s1);
-  if (lane == 0) red[warp] = s1;
-  __syncthreads();
-  double tot = 0.0;
-  for (int q = 0; q < nwarp; ++q) tot += red[q];
-  const double mean = tot / ((double)TH * (double)w);
-  for (int i = warp; i < TH; i += nwarp)
-    for (int jj = lane; jj < w; jj += 32) T[i * w + jj] = (float)((double)T[i * w + jj] - mean);
-  __syncthreads();
   const int b = warp & 7, c = warp >> 3, j = 32 * c + lane, dy0 = kBorderDY * b;
   float tr[TH];  // the thread's template column, pinned in registers (volatile loads: not re-read per use)
 #pragma unroll
