@@ -354,7 +354,7 @@ struct ncc_plan_s {
   TemplateStats* tst;
   unsigned long long* keys;
   // PIV
-  int Ky, Kx, OY, OX, sub_batch, piv_bp, piv_smem, map_w, map_h;
+  int Ky, Kx, OY, OX, sub_batch, host_chunk, piv_bp, piv_smem, map_w, map_h;
   int ws_smem, ws_grid;  // persistent warp-specialised PIV kernel (0: not used)
   int ws_bp;             // its staged pitch = TMA box width
   const PivVariant* pivv;
@@ -1061,41 +1061,59 @@ ncc_status create_piv(ncc_plan pl) {
   NCC_CUDA(cudaFuncSetAttribute((const void*)box_rows_kernel<kBoxRowsNT>,
                                 cudaFuncAttributeMaxDynamicSharedMemorySize, rows_smem));
 
-  // window-sum maps of frame B, processed in sub-batches of pairs (scratch budget ~2 GiB)
+  // window-sum maps of frame B, processed in sub-batches of pairs
   pl->rs_frame_stride = (int64_t)p.image_h * pl->map_w;
   pl->s_frame_stride = (int64_t)pl->map_h * pl->map_w;
   ncc_status st;
   if ((st = setup_box(pl, w))) return st;
-  const double per_pair = 16.0 * (double)((pl->box_smem ? 0 : pl->rs_frame_stride) + pl->s_frame_stride);
-  int sb = (int)(2.0 * 1024 * 1024 * 1024 / per_pair);
-  if (sb < 1) sb = 1;
-  if (const char* e = getenv("NCC_PIV_SUB_BATCH")) sb = std::min(sb, std::max(1, atoi(e)));  // tests / sweeps
-  if (sb > p.batch) sb = p.batch;
-  pl->sub_batch = sb;
-  if (!pl->box_smem) {
-    if ((st = dalloc(&pl->RS1, (size_t)sb * pl->rs_frame_stride))) return st;
-    if ((st = dalloc(&pl->RS2, (size_t)sb * pl->rs_frame_stride))) return st;
-  }
-  if ((st = dalloc(&pl->S1, (size_t)sb * pl->s_frame_stride))) return st;
-  if ((st = dalloc(&pl->S2, (size_t)sb * pl->s_frame_stride))) return st;
   // tensor-core numerator (f3 on the PIV path, ncc_piv_tc.cuh): NCC score, D_x = 2 m_x in {32, 64}
   // (R = 128 / D_x image rows per MMA), whole 16-column template chunks, and the overlapping windows
   // of a column strip fit the accumulator / operand slots.  NCC_PIV_TC=0 (or NCC_F_CUDA_CORES) keeps
   // the CUDA-core kernels.
+  const char* e_ptc = getenv("NCC_PIV_TC");
+  const int Dx = 2 * mx, R_ptc = (Dx == 32 || Dx == 64) ? 128 / Dx : 1, span_ptc = h + 2 * my;
+  const bool ptc_ok = p.score == NCC_SCORE_NCC && !(p.flags & NCC_F_CUDA_CORES) && !(e_ptc && atoi(e_ptc) == 0) &&
+                      (Dx == 32 || Dx == 64) && w % ptc::kKs == 0 && (h * w) % 128 == 0 &&
+                      h * w <= 128 * ptc::kPrepMax && p.step_y % R_ptc == 0 && p.step_y <= span_ptc &&
+                      (span_ptc + p.step_y - 1) / p.step_y <= ptc::kNSlot - 1 && p.step_x % 4 == 0 &&
+                      p.image_pitch % 4 == 0 && Dx + w <= 256 && ptc::tmem_cols(my, R_ptc, w) <= 512 &&
+                      ptc::smem_bytes(h, w, my, mx) <= maxsm && (2 * my + 1) * (2 * mx + 1) <= 128 * ptc::kEpiMax &&
+                      2 * my + 1 <= 8 * kBorderDY;
+  // default: the tensor cores where they measured faster (R = 2, +-32 search: cfg 4, 2.6x);
+  // at R = 4 (+-16, cfg 3) the CUDA-core kernel wins (EXPERIMENTS.md); NCC_PIV_TC=1 forces them
+  const bool use_ptc = ptc_ok && (R_ptc == 2 || (e_ptc && atoi(e_ptc) == 1));
+  // Sub-batch sizing.  The CUDA-core kernels read fp64 window sums (16 B per map position, scratch
+  // budget ~2 GiB); the tensor-core path reads only the fp32 factors (8 B) and its last-column
+  // numerators, so its budget is 8 GiB -- cfg 4's 256 pairs in ONE sub-batch: the persistent
+  // kernel's units (strips) then balance over the SMs to ~0.5 % instead of one partly filled wave
+  // per 34-pair sub-batch (~7 %).  Sub-batches are equal-sized.  The host path streams chunks of
+  // the 2 GiB size regardless (copy / compute overlap).
+  const double per_pair_fp64 = 16.0 * (double)((pl->box_smem ? 0 : pl->rs_frame_stride) + pl->s_frame_stride);
+  int sb_host = std::max(1, (int)(2.0 * 1024 * 1024 * 1024 / per_pair_fp64));
+  int sb = sb_host;
+  if (use_ptc && pl->box_smem) {
+    const double per_pair = 8.0 * (double)pl->s_frame_stride + 4.0 * (double)pl->Ky * pl->Kx * pl->OY;
+    sb = std::max(1, (int)(8.0 * 1024 * 1024 * 1024 / per_pair));
+  }
+  if (const char* e = getenv("NCC_PIV_SUB_BATCH")) {  // tests / sweeps
+    sb = std::min(sb, std::max(1, atoi(e)));
+    sb_host = std::min(sb_host, sb);
+  }
+  if (sb > p.batch) sb = p.batch;
+  sb = ceil_div(p.batch, ceil_div(p.batch, sb));  // equal sub-batches
+  pl->sub_batch = sb;
+  pl->host_chunk = std::min(sb, std::min(sb_host, p.batch));
+  if (!pl->box_smem) {
+    if ((st = dalloc(&pl->RS1, (size_t)sb * pl->rs_frame_stride))) return st;
+    if ((st = dalloc(&pl->RS2, (size_t)sb * pl->rs_frame_stride))) return st;
+  }
+  if (!(use_ptc && pl->box_smem)) {  // fp64 sums (the tensor-core path with the fused box kernel writes none)
+    if ((st = dalloc(&pl->S1, (size_t)sb * pl->s_frame_stride))) return st;
+    if ((st = dalloc(&pl->S2, (size_t)sb * pl->s_frame_stride))) return st;
+  }
   {
-    const char* e = getenv("NCC_PIV_TC");
-    const int Dx = 2 * mx, R = (Dx == 32 || Dx == 64) ? 128 / Dx : 1, span = h + 2 * my;
-    const bool ok = p.score == NCC_SCORE_NCC && !(p.flags & NCC_F_CUDA_CORES) && !(e && atoi(e) == 0) &&
-                    (Dx == 32 || Dx == 64) && w % ptc::kKs == 0 && (h * w) % 128 == 0 &&
-                    h * w <= 128 * ptc::kPrepMax && p.step_y % R == 0 && p.step_y <= span &&
-                    (span + p.step_y - 1) / p.step_y <= ptc::kNSlot - 1 && p.step_x % 4 == 0 &&
-                    p.image_pitch % 4 == 0 && Dx + w <= 256 && ptc::tmem_cols(my, R, w) <= 512 &&
-                    ptc::smem_bytes(h, w, my, mx) <= maxsm && (2 * my + 1) * (2 * mx + 1) <= 128 * ptc::kEpiMax &&
-                    2 * my + 1 <= 8 * kBorderDY;
-    // default: the tensor cores where they measured faster (R = 2, +-32 search: cfg 4, 1.6x);
-    // at R = 4 (+-16, cfg 3) the CUDA-core kernel wins (EXPERIMENTS.md); NCC_PIV_TC=1 forces them
-    const bool worth = R == 2 || (e && atoi(e) == 1);
-    if (ok && worth) {
+    const int R = R_ptc, span = span_ptc;
+    if (use_ptc) {
       pl->ptc = 1;
       pl->ptc_R = R;
       pl->ptc_smem = ptc::smem_bytes(h, w, my, mx);
@@ -2163,7 +2181,7 @@ ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, p
   const size_t fb = (size_t)p.batch * p.image_h * p.image_pitch * sizeof(float);
   const size_t vb = (size_t)p.batch * pl->Ky * pl->Kx * sizeof(piv_vector);
   ncc_status st;
-  const int chunk = pl->sub_batch;
+  const int chunk = pl->host_chunk;  // the copy / compute overlap granularity (<= the device sub-batch)
   if (p.batch <= chunk) {  // one chunk: copy in, run, copy out
     if ((st = stage((void**)&pl->st_a, &pl->st_a_bytes, fb))) return st;
     if ((st = stage((void**)&pl->st_b, &pl->st_b_bytes, fb))) return st;
@@ -2179,7 +2197,7 @@ ncc_status piv_correlate_host(ncc_plan pl, const float* h_a, const float* h_b, p
     NCC_CUDA(cudaMemcpyAsync(h_vec, pl->st_out, vb, cudaMemcpyDeviceToHost, s));
     return NCC_OK;
   }
-  // Streaming: chunks of sub_batch pairs through two device slots.  The host->device copy of
+  // Streaming: chunks of host_chunk pairs through two device slots.  The host->device copy of
   // chunk c + 1 runs on the plan's copy stream while chunk c is correlated on `stream`; a slot
   // is refilled only after the chunk that used it (and its vectors' copy-back) is done.
   if ((st = ensure_copy_stream(pl))) return st;
