@@ -195,3 +195,31 @@ def test_default_selection(monkeypatch):
         assert plan.info.variant_name.decode().startswith("piv_tc_bf16x3_64x64_m32x32_r2")
     with PivPlan(512, 512, 32, 16, 16, pairs=1) as plan:
         assert plan.info.variant_name.decode().startswith("piv_ws2")
+
+
+def test_equal_sub_batches_and_host_chunks_bitwise(monkeypatch):
+    """The tensor-core path's sub-batching (equal-sized sub-batches within an 8 GiB factors budget;
+    NCC_PIV_SUB_BATCH caps it) and the host path's streamed chunks change no bit: 5 pairs as one
+    launch, as sub-batches of 2 + 2 + 1, and through piv_correlate_host in chunks."""
+    cv, specs = synth.piv_batch_from_canvases(4, 5, canvases=2)
+    As = np.ascontiguousarray(np.stack([cv[ci][ay:ay + 384, ax:ax + 384] for (ci, ay, ax, by, bx, _) in specs]))
+    Bs = np.ascontiguousarray(np.stack([cv[ci][by:by + 384, bx:bx + 384] for (ci, ay, ax, by, bx, _) in specs]))
+    v0, s0, info = run(list(As), list(Bs), 64, 32, 32)
+    assert info["variant_name"].startswith("piv_tc"), info["variant_name"]
+    monkeypatch.setenv("NCC_PIV_SUB_BATCH", "2")
+    v1, s1, _ = run(list(As), list(Bs), 64, 32, 32)
+    np.testing.assert_array_equal(s0, s1)
+    for k in v0:
+        np.testing.assert_array_equal(v0[k], v1[k])
+    hA = torch.from_numpy(As).pin_memory()
+    hB = torch.from_numpy(Bs).pin_memory()
+    with PivPlan(384, 384, 64, 32, 32, pairs=5) as plan:
+        hv = torch.full((5,) + plan.grid + (6,), -1, dtype=torch.int32).pin_memory()
+        for _ in range(2):  # the second call reuses the chunk slots
+            plan.correlate_host(hA, hB, hv)
+        torch.cuda.synchronize()
+    d = {k: x.numpy() for k, x in decode_vectors(hv).items()}
+    for k in v0:
+        np.testing.assert_array_equal(d[k], v0[k])
+    for pi, (_, _, _, _, _, (dy, dx)) in enumerate(specs):
+        assert np.all(v0["iy"][pi] == dy) and np.all(v0["ix"][pi] == dx)
