@@ -374,6 +374,7 @@ struct ncc_plan_s {
                  // then window sums || template prep + ragged columns
   float *tcB, *tc_acc;     // reversed template-block operands; running numerator (one plane, chain mode)
   int tc_planes;           // planes mode (few template blocks): per-block partial planes + tm_tc_finish
+  int tc_clen, tc_nplanes; // blocks per chain (1: planes, nblk: one chain), planes tm_tc_finish sums
   int tc_box_late;         // planes mode: window sums after the numerator, as its programmatic dependent
   float* tc_part;          // [nblk][batch][Ub][V] partial numerators (planes mode)
   unsigned int* tc_done;   // finished tm_tc_tail CTAs (self-resetting)
@@ -667,18 +668,31 @@ ncc_status setup_tc(ncc_plan pl) {
   ncc_status st;
   if ((st = dalloc(&pl->tcB, (size_t)pl->n_tmpl * nblk * (tc::b_bytes(pl->tc_wc) / 4)))) return st;
   // Few template blocks (cfg2: 4): each block writes its own partial plane (no waiting between
-  // CTAs) and tm_tc_finish sums them in block order; many (cfg5: 64): the in-kernel chain, one
-  // plane whatever the block count (64 planes were 3.4 GB of writes per cfg5 call).
-  // NCC_TC_PLANES=0/1 overrides.
-  pl->tc_planes = nblk <= 8;
-  if (const char* e = getenv("NCC_TC_PLANES")) pl->tc_planes = atoi(e) != 0;
-  if (roi) pl->tc_planes = 1;  // ROI mode: planes (small per-ROI planes, any block count)
-  pl->tc_box_late = getenv("NCC_TC_BOX_LATE") ? atoi(getenv("NCC_TC_BOX_LATE")) : 0;  // measured: slower
-  if (pl->tc_planes) {
-    if ((st = dalloc(&pl->tc_part, (size_t)nblk * nsub * rows * cols))) return st;
-  } else if ((st = dalloc(&pl->tc_acc, (size_t)p.batch * pl->Ub * pl->V))) {
-    return st;
+  // CTAs) and tm_tc_finish sums them in block order.  Many (cfg5: 64): "chained planes" -- chains of
+  // ceil(nblk / 16) consecutive blocks accumulate in-kernel (block b adds its sums to the running
+  // numerator block b - 1 of its chain published), each chain's last block writes one plane, and
+  // tm_tc_finish sums the <= 16 planes in order: per output ((p_0 + p_1) + ...) in block order, as
+  // in both pure forms.  Measured at cfg5 (ms per step): one 64-block chain 19.4-20.3 (every CTA
+  // waits for its predecessors' start-up), 64 planes 18.3 (3.4 GB of writes), chains of 16 / 8 / 4
+  // blocks 18.8 / 18.8 / 18.3 (0.2 / 0.4 / 0.8 GB).  NCC_TC_PLANES=0 (one chain) / 1 (pure planes)
+  // and NCC_TC_CLEN override.
+  pl->tc_planes = 1;
+  pl->tc_clen = nblk <= 8 ? 1 : ceil_div(nblk, 16);
+  if (const char* e = getenv("NCC_TC_PLANES")) {
+    pl->tc_planes = atoi(e) != 0;
+    pl->tc_clen = pl->tc_planes ? 1 : nblk;
   }
+  if (const char* e = getenv("NCC_TC_CLEN")) pl->tc_clen = std::max(1, std::min(nblk, atoi(e)));
+  if (roi) {  // ROI mode: planes (small per-ROI planes, any block count)
+    pl->tc_planes = 1;
+    pl->tc_clen = 1;
+  }
+  pl->tc_nplanes = ceil_div(nblk, pl->tc_clen);
+  pl->tc_box_late = getenv("NCC_TC_BOX_LATE") ? atoi(getenv("NCC_TC_BOX_LATE")) : 0;  // measured: slower
+  if (pl->tc_planes && (st = dalloc(&pl->tc_part, (size_t)pl->tc_nplanes * nsub * rows * cols))) return st;
+  if ((pl->tc_clen > 1 || !pl->tc_planes) &&  // running numerators: one plane per chain
+      (st = dalloc(&pl->tc_acc, (size_t)pl->tc_nplanes * p.batch * pl->Ub * pl->V)))
+    return st;
   pl->tc_ngrp = ceil_div(pl->tc_useg + tc::kHB - 1, tc::kG);
   pl->tc_exp = getenv("NCC_TC_EXP") ? atoi(getenv("NCC_TC_EXP")) : 0;
   pl->tc_center = getenv("NCC_TC_CENTER") ? atoi(getenv("NCC_TC_CENTER")) : 0;
@@ -687,7 +701,7 @@ ncc_status setup_tc(ncc_plan pl) {
     if ((st = dalloc(&pl->tc_prof, n))) return st;
     NCC_CUDA(cudaMemset(pl->tc_prof, 0, n * 8));
   }
-  const size_t nflags = (size_t)p.batch * pl->tc_vtiles * pl->tc_nseg * pl->tc_ngrp * 4;
+  const size_t nflags = (size_t)p.batch * pl->tc_vtiles * pl->tc_nseg * pl->tc_nplanes * pl->tc_ngrp * 4;
   if ((st = dalloc(&pl->tc_flags, nflags))) return st;
   NCC_CUDA(cudaMemset(pl->tc_flags, 0, nflags * sizeof(unsigned int)));
   if ((st = dalloc(&pl->tc_ticket, (size_t)1))) return st;
@@ -706,8 +720,12 @@ ncc_status setup_tc(ncc_plan pl) {
                                 kPrepSmemFloats * 4));
   pl->tc = 1;
   ncc_plan_info& in = pl->info;
+  char mode_s[24];
+  if (!pl->tc_planes) snprintf(mode_s, sizeof(mode_s), "chain");
+  else if (pl->tc_clen == 1) snprintf(mode_s, sizeof(mode_s), "planes");
+  else snprintf(mode_s, sizeof(mode_s), "chain%d_planes%d", pl->tc_clen, pl->tc_nplanes);
   snprintf(in.variant_name, sizeof(in.variant_name), "tm_tc_bf16x3_hb%d_wc%d_seg%d_%s%s%s", tc::kHB, pl->tc_wc,
-           pl->tc_nseg, pl->tc_planes ? "planes" : "chain", pl->tc_vcols ? "_cols" : "", roi ? "_roi" : "");
+           pl->tc_nseg, mode_s, pl->tc_vcols ? "_cols" : "", roi ? "_roi" : "");
   fill_kernel_info(pl, (const void*)tm_tc_kernel, tc::kThreads, smem, nblk * pl->tc_vtiles * pl->tc_nseg, nsub, 1);
   in.specialized = 3;  // tensor-core tier: one kernel for every shape (h, w run-time evaluated), not an SK
   in.split = nblk;
@@ -1469,6 +1487,8 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
     t.vtiles = pl->tc_vtiles;
     t.acc = pl->tc_acc;
     t.planes = pl->tc_planes;
+    t.clen = pl->tc_clen;
+    t.acc_chain_stride = (int64_t)p.batch * pl->Ub * pl->V;
     t.rois = pl->roi_mode ? d_rois : nullptr;
     t.n_tmpl = pl->n_tmpl;
     t.roi_h = p.roi_h;
@@ -1513,7 +1533,7 @@ ncc_status run_match(ncc_plan pl, const float* d_images, const float* d_tmpl, in
           reinterpret_cast<PeakOut*>(d_peaks), nsub);
     } else if (pl->tc_planes) {
       tm_tc_finish<<<dim3(ceil_div(pl->V, 256 * kFinV), ceil_div(pl->Ub, kFinR), batch), 256, 0, s>>>(
-          pl->tc_part, nblk, (int64_t)p.batch * pl->Ub * pl->V, (int64_t)pl->Ub * pl->V, pl->tc_rsv, pl->tc_mean,
+          pl->tc_part, pl->tc_nplanes, (int64_t)p.batch * pl->Ub * pl->V, (int64_t)pl->Ub * pl->V, pl->tc_rsv, pl->tc_mean,
           pl->S1, pl->S2, pl->s_frame_stride, pl->tst, p.tmpl_h, p.tmpl_w, pl->V, pl->V - pl->tc_vcols, pl->u_begin,
           (p.flags & NCC_F_WRITE_SURFACE) ? d_scores : nullptr, (int64_t)pl->Ub * pl->V, pl->keys,
           p.score == NCC_SCORE_SSD, pl->tc_done, reinterpret_cast<PeakOut*>(d_peaks), batch, pl->Ub);

@@ -251,8 +251,11 @@ struct TcArgs {
   // gone): block b > 0 adds its drained rows to the running numerator block b - 1 left in `acc`
   // (per-row-group, per-warp flags), the last block normalises them in the same drain.
   float* acc;              // [batch][u_end - u_begin][V] running numerator (one plane; chain mode)
-  int planes;              // 1: planes mode -- block b writes its partial sums to part + b part_blk_stride
-  float* part;             //    (summed in block order by tm_tc_finish); 0: the chain
+  int planes;              // 1: planes mode -- the partial sums go to planes part + c part_blk_stride
+  float* part;             //    (summed in plane order by tm_tc_finish); 0: the chain normalises in-kernel
+  int clen;                // blocks per chain: planes mode 1 (plane c = block c), chain mode nblk (one chain);
+                           // between: "chained planes" -- chains of clen blocks, plane c = chain c's sum
+  int64_t acc_chain_stride;  // running-numerator plane of chain c: acc + c acc_chain_stride
   int64_t part_blk_stride;
   int64_t acc_frame_stride;
   unsigned int* flags;     // [batch][vtiles * nseg][ngrp_max][4]: blocks done with a row group
@@ -550,6 +553,12 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
     // independent of bands and segments.
     const int cw = warp - kChainWarp0;
     const bool last_blk = blk == nblk - 1;
+    // chain of this block (chained planes: the plane index too) and its position in the chain
+    const int cid = blk / a.clen, nchains = (nblk + a.clen - 1) / a.clen;
+    const bool chained = a.clen > 1, cfirst = blk % a.clen == 0, clast = blk % a.clen == a.clen - 1 || last_blk;
+    auto flag_ptr = [&](int g) {
+      return a.flags + (((int64_t)(f * a.vtiles * a.nseg + tile) * nchains + cid) * a.ngrp_max + g) * 4 + cw;
+    };
     const float* stg = reinterpret_cast<const float*>(smem_tc + stage_off(a.WC)) + cw * 64 + lane;
     unsigned long long* prof = (a.exp & 32) && lane == 0 && cw == 0 ? a.prof + (int64_t)tk * 8 : nullptr;
     unsigned long long p_flag = 0, p_grp = 0, p_chain = 0;
@@ -565,14 +574,14 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
       colok[j] = vcol[j] >= rv0 && vcol[j] < vend;
       cb[j] = (int64_t)(ua - ru0) * opitch + ((colok[j] ? vcol[j] : rv0) - rv0);
     }
-    float* accb = a.acc + (int64_t)f * a.acc_frame_stride;
+    float* accb = chained ? a.acc + (int64_t)f * a.acc_frame_stride + (int64_t)cid * a.acc_chain_stride : nullptr;
     const int64_t sfo = (int64_t)f * a.stat_frame_stride;
 #pragma unroll 1
     for (int gd = 0; gd < ngrp; ++gd) {
       const int up0 = gd * kG - kHB + 1;
       const bool has_rows = up0 + kG > 0 && up0 < nu && !TC_EXP(32) && !(a.exp & 2);
       const int slot = gd % kGRing;
-      unsigned int* fl = a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + gd) * 4 + cw;
+      unsigned int* fl = flag_ptr(gd);
       unsigned long long pt = prof ? gtimer() : 0ull;
       int64_t rowoff[kG];
 #pragma unroll
@@ -594,13 +603,11 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         if (pending >= 0) {
           __threadfence();  // each lane's stores before the flag (the threadFenceReduction pattern)
           __syncwarp();
-          if (lane == 0)
-            st_release_u32(a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + pending) * 4 + cw,
-                           (unsigned)(blk + 1));
+          if (lane == 0) st_release_u32(flag_ptr(pending), (unsigned)(blk + 1));
           pending = -1;
         }
       };
-      if (has_rows && blk > 0 && !(a.exp & 1) && !a.planes) {  // every lane acquires the flag itself
+      if (has_rows && chained && !cfirst && !(a.exp & 1)) {  // every lane acquires the flag itself
         unsigned int fv = ld_acquire_u32(fl);
         publish_pending();
         for (long long it = 0; fv < (unsigned)blk; ++it) {
@@ -611,7 +618,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         publish_pending();
       }
       if (prof) { const unsigned long long t = gtimer(); p_flag += t - pt; pt = t; }
-      if (has_rows && blk > 0 && !a.planes) {
+      if (has_rows && chained && !cfirst) {
 #pragma unroll
         for (int j = 0; j < 2; ++j)
 #pragma unroll
@@ -625,7 +632,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
 #pragma unroll
         for (int k = 0; k < kG; ++k) x[j][k] = stg[slot * (kG * 128) + k * 128 + 32 * j];
       mbar_arrive(&consumed[slot]);
-      if (has_rows && a.planes) {  // planes mode: this block's partial sums to its own plane (no waiting)
+      if (has_rows && a.planes && !chained) {  // planes mode: this block's partial sums to its own plane (no waiting)
         float* pb = a.part + (int64_t)blk * a.part_blk_stride + (int64_t)f * osub;
 #pragma unroll
         for (int j = 0; j < 2; ++j)
@@ -635,13 +642,23 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
             if (up >= 0 && up < nu && colok[j]) __stcg(pb + cb[j] + (int64_t)up * opitch, x[j][k]);
           }
       } else if (has_rows && !(a.exp & 16)) {
-        if (blk > 0) {
+        if (!cfirst) {
 #pragma unroll
           for (int j = 0; j < 2; ++j)
 #pragma unroll
             for (int k = 0; k < kG; ++k) x[j][k] = prev[j][k] + x[j][k];
         }
-        if (!last_blk) {
+        if (clast && a.planes) {  // chained planes: the chain's sum to plane cid (tm_tc_finish)
+          float* pb = a.part + (int64_t)cid * a.part_blk_stride + (int64_t)f * osub;
+#pragma unroll
+          for (int j = 0; j < 2; ++j)
+#pragma unroll
+            for (int k = 0; k < kG; ++k) {
+              const int up = up0 + k;
+              if (up >= 0 && up < nu && colok[j]) __stcg(pb + cb[j] + (int64_t)up * opitch, x[j][k]);
+            }
+          if (lane == 0 && !cfirst) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
+        } else if (!clast) {
 #pragma unroll
           for (int j = 0; j < 2; ++j)
 #pragma unroll
@@ -677,7 +694,7 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
               }
             }
           }
-          if (lane == 0 && blk > 0) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
+          if (lane == 0 && !cfirst) *fl = 0u;  // consumed: ready for the next call (stream-ordered)
         }
       }
       if (prof) {
@@ -689,12 +706,10 @@ __global__ void __launch_bounds__(tc::kThreads, 1) tm_tc_kernel(const TcArgs a,
         }
       }
     }
-    if (pending >= 0 && !a.planes) {  // the last group's running sums
+    if (pending >= 0) {  // the last group's running sums
       __threadfence();
       __syncwarp();
-      if (lane == 0)
-        st_release_u32(a.flags + ((int64_t)(f * a.vtiles * a.nseg + tile) * a.ngrp_max + pending) * 4 + cw,
-                       (unsigned)(blk + 1));
+      if (lane == 0) st_release_u32(flag_ptr(pending), (unsigned)(blk + 1));
     }
     if (last_blk && !a.planes) {
       wbest = warp_max_key(wbest);
